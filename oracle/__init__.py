@@ -1,0 +1,191 @@
+"""CPU oracle for the partitioned-communication hot path — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
+/ ``--impl reference`` legs may import this package.  The product path
+(``paper_conf_sc_temucinslsga24_b200``, ``libpc.so``) never imports it and shares
+no code with it.  See ``oracle.cpp`` for what each function follows in the paper
+(PAPER.md line citations) and DESIGN.md §"Readings of the paper" for R1..R23.
+
+Functions (numpy in, numpy out):
+  p2p(...)                O1  partitioned send/recv with aggregation + RTR
+  allreduce_def_i32(...)  O2  plain definition, int32 (sum wraps, max, min)
+  allreduce_def_f64(...)  O2  plain definition, fp32 inputs summed in fp64
+  pallreduce(...)         O3/O4  Alg 1 (ring) or RD schedule + Alg 2, P threads
+  alg1_table(P, r)        Alg 1 step tuples
+  ring_fold_f32 / rd_tree_f32   closed forms of O3 / O4 (pinned against them)
+  jacobi_seq / jacobi_decomp    O5
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+INT32, FLOAT32 = 0, 1
+SUM, MAX, MIN = 0, 1, 2
+RING, RD = 1, 2
+
+
+def build(force: bool = False) -> str:
+    src = os.path.join(_HERE, "oracle.cpp")
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
+        subprocess.check_call(["make", "-s", "-C", _HERE, "liboracle.so"])
+    return _SO
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        _lib = C.CDLL(_SO)
+        P = C.c_void_p
+        i32, i64, u64 = C.c_int, C.c_int64, C.c_uint64
+        _lib.orc_p2p.argtypes = [P, P, i32, i64, i32, i32, i32, P, i32, i32, u64, P]
+        _lib.orc_allreduce_def_i32.argtypes = [i32, i64, P, i32, P]
+        _lib.orc_allreduce_def_f64.argtypes = [i32, i64, P, P, P]
+        _lib.orc_pallreduce.argtypes = [i32, i32, i32, i64, i32, i32, i32, i32, P, P, P, u64, P, P]
+        _lib.orc_alg1_table.argtypes = [i32, i32, P]
+        _lib.orc_ring_fold_f32.argtypes = [i32, i64, P, P, P]
+        _lib.orc_rd_tree_f32.argtypes = [i32, i64, P, P]
+        _lib.orc_jacobi_seq.argtypes = [i32, i32, i32, P, P]
+        _lib.orc_jacobi_decomp.argtypes = [i32, i32, i32, i32, i32, P, P]
+    return _lib
+
+
+def _p(a: np.ndarray):
+    return a.ctypes.data_as(C.c_void_p)
+
+
+class OracleError(RuntimeError):
+    pass
+
+
+def _check(rc: int, what: str):
+    if rc < 0:
+        raise OracleError(f"{what} failed with {rc}")
+    return rc
+
+
+def p2p(send: np.ndarray, partitions: int, agg: int, orders: np.ndarray, workers: int = 4,
+        use_rtr: bool = True, recv_delay_us: int = 0, jitter_seed: int = 1):
+    """send: (epochs, total_bytes) uint8.  Returns (consumed, arrivals[epochs, n_transport])."""
+    send = np.ascontiguousarray(send, dtype=np.uint8)
+    epochs, total = send.shape
+    assert total % partitions == 0
+    nt = (partitions + agg - 1) // agg
+    consumed = np.zeros_like(send)
+    arrivals = np.zeros((epochs, nt), dtype=np.uint32)
+    orders = np.ascontiguousarray(orders, dtype=np.int32).reshape(epochs, partitions)
+    _check(lib().orc_p2p(_p(send), _p(consumed), partitions, total // partitions, agg, workers, epochs,
+                         _p(orders), int(use_rtr), recv_delay_us, jitter_seed, _p(arrivals)), "orc_p2p")
+    return consumed, arrivals
+
+
+def allreduce_def_i32(x: np.ndarray, op: int = SUM) -> np.ndarray:
+    """x: (P, n) int32 -> (n,) int32."""
+    x = np.ascontiguousarray(x, dtype=np.int32)
+    P, n = x.shape
+    y = np.zeros(n, dtype=np.int32)
+    _check(lib().orc_allreduce_def_i32(P, n, _p(x), op, _p(y)), "def_i32")
+    return y
+
+
+def allreduce_def_f64(x: np.ndarray):
+    """x: (P, n) float32 -> (fp64 sum, fp64 sum|x|)."""
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    P, n = x.shape
+    y = np.zeros(n, dtype=np.float64)
+    a = np.zeros(n, dtype=np.float64)
+    _check(lib().orc_allreduce_def_f64(P, n, _p(x), _p(y), _p(a)), "def_f64")
+    return y, a
+
+
+def n_steps(algo: int, P: int) -> int:
+    if algo == RING:
+        return 2 * (P - 1)
+    k = 0
+    while (1 << k) < P:
+        k += 1
+    return k
+
+
+def pallreduce(x: np.ndarray, partitions: int, algo: int = RING, op: int = SUM, inplace: bool = False,
+               orders: np.ndarray | None = None, jitter_seed: int = 1):
+    """x: (epochs, P, Np*L) int32 or float32 (or (P, Np*L) for one epoch).
+
+    Returns (y, reduces, arrivals): y has x's shape and holds each rank's recvbuf
+    after its MPI_Wait; reduces/arrivals are (P, Np, max(nsteps,1)) counts from
+    the last epoch."""
+    squeeze = x.ndim == 2
+    if squeeze:
+        x = x[None]
+    dtype = INT32 if x.dtype == np.int32 else FLOAT32
+    x = np.ascontiguousarray(x)
+    epochs, P, n = x.shape
+    assert n % partitions == 0
+    L = n // partitions
+    if orders is None:
+        orders = np.tile(np.arange(partitions, dtype=np.int32), (epochs, P, 1))
+    orders = np.ascontiguousarray(orders, dtype=np.int32).reshape(epochs, P, partitions)
+    ns = max(n_steps(algo, P), 1)
+    y = np.zeros_like(x)
+    red = np.zeros((P, partitions, ns), dtype=np.uint32)
+    arr = np.zeros((P, partitions, ns), dtype=np.uint32)
+    _check(lib().orc_pallreduce(algo, P, partitions, L, dtype, op, epochs, int(inplace), _p(x), _p(y),
+                                _p(orders), jitter_seed, _p(red), _p(arr)), "orc_pallreduce")
+    return (y[0] if squeeze else y), red, arr
+
+
+def alg1_table(P: int, r: int) -> np.ndarray:
+    """(2(P-1), 5) int32 rows (I, R, op, O, A)."""
+    out = np.zeros((max(2 * (P - 1), 1), 5), dtype=np.int32)
+    n = _check(lib().orc_alg1_table(P, r, _p(out)), "alg1_table")
+    return out[:n]
+
+
+def ring_fold_f32(x: np.ndarray, start: np.ndarray) -> np.ndarray:
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    P, n = x.shape
+    start = np.ascontiguousarray(start, dtype=np.int32)
+    out = np.zeros(n, dtype=np.float32)
+    _check(lib().orc_ring_fold_f32(P, n, _p(x), _p(start), _p(out)), "ring_fold")
+    return out
+
+
+def rd_tree_f32(x: np.ndarray) -> np.ndarray:
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    P, n = x.shape
+    out = np.zeros(n, dtype=np.float32)
+    _check(lib().orc_rd_tree_f32(P, n, _p(x), _p(out)), "rd_tree")
+    return out
+
+
+def chunk_ids(L: int, P: int, partitions: int) -> np.ndarray:
+    """Chunk id of every element of an (Np*L) buffer under reading R4
+    (q = ceil(L/(4P))*4 elements per chunk)."""
+    q = -(-L // (4 * P)) * 4 if L > 0 else 4
+    j = np.arange(L)
+    c = np.minimum(j // max(q, 1), P - 1).astype(np.int32)
+    return np.tile(c, partitions)
+
+
+def jacobi_seq(a0: np.ndarray, iters: int) -> np.ndarray:
+    a0 = np.ascontiguousarray(a0, dtype=np.float32)
+    ny, nx = a0.shape
+    out = np.zeros_like(a0)
+    _check(lib().orc_jacobi_seq(ny, nx, iters, _p(a0), _p(out)), "jacobi_seq")
+    return out
+
+
+def jacobi_decomp(a0: np.ndarray, iters: int, Py: int, Px: int) -> np.ndarray:
+    a0 = np.ascontiguousarray(a0, dtype=np.float32)
+    ny, nx = a0.shape
+    out = np.zeros_like(a0)
+    _check(lib().orc_jacobi_decomp(ny, nx, Py, Px, iters, _p(a0), _p(out)), "jacobi_decomp")
+    return out
