@@ -1,0 +1,177 @@
+/*
+ * include/pc.h — host C ABI of libpc: GPU-initiated MPI-Partitioned-style
+ * communication for B200 (NVLink 5 / NVSwitch), after Temuçin et al., SC'24
+ * ("Design and Implementation of MPI-Native GPU-Initiated MPI Partitioned
+ * Communication"; reference text PAPER.md, cited as P:Lnn §section).
+ *
+ * Plain C: pointers, sizes, ints.  No torch or C++ types cross this boundary.
+ * Every host call returns PC_SUCCESS (0) or a negative PC_ERR_* code and never
+ * throws.  Device-side bindings are in pc_device.cuh.
+ *
+ * Flow (Listing 2; Fig. 1; §IV-A):
+ *     pc_psend_init / pc_precv_init / pc_pallreduce_init      once
+ *     loop:  pc_start -> pc_pbuf_prepare -> [first: pc_prequest_create]
+ *            -> user kernel calling pc_pready*(p, preq) -> pc_wait
+ *
+ * Buffers: caller-owned device memory (cudaMalloc or the torch caching
+ * allocator WITHOUT expandable segments), 16-byte aligned, valid and unmoved
+ * until pc_request_free.  The library owns flags, counters, staging and the
+ * device request storage.  Host calls for one request come from one host
+ * thread at a time.
+ */
+#ifndef PC_H_
+#define PC_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* cudaStream_t without including cuda_runtime.h (ABI-identical pointer). */
+typedef struct CUstream_st *pc_stream_t;
+
+typedef struct pc_comm_s *pc_comm_t;            /* opaque: rank, size, device, peer mappings     */
+typedef struct pc_request_s *pc_request_t;      /* opaque: one persistent partitioned request    */
+typedef struct pc_local_group_s *pc_local_group_t; /* in-process rank group (virtual ranks)      */
+typedef struct pc_prequest_s pc_prequest_t;     /* POD device request, passed BY VALUE to kernels
+                                                   (MPIX_Prequest); layout in pc_device.cuh */
+
+typedef enum { PC_INT32 = 0, PC_FLOAT32 = 1, PC_BYTE = 2 } pc_dtype_t;
+typedef enum { PC_OP_SUM = 0, PC_OP_MAX = 1, PC_OP_MIN = 2 } pc_op_t;
+/* Granularity of the device Pready call: informational — the device
+ * function chosen (pc_pready / _warp / _block) decides who participates. */
+typedef enum { PC_GRAN_THREAD = 0, PC_GRAN_WARP = 1, PC_GRAN_BLOCK = 2 } pc_gran_t;
+/* Copy mechanism: INLINE = "Kernel Copy" — the contributor that
+ * completes a transport partition pushes it over NVLink from inside the user
+ * kernel; ENGINE = persistent library warps poll ready flags and push (the
+ * GPU-resident replacement of the paper's host Progression Engine). */
+typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1 } pc_copy_t;
+/* Allreduce schedule (§IV-B).  RING = Alg 1; RD = recursive
+ * doubling (BASELINE north_star; not in the paper; P a power of two);
+ * AUTO = RD below the size threshold (env PC_RD_MAX_BYTES), ring above. */
+typedef enum { PC_ALGO_AUTO = 0, PC_ALGO_RING = 1, PC_ALGO_RD = 2 } pc_algo_t;
+
+enum {
+  PC_SUCCESS = 0,
+  PC_ERR_ARG = -1,         /* bad argument (null, range, misaligned buffer)             */
+  PC_ERR_CUDA = -2,        /* a CUDA runtime/driver call failed                         */
+  PC_ERR_STATE = -3,       /* start on active / free of active / pready on inactive     */
+  PC_ERR_MATCH = -4,       /* send/recv (or allreduce) parameters disagree across ranks */
+  PC_ERR_TIMEOUT = -5,     /* a device spin exceeded PC_TIMEOUT_MS (sticky error word)   */
+  PC_ERR_DEVICE = -6,      /* a device call reported an error (bad partition, dup)       */
+  PC_ERR_NOMEM = -7,
+  PC_ERR_UNSUPPORTED = -8
+};
+
+/* ---------------------------------------------------------------- bootstrap
+ * All-gather callback supplied by the caller (a torch ProcessGroup, MPI, …):
+ * gather `nbytes` from every rank into recv[rank*nbytes].  Returns 0 on success.
+ * It is called only from pc_comm_create and from the FIRST pc_pbuf_prepare of
+ * a batch of new requests (see pc_pbuf_prepare), never on the hot path. */
+typedef int (*pc_allgather_fn)(const void *send, size_t nbytes, void *recv, void *ctx);
+
+/* cuda_device = -1 creates a host-only ("dry") comm: requests, matching and
+ * schedules work, nothing touches a GPU (used by CPU tests of the host logic). */
+int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void *ctx, pc_comm_t *comm);
+int pc_comm_destroy(pc_comm_t comm);
+int pc_comm_rank(pc_comm_t comm, int *rank);
+int pc_comm_size(pc_comm_t comm, int *size);
+/* Number of engine warps every rank uses (agreed at comm creation: identical
+ * on all ranks so per-warp work orders match — the deadlock-freedom argument
+ * of DESIGN.md §"Engine"). */
+int pc_comm_engine_warps(pc_comm_t comm, int *warps);
+
+/* In-process rank groups: several ranks of one comm living in ONE process
+ * (e.g. P virtual ranks sharing one GPU, or one process driving several GPUs).
+ * Peers in the same process are addressed directly, without CUDA IPC.  Each
+ * rank must be driven by its own host thread during pc_comm_create and the
+ * first pc_pbuf_prepare (the all-gather blocks until every rank arrived). */
+int pc_local_group_create(int size, pc_local_group_t *group);
+int pc_local_group_destroy(pc_local_group_t group);
+/* ctx to pass to pc_comm_create together with pc_local_allgather */
+void *pc_local_group_ctx(pc_local_group_t group, int rank);
+int pc_local_allgather(const void *send, size_t nbytes, void *recv, void *ctx);
+
+/* ---------------------------------------------------------------- init (non-blocking)
+ * MPI-4 partitioned semantics: `count` is elements PER PARTITION, the
+ * buffer holds partitions*count elements.  Matching is by (comm, peer, tag,
+ * posting order).  Nothing is exchanged here; mismatches surface as
+ * PC_ERR_MATCH at the first pc_pbuf_prepare. */
+int pc_psend_init(const void *buf, int partitions, size_t count, pc_dtype_t dtype, int dest, int tag,
+                  pc_comm_t comm, pc_request_t *req);
+int pc_precv_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, int source, int tag,
+                  pc_comm_t comm, pc_request_t *req);
+/* Partitioned allreduce (MPIX_Pallreduce_init; schedule S of
+ * P:L153-L155).  Collective: every rank calls it with identical arguments in
+ * the same order.  sendbuf == recvbuf (in place) is allowed.  dtype INT32 or
+ * FLOAT32; op SUM/MAX/MIN. */
+int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
+                       pc_op_t op, pc_algo_t algo, pc_comm_t comm, pc_request_t *req);
+
+/* ---------------------------------------------------------------- epoch
+ * MPI_Start: epoch e <- e+1, written stream-ordered to the device
+ * epoch word; for ENGINE copy and allreduce it also launches the engine on a
+ * library stream forked from `stream`.  PC_ERR_STATE if the request is active. */
+int pc_start(pc_request_t req, pc_stream_t stream);
+/* MPIX_Pbuf_prepare: guarantees the remote buffers are
+ * ready.  FIRST call (per batch of new requests): host-blocking exchange of
+ * request records + IPC handles through the comm's all-gather, matching,
+ * mapping of peer buffers.  Every call: stream-ordered "ready-to-receive"
+ * epoch write into each producer's RTR word (no host blocking); producers
+ * check it on the device before their first push of the epoch. */
+int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream);
+/* MPIX_Prequest_create: build the POD device request.  `aggregation`
+ * = g user partitions per transport partition (P:L129 threshold; 1 = none);
+ * allreduce requires g = 1.  Blocking.  Writes the transport layout into the
+ * receiver's control block. */
+int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_copy_t copy, pc_prequest_t *out);
+int pc_prequest_free(pc_prequest_t *preq);
+/* sizeof(pc_prequest_t) as compiled into the library (bindings check it). */
+size_t pc_prequest_size(void);
+
+/* ---------------------------------------------------------------- completion
+ * pc_parrived: host, non-blocking, 1 iff partition complete this epoch (P:L48,
+ * P:L143; allreduce: final result in recvbuf).
+ * pc_test: host, non-blocking MPI_Test.  pc_wait: host-blocking MPI_Wait
+ * (P:L50); returns PC_ERR_TIMEOUT / PC_ERR_DEVICE if the device
+ * reported one.  pc_wait_on_stream: enqueue "wait for completion" on `stream`
+ * without host blocking (the request becomes inactive for the host; later
+ * work on `stream` is ordered after completion).  Wait on an inactive request
+ * returns PC_SUCCESS. */
+int pc_parrived(pc_request_t req, int partition, int *flag);
+int pc_test(pc_request_t req, int *flag);
+int pc_wait(pc_request_t req);
+int pc_wait_on_stream(pc_request_t req, pc_stream_t stream);
+/* Host Pready bindings (MPI_Pready / MPI_Pready_range): enqueue a tiny kernel
+ * on `stream` that marks partitions [lo, hi] ready. */
+int pc_pready(int partition, pc_request_t req, pc_stream_t stream);
+int pc_pready_range(int lo, int hi, pc_request_t req, pc_stream_t stream);
+int pc_request_free(pc_request_t *req);
+
+/* ---------------------------------------------------------------- introspection
+ * (host logic exported for tests; pure functions, no GPU) */
+/* Ring schedule (Alg 1) of rank r: rows (I, R, op, O, A) for the 2(P-1)
+ * communicating steps; returns the number of steps. */
+int pc_schedule_ring(int P, int r, int32_t *out_rows5);
+/* Recursive-doubling schedule: rows (I, R=-1, op=1, O, A=-1); log2 P steps. */
+int pc_schedule_rd(int P, int r, int32_t *out_rows5);
+/* Chunk bounds of a partition of L elements split in P chunks (reading R4):
+ * out[c] = first element of chunk c, out[P] = L. */
+int pc_chunk_bounds(int64_t L, int P, int64_t *out);
+/* Request facts after the first pbuf_prepare: algo actually used, slices per
+ * chunk, slice elements, engine warps. */
+int pc_request_info(pc_request_t req, int *algo, int *slices, int64_t *slice_elems, int *engine_warps);
+/* Matched peer request id (debug; p2p) after the first pbuf_prepare. */
+int pc_request_match(pc_request_t req, int *peer, int *peer_request_index);
+/* Device error word of a request: code and partition (0,0 if none). */
+int pc_request_error(pc_request_t req, int *code, int *partition);
+const char *pc_strerror(int err);
+/* Library version string. */
+const char *pc_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PC_H_ */

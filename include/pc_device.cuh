@@ -1,0 +1,363 @@
+/*
+ * include/pc_device.cuh — device bindings of libpc (sm_100a).
+ *
+ *   PC_DEVICE int  pc_pready      (int partition, pc_prequest_t preq);  any thread
+ *   PC_DEVICE int  pc_pready_warp (int partition, pc_prequest_t preq);  warp-collective
+ *   PC_DEVICE int  pc_pready_block(int partition, pc_prequest_t preq);  block-collective
+ *   PC_DEVICE int  pc_parrived    (pc_prequest_t preq, int partition);
+ *   PC_DEVICE int  pc_wait_arrived(pc_prequest_t preq, int partition);
+ *
+ * Paper: MPIX_Pready / MPIX_Pready_{thread,warp,block} / MPIX_Parrived
+ * (Listing 2; §IV-A4).  PC_DEVICE plays the role of
+ * MPIX_Device.
+ *
+ * pc_pready* semantics: "user partition `partition` of the send buffer is
+ * final for the current epoch".  Call at most once per partition per epoch.
+ *   - Aggregation: user partition p belongs to transport
+ *     partition t = p / g.  Contributors increment a never-reset GPU-global
+ *     counter cnt[t] (target e*g_t, wrap-aware); thread-granularity callers are
+ *     first combined per warp with __match_any_sync so one atomic covers every
+ *     lane of the warp that targets the same t (the library-side aggregation
+ *     the paper recommends).
+ *   - INLINE copy ("Kernel Copy"): the warp/block whose contribution
+ *     completes t pushes t's bytes to the receiver's buffer over NVLink with
+ *     16-byte vector stores, then releases the receiver's flag[t] = e with a
+ *     system-scope fence + store (the completion the paper sent through the
+ *     host, done here on the device).  Before its first push of the
+ *     epoch it checks the ready-to-receive word (Pbuf_prepare).
+ *   - ENGINE copy: the completing contributor only release-stores ready[t] = e;
+ *     library engine warps move the data.
+ *   - Allreduce requests: marks user partition u ready (step S_0 is the
+ *     user's Pready); the library engine runs the schedule.
+ * Returns 0, or a PC_ERR_* code that is also recorded in the sticky error word
+ * (bad partition, duplicate Pready detected by counter overshoot).
+ *
+ * pc_parrived: 1 iff the partition is complete in this epoch (receive: its
+ * bytes are in recvbuf; allreduce: its final result is in recvbuf).
+ * It is an ld.acquire.sys of a flag in the caller's OWN memory (written
+ * remotely by the producer), not a host round trip.  Other threads
+ * of the block must synchronise with the polling thread before they read the
+ * partition.
+ */
+#ifndef PC_DEVICE_CUH_
+#define PC_DEVICE_CUH_
+
+#include <stdint.h>
+
+#include "pc_prequest.h"
+
+typedef struct pc_prequest_s pc_prequest_t;
+
+#define PC_DEVICE __device__ __forceinline__
+
+#ifndef PC_DEV_ERR_ARG
+#define PC_DEV_ERR_ARG (-1)
+#define PC_DEV_ERR_TIMEOUT (-5)
+#define PC_DEV_ERR_DEVICE (-6)
+#endif
+
+namespace pc_detail {
+
+PC_DEVICE uint32_t ld_acquire_sys(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+PC_DEVICE uint32_t ld_acquire_gpu(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+PC_DEVICE uint32_t ld_relaxed_sys(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+PC_DEVICE void st_release_sys(uint32_t *p, uint32_t v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+PC_DEVICE void st_relaxed_sys(uint32_t *p, uint32_t v) {
+  asm volatile("st.relaxed.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+PC_DEVICE void st_release_gpu(uint32_t *p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+PC_DEVICE uint32_t atom_add_acq_rel_gpu(uint32_t *p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+PC_DEVICE void red_add_release_gpu(uint32_t *p, uint32_t v) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+PC_DEVICE void fence_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+PC_DEVICE uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+PC_DEVICE uint32_t lane_id() {
+  uint32_t l;
+  asm("mov.u32 %0, %%laneid;" : "=r"(l));
+  return l;
+}
+/* wrap-aware "v has reached target" for monotonically increasing u32 words */
+PC_DEVICE bool reached(uint32_t v, uint32_t target) { return (int32_t)(v - target) >= 0; }
+
+PC_DEVICE void set_error(int32_t *err, int32_t code, int32_t part) {
+  if (atomicCAS(err, 0, code) == 0) {
+    err[1] = part;
+    __threadfence_system();
+  }
+}
+PC_DEVICE bool aborted(const int32_t *err) { return *(const volatile int32_t *)err != 0; }
+
+/* Spin until *p has reached `target`.  SYS: acquire at system scope (word
+ * written by another GPU); else GPU scope.  Bounded: after timeout_ms sets the
+ * sticky error word and returns false; also returns false as soon as another
+ * thread has set an error (so one failure drains every waiter instead of
+ * hanging the device). */
+template <bool SYS>
+PC_DEVICE bool spin_geq(const uint32_t *p, uint32_t target, int32_t *err, uint32_t timeout_ms, int32_t part) {
+  uint32_t v = SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p);
+  if (reached(v, target)) return true;
+  const uint64_t t0 = globaltimer();
+  uint32_t n = 0, ns = 0;
+  for (;;) {
+    if (ns) __nanosleep(ns);
+    v = SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p);
+    if (reached(v, target)) return true;
+    ++n;
+    if (n > 512) ns = ns ? (ns < 512 ? ns * 2 : 512) : 32;
+    if ((n & 127) == 0) {
+      if (aborted(err)) return false;
+      if (timeout_ms && globaltimer() - t0 > (uint64_t)timeout_ms * 1000000ull) {
+        set_error(err, PC_DEV_ERR_TIMEOUT, part);
+        return false;
+      }
+    }
+  }
+}
+
+/* Cooperative byte copy by `n` participants (participant index `idx`):
+ * 16-byte vector loads (L2, .cg) and stores when both pointers are 16-B
+ * aligned, 4 independent vectors in flight per participant; 4-byte and
+ * 1-byte fallbacks otherwise.  dst may be a peer-mapped (NVLink) address. */
+PC_DEVICE void copy_bytes(uint8_t *dst, const uint8_t *src, uint64_t nbytes, uint32_t idx, uint32_t n) {
+  if (((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src)) & 15) == 0) {
+    const uint64_t nv = nbytes >> 4;
+    const uint4 *s = reinterpret_cast<const uint4 *>(src);
+    uint4 *d = reinterpret_cast<uint4 *>(dst);
+    uint64_t k = idx;
+    for (; k + 3ull * n < nv; k += 4ull * n) {
+      uint4 a = __ldcg(s + k), b = __ldcg(s + k + n), c = __ldcg(s + k + 2 * n), e = __ldcg(s + k + 3 * n);
+      d[k] = a;
+      d[k + n] = b;
+      d[k + 2 * n] = c;
+      d[k + 3 * n] = e;
+    }
+    for (; k < nv; k += n) d[k] = __ldcg(s + k);
+    for (uint64_t b = (nv << 4) + idx; b < nbytes; b += n) dst[b] = src[b];
+  } else if (((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src) | nbytes) & 3) == 0) {
+    const uint32_t *s = reinterpret_cast<const uint32_t *>(src);
+    uint32_t *d = reinterpret_cast<uint32_t *>(dst);
+    for (uint64_t k = idx; k < (nbytes >> 2); k += n) d[k] = __ldcg(s + k);
+  } else {
+    for (uint64_t b = idx; b < nbytes; b += n) dst[b] = src[b];
+  }
+}
+
+PC_DEVICE uint32_t epoch_of(const pc_prequest_t &q) { return *(const volatile uint32_t *)q.epoch; }
+
+PC_DEVICE uint32_t transport_size(const pc_prequest_t &q, int t) {
+  const int rem = q.partitions - t * q.agg;
+  return (uint32_t)(rem < q.agg ? rem : q.agg);
+}
+
+/* Count `add` contributions to transport partition t; returns true for the
+ * single contribution that completes t in epoch e.  Flags a duplicate Pready
+ * (counter already at/over the target) in the sticky error word. */
+PC_DEVICE bool contribute(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, int part) {
+  const uint32_t target = e * transport_size(q, t);
+  const uint32_t old = atom_add_acq_rel_gpu(q.cnt + t, add);
+  const int32_t d = (int32_t)(target - old);
+  if (d <= 0) {
+    set_error(q.err, PC_DEV_ERR_DEVICE, part);
+    return false;
+  }
+  return d <= (int32_t)add;
+}
+
+/* INLINE push of transport partition t by the lanes in `mask` (warp scope). */
+PC_DEVICE void push_warp(const pc_prequest_t &q, int t, uint32_t e, unsigned mask) {
+  const uint32_t lane = lane_id();
+  const uint32_t first = __ffs(mask) - 1;
+  const uint32_t idx = __popc(mask & ((1u << lane) - 1));
+  const uint32_t n = __popc(mask);
+  bool ok = true;
+  if (lane == first) ok = spin_geq<true>(q.rtr, e, q.err, q.timeout_ms, t);
+  ok = __shfl_sync(mask, ok, first);
+  if (!ok) return;
+  const uint64_t off = (uint64_t)t * (uint64_t)q.agg * q.part_bytes;
+  const uint64_t len = (uint64_t)transport_size(q, t) * q.part_bytes;
+  copy_bytes(q.peer_rbuf + off, q.sbuf + off, len, idx, n);
+  fence_sys();
+  __syncwarp(mask);
+  if (lane == first) {
+    st_relaxed_sys(q.peer_flags + t, e);
+    st_release_gpu(q.sent + t, e);
+  }
+}
+
+/* INLINE push of transport partition t by the whole block. */
+PC_DEVICE void push_block(const pc_prequest_t &q, int t, uint32_t e) {
+  __shared__ int s_ok;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  const uint32_t nthr = blockDim.x * blockDim.y * blockDim.z;
+  if (tid == 0) s_ok = spin_geq<true>(q.rtr, e, q.err, q.timeout_ms, t);
+  __syncthreads();
+  if (!s_ok) return;
+  const uint64_t off = (uint64_t)t * (uint64_t)q.agg * q.part_bytes;
+  const uint64_t len = (uint64_t)transport_size(q, t) * q.part_bytes;
+  copy_bytes(q.peer_rbuf + off, q.sbuf + off, len, tid, nthr);
+  fence_sys();
+  __syncthreads();
+  if (tid == 0) {
+    st_relaxed_sys(q.peer_flags + t, e);
+    st_release_gpu(q.sent + t, e);
+  }
+}
+
+}  // namespace pc_detail
+
+/* ------------------------------------------------------------------ Pready */
+
+/* Thread granularity: any subset of threads, each for its own partition. */
+PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
+  using namespace pc_detail;
+  if (partition < 0 || partition >= preq.partitions) {
+    set_error(preq.err, PC_DEV_ERR_ARG, partition);
+    return PC_DEV_ERR_ARG;
+  }
+  const uint32_t e = epoch_of(preq);
+  if (preq.kind == PC_KIND_PALLREDUCE) {
+    st_release_gpu(preq.ready + partition, e);
+    return 0;
+  }
+  const unsigned mask = __activemask();
+  const uint32_t lane = lane_id();
+  const int t = partition / preq.agg;
+  const unsigned grp = __match_any_sync(mask, t);
+  const uint32_t leader = __ffs(grp) - 1;
+  __syncwarp(mask);  // every lane's data writes are ordered before the leader's release
+  bool completes = false;
+  if (lane == leader) completes = contribute(preq, t, __popc(grp), e, partition);
+  if (preq.copy == 1) {  // ENGINE
+    if (completes) st_release_gpu(preq.ready + t, e);
+    return 0;
+  }
+  unsigned cmask = __ballot_sync(mask, completes);
+  __syncwarp(mask);
+  while (cmask) {
+    const int src = __ffs(cmask) - 1;
+    cmask &= cmask - 1;
+    const int tt = __shfl_sync(mask, t, src);
+    push_warp(preq, tt, e, mask);
+  }
+  return 0;
+}
+
+/* Warp granularity: all active lanes of the warp call it with the same
+ * partition; one notification per warp (reading R11). */
+PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
+  using namespace pc_detail;
+  const unsigned mask = __activemask();
+  const uint32_t lane = lane_id();
+  const uint32_t first = __ffs(mask) - 1;
+  if (partition < 0 || partition >= preq.partitions) {
+    if (lane == first) set_error(preq.err, PC_DEV_ERR_ARG, partition);
+    return PC_DEV_ERR_ARG;
+  }
+  const uint32_t e = epoch_of(preq);
+  __syncwarp(mask);
+  if (preq.kind == PC_KIND_PALLREDUCE) {
+    if (lane == first) st_release_gpu(preq.ready + partition, e);
+    return 0;
+  }
+  const int t = partition / preq.agg;
+  bool completes = false;
+  if (lane == first) completes = contribute(preq, t, 1, e, partition);
+  completes = __shfl_sync(mask, completes, first);
+  if (!completes) return 0;
+  if (preq.copy == 1) {
+    if (lane == first) st_release_gpu(preq.ready + t, e);
+    return 0;
+  }
+  __syncwarp(mask);
+  push_warp(preq, t, e, mask);
+  return 0;
+}
+
+/* Block granularity: every thread of the block calls it with the same
+ * partition; __syncthreads() then one notification. */
+PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
+  using namespace pc_detail;
+  __shared__ int s_completes;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  if (partition < 0 || partition >= preq.partitions) {
+    if (tid == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);
+    return PC_DEV_ERR_ARG;
+  }
+  const uint32_t e = epoch_of(preq);
+  __syncthreads();
+  if (preq.kind == PC_KIND_PALLREDUCE) {
+    if (tid == 0) st_release_gpu(preq.ready + partition, e);
+    return 0;
+  }
+  const int t = partition / preq.agg;
+  if (tid == 0) s_completes = contribute(preq, t, 1, e, partition);
+  __syncthreads();
+  const bool completes = s_completes;
+  if (!completes) return 0;
+  if (preq.copy == 1) {
+    if (tid == 0) st_release_gpu(preq.ready + t, e);
+    return 0;
+  }
+  push_block(preq, t, e);
+  return 0;
+}
+
+/* ---------------------------------------------------------------- Parrived */
+PC_DEVICE int pc_parrived(pc_prequest_t preq, int partition) {
+  using namespace pc_detail;
+  if (partition < 0 || partition >= preq.partitions) return 0;
+  const uint32_t e = epoch_of(preq);
+  if (preq.kind == PC_KIND_PALLREDUCE) return reached(ld_acquire_gpu(preq.done + partition), e * preq.done_mul);
+  if (preq.kind == PC_KIND_PSEND) {
+    const int t = partition / preq.agg;
+    return reached(ld_acquire_gpu(preq.sent + t), e);
+  }
+  const uint32_t g = *(const volatile uint32_t *)preq.layout;
+  if (g == 0) return 0;  // sender has not published its transport layout yet
+  return reached(ld_acquire_sys(preq.flags + partition / (int)g), e);
+}
+
+/* Acquire-spin until pc_parrived(preq, partition) (bounded by timeout_ms). */
+PC_DEVICE int pc_wait_arrived(pc_prequest_t preq, int partition) {
+  using namespace pc_detail;
+  const uint64_t t0 = globaltimer();
+  uint32_t n = 0;
+  while (!pc_parrived(preq, partition)) {
+    if ((++n & 127) == 0) {
+      if (aborted(preq.err)) return PC_DEV_ERR_TIMEOUT;
+      if (preq.timeout_ms && globaltimer() - t0 > (uint64_t)preq.timeout_ms * 1000000ull) {
+        set_error(preq.err, PC_DEV_ERR_TIMEOUT, partition);
+        return PC_DEV_ERR_TIMEOUT;
+      }
+      if (n > 1024) __nanosleep(256);
+    }
+  }
+  return 0;
+}
+
+#endif /* PC_DEVICE_CUH_ */

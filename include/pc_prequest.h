@@ -1,0 +1,48 @@
+/*
+ * include/pc_prequest.h — layout of the device request pc_prequest_t
+ * (MPIX_Prequest: "a device specific request object ... containing only
+ * the necessary information for a GPU to conduct its duties"; copy
+ * mechanism, aggregation threshold, counters, remote address).
+ *
+ * Plain C, shared by the host library (which fills it) and device code (which
+ * receives it BY VALUE as a kernel argument: no pointer chasing).
+ * Every pointer is a device address valid in the owning rank's CUDA context;
+ * peer_* pointers are peer-mapped (CUDA IPC or same-process) addresses of the
+ * partner rank's memory.  The epoch is NOT baked in: pc_prequest_create is
+ * called once (Listing 2) and `epoch` points to the device word
+ * pc_start writes.
+ */
+#ifndef PC_PREQUEST_H_
+#define PC_PREQUEST_H_
+
+#include <stdint.h>
+
+#define PC_KIND_PSEND 1
+#define PC_KIND_PRECV 2
+#define PC_KIND_PALLREDUCE 3
+
+struct pc_prequest_s {
+  uint32_t kind;        /* PC_KIND_*                                                    */
+  uint32_t copy;        /* pc_copy_t: 0 INLINE ("Kernel Copy"), 1 ENGINE                 */
+  int32_t partitions;   /* N_p user partitions                                           */
+  int32_t agg;          /* g user partitions per transport partition (send side)         */
+  int32_t ntransport;   /* ceil(N_p / g)                                                 */
+  uint32_t timeout_ms;  /* device spin bound (0 = forever)                               */
+  uint64_t part_bytes;  /* bytes per user partition (count * sizeof(dtype))              */
+  const uint32_t *epoch;      /* local epoch word written by pc_start                    */
+  uint32_t *cnt;              /* [ntransport] aggregation counters (send), never reset   */
+  uint32_t *ready;            /* [ntransport] ENGINE ready flags / [N_p] allreduce ready */
+  uint32_t *sent;             /* [ntransport] "pushed and flagged" (send-side wait)      */
+  const uint8_t *sbuf;        /* local send buffer                                        */
+  uint8_t *peer_rbuf;         /* receiver's recv buffer (peer-mapped)                     */
+  uint32_t *peer_flags;       /* receiver's arrival flags (peer-mapped) [ntransport]     */
+  const uint32_t *rtr;        /* local ready-to-receive word, written by the consumer    */
+  const uint32_t *flags;      /* receive side: local arrival flags [N_p]                  */
+  const uint32_t *layout;     /* receive side: g, written by the sender at prequest time */
+  const uint32_t *done;       /* allreduce: [N_p] per-partition completion counters      */
+  uint32_t done_mul;          /* allreduce: partition u is final when done[u] >= e*done_mul */
+  int32_t rank;               /* owning rank                                              */
+  int32_t *err;               /* sticky device error word [2] = {code, partition}         */
+};
+
+#endif /* PC_PREQUEST_H_ */

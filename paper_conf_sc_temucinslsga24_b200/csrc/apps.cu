@@ -1,0 +1,178 @@
+// libpcapps: application / producer kernels that USE the device bindings of
+// pc_device.cuh the way a user kernel would (Listing 2).  They are
+// the "compute" side of the paper's experiments:
+//   vecadd       C = A + B, 8 B per thread, 1024-thread blocks, with
+//                pc_pready at thread / warp / block granularity (P:L223,
+//                P:L229; §VI-A)
+//   produce      copy a prepared input into the send buffer partition by
+//                partition and Pready each one (allreduce producer, §VI-B)
+//   check_recv   receiver kernel that waits pc_parrived per partition and
+//                consumes it (device Parrived)
+//   pingpong     Pready->Parrived latency inside one persistent kernel per side
+//   bare_pingpong  the same with raw flags and no library (latency floor)
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "pc_device.cuh"
+
+#define PCAPP_GRAN_NONE (-1)
+#define PCAPP_GRAN_THREAD 0
+#define PCAPP_GRAN_WARP 1
+#define PCAPP_GRAN_BLOCK 2
+
+namespace {
+
+__global__ void __launch_bounds__(1024) vecadd_kernel(const float2 *__restrict__ A, const float2 *__restrict__ B,
+                                                      float2 *__restrict__ C, int64_t n2, int gran,
+                                                      pc_prequest_t preq) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n2) {
+    const float2 a = A[i], b = B[i];
+    C[i] = make_float2(a.x + b.x, a.y + b.y);
+  }
+  if (gran == PCAPP_GRAN_THREAD) {
+    if (i < n2) pc_pready((int)i, preq);
+  } else if (gran == PCAPP_GRAN_WARP) {
+    pc_pready_warp((int)(i >> 5), preq);
+  } else if (gran == PCAPP_GRAN_BLOCK) {
+    pc_pready_block((int)blockIdx.x, preq);
+  }
+}
+
+// Each block produces partitions p = blockIdx.x, +gridDim.x, ...: copies
+// src -> dst for the partition, then marks it ready.
+__global__ void __launch_bounds__(512) produce_kernel(uint8_t *__restrict__ dst, const uint8_t *__restrict__ src,
+                                                     int partitions, int64_t part_bytes, int gran, int order_stride,
+                                                     pc_prequest_t preq) {
+  for (int k = blockIdx.x; k < partitions; k += gridDim.x) {
+    // a permuted production order (order_stride coprime with partitions)
+    const int p = (int)(((int64_t)k * order_stride) % partitions);
+    const int64_t off = (int64_t)p * part_bytes;
+    const uint4 *s4 = reinterpret_cast<const uint4 *>(src + off);
+    uint4 *d4 = reinterpret_cast<uint4 *>(dst + off);
+    const int64_t nv = ((((uintptr_t)(src + off)) | ((uintptr_t)(dst + off))) & 15) ? 0 : part_bytes / 16;
+    for (int64_t j = threadIdx.x; j < nv; j += blockDim.x) d4[j] = s4[j];
+    for (int64_t j = nv * 16 + threadIdx.x; j < part_bytes; j += blockDim.x) dst[off + j] = src[off + j];
+    if (gran == PCAPP_GRAN_BLOCK) {
+      pc_pready_block(p, preq);
+    } else if (gran == PCAPP_GRAN_WARP) {
+      __syncthreads();
+      if (threadIdx.x < 32) pc_pready_warp(p, preq);
+    } else {
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        __threadfence();
+        pc_pready(p, preq);
+      }
+    }
+  }
+}
+
+__global__ void check_recv_kernel(pc_prequest_t preq, const uint8_t *recvbuf, uint8_t *out, int partitions,
+                                  int64_t part_bytes, int *status) {
+  __shared__ int ok;
+  for (int p = blockIdx.x; p < partitions; p += gridDim.x) {
+    if (threadIdx.x == 0) ok = pc_wait_arrived(preq, p) == 0;
+    __syncthreads();
+    if (!ok) {
+      if (threadIdx.x == 0) atomicAdd(status, 1);
+      return;
+    }
+    const int64_t off = (int64_t)p * part_bytes;
+    for (int64_t j = threadIdx.x; j < part_bytes; j += blockDim.x) out[off + j] = __ldcg(recvbuf + off + j);
+    __syncthreads();
+  }
+}
+
+// Ping-pong: side 0 readies partition k of its send request and waits for
+// partition k of its receive request; side 1 mirrors.  One warp per side.
+// Partition k is used once per epoch (MPI rule).  out_ns[0] = total ns on
+// side 0 for `iters` round trips.
+__global__ void pingpong_kernel(pc_prequest_t sendq, pc_prequest_t recvq, int side, int iters, int gran,
+                                unsigned long long *out_ns) {
+  const uint64_t t0 = pc_detail::globaltimer();
+  for (int k = 0; k < iters; ++k) {
+    if (side == 1) {
+      if (threadIdx.x == 0) pc_wait_arrived(recvq, k);
+      __syncwarp();
+    }
+    if (gran == PCAPP_GRAN_THREAD) {
+      if (threadIdx.x == 0) pc_pready(k, sendq);
+    } else {
+      pc_pready_warp(k, sendq);
+    }
+    if (side == 0) {
+      if (threadIdx.x == 0) pc_wait_arrived(recvq, k);
+      __syncwarp();
+    }
+  }
+  if (threadIdx.x == 0) out_ns[0] = pc_detail::globaltimer() - t0;
+}
+
+// Latency floor: the same ping-pong with a bare flag and no library.
+__global__ void bare_pingpong_kernel(uint32_t *my_flag, uint32_t *peer_flag, int side, int iters, uint32_t base,
+                                     unsigned long long *out_ns) {
+  if (threadIdx.x != 0) return;
+  const uint64_t t0 = pc_detail::globaltimer();
+  for (int k = 1; k <= iters; ++k) {
+    const uint32_t v = base + (uint32_t)k;
+    if (side == 1)
+      while (!pc_detail::reached(pc_detail::ld_acquire_sys(my_flag), v)) {
+      }
+    pc_detail::st_release_sys(peer_flag, v);
+    if (side == 0)
+      while (!pc_detail::reached(pc_detail::ld_acquire_sys(my_flag), v)) {
+      }
+  }
+  out_ns[0] = pc_detail::globaltimer() - t0;
+}
+
+}  // namespace
+
+extern "C" {
+
+int pcapp_vecadd(const float *A, const float *B, float *C, int64_t n, int gran, const pc_prequest_t *preq,
+                 cudaStream_t s) {
+  if (n % 2) return -1;
+  const int64_t n2 = n / 2;
+  const int64_t blocks = (n2 + 1023) / 1024;
+  pc_prequest_t q{};
+  if (preq) q = *preq;
+  if (gran != PCAPP_GRAN_NONE && !preq) return -1;
+  vecadd_kernel<<<(unsigned)blocks, 1024, 0, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, gran, q);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_produce(void *dst, const void *src, int partitions, int64_t part_bytes, int gran, int order_stride,
+                  int blocks, const pc_prequest_t *preq, cudaStream_t s) {
+  if (!preq || partitions < 1) return -1;
+  if (blocks <= 0) blocks = partitions < 1184 ? partitions : 1184;
+  produce_kernel<<<blocks, 512, 0, s>>>((uint8_t *)dst, (const uint8_t *)src, partitions, part_bytes, gran,
+                                        order_stride < 1 ? 1 : order_stride, *preq);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_check_recv(const pc_prequest_t *preq, const void *recvbuf, void *out, int partitions, int64_t part_bytes,
+                     int blocks, int *status, cudaStream_t s) {
+  if (!preq) return -1;
+  check_recv_kernel<<<blocks, 256, 0, s>>>(*preq, (const uint8_t *)recvbuf, (uint8_t *)out, partitions, part_bytes,
+                                           status);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_pingpong(const pc_prequest_t *sendq, const pc_prequest_t *recvq, int side, int iters, int gran,
+                   unsigned long long *out_ns, cudaStream_t s) {
+  if (!sendq || !recvq) return -1;
+  pingpong_kernel<<<1, 32, 0, s>>>(*sendq, *recvq, side, iters, gran, out_ns);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_bare_pingpong(uint32_t *my_flag, uint32_t *peer_flag, int side, int iters, uint32_t base,
+                        unsigned long long *out_ns, cudaStream_t s) {
+  bare_pingpong_kernel<<<1, 32, 0, s>>>(my_flag, peer_flag, side, iters, base, out_ns);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+size_t pcapp_prequest_size(void) { return sizeof(pc_prequest_t); }
+
+}  // extern "C"

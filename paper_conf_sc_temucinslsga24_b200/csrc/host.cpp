@@ -1,0 +1,1150 @@
+// libpc host runtime: comm bootstrap, request lifecycle, matching, schedules.
+//
+// Paper mapping (§IV-A/§IV-B):
+//   pc_psend_init / pc_precv_init   MPI_Psend_init / MPI_Precv_init:
+//                                   record parameters only (non-blocking)
+//   pc_start                        MPI_Start: new epoch, stream-ordered
+//   pc_pbuf_prepare                 MPIX_Pbuf_prepare: first
+//                                   call = setup_t exchange + registration (here:
+//                                   all-gather of request records + CUDA IPC
+//                                   handles); every call = ready-to-receive
+//   pc_prequest_create              MPIX_Prequest_create
+//   pc_pallreduce_init              MPIX_Pallreduce_init (Alg 1)
+//   pc_wait                         MPI_Wait (Alg 2 P:L178 runs on the GPU)
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <random>
+#include <string>
+#include <tuple>
+
+#include "pc_internal.h"
+
+namespace pc {
+
+static bool env_flag(const char *n) {
+  const char *v = getenv(n);
+  return v && *v && strcmp(v, "0") != 0;
+}
+static long env_long(const char *n, long dflt) {
+  const char *v = getenv(n);
+  if (!v || !*v) return dflt;
+  return strtol(v, nullptr, 0);
+}
+
+void logf(const char *fmt, ...) {
+  if (!env_flag("PC_DEBUG")) return;
+  va_list ap;
+  va_start(ap, fmt);
+  fprintf(stderr, "[pc] ");
+  vfprintf(stderr, fmt, ap);
+  fprintf(stderr, "\n");
+  va_end(ap);
+}
+
+int cuda_err(cudaError_t e, const char *what) {
+  fprintf(stderr, "[pc] CUDA error %d (%s) in %s\n", (int)e, cudaGetErrorString(e), what);
+  return e == cudaErrorMemoryAllocation ? PC_ERR_NOMEM : PC_ERR_CUDA;
+}
+
+// ------------------------------------------------------------------ driver entry points
+typedef CUresult (*PFN_getAddrRange)(CUdeviceptr *, size_t *, CUdeviceptr);
+typedef CUresult (*PFN_writeValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+static PFN_getAddrRange g_getAddrRange = nullptr;
+static PFN_writeValue32 g_writeValue32 = nullptr;
+static std::once_flag g_drv_once;
+
+static void load_driver_entry_points() {
+  std::call_once(g_drv_once, [] {
+    void *fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      g_getAddrRange = (PFN_getAddrRange)fn;
+    fn = nullptr;
+    if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      g_writeValue32 = (PFN_writeValue32)fn;
+    cudaGetLastError();
+  });
+}
+
+bool memops_available() {
+  load_driver_entry_points();
+  return g_writeValue32 != nullptr && !env_flag("PC_NO_MEMOPS");
+}
+
+int stream_write_u32(Comm *c, cudaStream_t s, uint32_t *addr, uint32_t value) {
+  if (c->memops) {
+    CUresult r = g_writeValue32((CUstream)s, (CUdeviceptr)addr, value, 0 /* with memory barrier */);
+    if (r == CUDA_SUCCESS) return 0;
+    logf("cuStreamWriteValue32 failed (%d); falling back to a 1-thread kernel", (int)r);
+    c->memops = false;
+  }
+  return launch_set_word(addr, value, s);
+}
+
+// ------------------------------------------------------------------ local groups
+static int local_allgather_impl(LocalGroup *g, int rank, const void *send, size_t nbytes, void *recv) {
+  std::unique_lock<std::mutex> lk(g->mu);
+  g->cv.wait(lk, [&] { return g->readers_left == 0; });  // previous round fully consumed
+  if (g->arrived == 0) {
+    g->nbytes = nbytes;
+    g->buf.assign(nbytes * (size_t)g->size, 0);
+  } else if (g->nbytes != nbytes) {
+    return PC_ERR_ARG;
+  }
+  memcpy(g->buf.data() + (size_t)rank * nbytes, send, nbytes);
+  const uint64_t gen = g->generation;
+  if (++g->arrived == g->size) {
+    g->generation++;
+    g->arrived = 0;
+    g->readers_left = g->size;
+    g->cv.notify_all();
+  } else {
+    g->cv.wait(lk, [&] { return g->generation != gen; });
+  }
+  memcpy(recv, g->buf.data(), nbytes * (size_t)g->size);
+  if (--g->readers_left == 0) g->cv.notify_all();
+  return 0;
+}
+
+// ------------------------------------------------------------------ bootstrap helpers
+int allgather(Comm *c, const void *send, size_t nbytes, void *recv) {
+  if (c->size == 1) {
+    memcpy(recv, send, nbytes);
+    return 0;
+  }
+  int r = c->ag(send, nbytes, recv, c->ag_ctx);
+  return r == 0 ? 0 : PC_ERR_ARG;
+}
+
+static bool need_ipc(Comm *c) {
+  if (c->dry) return false;
+  for (int q = 0; q < c->size; ++q)
+    if (q != c->rank && !c->same_proc[q]) return true;
+  return false;
+}
+
+int export_ptr(Comm *c, const void *p, uint64_t bytes, ShareRec *out) {
+  memset(out, 0, sizeof(*out));
+  out->raw = (uint64_t)(uintptr_t)p;
+  out->bytes = bytes;
+  if (!p || !need_ipc(c)) return 0;
+  load_driver_entry_points();
+  if (!g_getAddrRange) return PC_ERR_UNSUPPORTED;
+  CUdeviceptr base = 0;
+  size_t sz = 0;
+  if (g_getAddrRange(&base, &sz, (CUdeviceptr)p) != CUDA_SUCCESS) {
+    fprintf(stderr, "[pc] cuMemGetAddressRange failed for %p (not device memory?)\n", p);
+    return PC_ERR_ARG;
+  }
+  out->off = (uint64_t)((uintptr_t)p - (uintptr_t)base);
+  cudaError_t e = cudaIpcGetMemHandle(&out->h, (void *)base);
+  if (e != cudaSuccess) {
+    fprintf(stderr,
+            "[pc] cudaIpcGetMemHandle failed (%s): buffers must come from cudaMalloc / the torch caching "
+            "allocator without expandable segments\n",
+            cudaGetErrorString(e));
+    cudaGetLastError();
+    return PC_ERR_ARG;
+  }
+  return 0;
+}
+
+int import_ptr(Comm *c, int owner, const ShareRec &s, void **out) {
+  if (c->dry || s.raw == 0) {
+    *out = (void *)(uintptr_t)s.raw;
+    return 0;
+  }
+  if (owner == c->rank || c->same_proc[owner]) {
+    *out = (void *)(uintptr_t)s.raw;
+    return 0;
+  }
+  std::string key((const char *)&s.h, sizeof(s.h));
+  auto it = c->ipc_open.find(key);
+  void *base = nullptr;
+  if (it != c->ipc_open.end()) {
+    base = it->second;
+  } else {
+    PC_CUDA(cudaIpcOpenMemHandle(&base, s.h, cudaIpcMemLazyEnablePeerAccess));
+    c->ipc_open[key] = base;
+  }
+  *out = (uint8_t *)base + s.off;
+  return 0;
+}
+
+static uint64_t process_token() {
+  static uint64_t tok = [] {
+    std::random_device rd;
+    uint64_t t = ((uint64_t)rd() << 32) ^ rd();
+    t ^= (uint64_t)std::chrono::steady_clock::now().time_since_epoch().count();
+    t ^= (uint64_t)(uintptr_t)&tok;
+    return t ? t : 1;
+  }();
+  return tok;
+}
+
+// ------------------------------------------------------------------ schedules (host, pure)
+static int mod(int a, int p) { return ((a % p) + p) % p; }
+
+// Alg 1 with reading R1 (exclusive loop bound: 2(P-1) steps).
+static int ring_rows(int P, int r, int32_t *out) {
+  const int n = 2 * (P - 1);
+  for (int i = 0; i < n; ++i) {
+    int32_t *row = out + 5 * i;
+    row[0] = mod(r - 1, P);
+    row[1] = mod(r + 2 * P - i, P);
+    row[2] = i < P - 1 ? 1 : 0;
+    row[3] = mod(r + 1, P);
+    row[4] = mod(r + 2 * P - i - 1, P);
+  }
+  return n;
+}
+
+static int log2_exact(int P) {
+  int k = 0;
+  while ((1 << k) < P) ++k;
+  return (1 << k) == P ? k : -1;
+}
+
+static int rd_rows(int P, int r, int32_t *out) {
+  const int n = log2_exact(P);
+  if (n < 0) return PC_ERR_ARG;
+  for (int k = 0; k < n; ++k) {
+    int32_t *row = out + 5 * k;
+    row[0] = r ^ (1 << k);
+    row[1] = -1;
+    row[2] = 1;
+    row[3] = r ^ (1 << k);
+    row[4] = -1;
+  }
+  return n;
+}
+
+// Reading R4: q = ceil(L / (4P)) * 4 elements per chunk (16-byte multiples);
+// trailing chunks may be short or empty.
+static int64_t chunk_q(int64_t L, int P) { return ((L + 4LL * P - 1) / (4LL * P)) * 4; }
+
+// Slicing policy (deterministic from arguments every rank shares): split a
+// length of `len` elements into ns slices of qs elements (multiple of 4), with
+// about `target_units / nparts` slices per part but none below min_elems.
+static void choose_slices(int64_t len, int nparts, int target_units, int64_t min_elems, int *ns_out,
+                          int64_t *qs_out) {
+  long fixed = env_long("PC_SLICE_BYTES", 0);
+  int64_t qs;
+  if (fixed > 0) {
+    qs = std::max<int64_t>(4, (fixed / 4 + 3) / 4 * 4);
+  } else {
+    int64_t by_size = std::max<int64_t>(1, (len + min_elems - 1) / std::max<int64_t>(min_elems, 1));
+    int64_t by_units = std::max<int64_t>(1, target_units / std::max(nparts, 1));
+    int64_t ns = std::min(by_size, by_units);
+    qs = (len + ns - 1) / ns;
+    qs = std::max<int64_t>(4, (qs + 3) / 4 * 4);
+  }
+  int64_t ns = len > 0 ? (len + qs - 1) / qs : 1;
+  *ns_out = (int)std::max<int64_t>(1, ns);
+  *qs_out = qs;
+}
+
+// ------------------------------------------------------------------ request helpers
+static size_t dtype_size(int dt) { return dt == PC_BYTE ? 1 : 4; }
+
+static int alloc_ctrl(Request *q) {
+  Comm *c = q->comm;
+  if (c->dry) return 0;
+  PC_CUDA(cudaSetDevice(c->device));
+  int lo = 0, hi = 0;
+  PC_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+  PC_CUDA(cudaStreamCreateWithPriority(&q->side, cudaStreamNonBlocking, hi));
+  PC_CUDA(cudaEventCreateWithFlags(&q->ev_fork, cudaEventDisableTiming));
+  PC_CUDA(cudaEventCreateWithFlags(&q->ev_done, cudaEventDisableTiming));
+  PC_CUDA(cudaMalloc((void **)&q->ctrl, q->L.words * 4));
+  PC_CUDA(cudaMemsetAsync(q->ctrl, 0, q->L.words * 4, q->side));
+  if (q->staging_bytes) {
+    PC_CUDA(cudaMalloc((void **)&q->staging, q->staging_bytes));
+  }
+  PC_CUDA(cudaStreamSynchronize(q->side));
+  return 0;
+}
+
+static int check_buf(const void *p, uint64_t bytes) {
+  if (bytes == 0) return 0;
+  if (!p) return PC_ERR_ARG;
+  if (((uintptr_t)p) & 15) return PC_ERR_ARG;
+  return 0;
+}
+
+static void fill_prequest(Request *q, pc_prequest_t *o) {
+  memset(o, 0, sizeof(*o));
+  o->kind = (uint32_t)q->kind;
+  o->copy = (uint32_t)q->copy;
+  o->partitions = q->partitions;
+  o->agg = q->agg;
+  o->ntransport = q->ntransport;
+  o->timeout_ms = q->comm->timeout_ms;
+  o->part_bytes = q->part_bytes;
+  o->rank = q->comm->rank;
+  if (!q->ctrl) return;
+  o->epoch = q->ctrl + q->L.epoch;
+  o->cnt = q->ctrl + q->L.cnt;
+  o->ready = q->ctrl + q->L.ready;
+  o->sent = q->ctrl + q->L.sent;
+  o->sbuf = (const uint8_t *)q->sbuf;
+  o->rtr = q->ctrl + q->L.rtr;
+  o->flags = q->ctrl + q->L.flags;
+  o->layout = q->ctrl + q->L.layout;
+  o->done = q->ctrl + q->L.donecnt;
+  o->done_mul = (uint32_t)q->slices;
+  o->err = (int32_t *)(q->ctrl + q->L.err);
+  if (q->kind == PC_KIND_PSEND) {
+    o->peer_rbuf = q->peer_buf;
+    o->peer_flags = q->peer_ctrl ? q->peer_ctrl + q->L.flags : nullptr;
+  }
+}
+
+static int new_request(Comm *c, int kind, pc_request_t *out, Request **rq) {
+  if (!c || !out) return PC_ERR_ARG;
+  Request *q = new Request();
+  q->comm = c;
+  q->kind = kind;
+  q->index = (int)c->reqs.size();
+  c->reqs.push_back(q);
+  *rq = q;
+  *out = (pc_request_t)q;
+  return 0;
+}
+
+static int p2p_init(int kind, const void *sbuf, void *rbuf, int partitions, size_t count, int dtype, int peer,
+                    int tag, Comm *c, pc_request_t *out) {
+  if (!c || !out || partitions < 1 || dtype < 0 || dtype > 2 || peer < 0 || peer >= c->size || tag < 0)
+    return PC_ERR_ARG;
+  const uint64_t bytes = (uint64_t)partitions * count * dtype_size(dtype);
+  if (!c->dry && check_buf(kind == PC_KIND_PSEND ? sbuf : rbuf, bytes)) return PC_ERR_ARG;
+  Request *q;
+  int rc = new_request(c, kind, out, &q);
+  if (rc) return rc;
+  q->sbuf = sbuf;
+  q->rbuf = rbuf;
+  q->partitions = partitions;
+  q->count = count;
+  q->dtype = dtype;
+  q->esize = dtype_size(dtype);
+  q->peer = peer;
+  q->tag = tag;
+  q->part_bytes = count * q->esize;
+  q->total_bytes = bytes;
+  q->seq = c->post_seq[std::make_tuple(kind, peer, tag)]++;
+  q->L.build((size_t)partitions, (size_t)partitions);
+  q->agg = 1;
+  q->ntransport = partitions;
+  return alloc_ctrl(q);
+}
+
+// ------------------------------------------------------------------ exchange (first pbuf_prepare)
+static int make_rec(Request *q, ReqRec *r) {
+  Comm *c = q->comm;
+  memset(r, 0, sizeof(*r));
+  r->kind = q->kind;
+  r->peer = q->peer;
+  r->tag = q->tag;
+  r->partitions = q->partitions;
+  r->count = (int64_t)q->count;
+  r->dtype = q->dtype;
+  r->op = q->op;
+  r->algo = q->algo;
+  r->seq = q->seq;
+  r->owner = c->rank;
+  r->req_index = q->index;
+  int rc = 0;
+  if (q->kind == PC_KIND_PRECV || q->kind == PC_KIND_PALLREDUCE)
+    if ((rc = export_ptr(c, q->rbuf, q->total_bytes, &r->buf))) return rc;
+  if ((rc = export_ptr(c, q->ctrl, q->L.words * 4, &r->ctrl))) return rc;
+  if (q->staging && (rc = export_ptr(c, q->staging, q->staging_bytes, &r->stage))) return rc;
+  return 0;
+}
+
+static const ReqRec *find_rec(const std::vector<ReqRec> &all, int M, int owner, int kind, int peer, int tag,
+                              int seq, const std::vector<int> &counts) {
+  for (int k = 0; k < counts[owner]; ++k) {
+    const ReqRec &r = all[(size_t)owner * M + k];
+    if (r.kind == kind && r.peer == peer && r.tag == tag && r.seq == seq) return &r;
+  }
+  return nullptr;
+}
+
+static int exchange_round(Comm *c, Request *target) {
+  std::vector<Request *> pending;
+  for (Request *q : c->reqs)
+    if (q && !q->exchanged) pending.push_back(q);
+  int32_t mine = (int32_t)pending.size();
+  std::vector<int32_t> counts(c->size);
+  int rc = allgather(c, &mine, sizeof(mine), counts.data());
+  if (rc) return rc;
+  int M = 0;
+  for (int v : counts) M = std::max(M, v);
+  if (M == 0) return PC_ERR_STATE;
+  std::vector<ReqRec> my(M), all((size_t)M * c->size);
+  for (size_t k = 0; k < pending.size(); ++k)
+    if ((rc = make_rec(pending[k], &my[k]))) return rc;
+  if ((rc = allgather(c, my.data(), sizeof(ReqRec) * M, all.data()))) return rc;
+  std::vector<int> cnt(counts.begin(), counts.end());
+
+  int target_rc = PC_ERR_MATCH;
+  for (Request *q : pending) {
+    int qrc = 0;
+    if (q->kind == PC_KIND_PSEND || q->kind == PC_KIND_PRECV) {
+      const int want = q->kind == PC_KIND_PSEND ? PC_KIND_PRECV : PC_KIND_PSEND;
+      const ReqRec *m = find_rec(all, M, q->peer, want, c->rank, q->tag, q->seq, cnt);
+      if (!m) {
+        qrc = PC_ERR_MATCH;
+      } else if (m->partitions != q->partitions || m->count != (int64_t)q->count || m->dtype != q->dtype) {
+        fprintf(stderr, "[pc] rank %d: %s to/from %d tag %d: partitions/count/dtype disagree (%d/%lld/%d vs %d/%lld/%d)\n",
+                c->rank, q->kind == PC_KIND_PSEND ? "psend" : "precv", q->peer, q->tag, q->partitions,
+                (long long)q->count, q->dtype, m->partitions, (long long)m->count, m->dtype);
+        qrc = PC_ERR_MATCH;
+        q->exchanged = true;  // matched but incompatible: report, do not retry
+        q->matched = false;
+      } else {
+        void *pctrl = nullptr, *pbuf = nullptr;
+        if ((qrc = import_ptr(c, m->owner, m->ctrl, &pctrl)) == 0) {
+          q->peer_ctrl = (uint32_t *)pctrl;
+          if (q->kind == PC_KIND_PSEND) {
+            qrc = import_ptr(c, m->owner, m->buf, &pbuf);
+            q->peer_buf = (uint8_t *)pbuf;
+          } else {
+            // the receiver is the consumer: it writes ready-to-receive into the sender's rtr[0]
+            q->rtr_targets.push_back({q->peer_ctrl, 0});
+          }
+        }
+        if (qrc == 0) {
+          q->exchanged = true;
+          q->matched = true;
+          q->match_peer_index = m->req_index;
+        }
+      }
+    } else {  // PALLREDUCE: the seq-th allreduce of every rank
+      std::vector<const ReqRec *> peers(c->size, nullptr);
+      for (int r = 0; r < c->size && !qrc; ++r) {
+        const ReqRec *m = find_rec(all, M, r, PC_KIND_PALLREDUCE, -1, 0, q->seq, cnt);
+        if (!m || m->partitions != q->partitions || m->count != (int64_t)q->count || m->dtype != q->dtype ||
+            m->op != q->op || m->algo != q->algo) {
+          fprintf(stderr, "[pc] rank %d: allreduce #%d disagrees with rank %d\n", c->rank, q->seq, r);
+          qrc = PC_ERR_MATCH;
+        }
+        peers[r] = m;
+      }
+      if (!qrc) {
+        const int P = c->size, r = c->rank;
+        auto imp = [&](int who, int slot) -> int {
+          void *b = nullptr, *ct = nullptr, *st = nullptr;
+          int e;
+          if ((e = import_ptr(c, who, peers[who]->buf, &b))) return e;
+          if ((e = import_ptr(c, who, peers[who]->ctrl, &ct))) return e;
+          if ((e = import_ptr(c, who, peers[who]->stage, &st))) return e;
+          q->nb_buf[slot] = (uint8_t *)b;
+          q->nb_ctrl[slot] = (uint32_t *)ct;
+          q->nb_stage[slot] = (uint8_t *)st;
+          return 0;
+        };
+        if (P > 1) {
+          if (q->algo == PC_ALGO_RING) {
+            qrc = imp(mod(r + 1, P), 0);  // O: where this rank's steps land
+            if (!qrc) {
+              // consumer-side RTR: this rank receives from I = r-1, so it
+              // tells I (rtr slot 0 of I's control block) when it is ready
+              void *ict = nullptr;
+              qrc = import_ptr(c, mod(r - 1, P), peers[mod(r - 1, P)]->ctrl, &ict);
+              if (!qrc) q->rtr_targets.push_back({(uint32_t *)ict, 0});
+            }
+          } else {
+            for (int k = 0; k < q->nsteps && !qrc; ++k) {
+              qrc = imp(r ^ (1 << k), k);
+              if (!qrc) q->rtr_targets.push_back({q->nb_ctrl[k], k});
+            }
+          }
+        }
+        if (!qrc) {
+          q->exchanged = true;
+          q->matched = true;
+        }
+      } else {
+        q->exchanged = true;
+      }
+    }
+    if (q == target) target_rc = qrc;
+    if (qrc) logf("rank %d: request %d exchange rc=%d", c->rank, q->index, qrc);
+  }
+  if (!c->dry) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_err(e, "exchange");
+  }
+  return target_rc;
+}
+
+// ------------------------------------------------------------------ engine launch
+static int maybe_launch_engine(Request *q) {
+  Comm *c = q->comm;
+  if (c->dry || !q->active || !q->exchanged || !q->matched || q->engine_launched) return 0;
+  const bool needs = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
+  if (!needs) return 0;
+  PC_CUDA(cudaSetDevice(c->device));
+  PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+  PC_CUDA(cudaStreamWaitEvent(q->side, q->ev_fork, 0));
+  int rc = 0;
+  int32_t *err = (int32_t *)(q->ctrl + q->L.err);
+  if (q->kind == PC_KIND_PALLREDUCE) {
+    const int P = c->size;
+    if (q->algo == PC_ALGO_RING) {
+      RingArgs a{};
+      a.e = q->epoch;
+      a.P = P;
+      a.r = c->rank;
+      a.Np = q->partitions;
+      a.ns = q->slices;
+      a.nunits = q->partitions * q->slices;
+      a.op = q->op;
+      a.dtype = q->dtype;
+      a.L = (int64_t)q->count;
+      a.q = q->chunk_elems;
+      a.qs = q->slice_elems;
+      a.sendbuf = (const uint8_t *)q->sbuf;
+      a.recvbuf = (uint8_t *)q->rbuf;
+      a.staging = q->staging;
+      a.flags = q->ctrl + q->L.flags;
+      a.ready = q->ctrl + q->L.ready;
+      a.rtr = q->ctrl + q->L.rtr;
+      a.done = q->ctrl + q->L.donecnt;
+      a.o_staging = q->nb_stage[0];
+      a.o_recvbuf = q->nb_buf[0];
+      a.o_flags = q->nb_ctrl[0] ? q->nb_ctrl[0] + q->L.flags : nullptr;
+      a.err = err;
+      a.timeout_ms = c->timeout_ms;
+      rc = launch_ring_engine(a, q->engine_warps, q->side);
+    } else {
+      RdArgs a{};
+      a.e = q->epoch;
+      a.P = P;
+      a.r = c->rank;
+      a.Np = q->partitions;
+      a.ns = q->slices;
+      a.nunits = q->partitions * q->slices;
+      a.op = q->op;
+      a.dtype = q->dtype;
+      a.nsteps = q->nsteps;
+      a.L = (int64_t)q->count;
+      a.qs = q->slice_elems;
+      a.sendbuf = (const uint8_t *)q->sbuf;
+      a.recvbuf = (uint8_t *)q->rbuf;
+      a.staging = q->staging;
+      a.flags = q->ctrl + q->L.flags;
+      a.ready = q->ctrl + q->L.ready;
+      a.rtr = q->ctrl + q->L.rtr;
+      a.done = q->ctrl + q->L.donecnt;
+      const int64_t slot_bytes = (int64_t)q->partitions * (int64_t)q->count * 4;
+      for (int k = 0; k < q->nsteps; ++k) {
+        a.p_staging[k] = q->nb_stage[k] + (int64_t)k * slot_bytes;
+        a.p_flags[k] = q->nb_ctrl[k] + q->L.flags;
+      }
+      a.err = err;
+      a.timeout_ms = c->timeout_ms;
+      rc = launch_rd_engine(a, q->engine_warps, q->side);
+    }
+  } else {
+    P2pEngineArgs a{};
+    a.e = q->epoch;
+    a.nt = q->ntransport;
+    a.agg = q->agg;
+    a.ns = q->slices;
+    a.nunits = q->ntransport * q->slices;
+    a.part_bytes = q->part_bytes;
+    a.slice_bytes = (uint64_t)q->slice_elems;
+    a.partitions = q->partitions;
+    a.sbuf = (const uint8_t *)q->sbuf;
+    a.peer_rbuf = q->peer_buf;
+    a.peer_flags = q->peer_ctrl + q->L.flags;
+    a.ready = q->ctrl + q->L.ready;
+    a.rtr = q->ctrl + q->L.rtr;
+    a.donecnt = q->ctrl + q->L.donecnt;
+    a.sent = q->ctrl + q->L.sent;
+    a.err = err;
+    a.timeout_ms = c->timeout_ms;
+    rc = launch_p2p_engine(a, q->engine_warps, q->side);
+  }
+  if (rc) return rc;
+  PC_CUDA(cudaEventRecord(q->ev_done, q->side));
+  q->engine_launched = true;
+  return 0;
+}
+
+static int read_error(Request *q, int *code, int *part) {
+  *code = 0;
+  *part = 0;
+  if (q->comm->dry || !q->ctrl) return 0;
+  int32_t h[2] = {0, 0};
+  PC_CUDA(cudaMemcpyAsync(h, q->ctrl + q->L.err, sizeof(h), cudaMemcpyDeviceToHost, q->side));
+  PC_CUDA(cudaStreamSynchronize(q->side));
+  *code = h[0];
+  *part = h[1];
+  return 0;
+}
+
+static int error_rc(Request *q) {
+  int code, part;
+  int rc = read_error(q, &code, &part);
+  if (rc) return rc;
+  if (code == 0) return 0;
+  fprintf(stderr, "[pc] rank %d request %d: device error %d (partition %d)\n", q->comm->rank, q->index, code, part);
+  return code == PC_ERR_TIMEOUT ? PC_ERR_TIMEOUT : PC_ERR_DEVICE;
+}
+
+}  // namespace pc
+
+using namespace pc;
+
+// ====================================================================== C ABI
+extern "C" {
+
+const char *pc_version(void) { return "libpc 0.1 (sm_100a)"; }
+
+const char *pc_strerror(int err) {
+  switch (err) {
+    case PC_SUCCESS: return "success";
+    case PC_ERR_ARG: return "invalid argument";
+    case PC_ERR_CUDA: return "CUDA error";
+    case PC_ERR_STATE: return "invalid request state";
+    case PC_ERR_MATCH: return "send/recv or collective parameters do not match";
+    case PC_ERR_TIMEOUT: return "device wait timed out";
+    case PC_ERR_DEVICE: return "device-side error (bad partition / duplicate Pready)";
+    case PC_ERR_NOMEM: return "out of memory";
+    case PC_ERR_UNSUPPORTED: return "unsupported";
+    default: return "unknown error";
+  }
+}
+
+size_t pc_prequest_size(void) { return sizeof(pc_prequest_t); }
+
+int pc_local_group_create(int size, pc_local_group_t *group) {
+  if (size < 1 || !group) return PC_ERR_ARG;
+  LocalGroup *g = new LocalGroup();
+  g->size = size;
+  g->ctxs.resize(size);
+  for (int r = 0; r < size; ++r) g->ctxs[r] = {g, r};
+  *group = (pc_local_group_t)g;
+  return 0;
+}
+
+int pc_local_group_destroy(pc_local_group_t group) {
+  delete (LocalGroup *)group;
+  return 0;
+}
+
+void *pc_local_group_ctx(pc_local_group_t group, int rank) {
+  LocalGroup *g = (LocalGroup *)group;
+  if (!g || rank < 0 || rank >= g->size) return nullptr;
+  return &g->ctxs[rank];
+}
+
+int pc_local_allgather(const void *send, size_t nbytes, void *recv, void *ctx) {
+  auto *p = (std::pair<LocalGroup *, int> *)ctx;
+  if (!p) return PC_ERR_ARG;
+  return local_allgather_impl(p->first, p->second, send, nbytes, recv);
+}
+
+int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void *ctx, pc_comm_t *comm) {
+  if (!comm || size < 1 || size > kMaxRanks || rank < 0 || rank >= size || (size > 1 && !ag)) return PC_ERR_ARG;
+  Comm *c = new Comm();
+  c->rank = rank;
+  c->size = size;
+  c->device = cuda_device;
+  c->dry = cuda_device < 0;
+  c->ag = ag;
+  c->ag_ctx = ctx;
+  c->timeout_ms = (uint32_t)env_long("PC_TIMEOUT_MS", 20000);
+  RankRec me{};
+  me.magic = 0x50432431u;
+  me.rank = rank;
+  me.size = size;
+  me.device = cuda_device;
+  me.dry = c->dry;
+  me.pid = (int64_t)getpid();
+  me.proc_token = process_token();
+  if (!c->dry) {
+    cudaError_t e = cudaSetDevice(cuda_device);
+    if (e != cudaSuccess) {
+      delete c;
+      return cuda_err(e, "cudaSetDevice");
+    }
+    cudaFree(nullptr);
+    cudaDeviceProp prop;
+    e = cudaGetDeviceProperties(&prop, cuda_device);
+    if (e != cudaSuccess) {
+      delete c;
+      return cuda_err(e, "cudaGetDeviceProperties");
+    }
+    memcpy(me.uuid, &prop.uuid, 16);
+    me.sms = prop.multiProcessorCount;
+    int occ = 0;
+    int rc = engine_occupancy_ctas_per_sm(&occ);
+    if (rc) {
+      delete c;
+      return rc;
+    }
+    const int want = (int)env_long("PC_ENGINE_CTAS_PER_SM", 2);
+    me.engine_warps = me.sms * std::max(1, std::min(occ, want)) * (kEngineBlock / 32);
+    c->sms = me.sms;
+    c->memops = memops_available();
+  }
+  std::vector<RankRec> all(size);
+  int rc = allgather(c, &me, sizeof(me), all.data());
+  if (rc) {
+    delete c;
+    return rc;
+  }
+  c->ranks = all;
+  c->same_proc.assign(size, false);
+  int ew = INT32_MAX;
+  for (int q = 0; q < size; ++q) {
+    const RankRec &r = all[q];
+    if (r.magic != me.magic || r.size != size || r.rank != q || r.dry != me.dry) {
+      fprintf(stderr, "[pc] comm_create: inconsistent bootstrap record from rank %d\n", q);
+      delete c;
+      return PC_ERR_ARG;
+    }
+    c->same_proc[q] = (r.pid == me.pid && r.proc_token == me.proc_token);
+    if (!c->dry) {
+      int on_dev = 0;
+      for (int k = 0; k < size; ++k)
+        if (memcmp(all[k].uuid, r.uuid, 16) == 0) ++on_dev;
+      ew = std::min(ew, r.engine_warps / std::max(on_dev, 1));
+    }
+  }
+  c->engine_warps = c->dry ? 1184 : std::max(8, (int)env_long("PC_ENGINE_WARPS", ew));
+  if (!c->dry) {
+    for (int q = 0; q < size; ++q) {
+      if (q == rank || !c->same_proc[q] || all[q].device == cuda_device) continue;
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, cuda_device, all[q].device);
+      if (can) {
+        cudaError_t e = cudaDeviceEnablePeerAccess(all[q].device, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) {
+          delete c;
+          return cuda_err(e, "cudaDeviceEnablePeerAccess");
+        }
+        cudaGetLastError();
+      }
+    }
+  }
+  logf("comm rank %d/%d dev %d engine_warps %d memops %d", rank, size, cuda_device, c->engine_warps, (int)c->memops);
+  *comm = (pc_comm_t)c;
+  return 0;
+}
+
+int pc_comm_destroy(pc_comm_t comm) {
+  Comm *c = (Comm *)comm;
+  if (!c) return PC_ERR_ARG;
+  for (Request *q : c->reqs)
+    if (q) return PC_ERR_STATE;  // free requests first
+  if (!c->dry) {
+    cudaSetDevice(c->device);
+    for (auto &kv : c->ipc_open) cudaIpcCloseMemHandle(kv.second);
+  }
+  delete c;
+  return 0;
+}
+
+int pc_comm_rank(pc_comm_t comm, int *rank) {
+  if (!comm || !rank) return PC_ERR_ARG;
+  *rank = ((Comm *)comm)->rank;
+  return 0;
+}
+int pc_comm_size(pc_comm_t comm, int *size) {
+  if (!comm || !size) return PC_ERR_ARG;
+  *size = ((Comm *)comm)->size;
+  return 0;
+}
+int pc_comm_engine_warps(pc_comm_t comm, int *warps) {
+  if (!comm || !warps) return PC_ERR_ARG;
+  *warps = ((Comm *)comm)->engine_warps;
+  return 0;
+}
+
+int pc_psend_init(const void *buf, int partitions, size_t count, pc_dtype_t dtype, int dest, int tag,
+                  pc_comm_t comm, pc_request_t *req) {
+  return p2p_init(PC_KIND_PSEND, buf, nullptr, partitions, count, dtype, dest, tag, (Comm *)comm, req);
+}
+
+int pc_precv_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, int source, int tag, pc_comm_t comm,
+                  pc_request_t *req) {
+  return p2p_init(PC_KIND_PRECV, nullptr, buf, partitions, count, dtype, source, tag, (Comm *)comm, req);
+}
+
+int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
+                       pc_op_t op, pc_algo_t algo, pc_comm_t comm, pc_request_t *req) {
+  Comm *c = (Comm *)comm;
+  if (!c || !req || partitions < 1 || (dtype != PC_INT32 && dtype != PC_FLOAT32) || op < 0 || op > 2 ||
+      algo < 0 || algo > 2)
+    return PC_ERR_ARG;
+  const int P = c->size;
+  const uint64_t bytes = (uint64_t)partitions * count * 4;
+  if (!c->dry && (check_buf(sendbuf, bytes) || check_buf(recvbuf, bytes))) return PC_ERR_ARG;
+  int a = algo;
+  const bool pow2 = log2_exact(P) >= 0;
+  if (a == PC_ALGO_AUTO) {
+    const long rd_max = env_long("PC_RD_MAX_BYTES", 512 * 1024);
+    a = (pow2 && (long long)bytes <= rd_max && P > 1) ? PC_ALGO_RD : PC_ALGO_RING;
+  }
+  if (a == PC_ALGO_RD && !pow2) return PC_ERR_UNSUPPORTED;
+  Request *q;
+  int rc = new_request(c, PC_KIND_PALLREDUCE, req, &q);
+  if (rc) return rc;
+  q->sbuf = sendbuf;
+  q->rbuf = recvbuf;
+  q->partitions = partitions;
+  q->count = count;
+  q->dtype = dtype;
+  q->op = op;
+  q->algo_req = algo;
+  q->algo = a;
+  q->esize = 4;
+  q->peer = -1;
+  q->tag = 0;
+  q->part_bytes = count * 4;
+  q->total_bytes = bytes;
+  q->seq = c->allreduce_seq++;
+  q->agg = 1;
+  q->ntransport = partitions;
+  q->engine_warps = c->engine_warps;
+  const int64_t L = (int64_t)count;
+  const int64_t min_elems = env_long("PC_MIN_SLICE_BYTES", 8192) / 4;
+  if (a == PC_ALGO_RING) {
+    q->nsteps = 2 * (P - 1);
+    q->chunk_elems = chunk_q(L, P);
+    choose_slices(q->chunk_elems, partitions, c->engine_warps, min_elems, &q->slices, &q->slice_elems);
+    q->staging_bytes = P > 1 ? bytes : 0;
+  } else {
+    q->nsteps = log2_exact(P);
+    q->chunk_elems = L;
+    choose_slices(L, partitions, c->engine_warps, min_elems, &q->slices, &q->slice_elems);
+    q->staging_bytes = bytes * (uint64_t)q->nsteps;
+  }
+  const size_t nflags = (size_t)partitions * (size_t)std::max(q->nsteps, 1) * (size_t)q->slices;
+  q->L.build((size_t)partitions, nflags);
+  return alloc_ctrl(q);
+}
+
+int pc_start(pc_request_t req, pc_stream_t stream) {
+  Request *q = (Request *)req;
+  if (!q) return PC_ERR_ARG;
+  if (q->active) return PC_ERR_STATE;
+  Comm *c = q->comm;
+  q->epoch++;
+  q->active = true;
+  q->engine_launched = false;
+  q->prepared_this_epoch = false;
+  q->user_stream = (cudaStream_t)stream;
+  if (c->dry) return 0;
+  PC_CUDA(cudaSetDevice(c->device));
+  return stream_write_u32(c, (cudaStream_t)stream, q->ctrl + q->L.epoch, q->epoch);
+}
+
+int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
+  Request *q = (Request *)req;
+  if (!q) return PC_ERR_ARG;
+  if (!q->active) return PC_ERR_STATE;
+  Comm *c = q->comm;
+  if (!c->dry) PC_CUDA(cudaSetDevice(c->device));
+  if (!q->exchanged) {
+    int rc = exchange_round(c, q);
+    if (rc) return rc;
+  }
+  if (!q->matched) return PC_ERR_MATCH;
+  if (c->dry) return 0;
+  q->user_stream = (cudaStream_t)stream;
+  if (!q->prepared_this_epoch) {
+    for (auto &t : q->rtr_targets) {
+      int rc = stream_write_u32(c, (cudaStream_t)stream, t.first + q->L.rtr + t.second, q->epoch);
+      if (rc) return rc;
+    }
+    q->prepared_this_epoch = true;
+  }
+  return maybe_launch_engine(q);
+}
+
+int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_copy_t copy, pc_prequest_t *out) {
+  Request *q = (Request *)req;
+  if (!q || !out || gran < 0 || gran > 2 || copy < 0 || copy > 1) return PC_ERR_ARG;
+  Comm *c = q->comm;
+  if (!q->exchanged || !q->matched) return PC_ERR_STATE;  // after the first pbuf_prepare (Listing 2)
+  if (q->kind == PC_KIND_PALLREDUCE && aggregation != 1) return PC_ERR_ARG;
+  if (q->kind == PC_KIND_PSEND) {
+    if (aggregation < 1 || aggregation > q->partitions) return PC_ERR_ARG;
+    if (q->has_preq && (aggregation != q->agg)) return PC_ERR_STATE;  // the transport layout is fixed
+    q->agg = aggregation;
+    q->ntransport = (q->partitions + aggregation - 1) / aggregation;
+    q->copy = copy;
+    const uint64_t tb = (uint64_t)aggregation * q->part_bytes;
+    const int64_t min_bytes = env_long("PC_MIN_SLICE_BYTES", 16384);
+    int ns;
+    int64_t sl;
+    // slices in 4-byte "elements" of the transport partition's bytes
+    choose_slices((int64_t)((tb + 3) / 4), q->ntransport, c->engine_warps, std::max<int64_t>(1, min_bytes / 4), &ns,
+                  &sl);
+    q->slices = ns;
+    q->slice_elems = sl * 4;  // bytes per slice
+    q->engine_warps = c->engine_warps;
+    if (!c->dry) {
+      PC_CUDA(cudaSetDevice(c->device));
+      // publish the transport layout (g) in the receiver's control block
+      uint32_t g = (uint32_t)aggregation;
+      PC_CUDA(cudaMemcpyAsync(q->peer_ctrl + q->L.layout, &g, 4, cudaMemcpyHostToDevice, q->side));
+      PC_CUDA(cudaStreamSynchronize(q->side));
+    }
+  } else {
+    q->copy = copy;
+  }
+  q->has_preq = true;
+  fill_prequest(q, out);
+  if (q->kind == PC_KIND_PSEND) return maybe_launch_engine(q);
+  return 0;
+}
+
+int pc_prequest_free(pc_prequest_t *preq) {
+  if (!preq) return PC_ERR_ARG;
+  memset(preq, 0, sizeof(*preq));
+  return 0;
+}
+
+static int wait_common(Request *q, cudaStream_t s, bool host) {
+  Comm *c = q->comm;
+  if (!q->active) return 0;
+  if (c->dry) {
+    q->active = false;
+    return 0;
+  }
+  PC_CUDA(cudaSetDevice(c->device));
+  if (!q->exchanged || !q->matched) return PC_ERR_STATE;
+  int rc = maybe_launch_engine(q);
+  if (rc) return rc;
+  int32_t *err = (int32_t *)(q->ctrl + q->L.err);
+  const bool engine = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->copy == 1);
+  if (engine) {
+    if (!q->engine_launched) return PC_ERR_STATE;
+    if (host) {
+      PC_CUDA(cudaEventSynchronize(q->ev_done));
+    } else {
+      PC_CUDA(cudaStreamWaitEvent(s, q->ev_done, 0));
+    }
+  } else {
+    cudaStream_t ws = host ? q->side : s;
+    if (host) {
+      // ordered after the work the user enqueued before pc_wait on the epoch's stream
+      PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+      PC_CUDA(cudaStreamWaitEvent(q->side, q->ev_fork, 0));
+    }
+    if (q->kind == PC_KIND_PSEND) {
+      if (!q->has_preq) return PC_ERR_STATE;
+      rc = launch_wait_words(q->ctrl + q->L.sent, q->ntransport, q->epoch, nullptr, q->partitions, err, c->timeout_ms,
+                             ws, false);
+    } else {
+      rc = launch_wait_words(q->ctrl + q->L.flags, 0, q->epoch, q->ctrl + q->L.layout, q->partitions, err,
+                             c->timeout_ms, ws, true);
+    }
+    if (rc) return rc;
+    if (host) PC_CUDA(cudaStreamSynchronize(q->side));
+  }
+  q->active = false;
+  if (host) return error_rc(q);
+  return 0;
+}
+
+int pc_wait(pc_request_t req) {
+  Request *q = (Request *)req;
+  if (!q) return PC_ERR_ARG;
+  return wait_common(q, nullptr, true);
+}
+
+int pc_wait_on_stream(pc_request_t req, pc_stream_t stream) {
+  Request *q = (Request *)req;
+  if (!q) return PC_ERR_ARG;
+  return wait_common(q, (cudaStream_t)stream, false);
+}
+
+static int read_words(Request *q, size_t off, size_t n, uint32_t *h) {
+  PC_CUDA(cudaMemcpyAsync(h, q->ctrl + off, n * 4, cudaMemcpyDeviceToHost, q->side));
+  PC_CUDA(cudaStreamSynchronize(q->side));
+  return 0;
+}
+
+static bool reached_h(uint32_t v, uint32_t t) { return (int32_t)(v - t) >= 0; }
+
+int pc_parrived(pc_request_t req, int partition, int *flag) {
+  Request *q = (Request *)req;
+  if (!q || !flag || partition < 0 || partition >= q->partitions) return PC_ERR_ARG;
+  *flag = 0;
+  if (q->comm->dry) return 0;
+  PC_CUDA(cudaSetDevice(q->comm->device));
+  uint32_t v = 0;
+  int rc;
+  if (q->kind == PC_KIND_PALLREDUCE) {
+    if ((rc = read_words(q, q->L.donecnt + partition, 1, &v))) return rc;
+    *flag = reached_h(v, q->epoch * (uint32_t)q->slices);
+  } else if (q->kind == PC_KIND_PRECV) {
+    uint32_t g = 0;
+    if ((rc = read_words(q, q->L.layout, 1, &g))) return rc;
+    if (g == 0) return 0;
+    if ((rc = read_words(q, q->L.flags + partition / g, 1, &v))) return rc;
+    *flag = reached_h(v, q->epoch);
+  } else {
+    if ((rc = read_words(q, q->L.sent + partition / q->agg, 1, &v))) return rc;
+    *flag = reached_h(v, q->epoch);
+  }
+  return 0;
+}
+
+int pc_test(pc_request_t req, int *flag) {
+  Request *q = (Request *)req;
+  if (!q || !flag) return PC_ERR_ARG;
+  *flag = 1;
+  if (!q->active || q->comm->dry) {
+    if (q->active) q->active = false;
+    return 0;
+  }
+  PC_CUDA(cudaSetDevice(q->comm->device));
+  int rc = maybe_launch_engine(q);
+  if (rc) return rc;
+  const bool engine = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->copy == 1);
+  bool done = false;
+  if (engine) {
+    if (!q->engine_launched) {
+      *flag = 0;
+      return 0;
+    }
+    cudaError_t e = cudaEventQuery(q->ev_done);
+    if (e == cudaErrorNotReady) {
+      cudaGetLastError();
+      done = false;
+    } else if (e == cudaSuccess) {
+      done = true;
+    } else {
+      return cuda_err(e, "cudaEventQuery");
+    }
+  } else {
+    int n = q->kind == PC_KIND_PSEND ? q->ntransport : 0;
+    size_t off = q->kind == PC_KIND_PSEND ? q->L.sent : q->L.flags;
+    if (q->kind == PC_KIND_PRECV) {
+      uint32_t g = 0;
+      if ((rc = read_words(q, q->L.layout, 1, &g))) return rc;
+      n = g ? (q->partitions + (int)g - 1) / (int)g : -1;
+    }
+    done = n >= 0;
+    if (n > 0) {
+      std::vector<uint32_t> h((size_t)n);
+      if ((rc = read_words(q, off, (size_t)n, h.data()))) return rc;
+      for (uint32_t v : h) done = done && reached_h(v, q->epoch);
+    }
+  }
+  int erc = error_rc(q);
+  if (erc) {
+    q->active = false;
+    return erc;
+  }
+  *flag = done ? 1 : 0;
+  if (done) q->active = false;
+  return 0;
+}
+
+int pc_pready_range(int lo, int hi, pc_request_t req, pc_stream_t stream) {
+  Request *q = (Request *)req;
+  if (!q || lo < 0 || hi < lo || hi >= q->partitions) return PC_ERR_ARG;
+  if (!q->active) return PC_ERR_STATE;
+  if (q->kind == PC_KIND_PRECV) return PC_ERR_ARG;
+  if (q->comm->dry) return 0;
+  if (q->kind == PC_KIND_PSEND && !q->has_preq) return PC_ERR_STATE;
+  PC_CUDA(cudaSetDevice(q->comm->device));
+  pc_prequest_t p;
+  fill_prequest(q, &p);
+  return launch_pready_range(p, lo, hi, (cudaStream_t)stream);
+}
+
+int pc_pready(int partition, pc_request_t req, pc_stream_t stream) {
+  return pc_pready_range(partition, partition, req, stream);
+}
+
+int pc_request_free(pc_request_t *req) {
+  if (!req || !*req) return PC_ERR_ARG;
+  Request *q = (Request *)*req;
+  if (q->active) return PC_ERR_STATE;
+  Comm *c = q->comm;
+  if (!c->dry) {
+    cudaSetDevice(c->device);
+    if (q->side) cudaStreamSynchronize(q->side);
+    if (q->ctrl) cudaFree(q->ctrl);
+    if (q->staging) cudaFree(q->staging);
+    if (q->side) cudaStreamDestroy(q->side);
+    if (q->ev_fork) cudaEventDestroy(q->ev_fork);
+    if (q->ev_done) cudaEventDestroy(q->ev_done);
+  }
+  c->reqs[q->index] = nullptr;
+  delete q;
+  *req = nullptr;
+  return 0;
+}
+
+int pc_schedule_ring(int P, int r, int32_t *out_rows5) {
+  if (P < 1 || P > kMaxRanks || r < 0 || r >= P || !out_rows5) return PC_ERR_ARG;
+  return ring_rows(P, r, out_rows5);
+}
+
+int pc_schedule_rd(int P, int r, int32_t *out_rows5) {
+  if (P < 1 || P > kMaxRanks || r < 0 || r >= P || !out_rows5) return PC_ERR_ARG;
+  return rd_rows(P, r, out_rows5);
+}
+
+int pc_chunk_bounds(int64_t L, int P, int64_t *out) {
+  if (L < 0 || P < 1 || !out) return PC_ERR_ARG;
+  const int64_t q = chunk_q(L, P);
+  for (int c = 0; c < P; ++c) out[c] = std::min<int64_t>((int64_t)c * q, L);
+  out[P] = L;
+  return 0;
+}
+
+int pc_request_info(pc_request_t req, int *algo, int *slices, int64_t *slice_elems, int *engine_warps) {
+  Request *q = (Request *)req;
+  if (!q) return PC_ERR_ARG;
+  if (algo) *algo = q->algo;
+  if (slices) *slices = q->slices;
+  if (slice_elems) *slice_elems = q->slice_elems;
+  if (engine_warps) *engine_warps = q->engine_warps;
+  return 0;
+}
+
+int pc_request_match(pc_request_t req, int *peer, int *peer_request_index) {
+  Request *q = (Request *)req;
+  if (!q || !peer || !peer_request_index) return PC_ERR_ARG;
+  if (!q->exchanged || !q->matched) return PC_ERR_STATE;
+  *peer = q->peer;
+  *peer_request_index = q->match_peer_index;
+  return 0;
+}
+
+int pc_request_error(pc_request_t req, int *code, int *partition) {
+  Request *q = (Request *)req;
+  if (!q || !code || !partition) return PC_ERR_ARG;
+  if (q->comm->dry) {
+    *code = 0;
+    *partition = 0;
+    return 0;
+  }
+  PC_CUDA(cudaSetDevice(q->comm->device));
+  return read_error(q, code, partition);
+}
+
+}  // extern "C"

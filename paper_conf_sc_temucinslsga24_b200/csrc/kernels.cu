@@ -1,0 +1,403 @@
+// libpc device engines (sm_100a).
+//
+//  ring_engine   partitioned allreduce, Alg 1 schedule progressed
+//                on the GPU: the host Progression Engine of Alg 2
+//                and its per-step reduce kernel + cudaStreamSynchronize
+//                 are replaced by warps that wait on a flag,
+//                reduce the arriving slice in registers and forward it to the
+//                next rank in the same pass (the "computation inside the device
+//                call" the paper proposes).
+//  rd_engine     the same over a recursive-doubling schedule (north_star).
+//  p2p_engine    ENGINE copy mode of partitioned send: poll local ready flags,
+//                push slices over NVLink, publish the receiver's flag.
+//  wait_words    stream-ordered MPI_Wait for send/recv requests.
+//
+// Unit of work = (user partition u, slice s) handled by ONE warp through all
+// steps of the schedule ("each partition independently executes that
+// schedule").  Warps take units in increasing order, x = gw, gw+W, ...
+// with W identical on every rank (agreed at comm creation), so the dependency
+// (unit x, step i) at rank r -> (unit x, step i-1) at rank r-1 can never form a
+// cycle while all engine warps are resident.
+#include <cuda_runtime.h>
+
+#include "pc_device.cuh"
+#include "pc_internal.h"
+
+namespace pc {
+namespace {
+
+using namespace pc_detail;
+
+// Warp-wide bounded wait on a flag word; lane 0 polls, the warp follows.
+template <bool SYS>
+__device__ __forceinline__ bool warp_wait(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo,
+                                          int part) {
+  bool ok = true;
+  if ((threadIdx.x & 31) == 0) ok = spin_geq<SYS>(p, target, err, tmo, part);
+  ok = __shfl_sync(0xffffffffu, ok, 0);
+  __syncwarp();
+  return ok;
+}
+
+// Publish: every lane's (peer) stores are made visible at system scope, then
+// lane 0 stores the epoch into the consumer's flag.
+__device__ __forceinline__ void warp_signal(uint32_t *flag, uint32_t e) {
+  fence_sys();
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) st_relaxed_sys(flag, e);
+}
+
+template <int DT, int OP>
+struct Op;
+template <int OP>
+struct Op<0, OP> {  // int32: sum wraps mod 2^32
+  using T = int32_t;
+  static __device__ __forceinline__ int32_t f(int32_t a, int32_t b) {
+    if (OP == 0) return (int32_t)((uint32_t)a + (uint32_t)b);
+    if (OP == 1) return a > b ? a : b;
+    return a < b ? a : b;
+  }
+};
+template <int OP>
+struct Op<1, OP> {  // fp32: one IEEE add, round to nearest even, no contraction
+  using T = float;
+  static __device__ __forceinline__ float f(float a, float b) {
+    if (OP == 0) return __fadd_rn(a, b);
+    if (OP == 1) return fmaxf(a, b);
+    return fminf(a, b);
+  }
+};
+
+template <int DT, int OP>
+__device__ __forceinline__ uint4 vop(uint4 a, uint4 b) {
+  using O = Op<DT, OP>;
+  using T = typename O::T;
+  uint4 r;
+  T *ra = reinterpret_cast<T *>(&r);
+  const T *pa = reinterpret_cast<const T *>(&a);
+  const T *pb = reinterpret_cast<const T *>(&b);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) ra[j] = O::f(pa[j], pb[j]);
+  return r;
+}
+
+// out1[k] (and out2[k]) = local[k] ⊕ incoming[k], k < n elements, by one warp.
+template <int DT, int OP>
+__device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *local, const void *incoming,
+                                            int64_t n) {
+  using O = Op<DT, OP>;
+  using T = typename O::T;
+  const uint32_t lane = threadIdx.x & 31;
+  const uintptr_t al = reinterpret_cast<uintptr_t>(out1) | reinterpret_cast<uintptr_t>(out2) |
+                       reinterpret_cast<uintptr_t>(local) | reinterpret_cast<uintptr_t>(incoming);
+  int64_t done = 0;
+  if ((al & 15) == 0) {
+    const int64_t nv = n >> 2;
+    const uint4 *a = reinterpret_cast<const uint4 *>(local);
+    const uint4 *b = reinterpret_cast<const uint4 *>(incoming);
+    uint4 *o1 = reinterpret_cast<uint4 *>(out1);
+    uint4 *o2 = reinterpret_cast<uint4 *>(out2);
+    int64_t k = lane;
+    for (; k + 96 < nv; k += 128) {
+      uint4 a0 = __ldcg(a + k), a1 = __ldcg(a + k + 32), a2 = __ldcg(a + k + 64), a3 = __ldcg(a + k + 96);
+      uint4 b0 = __ldcg(b + k), b1 = __ldcg(b + k + 32), b2 = __ldcg(b + k + 64), b3 = __ldcg(b + k + 96);
+      uint4 r0 = vop<DT, OP>(a0, b0), r1 = vop<DT, OP>(a1, b1), r2 = vop<DT, OP>(a2, b2),
+            r3 = vop<DT, OP>(a3, b3);
+      o1[k] = r0;
+      o1[k + 32] = r1;
+      o1[k + 64] = r2;
+      o1[k + 96] = r3;
+      if (out2) {
+        o2[k] = r0;
+        o2[k + 32] = r1;
+        o2[k + 64] = r2;
+        o2[k + 96] = r3;
+      }
+    }
+    for (; k < nv; k += 32) {
+      uint4 r0 = vop<DT, OP>(__ldcg(a + k), __ldcg(b + k));
+      o1[k] = r0;
+      if (out2) o2[k] = r0;
+    }
+    done = nv << 2;
+  }
+  const T *a = reinterpret_cast<const T *>(local);
+  const T *b = reinterpret_cast<const T *>(incoming);
+  T *o1 = reinterpret_cast<T *>(out1);
+  T *o2 = reinterpret_cast<T *>(out2);
+  for (int64_t k = done + lane; k < n; k += 32) {
+    const T r = O::f(__ldcg(a + k), __ldcg(b + k));
+    o1[k] = r;
+    if (o2) o2[k] = r;
+  }
+}
+
+__device__ __forceinline__ void warp_copy(void *dst, const void *src, int64_t nbytes) {
+  copy_bytes(reinterpret_cast<uint8_t *>(dst), reinterpret_cast<const uint8_t *>(src), (uint64_t)nbytes,
+             threadIdx.x & 31, 32);
+}
+
+__device__ __forceinline__ int modp(int a, int p) { return ((a % p) + p) % p; }
+
+// ---------------------------------------------------------------------------
+// Ring (Alg 1).  Paper indexing: at step i rank r sends chunk R_i = r - i and
+// receives chunk A_i = r - i - 1 (mod P).  Fused engine step E_i (i >= 1)
+// consumes the arrival of step i-1 (chunk A_{i-1} = R_i) and sends step i:
+//   1 <= i <= P-2 : acc = send[c] ⊕ staging[c]  -> O.staging[c]        (RS)
+//   i  = P-1      : acc = send[c] ⊕ staging[c]  -> recv[c], O.recv[c]  (final)
+//   P <= i <= 2P-3:        recv[c]              -> O.recv[c]           (AG)
+// E_0 sends send[r] -> O.staging[r]; completion waits for step 2P-3.
+// Operand order local ⊕ incoming (reading R5); flags are per (u, step, slice)
+// (reading R3) and hold epoch values, so they are never reset.
+// ---------------------------------------------------------------------------
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) ring_engine(RingArgs a) {
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int W = (gridDim.x * blockDim.x) >> 5;
+  const int P = a.P, r = a.r, NS = 2 * (P - 1);
+  const uint32_t e = a.e;
+  const int64_t es = 4;
+  bool rtr_ok = false;
+  for (int x = gw; x < a.nunits; x += W) {
+    const int u = x / a.ns, s = x % a.ns;
+    const int64_t base = (int64_t)u * a.L;
+    if (!warp_wait<false>(a.ready + u, e, a.err, a.timeout_ms, u)) return;
+    if (P == 1) {
+      const int64_t lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
+      if (hi > lo && a.sendbuf != a.recvbuf)
+        warp_copy(a.recvbuf + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
+      __syncwarp();
+      if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+      continue;
+    }
+    if (!rtr_ok) {
+      if (!warp_wait<true>(a.rtr, e, a.err, a.timeout_ms, -1)) return;
+      rtr_ok = true;
+    }
+    const int64_t fbase = (int64_t)u * NS * a.ns + s;  // flag (u, i, s) = fbase + i * ns
+    // E_0: the user's Pready of step S_0
+    {
+      const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
+      const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
+      if (hi > lo) warp_copy(a.o_staging + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
+      warp_signal(a.o_flags + fbase, e);
+    }
+    for (int i = 1; i <= 2 * P - 3; ++i) {
+      const int c = modp(r - i, P);
+      if (!warp_wait<true>(a.flags + fbase + (int64_t)(i - 1) * a.ns, e, a.err, a.timeout_ms, u)) return;
+      const int64_t c_lo = min((int64_t)c * a.q, a.L), c_hi = min((int64_t)(c + 1) * a.q, a.L);
+      const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
+      const int64_t n = hi > lo ? hi - lo : 0;
+      const int64_t off = (base + lo) * es;
+      if (n) {
+        if (i <= P - 2)
+          warp_reduce<DT, OP>(a.o_staging + off, nullptr, a.sendbuf + off, a.staging + off, n);
+        else if (i == P - 1)
+          warp_reduce<DT, OP>(a.recvbuf + off, a.o_recvbuf + off, a.sendbuf + off, a.staging + off, n);
+        else
+          warp_copy(a.o_recvbuf + off, a.recvbuf + off, n * es);
+      }
+      warp_signal(a.o_flags + fbase + (int64_t)i * a.ns, e);
+    }
+    if (!warp_wait<true>(a.flags + fbase + (int64_t)(2 * P - 3) * a.ns, e, a.err, a.timeout_ms, u)) return;
+    if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Recursive doubling: step k exchanges the whole slice with partner r ^ 2^k
+// (its staging slot k); acc_{k+1} = acc_k ⊕ in_k is written to recv (the
+// accumulator) and pushed to the next partner in the same pass.
+// ---------------------------------------------------------------------------
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) rd_engine(RdArgs a) {
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int W = (gridDim.x * blockDim.x) >> 5;
+  const int NS = a.nsteps;
+  const uint32_t e = a.e;
+  const int64_t es = 4;
+  const int64_t stride = (int64_t)a.Np * a.L * es;  // bytes per staging slot
+  uint32_t rtr_ok = 0;
+  for (int x = gw; x < a.nunits; x += W) {
+    const int u = x / a.ns, s = x % a.ns;
+    const int64_t lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
+    const int64_t n = hi > lo ? hi - lo : 0;
+    const int64_t off = ((int64_t)u * a.L + lo) * es;
+    if (!warp_wait<false>(a.ready + u, e, a.err, a.timeout_ms, u)) return;
+    if (NS == 0) {
+      if (n && a.sendbuf != a.recvbuf) warp_copy(a.recvbuf + off, a.sendbuf + off, n * es);
+      __syncwarp();
+      if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+      continue;
+    }
+    auto fidx = [&](int k) { return ((int64_t)u * NS + k) * a.ns + s; };
+    if (!(rtr_ok & 1u)) {
+      if (!warp_wait<true>(a.rtr + 0, e, a.err, a.timeout_ms, -1)) return;
+      rtr_ok |= 1u;
+    }
+    if (n) warp_copy(a.p_staging[0] + off, a.sendbuf + off, n * es);
+    warp_signal(a.p_flags[0] + fidx(0), e);
+    for (int k = 0; k < NS; ++k) {
+      if (!warp_wait<true>(a.flags + fidx(k), e, a.err, a.timeout_ms, u)) return;
+      const uint8_t *acc = (k == 0) ? a.sendbuf : a.recvbuf;
+      const uint8_t *in = a.staging + (int64_t)k * stride;
+      if (k < NS - 1) {
+        if (!(rtr_ok & (1u << (k + 1)))) {
+          if (!warp_wait<true>(a.rtr + k + 1, e, a.err, a.timeout_ms, -1)) return;
+          rtr_ok |= 1u << (k + 1);
+        }
+        if (n) warp_reduce<DT, OP>(a.recvbuf + off, a.p_staging[k + 1] + off, acc + off, in + off, n);
+        warp_signal(a.p_flags[k + 1] + fidx(k + 1), e);
+      } else {
+        if (n) warp_reduce<DT, OP>(a.recvbuf + off, nullptr, acc + off, in + off, n);
+        __syncwarp();
+      }
+    }
+    if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// ENGINE copy mode of partitioned send: unit = (transport partition t, slice s).
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int W = (gridDim.x * blockDim.x) >> 5;
+  const uint32_t e = a.e;
+  bool rtr_ok = false;
+  for (int x = gw; x < a.nunits; x += W) {
+    const int t = x / a.ns, s = x % a.ns;
+    if (!warp_wait<false>(a.ready + t, e, a.err, a.timeout_ms, t)) return;
+    if (!rtr_ok) {
+      if (!warp_wait<true>(a.rtr, e, a.err, a.timeout_ms, -1)) return;
+      rtr_ok = true;
+    }
+    const int rem = a.partitions - t * a.agg;
+    const uint64_t len = (uint64_t)(rem < a.agg ? rem : a.agg) * a.part_bytes;
+    const uint64_t off = (uint64_t)t * a.agg * a.part_bytes;
+    const uint64_t slo = (uint64_t)s * a.slice_bytes;
+    const uint64_t n = slo < len ? min(a.slice_bytes, len - slo) : 0;
+    if (n) warp_copy(a.peer_rbuf + off + slo, a.sbuf + off + slo, (int64_t)n);
+    fence_sys();
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) {
+      const uint32_t old = atom_add_acq_rel_gpu(a.donecnt + t, 1);
+      if (old + 1 == e * (uint32_t)a.ns) {
+        st_relaxed_sys(a.peer_flags + t, e);
+        st_release_gpu(a.sent + t, e);
+      }
+    }
+  }
+}
+
+__global__ void wait_words_kernel(const uint32_t *words, int n, uint32_t target, const uint32_t *layout,
+                                  int partitions, int32_t *err, uint32_t tmo, int sys) {
+  __shared__ int s_n;
+  if (threadIdx.x == 0) {
+    int nn = n;
+    if (layout) {
+      // receiver: the sender publishes g at pc_prequest_create
+      const uint64_t t0 = globaltimer();
+      uint32_t g;
+      while ((g = *(const volatile uint32_t *)layout) == 0) {
+        if (aborted(err)) break;
+        if (tmo && globaltimer() - t0 > (uint64_t)tmo * 1000000ull) {
+          set_error(err, PC_DEV_ERR_TIMEOUT, -2);
+          break;
+        }
+        __nanosleep(256);
+      }
+      nn = g ? (partitions + (int)g - 1) / (int)g : 0;
+    }
+    s_n = nn;
+  }
+  __syncthreads();
+  const int nn = s_n;
+  for (int i = threadIdx.x; i < nn; i += blockDim.x) {
+    bool ok = sys ? spin_geq<true>(words + i, target, err, tmo, i) : spin_geq<false>(words + i, target, err, tmo, i);
+    if (!ok) break;
+  }
+}
+
+__global__ void set_word_kernel(uint32_t *addr, uint32_t v) { st_release_sys(addr, v); }
+
+__global__ void pready_range_kernel(pc_prequest_t q, int lo, int hi) {
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int W = (gridDim.x * blockDim.x) >> 5;
+  for (int p = lo + gw; p <= hi; p += W) pc_pready_warp(p, q);
+}
+
+template <typename F>
+int dispatch(int dtype, int op, F f) {
+  if (dtype == PC_INT32) {
+    if (op == PC_OP_SUM) return f(std::integral_constant<int, 0>(), std::integral_constant<int, 0>());
+    if (op == PC_OP_MAX) return f(std::integral_constant<int, 0>(), std::integral_constant<int, 1>());
+    return f(std::integral_constant<int, 0>(), std::integral_constant<int, 2>());
+  }
+  if (op == PC_OP_SUM) return f(std::integral_constant<int, 1>(), std::integral_constant<int, 0>());
+  if (op == PC_OP_MAX) return f(std::integral_constant<int, 1>(), std::integral_constant<int, 1>());
+  return f(std::integral_constant<int, 1>(), std::integral_constant<int, 2>());
+}
+
+int grid_for(int warps, int nunits) {
+  int w = warps < nunits ? warps : nunits;
+  if (w < 1) w = 1;
+  return (w * 32 + kEngineBlock - 1) / kEngineBlock;
+}
+
+}  // namespace
+
+int launch_ring_engine(const RingArgs &a, int warps, cudaStream_t s) {
+  return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
+    ring_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  });
+}
+
+int launch_rd_engine(const RdArgs &a, int warps, cudaStream_t s) {
+  return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
+    rd_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  });
+}
+
+int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
+  p2p_engine<<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_wait_words(const uint32_t *words, int n, uint32_t target, const uint32_t *layout, int partitions,
+                      int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys) {
+  wait_words_kernel<<<1, 256, 0, s>>>(words, n, target, layout, partitions, err, timeout_ms, sys ? 1 : 0);
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s) {
+  set_word_kernel<<<1, 1, 0, s>>>(addr, value);
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s) {
+  const int n = hi - lo + 1;
+  int blocks = (n + 7) / 8;
+  if (blocks > 148) blocks = 148;
+  if (blocks < 1) blocks = 1;
+  pready_range_kernel<<<blocks, 256, 0, s>>>(q, lo, hi);
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int engine_occupancy_ctas_per_sm(int *ctas) {
+  int a = 0, b = 0;
+  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, ring_engine<1, 0>, kEngineBlock, 0));
+  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, rd_engine<1, 0>, kEngineBlock, 0));
+  *ctas = a < b ? a : b;
+  return 0;
+}
+
+}  // namespace pc

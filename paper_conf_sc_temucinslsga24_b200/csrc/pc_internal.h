@@ -1,0 +1,231 @@
+// Internal host-side structures of libpc (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <condition_variable>
+#include <cstdint>
+#include <map>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "pc.h"
+#include "pc_prequest.h"
+
+namespace pc {
+
+constexpr int kMaxRanks = 64;
+constexpr int kMaxRdSteps = 6;        // log2(kMaxRanks)
+constexpr int kEngineBlock = 256;     // threads per engine CTA (8 warps)
+
+// ------------------------------------------------------------------ errors
+int cuda_err(cudaError_t e, const char *what);
+#define PC_CUDA(call)                                     \
+  do {                                                    \
+    cudaError_t _e = (call);                              \
+    if (_e != cudaSuccess) return ::pc::cuda_err(_e, #call); \
+  } while (0)
+void logf(const char *fmt, ...);
+
+// ------------------------------------------------------------------ bootstrap records
+struct RankRec {
+  uint32_t magic;
+  int32_t rank, size, device, dry;
+  int32_t sms, engine_warps;  // this rank's engine capacity (already divided by ranks on its device)
+  int32_t pad;
+  int64_t pid;
+  uint64_t proc_token;
+  uint8_t uuid[16];
+};
+
+struct ShareRec {  // one exported allocation
+  cudaIpcMemHandle_t h;
+  uint64_t off;    // offset of the pointer inside its allocation
+  uint64_t raw;    // raw pointer (valid in the exporting process)
+  uint64_t bytes;  // bytes meaningful from the pointer
+};
+
+struct ReqRec {
+  int32_t kind, peer, tag, partitions;
+  int64_t count;
+  int32_t dtype, op, algo, seq;
+  int32_t owner;     // exporting rank
+  int32_t req_index; // index in the owner's request list
+  ShareRec buf;      // p2p: user buffer; allreduce: recvbuf
+  ShareRec ctrl;     // control block
+  ShareRec stage;    // allreduce staging
+};
+
+// ------------------------------------------------------------------ local group
+struct LocalGroup {
+  int size;
+  std::mutex mu;
+  std::condition_variable cv;
+  uint64_t generation = 0;
+  int arrived = 0;
+  int readers_left = 0;
+  std::vector<uint8_t> buf;
+  size_t nbytes = 0;
+  std::vector<std::pair<LocalGroup *, int>> ctxs;
+};
+
+// ------------------------------------------------------------------ control block layout
+// One device allocation per request.  Words are u32.  Offsets in words.
+struct CtrlLayout {
+  size_t epoch = 0;        // [1]
+  size_t rtr = 1;          // [kMaxRdSteps + 2] ready-to-receive words (per incoming producer slot)
+  size_t layout = 10;      // [1] g published by the sender (receive side)
+  size_t err = 12;         // [2] sticky device error (int32 code, partition)
+  size_t cnt = 16;         // [n1] aggregation counters
+  size_t ready = 0;        // [n1]
+  size_t sent = 0;         // [n1]
+  size_t donecnt = 0;      // [n1] engine slice-completion counters / allreduce done[u]
+  size_t flags = 0;        // [nflags] arrival flags
+  size_t words = 0;
+  void build(size_t n1, size_t nflags) {
+    ready = cnt + n1;
+    sent = ready + n1;
+    donecnt = sent + n1;
+    flags = donecnt + n1;
+    words = flags + nflags;
+    words = (words + 63) & ~size_t(63);
+  }
+};
+
+struct Comm;
+
+struct Request {
+  Comm *comm = nullptr;
+  int index = -1;  // position in comm->reqs
+  int kind = 0;    // PC_KIND_*
+  const void *sbuf = nullptr;
+  void *rbuf = nullptr;
+  int partitions = 0;
+  size_t count = 0;
+  int dtype = 0, op = 0, algo_req = 0, algo = 0;
+  int peer = -1, tag = 0, seq = 0;
+  size_t esize = 4;
+  uint64_t part_bytes = 0, total_bytes = 0;
+
+  // state
+  uint32_t epoch = 0;
+  bool active = false;
+  bool exchanged = false;
+  bool prepared_this_epoch = false;
+  bool engine_launched = false;
+  bool matched = false;
+  int match_peer_index = -1;
+
+  // device resources
+  uint32_t *ctrl = nullptr;  // device control block
+  CtrlLayout L;
+  uint8_t *staging = nullptr;
+  size_t staging_bytes = 0;
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_done = nullptr;
+  cudaStream_t user_stream = nullptr;
+
+  // peer addresses (after exchange)
+  uint8_t *peer_buf = nullptr;       // p2p send: receiver's recvbuf
+  uint32_t *peer_ctrl = nullptr;     // p2p: partner ctrl; allreduce ring: ctrl of O
+  uint8_t *peer_stage = nullptr;     // allreduce ring: staging of O
+  // allreduce RD: per step partner addresses; ring uses index 0 (= O)
+  uint8_t *nb_buf[kMaxRdSteps + 1] = {};
+  uint32_t *nb_ctrl[kMaxRdSteps + 1] = {};
+  uint8_t *nb_stage[kMaxRdSteps + 1] = {};
+  // consumers of this rank (they get an RTR write from us): ctrl + rtr slot
+  std::vector<std::pair<uint32_t *, int>> rtr_targets;
+
+  // prequest (p2p)
+  bool has_preq = false;
+  int agg = 1, ntransport = 0, copy = 0;
+  // engine slicing
+  int nsteps = 0;
+  int slices = 1;          // ns: slices per chunk (allreduce) or per transport partition (p2p ENGINE)
+  int64_t slice_elems = 0; // allreduce: elements per slice; p2p: bytes per slice
+  int64_t chunk_elems = 0; // allreduce ring: q
+  int engine_warps = 0;
+};
+
+struct Comm {
+  int rank = 0, size = 1, device = -1;
+  bool dry = false;
+  pc_allgather_fn ag = nullptr;
+  void *ag_ctx = nullptr;
+  std::vector<RankRec> ranks;
+  std::vector<bool> same_proc;
+  int engine_warps = 0;  // agreed (min over ranks)
+  int sms = 0;
+  std::vector<Request *> reqs;
+  std::map<std::tuple<int, int, int>, int> post_seq;  // (kind, peer, tag) -> next seq
+  int allreduce_seq = 0;
+  // IPC mappings opened by this comm: key = handle bytes
+  std::map<std::string, void *> ipc_open;
+  uint32_t timeout_ms = 10000;
+  bool memops = false;  // cuStreamWriteValue32 usable
+};
+
+// ------------------------------------------------------------------ helpers
+int allgather(Comm *c, const void *send, size_t nbytes, void *recv);
+int export_ptr(Comm *c, const void *p, uint64_t bytes, ShareRec *out);
+int import_ptr(Comm *c, int owner, const ShareRec &s, void **out);
+int stream_write_u32(Comm *c, cudaStream_t s, uint32_t *addr, uint32_t value);
+bool memops_available();
+
+// ------------------------------------------------------------------ kernel launchers (kernels.cu)
+struct RingArgs {
+  uint32_t e;
+  int P, r, Np, ns, nunits, op, dtype;
+  int64_t L, q, qs;
+  const uint8_t *sendbuf;
+  uint8_t *recvbuf;
+  const uint8_t *staging;
+  const uint32_t *flags, *ready, *rtr;
+  uint32_t *done;
+  uint8_t *o_staging, *o_recvbuf;
+  uint32_t *o_flags;
+  int32_t *err;
+  uint32_t timeout_ms;
+};
+struct RdArgs {
+  uint32_t e;
+  int P, r, Np, ns, nunits, op, dtype, nsteps;
+  int64_t L, qs;
+  const uint8_t *sendbuf;
+  uint8_t *recvbuf;
+  const uint8_t *staging;  // [nsteps][Np*L]
+  const uint32_t *flags, *ready, *rtr;
+  uint32_t *done;
+  uint8_t *p_staging[kMaxRdSteps];
+  uint32_t *p_flags[kMaxRdSteps];
+  int32_t *err;
+  uint32_t timeout_ms;
+};
+struct P2pEngineArgs {
+  uint32_t e;
+  int nt, agg, ns, nunits;
+  uint64_t part_bytes, slice_bytes;
+  int partitions;
+  const uint8_t *sbuf;
+  uint8_t *peer_rbuf;
+  uint32_t *peer_flags;
+  const uint32_t *ready, *rtr;
+  uint32_t *donecnt, *sent;
+  int32_t *err;
+  uint32_t timeout_ms;
+};
+
+int launch_ring_engine(const RingArgs &a, int warps, cudaStream_t s);
+int launch_rd_engine(const RdArgs &a, int warps, cudaStream_t s);
+int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s);
+// wait until words[i*stride] reached target (i < n); layout!=null: n derived
+// as ceil(partitions / *layout) (receiver side)
+int launch_wait_words(const uint32_t *words, int n, uint32_t target, const uint32_t *layout, int partitions,
+                      int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys);
+int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s);
+int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s);
+int engine_occupancy_ctas_per_sm(int *ctas);
+
+}  // namespace pc

@@ -1,0 +1,189 @@
+"""GPU parity: partitioned allreduce (ring = Alg 1, RD) through the C ABI vs
+the CPU oracle, with P virtual ranks on one B200 (tests/gpu_util.py).
+
+Bar: int32 bit-exact against the oracle's plain
+definition; fp32 bit-exact against the schedule-faithful oracle (O3 ring fold /
+O4 RD tree) AND |y - y64| <= 1e-5 * sum|x| against fp64 (reading R16).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_sc_temucinslsga24_b200 as pc
+import synth
+from paper_conf_sc_temucinslsga24_b200 import apps
+
+from gpu_util import comms, first_prepare, to_dev
+
+pytestmark = pytest.mark.gpu
+
+SEED = synth.BASE_SEED
+
+
+def run_allreduce(P, Np, L, xs_epochs, algo, op=pc.SUM, inplace=False, producer=None, gran=apps.GRAN_BLOCK):
+    """xs_epochs: list over epochs of (P, Np*L) host arrays.  Returns a list over
+    epochs of (P, Np*L) results (each rank's recvbuf after its wait)."""
+    dt = pc.INT32 if xs_epochs[0].dtype == np.int32 else pc.FLOAT32
+    n = Np * L
+    outs = []
+    with comms(P) as cs:
+        streams = [torch.cuda.Stream() for _ in range(P)]
+        nd = max(n, 4)
+        tdtype = torch.int32 if dt == pc.INT32 else torch.float32
+        send = [torch.zeros(nd, dtype=tdtype, device="cuda") for _ in range(P)]
+        recv = send if inplace else [torch.zeros(nd, dtype=tdtype, device="cuda") for _ in range(P)]
+        src = [torch.zeros(nd, dtype=tdtype, device="cuda") for _ in range(P)]
+        reqs = [pc.pallreduce_init(send[r], recv[r], Np, L, dt, op, algo, cs[r]) for r in range(P)]
+        preqs = None
+        for e, xs in enumerate(xs_epochs):
+            for r in range(P):
+                with torch.cuda.stream(streams[r]):
+                    if producer:
+                        src[r][:n].copy_(torch.from_numpy(xs[r]).to("cuda", non_blocking=False))
+                    else:
+                        send[r][:n].copy_(torch.from_numpy(xs[r]).to("cuda", non_blocking=False))
+            torch.cuda.synchronize()
+            for r in range(P):
+                reqs[r].start(streams[r])
+            if e == 0:
+                first_prepare([[reqs[r]] for r in range(P)], streams)
+                preqs = [reqs[r].prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_ENGINE) for r in range(P)]
+            else:
+                for r in range(P):
+                    reqs[r].pbuf_prepare(streams[r])
+            for r in range(P):
+                if producer:
+                    apps.produce(send[r], src[r], Np, L * 4, gran, preqs[r], order_stride=producer,
+                                 stream=streams[r])
+                else:
+                    reqs[r].pready_range(0, Np - 1, streams[r])
+            for r in range(P):
+                reqs[r].wait_on_stream(streams[r])
+            torch.cuda.synchronize()
+            for r in range(P):
+                code, part = reqs[r].error()
+                assert code == 0, f"rank {r} device error {code} at {part}"
+            outs.append(np.stack([recv[r][:n].cpu().numpy() for r in range(P)]))
+        for q in reqs:
+            q.free()
+    return outs
+
+
+def wrap_sum(x):
+    s = x.astype(np.int64).sum(axis=0)
+    return ((s + 2**31) % 2**32 - 2**31).astype(np.int32)
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 5, 8])
+@pytest.mark.parametrize("Np,L", [(1, 1), (3, 17), (7, 64), (8, 5), (2, 1000), (1, 4)])
+def test_ring_int32_sum(P, Np, L):
+    x = np.stack([synth.int32_full(SEED, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_RING)
+    ref = oracle.allreduce_def_i32(x)
+    for r in range(P):
+        np.testing.assert_array_equal(y[r], ref)
+
+
+@pytest.mark.parametrize("P", [1, 2, 4, 8])
+@pytest.mark.parametrize("Np,L", [(1, 1), (3, 17), (8, 5), (2, 1000)])
+def test_rd_int32_sum(P, Np, L):
+    x = np.stack([synth.int32_full(SEED + 1, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_RD)
+    ref = oracle.allreduce_def_i32(x)
+    for r in range(P):
+        np.testing.assert_array_equal(y[r], ref)
+
+
+@pytest.mark.parametrize("op", [pc.MAX, pc.MIN])
+@pytest.mark.parametrize("algo,P", [(pc.ALGO_RING, 3), (pc.ALGO_RING, 8), (pc.ALGO_RD, 4)])
+def test_int32_maxmin(op, algo, P):
+    Np, L = 4, 333
+    x = np.stack([synth.int32_full(SEED + 2, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], algo, op=op)
+    ref = oracle.allreduce_def_i32(x, op)
+    for r in range(P):
+        np.testing.assert_array_equal(y[r], ref)
+
+
+def check_fp32(x, y, algo, Np, L):
+    P = x.shape[0]
+    y64, sabs = oracle.allreduce_def_f64(x)
+    if algo == pc.ALGO_RING:
+        lit, _, _ = oracle.pallreduce(x, Np, oracle.RING) if x.size <= 4_000_000 else (None, 0, 0)
+        cf = oracle.ring_fold_f32(x, oracle.chunk_ids(L, P, Np))
+    else:
+        lit, _, _ = oracle.pallreduce(x, Np, oracle.RD) if x.size <= 4_000_000 else (None, 0, 0)
+        cf = oracle.rd_tree_f32(x)
+    for r in range(P):
+        np.testing.assert_array_equal(y[r].view(np.uint32), cf.view(np.uint32))
+        if lit is not None:
+            np.testing.assert_array_equal(y[r].view(np.uint32), lit[r].view(np.uint32))
+    assert (np.abs(y[0].astype(np.float64) - y64) <= 1e-5 * sabs).all()
+
+
+@pytest.mark.parametrize("P", [2, 3, 5, 8])
+@pytest.mark.parametrize("Np,L", [(1, 1), (3, 17), (7, 64), (2, 4099)])
+def test_ring_fp32_bitexact(P, Np, L):
+    x = np.stack([synth.normal_f32(SEED + 3, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_RING)
+    check_fp32(x, y, pc.ALGO_RING, Np, L)
+
+
+@pytest.mark.parametrize("P", [2, 4, 8])
+@pytest.mark.parametrize("Np,L", [(1, 1), (3, 17), (2, 4099)])
+def test_rd_fp32_bitexact(P, Np, L):
+    x = np.stack([synth.normal_f32(SEED + 4, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_RD)
+    check_fp32(x, y, pc.ALGO_RD, Np, L)
+
+
+@pytest.mark.parametrize("algo,P", [(pc.ALGO_RING, 4), (pc.ALGO_RING, 8), (pc.ALGO_RD, 8)])
+def test_multi_slice_ragged_epochs_inplace(algo, P):
+    """Sizes spanning many slices per chunk with a ragged tail (L % 4 != 0 so
+    partitions are not 16-B aligned), 3 epochs with epoch-tagged inputs,
+    in place (sendbuf == recvbuf, reading R22), device producer with a
+    permuted Pready order."""
+    Np, L = 3, 300_001
+    xs = [np.stack([synth.normal_f32(SEED + 5, r, e, Np * L) for r in range(P)]) for e in range(3)]
+    ys = run_allreduce(P, Np, L, xs, algo, inplace=True, producer=2)
+    for x, y in zip(xs, ys):
+        check_fp32(x, y, algo, Np, L)
+
+
+@pytest.mark.parametrize("gran", [apps.GRAN_THREAD, apps.GRAN_WARP, apps.GRAN_BLOCK])
+def test_device_producer_granularities(gran):
+    P, Np, L = 4, 16, 4096
+    x = np.stack([synth.int32_full(SEED + 6, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_RING, producer=5, gran=gran)
+    for r in range(P):
+        np.testing.assert_array_equal(y[r], wrap_sum(x))
+
+
+def test_many_epochs_int():
+    """50 back-to-back epochs with epoch-tagged inputs: no stale or early reads."""
+    P, Np, L = 4, 5, 777
+    xs = [np.stack([synth.int32_full(SEED + 7, r, e, Np * L) for r in range(P)]) for e in range(50)]
+    ys = run_allreduce(P, Np, L, xs, pc.ALGO_RING)
+    for x, y in zip(xs, ys):
+        for r in range(P):
+            np.testing.assert_array_equal(y[r], wrap_sum(x))
+
+
+def test_nan_propagates():
+    P, Np, L = 4, 2, 64
+    x = np.stack([synth.normal_f32(SEED + 8, r, 0, Np * L) for r in range(P)])
+    x[1, 7] = np.nan
+    for algo in (pc.ALGO_RING, pc.ALGO_RD):
+        (y,) = run_allreduce(P, Np, L, [x], algo)
+        assert np.isnan(y[:, 7]).all() and not np.isnan(np.delete(y, 7, axis=1)).any()
+
+
+def test_integer_valued_fp32_exact():
+    P, Np, L = 8, 4, 10_000
+    x = np.stack([synth.int_valued_f32(SEED + 9, r, 0, Np * L, (1 << 24) // P) for r in range(P)])
+    for algo in (pc.ALGO_RING, pc.ALGO_RD):
+        (y,) = run_allreduce(P, Np, L, [x], algo)
+        ref = x.astype(np.int64).sum(0).astype(np.float32)
+        for r in range(P):
+            np.testing.assert_array_equal(y[r], ref)

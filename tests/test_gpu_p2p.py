@@ -1,0 +1,232 @@
+"""GPU parity: partitioned send/recv (Pready at thread / warp / block
+granularity, aggregation, INLINE "Kernel Copy" and ENGINE copy) through the C
+ABI vs the CPU oracle O1 (byte-exact), with 2 virtual ranks on one B200."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_sc_temucinslsga24_b200 as pc
+import synth
+from paper_conf_sc_temucinslsga24_b200 import apps
+
+from gpu_util import comms, first_prepare
+
+pytestmark = pytest.mark.gpu
+SEED = synth.BASE_SEED
+
+GRAN_ELEMS = {apps.GRAN_THREAD: 2, apps.GRAN_WARP: 64, apps.GRAN_BLOCK: 2048}  # 8 B / 256 B / 8 KiB
+
+
+def run_vecadd(n, gran, agg, copy, epochs=3, check_in_kernel=True):
+    """C1/C2 shape: sender computes C = A + B and Preadies from the kernel."""
+    count = GRAN_ELEMS[gran]
+    partitions = n // count
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        A = torch.empty(n, device="cuda")
+        B = torch.empty(n, device="cuda")
+        Cb = torch.empty(n, device="cuda")
+        R = torch.full((n,), -1.0, device="cuda")
+        out = torch.zeros(n, device="cuda")
+        status = torch.zeros(1, dtype=torch.int32, device="cuda")
+        snd = pc.psend_init(Cb, partitions, count, pc.FLOAT32, 1, 7, cs[0])
+        rcv = pc.precv_init(R, partitions, count, pc.FLOAT32, 0, 7, cs[1])
+        sent_all, got_all, got_kernel = [], [], []
+        for e in range(epochs):
+            a = synth.uniform_f32(SEED, 0, 2 * e, n)
+            b = synth.uniform_f32(SEED, 0, 2 * e + 1, n)
+            A.copy_(torch.from_numpy(a))
+            B.copy_(torch.from_numpy(b))
+            torch.cuda.synchronize()
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                sq = snd.prequest_create(gran, agg, copy)
+                rq = rcv.prequest_create(gran, 1, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            if check_in_kernel:
+                apps.check_recv(rq, R, out, partitions, count * 4, status, blocks=64, stream=s1)
+            apps.vecadd(A, B, Cb, n, gran, sq, s0)
+            snd.wait_on_stream(s0)
+            rcv.wait_on_stream(s1)
+            torch.cuda.synchronize()
+            assert snd.error()[0] == 0 and rcv.error()[0] == 0
+            sent_all.append((a + b).astype(np.float32))
+            got_all.append(R.cpu().numpy().copy())
+            got_kernel.append(out.cpu().numpy().copy())
+        assert int(status.item()) == 0
+        snd.free()
+        rcv.free()
+    send = np.stack(sent_all).view(np.uint8).reshape(epochs, -1)
+    orders = np.stack([synth.permutation(SEED, 0, e, partitions) for e in range(epochs)])
+    consumed, arrivals = oracle.p2p(send, partitions, agg, orders)
+    assert (arrivals == 1).all()
+    got = np.stack(got_all).view(np.uint8).reshape(epochs, -1)
+    np.testing.assert_array_equal(got, consumed)
+    if check_in_kernel:
+        np.testing.assert_array_equal(np.stack(got_kernel).view(np.uint8).reshape(epochs, -1), consumed)
+
+
+def test_c1_block_agg16_inline():
+    """C1: 1 MiB fp32, block Pready (128 x 8 KiB user partitions) aggregated
+    16 per transport partition -> 8 transport partitions (reading R24)."""
+    run_vecadd(1 << 18, apps.GRAN_BLOCK, 16, pc.COPY_INLINE, epochs=5)
+
+
+@pytest.mark.parametrize("gran", [apps.GRAN_THREAD, apps.GRAN_WARP, apps.GRAN_BLOCK])
+@pytest.mark.parametrize("agg_kind", ["none", "odd", "all"])
+@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE])
+def test_granularity_aggregation_copy(gran, agg_kind, copy):
+    n = 3 * 2048 * 5 + 0  # 15 blocks of 1024 threads
+    partitions = n // GRAN_ELEMS[gran]
+    agg = {"none": 1, "odd": max(1, partitions // 3 - 1), "all": partitions}[agg_kind]
+    run_vecadd(n, gran, agg, copy, epochs=2)
+
+
+def test_thread_granularity_warp_aggregation_large():
+    """Thread granularity with g = 1024 (one transport partition per block):
+    the library's warp aggregation of thread Preadies."""
+    run_vecadd(1 << 20, apps.GRAN_THREAD, 1024, pc.COPY_INLINE, epochs=2)
+
+
+def test_many_epochs_tagged_bytes():
+    """>= 200 back-to-back epochs of epoch-tagged bytes with a permuted Pready
+    order: every epoch's bytes arrive intact and exactly once."""
+    partitions, pbytes, E = 16, 4096, 200
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        src = torch.empty(partitions * pbytes, dtype=torch.uint8, device="cuda")
+        sbuf = torch.empty_like(src)
+        rbuf = torch.empty_like(src)
+        snd = pc.psend_init(sbuf, partitions, pbytes, pc.BYTE, 1, 1, cs[0])
+        rcv = pc.precv_init(rbuf, partitions, pbytes, pc.BYTE, 0, 1, cs[1])
+        for e in range(E):
+            payload = synth.bytes_tagged(SEED, 0, e, partitions * pbytes)
+            src.copy_(torch.from_numpy(payload))
+            torch.cuda.synchronize()
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                sq = snd.prequest_create(pc.GRAN_BLOCK, 4, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            apps.produce(sbuf, src, partitions, pbytes, apps.GRAN_BLOCK, sq, order_stride=5, stream=s0)
+            snd.wait_on_stream(s0)
+            rcv.wait_on_stream(s1)
+            s1.synchronize()
+            np.testing.assert_array_equal(rbuf.cpu().numpy(), payload)
+        snd.wait()
+        assert snd.error()[0] == 0 and rcv.error()[0] == 0
+        snd.free()
+        rcv.free()
+
+
+def test_host_wait_and_test():
+    n = 2048 * 4
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        A = torch.ones(n, device="cuda")
+        Cb = torch.empty(n, device="cuda")
+        R = torch.zeros(n, device="cuda")
+        snd = pc.psend_init(Cb, 4, 2048, pc.FLOAT32, 1, 0, cs[0])
+        rcv = pc.precv_init(R, 4, 2048, pc.FLOAT32, 0, 0, cs[1])
+        snd.start(s0)
+        rcv.start(s1)
+        first_prepare([[snd], [rcv]], [s0, s1])
+        sq = snd.prequest_create(pc.GRAN_BLOCK, 2, pc.COPY_ENGINE)
+        assert not rcv.parrived(0)
+        apps.vecadd(A, A, Cb, n, apps.GRAN_BLOCK, sq, s0)
+        snd.wait()
+        rcv.wait()
+        assert rcv.parrived(3)
+        assert (R.cpu().numpy() == 2.0).all()
+        assert rcv.test()  # inactive request: complete
+        snd.free()
+        rcv.free()
+
+
+def test_duplicate_pready_is_reported():
+    n = 2048 * 2
+    with comms(2, timeout_ms=2000) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        Cb = torch.zeros(n, device="cuda")
+        R = torch.zeros(n, device="cuda")
+        snd = pc.psend_init(Cb, 2, 2048, pc.FLOAT32, 1, 0, cs[0])
+        rcv = pc.precv_init(R, 2, 2048, pc.FLOAT32, 0, 0, cs[1])
+        snd.start(s0)
+        rcv.start(s1)
+        first_prepare([[snd], [rcv]], [s0, s1])
+        snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+        snd.pready(0, s0)
+        snd.pready(0, s0)  # duplicate in the same epoch
+        snd.pready(1, s0)
+        rcv.wait()
+        with pytest.raises(pc.PcError) as ei:
+            snd.wait()
+        assert ei.value.code == pc.ERR_DEVICE
+        snd.free()
+        rcv.free()
+
+
+def test_missing_pready_times_out():
+    n = 2048 * 2
+    with comms(2, timeout_ms=300) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        Cb = torch.zeros(n, device="cuda")
+        R = torch.zeros(n, device="cuda")
+        snd = pc.psend_init(Cb, 2, 2048, pc.FLOAT32, 1, 0, cs[0])
+        rcv = pc.precv_init(R, 2, 2048, pc.FLOAT32, 0, 0, cs[1])
+        snd.start(s0)
+        rcv.start(s1)
+        first_prepare([[snd], [rcv]], [s0, s1])
+        snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+        snd.pready(0, s0)  # partition 1 never readied
+        with pytest.raises(pc.PcError) as ei:
+            rcv.wait()
+        assert ei.value.code == pc.ERR_TIMEOUT
+        with pytest.raises(pc.PcError):
+            snd.wait()
+        snd.free()
+        rcv.free()
+
+
+@pytest.mark.parametrize("payload", [0, 8, 256, 8192])
+def test_pingpong_latency_roundtrip(payload):
+    """Pready->Parrived ping-pong inside persistent kernels (one per side)."""
+    iters = 2000
+    cnt = payload // 4
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        bufs = [torch.zeros(max(iters * cnt, 4), device="cuda") for _ in range(4)]
+        a2b = pc.psend_init(bufs[0], iters, cnt, pc.FLOAT32, 1, 1, cs[0])
+        b_in = pc.precv_init(bufs[1], iters, cnt, pc.FLOAT32, 0, 1, cs[1])
+        b2a = pc.psend_init(bufs[2], iters, cnt, pc.FLOAT32, 0, 2, cs[1])
+        a_in = pc.precv_init(bufs[3], iters, cnt, pc.FLOAT32, 1, 2, cs[0])
+        bufs[0].copy_(torch.arange(bufs[0].numel(), dtype=torch.float32))
+        for q, s in ((a2b, s0), (a_in, s0), (b_in, s1), (b2a, s1)):
+            q.start(s)
+        first_prepare([[a2b, a_in], [b_in, b2a]], [s0, s1])
+        pa = a2b.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
+        pai = a_in.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
+        pb = b2a.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
+        pbi = b_in.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
+        t = torch.zeros(2, dtype=torch.int64, device="cuda")
+        apps.pingpong(pb, pbi, 1, iters, apps.GRAN_WARP, t[1:], s1)
+        apps.pingpong(pa, pai, 0, iters, apps.GRAN_WARP, t[:1], s0)
+        for q, s in ((a2b, s0), (a_in, s0), (b_in, s1), (b2a, s1)):
+            q.wait_on_stream(s)
+        torch.cuda.synchronize()
+        ns = int(t[0].item()) / iters / 2
+        print(f"payload {payload} B: one-way {ns:.0f} ns (same-GPU virtual ranks)")
+        assert ns > 0
+        if cnt:
+            np.testing.assert_array_equal(bufs[1].cpu().numpy(), bufs[0].cpu().numpy())
+        for q in (a2b, a_in, b_in, b2a):
+            assert q.error()[0] == 0
+            q.free()
