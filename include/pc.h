@@ -165,6 +165,10 @@ int pc_chunk_bounds(int64_t L, int P, int64_t *out);
 int pc_request_info(pc_request_t req, int *algo, int *slices, int64_t *slice_elems, int *engine_warps);
 /* Matched peer request id (debug; p2p) after the first pbuf_prepare. */
 int pc_request_match(pc_request_t req, int *peer, int *peer_request_index);
+/* Read n control words of a request (which: 0 arrival flags, 1 sent, 2
+ * aggregation counters, 3 ready, 4 done/slice counters, 5 RTR words, 6 epoch)
+ * starting at `offset` into host memory `out` (debug / tests; blocking). */
+int pc_request_words(pc_request_t req, int which, int offset, int n, uint32_t *out);
 /* Device error word of a request: code and partition (0,0 if none). */
 int pc_request_error(pc_request_t req, int *code, int *partition);
 const char *pc_strerror(int err);

@@ -267,34 +267,37 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
   return 0;
 }
 
-/* Warp granularity: all active lanes of the warp call it with the same
- * partition; one notification per warp (reading R11). */
+/* Warp granularity: warp-collective — ALL 32 lanes of the warp call it with
+ * the same partition (like __syncwarp()); one notification per warp (P:L137,
+ * reading R11).  (__activemask() cannot be used to find the participants: with
+ * independent thread scheduling a converged-looking warp may run this code as
+ * several subsets, which would count the warp more than once.) */
 PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   using namespace pc_detail;
-  const unsigned mask = __activemask();
+  const unsigned full = 0xffffffffu;
   const uint32_t lane = lane_id();
-  const uint32_t first = __ffs(mask) - 1;
+  __syncwarp(full);  // every lane's data writes are ordered before lane 0's release
   if (partition < 0 || partition >= preq.partitions) {
-    if (lane == first) set_error(preq.err, PC_DEV_ERR_ARG, partition);
+    if (lane == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);
     return PC_DEV_ERR_ARG;
   }
   const uint32_t e = epoch_of(preq);
-  __syncwarp(mask);
   if (preq.kind == PC_KIND_PALLREDUCE) {
-    if (lane == first) st_release_gpu(preq.ready + partition, e);
+    if (lane == 0) st_release_gpu(preq.ready + partition, e);
+    __syncwarp(full);
     return 0;
   }
   const int t = partition / preq.agg;
   bool completes = false;
-  if (lane == first) completes = contribute(preq, t, 1, e, partition);
-  completes = __shfl_sync(mask, completes, first);
+  if (lane == 0) completes = contribute(preq, t, 1, e, partition);
+  completes = __shfl_sync(full, completes, 0);
   if (!completes) return 0;
   if (preq.copy == 1) {
-    if (lane == first) st_release_gpu(preq.ready + t, e);
+    if (lane == 0) st_release_gpu(preq.ready + t, e);
+    __syncwarp(full);
     return 0;
   }
-  __syncwarp(mask);
-  push_warp(preq, t, e, mask);
+  push_warp(preq, t, e, full);
   return 0;
 }
 

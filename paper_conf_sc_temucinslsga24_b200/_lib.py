@@ -60,6 +60,7 @@ _PC_PROTOS = {
     "pc_request_info": (I32, [P, PI32, PI32, PI64, PI32]),
     "pc_request_match": (I32, [P, PI32, PI32]),
     "pc_request_error": (I32, [P, PI32, PI32]),
+    "pc_request_words": (I32, [P, I32, I32, I32, P]),
     "pc_strerror": (C.c_char_p, [I32]),
     "pc_version": (C.c_char_p, []),
 }
@@ -70,6 +71,8 @@ _APP_PROTOS = {
     "pcapp_check_recv": (I32, [P, P, P, I32, I64, I32, P, P]),
     "pcapp_pingpong": (I32, [P, P, I32, I32, I32, P, P]),
     "pcapp_bare_pingpong": (I32, [P, P, I32, I32, C.c_uint32, P, P]),
+    "pcapp_pingpong_pair": (I32, [P, P, P, P, I32, I32, P, P]),
+    "pcapp_bare_pingpong_pair": (I32, [P, P, I32, C.c_uint32, P, P]),
     "pcapp_prequest_size": (SZ, []),
 }
 

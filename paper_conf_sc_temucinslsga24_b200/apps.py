@@ -43,3 +43,15 @@ def pingpong(sendq: Prequest, recvq: Prequest, side: int, iters: int, gran: int,
 def bare_pingpong(my_flag, peer_flag, side: int, iters: int, base: int, out_ns, stream=None):
     _ok(_lib.apps().pcapp_bare_pingpong(_ptr(my_flag), _ptr(peer_flag), side, iters, base, _ptr(out_ns),
                                         _stream(stream)), "bare_pingpong")
+
+
+def pingpong_pair(sendA: Prequest, recvA: Prequest, sendB: Prequest, recvB: Prequest, iters: int, gran: int,
+                  out_ns, stream=None):
+    """Both sides in one launch (virtual ranks on one GPU)."""
+    _ok(_lib.apps().pcapp_pingpong_pair(sendA.ptr, recvA.ptr, sendB.ptr, recvB.ptr, iters, gran, _ptr(out_ns),
+                                        _stream(stream)), "pingpong_pair")
+
+
+def bare_pingpong_pair(flagA, flagB, iters: int, base: int, out_ns, stream=None):
+    _ok(_lib.apps().pcapp_bare_pingpong_pair(_ptr(flagA), _ptr(flagB), iters, base, _ptr(out_ns),
+                                             _stream(stream)), "bare_pingpong_pair")

@@ -109,6 +109,53 @@ __global__ void pingpong_kernel(pc_prequest_t sendq, pc_prequest_t recvq, int si
   if (threadIdx.x == 0) out_ns[0] = pc_detail::globaltimer() - t0;
 }
 
+// Both sides in ONE launch (block 0 = side 0, block 1 = side 1): for virtual
+// ranks sharing a GPU, so the two spinning sides are co-resident by
+// construction.
+__global__ void pingpong_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, pc_prequest_t sendB,
+                                     pc_prequest_t recvB, int iters, int gran, unsigned long long *out_ns) {
+  const int side = blockIdx.x;
+  const pc_prequest_t &sq = side ? sendB : sendA;
+  const pc_prequest_t &rq = side ? recvB : recvA;
+  const uint64_t t0 = pc_detail::globaltimer();
+  for (int k = 0; k < iters; ++k) {
+    if (side == 1) {
+      if (threadIdx.x == 0) pc_wait_arrived(rq, k);
+      __syncwarp();
+    }
+    if (gran == PCAPP_GRAN_THREAD) {
+      if (threadIdx.x == 0) pc_pready(k, sq);
+    } else {
+      pc_pready_warp(k, sq);
+    }
+    if (side == 0) {
+      if (threadIdx.x == 0) pc_wait_arrived(rq, k);
+      __syncwarp();
+    }
+  }
+  if (threadIdx.x == 0) out_ns[side] = pc_detail::globaltimer() - t0;
+}
+
+__global__ void bare_pingpong_pair_kernel(uint32_t *flagA, uint32_t *flagB, int iters, uint32_t base,
+                                          unsigned long long *out_ns) {
+  if (threadIdx.x != 0) return;
+  const int side = blockIdx.x;
+  uint32_t *mine = side ? flagB : flagA;
+  uint32_t *peer = side ? flagA : flagB;
+  const uint64_t t0 = pc_detail::globaltimer();
+  for (int k = 1; k <= iters; ++k) {
+    const uint32_t v = base + (uint32_t)k;
+    if (side == 1)
+      while (!pc_detail::reached(pc_detail::ld_acquire_sys(mine), v)) {
+      }
+    pc_detail::st_release_sys(peer, v);
+    if (side == 0)
+      while (!pc_detail::reached(pc_detail::ld_acquire_sys(mine), v)) {
+      }
+  }
+  out_ns[side] = pc_detail::globaltimer() - t0;
+}
+
 // Latency floor: the same ping-pong with a bare flag and no library.
 __global__ void bare_pingpong_kernel(uint32_t *my_flag, uint32_t *peer_flag, int side, int iters, uint32_t base,
                                      unsigned long long *out_ns) {
@@ -170,6 +217,19 @@ int pcapp_pingpong(const pc_prequest_t *sendq, const pc_prequest_t *recvq, int s
 int pcapp_bare_pingpong(uint32_t *my_flag, uint32_t *peer_flag, int side, int iters, uint32_t base,
                         unsigned long long *out_ns, cudaStream_t s) {
   bare_pingpong_kernel<<<1, 32, 0, s>>>(my_flag, peer_flag, side, iters, base, out_ns);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_pingpong_pair(const pc_prequest_t *sendA, const pc_prequest_t *recvA, const pc_prequest_t *sendB,
+                        const pc_prequest_t *recvB, int iters, int gran, unsigned long long *out_ns, cudaStream_t s) {
+  if (!sendA || !recvA || !sendB || !recvB) return -1;
+  pingpong_pair_kernel<<<2, 32, 0, s>>>(*sendA, *recvA, *sendB, *recvB, iters, gran, out_ns);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_bare_pingpong_pair(uint32_t *flagA, uint32_t *flagB, int iters, uint32_t base, unsigned long long *out_ns,
+                             cudaStream_t s) {
+  bare_pingpong_pair_kernel<<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

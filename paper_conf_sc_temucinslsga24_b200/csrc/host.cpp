@@ -266,6 +266,7 @@ static int alloc_ctrl(Request *q) {
   PC_CUDA(cudaStreamCreateWithPriority(&q->side, cudaStreamNonBlocking, hi));
   PC_CUDA(cudaEventCreateWithFlags(&q->ev_fork, cudaEventDisableTiming));
   PC_CUDA(cudaEventCreateWithFlags(&q->ev_done, cudaEventDisableTiming));
+  PC_CUDA(cudaEventCreateWithFlags(&q->gs.ev, cudaEventDisableTiming));
   PC_CUDA(cudaMalloc((void **)&q->ctrl, q->L.words * 4));
   PC_CUDA(cudaMemsetAsync(q->ctrl, 0, q->L.words * 4, q->side));
   if (q->staging_bytes) {
@@ -363,6 +364,7 @@ static int make_rec(Request *q, ReqRec *r) {
   r->seq = q->seq;
   r->owner = c->rank;
   r->req_index = q->index;
+  r->host_req = (uint64_t)(uintptr_t)q;
   int rc = 0;
   if (q->kind == PC_KIND_PRECV || q->kind == PC_KIND_PALLREDUCE)
     if ((rc = export_ptr(c, q->rbuf, q->total_bytes, &r->buf))) return rc;
@@ -474,6 +476,25 @@ static int exchange_round(Comm *c, Request *target) {
         if (!qrc) {
           q->exchanged = true;
           q->matched = true;
+          // ranks of this comm sharing this GPU inside this process run their
+          // engines as one grouped launch
+          std::vector<int> loc;
+          for (int k = 0; k < P; ++k)
+            if (c->same_proc[k] && c->ranks[k].device == c->device &&
+                memcmp(c->ranks[k].uuid, c->ranks[c->rank].uuid, 16) == 0)
+              loc.push_back(k);
+          if (loc.size() > 1) {
+            if ((int)loc.size() > kMaxLocal) {
+              qrc = PC_ERR_UNSUPPORTED;
+            } else {
+              Request *ld = (Request *)(uintptr_t)peers[loc[0]]->host_req;
+              q->leader = ld;
+              std::lock_guard<std::mutex> lk(ld->gs.mu);
+              ld->gs.members.push_back(q);
+              std::sort(ld->gs.members.begin(), ld->gs.members.end(),
+                        [](Request *a, Request *b) { return a->comm->rank < b->comm->rank; });
+            }
+          }
         }
       } else {
         q->exchanged = true;
@@ -490,73 +511,83 @@ static int exchange_round(Comm *c, Request *target) {
 }
 
 // ------------------------------------------------------------------ engine launch
-static int maybe_launch_engine(Request *q) {
+// The engine is launched lazily, from pc_wait / pc_wait_on_stream / pc_test,
+// i.e. AFTER the user enqueued the producer kernel of the epoch (Listing 2
+// order: Start, Pbuf_prepare, kernel, Wait).  A spinning engine can therefore
+// never sit in front of the producer it waits for in a shared hardware queue
+// (streams beyond CUDA_DEVICE_MAX_CONNECTIONS share queues).
+static RingArgs make_ring_args(Request *q) {
   Comm *c = q->comm;
-  if (c->dry || !q->active || !q->exchanged || !q->matched || q->engine_launched) return 0;
-  const bool needs = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
-  if (!needs) return 0;
-  PC_CUDA(cudaSetDevice(c->device));
+  RingArgs a{};
+  a.e = q->epoch;
+  a.P = c->size;
+  a.r = c->rank;
+  a.Np = q->partitions;
+  a.ns = q->slices;
+  a.nunits = q->partitions * q->slices;
+  a.op = q->op;
+  a.dtype = q->dtype;
+  a.L = (int64_t)q->count;
+  a.q = q->chunk_elems;
+  a.qs = q->slice_elems;
+  a.sendbuf = (const uint8_t *)q->sbuf;
+  a.recvbuf = (uint8_t *)q->rbuf;
+  a.staging = q->staging;
+  a.flags = q->ctrl + q->L.flags;
+  a.ready = q->ctrl + q->L.ready;
+  a.rtr = q->ctrl + q->L.rtr;
+  a.done = q->ctrl + q->L.donecnt;
+  a.o_staging = q->nb_stage[0];
+  a.o_recvbuf = q->nb_buf[0];
+  a.o_flags = q->nb_ctrl[0] ? q->nb_ctrl[0] + q->L.flags : nullptr;
+  a.err = (int32_t *)(q->ctrl + q->L.err);
+  a.timeout_ms = c->timeout_ms;
+  return a;
+}
+
+static RdArgs make_rd_args(Request *q) {
+  Comm *c = q->comm;
+  RdArgs a{};
+  a.e = q->epoch;
+  a.P = c->size;
+  a.r = c->rank;
+  a.Np = q->partitions;
+  a.ns = q->slices;
+  a.nunits = q->partitions * q->slices;
+  a.op = q->op;
+  a.dtype = q->dtype;
+  a.nsteps = q->nsteps;
+  a.L = (int64_t)q->count;
+  a.qs = q->slice_elems;
+  a.sendbuf = (const uint8_t *)q->sbuf;
+  a.recvbuf = (uint8_t *)q->rbuf;
+  a.staging = q->staging;
+  a.flags = q->ctrl + q->L.flags;
+  a.ready = q->ctrl + q->L.ready;
+  a.rtr = q->ctrl + q->L.rtr;
+  a.done = q->ctrl + q->L.donecnt;
+  const int64_t slot_bytes = (int64_t)q->partitions * (int64_t)q->count * 4;
+  for (int k = 0; k < q->nsteps; ++k) {
+    a.p_staging[k] = q->nb_stage[k] + (int64_t)k * slot_bytes;
+    a.p_flags[k] = q->nb_ctrl[k] + q->L.flags;
+  }
+  a.err = (int32_t *)(q->ctrl + q->L.err);
+  a.timeout_ms = c->timeout_ms;
+  return a;
+}
+
+static bool needs_engine(Request *q) {
+  return q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
+}
+
+// Single-rank launch on the request's side stream, forked from its user stream.
+static int launch_single(Request *q) {
   PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
   PC_CUDA(cudaStreamWaitEvent(q->side, q->ev_fork, 0));
-  int rc = 0;
-  int32_t *err = (int32_t *)(q->ctrl + q->L.err);
+  int rc;
   if (q->kind == PC_KIND_PALLREDUCE) {
-    const int P = c->size;
-    if (q->algo == PC_ALGO_RING) {
-      RingArgs a{};
-      a.e = q->epoch;
-      a.P = P;
-      a.r = c->rank;
-      a.Np = q->partitions;
-      a.ns = q->slices;
-      a.nunits = q->partitions * q->slices;
-      a.op = q->op;
-      a.dtype = q->dtype;
-      a.L = (int64_t)q->count;
-      a.q = q->chunk_elems;
-      a.qs = q->slice_elems;
-      a.sendbuf = (const uint8_t *)q->sbuf;
-      a.recvbuf = (uint8_t *)q->rbuf;
-      a.staging = q->staging;
-      a.flags = q->ctrl + q->L.flags;
-      a.ready = q->ctrl + q->L.ready;
-      a.rtr = q->ctrl + q->L.rtr;
-      a.done = q->ctrl + q->L.donecnt;
-      a.o_staging = q->nb_stage[0];
-      a.o_recvbuf = q->nb_buf[0];
-      a.o_flags = q->nb_ctrl[0] ? q->nb_ctrl[0] + q->L.flags : nullptr;
-      a.err = err;
-      a.timeout_ms = c->timeout_ms;
-      rc = launch_ring_engine(a, q->engine_warps, q->side);
-    } else {
-      RdArgs a{};
-      a.e = q->epoch;
-      a.P = P;
-      a.r = c->rank;
-      a.Np = q->partitions;
-      a.ns = q->slices;
-      a.nunits = q->partitions * q->slices;
-      a.op = q->op;
-      a.dtype = q->dtype;
-      a.nsteps = q->nsteps;
-      a.L = (int64_t)q->count;
-      a.qs = q->slice_elems;
-      a.sendbuf = (const uint8_t *)q->sbuf;
-      a.recvbuf = (uint8_t *)q->rbuf;
-      a.staging = q->staging;
-      a.flags = q->ctrl + q->L.flags;
-      a.ready = q->ctrl + q->L.ready;
-      a.rtr = q->ctrl + q->L.rtr;
-      a.done = q->ctrl + q->L.donecnt;
-      const int64_t slot_bytes = (int64_t)q->partitions * (int64_t)q->count * 4;
-      for (int k = 0; k < q->nsteps; ++k) {
-        a.p_staging[k] = q->nb_stage[k] + (int64_t)k * slot_bytes;
-        a.p_flags[k] = q->nb_ctrl[k] + q->L.flags;
-      }
-      a.err = err;
-      a.timeout_ms = c->timeout_ms;
-      rc = launch_rd_engine(a, q->engine_warps, q->side);
-    }
+    rc = q->algo == PC_ALGO_RING ? launch_ring_engine(make_ring_args(q), q->engine_warps, q->side)
+                                 : launch_rd_engine(make_rd_args(q), q->engine_warps, q->side);
   } else {
     P2pEngineArgs a{};
     a.e = q->epoch;
@@ -574,13 +605,58 @@ static int maybe_launch_engine(Request *q) {
     a.rtr = q->ctrl + q->L.rtr;
     a.donecnt = q->ctrl + q->L.donecnt;
     a.sent = q->ctrl + q->L.sent;
-    a.err = err;
-    a.timeout_ms = c->timeout_ms;
+    a.err = (int32_t *)(q->ctrl + q->L.err);
+    a.timeout_ms = q->comm->timeout_ms;
     rc = launch_p2p_engine(a, q->engine_warps, q->side);
   }
   if (rc) return rc;
   PC_CUDA(cudaEventRecord(q->ev_done, q->side));
   q->engine_launched = true;
+  return 0;
+}
+
+// Co-located ranks (same process, same GPU): register this rank's epoch; the
+// last rank to register launches ONE kernel running every member's engine,
+// ordered after every member's producer work (their ev_fork events).
+// *launched tells whether that launch has happened (then q->ev_done of the
+// group leader marks completion).  block: wait (host) until it has.
+static int group_register(Request *q, bool block, bool *launched) {
+  Request *ld = q->leader;
+  GroupState &g = ld->gs;
+  std::unique_lock<std::mutex> lk(g.mu);
+  if (g.epoch != q->epoch) {
+    if (g.pending > 0 && !g.launched) return PC_ERR_STATE;  // a member is still in the previous epoch
+    g.epoch = q->epoch;
+    g.pending = 0;
+    g.launched = false;
+  }
+  if (!q->engine_registered) {
+    PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+    q->engine_registered = true;
+    g.pending++;
+  }
+  if (!g.launched && g.pending == (int)g.members.size()) {
+    for (Request *m : g.members) PC_CUDA(cudaStreamWaitEvent(q->side, m->ev_fork, 0));
+    int rc;
+    if (q->algo == PC_ALGO_RING) {
+      RingGroupArgs ga{};
+      ga.n = (int)g.members.size();
+      for (int k = 0; k < ga.n; ++k) ga.a[k] = make_ring_args(g.members[k]);
+      rc = launch_ring_engine_group(ga, q->engine_warps, q->side);
+    } else {
+      RdGroupArgs ga{};
+      ga.n = (int)g.members.size();
+      for (int k = 0; k < ga.n; ++k) ga.a[k] = make_rd_args(g.members[k]);
+      rc = launch_rd_engine_group(ga, q->engine_warps, q->side);
+    }
+    if (rc) return rc;
+    PC_CUDA(cudaEventRecord(g.ev, q->side));
+    g.launched = true;
+    g.cv.notify_all();
+  }
+  if (block) g.cv.wait(lk, [&] { return g.launched || g.epoch != q->epoch; });
+  *launched = g.launched && g.epoch == q->epoch;
+  if (*launched) q->engine_launched = true;
   return 0;
 }
 
@@ -848,6 +924,7 @@ int pc_start(pc_request_t req, pc_stream_t stream) {
   q->epoch++;
   q->active = true;
   q->engine_launched = false;
+  q->engine_registered = false;
   q->prepared_this_epoch = false;
   q->user_stream = (cudaStream_t)stream;
   if (c->dry) return 0;
@@ -875,7 +952,7 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
     }
     q->prepared_this_epoch = true;
   }
-  return maybe_launch_engine(q);
+  return 0;
 }
 
 int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_copy_t copy, pc_prequest_t *out) {
@@ -912,13 +989,31 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
   }
   q->has_preq = true;
   fill_prequest(q, out);
-  if (q->kind == PC_KIND_PSEND) return maybe_launch_engine(q);
   return 0;
 }
 
 int pc_prequest_free(pc_prequest_t *preq) {
   if (!preq) return PC_ERR_ARG;
   memset(preq, 0, sizeof(*preq));
+  return 0;
+}
+
+// Make sure this epoch's engine is (or will be) launched; *ev = the event that
+// completes with it, or null when a co-located group is still incomplete.
+static int ensure_engine(Request *q, bool block, cudaEvent_t *ev) {
+  *ev = nullptr;
+  if (!needs_engine(q)) return 0;
+  if (q->leader) {
+    bool launched = false;
+    int rc = group_register(q, block, &launched);
+    if (launched) *ev = q->leader->gs.ev;
+    return rc;
+  }
+  if (!q->engine_launched) {
+    int rc = launch_single(q);
+    if (rc) return rc;
+  }
+  *ev = q->ev_done;
   return 0;
 }
 
@@ -931,17 +1026,21 @@ static int wait_common(Request *q, cudaStream_t s, bool host) {
   }
   PC_CUDA(cudaSetDevice(c->device));
   if (!q->exchanged || !q->matched) return PC_ERR_STATE;
-  int rc = maybe_launch_engine(q);
-  if (rc) return rc;
   int32_t *err = (int32_t *)(q->ctrl + q->L.err);
   const bool engine = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->copy == 1);
+  int rc;
   if (engine) {
-    if (!q->engine_launched) return PC_ERR_STATE;
+    if (q->kind == PC_KIND_PSEND && !q->has_preq) return PC_ERR_STATE;
+    cudaEvent_t ev = nullptr;
+    if ((rc = ensure_engine(q, host, &ev))) return rc;
     if (host) {
-      PC_CUDA(cudaEventSynchronize(q->ev_done));
-    } else {
-      PC_CUDA(cudaStreamWaitEvent(s, q->ev_done, 0));
+      if (!ev) return PC_ERR_STATE;
+      PC_CUDA(cudaEventSynchronize(ev));
+    } else if (ev) {
+      PC_CUDA(cudaStreamWaitEvent(s, ev, 0));
     }
+    // (co-located group not complete yet: the last local rank's wait launches
+    //  the grouped engine on its stream; see pc.h "In-process rank groups")
   } else {
     cudaStream_t ws = host ? q->side : s;
     if (host) {
@@ -1018,16 +1117,21 @@ int pc_test(pc_request_t req, int *flag) {
     return 0;
   }
   PC_CUDA(cudaSetDevice(q->comm->device));
-  int rc = maybe_launch_engine(q);
-  if (rc) return rc;
+  int rc;
   const bool engine = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->copy == 1);
   bool done = false;
   if (engine) {
-    if (!q->engine_launched) {
+    cudaEvent_t ev = nullptr;
+    if (q->kind == PC_KIND_PSEND && !q->has_preq) {
       *flag = 0;
       return 0;
     }
-    cudaError_t e = cudaEventQuery(q->ev_done);
+    if ((rc = ensure_engine(q, false, &ev))) return rc;
+    if (!ev) {
+      *flag = 0;
+      return 0;
+    }
+    cudaError_t e = cudaEventQuery(ev);
     if (e == cudaErrorNotReady) {
       cudaGetLastError();
       done = false;
@@ -1081,7 +1185,7 @@ int pc_pready(int partition, pc_request_t req, pc_stream_t stream) {
 int pc_request_free(pc_request_t *req) {
   if (!req || !*req) return PC_ERR_ARG;
   Request *q = (Request *)*req;
-  if (q->active) return PC_ERR_STATE;
+  if (q->active && q->matched) return PC_ERR_STATE;  // an unmatched request has nothing in flight
   Comm *c = q->comm;
   if (!c->dry) {
     cudaSetDevice(c->device);
@@ -1091,6 +1195,7 @@ int pc_request_free(pc_request_t *req) {
     if (q->side) cudaStreamDestroy(q->side);
     if (q->ev_fork) cudaEventDestroy(q->ev_fork);
     if (q->ev_done) cudaEventDestroy(q->ev_done);
+    if (q->gs.ev) cudaEventDestroy(q->gs.ev);
   }
   c->reqs[q->index] = nullptr;
   delete q;
@@ -1133,6 +1238,26 @@ int pc_request_match(pc_request_t req, int *peer, int *peer_request_index) {
   *peer = q->peer;
   *peer_request_index = q->match_peer_index;
   return 0;
+}
+
+int pc_request_words(pc_request_t req, int which, int offset, int n, uint32_t *out) {
+  Request *q = (Request *)req;
+  if (!q || !out || which < 0 || which > 8 || offset < 0 || n < 0) return PC_ERR_ARG;
+  if (q->comm->dry || !q->ctrl) return PC_ERR_STATE;
+  const size_t base[9] = {q->L.flags, q->L.sent, q->L.cnt, q->L.ready, q->L.donecnt, q->L.rtr, q->L.epoch, q->L.layout, q->L.err};
+  const size_t lim[9] = {q->L.words - q->L.flags, q->L.donecnt - q->L.sent, q->L.ready - q->L.cnt,
+                         q->L.sent - q->L.ready, q->L.flags - q->L.donecnt, 8, 1, 1, 2};
+  if ((size_t)offset + (size_t)n > lim[which]) return PC_ERR_ARG;
+  PC_CUDA(cudaSetDevice(q->comm->device));
+  uint32_t *tmp = nullptr;
+  PC_CUDA(cudaMallocHost((void **)&tmp, (size_t)std::max(n, 1) * 4));
+  int rc = 0;
+  cudaError_t e = cudaMemcpyAsync(tmp, q->ctrl + base[which] + offset, (size_t)n * 4, cudaMemcpyDeviceToHost, q->side);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(q->side);
+  if (e != cudaSuccess) rc = cuda_err(e, "pc_request_words");
+  else memcpy(out, tmp, (size_t)n * 4);
+  cudaFreeHost(tmp);
+  return rc;
 }
 
 int pc_request_error(pc_request_t req, int *code, int *partition) {

@@ -151,9 +151,7 @@ __device__ __forceinline__ int modp(int a, int p) { return ((a % p) + p) % p; }
 // (reading R3) and hold epoch values, so they are never reset.
 // ---------------------------------------------------------------------------
 template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) ring_engine(RingArgs a) {
-  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int W = (gridDim.x * blockDim.x) >> 5;
+__device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const int W) {
   const int P = a.P, r = a.r, NS = 2 * (P - 1);
   const uint32_t e = a.e;
   const int64_t es = 4;
@@ -210,9 +208,7 @@ __global__ void __launch_bounds__(kEngineBlock) ring_engine(RingArgs a) {
 // accumulator) and pushed to the next partner in the same pass.
 // ---------------------------------------------------------------------------
 template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) rd_engine(RdArgs a) {
-  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int W = (gridDim.x * blockDim.x) >> 5;
+__device__ __forceinline__ void rd_body(const RdArgs &a, const int gw, const int W) {
   const int NS = a.nsteps;
   const uint32_t e = a.e;
   const int64_t es = 4;
@@ -255,6 +251,39 @@ __global__ void __launch_bounds__(kEngineBlock) rd_engine(RdArgs a) {
     }
     if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
   }
+}
+
+// Single-rank launches (one rank per GPU / process).
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) ring_engine(RingArgs a) {
+  ring_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
+}
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) rd_engine(RdArgs a) {
+  rd_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
+}
+
+// Grouped launches: the engines of every rank that shares this GPU inside one
+// process (virtual ranks) run as ONE kernel, so they are co-resident by
+// construction and no engine can sit behind another in a hardware queue
+// (DESIGN.md §"Virtual ranks").  Block b belongs to the rank whose block range
+// contains it; warps are numbered within that rank exactly as in the
+// single-rank launch.
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) ring_engine_group(RingGroupArgs g) {
+  int k = 0;
+  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
+  const int b = blockIdx.x - g.block_start[k];
+  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
+  ring_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
+}
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) rd_engine_group(RdGroupArgs g) {
+  int k = 0;
+  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
+  const int b = blockIdx.x - g.block_start[k];
+  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
+  rd_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
 }
 
 // ---------------------------------------------------------------------------
@@ -358,6 +387,34 @@ int launch_ring_engine(const RingArgs &a, int warps, cudaStream_t s) {
 int launch_rd_engine(const RdArgs &a, int warps, cudaStream_t s) {
   return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
     rd_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  });
+}
+
+int launch_ring_engine_group(const RingGroupArgs &g, int warps, cudaStream_t s) {
+  RingGroupArgs h = g;
+  int blocks = 0;
+  for (int k = 0; k < g.n; ++k) {
+    h.block_start[k] = blocks;
+    blocks += grid_for(warps, g.a[k].nunits);
+  }
+  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
+    ring_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  });
+}
+
+int launch_rd_engine_group(const RdGroupArgs &g, int warps, cudaStream_t s) {
+  RdGroupArgs h = g;
+  int blocks = 0;
+  for (int k = 0; k < g.n; ++k) {
+    h.block_start[k] = blocks;
+    blocks += grid_for(warps, g.a[k].nunits);
+  }
+  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
+    rd_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
     PC_CUDA(cudaGetLastError());
     return 0;
   });

@@ -53,6 +53,7 @@ struct ReqRec {
   int32_t dtype, op, algo, seq;
   int32_t owner;     // exporting rank
   int32_t req_index; // index in the owner's request list
+  uint64_t host_req; // Request* in the owner's process (co-located grouping)
   ShareRec buf;      // p2p: user buffer; allreduce: recvbuf
   ShareRec ctrl;     // control block
   ShareRec stage;    // allreduce staging
@@ -95,6 +96,18 @@ struct CtrlLayout {
 };
 
 struct Comm;
+struct Request;
+
+// Grouped engine launch state of co-located ranks (lives in the leader).
+struct GroupState {
+  std::mutex mu;
+  std::condition_variable cv;
+  uint32_t epoch = 0;
+  int pending = 0;
+  bool launched = false;
+  cudaEvent_t ev = nullptr;
+  std::vector<Request *> members;  // sorted by rank
+};
 
 struct Request {
   Comm *comm = nullptr;
@@ -115,7 +128,10 @@ struct Request {
   bool exchanged = false;
   bool prepared_this_epoch = false;
   bool engine_launched = false;
+  bool engine_registered = false;
   bool matched = false;
+  Request *leader = nullptr;  // co-located group leader (allreduce), or null
+  GroupState gs;
   int match_peer_index = -1;
 
   // device resources
@@ -217,7 +233,20 @@ struct P2pEngineArgs {
   uint32_t timeout_ms;
 };
 
+constexpr int kMaxLocal = 8;  // ranks of one comm sharing one GPU in one process
+struct RingGroupArgs {
+  int n;
+  int block_start[kMaxLocal];
+  RingArgs a[kMaxLocal];
+};
+struct RdGroupArgs {
+  int n;
+  int block_start[kMaxLocal];
+  RdArgs a[kMaxLocal];
+};
 int launch_ring_engine(const RingArgs &a, int warps, cudaStream_t s);
+int launch_ring_engine_group(const RingGroupArgs &g, int warps, cudaStream_t s);
+int launch_rd_engine_group(const RdGroupArgs &g, int warps, cudaStream_t s);
 int launch_rd_engine(const RdArgs &a, int warps, cudaStream_t s);
 int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s);
 // wait until words[i*stride] reached target (i < n); layout!=null: n derived

@@ -257,6 +257,16 @@ class Request:
         check(_lib.pc().pc_request_match(self.handle, C.byref(p), C.byref(i)), "pc_request_match")
         return p.value, i.value
 
+    WORDS = {"flags": 0, "sent": 1, "cnt": 2, "ready": 3, "done": 4, "rtr": 5, "epoch": 6, "layout": 7, "err": 8}
+
+    def words(self, which: str, offset: int, n: int):
+        """Read control words (debug/tests): flags, sent, cnt, ready, done, rtr, epoch."""
+        import numpy as np
+        out = np.zeros(max(n, 1), dtype=np.uint32)
+        check(_lib.pc().pc_request_words(self.handle, self.WORDS[which], offset, n, out.ctypes.data),
+              "pc_request_words")
+        return out[:n]
+
     def error(self) -> tuple[int, int]:
         c, p = C.c_int32(), C.c_int32()
         check(_lib.pc().pc_request_error(self.handle, C.byref(c), C.byref(p)), "pc_request_error")

@@ -1,6 +1,10 @@
 import os
 import sys
 
+# More hardware work queues: fewer false dependencies between the streams of
+# virtual ranks (must be set before the CUDA context exists).
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)

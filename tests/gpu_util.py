@@ -21,7 +21,7 @@ def dev():
 
 
 @contextlib.contextmanager
-def comms(P: int, timeout_ms: int = 20000):
+def comms(P: int, timeout_ms: int = 5000):
     old = os.environ.get("PC_TIMEOUT_MS")
     os.environ["PC_TIMEOUT_MS"] = str(timeout_ms)
     try:

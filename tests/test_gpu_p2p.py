@@ -48,13 +48,25 @@ def run_vecadd(n, gran, agg, copy, epochs=3, check_in_kernel=True):
             else:
                 rcv.pbuf_prepare(s1)
                 snd.pbuf_prepare(s0)
-            if check_in_kernel:
-                apps.check_recv(rq, R, out, partitions, count * 4, status, blocks=64, stream=s1)
+            # Producers first, consumers second: virtual ranks share hardware
+            # queues, so a spinning consumer must never be enqueued before the
+            # work it waits for.  The sender's wait launches its ENGINE (lazy
+            # launch), so it precedes the in-kernel Parrived consumer.
             apps.vecadd(A, B, Cb, n, gran, sq, s0)
             snd.wait_on_stream(s0)
+            if check_in_kernel:
+                apps.check_recv(rq, R, out, partitions, count * 4, status, blocks=64, stream=s1)
             rcv.wait_on_stream(s1)
             torch.cuda.synchronize()
-            assert snd.error()[0] == 0 and rcv.error()[0] == 0
+            if snd.error()[0] != 0 or rcv.error()[0] != 0:
+                f = rcv.words("flags", 0, -(-partitions // agg))
+                st = snd.words("sent", 0, -(-partitions // agg))
+                raise AssertionError(
+                    f"epoch {e}: snd err {snd.error()} rcv err {rcv.error()} status {int(status.item())} "
+                    f"flags<e+1 at {np.nonzero(f < e + 1)[0][:8]} vals {f[np.nonzero(f < e + 1)[0][:4]]} "
+                    f"sent<e+1 at {np.nonzero(st < e + 1)[0][:8]} layout/epoch {rcv.words('epoch', 0, 1)} "
+                    f"rtr {snd.words('rtr', 0, 2)} raw flags {[hex(v) for v in f[:12]]} max {hex(f.max())} "
+                    f"R[:4] {R[:4].tolist()} out[:4] {out[:4].tolist()}")
             sent_all.append((a + b).astype(np.float32))
             got_all.append(R.cpu().numpy().copy())
             got_kernel.append(out.cpu().numpy().copy())
@@ -209,18 +221,18 @@ def test_pingpong_latency_roundtrip(payload):
         b2a = pc.psend_init(bufs[2], iters, cnt, pc.FLOAT32, 0, 2, cs[1])
         a_in = pc.precv_init(bufs[3], iters, cnt, pc.FLOAT32, 1, 2, cs[0])
         bufs[0].copy_(torch.arange(bufs[0].numel(), dtype=torch.float32))
-        for q, s in ((a2b, s0), (a_in, s0), (b_in, s1), (b2a, s1)):
-            q.start(s)
-        first_prepare([[a2b, a_in], [b_in, b2a]], [s0, s1])
+        # the pair kernel runs on s0: every epoch word it reads is written on s0
+        for q in (a2b, a_in, b_in, b2a):
+            q.start(s0)
+        first_prepare([[a2b, a_in], [b_in, b2a]], [s0, s0])
         pa = a2b.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
         pai = a_in.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
         pb = b2a.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
         pbi = b_in.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
         t = torch.zeros(2, dtype=torch.int64, device="cuda")
-        apps.pingpong(pb, pbi, 1, iters, apps.GRAN_WARP, t[1:], s1)
-        apps.pingpong(pa, pai, 0, iters, apps.GRAN_WARP, t[:1], s0)
-        for q, s in ((a2b, s0), (a_in, s0), (b_in, s1), (b2a, s1)):
-            q.wait_on_stream(s)
+        apps.pingpong_pair(pa, pai, pb, pbi, iters, apps.GRAN_WARP, t, s0)
+        for q in (a2b, b2a, a_in, b_in):
+            q.wait_on_stream(s0)
         torch.cuda.synchronize()
         ns = int(t[0].item()) / iters / 2
         print(f"payload {payload} B: one-way {ns:.0f} ns (same-GPU virtual ranks)")

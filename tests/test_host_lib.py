@@ -1,0 +1,224 @@
+"""CPU tests of the C-ABI library: it loads, exports every symbol include/*.h
+declares, and its pure host logic (schedules, chunking, matching, request
+state machine) is right.  No compute calls — there is no GPU here.  Host-only
+("dry", device = -1) comms run the real bootstrap / exchange / matching code."""
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_temucinslsga24_b200 as pc
+from paper_conf_sc_temucinslsga24_b200 import _lib
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_library_exports_every_header_symbol():
+    lib = _lib.pc()
+    syms = _lib.header_symbols("pc.h")
+    assert len(syms) >= 30
+    for s in syms:
+        assert hasattr(lib, s), f"libpc.so does not export {s}"
+    assert lib.pc_prequest_size() == _lib.apps().pcapp_prequest_size()
+
+
+def test_no_oracle_in_product():
+    """The product never links or imports the oracle."""
+    out = subprocess.run(["nm", "-D", "--defined-only", _lib.LIBPC], capture_output=True, text=True).stdout
+    assert "orc_" not in out
+    for f in os.listdir(os.path.join(ROOT, "paper_conf_sc_temucinslsga24_b200")):
+        if f.endswith(".py"):
+            src = open(os.path.join(ROOT, "paper_conf_sc_temucinslsga24_b200", f)).read()
+            assert "import oracle" not in src and "from oracle" not in src
+
+
+@pytest.mark.parametrize("P", range(1, 9))
+def test_ring_schedule_matches_oracle_alg1(P):
+    """Two independent implementations of Alg 1 agree."""
+    for r in range(P):
+        np.testing.assert_array_equal(pc.schedule_ring(P, r), oracle.alg1_table(P, r))
+
+
+@pytest.mark.parametrize("P", [1, 2, 4, 8, 16])
+def test_rd_schedule(P):
+    k = int(np.log2(P))
+    for r in range(P):
+        t = pc.schedule_rd(P, r)
+        assert len(t) == k
+        partners = sorted(int(row[0]) for row in t)
+        assert partners == sorted(r ^ (1 << j) for j in range(k))
+        # symmetric: my partner at step j has me as its partner at step j
+        for j, row in enumerate(t):
+            assert pc.schedule_rd(P, int(row[0]))[j][0] == r
+
+
+def test_rd_schedule_rejects_non_power_of_two():
+    with pytest.raises(pc.PcError):
+        pc.schedule_rd(6, 0)
+
+
+@pytest.mark.parametrize("L", [0, 1, 3, 4, 5, 16, 17, 64, 1000, 300001])
+@pytest.mark.parametrize("P", [1, 2, 3, 5, 8])
+def test_chunk_bounds_match_oracle(L, P):
+    b = pc.chunk_bounds(L, P)
+    assert b[0] == 0 and b[-1] == L and (np.diff(b) >= 0).all()
+    ids = oracle.chunk_ids(L, P, 1)
+    for c in range(P):
+        assert (ids[b[c]:b[c + 1]] == c).all()
+    for c in range(1, P):
+        if b[c] < L:
+            assert b[c] % 4 == 0, "chunk starts are 16-byte aligned (reading R4)"
+
+
+def _dry(P):
+    return pc.local_comms(P, -1)
+
+
+def test_dry_p2p_matching_by_tag_and_order():
+    g, cs = _dry(2)
+    # rank 0 posts two sends with tag 5 and one with tag 9; rank 1 posts the
+    # receives in a different order: matching is by (peer, tag, posting order)
+    s = [pc.psend_init(0x1000, 4, 8, pc.FLOAT32, 1, 5, cs[0]), pc.psend_init(0x2000, 4, 8, pc.FLOAT32, 1, 9, cs[0]),
+         pc.psend_init(0x3000, 4, 8, pc.FLOAT32, 1, 5, cs[0])]
+    r = [pc.precv_init(0x4000, 4, 8, pc.FLOAT32, 0, 9, cs[1]), pc.precv_init(0x5000, 4, 8, pc.FLOAT32, 0, 5, cs[1]),
+         pc.precv_init(0x6000, 4, 8, pc.FLOAT32, 0, 5, cs[1])]
+    for q in s + r:
+        q.start()
+    pc.run_ranks([lambda: [q.pbuf_prepare() for q in s], lambda: [q.pbuf_prepare() for q in r]])
+    # request indices on the peer: s[0] <-> r[1], s[1] <-> r[0], s[2] <-> r[2]
+    assert s[0].match() == (1, 1) and s[1].match() == (1, 0) and s[2].match() == (1, 2)
+    assert r[1].match() == (0, 0) and r[0].match() == (0, 1) and r[2].match() == (0, 2)
+    for q in s + r:
+        q.wait()
+        q.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
+
+
+def test_dry_p2p_mismatch_is_reported():
+    g, cs = _dry(2)
+    a = pc.psend_init(0x1000, 4, 8, pc.FLOAT32, 1, 1, cs[0])
+    b = pc.precv_init(0x2000, 8, 4, pc.FLOAT32, 0, 1, cs[1])  # same bytes, different partitions
+    a.start()
+    b.start()
+    res = pc.run_ranks([lambda: _try(a.pbuf_prepare), lambda: _try(b.pbuf_prepare)])
+    assert res == [pc.ERR_MATCH, pc.ERR_MATCH]
+    for c in cs:
+        c.destroy()
+    g.destroy()
+
+
+def _try(f):
+    try:
+        f()
+        return 0
+    except pc.PcError as e:
+        return e.code
+
+
+def test_dry_allreduce_agreement_and_algo_choice():
+    g, cs = _dry(4)
+    reqs = [pc.pallreduce_init(0, 0, 2, 1 << 20, pc.FLOAT32, pc.SUM, pc.ALGO_AUTO, c) for c in cs]
+    small = [pc.pallreduce_init(0, 0, 1, 256, pc.FLOAT32, pc.SUM, pc.ALGO_AUTO, c) for c in cs]
+    for q in reqs + small:
+        q.start()
+    pc.run_ranks([(lambda r=r: (reqs[r].pbuf_prepare(), small[r].pbuf_prepare())) for r in range(4)])
+    assert all(q.info()["algo"] == pc.ALGO_RING for q in reqs)
+    assert all(q.info()["algo"] == pc.ALGO_RD for q in small)
+    infos = {tuple(sorted(q.info().items())) for q in reqs}
+    assert len(infos) == 1, "every rank must derive the same slicing"
+    # disagreeing allreduce (different count on rank 3) -> PC_ERR_MATCH everywhere it is checked
+    bad = [pc.pallreduce_init(0, 0, 1, 100 if r < 3 else 101, pc.INT32, pc.SUM, pc.ALGO_RING, cs[r]) for r in range(4)]
+    for q in bad:
+        q.start()
+    res = pc.run_ranks([(lambda r=r: _try(bad[r].pbuf_prepare)) for r in range(4)])
+    assert all(x == pc.ERR_MATCH for x in res)
+    for q in reqs + small:
+        q.wait()
+    for c in cs:
+        c.destroy()
+    g.destroy()
+
+
+def test_dry_state_errors():
+    g, cs = _dry(1)
+    q = pc.pallreduce_init(0, 0, 1, 16, pc.FLOAT32, pc.SUM, pc.ALGO_RING, cs[0])
+    with pytest.raises(pc.PcError) as e:
+        q.pbuf_prepare()  # not started
+    assert e.value.code == pc.ERR_STATE
+    q.start()
+    with pytest.raises(pc.PcError) as e:
+        q.start()  # start on an active request
+    assert e.value.code == pc.ERR_STATE
+    q.pbuf_prepare()
+    with pytest.raises(pc.PcError) as e:
+        q.free()  # free of an active (matched) request
+    assert e.value.code == pc.ERR_STATE
+    q.wait()
+    q.wait()  # wait on an inactive request: success
+    q.free()
+    cs[0].destroy()
+    g.destroy()
+
+
+def test_bad_arguments():
+    g, cs = _dry(2)
+    for f in (lambda: pc.psend_init(0, 0, 8, pc.FLOAT32, 1, 0, cs[0]),      # no partitions
+              lambda: pc.psend_init(0, 4, 8, pc.FLOAT32, 5, 0, cs[0]),      # bad peer
+              lambda: pc.pallreduce_init(0, 0, 1, 8, pc.BYTE, pc.SUM, 0, cs[0]),  # bad dtype
+              lambda: pc.pallreduce_init(0, 0, 1, 8, pc.FLOAT32, 7, 0, cs[0])):   # bad op
+        with pytest.raises(pc.PcError) as e:
+            f()
+        assert e.value.code == pc.ERR_ARG
+    for c in cs:
+        c.destroy()
+    g.destroy()
+
+
+_GLOO_WORKER = r"""
+import os, sys
+sys.path.insert(0, {root!r})
+import torch.distributed as dist
+import paper_conf_sc_temucinslsga24_b200 as pc
+dist.init_process_group("gloo", rank=int(os.environ["RANK"]), world_size=2)
+r = dist.get_rank()
+comm = pc.Comm.from_process_group(-1)
+assert comm.rank == r and comm.size == 2
+if r == 0:
+    a = pc.psend_init(0x1000, 4, 8, pc.FLOAT32, 1, 3, comm)
+    b = pc.precv_init(0x2000, 4, 8, pc.FLOAT32, 1, 4, comm)
+else:
+    b = pc.psend_init(0x1000, 4, 8, pc.FLOAT32, 0, 4, comm)
+    a = pc.precv_init(0x2000, 4, 8, pc.FLOAT32, 0, 3, comm)
+ar = pc.pallreduce_init(0, 0, 3, 1000, pc.FLOAT32, pc.SUM, pc.ALGO_RING, comm)
+for q in (a, b, ar):
+    q.start()
+for q in (a, b, ar):
+    q.pbuf_prepare()
+assert a.match() == (1 - r, 0) and b.match() == (1 - r, 1), (a.match(), b.match())
+info = ar.info()
+for q in (a, b, ar):
+    q.wait()
+    q.free()
+comm.destroy()
+print("OK", r, info["slices"])
+dist.destroy_process_group()
+"""
+
+
+def test_gloo_two_process_bootstrap_and_matching(tmp_path):
+    """The N>1 host path: two processes, torch.distributed gloo all-gather as
+    the bootstrap, request exchange + matching across processes."""
+    script = tmp_path / "w.py"
+    script.write_text(_GLOO_WORKER.format(root=ROOT))
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT=str(29500 + os.getpid() % 1000), WORLD_SIZE="2")
+    procs = [subprocess.Popen([sys.executable, str(script)], env=dict(env, RANK=str(r)), stdout=subprocess.PIPE,
+                              stderr=subprocess.STDOUT, text=True) for r in range(2)]
+    outs = [p.communicate(timeout=120)[0] for p in procs]
+    for r, (p, o) in enumerate(zip(procs, outs)):
+        assert p.returncode == 0, o
+        assert f"OK {r}" in o
