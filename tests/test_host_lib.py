@@ -199,7 +199,9 @@ for q in (a, b, ar):
     q.start()
 for q in (a, b, ar):
     q.pbuf_prepare()
-assert a.match() == (1 - r, 0) and b.match() == (1 - r, 1), (a.match(), b.match())
+# request indices on the peer: rank 0 created (a, b), rank 1 created (b, a)
+exp = ((1, 1), (1, 0)) if r == 0 else ((0, 0), (0, 1))
+assert (a.match(), b.match()) == exp, (a.match(), b.match())
 info = ar.info()
 for q in (a, b, ar):
     q.wait()
