@@ -169,6 +169,15 @@ int pc_request_match(pc_request_t req, int *peer, int *peer_request_index);
  * aggregation counters, 3 ready, 4 done/slice counters, 5 RTR words, 6 epoch)
  * starting at `offset` into host memory `out` (debug / tests; blocking). */
 int pc_request_words(pc_request_t req, int which, int offset, int n, uint32_t *out);
+/* Engine timing for benchmarks: when on, every engine launch of the request
+ * (or of its co-located group) is bracketed by CUDA events on the stream it
+ * runs on; pc_request_engine_times drains the durations (ms) of the launches
+ * since the last call into ms[0..max) and returns how many it wrote. */
+int pc_request_set_timing(pc_request_t req, int on);
+int pc_request_engine_times(pc_request_t req, float *ms, int max);
+/* Number of kernels libpc has launched in this process (for the bench's
+ * gpu_launches claim). */
+uint64_t pc_launch_count(void);
 /* Device error word of a request: code and partition (0,0 if none). */
 int pc_request_error(pc_request_t req, int *code, int *partition);
 const char *pc_strerror(int err);

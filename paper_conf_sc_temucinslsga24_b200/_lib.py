@@ -61,6 +61,9 @@ _PC_PROTOS = {
     "pc_request_match": (I32, [P, PI32, PI32]),
     "pc_request_error": (I32, [P, PI32, PI32]),
     "pc_request_words": (I32, [P, I32, I32, I32, P]),
+    "pc_request_set_timing": (I32, [P, I32]),
+    "pc_request_engine_times": (I32, [P, P, I32]),
+    "pc_launch_count": (C.c_uint64, []),
     "pc_strerror": (C.c_char_p, [I32]),
     "pc_version": (C.c_char_p, []),
 }
@@ -71,7 +74,7 @@ _APP_PROTOS = {
     "pcapp_check_recv": (I32, [P, P, P, I32, I64, I32, P, P]),
     "pcapp_pingpong": (I32, [P, P, I32, I32, I32, P, P]),
     "pcapp_bare_pingpong": (I32, [P, P, I32, I32, C.c_uint32, P, P]),
-    "pcapp_pingpong_pair": (I32, [P, P, P, P, I32, I32, P, P]),
+    "pcapp_pingpong_pair": (I32, [P, P, P, P, I32, I32, P, P, P]),
     "pcapp_bare_pingpong_pair": (I32, [P, P, I32, C.c_uint32, P, P]),
     "pcapp_prequest_size": (SZ, []),
 }

@@ -46,10 +46,11 @@ def bare_pingpong(my_flag, peer_flag, side: int, iters: int, base: int, out_ns, 
 
 
 def pingpong_pair(sendA: Prequest, recvA: Prequest, sendB: Prequest, recvB: Prequest, iters: int, gran: int,
-                  out_ns, stream=None):
-    """Both sides in one launch (virtual ranks on one GPU)."""
+                  out_ns, stream=None, rt_ns=None):
+    """Both sides in one launch (virtual ranks on one GPU).  rt_ns (optional,
+    int64[iters]) receives every round-trip time seen by side 0."""
     _ok(_lib.apps().pcapp_pingpong_pair(sendA.ptr, recvA.ptr, sendB.ptr, recvB.ptr, iters, gran, _ptr(out_ns),
-                                        _stream(stream)), "pingpong_pair")
+                                        _ptr(rt_ns), _stream(stream)), "pingpong_pair")
 
 
 def bare_pingpong_pair(flagA, flagB, iters: int, base: int, out_ns, stream=None):

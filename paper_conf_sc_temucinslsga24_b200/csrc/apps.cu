@@ -113,11 +113,13 @@ __global__ void pingpong_kernel(pc_prequest_t sendq, pc_prequest_t recvq, int si
 // ranks sharing a GPU, so the two spinning sides are co-resident by
 // construction.
 __global__ void pingpong_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, pc_prequest_t sendB,
-                                     pc_prequest_t recvB, int iters, int gran, unsigned long long *out_ns) {
+                                     pc_prequest_t recvB, int iters, int gran, unsigned long long *out_ns,
+                                     unsigned long long *rt_ns) {
   const int side = blockIdx.x;
   const pc_prequest_t &sq = side ? sendB : sendA;
   const pc_prequest_t &rq = side ? recvB : recvA;
   const uint64_t t0 = pc_detail::globaltimer();
+  uint64_t tk = t0;
   for (int k = 0; k < iters; ++k) {
     if (side == 1) {
       if (threadIdx.x == 0) pc_wait_arrived(rq, k);
@@ -129,7 +131,12 @@ __global__ void pingpong_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, p
       pc_pready_warp(k, sq);
     }
     if (side == 0) {
-      if (threadIdx.x == 0) pc_wait_arrived(rq, k);
+      if (threadIdx.x == 0) {
+        pc_wait_arrived(rq, k);
+        const uint64_t t = pc_detail::globaltimer();
+        if (rt_ns) rt_ns[k] = t - tk;  // one round trip = two Pready->Parrived hops
+        tk = t;
+      }
       __syncwarp();
     }
   }
@@ -221,9 +228,10 @@ int pcapp_bare_pingpong(uint32_t *my_flag, uint32_t *peer_flag, int side, int it
 }
 
 int pcapp_pingpong_pair(const pc_prequest_t *sendA, const pc_prequest_t *recvA, const pc_prequest_t *sendB,
-                        const pc_prequest_t *recvB, int iters, int gran, unsigned long long *out_ns, cudaStream_t s) {
+                        const pc_prequest_t *recvB, int iters, int gran, unsigned long long *out_ns,
+                        unsigned long long *rt_ns, cudaStream_t s) {
   if (!sendA || !recvA || !sendB || !recvB) return -1;
-  pingpong_pair_kernel<<<2, 32, 0, s>>>(*sendA, *recvA, *sendB, *recvB, iters, gran, out_ns);
+  pingpong_pair_kernel<<<2, 32, 0, s>>>(*sendA, *recvA, *sendB, *recvB, iters, gran, out_ns, rt_ns);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -580,11 +580,31 @@ static bool needs_engine(Request *q) {
   return q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
 }
 
+// Optional CUDA-event timing around an engine launch (pc_request_set_timing).
+static int timing_begin(TimingLog &T, cudaStream_t s, int *a) {
+  *a = -1;
+  if (!T.on || T.pending.size() >= 16384) return 0;
+  cudaEvent_t e;
+  if ((*a = T.get(&e)) < 0) return PC_ERR_CUDA;
+  PC_CUDA(cudaEventRecord(e, s));
+  return 0;
+}
+static int timing_end(TimingLog &T, cudaStream_t s, int a) {
+  if (a < 0) return 0;
+  cudaEvent_t e;
+  int b = T.get(&e);
+  if (b < 0) return PC_ERR_CUDA;
+  PC_CUDA(cudaEventRecord(e, s));
+  T.pending.push_back({(size_t)a, (size_t)b});
+  return 0;
+}
+
 // Single-rank launch on the request's side stream, forked from its user stream.
 static int launch_single(Request *q) {
   PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
   PC_CUDA(cudaStreamWaitEvent(q->side, q->ev_fork, 0));
-  int rc;
+  int rc, tk;
+  if ((rc = timing_begin(q->tlog, q->side, &tk))) return rc;
   if (q->kind == PC_KIND_PALLREDUCE) {
     rc = q->algo == PC_ALGO_RING ? launch_ring_engine(make_ring_args(q), q->engine_warps, q->side)
                                  : launch_rd_engine(make_rd_args(q), q->engine_warps, q->side);
@@ -610,6 +630,7 @@ static int launch_single(Request *q) {
     rc = launch_p2p_engine(a, q->engine_warps, q->side);
   }
   if (rc) return rc;
+  if ((rc = timing_end(q->tlog, q->side, tk))) return rc;
   PC_CUDA(cudaEventRecord(q->ev_done, q->side));
   q->engine_launched = true;
   return 0;
@@ -637,7 +658,8 @@ static int group_register(Request *q, bool block, bool *launched) {
   }
   if (!g.launched && g.pending == (int)g.members.size()) {
     for (Request *m : g.members) PC_CUDA(cudaStreamWaitEvent(q->side, m->ev_fork, 0));
-    int rc;
+    int rc, tk;
+    if ((rc = timing_begin(g.tlog, q->side, &tk))) return rc;
     if (q->algo == PC_ALGO_RING) {
       RingGroupArgs ga{};
       ga.n = (int)g.members.size();
@@ -650,6 +672,7 @@ static int group_register(Request *q, bool block, bool *launched) {
       rc = launch_rd_engine_group(ga, q->engine_warps, q->side);
     }
     if (rc) return rc;
+    if ((rc = timing_end(g.tlog, q->side, tk))) return rc;
     PC_CUDA(cudaEventRecord(g.ev, q->side));
     g.launched = true;
     g.cv.notify_all();
@@ -1196,6 +1219,8 @@ int pc_request_free(pc_request_t *req) {
     if (q->ev_fork) cudaEventDestroy(q->ev_fork);
     if (q->ev_done) cudaEventDestroy(q->ev_done);
     if (q->gs.ev) cudaEventDestroy(q->gs.ev);
+    for (cudaEvent_t e : q->gs.tlog.pool) cudaEventDestroy(e);
+    for (cudaEvent_t e : q->tlog.pool) cudaEventDestroy(e);
   }
   c->reqs[q->index] = nullptr;
   delete q;
@@ -1238,6 +1263,36 @@ int pc_request_match(pc_request_t req, int *peer, int *peer_request_index) {
   *peer = q->peer;
   *peer_request_index = q->match_peer_index;
   return 0;
+}
+
+uint64_t pc_launch_count(void) { return launch_count(); }
+
+int pc_request_set_timing(pc_request_t req, int on) {
+  Request *q = (Request *)req;
+  if (!q) return PC_ERR_ARG;
+  TimingLog &T = q->leader ? q->leader->gs.tlog : q->tlog;
+  T.on = on != 0;
+  q->tlog.on = on != 0;
+  return 0;
+}
+
+int pc_request_engine_times(pc_request_t req, float *ms, int max) {
+  Request *q = (Request *)req;
+  if (!q || (max > 0 && !ms)) return PC_ERR_ARG;
+  if (q->comm->dry) return 0;
+  PC_CUDA(cudaSetDevice(q->comm->device));
+  TimingLog &T = q->leader ? q->leader->gs.tlog : q->tlog;
+  int n = 0;
+  for (auto &pr : T.pending) {
+    PC_CUDA(cudaEventSynchronize(T.pool[pr.second]));
+    float v = 0.f;
+    PC_CUDA(cudaEventElapsedTime(&v, T.pool[pr.first], T.pool[pr.second]));
+    if (n < max) ms[n] = v;
+    ++n;
+  }
+  T.pending.clear();
+  T.next = 0;
+  return n < max ? n : max;
 }
 
 int pc_request_words(pc_request_t req, int which, int offset, int n, uint32_t *out) {

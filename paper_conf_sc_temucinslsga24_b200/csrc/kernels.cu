@@ -20,6 +20,8 @@
 // cycle while all engine warps are resident.
 #include <cuda_runtime.h>
 
+#include <atomic>
+
 #include "pc_device.cuh"
 #include "pc_internal.h"
 
@@ -368,6 +370,8 @@ int dispatch(int dtype, int op, F f) {
   return f(std::integral_constant<int, 1>(), std::integral_constant<int, 2>());
 }
 
+std::atomic<uint64_t> g_launches{0};
+
 int grid_for(int warps, int nunits) {
   int w = warps < nunits ? warps : nunits;
   if (w < 1) w = 1;
@@ -379,6 +383,7 @@ int grid_for(int warps, int nunits) {
 int launch_ring_engine(const RingArgs &a, int warps, cudaStream_t s) {
   return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
     ring_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    g_launches++;
     PC_CUDA(cudaGetLastError());
     return 0;
   });
@@ -387,6 +392,7 @@ int launch_ring_engine(const RingArgs &a, int warps, cudaStream_t s) {
 int launch_rd_engine(const RdArgs &a, int warps, cudaStream_t s) {
   return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
     rd_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    g_launches++;
     PC_CUDA(cudaGetLastError());
     return 0;
   });
@@ -401,6 +407,7 @@ int launch_ring_engine_group(const RingGroupArgs &g, int warps, cudaStream_t s) 
   }
   return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
     ring_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
+    g_launches++;
     PC_CUDA(cudaGetLastError());
     return 0;
   });
@@ -415,6 +422,7 @@ int launch_rd_engine_group(const RdGroupArgs &g, int warps, cudaStream_t s) {
   }
   return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
     rd_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
+    g_launches++;
     PC_CUDA(cudaGetLastError());
     return 0;
   });
@@ -422,6 +430,7 @@ int launch_rd_engine_group(const RdGroupArgs &g, int warps, cudaStream_t s) {
 
 int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
   p2p_engine<<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+  g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
 }
@@ -429,12 +438,14 @@ int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
 int launch_wait_words(const uint32_t *words, int n, uint32_t target, const uint32_t *layout, int partitions,
                       int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys) {
   wait_words_kernel<<<1, 256, 0, s>>>(words, n, target, layout, partitions, err, timeout_ms, sys ? 1 : 0);
+  g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
 }
 
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s) {
   set_word_kernel<<<1, 1, 0, s>>>(addr, value);
+  g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
 }
@@ -445,9 +456,12 @@ int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s) {
   if (blocks > 148) blocks = 148;
   if (blocks < 1) blocks = 1;
   pready_range_kernel<<<blocks, 256, 0, s>>>(q, lo, hi);
+  g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
 }
+
+uint64_t launch_count() { return g_launches.load(); }
 
 int engine_occupancy_ctas_per_sm(int *ctas) {
   int a = 0, b = 0;

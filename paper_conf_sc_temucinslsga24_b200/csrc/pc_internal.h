@@ -98,6 +98,24 @@ struct CtrlLayout {
 struct Comm;
 struct Request;
 
+// CUDA-event timing of engine launches (bench roofline: the dominant kernel's
+// duration measured live on the stream it runs on).
+struct TimingLog {
+  bool on = false;
+  std::vector<cudaEvent_t> pool;
+  size_t next = 0;
+  std::vector<std::pair<size_t, size_t>> pending;
+  int get(cudaEvent_t *ev) {  // returns pool index or -1
+    if (next == pool.size()) {
+      cudaEvent_t e;
+      if (cudaEventCreate(&e) != cudaSuccess) return -1;
+      pool.push_back(e);
+    }
+    *ev = pool[next];
+    return (int)next++;
+  }
+};
+
 // Grouped engine launch state of co-located ranks (lives in the leader).
 struct GroupState {
   std::mutex mu;
@@ -107,6 +125,7 @@ struct GroupState {
   bool launched = false;
   cudaEvent_t ev = nullptr;
   std::vector<Request *> members;  // sorted by rank
+  TimingLog tlog;
 };
 
 struct Request {
@@ -132,6 +151,7 @@ struct Request {
   bool matched = false;
   Request *leader = nullptr;  // co-located group leader (allreduce), or null
   GroupState gs;
+  TimingLog tlog;
   int match_peer_index = -1;
 
   // device resources
@@ -256,5 +276,6 @@ int launch_wait_words(const uint32_t *words, int n, uint32_t target, const uint3
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s);
 int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s);
 int engine_occupancy_ctas_per_sm(int *ctas);
+uint64_t launch_count();
 
 }  // namespace pc

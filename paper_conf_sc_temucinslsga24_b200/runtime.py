@@ -267,6 +267,16 @@ class Request:
               "pc_request_words")
         return out[:n]
 
+    def set_timing(self, on: bool = True):
+        check(_lib.pc().pc_request_set_timing(self.handle, int(on)), "pc_request_set_timing")
+
+    def engine_times(self, max_n: int = 65536):
+        """Durations (ms) of the engine launches since the last call (timing on)."""
+        import numpy as np
+        out = np.zeros(max_n, dtype=np.float32)
+        n = check(_lib.pc().pc_request_engine_times(self.handle, out.ctypes.data, max_n), "engine_times")
+        return out[:n]
+
     def error(self) -> tuple[int, int]:
         c, p = C.c_int32(), C.c_int32()
         check(_lib.pc().pc_request_error(self.handle, C.byref(c), C.byref(p)), "pc_request_error")
@@ -306,6 +316,11 @@ def pallreduce_init(sendbuf, recvbuf, partitions: int, count: int, dtype: int, o
 
 
 # ------------------------------------------------------------------ pure host logic
+def launch_count() -> int:
+    """Kernels libpc launched in this process so far."""
+    return int(_lib.pc().pc_launch_count())
+
+
 def schedule_ring(P: int, r: int):
     import numpy as np
     out = np.zeros((max(2 * (P - 1), 1), 5), dtype=np.int32)
