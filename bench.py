@@ -36,7 +36,7 @@ METRIC = "partitioned allreduce bus GB/s vs msg size at 2/4/8 B200; Pready→Par
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="pc", choices=["pc", "reference"])
     ap.add_argument("--bytes", type=int, default=256 << 20, help="bytes per rank (S)")
@@ -48,6 +48,13 @@ def parse():
     ap.add_argument("--no-latency", action="store_true")
     ap.add_argument("--quiet", action="store_true", help="only the JSON line")
     return ap.parse_args()
+
+
+T0 = time.time()
+
+
+def log(*a):
+    print(f"[bench {time.time() - T0:7.1f}s]", *a, file=sys.stderr, flush=True)
 
 
 def busbw(S, sec, P):
@@ -236,10 +243,14 @@ def run_virtual(args):
         for q in reqs:
             q.wait_on_stream(st)
 
+    log("init done; first step")
     step(first=True)
+    torch.cuda.synchronize()
+    log("first step done")
     for _ in range(max(args.warmup - 1, 0)):
         step()
     torch.cuda.synchronize()
+    log("warmup done")
     for q in reqs:
         assert q.error()[0] == 0, f"device error {q.error()}"
     info = reqs[0].info()
@@ -256,6 +267,7 @@ def run_virtual(args):
         torch.cuda.synchronize()
     launches = pc.launch_count() - n0
     ms = e0.elapsed_time(e1) / args.steps
+    log(f"timed: {ms:.3f} ms/step")
     eng = reqs[0].engine_times()
     reqs[0].set_timing(False)
     for q in reqs:
@@ -305,21 +317,28 @@ def run_virtual(args):
     f1.record(st)
     torch.cuda.synchronize()
     e2e_ms = f0.elapsed_time(f1) / ke
+    log(f"e2e: {e2e_ms:.3f} ms/step")
     e2e = {"value": busbw(S, e2e_ms / 1e3, P), "unit": "GB/s", "h2d_bytes_per_step": P * S, "d2h_bytes_per_step": S,
            "ms_per_step": e2e_ms, "api": "pc_start/pc_pbuf_prepare/pc_pready_range/pc_wait_on_stream per rank"}
 
     for q in reqs:
         q.free()
-    lat = None
-    if not args.no_latency:
-        lat = {"flag_only": latency_pair(pc, apps, torch, comms, payload=0),
-               "8B": latency_pair(pc, apps, torch, comms, payload=8),
-               "note": "2 virtual ranks on one B200 (flags/payload in the same HBM/L2, not NVLink)"}
     for c in comms:
         c.destroy()
     g.destroy()
+    lat = None
+    if not args.no_latency:
+        g2, c2 = pc.local_comms(2, 0)  # the exchange of new requests is collective over the comm
+        lat = {"flag_only": latency_pair(pc, apps, torch, c2, payload=0),
+               "8B": latency_pair(pc, apps, torch, c2, payload=8),
+               "note": "2 virtual ranks on one B200 (flags/payload in the same HBM/L2, not NVLink)"}
+        for c in c2:
+            c.destroy()
+        g2.destroy()
 
+    log("latency done")
     cpu = None if args.no_cpu_baseline else oracle_sample(P=P)
+    log("cpu baseline done")
     out = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": 1, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
