@@ -56,3 +56,150 @@ def pingpong_pair(sendA: Prequest, recvA: Prequest, sendB: Prequest, recvB: Preq
 def bare_pingpong_pair(flagA, flagB, iters: int, base: int, out_ns, stream=None):
     _ok(_lib.apps().pcapp_bare_pingpong_pair(_ptr(flagA), _ptr(flagB), iters, base, _ptr(out_ns),
                                              _stream(stream)), "bare_pingpong_pair")
+
+
+# --------------------------------------------------------------------------- Jacobi (a8)
+T, B, L, R = 0, 1, 2, 3
+_SEND_TAG = {T: 1, B: 2, L: 3, R: 4}   # tag = side of the SENDER the data leaves from
+_RECV_TAG = {T: 2, B: 1, L: 4, R: 3}   # halo on my side d comes from the neighbour's opposite side
+STRIP = 128
+
+
+class JacobiSolver:
+    """2D Jacobi over a Py x Px decomposition with intra-kernel partitioned
+    halo exchange.  `comms` holds the ranks this process
+    drives (all P virtual ranks, or the single rank of a multi-GPU process);
+    `ranks` are their comm ranks.  One epoch = one solve of `iters` iterations:
+    every halo partition is (iteration slot, edge segment), readied once."""
+
+    def __init__(self, comms, ranks, N: int, Py: int, Px: int, iters: int, H: int = 32, device: int = 0):
+        import torch
+        from . import runtime as rt
+        self.torch, self.rt = torch, rt
+        self.N, self.Py, self.Px, self.K, self.H = N, Py, Px, iters, H
+        assert N % Py == 0 and N % Px == 0
+        self.ly, self.lx = N // Py, N // Px
+        assert self.lx % STRIP == 0 and self.ly % H == 0, "lx must be a multiple of 128, ly of H"
+        self.comms, self.ranks = comms, ranks
+        dev = torch.device("cuda", device)
+        self.dev = dev
+        self.local = []
+        for comm, r in zip(comms, ranks):
+            py, px = divmod(r, Px)
+            nb = {T: (py - 1) * Px + px if py > 0 else -1, B: (py + 1) * Px + px if py < Py - 1 else -1,
+                  L: py * Px + px - 1 if px > 0 else -1, R: py * Px + px + 1 if px < Px - 1 else -1}
+            st = {"r": r, "py": py, "px": px, "nb": nb, "comm": comm,
+                  "grid": [torch.zeros(self.ly * self.lx, device=dev) for _ in range(2)],
+                  "send": {}, "halo": {}, "sreq": {}, "rreq": {}, "sq": {}, "rq": {}}
+            for d, q in nb.items():
+                if q < 0:
+                    continue
+                seg = STRIP if d in (T, B) else H
+                nseg = (self.lx if d in (T, B) else self.ly) // seg
+                parts = (iters + 1) * nseg
+                st["send"][d] = torch.zeros(parts * seg, device=dev)
+                st["halo"][d] = torch.zeros(parts * seg, device=dev)
+                st["sreq"][d] = rt.psend_init(st["send"][d], parts, seg, rt.FLOAT32, q, _SEND_TAG[d], comm)
+                st["rreq"][d] = rt.precv_init(st["halo"][d], parts, seg, rt.FLOAT32, q, _RECV_TAG[d], comm)
+            self.local.append(st)
+        self.desc = None
+        self.epochs = 0
+
+    def set_initial(self, a0):
+        """a0: full N x N host array (numpy) or None for the perf init (top edge 1)."""
+        import numpy as np
+        torch = self.torch
+        for st in self.local:
+            blk = a0[st["py"] * self.ly:(st["py"] + 1) * self.ly, st["px"] * self.lx:(st["px"] + 1) * self.lx]
+            st["grid"][0].copy_(torch.from_numpy(np.ascontiguousarray(blk, dtype=np.float32).reshape(-1)))
+            st["grid"][1].copy_(st["grid"][0])
+
+    def result(self):
+        """Gather the local blocks after the last solve into an N x N array."""
+        import numpy as np
+        out = np.zeros((self.N, self.N), dtype=np.float32)
+        for st in self.local:
+            g = st["grid"][self.K & 1].cpu().numpy().reshape(self.ly, self.lx)
+            out[st["py"] * self.ly:(st["py"] + 1) * self.ly, st["px"] * self.lx:(st["px"] + 1) * self.lx] = g
+        return out
+
+    def _reqs(self, st):
+        return list(st["sreq"].values()) + list(st["rreq"].values())
+
+    def _build_desc(self):
+        import ctypes as C
+        torch = self.torch
+        lib = _lib.apps()
+        sz = lib.pcapp_jacobi_rank_size()
+        raw = bytearray(sz * len(self.local))
+        starts = []
+        blocks = 0
+        for i, st in enumerate(self.local):
+            has = (C.c_int * 4)(*[1 if st["nb"][d] >= 0 else 0 for d in range(4)])
+            sendp = (C.c_void_p * 4)(*[st["send"][d].data_ptr() if d in st["send"] else 0 for d in range(4)])
+            halop = (C.c_void_p * 4)(*[st["halo"][d].data_ptr() if d in st["halo"] else 0 for d in range(4)])
+            sqp = (C.c_void_p * 4)(*[st["sq"][d].ptr if d in st["sq"] else 0 for d in range(4)])
+            rqp = (C.c_void_p * 4)(*[st["rq"][d].ptr if d in st["rq"] else 0 for d in range(4)])
+            buf = C.create_string_buffer(sz)
+            rc = lib.pcapp_jacobi_describe(buf, st["grid"][0].data_ptr(), st["grid"][1].data_ptr(), self.ly,
+                                           self.lx, self.H, st["py"] * self.ly, st["px"] * self.lx, self.N,
+                                           has, sendp, halop, sqp, rqp)
+            if rc != 0:
+                raise RuntimeError("pcapp_jacobi_describe failed")
+            raw[i * sz:(i + 1) * sz] = buf.raw
+            starts.append(blocks)
+            tiles = (self.ly // self.H) * (self.lx // STRIP)
+            blocks += (tiles + 7) // 8
+        self.desc = torch.frombuffer(raw, dtype=torch.uint8).to(self.dev)
+        self.starts = torch.tensor(starts, dtype=torch.int32, device=self.dev)
+        self.blocks = blocks
+
+    def solve(self, stream, first_prepare=None):
+        """One epoch: start + pbuf_prepare every request, the init push, K
+        iteration launches, then wait_on_stream (senders before receivers).
+        first_prepare(list_of_request_lists) runs the blocking first
+        pbuf_prepare across ranks (threads for co-located ranks)."""
+        lib = _lib.apps()
+        for st in self.local:
+            for q in self._reqs(st):
+                q.start(stream)
+        if self.epochs == 0:
+            lists = [self._reqs(st) for st in self.local]
+            if first_prepare is not None:
+                first_prepare(lists)
+            else:
+                for lst in lists:
+                    for q in lst:
+                        q.pbuf_prepare(stream)
+            for st in self.local:
+                for d, q in st["sreq"].items():
+                    st["sq"][d] = q.prequest_create(self.rt.GRAN_WARP, 1, self.rt.COPY_INLINE)
+                for d, q in st["rreq"].items():
+                    st["rq"][d] = q.prequest_create(self.rt.GRAN_WARP, 1, self.rt.COPY_INLINE)
+            self._build_desc()
+        else:
+            for st in self.local:
+                for q in self._reqs(st):
+                    q.pbuf_prepare(stream)
+        s = stream.cuda_stream if hasattr(stream, "cuda_stream") else (stream or 0)
+        n = len(self.local)
+        _ok(lib.pcapp_jacobi_launch(self.desc.data_ptr(), self.starts.data_ptr(), n, self.blocks, 0, 1, s),
+            "jacobi init")
+        for k in range(self.K):
+            _ok(lib.pcapp_jacobi_launch(self.desc.data_ptr(), self.starts.data_ptr(), n, self.blocks, k, 0, s),
+                "jacobi iter")
+        for st in self.local:
+            for q in st["sreq"].values():
+                q.wait_on_stream(stream)
+        for st in self.local:
+            for q in st["rreq"].values():
+                q.wait_on_stream(stream)
+        self.epochs += 1
+
+    def errors(self):
+        return [q.error() for st in self.local for q in self._reqs(st) if q.error()[0] != 0]
+
+    def free(self):
+        for st in self.local:
+            for q in self._reqs(st):
+                q.free()
