@@ -46,6 +46,9 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-latency", action="store_true")
+    ap.add_argument("--no-jacobi", action="store_true")
+    ap.add_argument("--jacobi-n", type=int, default=16384)
+    ap.add_argument("--jacobi-iters", type=int, default=50)
     ap.add_argument("--quiet", action="store_true", help="only the JSON line")
     return ap.parse_args()
 
@@ -209,6 +212,49 @@ def latency_pair(pc, apps, torch, comms, iters=5000, payload=0):
             "mean": float(rts.mean()), "payload_bytes": payload, "iters": iters, "errors": errs}
 
 
+def jacobi_bench(pc, apps, torch, args):
+    """C4: Jacobi 16384^2 fp32, 1 rank and 4x2 virtual ranks (intra-kernel
+    partitioned halos), GFLOP/s at 4 flops per interior cell update (R17) and
+    the HBM fraction at 8 B per cell update."""
+    import numpy as np
+    N, K = args.jacobi_n, args.jacobi_iters
+    hbm_peak, _ = peaks()
+    res = {}
+    for Py, Px in ((1, 1), (4, 2)):
+        P = Py * Px
+        g, cs = pc.local_comms(P, 0)
+        st = torch.cuda.Stream()
+        js = apps.JacobiSolver(cs, list(range(P)), N, Py, Px, K, H=32)
+        for s in js.local:  # perf init: top edge 1.0, rest 0
+            s["grid"][0].zero_()
+            if s["py"] == 0:
+                s["grid"][0][: js.lx].fill_(1.0)
+            s["grid"][1].copy_(s["grid"][0])
+        torch.cuda.synchronize()
+        fp = lambda lists: pc.run_ranks([(lambda l=l: [q.pbuf_prepare(st) for q in l]) for l in lists])
+        js.solve(st, first_prepare=fp)  # warm-up epoch
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = 3
+        e0.record(st)
+        for _ in range(reps):
+            js.solve(st)
+        e1.record(st)
+        torch.cuda.synchronize()
+        errs = js.errors()
+        ms_iter = e0.elapsed_time(e1) / (reps * (K + 1))  # K iterations + the init push
+        cells = (N - 2) * (N - 2)
+        res[f"{Py}x{Px}"] = {"gflops": 4.0 * cells / (ms_iter / 1e3) / 1e9, "us_per_iter": ms_iter * 1e3,
+                             "hbm_frac": (8.0 * N * N / (ms_iter / 1e3) / 1e9) / hbm_peak,
+                             "ranks": P, "errors": errs}
+        js.free()
+        for c in cs:
+            c.destroy()
+        g.destroy()
+    res["config"] = f"{N}^2 fp32, {K} iterations per epoch, virtual ranks on one B200, 8 B/cell-update roofline"
+    return res
+
+
 def run_virtual(args):
     import numpy as np
     import torch
@@ -337,6 +383,8 @@ def run_virtual(args):
         g2.destroy()
 
     log("latency done")
+    jac = None if args.no_jacobi else jacobi_bench(pc, apps, torch, args)
+    log("jacobi done")
     cpu = None if args.no_cpu_baseline else oracle_sample(P=P)
     log("cpu baseline done")
     out = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": 1, "steps": args.steps,
@@ -350,7 +398,7 @@ def run_virtual(args):
                       "l2": f"no flush: working set {3 * P * S >> 20} MiB >> 126 MB L2",
                       "parallelism": f"{P} virtual ranks / 1 GPU"},
            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-           "clocks": clk.summary(), "latency_ns": lat, "nccl": None}
+           "clocks": clk.summary(), "latency_ns": lat, "jacobi": jac, "nccl": None}
     print(json.dumps(out), flush=True)
 
 

@@ -30,12 +30,41 @@ namespace {
 
 using namespace pc_detail;
 
+#ifndef PC_ENGINE_UNROLL
+#define PC_ENGINE_UNROLL 8
+#endif
+constexpr int kU = PC_ENGINE_UNROLL;  // 16-B vectors in flight per operand per lane
+
+// Engine-side bounded spin: the awaited event is a whole slice step of the
+// upstream rank (tens of microseconds), so back off with __nanosleep early and
+// keep the L2 free of polling traffic.
+template <bool SYS>
+__device__ __forceinline__ bool engine_spin(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo, int part) {
+  uint32_t v = SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p);
+  if (reached(v, target)) return true;
+  const uint64_t t0 = globaltimer();
+  uint32_t ns = 64, n = 0;
+  for (;;) {
+    __nanosleep(ns);
+    if (ns < 1024) ns <<= 1;
+    v = SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p);
+    if (reached(v, target)) return true;
+    if ((++n & 15) == 0) {
+      if (aborted(err)) return false;
+      if (tmo && globaltimer() - t0 > (uint64_t)tmo * 1000000ull) {
+        set_error(err, PC_DEV_ERR_TIMEOUT, part);
+        return false;
+      }
+    }
+  }
+}
+
 // Warp-wide bounded wait on a flag word; lane 0 polls, the warp follows.
 template <bool SYS>
 __device__ __forceinline__ bool warp_wait(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo,
                                           int part) {
   bool ok = true;
-  if ((threadIdx.x & 31) == 0) ok = spin_geq<SYS>(p, target, err, tmo, part);
+  if ((threadIdx.x & 31) == 0) ok = engine_spin<SYS>(p, target, err, tmo, part);
   ok = __shfl_sync(0xffffffffu, ok, 0);
   __syncwarp();
   return ok;
@@ -100,20 +129,17 @@ __device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *
     uint4 *o1 = reinterpret_cast<uint4 *>(out1);
     uint4 *o2 = reinterpret_cast<uint4 *>(out2);
     int64_t k = lane;
-    for (; k + 96 < nv; k += 128) {
-      uint4 a0 = __ldcg(a + k), a1 = __ldcg(a + k + 32), a2 = __ldcg(a + k + 64), a3 = __ldcg(a + k + 96);
-      uint4 b0 = __ldcg(b + k), b1 = __ldcg(b + k + 32), b2 = __ldcg(b + k + 64), b3 = __ldcg(b + k + 96);
-      uint4 r0 = vop<DT, OP>(a0, b0), r1 = vop<DT, OP>(a1, b1), r2 = vop<DT, OP>(a2, b2),
-            r3 = vop<DT, OP>(a3, b3);
-      o1[k] = r0;
-      o1[k + 32] = r1;
-      o1[k + 64] = r2;
-      o1[k + 96] = r3;
-      if (out2) {
-        o2[k] = r0;
-        o2[k + 32] = r1;
-        o2[k + 64] = r2;
-        o2[k + 96] = r3;
+    for (; k + 32 * (kU - 1) < nv; k += 32 * kU) {
+      uint4 x[kU], y[kU];
+#pragma unroll
+      for (int j = 0; j < kU; ++j) x[j] = __ldcg(a + k + 32 * j);
+#pragma unroll
+      for (int j = 0; j < kU; ++j) y[j] = __ldcg(b + k + 32 * j);
+#pragma unroll
+      for (int j = 0; j < kU; ++j) {
+        const uint4 r = vop<DT, OP>(x[j], y[j]);
+        o1[k + 32 * j] = r;
+        if (out2) o2[k + 32 * j] = r;
       }
     }
     for (; k < nv; k += 32) {
@@ -135,8 +161,26 @@ __device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *
 }
 
 __device__ __forceinline__ void warp_copy(void *dst, const void *src, int64_t nbytes) {
-  copy_bytes(reinterpret_cast<uint8_t *>(dst), reinterpret_cast<const uint8_t *>(src), (uint64_t)nbytes,
-             threadIdx.x & 31, 32);
+  const uint32_t lane = threadIdx.x & 31;
+  if (((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src)) & 15) == 0) {
+    const int64_t nv = nbytes >> 4;
+    const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
+    uint4 *d4 = reinterpret_cast<uint4 *>(dst);
+    int64_t k = lane;
+    for (; k + 32 * (kU - 1) < nv; k += 32 * kU) {
+      uint4 x[kU];
+#pragma unroll
+      for (int j = 0; j < kU; ++j) x[j] = __ldcg(s4 + k + 32 * j);
+#pragma unroll
+      for (int j = 0; j < kU; ++j) d4[k + 32 * j] = x[j];
+    }
+    for (; k < nv; k += 32) d4[k] = __ldcg(s4 + k);
+    const int64_t done = nv << 4;
+    if (done < nbytes) copy_bytes(reinterpret_cast<uint8_t *>(dst) + done, reinterpret_cast<const uint8_t *>(src) + done,
+                                  (uint64_t)(nbytes - done), lane, 32);
+    return;
+  }
+  copy_bytes(reinterpret_cast<uint8_t *>(dst), reinterpret_cast<const uint8_t *>(src), (uint64_t)nbytes, lane, 32);
 }
 
 __device__ __forceinline__ int modp(int a, int p) { return ((a % p) + p) % p; }
