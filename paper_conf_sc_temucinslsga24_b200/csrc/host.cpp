@@ -923,15 +923,18 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   q->engine_warps = c->engine_warps;
   const int64_t L = (int64_t)count;
   const int64_t min_elems = env_long("PC_MIN_SLICE_BYTES", 8192) / 4;
+  // units (partition slices) per engine warp: each warp sweeps its units
+  // round-robin (Alg 2), so a few per warp absorb upstream skew
+  const int upw = (int)std::max(1L, std::min(8L, env_long("PC_UNITS_PER_WARP", 4)));
   if (a == PC_ALGO_RING) {
     q->nsteps = 2 * (P - 1);
     q->chunk_elems = chunk_q(L, P);
-    choose_slices(q->chunk_elems, partitions, c->engine_warps, min_elems, &q->slices, &q->slice_elems);
+    choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems);
     q->staging_bytes = P > 1 ? bytes : 0;
   } else {
     q->nsteps = log2_exact(P);
     q->chunk_elems = L;
-    choose_slices(L, partitions, c->engine_warps, min_elems, &q->slices, &q->slice_elems);
+    choose_slices(L, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems);
     q->staging_bytes = bytes * (uint64_t)q->nsteps;
   }
   const size_t nflags = (size_t)partitions * (size_t)std::max(q->nsteps, 1) * (size_t)q->slices;

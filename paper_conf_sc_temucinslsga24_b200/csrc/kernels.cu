@@ -196,55 +196,121 @@ __device__ __forceinline__ int modp(int a, int p) { return ((a % p) + p) % p; }
 // Operand order local ⊕ incoming (reading R5); flags are per (u, step, slice)
 // (reading R3) and hold epoch values, so they are never reset.
 // ---------------------------------------------------------------------------
+// Alg 2 on a warp: the warp owns up to kMaxActive units and
+// sweeps them round-robin, polling each unit's next dependency once and
+// performing the step of every unit that is ready — exactly the per-partition
+// state machine of Alg 2, with the progression thread replaced by the warp.
+// A slow upstream unit therefore never idles the warp while another of its
+// units can advance.  Dependencies form a DAG over (unit, step, rank), so
+// progress only needs every engine warp to be resident.
+constexpr int kMaxActive = 8;
+
+__device__ __forceinline__ bool warp_poll(const uint32_t *p, uint32_t target, bool sys) {
+  bool ok = false;
+  if ((threadIdx.x & 31) == 0) ok = reached(sys ? ld_acquire_sys(p) : ld_acquire_gpu(p), target);
+  return __shfl_sync(0xffffffffu, ok, 0);
+}
+
+// Idle backoff shared by the sweeping engines; false on abort / timeout.
+struct Idle {
+  uint64_t since = 0;
+  uint32_t ns = 0;
+  __device__ __forceinline__ void progressed() {
+    since = 0;
+    ns = 0;
+  }
+  __device__ __forceinline__ bool wait(int32_t *err, uint32_t tmo, int part) {
+    if (since == 0) since = globaltimer();
+    ns = ns ? (ns < 1024 ? ns * 2 : 1024) : 64;
+    __nanosleep(ns);
+    if (aborted(err)) return false;
+    if (tmo && globaltimer() - since > (uint64_t)tmo * 1000000ull) {
+      if ((threadIdx.x & 31) == 0) set_error(err, PC_DEV_ERR_TIMEOUT, part);
+      return false;
+    }
+    return true;
+  }
+};
+
+template <int DT, int OP>
+__device__ __forceinline__ void ring_step(const RingArgs &a, int u, int s, int i) {
+  const int P = a.P, r = a.r, NS = 2 * (P - 1);
+  const int64_t es = 4;
+  const int64_t base = (int64_t)u * a.L;
+  const int64_t fbase = (int64_t)u * NS * a.ns + s;  // flag (u, i, s) = fbase + i * ns
+  const int c = modp(r - i, P);                     // R_i = A_{i-1}
+  const int64_t c_lo = min((int64_t)c * a.q, a.L), c_hi = min((int64_t)(c + 1) * a.q, a.L);
+  const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
+  const int64_t n = hi > lo ? hi - lo : 0;
+  const int64_t off = (base + lo) * es;
+  if (n) {
+    if (i == 0)  // E_0: the user's Pready of S_0
+      warp_copy(a.o_staging + off, a.sendbuf + off, n * es);
+    else if (i <= P - 2)
+      warp_reduce<DT, OP>(a.o_staging + off, nullptr, a.sendbuf + off, a.staging + off, n);
+    else if (i == P - 1)
+      warp_reduce<DT, OP>(a.recvbuf + off, a.o_recvbuf + off, a.sendbuf + off, a.staging + off, n);
+    else
+      warp_copy(a.o_recvbuf + off, a.recvbuf + off, n * es);
+  }
+  warp_signal(a.o_flags + fbase + (int64_t)i * a.ns, a.e);
+}
+
 template <int DT, int OP>
 __device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const int W) {
-  const int P = a.P, r = a.r, NS = 2 * (P - 1);
+  const int P = a.P, NS = 2 * (P - 1);
   const uint32_t e = a.e;
   const int64_t es = 4;
-  bool rtr_ok = false;
-  for (int x = gw; x < a.nunits; x += W) {
-    const int u = x / a.ns, s = x % a.ns;
-    const int64_t base = (int64_t)u * a.L;
-    if (!warp_wait<false>(a.ready + u, e, a.err, a.timeout_ms, u)) return;
-    if (P == 1) {
-      const int64_t lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
+  if (gw >= a.nunits) return;
+  if (P == 1) {
+    for (int x = gw; x < a.nunits; x += W) {
+      const int u = x / a.ns, s = x % a.ns;
+      if (!warp_wait<false>(a.ready + u, e, a.err, a.timeout_ms, u)) return;
+      const int64_t base = (int64_t)u * a.L, lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
       if (hi > lo && a.sendbuf != a.recvbuf)
         warp_copy(a.recvbuf + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
       __syncwarp();
       if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-      continue;
     }
-    if (!rtr_ok) {
-      if (!warp_wait<true>(a.rtr, e, a.err, a.timeout_ms, -1)) return;
-      rtr_ok = true;
+    return;
+  }
+  // the consumer's ready-to-receive (written by a stream memop, never by an engine)
+  if (!warp_wait<true>(a.rtr, e, a.err, a.timeout_ms, -1)) return;
+  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
+    int step[kMaxActive];
+    int remaining = 0;
+#pragma unroll
+    for (int j = 0; j < kMaxActive; ++j) {
+      const bool mine = gw + (j0 + j) * W < a.nunits;
+      step[j] = mine ? 0 : NS + 1;
+      remaining += mine;
     }
-    const int64_t fbase = (int64_t)u * NS * a.ns + s;  // flag (u, i, s) = fbase + i * ns
-    // E_0: the user's Pready of step S_0
-    {
-      const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
-      const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-      if (hi > lo) warp_copy(a.o_staging + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
-      warp_signal(a.o_flags + fbase, e);
-    }
-    for (int i = 1; i <= 2 * P - 3; ++i) {
-      const int c = modp(r - i, P);
-      if (!warp_wait<true>(a.flags + fbase + (int64_t)(i - 1) * a.ns, e, a.err, a.timeout_ms, u)) return;
-      const int64_t c_lo = min((int64_t)c * a.q, a.L), c_hi = min((int64_t)(c + 1) * a.q, a.L);
-      const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-      const int64_t n = hi > lo ? hi - lo : 0;
-      const int64_t off = (base + lo) * es;
-      if (n) {
-        if (i <= P - 2)
-          warp_reduce<DT, OP>(a.o_staging + off, nullptr, a.sendbuf + off, a.staging + off, n);
-        else if (i == P - 1)
-          warp_reduce<DT, OP>(a.recvbuf + off, a.o_recvbuf + off, a.sendbuf + off, a.staging + off, n);
-        else
-          warp_copy(a.o_recvbuf + off, a.recvbuf + off, n * es);
+    Idle idle;
+    while (remaining) {
+      bool progressed = false;
+#pragma unroll
+      for (int j = 0; j < kMaxActive; ++j) {
+        if (step[j] > NS) continue;
+        const int x = gw + (j0 + j) * W;
+        const int u = x / a.ns, s = x % a.ns;
+        const int i = step[j];
+        const uint32_t *dep = i == 0 ? a.ready + u : a.flags + ((int64_t)u * NS + (i - 1)) * a.ns + s;
+        if (!warp_poll(dep, e, i != 0)) continue;
+        progressed = true;
+        if (i < NS) {
+          ring_step<DT, OP>(a, u, s, i);
+          step[j] = i + 1;
+        } else {  // arrival of the last AG step: partition slice final here
+          if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+          step[j] = NS + 1;
+          --remaining;
+        }
       }
-      warp_signal(a.o_flags + fbase + (int64_t)i * a.ns, e);
+      if (progressed)
+        idle.progressed();
+      else if (!idle.wait(a.err, a.timeout_ms, gw))
+        return;
     }
-    if (!warp_wait<true>(a.flags + fbase + (int64_t)(2 * P - 3) * a.ns, e, a.err, a.timeout_ms, u)) return;
-    if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
   }
 }
 
