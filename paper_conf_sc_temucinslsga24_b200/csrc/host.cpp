@@ -925,7 +925,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   const int64_t min_elems = env_long("PC_MIN_SLICE_BYTES", 8192) / 4;
   // units (partition slices) per engine warp: each warp sweeps its units
   // round-robin (Alg 2), so a few per warp absorb upstream skew
-  const int upw = (int)std::max(1L, std::min(8L, env_long("PC_UNITS_PER_WARP", 4)));
+  const int upw = (int)std::max(1L, std::min(8L, env_long("PC_UNITS_PER_WARP", 1)));
   if (a == PC_ALGO_RING) {
     q->nsteps = 2 * (P - 1);
     q->chunk_elems = chunk_q(L, P);
