@@ -68,6 +68,16 @@ PC_DEVICE uint32_t ld_acquire_gpu(const uint32_t *p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+/* {p[0], p[1]} in one system-scope acquire (the epoch word and the RTR word
+ * are adjacent in the control block: one L2 round trip for both). */
+PC_DEVICE uint2 ld_acquire_sys_v2(const uint32_t *p) {
+  uint2 v;
+  asm volatile("ld.acquire.sys.global.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p) : "memory");
+  return v;
+}
+PC_DEVICE void st_relaxed_gpu(uint32_t *p, uint32_t v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 PC_DEVICE uint32_t ld_relaxed_sys(const uint32_t *p) {
   uint32_t v;
   asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -176,8 +186,11 @@ PC_DEVICE uint32_t transport_size(const pc_prequest_t &q, int t) {
 
 /* Count `add` contributions to transport partition t; returns true for the
  * single contribution that completes t in epoch e.  Flags a duplicate Pready
- * (counter already at/over the target) in the sticky error word. */
+ * (counter already at/over the target) in the sticky error word.  With g = 1
+ * every Pready completes its own transport partition: no counter (the
+ * latency-critical path; duplicate detection needs g > 1). */
 PC_DEVICE bool contribute(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, int part) {
+  if (q.agg == 1) return true;
   const uint32_t target = e * transport_size(q, t);
   const uint32_t old = atom_add_acq_rel_gpu(q.cnt + t, add);
   const int32_t d = (int32_t)(target - old);
@@ -188,14 +201,15 @@ PC_DEVICE bool contribute(const pc_prequest_t &q, int t, uint32_t add, uint32_t 
   return d <= (int32_t)add;
 }
 
-/* INLINE push of transport partition t by the lanes in `mask` (warp scope). */
-PC_DEVICE void push_warp(const pc_prequest_t &q, int t, uint32_t e, unsigned mask) {
+/* INLINE push of transport partition t by the lanes in `mask` (warp scope).
+ * rtr0: the RTR value the caller already loaded together with the epoch. */
+PC_DEVICE void push_warp(const pc_prequest_t &q, int t, uint32_t e, unsigned mask, uint32_t rtr0 = 0) {
   const uint32_t lane = lane_id();
   const uint32_t first = __ffs(mask) - 1;
   const uint32_t idx = __popc(mask & ((1u << lane) - 1));
   const uint32_t n = __popc(mask);
   bool ok = true;
-  if (lane == first) ok = spin_geq<true>(q.rtr, e, q.err, q.timeout_ms, t);
+  if (lane == first && !reached(rtr0, e)) ok = spin_geq<true>(q.rtr, e, q.err, q.timeout_ms, t);
   ok = __shfl_sync(mask, ok, first);
   if (!ok) return;
   const uint64_t off = (uint64_t)t * (uint64_t)q.agg * q.part_bytes;
@@ -205,7 +219,7 @@ PC_DEVICE void push_warp(const pc_prequest_t &q, int t, uint32_t e, unsigned mas
   __syncwarp(mask);
   if (lane == first) {
     st_relaxed_sys(q.peer_flags + t, e);
-    st_release_gpu(q.sent + t, e);
+    st_relaxed_gpu(q.sent + t, e);  // ordered by the fence above
   }
 }
 
@@ -224,7 +238,7 @@ PC_DEVICE void push_block(const pc_prequest_t &q, int t, uint32_t e) {
   __syncthreads();
   if (tid == 0) {
     st_relaxed_sys(q.peer_flags + t, e);
-    st_release_gpu(q.sent + t, e);
+    st_relaxed_gpu(q.sent + t, e);  // ordered by the fence above
   }
 }
 
@@ -281,23 +295,29 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
     if (lane == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);
     return PC_DEV_ERR_ARG;
   }
-  const uint32_t e = epoch_of(preq);
   if (preq.kind == PC_KIND_PALLREDUCE) {
-    if (lane == 0) st_release_gpu(preq.ready + partition, e);
+    if (lane == 0) st_release_gpu(preq.ready + partition, epoch_of(preq));
     __syncwarp(full);
     return 0;
   }
   const int t = partition / preq.agg;
   bool completes = false;
-  if (lane == 0) completes = contribute(preq, t, 1, e, partition);
+  uint32_t e = 0, rtr0 = 0;
+  if (lane == 0) {
+    const uint2 er = ld_acquire_sys_v2(preq.epoch);  // {epoch, rtr[0]}
+    e = er.x;
+    rtr0 = er.y;
+    completes = contribute(preq, t, 1, e, partition);
+  }
   completes = __shfl_sync(full, completes, 0);
   if (!completes) return 0;
+  e = __shfl_sync(full, e, 0);
   if (preq.copy == 1) {
     if (lane == 0) st_release_gpu(preq.ready + t, e);
     __syncwarp(full);
     return 0;
   }
-  push_warp(preq, t, e, full);
+  push_warp(preq, t, e, full, rtr0);
   return 0;
 }
 
@@ -345,19 +365,47 @@ PC_DEVICE int pc_parrived(pc_prequest_t preq, int partition) {
   return reached(ld_acquire_sys(preq.flags + partition / (int)g), e);
 }
 
-/* Acquire-spin until pc_parrived(preq, partition) (bounded by timeout_ms). */
+/* Acquire-spin until pc_parrived(preq, partition) (bounded by timeout_ms).
+ * The epoch and the transport layout are read once; the loop is a single
+ * ld.acquire of the partition's flag (one L2 round trip per poll). */
 PC_DEVICE int pc_wait_arrived(pc_prequest_t preq, int partition) {
   using namespace pc_detail;
+  if (partition < 0 || partition >= preq.partitions) return PC_DEV_ERR_ARG;
   const uint64_t t0 = globaltimer();
+  const uint32_t e = epoch_of(preq);
+  const uint32_t *w;
+  uint32_t target = e;
+  bool sys = false;
+  if (preq.kind == PC_KIND_PALLREDUCE) {
+    w = preq.done + partition;
+    target = e * preq.done_mul;
+  } else if (preq.kind == PC_KIND_PSEND) {
+    w = preq.sent + partition / preq.agg;
+  } else {
+    uint32_t g;
+    uint32_t n = 0;
+    while ((g = *(const volatile uint32_t *)preq.layout) == 0) {  // sender not set up yet
+      if ((++n & 127) == 0) {
+        if (aborted(preq.err)) return PC_DEV_ERR_TIMEOUT;
+        if (preq.timeout_ms && globaltimer() - t0 > (uint64_t)preq.timeout_ms * 1000000ull) {
+          set_error(preq.err, PC_DEV_ERR_TIMEOUT, partition);
+          return PC_DEV_ERR_TIMEOUT;
+        }
+        __nanosleep(256);
+      }
+    }
+    w = preq.flags + partition / (int)g;
+    sys = true;
+  }
   uint32_t n = 0;
-  while (!pc_parrived(preq, partition)) {
+  while (!reached(sys ? ld_acquire_sys(w) : ld_acquire_gpu(w), target)) {
     if ((++n & 127) == 0) {
       if (aborted(preq.err)) return PC_DEV_ERR_TIMEOUT;
       if (preq.timeout_ms && globaltimer() - t0 > (uint64_t)preq.timeout_ms * 1000000ull) {
         set_error(preq.err, PC_DEV_ERR_TIMEOUT, partition);
         return PC_DEV_ERR_TIMEOUT;
       }
-      if (n > 1024) __nanosleep(256);
+      if (n > 4096) __nanosleep(128);
     }
   }
   return 0;

@@ -75,7 +75,7 @@ struct LocalGroup {
 // ------------------------------------------------------------------ control block layout
 // One device allocation per request.  Words are u32.  Offsets in words.
 struct CtrlLayout {
-  size_t epoch = 0;        // [1]
+  size_t epoch = 0;        // [1]   (pc_device.cuh loads {epoch, rtr[0]} as one 8-byte word)
   size_t rtr = 1;          // [kMaxRdSteps + 2] ready-to-receive words (per incoming producer slot)
   size_t layout = 10;      // [1] g published by the sender (receive side)
   size_t err = 12;         // [2] sticky device error (int32 code, partition)

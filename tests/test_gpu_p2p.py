@@ -174,7 +174,9 @@ def test_duplicate_pready_is_reported():
         snd.start(s0)
         rcv.start(s1)
         first_prepare([[snd], [rcv]], [s0, s1])
-        snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+        # g = 2: both partitions feed one transport partition, so a duplicate
+        # Pready overshoots the aggregation counter (g = 1 has no counter)
+        snd.prequest_create(pc.GRAN_BLOCK, 2, pc.COPY_INLINE)
         snd.pready(0, s0)
         snd.pready(0, s0)  # duplicate in the same epoch
         snd.pready(1, s0)
