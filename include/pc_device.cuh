@@ -75,6 +75,11 @@ PC_DEVICE uint2 ld_acquire_sys_v2(const uint32_t *p) {
   asm volatile("ld.acquire.sys.global.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p) : "memory");
   return v;
 }
+PC_DEVICE uint2 ld_acquire_gpu_v2(const uint32_t *p) {
+  uint2 v;
+  asm volatile("ld.acquire.gpu.global.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p) : "memory");
+  return v;
+}
 PC_DEVICE void st_relaxed_gpu(uint32_t *p, uint32_t v) {
   asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -101,6 +106,18 @@ PC_DEVICE void red_add_release_gpu(uint32_t *p, uint32_t v) {
   asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 PC_DEVICE void fence_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+PC_DEVICE void fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+/* Release fence at the scope the request needs: system scope when a peer is
+ * another GPU (NVLink), GPU scope when every peer shares this GPU. */
+PC_DEVICE void fence_scope(uint32_t sys) {
+  if (sys)
+    fence_sys();
+  else
+    fence_gpu();
+}
+PC_DEVICE uint32_t ld_acquire_scope(const uint32_t *p, uint32_t sys) {
+  return sys ? ld_acquire_sys(p) : ld_acquire_gpu(p);
+}
 PC_DEVICE uint64_t globaltimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -208,14 +225,21 @@ PC_DEVICE void push_warp(const pc_prequest_t &q, int t, uint32_t e, unsigned mas
   const uint32_t first = __ffs(mask) - 1;
   const uint32_t idx = __popc(mask & ((1u << lane) - 1));
   const uint32_t n = __popc(mask);
+  const uint64_t off = (uint64_t)t * (uint64_t)q.agg * q.part_bytes;
+  const uint64_t len = (uint64_t)transport_size(q, t) * q.part_bytes;
+  if (len == 0) {  // flag only: no data to protect or order -> no RTR wait, no fence
+    if (lane == first) {
+      st_relaxed_sys(q.peer_flags + t, e);
+      st_relaxed_gpu(q.sent + t, e);
+    }
+    return;
+  }
   bool ok = true;
   if (lane == first && !reached(rtr0, e)) ok = spin_geq<true>(q.rtr, e, q.err, q.timeout_ms, t);
   ok = __shfl_sync(mask, ok, first);
   if (!ok) return;
-  const uint64_t off = (uint64_t)t * (uint64_t)q.agg * q.part_bytes;
-  const uint64_t len = (uint64_t)transport_size(q, t) * q.part_bytes;
   copy_bytes(q.peer_rbuf + off, q.sbuf + off, len, idx, n);
-  fence_sys();
+  fence_scope(q.sys_scope);
   __syncwarp(mask);
   if (lane == first) {
     st_relaxed_sys(q.peer_flags + t, e);
@@ -234,7 +258,7 @@ PC_DEVICE void push_block(const pc_prequest_t &q, int t, uint32_t e) {
   const uint64_t off = (uint64_t)t * (uint64_t)q.agg * q.part_bytes;
   const uint64_t len = (uint64_t)transport_size(q, t) * q.part_bytes;
   copy_bytes(q.peer_rbuf + off, q.sbuf + off, len, tid, nthr);
-  fence_sys();
+  fence_scope(q.sys_scope);
   __syncthreads();
   if (tid == 0) {
     st_relaxed_sys(q.peer_flags + t, e);
@@ -304,7 +328,7 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   bool completes = false;
   uint32_t e = 0, rtr0 = 0;
   if (lane == 0) {
-    const uint2 er = ld_acquire_sys_v2(preq.epoch);  // {epoch, rtr[0]}
+    const uint2 er = preq.sys_scope ? ld_acquire_sys_v2(preq.epoch) : ld_acquire_gpu_v2(preq.epoch);  // {epoch, rtr[0]}
     e = er.x;
     rtr0 = er.y;
     completes = contribute(preq, t, 1, e, partition);
@@ -362,7 +386,7 @@ PC_DEVICE int pc_parrived(pc_prequest_t preq, int partition) {
   }
   const uint32_t g = *(const volatile uint32_t *)preq.layout;
   if (g == 0) return 0;  // sender has not published its transport layout yet
-  return reached(ld_acquire_sys(preq.flags + partition / (int)g), e);
+  return reached(ld_acquire_scope(preq.flags + partition / (int)g, preq.sys_scope), e);
 }
 
 /* Acquire-spin until pc_parrived(preq, partition) (bounded by timeout_ms).
@@ -395,10 +419,12 @@ PC_DEVICE int pc_wait_arrived(pc_prequest_t preq, int partition) {
       }
     }
     w = preq.flags + partition / (int)g;
-    sys = true;
+    sys = preq.sys_scope != 0;
   }
+  // no bytes to read after the flag -> a relaxed poll is enough
+  const bool relaxed = preq.part_bytes == 0;
   uint32_t n = 0;
-  while (!reached(sys ? ld_acquire_sys(w) : ld_acquire_gpu(w), target)) {
+  while (!reached(relaxed ? ld_relaxed_sys(w) : (sys ? ld_acquire_sys(w) : ld_acquire_gpu(w)), target)) {
     if ((++n & 127) == 0) {
       if (aborted(preq.err)) return PC_DEV_ERR_TIMEOUT;
       if (preq.timeout_ms && globaltimer() - t0 > (uint64_t)preq.timeout_ms * 1000000ull) {

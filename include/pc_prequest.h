@@ -42,6 +42,9 @@ struct pc_prequest_s {
   const uint32_t *done;       /* allreduce: [N_p] per-partition completion counters      */
   uint32_t done_mul;          /* allreduce: partition u is final when done[u] >= e*done_mul */
   int32_t rank;               /* owning rank                                              */
+  uint32_t sys_scope;         /* 1: a peer is on another GPU -> system-scope fences /
+                                 acquires; 0: every peer shares this GPU -> GPU scope
+                                 (a system-scope fence costs ~1.5 us on B200)           */
   int32_t *err;               /* sticky device error word [2] = {code, partition}         */
 };
 

@@ -163,6 +163,50 @@ __global__ void bare_pingpong_pair_kernel(uint32_t *flagA, uint32_t *flagB, int 
   out_ns[side] = pc_detail::globaltimer() - t0;
 }
 
+// Flag ping-pong microbenchmark over memory-order variants (latency floor
+// study): 0 st.release.sys/ld.acquire.sys, 1 relaxed.sys,
+// 2 release/acquire.gpu, 3 relaxed.gpu, 4 fence.acq_rel.sys+st.relaxed.sys /
+// ld.acquire.sys, 5 volatile.
+template <int V>
+__device__ __forceinline__ void vstore(uint32_t *p, uint32_t v) {
+  if (V == 0) asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+  if (V == 1) asm volatile("st.relaxed.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+  if (V == 2) asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+  if (V == 3) asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+  if (V == 4) asm volatile("fence.acq_rel.sys;\n\tst.relaxed.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+  if (V == 5) asm volatile("st.volatile.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+template <int V>
+__device__ __forceinline__ uint32_t vload(const uint32_t *p) {
+  uint32_t v;
+  if (V == 0 || V == 4) asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  if (V == 1) asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  if (V == 2) asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  if (V == 3) asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  if (V == 5) asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+template <int V>
+__global__ void flag_variant_kernel(uint32_t *flagA, uint32_t *flagB, int iters, uint32_t base,
+                                    unsigned long long *out_ns) {
+  if (threadIdx.x != 0) return;
+  const int side = blockIdx.x;
+  uint32_t *mine = side ? flagB : flagA;
+  uint32_t *peer = side ? flagA : flagB;
+  const uint64_t t0 = pc_detail::globaltimer();
+  for (int k = 1; k <= iters; ++k) {
+    const uint32_t v = base + (uint32_t)k;
+    if (side == 1)
+      while (!pc_detail::reached(vload<V>(mine), v)) {
+      }
+    vstore<V>(peer, v);
+    if (side == 0)
+      while (!pc_detail::reached(vload<V>(mine), v)) {
+      }
+  }
+  out_ns[side] = pc_detail::globaltimer() - t0;
+}
+
 // Latency floor: the same ping-pong with a bare flag and no library.
 __global__ void bare_pingpong_kernel(uint32_t *my_flag, uint32_t *peer_flag, int side, int iters, uint32_t base,
                                      unsigned long long *out_ns) {
@@ -238,6 +282,19 @@ int pcapp_pingpong_pair(const pc_prequest_t *sendA, const pc_prequest_t *recvA, 
 int pcapp_bare_pingpong_pair(uint32_t *flagA, uint32_t *flagB, int iters, uint32_t base, unsigned long long *out_ns,
                              cudaStream_t s) {
   bare_pingpong_pair_kernel<<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_flag_variant(uint32_t *flagA, uint32_t *flagB, int variant, int iters, uint32_t base,
+                       unsigned long long *out_ns, cudaStream_t s) {
+  switch (variant) {
+    case 0: flag_variant_kernel<0><<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns); break;
+    case 1: flag_variant_kernel<1><<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns); break;
+    case 2: flag_variant_kernel<2><<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns); break;
+    case 3: flag_variant_kernel<3><<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns); break;
+    case 4: flag_variant_kernel<4><<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns); break;
+    default: flag_variant_kernel<5><<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns); break;
+  }
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

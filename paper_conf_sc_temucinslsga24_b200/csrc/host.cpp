@@ -304,6 +304,7 @@ static void fill_prequest(Request *q, pc_prequest_t *o) {
   o->layout = q->ctrl + q->L.layout;
   o->done = q->ctrl + q->L.donecnt;
   o->done_mul = (uint32_t)q->slices;
+  o->sys_scope = (uint32_t)q->sys_scope;
   o->err = (int32_t *)(q->ctrl + q->L.err);
   if (q->kind == PC_KIND_PSEND) {
     o->peer_rbuf = q->peer_buf;
@@ -430,6 +431,7 @@ static int exchange_round(Comm *c, Request *target) {
           q->exchanged = true;
           q->matched = true;
           q->match_peer_index = m->req_index;
+          q->sys_scope = c->dry || memcmp(c->ranks[q->peer].uuid, c->ranks[c->rank].uuid, 16) != 0;
         }
       }
     } else {  // PALLREDUCE: the seq-th allreduce of every rank
@@ -476,6 +478,9 @@ static int exchange_round(Comm *c, Request *target) {
         if (!qrc) {
           q->exchanged = true;
           q->matched = true;
+          q->sys_scope = c->dry ? 1 : 0;
+          for (int k = 0; k < P; ++k)
+            if (memcmp(c->ranks[k].uuid, c->ranks[c->rank].uuid, 16) != 0) q->sys_scope = 1;
           // ranks of this comm sharing this GPU inside this process run their
           // engines as one grouped launch
           std::vector<int> loc;
@@ -542,6 +547,7 @@ static RingArgs make_ring_args(Request *q) {
   a.o_flags = q->nb_ctrl[0] ? q->nb_ctrl[0] + q->L.flags : nullptr;
   a.err = (int32_t *)(q->ctrl + q->L.err);
   a.timeout_ms = c->timeout_ms;
+  a.sys = q->sys_scope;
   return a;
 }
 
@@ -573,6 +579,7 @@ static RdArgs make_rd_args(Request *q) {
   }
   a.err = (int32_t *)(q->ctrl + q->L.err);
   a.timeout_ms = c->timeout_ms;
+  a.sys = q->sys_scope;
   return a;
 }
 
@@ -627,6 +634,7 @@ static int launch_single(Request *q) {
     a.sent = q->ctrl + q->L.sent;
     a.err = (int32_t *)(q->ctrl + q->L.err);
     a.timeout_ms = q->comm->timeout_ms;
+    a.sys = q->sys_scope;
     rc = launch_p2p_engine(a, q->engine_warps, q->side);
   }
   if (rc) return rc;

@@ -38,8 +38,8 @@ constexpr int kU = PC_ENGINE_UNROLL;  // 16-B vectors in flight per operand per 
 // Engine-side bounded spin: the awaited event is a whole slice step of the
 // upstream rank (tens of microseconds), so back off with __nanosleep early and
 // keep the L2 free of polling traffic.
-template <bool SYS>
-__device__ __forceinline__ bool engine_spin(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo, int part) {
+__device__ __forceinline__ bool engine_spin(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo, int part,
+                                            bool SYS) {
   uint32_t v = SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p);
   if (reached(v, target)) return true;
   const uint64_t t0 = globaltimer();
@@ -60,20 +60,21 @@ __device__ __forceinline__ bool engine_spin(const uint32_t *p, uint32_t target, 
 }
 
 // Warp-wide bounded wait on a flag word; lane 0 polls, the warp follows.
-template <bool SYS>
-__device__ __forceinline__ bool warp_wait(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo,
-                                          int part) {
+// sys: acquire at system scope (word written from another GPU).
+__device__ __forceinline__ bool warp_wait(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo, int part,
+                                          bool sys) {
   bool ok = true;
-  if ((threadIdx.x & 31) == 0) ok = engine_spin<SYS>(p, target, err, tmo, part);
+  if ((threadIdx.x & 31) == 0) ok = engine_spin(p, target, err, tmo, part, sys);
   ok = __shfl_sync(0xffffffffu, ok, 0);
   __syncwarp();
   return ok;
 }
 
-// Publish: every lane's (peer) stores are made visible at system scope, then
-// lane 0 stores the epoch into the consumer's flag.
-__device__ __forceinline__ void warp_signal(uint32_t *flag, uint32_t e) {
-  fence_sys();
+// Publish: every lane's (peer) stores are made visible at the request's scope
+// (system scope for a peer on another GPU), then lane 0 stores the epoch into
+// the consumer's flag.
+__device__ __forceinline__ void warp_signal(uint32_t *flag, uint32_t e, bool sys) {
+  fence_scope(sys);
   __syncwarp();
   if ((threadIdx.x & 31) == 0) st_relaxed_sys(flag, e);
 }
@@ -253,7 +254,7 @@ __device__ __forceinline__ void ring_step(const RingArgs &a, int u, int s, int i
     else
       warp_copy(a.o_recvbuf + off, a.recvbuf + off, n * es);
   }
-  warp_signal(a.o_flags + fbase + (int64_t)i * a.ns, a.e);
+  warp_signal(a.o_flags + fbase + (int64_t)i * a.ns, a.e, a.sys);
 }
 
 template <int DT, int OP>
@@ -265,7 +266,7 @@ __device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const
   if (P == 1) {
     for (int x = gw; x < a.nunits; x += W) {
       const int u = x / a.ns, s = x % a.ns;
-      if (!warp_wait<false>(a.ready + u, e, a.err, a.timeout_ms, u)) return;
+      if (!warp_wait(a.ready + u, e, a.err, a.timeout_ms, u, false)) return;
       const int64_t base = (int64_t)u * a.L, lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
       if (hi > lo && a.sendbuf != a.recvbuf)
         warp_copy(a.recvbuf + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
@@ -275,7 +276,7 @@ __device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const
     return;
   }
   // the consumer's ready-to-receive (written by a stream memop, never by an engine)
-  if (!warp_wait<true>(a.rtr, e, a.err, a.timeout_ms, -1)) return;
+  if (!warp_wait(a.rtr, e, a.err, a.timeout_ms, -1, a.sys)) return;
   for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
     int step[kMaxActive];
     int remaining = 0;
@@ -295,7 +296,7 @@ __device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const
         const int u = x / a.ns, s = x % a.ns;
         const int i = step[j];
         const uint32_t *dep = i == 0 ? a.ready + u : a.flags + ((int64_t)u * NS + (i - 1)) * a.ns + s;
-        if (!warp_poll(dep, e, i != 0)) continue;
+        if (!warp_poll(dep, e, i != 0 && a.sys)) continue;
         progressed = true;
         if (i < NS) {
           ring_step<DT, OP>(a, u, s, i);
@@ -331,7 +332,7 @@ __device__ __forceinline__ void rd_body(const RdArgs &a, const int gw, const int
     const int64_t lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
     const int64_t n = hi > lo ? hi - lo : 0;
     const int64_t off = ((int64_t)u * a.L + lo) * es;
-    if (!warp_wait<false>(a.ready + u, e, a.err, a.timeout_ms, u)) return;
+    if (!warp_wait(a.ready + u, e, a.err, a.timeout_ms, u, false)) return;
     if (NS == 0) {
       if (n && a.sendbuf != a.recvbuf) warp_copy(a.recvbuf + off, a.sendbuf + off, n * es);
       __syncwarp();
@@ -340,22 +341,22 @@ __device__ __forceinline__ void rd_body(const RdArgs &a, const int gw, const int
     }
     auto fidx = [&](int k) { return ((int64_t)u * NS + k) * a.ns + s; };
     if (!(rtr_ok & 1u)) {
-      if (!warp_wait<true>(a.rtr + 0, e, a.err, a.timeout_ms, -1)) return;
+      if (!warp_wait(a.rtr + 0, e, a.err, a.timeout_ms, -1, a.sys)) return;
       rtr_ok |= 1u;
     }
     if (n) warp_copy(a.p_staging[0] + off, a.sendbuf + off, n * es);
-    warp_signal(a.p_flags[0] + fidx(0), e);
+    warp_signal(a.p_flags[0] + fidx(0), e, a.sys);
     for (int k = 0; k < NS; ++k) {
-      if (!warp_wait<true>(a.flags + fidx(k), e, a.err, a.timeout_ms, u)) return;
+      if (!warp_wait(a.flags + fidx(k), e, a.err, a.timeout_ms, u, a.sys)) return;
       const uint8_t *acc = (k == 0) ? a.sendbuf : a.recvbuf;
       const uint8_t *in = a.staging + (int64_t)k * stride;
       if (k < NS - 1) {
         if (!(rtr_ok & (1u << (k + 1)))) {
-          if (!warp_wait<true>(a.rtr + k + 1, e, a.err, a.timeout_ms, -1)) return;
+          if (!warp_wait(a.rtr + k + 1, e, a.err, a.timeout_ms, -1, a.sys)) return;
           rtr_ok |= 1u << (k + 1);
         }
         if (n) warp_reduce<DT, OP>(a.recvbuf + off, a.p_staging[k + 1] + off, acc + off, in + off, n);
-        warp_signal(a.p_flags[k + 1] + fidx(k + 1), e);
+        warp_signal(a.p_flags[k + 1] + fidx(k + 1), e, a.sys);
       } else {
         if (n) warp_reduce<DT, OP>(a.recvbuf + off, nullptr, acc + off, in + off, n);
         __syncwarp();
@@ -408,9 +409,9 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
   bool rtr_ok = false;
   for (int x = gw; x < a.nunits; x += W) {
     const int t = x / a.ns, s = x % a.ns;
-    if (!warp_wait<false>(a.ready + t, e, a.err, a.timeout_ms, t)) return;
+    if (!warp_wait(a.ready + t, e, a.err, a.timeout_ms, t, false)) return;
     if (!rtr_ok) {
-      if (!warp_wait<true>(a.rtr, e, a.err, a.timeout_ms, -1)) return;
+      if (!warp_wait(a.rtr, e, a.err, a.timeout_ms, -1, a.sys)) return;
       rtr_ok = true;
     }
     const int rem = a.partitions - t * a.agg;
@@ -419,7 +420,7 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
     const uint64_t slo = (uint64_t)s * a.slice_bytes;
     const uint64_t n = slo < len ? min(a.slice_bytes, len - slo) : 0;
     if (n) warp_copy(a.peer_rbuf + off + slo, a.sbuf + off + slo, (int64_t)n);
-    fence_sys();
+    fence_scope(a.sys);
     __syncwarp();
     if ((threadIdx.x & 31) == 0) {
       const uint32_t old = atom_add_acq_rel_gpu(a.donecnt + t, 1);

@@ -174,6 +174,8 @@ struct Request {
   // consumers of this rank (they get an RTR write from us): ctrl + rtr slot
   std::vector<std::pair<uint32_t *, int>> rtr_targets;
 
+  // memory-model scope: 1 when a peer of this request is on another GPU
+  int sys_scope = 1;
   // prequest (p2p)
   bool has_preq = false;
   int agg = 1, ntransport = 0, copy = 0;
@@ -224,6 +226,7 @@ struct RingArgs {
   uint32_t *o_flags;
   int32_t *err;
   uint32_t timeout_ms;
+  int sys;  // 1: some peer is another GPU -> system-scope fences/acquires
 };
 struct RdArgs {
   uint32_t e;
@@ -238,6 +241,7 @@ struct RdArgs {
   uint32_t *p_flags[kMaxRdSteps];
   int32_t *err;
   uint32_t timeout_ms;
+  int sys;
 };
 struct P2pEngineArgs {
   uint32_t e;
@@ -251,6 +255,7 @@ struct P2pEngineArgs {
   uint32_t *donecnt, *sent;
   int32_t *err;
   uint32_t timeout_ms;
+  int sys;
 };
 
 constexpr int kMaxLocal = 8;  // ranks of one comm sharing one GPU in one process
