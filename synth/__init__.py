@@ -129,3 +129,8 @@ def jacobi_init(ny: int, nx: int, kind: str = "perf", seed: int = BASE_SEED) -> 
     if kind == "random":
         return uniform_f32(seed, 0, 0, ny * nx, 0.0, 1.0).reshape(ny, nx)
     raise ValueError(kind)
+
+
+def uniform_f32_at(seed, rank, epoch, idx, lo=-1.0, hi=1.0) -> np.ndarray:
+    """uniform_f32 values at arbitrary indices (sampled parity at full size)."""
+    return (lo + (hi - lo) * _unit(u64_at(seed, rank, epoch, idx))).astype(np.float32)

@@ -1,0 +1,62 @@
+"""Worker for test_gpu_multiproc: one process per rank, every rank on cuda:0
+(the box has one GPU), bootstrap over a gloo process group, peers mapped with
+CUDA IPC — the N > 1 code path of bench.py except that ranks share a GPU."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+import torch.distributed as dist  # noqa: E402
+
+import paper_conf_sc_temucinslsga24_b200 as pc  # noqa: E402
+import synth  # noqa: E402
+from paper_conf_sc_temucinslsga24_b200 import apps  # noqa: E402
+
+out_dir = sys.argv[1]
+dist.init_process_group("gloo")
+r, P = dist.get_rank(), dist.get_world_size()
+torch.cuda.set_device(0)
+comm = pc.Comm.from_process_group(0)
+st = torch.cuda.Stream()
+res = {}
+for name, algo in (("ring", pc.ALGO_RING), ("rd", pc.ALGO_RD)):
+    Np, L = 3, 1000
+    x = synth.normal_f32(synth.BASE_SEED, r, 0, Np * L)
+    send = torch.from_numpy(x).cuda()
+    recv = torch.zeros_like(send)
+    q = pc.pallreduce_init(send, recv, Np, L, pc.FLOAT32, pc.SUM, algo, comm)
+    for e in range(2):
+        q.start(st)
+        q.pbuf_prepare(st)
+        q.pready_range(0, Np - 1, st)
+        q.wait_on_stream(st)
+    st.synchronize()
+    assert q.error() == (0, 0), q.error()
+    res[name] = recv.cpu().numpy()
+    q.free()
+# p2p 0 -> 1 with block-granularity Pready from the producer kernel
+n = 2048 * 8
+if r == 0:
+    a = torch.from_numpy(synth.uniform_f32(synth.BASE_SEED, 0, 0, n)).cuda()
+    b = torch.from_numpy(synth.uniform_f32(synth.BASE_SEED, 0, 1, n)).cuda()
+    c = torch.empty(n, device="cuda")
+    q = pc.psend_init(c, 8, 2048, pc.FLOAT32, 1, 9, comm)
+else:
+    rb = torch.zeros(n, device="cuda")
+    q = pc.precv_init(rb, 8, 2048, pc.FLOAT32, 0, 9, comm)
+q.start(st)
+q.pbuf_prepare(st)
+pq = q.prequest_create(pc.GRAN_BLOCK, 2, pc.COPY_INLINE)
+if r == 0:
+    apps.vecadd(a, b, c, n, apps.GRAN_BLOCK, pq, st)
+q.wait()
+assert q.error() == (0, 0), q.error()
+if r == 1:
+    res["p2p"] = rb.cpu().numpy()
+q.free()
+np.savez(os.path.join(out_dir, f"rank{r}.npz"), **res)
+comm.destroy()
+dist.destroy_process_group()
+print("worker OK", r)
