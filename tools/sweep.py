@@ -1,0 +1,198 @@
+"""C5 / C3 / C2 sweeps on one B200 (virtual ranks), JSONL to stdout.
+
+  python tools/sweep.py allreduce [--ranks 2,4,8] [--algos ring,rd]
+  python tools/sweep.py dl                      # ResNet-50 / BERT-large gradient buffers
+  python tools/sweep.py p2p                     # C2: Pready granularity x aggregation x copy mode
+
+Each point: busBW (allreduce) or GB/s (p2p) from CUDA events over many
+back-to-back epochs on one stream (the bench step), median of 3 blocks."""
+import argparse
+import json
+import os
+import statistics
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
+import torch  # noqa: E402
+
+import paper_conf_sc_temucinslsga24_b200 as pc  # noqa: E402
+import synth  # noqa: E402
+from paper_conf_sc_temucinslsga24_b200 import apps  # noqa: E402
+
+
+def busbw(S, sec, P):
+    return S / sec * 2.0 * (P - 1) / P / 1e9 if P > 1 else S / sec / 1e9
+
+
+def time_allreduce(cs, S, Np, algo, min_ms=30.0):
+    P = len(cs)
+    count = max(S // 4 // Np, 1)
+    n = count * Np
+    st = torch.cuda.Stream()
+    send = [torch.randn(n, device="cuda") for _ in range(P)]
+    recv = [torch.empty(n, device="cuda") for _ in range(P)]
+    reqs = [pc.pallreduce_init(send[r], recv[r], Np, count, pc.FLOAT32, pc.SUM, algo, cs[r]) for r in range(P)]
+
+    def step(first=False):
+        for q in reqs:
+            q.start(st)
+        if first:
+            pc.run_ranks([(lambda q=q: q.pbuf_prepare(st)) for q in reqs])
+        else:
+            for q in reqs:
+                q.pbuf_prepare(st)
+        for q in reqs:
+            q.pready_range(0, Np - 1, st)
+        for q in reqs:
+            q.wait_on_stream(st)
+
+    step(True)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    step()
+    e1.record(st)
+    torch.cuda.synchronize()
+    one = max(e0.elapsed_time(e1), 1e-3)
+    iters = int(max(5, min(2000, min_ms / one)))
+    blocks = []
+    for _ in range(3):
+        e0.record(st)
+        for _ in range(iters):
+            step()
+        e1.record(st)
+        torch.cuda.synchronize()
+        blocks.append(e0.elapsed_time(e1) / iters)
+    errs = [q.error() for q in reqs if q.error()[0] != 0]
+    info = reqs[0].info()
+    for q in reqs:
+        q.free()
+    ms = statistics.median(blocks)
+    return {"bytes_per_rank": n * 4, "partitions": Np, "ranks": P, "algo": ["auto", "ring", "rd"][algo],
+            "us_per_step": ms * 1e3, "busbw_gbs": busbw(n * 4, ms / 1e3, P), "slices": info["slices"],
+            "errors": errs}
+
+
+def sweep_allreduce(args):
+    for P in [int(x) for x in args.ranks.split(",")]:
+        g, cs = pc.local_comms(P, 0)
+        for algo in args.algos.split(","):
+            a = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "auto": pc.ALGO_AUTO}[algo]
+            if a == pc.ALGO_RD and P & (P - 1):
+                continue
+            S = 1 << 10
+            while S <= args.max_bytes:
+                for Np in [int(x) for x in args.partitions.split(",")]:
+                    if S // 4 // Np < P:
+                        continue
+                    r = time_allreduce(cs, S, Np, a)
+                    print(json.dumps(r), flush=True)
+                S <<= 2
+        for c in cs:
+            c.destroy()
+        g.destroy()
+
+
+def sweep_dl(args):
+    for P in [int(x) for x in args.ranks.split(",")]:
+        g, cs = pc.local_comms(P, 0)
+        for name, sizes, part_bytes in (("resnet50", synth.RESNET50_SIZES, 1 << 20),
+                                        ("bert_large", synth.BERT_LARGE_SIZES, 4 << 20)):
+            total = sum(sizes) * 4
+            Np = max(1, total // part_bytes)
+            r = time_allreduce(cs, total, Np, pc.ALGO_RING)
+            r["model"] = name
+            r["tensors"] = len(sizes)
+            print(json.dumps(r), flush=True)
+        for c in cs:
+            c.destroy()
+        g.destroy()
+
+
+def sweep_p2p(args):
+    """C2: vector-add producer + Pready at thread/warp/block granularity with
+    aggregation g, INLINE vs ENGINE; goodput = bytes / (kernel + comm) time."""
+    g2, cs = pc.local_comms(2, 0)
+    st = torch.cuda.Stream()
+    elems = {apps.GRAN_THREAD: 2, apps.GRAN_WARP: 64, apps.GRAN_BLOCK: 2048}
+    for S in [64 << 10, 1 << 20, 16 << 20, 256 << 20]:
+        n = S // 4
+        A = torch.randn(n, device="cuda")
+        B = torch.randn(n, device="cuda")
+        Cb = torch.empty(n, device="cuda")
+        R = torch.empty(n, device="cuda")
+        # traditional baseline: kernel, then a device copy (no library)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        it = 20
+        e0.record(st)
+        for _ in range(it):
+            apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st)
+            with torch.cuda.stream(st):
+                R.copy_(Cb)
+        e1.record(st)
+        torch.cuda.synchronize()
+        print(json.dumps({"bytes": S, "mode": "kernel+copy (traditional, same GPU)",
+                          "us": e0.elapsed_time(e1) / it * 1e3,
+                          "gbs": S / (e0.elapsed_time(e1) / it / 1e3) / 1e9}), flush=True)
+        for gran in (apps.GRAN_BLOCK, apps.GRAN_WARP, apps.GRAN_THREAD):
+            cnt = elems[gran]
+            parts = n // cnt
+            for agg_name, agg in (("none", 1), ("block", max(1, 2048 // cnt)), ("1MiB", max(1, (1 << 18) // cnt)),
+                                  ("all", parts)):
+                agg = min(agg, parts)
+                for copy in (pc.COPY_INLINE, pc.COPY_ENGINE):
+                    if gran == apps.GRAN_THREAD and agg == 1 and S > (16 << 20):
+                        continue  # 33 M flags: covered up to 16 MiB
+                    snd = pc.psend_init(Cb, parts, cnt, pc.FLOAT32, 1, 5, cs[0])
+                    rcv = pc.precv_init(R, parts, cnt, pc.FLOAT32, 0, 5, cs[1])
+
+                    def epoch(first=False):
+                        snd.start(st)
+                        rcv.start(st)
+                        if first:
+                            pc.run_ranks([lambda: snd.pbuf_prepare(st), lambda: rcv.pbuf_prepare(st)])
+                        else:
+                            rcv.pbuf_prepare(st)
+                            snd.pbuf_prepare(st)
+                        apps.vecadd(A, B, Cb, n, gran, sq[0], st)
+                        snd.wait_on_stream(st)
+                        rcv.wait_on_stream(st)
+
+                    snd.start(st)
+                    rcv.start(st)
+                    pc.run_ranks([lambda: snd.pbuf_prepare(st), lambda: rcv.pbuf_prepare(st)])
+                    sq = [snd.prequest_create(gran, agg, copy)]
+                    apps.vecadd(A, B, Cb, n, gran, sq[0], st)
+                    snd.wait_on_stream(st)
+                    rcv.wait_on_stream(st)
+                    torch.cuda.synchronize()
+                    e0.record(st)
+                    for _ in range(it):
+                        epoch()
+                    e1.record(st)
+                    torch.cuda.synchronize()
+                    us = e0.elapsed_time(e1) / it * 1e3
+                    errs = [q.error() for q in (snd, rcv) if q.error()[0] != 0]
+                    ok = torch.equal(R, Cb)
+                    print(json.dumps({"bytes": S, "gran": ["thread", "warp", "block"][gran], "agg": agg_name,
+                                      "g": agg, "copy": ["inline", "engine"][copy], "us": us,
+                                      "goodput_gbs": S / (us / 1e6) / 1e9, "ok": ok, "errors": errs}), flush=True)
+                    snd.free()
+                    rcv.free()
+    for c in cs:
+        c.destroy()
+    g2.destroy()
+
+
+if __name__ == "__main__":
+    ap = argparse.ArgumentParser()
+    ap.add_argument("what", choices=["allreduce", "dl", "p2p"])
+    ap.add_argument("--ranks", default="8")
+    ap.add_argument("--algos", default="ring,rd")
+    ap.add_argument("--partitions", default="1,16,64")
+    ap.add_argument("--max-bytes", type=int, default=1 << 30)
+    a = ap.parse_args()
+    {"allreduce": sweep_allreduce, "dl": sweep_dl, "p2p": sweep_p2p}[a.what](a)
