@@ -171,6 +171,15 @@ PC_DEVICE bool spin_geq(const uint32_t *p, uint32_t target, int32_t *err, uint32
  * aligned, 4 independent vectors in flight per participant; 4-byte and
  * 1-byte fallbacks otherwise.  dst may be a peer-mapped (NVLink) address. */
 PC_DEVICE void copy_bytes(uint8_t *dst, const uint8_t *src, uint64_t nbytes, uint32_t idx, uint32_t n) {
+  const uintptr_t mis = reinterpret_cast<uintptr_t>(dst) & 15;
+  if (mis && (reinterpret_cast<uintptr_t>(src) & 15) == mis && nbytes > 16 - mis) {
+    // shared misalignment: bytes up to the 16-B boundary, then vectors
+    const uint64_t h = 16 - mis;
+    for (uint64_t b = idx; b < h; b += n) dst[b] = src[b];
+    dst += h;
+    src += h;
+    nbytes -= h;
+  }
   if (((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src)) & 15) == 0) {
     const uint64_t nv = nbytes >> 4;
     const uint4 *s = reinterpret_cast<const uint4 *>(src);

@@ -114,46 +114,60 @@ __device__ __forceinline__ uint4 vop(uint4 a, uint4 b) {
 }
 
 // out1[k] (and out2[k]) = local[k] ⊕ incoming[k], k < n elements, by one warp.
+// All operands of one call sit at the same element offset of 16-B aligned
+// buffers, so they share one misalignment: a scalar head of < 4 elements
+// brings them to a 16-B boundary, the body runs on 16-B vectors (kU in flight
+// per operand per lane), a scalar tail finishes.  (Gradient buffers of
+// arbitrary tensor sizes, C3, make unaligned partitions the common case.)
 template <int DT, int OP>
 __device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *local, const void *incoming,
                                             int64_t n) {
   using O = Op<DT, OP>;
   using T = typename O::T;
   const uint32_t lane = threadIdx.x & 31;
-  const uintptr_t al = reinterpret_cast<uintptr_t>(out1) | reinterpret_cast<uintptr_t>(out2) |
-                       reinterpret_cast<uintptr_t>(local) | reinterpret_cast<uintptr_t>(incoming);
-  int64_t done = 0;
-  if ((al & 15) == 0) {
-    const int64_t nv = n >> 2;
-    const uint4 *a = reinterpret_cast<const uint4 *>(local);
-    const uint4 *b = reinterpret_cast<const uint4 *>(incoming);
-    uint4 *o1 = reinterpret_cast<uint4 *>(out1);
-    uint4 *o2 = reinterpret_cast<uint4 *>(out2);
-    int64_t k = lane;
-    for (; k + 32 * (kU - 1) < nv; k += 32 * kU) {
-      uint4 x[kU], y[kU];
-#pragma unroll
-      for (int j = 0; j < kU; ++j) x[j] = __ldcg(a + k + 32 * j);
-#pragma unroll
-      for (int j = 0; j < kU; ++j) y[j] = __ldcg(b + k + 32 * j);
-#pragma unroll
-      for (int j = 0; j < kU; ++j) {
-        const uint4 r = vop<DT, OP>(x[j], y[j]);
-        o1[k + 32 * j] = r;
-        if (out2) o2[k + 32 * j] = r;
-      }
-    }
-    for (; k < nv; k += 32) {
-      uint4 r0 = vop<DT, OP>(__ldcg(a + k), __ldcg(b + k));
-      o1[k] = r0;
-      if (out2) o2[k] = r0;
-    }
-    done = nv << 2;
-  }
   const T *a = reinterpret_cast<const T *>(local);
   const T *b = reinterpret_cast<const T *>(incoming);
   T *o1 = reinterpret_cast<T *>(out1);
   T *o2 = reinterpret_cast<T *>(out2);
+  const uintptr_t m = reinterpret_cast<uintptr_t>(out1) & 15;
+  const bool same = ((reinterpret_cast<uintptr_t>(local) & 15) == m) &&
+                    ((reinterpret_cast<uintptr_t>(incoming) & 15) == m) &&
+                    (!out2 || (reinterpret_cast<uintptr_t>(out2) & 15) == m) && (m & 3) == 0;
+  int64_t head = same ? (int64_t)(((16 - m) & 15) >> 2) : n;
+  if (head > n) head = n;
+  for (int64_t k = lane; k < head; k += 32) {
+    const T r = O::f(__ldcg(a + k), __ldcg(b + k));
+    o1[k] = r;
+    if (o2) o2[k] = r;
+  }
+  int64_t done = head;
+  if (same && n > head) {
+    const int64_t nv = (n - head) >> 2;
+    const uint4 *av = reinterpret_cast<const uint4 *>(a + head);
+    const uint4 *bv = reinterpret_cast<const uint4 *>(b + head);
+    uint4 *o1v = reinterpret_cast<uint4 *>(o1 + head);
+    uint4 *o2v = o2 ? reinterpret_cast<uint4 *>(o2 + head) : nullptr;
+    int64_t k = lane;
+    for (; k + 32 * (kU - 1) < nv; k += 32 * kU) {
+      uint4 x[kU], y[kU];
+#pragma unroll
+      for (int j = 0; j < kU; ++j) x[j] = __ldcg(av + k + 32 * j);
+#pragma unroll
+      for (int j = 0; j < kU; ++j) y[j] = __ldcg(bv + k + 32 * j);
+#pragma unroll
+      for (int j = 0; j < kU; ++j) {
+        const uint4 r = vop<DT, OP>(x[j], y[j]);
+        o1v[k + 32 * j] = r;
+        if (o2v) o2v[k + 32 * j] = r;
+      }
+    }
+    for (; k < nv; k += 32) {
+      const uint4 r = vop<DT, OP>(__ldcg(av + k), __ldcg(bv + k));
+      o1v[k] = r;
+      if (o2v) o2v[k] = r;
+    }
+    done = head + (nv << 2);
+  }
   for (int64_t k = done + lane; k < n; k += 32) {
     const T r = O::f(__ldcg(a + k), __ldcg(b + k));
     o1[k] = r;
@@ -163,6 +177,15 @@ __device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *
 
 __device__ __forceinline__ void warp_copy(void *dst, const void *src, int64_t nbytes) {
   const uint32_t lane = threadIdx.x & 31;
+  const uintptr_t m = reinterpret_cast<uintptr_t>(dst) & 15;
+  if (m && (reinterpret_cast<uintptr_t>(src) & 15) == m && nbytes > (int64_t)(16 - m)) {
+    // shared misalignment: copy a head up to the 16-B boundary, then vectors
+    const int64_t h = (int64_t)(16 - m);
+    copy_bytes(reinterpret_cast<uint8_t *>(dst), reinterpret_cast<const uint8_t *>(src), (uint64_t)h, lane, 32);
+    dst = reinterpret_cast<uint8_t *>(dst) + h;
+    src = reinterpret_cast<const uint8_t *>(src) + h;
+    nbytes -= h;
+  }
   if (((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src)) & 15) == 0) {
     const int64_t nv = nbytes >> 4;
     const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
