@@ -243,10 +243,23 @@ static void choose_slices(int64_t len, int nparts, int target_units, int64_t min
   if (fixed > 0) {
     qs = std::max<int64_t>(4, (fixed / 4 + 3) / 4 * 4);
   } else {
-    int64_t by_size = std::max<int64_t>(1, (len + min_elems - 1) / std::max<int64_t>(min_elems, 1));
-    int64_t by_units = std::max<int64_t>(1, target_units / std::max(nparts, 1));
-    int64_t ns = std::min(by_size, by_units);
-    qs = (len + ns - 1) / ns;
+    // Balance: with W = target_units warps taking units in turn, the engine
+    // time is ~ ceil(nparts*ns / W) slices of len/ns elements each; pick the
+    // ns (not below min_elems per slice) that minimises ceil(nparts*ns/W)/ns,
+    // preferring fewer, larger slices within 3%.
+    const int64_t by_size = std::max<int64_t>(1, (len + min_elems - 1) / std::max<int64_t>(min_elems, 1));
+    const int64_t W = std::max(target_units, 1), np = std::max(nparts, 1);
+    const int64_t max_ns = std::min<int64_t>(by_size, std::max<int64_t>(1, (4 * W + np - 1) / np));
+    int64_t best = 1;
+    double best_cost = 1e300;
+    for (int64_t ns = 1; ns <= max_ns; ++ns) {
+      const double cost = (double)((np * ns + W - 1) / W) / (double)ns;
+      if (cost < best_cost * 0.97) {
+        best_cost = cost;
+        best = ns;
+      }
+    }
+    qs = (len + best - 1) / best;
     qs = std::max<int64_t>(4, (qs + 3) / 4 * 4);
   }
   int64_t ns = len > 0 ? (len + qs - 1) / qs : 1;
