@@ -26,6 +26,7 @@
 namespace {
 
 constexpr int kStrip = 128;  // columns per warp tile (32 lanes x float4)
+constexpr int kRB = 4;       // rows loaded together per batch (tile height H % kRB == 0)
 enum { T = 0, B = 1, L = 2, R = 3 };
 
 struct JacobiRank {
@@ -74,33 +75,51 @@ __device__ void tile_iter(const JacobiRank &d, int tile, int k) {
   else up = cur;  // global boundary row: not used
   const int gx = d.gx0 + x0;
   const bool colfix0 = gx == 0, colfix3 = gx + 3 == d.N - 1;
-  for (int r = r0; r < r0 + d.H; ++r) {
-    float4 dn;
-    if (r + 1 < ly) dn = ld4(a + (size_t)(r + 1) * lx + x0);
-    else if (d.has[B]) dn = ld4(hB + x0);
-    else dn = cur;
-    float lf = __shfl_up_sync(0xffffffffu, cur.w, 1);
-    float rt = __shfl_down_sync(0xffffffffu, cur.x, 1);
-    if (lane == 0) lf = x0 > 0 ? __ldcg(a + (size_t)r * lx + x0 - 1) : (d.has[L] ? __ldcg(hL + r) : cur.x);
-    if (lane == 31) rt = x0 + 4 < lx ? __ldcg(a + (size_t)r * lx + x0 + 4) : (d.has[R] ? __ldcg(hR + r) : cur.w);
-    const int gy = d.gy0 + r;
-    float4 o;
-    if (gy == 0 || gy == d.N - 1) {
-      o = cur;  // Dirichlet row
-    } else {
-      o.x = colfix0 ? cur.x : stencil(up.x, dn.x, lf, cur.y);
-      o.y = stencil(up.y, dn.y, cur.x, cur.z);
-      o.z = stencil(up.z, dn.z, cur.y, cur.w);
-      o.w = colfix3 ? cur.w : stencil(up.w, dn.w, cur.z, rt);
+  // Rows in batches of kRB: the kRB next rows (and the lane-0 / lane-31 edge
+  // scalars) are loaded together so each warp keeps kRB 512-B loads in flight.
+  for (int r = r0; r < r0 + d.H; r += kRB) {
+    float4 nx[kRB];
+    float le[kRB], re[kRB];
+#pragma unroll
+    for (int j = 0; j < kRB; ++j) {
+      const int rr = r + 1 + j;
+      nx[j] = rr < ly ? ld4(a + (size_t)rr * lx + x0) : (d.has[B] ? ld4(hB + x0) : cur);
     }
-    *reinterpret_cast<float4 *>(b + (size_t)r * lx + x0) = o;
-    // edge staging for the neighbours (slot k+1)
-    if (r == 0 && d.has[T]) *reinterpret_cast<float4 *>(d.sendbuf[T] + (size_t)(k + 1) * lx + x0) = o;
-    if (r == ly - 1 && d.has[B]) *reinterpret_cast<float4 *>(d.sendbuf[B] + (size_t)(k + 1) * lx + x0) = o;
-    if (left && lane == 0) d.sendbuf[L][(size_t)(k + 1) * ly + r] = o.x;
-    if (right && lane == 31) d.sendbuf[R][(size_t)(k + 1) * ly + r] = o.w;
-    up = cur;
-    cur = dn;
+#pragma unroll
+    for (int j = 0; j < kRB; ++j) {
+      const int rr = r + j;
+      le[j] = 0.f;
+      re[j] = 0.f;
+      if (lane == 0) le[j] = x0 > 0 ? __ldcg(a + (size_t)rr * lx + x0 - 1) : (d.has[L] ? __ldcg(hL + rr) : 0.f);
+      if (lane == 31) re[j] = x0 + 4 < lx ? __ldcg(a + (size_t)rr * lx + x0 + 4) : (d.has[R] ? __ldcg(hR + rr) : 0.f);
+    }
+#pragma unroll
+    for (int j = 0; j < kRB; ++j) {
+      const int rr = r + j;
+      const float4 dn = nx[j];
+      float lf = __shfl_up_sync(0xffffffffu, cur.w, 1);
+      float rt = __shfl_down_sync(0xffffffffu, cur.x, 1);
+      if (lane == 0) lf = le[j];
+      if (lane == 31) rt = re[j];
+      const int gy = d.gy0 + rr;
+      float4 o;
+      if (gy == 0 || gy == d.N - 1) {
+        o = cur;  // Dirichlet row
+      } else {
+        o.x = colfix0 ? cur.x : stencil(up.x, dn.x, lf, cur.y);
+        o.y = stencil(up.y, dn.y, cur.x, cur.z);
+        o.z = stencil(up.z, dn.z, cur.y, cur.w);
+        o.w = colfix3 ? cur.w : stencil(up.w, dn.w, cur.z, rt);
+      }
+      *reinterpret_cast<float4 *>(b + (size_t)rr * lx + x0) = o;
+      // edge staging for the neighbours (slot k+1)
+      if (rr == 0 && d.has[T]) *reinterpret_cast<float4 *>(d.sendbuf[T] + (size_t)(k + 1) * lx + x0) = o;
+      if (rr == ly - 1 && d.has[B]) *reinterpret_cast<float4 *>(d.sendbuf[B] + (size_t)(k + 1) * lx + x0) = o;
+      if (left && lane == 0) d.sendbuf[L][(size_t)(k + 1) * ly + rr] = o.x;
+      if (right && lane == 31) d.sendbuf[R][(size_t)(k + 1) * ly + rr] = o.w;
+      up = cur;
+      cur = dn;
+    }
   }
   // Pready: push my edge segments of slot k+1 (INLINE copy by this warp)
   if (top) pc_pready_warp((k + 1) * d.nsegR + sx, d.sq[T]);
@@ -165,7 +184,7 @@ int pcapp_jacobi_launch(const void *ranks, const int *block_start, int nranks, i
 int pcapp_jacobi_describe(void *out, float *grid0, float *grid1, int ly, int lx, int H, int gy0, int gx0, int N,
                           const int *has, float *const *sendbuf, const float *const *halo,
                           const pc_prequest_t *const *sq, const pc_prequest_t *const *rq) {
-  if (lx % kStrip || ly % H || H < 1) return -1;
+  if (lx % kStrip || ly % H || H < kRB || H % kRB) return -1;
   JacobiRank d{};
   d.grid[0] = grid0;
   d.grid[1] = grid1;
