@@ -249,7 +249,7 @@ def jacobi_bench(pc, apps, torch, args):
         e1.record(st)
         torch.cuda.synchronize()
         errs = js.errors()
-        ms_iter = e0.elapsed_time(e1) / (reps * (K + 1))  # K iterations + the init push
+        ms_iter = e0.elapsed_time(e1) / (reps * K)  # per iteration, the per-epoch init push included
         cells = (N - 2) * (N - 2)
         res[f"{Py}x{Px}"] = {"gflops": 4.0 * cells / (ms_iter / 1e3) / 1e9, "us_per_iter": ms_iter * 1e3,
                              "hbm_frac": (8.0 * N * N / (ms_iter / 1e3) / 1e9) / hbm_peak,

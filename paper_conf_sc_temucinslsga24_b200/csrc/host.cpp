@@ -538,7 +538,7 @@ static int exchange_round(Comm *c, Request *target) {
 static RingArgs make_ring_args(Request *q) {
   Comm *c = q->comm;
   RingArgs a{};
-  a.e = q->epoch;
+  a.epoch = q->ctrl + q->L.epoch;
   a.P = c->size;
   a.r = c->rank;
   a.Np = q->partitions;
@@ -568,7 +568,7 @@ static RingArgs make_ring_args(Request *q) {
 static RdArgs make_rd_args(Request *q) {
   Comm *c = q->comm;
   RdArgs a{};
-  a.e = q->epoch;
+  a.epoch = q->ctrl + q->L.epoch;
   a.P = c->size;
   a.r = c->rank;
   a.Np = q->partitions;
@@ -631,7 +631,7 @@ static int launch_single(Request *q) {
                                  : launch_rd_engine(make_rd_args(q), q->engine_warps, q->side);
   } else {
     P2pEngineArgs a{};
-    a.e = q->epoch;
+    a.epoch = q->ctrl + q->L.epoch;
     a.nt = q->ntransport;
     a.agg = q->agg;
     a.ns = q->slices;
@@ -977,7 +977,9 @@ int pc_start(pc_request_t req, pc_stream_t stream) {
   q->user_stream = (cudaStream_t)stream;
   if (c->dry) return 0;
   PC_CUDA(cudaSetDevice(c->device));
-  return stream_write_u32(c, (cudaStream_t)stream, q->ctrl + q->L.epoch, q->epoch);
+  // the device epoch word is advanced on the device (not written from a host
+  // value), so a CUDA graph that captured Start...Wait replays new epochs
+  return launch_epoch_bump(q->ctrl + q->L.epoch, (cudaStream_t)stream);
 }
 
 int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
@@ -994,8 +996,15 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
   if (c->dry) return 0;
   q->user_stream = (cudaStream_t)stream;
   if (!q->prepared_this_epoch) {
-    for (auto &t : q->rtr_targets) {
-      int rc = stream_write_u32(c, (cudaStream_t)stream, t.first + q->L.rtr + t.second, q->epoch);
+    if (!q->rtr_targets.empty()) {
+      RtrArgs a{};
+      a.epoch = q->ctrl + q->L.epoch;
+      a.sys = q->sys_scope;
+      for (auto &t : q->rtr_targets) {
+        if (a.n == kMaxRdSteps + 2) return PC_ERR_UNSUPPORTED;
+        a.dst[a.n++] = t.first + q->L.rtr + t.second;
+      }
+      int rc = launch_rtr(a, (cudaStream_t)stream);
       if (rc) return rc;
     }
     q->prepared_this_epoch = true;
@@ -1098,11 +1107,11 @@ static int wait_common(Request *q, cudaStream_t s, bool host) {
     }
     if (q->kind == PC_KIND_PSEND) {
       if (!q->has_preq) return PC_ERR_STATE;
-      rc = launch_wait_words(q->ctrl + q->L.sent, q->ntransport, q->epoch, nullptr, q->partitions, err, c->timeout_ms,
-                             ws, false);
+      rc = launch_wait_words(q->ctrl + q->L.sent, q->ntransport, q->ctrl + q->L.epoch, 1, nullptr, q->partitions, err,
+                             c->timeout_ms, ws, false);
     } else {
-      rc = launch_wait_words(q->ctrl + q->L.flags, 0, q->epoch, q->ctrl + q->L.layout, q->partitions, err,
-                             c->timeout_ms, ws, true);
+      rc = launch_wait_words(q->ctrl + q->L.flags, 0, q->ctrl + q->L.epoch, 1, q->ctrl + q->L.layout, q->partitions,
+                             err, c->timeout_ms, ws, q->sys_scope != 0);
     }
     if (rc) return rc;
     if (host) PC_CUDA(cudaStreamSynchronize(q->side));
@@ -1132,26 +1141,39 @@ static int read_words(Request *q, size_t off, size_t n, uint32_t *h) {
 
 static bool reached_h(uint32_t v, uint32_t t) { return (int32_t)(v - t) >= 0; }
 
+// The epoch a host-side query compares against: the later of the host's count
+// of pc_start calls and the device epoch word (which CUDA-graph replays of a
+// captured Start advance without the host seeing it).
+static int current_epoch(Request *q, uint32_t *e) {
+  uint32_t d = 0;
+  int rc = read_words(q, q->L.epoch, 1, &d);
+  if (rc) return rc;
+  if (reached_h(d, q->epoch)) q->epoch = d;
+  *e = q->epoch;
+  return 0;
+}
+
 int pc_parrived(pc_request_t req, int partition, int *flag) {
   Request *q = (Request *)req;
   if (!q || !flag || partition < 0 || partition >= q->partitions) return PC_ERR_ARG;
   *flag = 0;
   if (q->comm->dry) return 0;
   PC_CUDA(cudaSetDevice(q->comm->device));
-  uint32_t v = 0;
+  uint32_t v = 0, e = 0;
   int rc;
+  if ((rc = current_epoch(q, &e))) return rc;
   if (q->kind == PC_KIND_PALLREDUCE) {
     if ((rc = read_words(q, q->L.donecnt + partition, 1, &v))) return rc;
-    *flag = reached_h(v, q->epoch * (uint32_t)q->slices);
+    *flag = reached_h(v, e * (uint32_t)q->slices);
   } else if (q->kind == PC_KIND_PRECV) {
     uint32_t g = 0;
     if ((rc = read_words(q, q->L.layout, 1, &g))) return rc;
     if (g == 0) return 0;
     if ((rc = read_words(q, q->L.flags + partition / g, 1, &v))) return rc;
-    *flag = reached_h(v, q->epoch);
+    *flag = reached_h(v, e);
   } else {
     if ((rc = read_words(q, q->L.sent + partition / q->agg, 1, &v))) return rc;
-    *flag = reached_h(v, q->epoch);
+    *flag = reached_h(v, e);
   }
   return 0;
 }
@@ -1198,9 +1220,11 @@ int pc_test(pc_request_t req, int *flag) {
     }
     done = n >= 0;
     if (n > 0) {
+      uint32_t e = 0;
+      if ((rc = current_epoch(q, &e))) return rc;
       std::vector<uint32_t> h((size_t)n);
       if ((rc = read_words(q, off, (size_t)n, h.data()))) return rc;
-      for (uint32_t v : h) done = done && reached_h(v, q->epoch);
+      for (uint32_t v : h) done = done && reached_h(v, e);
     }
   }
   int erc = error_rc(q);

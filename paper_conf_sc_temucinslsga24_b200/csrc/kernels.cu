@@ -257,7 +257,7 @@ struct Idle {
 };
 
 template <int DT, int OP>
-__device__ __forceinline__ void ring_step(const RingArgs &a, int u, int s, int i) {
+__device__ __forceinline__ void ring_step(const RingArgs &a, int u, int s, int i, uint32_t e) {
   const int P = a.P, r = a.r, NS = 2 * (P - 1);
   const int64_t es = 4;
   const int64_t base = (int64_t)u * a.L;
@@ -277,13 +277,13 @@ __device__ __forceinline__ void ring_step(const RingArgs &a, int u, int s, int i
     else
       warp_copy(a.o_recvbuf + off, a.recvbuf + off, n * es);
   }
-  warp_signal(a.o_flags + fbase + (int64_t)i * a.ns, a.e, a.sys);
+  warp_signal(a.o_flags + fbase + (int64_t)i * a.ns, e, a.sys);
 }
 
 template <int DT, int OP>
 __device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const int W) {
   const int P = a.P, NS = 2 * (P - 1);
-  const uint32_t e = a.e;
+  const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
   const int64_t es = 4;
   if (gw >= a.nunits) return;
   if (P == 1) {
@@ -322,7 +322,7 @@ __device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const
         if (!warp_poll(dep, e, i != 0 && a.sys)) continue;
         progressed = true;
         if (i < NS) {
-          ring_step<DT, OP>(a, u, s, i);
+          ring_step<DT, OP>(a, u, s, i, e);
           step[j] = i + 1;
         } else {  // arrival of the last AG step: partition slice final here
           if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
@@ -346,7 +346,7 @@ __device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const
 template <int DT, int OP>
 __device__ __forceinline__ void rd_body(const RdArgs &a, const int gw, const int W) {
   const int NS = a.nsteps;
-  const uint32_t e = a.e;
+  const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
   const int64_t es = 4;
   const int64_t stride = (int64_t)a.Np * a.L * es;  // bytes per staging slot
   uint32_t rtr_ok = 0;
@@ -428,7 +428,7 @@ __global__ void __launch_bounds__(kEngineBlock) rd_engine_group(RdGroupArgs g) {
 __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int W = (gridDim.x * blockDim.x) >> 5;
-  const uint32_t e = a.e;
+  const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
   bool rtr_ok = false;
   for (int x = gw; x < a.nunits; x += W) {
     const int t = x / a.ns, s = x % a.ns;
@@ -455,9 +455,10 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
   }
 }
 
-__global__ void wait_words_kernel(const uint32_t *words, int n, uint32_t target, const uint32_t *layout,
-                                  int partitions, int32_t *err, uint32_t tmo, int sys) {
+__global__ void wait_words_kernel(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul,
+                                  const uint32_t *layout, int partitions, int32_t *err, uint32_t tmo, int sys) {
   __shared__ int s_n;
+  const uint32_t target = *(const volatile uint32_t *)epoch * mul;
   if (threadIdx.x == 0) {
     int nn = n;
     if (layout) {
@@ -485,6 +486,23 @@ __global__ void wait_words_kernel(const uint32_t *words, int n, uint32_t target,
 }
 
 __global__ void set_word_kernel(uint32_t *addr, uint32_t v) { st_release_sys(addr, v); }
+
+// pc_start: the epoch lives on the device and is advanced in stream order, so
+// a captured CUDA graph replays correct epochs (the host never writes it).
+__global__ void epoch_bump_kernel(uint32_t *epoch) { *epoch = *epoch + 1; }
+
+// pc_pbuf_prepare: ready-to-receive = this rank's current epoch, written into
+// every producer's RTR slot (remote stores; release so that everything this
+// rank did to the buffers before is ordered first).
+__global__ void rtr_kernel(RtrArgs a) {
+  const uint32_t e = *(const volatile uint32_t *)a.epoch;
+  for (int i = 0; i < a.n; ++i) {
+    if (a.sys)
+      st_release_sys(a.dst[i], e);
+    else
+      st_release_gpu(a.dst[i], e);
+  }
+}
 
 __global__ void pready_range_kernel(pc_prequest_t q, int lo, int hi) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -569,9 +587,23 @@ int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
   return 0;
 }
 
-int launch_wait_words(const uint32_t *words, int n, uint32_t target, const uint32_t *layout, int partitions,
-                      int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys) {
-  wait_words_kernel<<<1, 256, 0, s>>>(words, n, target, layout, partitions, err, timeout_ms, sys ? 1 : 0);
+int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul, const uint32_t *layout,
+                      int partitions, int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys) {
+  wait_words_kernel<<<1, 256, 0, s>>>(words, n, epoch, mul, layout, partitions, err, timeout_ms, sys ? 1 : 0);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_epoch_bump(uint32_t *epoch, cudaStream_t s) {
+  epoch_bump_kernel<<<1, 1, 0, s>>>(epoch);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_rtr(const RtrArgs &a, cudaStream_t s) {
+  rtr_kernel<<<1, 1, 0, s>>>(a);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;

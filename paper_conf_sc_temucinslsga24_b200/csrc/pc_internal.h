@@ -214,7 +214,7 @@ bool memops_available();
 
 // ------------------------------------------------------------------ kernel launchers (kernels.cu)
 struct RingArgs {
-  uint32_t e;
+  const uint32_t *epoch;  // device epoch word (read at kernel start)
   int P, r, Np, ns, nunits, op, dtype;
   int64_t L, q, qs;
   const uint8_t *sendbuf;
@@ -229,7 +229,7 @@ struct RingArgs {
   int sys;  // 1: some peer is another GPU -> system-scope fences/acquires
 };
 struct RdArgs {
-  uint32_t e;
+  const uint32_t *epoch;
   int P, r, Np, ns, nunits, op, dtype, nsteps;
   int64_t L, qs;
   const uint8_t *sendbuf;
@@ -244,7 +244,7 @@ struct RdArgs {
   int sys;
 };
 struct P2pEngineArgs {
-  uint32_t e;
+  const uint32_t *epoch;
   int nt, agg, ns, nunits;
   uint64_t part_bytes, slice_bytes;
   int partitions;
@@ -276,7 +276,15 @@ int launch_rd_engine(const RdArgs &a, int warps, cudaStream_t s);
 int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s);
 // wait until words[i*stride] reached target (i < n); layout!=null: n derived
 // as ceil(partitions / *layout) (receiver side)
-int launch_wait_words(const uint32_t *words, int n, uint32_t target, const uint32_t *layout, int partitions,
+struct RtrArgs {
+  const uint32_t *epoch;
+  int n, sys;
+  uint32_t *dst[kMaxRdSteps + 2];
+};
+int launch_epoch_bump(uint32_t *epoch, cudaStream_t s);
+int launch_rtr(const RtrArgs &a, cudaStream_t s);
+int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul, const uint32_t *layout,
+                      int partitions,
                       int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys);
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s);
 int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s);

@@ -187,3 +187,49 @@ def test_integer_valued_fp32_exact():
         ref = x.astype(np.int64).sum(0).astype(np.float32)
         for r in range(P):
             np.testing.assert_array_equal(y[r], ref)
+
+
+def test_cuda_graph_replay_of_epochs():
+    """Start -> Pbuf_prepare -> Pready -> Wait of every rank captured once into
+    a CUDA graph and replayed: the epoch lives on the device (pc_start bumps it
+    there), so each replay is a new, correct epoch."""
+    P, Np, L = 4, 3, 5000
+    with comms(P) as cs:
+        st = torch.cuda.Stream()
+        send = [torch.zeros(Np * L, device="cuda") for _ in range(P)]
+        recv = [torch.zeros(Np * L, device="cuda") for _ in range(P)]
+        reqs = [pc.pallreduce_init(send[r], recv[r], Np, L, pc.FLOAT32, pc.SUM, pc.ALGO_RING, cs[r]) for r in range(P)]
+
+        def step(first=False):
+            for q in reqs:
+                q.start(st)
+            if first:
+                first_prepare([[q] for q in reqs], [st] * P)
+            else:
+                for q in reqs:
+                    q.pbuf_prepare(st)
+            for q in reqs:
+                q.pready_range(0, Np - 1, st)
+            for q in reqs:
+                q.wait_on_stream(st)
+
+        step(first=True)  # eager first epoch: exchange, mapping
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            step()
+        for e in range(6):
+            x = np.stack([synth.normal_f32(SEED + 20, r, e, Np * L) for r in range(P)])
+            for r in range(P):
+                send[r].copy_(torch.from_numpy(x[r]))
+            torch.cuda.synchronize()
+            g.replay()
+            torch.cuda.synchronize()
+            ref = oracle.ring_fold_f32(x, oracle.chunk_ids(L, P, Np))
+            for r in range(P):
+                np.testing.assert_array_equal(recv[r].cpu().numpy().view(np.uint32), ref.view(np.uint32))
+        # 1 eager + 1 captured (not executed at capture) + 6 replays
+        assert int(reqs[0].words("epoch", 0, 1)[0]) == 7
+        for q in reqs:
+            assert q.error() == (0, 0)
+            q.free()
