@@ -27,7 +27,7 @@ def busbw(S, sec, P):
     return S / sec * 2.0 * (P - 1) / P / 1e9 if P > 1 else S / sec / 1e9
 
 
-def time_allreduce(cs, S, Np, algo, min_ms=30.0):
+def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
     P = len(cs)
     count = max(S // 4 // Np, 1)
     n = count * Np
@@ -51,9 +51,15 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0):
 
     step(True)
     torch.cuda.synchronize()
+    run = step
+    if graph:  # capture one epoch of every rank; each replay is a new epoch
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            step()
+        run = g.replay
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(st)
-    step()
+    run()
     e1.record(st)
     torch.cuda.synchronize()
     one = max(e0.elapsed_time(e1), 1e-3)
@@ -62,7 +68,7 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0):
     for _ in range(3):
         e0.record(st)
         for _ in range(iters):
-            step()
+            run()
         e1.record(st)
         torch.cuda.synchronize()
         blocks.append(e0.elapsed_time(e1) / iters)
@@ -73,7 +79,7 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0):
     ms = statistics.median(blocks)
     return {"bytes_per_rank": n * 4, "partitions": Np, "ranks": P, "algo": ["auto", "ring", "rd"][algo],
             "us_per_step": ms * 1e3, "busbw_gbs": busbw(n * 4, ms / 1e3, P), "slices": info["slices"],
-            "errors": errs}
+            "graph": graph, "errors": errs}
 
 
 def sweep_allreduce(args):
@@ -88,7 +94,7 @@ def sweep_allreduce(args):
                 for Np in [int(x) for x in args.partitions.split(",")]:
                     if S // 4 // Np < P:
                         continue
-                    r = time_allreduce(cs, S, Np, a)
+                    r = time_allreduce(cs, S, Np, a, graph=args.graph)
                     print(json.dumps(r), flush=True)
                 S <<= 2
         for c in cs:
@@ -194,5 +200,6 @@ if __name__ == "__main__":
     ap.add_argument("--algos", default="ring,rd")
     ap.add_argument("--partitions", default="1,16,64")
     ap.add_argument("--max-bytes", type=int, default=1 << 30)
+    ap.add_argument("--graph", action="store_true", help="replay a captured CUDA graph of the epoch")
     a = ap.parse_args()
     {"allreduce": sweep_allreduce, "dl": sweep_dl, "p2p": sweep_p2p}[a.what](a)
