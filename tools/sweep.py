@@ -56,7 +56,10 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=st):
             step()
-        run = g.replay
+
+        def run():
+            with torch.cuda.stream(st):  # replay on the timed stream
+                g.replay()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(st)
     run()
