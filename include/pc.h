@@ -122,6 +122,13 @@ int pc_start(pc_request_t req, pc_stream_t stream);
  * epoch write into each producer's RTR word (no host blocking); producers
  * check it on the device before their first push of the epoch. */
 int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream);
+/* MPI_Startall analogue: pc_start for n requests of one GPU, with a single
+ * device kernel advancing all n epochs (CUDA-graph capturable). */
+int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream);
+/* pc_pbuf_prepare for n requests whose first pc_pbuf_prepare (exchange +
+ * mapping) already happened: all ready-to-receive writes in one kernel.
+ * PC_ERR_STATE if a request is inactive or not yet exchanged. */
+int pc_pbuf_prepare_all(int n, pc_request_t *reqs, pc_stream_t stream);
 /* MPIX_Prequest_create: build the POD device request.  `aggregation`
  * = g user partitions per transport partition (P:L129 threshold; 1 = none);
  * allreduce requires g = 1.  Blocking.  Writes the transport layout into the

@@ -43,6 +43,8 @@ _PC_PROTOS = {
     "pc_precv_init": (I32, [P, I32, SZ, I32, I32, I32, P, C.POINTER(P)]),
     "pc_pallreduce_init": (I32, [P, P, I32, SZ, I32, I32, I32, P, C.POINTER(P)]),
     "pc_start": (I32, [P, P]),
+    "pc_startall": (I32, [I32, P, P]),
+    "pc_pbuf_prepare_all": (I32, [I32, P, P]),
     "pc_pbuf_prepare": (I32, [P, P]),
     "pc_prequest_create": (I32, [P, I32, I32, I32, P]),
     "pc_prequest_free": (I32, [P]),

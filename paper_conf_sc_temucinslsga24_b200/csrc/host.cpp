@@ -1012,6 +1012,79 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
   return 0;
 }
 
+// MPI_Startall: one device kernel advances the epochs of all n requests.
+int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream) {
+  if (n < 0 || (n > 0 && !reqs)) return PC_ERR_ARG;
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    if (!q) return PC_ERR_ARG;
+    if (q->active) return PC_ERR_STATE;
+    if (q->comm->device != ((Request *)reqs[0])->comm->device || q->comm->dry != ((Request *)reqs[0])->comm->dry)
+      return PC_ERR_ARG;
+  }
+  CtlArgs a{};
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    q->epoch++;
+    q->active = true;
+    q->engine_launched = false;
+    q->engine_registered = false;
+    q->prepared_this_epoch = false;
+    q->user_stream = (cudaStream_t)stream;
+    if (q->comm->dry) continue;
+    a.epoch[a.n] = q->ctrl + q->L.epoch;
+    a.dst[a.n] = nullptr;
+    if (++a.n == kMaxCtl) {
+      PC_CUDA(cudaSetDevice(q->comm->device));
+      int rc = launch_ctl(a, (cudaStream_t)stream);
+      if (rc) return rc;
+      a.n = 0;
+    }
+  }
+  if (a.n) {
+    PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
+    return launch_ctl(a, (cudaStream_t)stream);
+  }
+  return 0;
+}
+
+// Ready-to-receive for n already-exchanged requests in one kernel (the first
+// pc_pbuf_prepare of each request, which exchanges and maps, must be a
+// pc_pbuf_prepare call).
+int pc_pbuf_prepare_all(int n, pc_request_t *reqs, pc_stream_t stream) {
+  if (n < 0 || (n > 0 && !reqs)) return PC_ERR_ARG;
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    if (!q) return PC_ERR_ARG;
+    if (!q->active) return PC_ERR_STATE;
+    if (!q->exchanged) return PC_ERR_STATE;
+    if (!q->matched) return PC_ERR_MATCH;
+  }
+  CtlArgs a{};
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    q->user_stream = (cudaStream_t)stream;
+    if (q->comm->dry || q->prepared_this_epoch) continue;
+    for (auto &t : q->rtr_targets) {
+      a.epoch[a.n] = q->ctrl + q->L.epoch;
+      a.dst[a.n] = t.first + q->L.rtr + t.second;
+      a.sys[a.n] = q->sys_scope;
+      if (++a.n == kMaxCtl) {
+        PC_CUDA(cudaSetDevice(q->comm->device));
+        int rc = launch_ctl(a, (cudaStream_t)stream);
+        if (rc) return rc;
+        a.n = 0;
+      }
+    }
+    q->prepared_this_epoch = true;
+  }
+  if (a.n) {
+    PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
+    return launch_ctl(a, (cudaStream_t)stream);
+  }
+  return 0;
+}
+
 int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_copy_t copy, pc_prequest_t *out) {
   Request *q = (Request *)req;
   if (!q || !out || gran < 0 || gran > 2 || copy < 0 || copy > 1) return PC_ERR_ARG;

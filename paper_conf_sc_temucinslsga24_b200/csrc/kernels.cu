@@ -491,6 +491,21 @@ __global__ void set_word_kernel(uint32_t *addr, uint32_t v) { st_release_sys(add
 // a captured CUDA graph replays correct epochs (the host never writes it).
 __global__ void epoch_bump_kernel(uint32_t *epoch) { *epoch = *epoch + 1; }
 
+__global__ void ctl_kernel(CtlArgs a) {
+  const int i = threadIdx.x;
+  if (i >= a.n) return;
+  uint32_t *ep = const_cast<uint32_t *>(a.epoch[i]);
+  if (!a.dst[i]) {
+    *ep = *ep + 1;
+  } else {
+    const uint32_t e = *(const volatile uint32_t *)ep;
+    if (a.sys[i])
+      st_release_sys(a.dst[i], e);
+    else
+      st_release_gpu(a.dst[i], e);
+  }
+}
+
 // pc_pbuf_prepare: ready-to-receive = this rank's current epoch, written into
 // every producer's RTR slot (remote stores; release so that everything this
 // rank did to the buffers before is ordered first).
@@ -590,6 +605,14 @@ int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
 int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul, const uint32_t *layout,
                       int partitions, int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys) {
   wait_words_kernel<<<1, 256, 0, s>>>(words, n, epoch, mul, layout, partitions, err, timeout_ms, sys ? 1 : 0);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_ctl(const CtlArgs &a, cudaStream_t s) {
+  if (a.n <= 0) return 0;
+  ctl_kernel<<<1, kMaxCtl, 0, s>>>(a);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;

@@ -281,6 +281,16 @@ struct RtrArgs {
   int n, sys;
   uint32_t *dst[kMaxRdSteps + 2];
 };
+// Batched control ops (pc_startall / pc_pbuf_prepare_all): entry i either
+// bumps epoch[i] (dst == null) or stores *epoch[i] into dst[i] (RTR).
+constexpr int kMaxCtl = 64;
+struct CtlArgs {
+  int n;
+  const uint32_t *epoch[kMaxCtl];
+  uint32_t *dst[kMaxCtl];
+  int sys[kMaxCtl];
+};
+int launch_ctl(const CtlArgs &a, cudaStream_t s);
 int launch_epoch_bump(uint32_t *epoch, cudaStream_t s);
 int launch_rtr(const RtrArgs &a, cudaStream_t s);
 int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul, const uint32_t *layout,

@@ -291,6 +291,21 @@ class Request:
                 self.comm.requests.remove(self)
 
 
+def _handles(reqs):
+    arr = (C.c_void_p * len(reqs))(*[q.handle for q in reqs])
+    return arr
+
+
+def startall(reqs, stream=None):
+    """MPI_Startall: one kernel advances every request's epoch."""
+    check(_lib.pc().pc_startall(len(reqs), _handles(reqs), _stream(stream)), "pc_startall")
+
+
+def pbuf_prepare_all(reqs, stream=None):
+    """Ready-to-receive of already-exchanged requests in one kernel."""
+    check(_lib.pc().pc_pbuf_prepare_all(len(reqs), _handles(reqs), _stream(stream)), "pc_pbuf_prepare_all")
+
+
 def psend_init(buf, partitions: int, count: int, dtype: int, dest: int, tag: int, comm: Comm) -> Request:
     h = C.c_void_p()
     check(_lib.pc().pc_psend_init(_ptr(buf), partitions, count, dtype, dest, tag, comm.handle, C.byref(h)),

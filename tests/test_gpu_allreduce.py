@@ -201,13 +201,13 @@ def test_cuda_graph_replay_of_epochs():
         reqs = [pc.pallreduce_init(send[r], recv[r], Np, L, pc.FLOAT32, pc.SUM, pc.ALGO_RING, cs[r]) for r in range(P)]
 
         def step(first=False):
-            for q in reqs:
-                q.start(st)
             if first:
-                first_prepare([[q] for q in reqs], [st] * P)
-            else:
                 for q in reqs:
-                    q.pbuf_prepare(st)
+                    q.start(st)
+                first_prepare([[q] for q in reqs], [st] * P)
+            else:  # MPI_Startall analogue + batched ready-to-receive
+                pc.startall(reqs, st)
+                pc.pbuf_prepare_all(reqs, st)
             for q in reqs:
                 q.pready_range(0, Np - 1, st)
             for q in reqs:

@@ -37,13 +37,13 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
     reqs = [pc.pallreduce_init(send[r], recv[r], Np, count, pc.FLOAT32, pc.SUM, algo, cs[r]) for r in range(P)]
 
     def step(first=False):
-        for q in reqs:
-            q.start(st)
         if first:
+            for q in reqs:
+                q.start(st)
             pc.run_ranks([(lambda q=q: q.pbuf_prepare(st)) for q in reqs])
         else:
-            for q in reqs:
-                q.pbuf_prepare(st)
+            pc.startall(reqs, st)  # one kernel for every rank's epoch
+            pc.pbuf_prepare_all(reqs, st)  # one kernel for every RTR
         for q in reqs:
             q.pready_range(0, Np - 1, st)
         for q in reqs:
