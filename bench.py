@@ -291,8 +291,7 @@ def run_virtual(args):
         else:
             pc.startall(reqs, st)  # one kernel for every rank's epoch
             pc.pbuf_prepare_all(reqs, st)  # one kernel for every RTR
-        for q in reqs:
-            q.pready_range(0, Np - 1, st)
+        pc.preadyall(reqs, st)  # S_0: the user's Pready of every partition, one kernel
         for q in reqs:
             q.wait_on_stream(st)
 

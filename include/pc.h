@@ -154,6 +154,8 @@ int pc_wait_on_stream(pc_request_t req, pc_stream_t stream);
 /* Host Pready bindings (MPI_Pready / MPI_Pready_range): enqueue a tiny kernel
  * on `stream` that marks partitions [lo, hi] ready. */
 int pc_pready(int partition, pc_request_t req, pc_stream_t stream);
+/* Host Pready of EVERY partition of n requests (one GPU) in one kernel. */
+int pc_preadyall(int n, pc_request_t *reqs, pc_stream_t stream);
 int pc_pready_range(int lo, int hi, pc_request_t req, pc_stream_t stream);
 int pc_request_free(pc_request_t *req);
 

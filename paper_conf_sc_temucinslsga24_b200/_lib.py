@@ -55,6 +55,7 @@ _PC_PROTOS = {
     "pc_wait_on_stream": (I32, [P, P]),
     "pc_pready": (I32, [I32, P, P]),
     "pc_pready_range": (I32, [I32, I32, P, P]),
+    "pc_preadyall": (I32, [I32, P, P]),
     "pc_request_free": (I32, [C.POINTER(P)]),
     "pc_schedule_ring": (I32, [I32, I32, PI32]),
     "pc_schedule_rd": (I32, [I32, I32, PI32]),

@@ -1310,6 +1310,32 @@ int pc_test(pc_request_t req, int *flag) {
   return 0;
 }
 
+int pc_preadyall(int n, pc_request_t *reqs, pc_stream_t stream) {
+  if (n < 0 || (n > 0 && !reqs)) return PC_ERR_ARG;
+  PreadyAllArgs a{};
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    if (!q) return PC_ERR_ARG;
+    if (!q->active) return PC_ERR_STATE;
+    if (q->kind == PC_KIND_PRECV) return PC_ERR_ARG;
+    if (q->kind == PC_KIND_PSEND && !q->has_preq) return PC_ERR_STATE;
+    if (q->comm->device != ((Request *)reqs[0])->comm->device) return PC_ERR_ARG;
+    if (q->comm->dry) continue;
+    fill_prequest(q, &a.q[a.n]);
+    if (++a.n == kMaxPreadyAll) {
+      PC_CUDA(cudaSetDevice(q->comm->device));
+      int rc = launch_pready_all(a, (cudaStream_t)stream);
+      if (rc) return rc;
+      a.n = 0;
+    }
+  }
+  if (a.n) {
+    PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
+    return launch_pready_all(a, (cudaStream_t)stream);
+  }
+  return 0;
+}
+
 int pc_pready_range(int lo, int hi, pc_request_t req, pc_stream_t stream) {
   Request *q = (Request *)req;
   if (!q || lo < 0 || hi < lo || hi >= q->partitions) return PC_ERR_ARG;

@@ -238,15 +238,20 @@ __device__ __forceinline__ bool warp_poll(const uint32_t *p, uint32_t target, bo
 // Idle backoff shared by the sweeping engines; false on abort / timeout.
 struct Idle {
   uint64_t since = 0;
-  uint32_t ns = 0;
+  uint32_t ns = 0, spins = 0;
   __device__ __forceinline__ void progressed() {
     since = 0;
     ns = 0;
+    spins = 0;
   }
   __device__ __forceinline__ bool wait(int32_t *err, uint32_t tmo, int part) {
     if (since == 0) since = globaltimer();
-    ns = ns ? (ns < 1024 ? ns * 2 : 1024) : 64;
-    __nanosleep(ns);
+    // poll back-to-back first (a hop of a small message is ~1 us away), then
+    // back off so long waits (large slices upstream) leave the L2 alone
+    if (++spins > 64) {
+      ns = ns ? (ns < 512 ? ns * 2 : 512) : 32;
+      __nanosleep(ns);
+    }
     if (aborted(err)) return false;
     if (tmo && globaltimer() - since > (uint64_t)tmo * 1000000ull) {
       if ((threadIdx.x & 31) == 0) set_error(err, PC_DEV_ERR_TIMEOUT, part);
@@ -519,6 +524,18 @@ __global__ void rtr_kernel(RtrArgs a) {
   }
 }
 
+__global__ void pready_all_kernel(PreadyAllArgs a) {
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int W = (gridDim.x * blockDim.x) >> 5;
+  int base = 0;
+  for (int k = 0; k < a.n; ++k) {
+    const int np = a.q[k].partitions;
+    // global index base + j is taken by warp (base + j) mod W
+    for (int j = ((gw - base) % W + W) % W; j < np; j += W) pc_pready_warp(j, a.q[k]);
+    base += np;
+  }
+}
+
 __global__ void pready_range_kernel(pc_prequest_t q, int lo, int hi) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int W = (gridDim.x * blockDim.x) >> 5;
@@ -634,6 +651,18 @@ int launch_rtr(const RtrArgs &a, cudaStream_t s) {
 
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s) {
   set_word_kernel<<<1, 1, 0, s>>>(addr, value);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_pready_all(const PreadyAllArgs &a, cudaStream_t s) {
+  int total = 0;
+  for (int k = 0; k < a.n; ++k) total += a.q[k].partitions;
+  int blocks = (total + 7) / 8;
+  if (blocks > 148) blocks = 148;
+  if (blocks < 1) blocks = 1;
+  pready_all_kernel<<<blocks, 256, 0, s>>>(a);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;

@@ -298,6 +298,12 @@ int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint3
                       int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys);
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s);
 int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s);
+constexpr int kMaxPreadyAll = 16;
+struct PreadyAllArgs {
+  int n;
+  pc_prequest_t q[kMaxPreadyAll];
+};
+int launch_pready_all(const PreadyAllArgs &a, cudaStream_t s);
 int engine_occupancy_ctas_per_sm(int *ctas);
 uint64_t launch_count();
 

@@ -306,6 +306,11 @@ def pbuf_prepare_all(reqs, stream=None):
     check(_lib.pc().pc_pbuf_prepare_all(len(reqs), _handles(reqs), _stream(stream)), "pc_pbuf_prepare_all")
 
 
+def preadyall(reqs, stream=None):
+    """Host Pready of every partition of every request, one kernel."""
+    check(_lib.pc().pc_preadyall(len(reqs), _handles(reqs), _stream(stream)), "pc_preadyall")
+
+
 def psend_init(buf, partitions: int, count: int, dtype: int, dest: int, tag: int, comm: Comm) -> Request:
     h = C.c_void_p()
     check(_lib.pc().pc_psend_init(_ptr(buf), partitions, count, dtype, dest, tag, comm.handle, C.byref(h)),

@@ -208,8 +208,11 @@ def test_cuda_graph_replay_of_epochs():
             else:  # MPI_Startall analogue + batched ready-to-receive
                 pc.startall(reqs, st)
                 pc.pbuf_prepare_all(reqs, st)
-            for q in reqs:
-                q.pready_range(0, Np - 1, st)
+            if first:
+                for q in reqs:
+                    q.pready_range(0, Np - 1, st)
+            else:
+                pc.preadyall(reqs, st)
             for q in reqs:
                 q.wait_on_stream(st)
 
