@@ -219,6 +219,71 @@ def latency_pair(pc, apps, torch, comms, iters=5000, payload=0):
             "bare_flag_floor_mean": bare, "frac_of_floor": bare / float(np.percentile(rts, 50))}
 
 
+def c1_bench(pc, apps, torch, epochs=200):
+    """C1: 2 ranks, 1 MiB fp32 produced by a vector-add kernel (8 B/thread,
+    1024-thread blocks) with block-granularity Pready: 128 user partitions of
+    8 KiB aggregated g = 16 -> 8 transport partitions (reading R24), INLINE
+    "Kernel Copy".  Goodput (P:L223) = bytes / (kernel + communication) time,
+    against the traditional model (kernel -> cudaStreamSynchronize -> copy,
+    Listing 1)."""
+    import time as _t
+    n = 1 << 18
+    g, cs = pc.local_comms(2, 0)
+    st = torch.cuda.Stream()
+    A, B = torch.randn(n, device="cuda"), torch.randn(n, device="cuda")
+    Cb, R = torch.empty(n, device="cuda"), torch.empty(n, device="cuda")
+    snd = pc.psend_init(Cb, 128, 2048, pc.FLOAT32, 1, 11, cs[0])
+    rcv = pc.precv_init(R, 128, 2048, pc.FLOAT32, 0, 11, cs[1])
+    snd.start(st)
+    rcv.start(st)
+    pc.run_ranks([lambda: snd.pbuf_prepare(st), lambda: rcv.pbuf_prepare(st)])
+    sq = snd.prequest_create(pc.GRAN_BLOCK, 16, pc.COPY_INLINE)
+    apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
+    snd.wait_on_stream(st)
+    rcv.wait_on_stream(st)
+    torch.cuda.synchronize()
+
+    def epoch():
+        pc.startall([snd, rcv], st)
+        pc.pbuf_prepare_all([snd, rcv], st)
+        apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
+        snd.wait_on_stream(st)
+        rcv.wait_on_stream(st)
+
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    for _ in range(epochs):
+        epoch()
+    e1.record(st)
+    torch.cuda.synchronize()
+    part_us = e0.elapsed_time(e1) / epochs * 1e3
+    ok = bool(torch.equal(R, Cb)) and snd.error()[0] == 0 and rcv.error()[0] == 0
+    # traditional: kernel, host synchronisation, then the copy (Listing 1)
+    t0 = _t.perf_counter()
+    for _ in range(epochs):
+        apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st)
+        st.synchronize()
+        with torch.cuda.stream(st):
+            R.copy_(Cb)
+        st.synchronize()
+    trad_us = (_t.perf_counter() - t0) / epochs * 1e6
+    # partitioned, host-observed the same way (Listing 2: ... kernel; MPI_Wait)
+    t0 = _t.perf_counter()
+    for _ in range(epochs):
+        epoch()
+        st.synchronize()
+    part_host_us = (_t.perf_counter() - t0) / epochs * 1e6
+    snd.free()
+    rcv.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
+    return {"bytes": 4 * n, "partitions": 128, "transport_partitions": 8, "gran": "block", "copy": "inline",
+            "partitioned_us_device": part_us, "partitioned_us_host": part_host_us, "traditional_us_host": trad_us,
+            "goodput_gbs": 4 * n / (part_host_us / 1e6) / 1e9, "speedup_vs_traditional": trad_us / part_host_us,
+            "ok": ok, "note": "2 virtual ranks on one B200; paper: Kernel Copy up to 2.34x (P:L245, GH200)"}
+
+
 def jacobi_bench(pc, apps, torch, args):
     """C4: Jacobi 16384^2 fp32, 1 rank and 4x2 virtual ranks (intra-kernel
     partitioned halos), GFLOP/s at 4 flops per interior cell update (R17) and
@@ -391,6 +456,8 @@ def run_virtual(args):
     log("latency done")
     jac = None if args.no_jacobi else jacobi_bench(pc, apps, torch, args)
     log("jacobi done")
+    c1 = c1_bench(pc, apps, torch)
+    log("c1 done")
     cpu = None if args.no_cpu_baseline else oracle_sample(P=P)
     log("cpu baseline done")
     out = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": 1, "steps": args.steps,
@@ -404,7 +471,7 @@ def run_virtual(args):
                       "l2": f"no flush: working set {3 * P * S >> 20} MiB >> 126 MB L2",
                       "parallelism": f"{P} virtual ranks / 1 GPU"},
            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-           "clocks": clk.summary(), "latency_ns": lat, "jacobi": jac, "nccl": None}
+           "clocks": clk.summary(), "latency_ns": lat, "jacobi": jac, "c1_p2p": c1, "nccl": None}
     print(json.dumps(out), flush=True)
 
 
@@ -417,8 +484,14 @@ def run_multi(args):
 
     rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
     local = int(os.environ.get("LOCAL_RANK", rank))
+    ngpu = torch.cuda.device_count()
+    shared = ngpu < int(os.environ.get("LOCAL_WORLD_SIZE", world))  # ranks share GPUs (debug on a 1-GPU box)
+    local = local % ngpu
     torch.cuda.set_device(local)
-    dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if shared:  # NCCL refuses two ranks on one GPU: bootstrap over gloo, no NCCL baseline
+        dist.init_process_group("gloo")
+    else:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     P, S, Np = world, args.bytes, args.partitions
     count = S // 4 // Np
     S = count * 4 * Np
@@ -455,29 +528,32 @@ def run_multi(args):
         torch.cuda.synchronize()
         dist.barrier()
     launches = pc.launch_count() - n0
-    ms = torch.tensor([e0.elapsed_time(e1) / args.steps], device="cuda")
-    dist.all_reduce(ms, op=dist.ReduceOp.MAX)
-    ms = float(ms.item())
+    dev = "cpu" if shared else "cuda"
+
+    def max_over_ranks(v):
+        t = torch.tensor([v], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
     eng = q.engine_times()
-    eng_ms = torch.tensor([float(np.mean(eng)) if len(eng) else 0.0], device="cuda")
-    dist.all_reduce(eng_ms, op=dist.ReduceOp.MAX)
+    eng_ms = max_over_ranks(float(np.mean(eng)) if len(eng) else 0.0)
     assert q.error()[0] == 0
 
-    # NCCL baseline on the same bytes, same stream discipline
-    x = send.clone()
-    for _ in range(3):
-        dist.all_reduce(x)
-    torch.cuda.synchronize()
-    dist.barrier()
-    n0e, n1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    n0e.record()
-    for _ in range(args.steps):
-        dist.all_reduce(x)
-    n1e.record()
-    torch.cuda.synchronize()
-    nms = torch.tensor([n0e.elapsed_time(n1e) / args.steps], device="cuda")
-    dist.all_reduce(nms, op=dist.ReduceOp.MAX)
-    nms = float(nms.item())
+    nms = None
+    if not shared:  # NCCL baseline on the same bytes, same stream discipline
+        x = send.clone()
+        for _ in range(3):
+            dist.all_reduce(x)
+        torch.cuda.synchronize()
+        dist.barrier()
+        n0e, n1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        n0e.record()
+        for _ in range(args.steps):
+            dist.all_reduce(x)
+        n1e.record()
+        torch.cuda.synchronize()
+        nms = max_over_ranks(n0e.elapsed_time(n1e) / args.steps)
 
     # e2e: H2D input, allreduce, D2H result
     host_in = send.cpu().pin_memory()
@@ -495,13 +571,11 @@ def run_multi(args):
             host_out.copy_(recv, non_blocking=True)
     f1.record(st)
     torch.cuda.synchronize()
-    ems = torch.tensor([f0.elapsed_time(f1) / ke], device="cuda")
-    dist.all_reduce(ems, op=dist.ReduceOp.MAX)
-    ems = float(ems.item())
+    ems = max_over_ranks(f0.elapsed_time(f1) / ke)
     q.free()
     comm.destroy()
     if rank == 0:
-        eng_ms_v = float(eng_ms.item()) or None
+        eng_ms_v = eng_ms or None
         nvl_bytes = 2 * (P - 1) / P * S  # per rank per direction (ring)
         achieved = nvl_bytes / (eng_ms_v / 1e3) / 1e9 if eng_ms_v else None
         out = {"metric": METRIC, "value": busbw(S, ms / 1e3, P), "unit": "GB/s", "n_gpus": world,
@@ -518,8 +592,9 @@ def run_multi(args):
                "cpu_baseline": None, "e2e": {"value": busbw(S, ems / 1e3, P), "unit": "GB/s",
                                              "h2d_bytes_per_step": S, "d2h_bytes_per_step": S, "ms_per_step": ems},
                "gpu_launches": launches, "clocks": clk.summary(),
-               "nccl": {"value": busbw(S, nms / 1e3, P), "ms_per_step": nms, "unit": "GB/s",
-                        "call": "torch.distributed.all_reduce (NCCL 2.28.9)"}}
+               "nccl": ({"value": busbw(S, nms / 1e3, P), "ms_per_step": nms, "unit": "GB/s",
+                         "call": "torch.distributed.all_reduce (NCCL 2.28.9)"} if nms else
+                        {"skipped": "ranks share a GPU (debug run): NCCL needs one GPU per rank"})}
         print(json.dumps(out), flush=True)
     dist.destroy_process_group()
 
