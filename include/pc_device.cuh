@@ -19,12 +19,12 @@
  *     first combined per warp with __match_any_sync so one atomic covers every
  *     lane of the warp that targets the same t (the library-side aggregation
  *     the paper recommends).
- *   - INLINE copy ("Kernel Copy"): the warp/block whose contribution
- *     completes t pushes t's bytes to the receiver's buffer over NVLink with
- *     16-byte vector stores, then releases the receiver's flag[t] = e with a
- *     system-scope fence + store (the completion the paper sent through the
- *     host, done here on the device).  Before its first push of the
- *     epoch it checks the ready-to-receive word (Pbuf_prepare).
+ *   - INLINE copy ("Kernel Copy"): every caller pushes ITS OWN
+ *     partition's bytes to the receiver's buffer (16-byte vector stores over
+ *     NVLink, after checking the ready-to-receive word, Pbuf_prepare P:L62),
+ *     fences at the request's scope, then counts; the contribution that
+ *     completes t releases the receiver's flag[t] = e (the completion the
+ *     paper sent through the host, done here on the device).
  *   - ENGINE copy: the completing contributor only release-stores ready[t] = e;
  *     library engine warps move the data.
  *   - Allreduce requests: marks user partition u ready (step S_0 is the
@@ -227,90 +227,79 @@ PC_DEVICE bool contribute(const pc_prequest_t &q, int t, uint32_t add, uint32_t 
   return d <= (int32_t)add;
 }
 
-/* INLINE push of transport partition t by the lanes in `mask` (warp scope).
- * rtr0: the RTR value the caller already loaded together with the epoch. */
-PC_DEVICE void push_warp(const pc_prequest_t &q, int t, uint32_t e, unsigned mask, uint32_t rtr0 = 0) {
-  const uint32_t lane = lane_id();
-  const uint32_t first = __ffs(mask) - 1;
-  const uint32_t idx = __popc(mask & ((1u << lane) - 1));
-  const uint32_t n = __popc(mask);
-  const uint64_t off = (uint64_t)t * (uint64_t)q.agg * q.part_bytes;
-  const uint64_t len = (uint64_t)transport_size(q, t) * q.part_bytes;
-  if (len == 0) {  // flag only: no data to protect or order -> no RTR wait, no fence
-    if (lane == first) {
-      st_relaxed_sys(q.peer_flags + t, e);
-      st_relaxed_gpu(q.sent + t, e);
-    }
+/* Publish transport partition t once this contributor's own bytes are in
+ * place ("Kernel Copy": every contributor assigns its data to the
+ * peer address, counters aggregate, then the partition is marked).  The
+ * caller has already fenced its pushes at the request's scope.  g = 1: the
+ * contribution is the whole transport partition, flag it directly; g > 1: the
+ * acq_rel counter add orders every other contributor's (fenced) pushes before
+ * the completing contributor, which fences again and flags. */
+PC_DEVICE void publish(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, int part) {
+  if (q.agg == 1) {
+    st_relaxed_sys(q.peer_flags + t, e);
+    st_relaxed_gpu(q.sent + t, e);
     return;
   }
-  bool ok = true;
-  if (lane == first && !reached(rtr0, e)) ok = spin_geq<true>(q.rtr, e, q.err, q.timeout_ms, t);
-  ok = __shfl_sync(mask, ok, first);
-  if (!ok) return;
-  copy_bytes(q.peer_rbuf + off, q.sbuf + off, len, idx, n);
-  fence_scope(q.sys_scope);
-  __syncwarp(mask);
-  if (lane == first) {
+  if (contribute(q, t, add, e, part)) {
+    fence_scope(q.sys_scope);
     st_relaxed_sys(q.peer_flags + t, e);
-    st_relaxed_gpu(q.sent + t, e);  // ordered by the fence above
+    st_relaxed_gpu(q.sent + t, e);
   }
 }
 
-/* INLINE push of transport partition t by the whole block. */
-PC_DEVICE void push_block(const pc_prequest_t &q, int t, uint32_t e) {
-  __shared__ int s_ok;
-  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
-  const uint32_t nthr = blockDim.x * blockDim.y * blockDim.z;
-  if (tid == 0) s_ok = spin_geq<true>(q.rtr, e, q.err, q.timeout_ms, t);
-  __syncthreads();
-  if (!s_ok) return;
-  const uint64_t off = (uint64_t)t * (uint64_t)q.agg * q.part_bytes;
-  const uint64_t len = (uint64_t)transport_size(q, t) * q.part_bytes;
-  copy_bytes(q.peer_rbuf + off, q.sbuf + off, len, tid, nthr);
-  fence_scope(q.sys_scope);
-  __syncthreads();
-  if (tid == 0) {
-    st_relaxed_sys(q.peer_flags + t, e);
-    st_relaxed_gpu(q.sent + t, e);  // ordered by the fence above
-  }
+/* {epoch, rtr[0]} in one acquire at the request's scope (adjacent words). */
+PC_DEVICE uint2 epoch_rtr(const pc_prequest_t &q) {
+  return q.sys_scope ? ld_acquire_sys_v2(q.epoch) : ld_acquire_gpu_v2(q.epoch);
 }
 
 }  // namespace pc_detail
 
 /* ------------------------------------------------------------------ Pready */
 
-/* Thread granularity: any subset of threads, each for its own partition. */
+/* Thread granularity: any subset of threads, each for its own partition.
+ * INLINE: every lane pushes its own partition's bytes, lanes of the warp that
+ * share a transport partition are combined (__match_any_sync) into one counter
+ * update, the completing contribution flags it (P:L231's "aggregate to the
+ * block level internally", done per warp).  ENGINE: count, the completing
+ * contribution marks the transport partition ready for the engine. */
 PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
   using namespace pc_detail;
   if (partition < 0 || partition >= preq.partitions) {
     set_error(preq.err, PC_DEV_ERR_ARG, partition);
     return PC_DEV_ERR_ARG;
   }
-  const uint32_t e = epoch_of(preq);
   if (preq.kind == PC_KIND_PALLREDUCE) {
-    st_release_gpu(preq.ready + partition, e);
+    st_release_gpu(preq.ready + partition, epoch_of(preq));
     return 0;
   }
   const unsigned mask = __activemask();
   const uint32_t lane = lane_id();
+  const uint32_t first = __ffs(mask) - 1;
   const int t = partition / preq.agg;
   const unsigned grp = __match_any_sync(mask, t);
   const uint32_t leader = __ffs(grp) - 1;
-  __syncwarp(mask);  // every lane's data writes are ordered before the leader's release
-  bool completes = false;
-  if (lane == leader) completes = contribute(preq, t, __popc(grp), e, partition);
+  uint32_t e = 0, rtr0 = 0;
+  if (lane == first) {
+    const uint2 er = epoch_rtr(preq);
+    e = er.x;
+    rtr0 = er.y;
+  }
+  e = __shfl_sync(mask, e, first);
   if (preq.copy == 1) {  // ENGINE
-    if (completes) st_release_gpu(preq.ready + t, e);
+    __syncwarp(mask);    // every lane's data writes are ordered before the leader's release
+    if (lane == leader && contribute(preq, t, __popc(grp), e, partition)) st_release_gpu(preq.ready + t, e);
     return 0;
   }
-  unsigned cmask = __ballot_sync(mask, completes);
-  __syncwarp(mask);
-  while (cmask) {
-    const int src = __ffs(cmask) - 1;
-    cmask &= cmask - 1;
-    const int tt = __shfl_sync(mask, t, src);
-    push_warp(preq, tt, e, mask);
+  if (preq.part_bytes) {
+    bool ok = true;
+    if (lane == first && !reached(rtr0, e)) ok = spin_geq<true>(preq.rtr, e, preq.err, preq.timeout_ms, partition);
+    if (!__shfl_sync(mask, ok, first)) return PC_DEV_ERR_TIMEOUT;
+    const uint64_t off = (uint64_t)partition * preq.part_bytes;
+    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, 0, 1);
+    fence_scope(preq.sys_scope);
   }
+  __syncwarp(mask);
+  if (lane == leader) publish(preq, t, __popc(grp), e, partition);
   return 0;
 }
 
@@ -318,7 +307,8 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
  * the same partition (like __syncwarp()); one notification per warp (P:L137,
  * reading R11).  (__activemask() cannot be used to find the participants: with
  * independent thread scheduling a converged-looking warp may run this code as
- * several subsets, which would count the warp more than once.) */
+ * several subsets, which would count the warp more than once.)  INLINE: the
+ * warp pushes its partition with 16-B stores, then publishes. */
 PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   using namespace pc_detail;
   const unsigned full = 0xffffffffu;
@@ -334,52 +324,72 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
     return 0;
   }
   const int t = partition / preq.agg;
-  bool completes = false;
-  uint32_t e = 0, rtr0 = 0;
+  uint32_t e = 0;
+  bool ok = true;
   if (lane == 0) {
-    const uint2 er = preq.sys_scope ? ld_acquire_sys_v2(preq.epoch) : ld_acquire_gpu_v2(preq.epoch);  // {epoch, rtr[0]}
+    const uint2 er = epoch_rtr(preq);
     e = er.x;
-    rtr0 = er.y;
-    completes = contribute(preq, t, 1, e, partition);
+    if (preq.copy == 0 && preq.part_bytes && !reached(er.y, e))
+      ok = spin_geq<true>(preq.rtr, e, preq.err, preq.timeout_ms, partition);
   }
-  completes = __shfl_sync(full, completes, 0);
-  if (!completes) return 0;
   e = __shfl_sync(full, e, 0);
-  if (preq.copy == 1) {
-    if (lane == 0) st_release_gpu(preq.ready + t, e);
+  if (!__shfl_sync(full, ok, 0)) return PC_DEV_ERR_TIMEOUT;
+  if (preq.copy == 1) {  // ENGINE
+    if (lane == 0 && contribute(preq, t, 1, e, partition)) st_release_gpu(preq.ready + t, e);
     __syncwarp(full);
     return 0;
   }
-  push_warp(preq, t, e, full, rtr0);
+  if (preq.part_bytes) {
+    const uint64_t off = (uint64_t)partition * preq.part_bytes;
+    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, lane, 32);
+    fence_scope(preq.sys_scope);
+    __syncwarp(full);
+  }
+  if (lane == 0) publish(preq, t, 1, e, partition);
+  __syncwarp(full);
   return 0;
 }
 
 /* Block granularity: every thread of the block calls it with the same
- * partition; __syncthreads() then one notification. */
+ * partition; __syncthreads() then one notification.  INLINE: the
+ * block pushes its partition, then thread 0 publishes. */
 PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
   using namespace pc_detail;
-  __shared__ int s_completes;
+  __shared__ uint32_t s_e;
+  __shared__ int s_ok;
   const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  const uint32_t nthr = blockDim.x * blockDim.y * blockDim.z;
   if (partition < 0 || partition >= preq.partitions) {
     if (tid == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);
     return PC_DEV_ERR_ARG;
   }
-  const uint32_t e = epoch_of(preq);
-  __syncthreads();
+  __syncthreads();  // the block's data writes are complete
   if (preq.kind == PC_KIND_PALLREDUCE) {
-    if (tid == 0) st_release_gpu(preq.ready + partition, e);
+    if (tid == 0) st_release_gpu(preq.ready + partition, epoch_of(preq));
     return 0;
   }
   const int t = partition / preq.agg;
-  if (tid == 0) s_completes = contribute(preq, t, 1, e, partition);
+  if (tid == 0) {
+    const uint2 er = epoch_rtr(preq);
+    s_e = er.x;
+    s_ok = 1;
+    if (preq.copy == 0 && preq.part_bytes && !reached(er.y, er.x))
+      s_ok = spin_geq<true>(preq.rtr, er.x, preq.err, preq.timeout_ms, partition);
+  }
   __syncthreads();
-  const bool completes = s_completes;
-  if (!completes) return 0;
-  if (preq.copy == 1) {
-    if (tid == 0) st_release_gpu(preq.ready + t, e);
+  const uint32_t e = s_e;
+  if (!s_ok) return PC_DEV_ERR_TIMEOUT;
+  if (preq.copy == 1) {  // ENGINE
+    if (tid == 0 && contribute(preq, t, 1, e, partition)) st_release_gpu(preq.ready + t, e);
     return 0;
   }
-  push_block(preq, t, e);
+  if (preq.part_bytes) {
+    const uint64_t off = (uint64_t)partition * preq.part_bytes;
+    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, tid, nthr);
+    fence_scope(preq.sys_scope);
+    __syncthreads();
+  }
+  if (tid == 0) publish(preq, t, 1, e, partition);
   return 0;
 }
 
