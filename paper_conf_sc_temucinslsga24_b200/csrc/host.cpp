@@ -977,8 +977,14 @@ int pc_start(pc_request_t req, pc_stream_t stream) {
   q->user_stream = (cudaStream_t)stream;
   if (c->dry) return 0;
   PC_CUDA(cudaSetDevice(c->device));
-  // the device epoch word is advanced on the device (not written from a host
-  // value), so a CUDA graph that captured Start...Wait replays new epochs
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+  if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
+  // Eager requests write the epoch with a stream memop (cheapest); once a
+  // request has been captured into a CUDA graph its epoch is advanced on the
+  // device, so replays produce new epochs without the host.
+  if (!q->graph_mode && c->memops) return stream_write_u32(c, (cudaStream_t)stream, q->ctrl + q->L.epoch, q->epoch);
+  q->graph_mode = true;
   return launch_epoch_bump(q->ctrl + q->L.epoch, (cudaStream_t)stream);
 }
 
@@ -996,7 +1002,15 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
   if (c->dry) return 0;
   q->user_stream = (cudaStream_t)stream;
   if (!q->prepared_this_epoch) {
-    if (!q->rtr_targets.empty()) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+    if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
+    if (!q->graph_mode && c->memops) {  // eager: host epoch == device epoch
+      for (auto &t : q->rtr_targets) {
+        int rc = stream_write_u32(c, (cudaStream_t)stream, t.first + q->L.rtr + t.second, q->epoch);
+        if (rc) return rc;
+      }
+    } else if (!q->rtr_targets.empty()) {
       RtrArgs a{};
       a.epoch = q->ctrl + q->L.epoch;
       a.sys = q->sys_scope;
@@ -1022,9 +1036,12 @@ int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream) {
     if (q->comm->device != ((Request *)reqs[0])->comm->device || q->comm->dry != ((Request *)reqs[0])->comm->dry)
       return PC_ERR_ARG;
   }
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (n > 0 && !((Request *)reqs[0])->comm->dry) PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
   CtlArgs a{};
   for (int i = 0; i < n; ++i) {
     Request *q = (Request *)reqs[i];
+    if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
     q->epoch++;
     q->active = true;
     q->engine_launched = false;

@@ -148,6 +148,7 @@ struct Request {
   bool prepared_this_epoch = false;
   bool engine_launched = false;
   bool engine_registered = false;
+  bool graph_mode = false;  // captured into a CUDA graph: epochs advance on the device only
   bool matched = false;
   Request *leader = nullptr;  // co-located group leader (allreduce), or null
   GroupState gs;
