@@ -10,7 +10,7 @@ Functions (numpy in, numpy out):
   p2p(...)                O1  partitioned send/recv with aggregation + RTR
   allreduce_def_i32(...)  O2  plain definition, int32 (sum wraps, max, min)
   allreduce_def_f64(...)  O2  plain definition, fp32 inputs summed in fp64
-  pallreduce(...)         O3/O4  Alg 1 (ring) or RD schedule + Alg 2, P threads
+  pallreduce(...)         O3/O4/O6  Alg 1 (ring), RD or DIRECT schedule + Alg 2, P threads
   alg1_table(P, r)        Alg 1 step tuples
   ring_fold_f32 / rd_tree_f32   closed forms of O3 / O4 (pinned against them)
   jacobi_seq / jacobi_decomp    O5
@@ -29,7 +29,7 @@ _lib = None
 
 INT32, FLOAT32 = 0, 1
 SUM, MAX, MIN = 0, 1, 2
-RING, RD = 1, 2
+RING, RD, DIRECT = 1, 2, 3
 
 
 def build(force: bool = False) -> str:
@@ -50,6 +50,7 @@ def lib():
         _lib.orc_allreduce_def_i32.argtypes = [i32, i64, P, i32, P]
         _lib.orc_allreduce_def_f64.argtypes = [i32, i64, P, P, P]
         _lib.orc_pallreduce.argtypes = [i32, i32, i32, i64, i32, i32, i32, i32, P, P, P, u64, P, P]
+        _lib.orc_pallreduce_direct.argtypes = [i32, i32, i64, i32, i32, i32, i32, P, P, P, u64, P, P]
         _lib.orc_alg1_table.argtypes = [i32, i32, P]
         _lib.orc_ring_fold_f32.argtypes = [i32, i64, P, P, P]
         _lib.orc_rd_tree_f32.argtypes = [i32, i64, P, P]
@@ -109,6 +110,8 @@ def allreduce_def_f64(x: np.ndarray):
 def n_steps(algo: int, P: int) -> int:
     if algo == RING:
         return 2 * (P - 1)
+    if algo == DIRECT:
+        return 2
     k = 0
     while (1 << k) < P:
         k += 1
@@ -137,8 +140,12 @@ def pallreduce(x: np.ndarray, partitions: int, algo: int = RING, op: int = SUM, 
     y = np.zeros_like(x)
     red = np.zeros((P, partitions, ns), dtype=np.uint32)
     arr = np.zeros((P, partitions, ns), dtype=np.uint32)
-    _check(lib().orc_pallreduce(algo, P, partitions, L, dtype, op, epochs, int(inplace), _p(x), _p(y),
-                                _p(orders), jitter_seed, _p(red), _p(arr)), "orc_pallreduce")
+    if algo == DIRECT:
+        _check(lib().orc_pallreduce_direct(P, partitions, L, dtype, op, epochs, int(inplace), _p(x), _p(y),
+                                           _p(orders), jitter_seed, _p(red), _p(arr)), "orc_pallreduce_direct")
+    else:
+        _check(lib().orc_pallreduce(algo, P, partitions, L, dtype, op, epochs, int(inplace), _p(x), _p(y),
+                                    _p(orders), jitter_seed, _p(red), _p(arr)), "orc_pallreduce")
     return (y[0] if squeeze else y), red, arr
 
 

@@ -474,6 +474,157 @@ int orc_pallreduce(int algo, int P, int Np, int64_t L, int dtype, int op, int ep
   return failed ? ORC_ERR_TIMEOUT : ORC_OK;
 }
 
+// ===========================================================================
+// O6: partitioned allreduce over the DIRECT two-step schedule (
+// the generic schedule of P:L151-L155 with neighbour SETS, progressed by Alg 2
+// with |I| = |O| = P-1):
+//   S_0 = (I = all others, R = chunk o for each O_o, MPI_Op, O = all others,
+//          A = my chunk r from every I)          -- reduce-scatter to owners
+//   S_1 = (I = all others, R = my chunk r (final), NOP, O = all others,
+//          A = chunk i from every I_i)           -- allgather of owned chunks
+// Chunk c (reading R4) is owned by rank c.  Reading R25: with |I| > 1 the
+// arrivals of a step are reduced in rank order (reduceData of contribution k
+// only after 0..k-1), so the fp32 result is the left fold over ranks
+// 0..P-1, independent of arrival order.
+// ===========================================================================
+int orc_pallreduce_direct(int P, int Np, int64_t L, int dtype, int op, int epochs, int inplace, const void *x,
+                          void *y, const int32_t *orders, uint64_t jitter_seed, uint32_t *reduces,
+                          uint32_t *arrivals) {
+  if (P < 1 || Np < 1 || L < 0 || epochs < 1) return ORC_ERR_ARG;
+  const int64_t esz = 4, part_bytes = L * esz, nbytes = (int64_t)Np * part_bytes;
+  const int64_t q = ((L + 4 * P - 1) / (4 * P)) * 4;  // R4
+  auto chunk_lo = [&](int c) { return std::min<int64_t>((int64_t)c * q, L); };
+  auto chunk_n = [&](int c) { return std::min<int64_t>((int64_t)(c + 1) * q, L) - chunk_lo(c); };
+  struct Rk {
+    std::vector<uint8_t> send, recv, staging;  // staging[u][sender][chunk r]
+    uint8_t *sendbuf = nullptr, *recvbuf = nullptr;
+    std::vector<std::atomic<uint32_t>> flag;  // [u][step][sender], value = epoch
+    std::vector<std::atomic<uint32_t>> local_ready;
+    std::atomic<uint32_t> rtr{0};
+  };
+  std::vector<Rk> R(P);
+  for (int r = 0; r < P; ++r) {
+    R[r].send.assign((size_t)nbytes, 0);
+    R[r].recv.assign((size_t)nbytes, 0);
+    R[r].staging.assign((size_t)(Np * P * q * esz + 16), 0);
+    R[r].recvbuf = R[r].recv.data();
+    R[r].sendbuf = inplace ? R[r].recvbuf : R[r].send.data();
+    R[r].flag = std::vector<std::atomic<uint32_t>>((size_t)Np * 2 * P);
+    for (auto &f : R[r].flag) f.store(0);
+    R[r].local_ready = std::vector<std::atomic<uint32_t>>(Np);
+  }
+  std::vector<std::atomic<uint32_t>> red((size_t)P * Np * 2), arr((size_t)P * Np * 2);
+  std::atomic<int> failed{0};
+  auto stage_ptr = [&](int owner, int u, int sender) {
+    return R[owner].staging.data() + (((int64_t)u * P + sender) * q) * esz;
+  };
+  for (uint32_t e = 1; e <= (uint32_t)epochs; ++e) {
+    const bool last = e == (uint32_t)epochs;
+    for (int r = 0; r < P; ++r) {  // MPI_Start + the user's kernel producing sendbuf
+      std::memcpy(R[r].sendbuf, (const uint8_t *)x + ((int64_t)(e - 1) * P + r) * nbytes, (size_t)nbytes);
+      for (auto &f : R[r].local_ready) f.store(0);
+    }
+    for (int r = 0; r < P; ++r) R[r].rtr.store(e, std::memory_order_release);  // MPIX_Pbuf_prepare
+    std::vector<std::thread> th;
+    for (int r = 0; r < P; ++r) {
+      th.emplace_back([&, r] {  // user: Pready(u) = the step-0 Pready to every O
+        Jitter jit(jitter_seed + 7919u * e + r);
+        const int32_t *ord = orders + ((int64_t)(e - 1) * P + r) * Np;
+        for (int k = 0; k < Np; ++k) {
+          const int u = ord[k];
+          jit.maybe_yield();
+          R[r].local_ready[u].store(1, std::memory_order_release);
+          for (int o = 0; o < P; ++o) {
+            if (o == r) continue;
+            if (!spin_until([&] { return R[o].rtr.load(std::memory_order_acquire) >= e; })) failed = 1;
+            std::memcpy(stage_ptr(o, u, r), R[r].sendbuf + (int64_t)u * part_bytes + chunk_lo(o) * esz,
+                        (size_t)(chunk_n(o) * esz));
+            R[o].flag[((size_t)u * 2 + 0) * P + r].store(e, std::memory_order_release);
+          }
+        }
+      });
+      th.emplace_back([&, r] {  // MPI_Wait: Alg 2 over the two steps
+        auto &me = R[r];
+        std::vector<int> step(Np, 0), next(Np, 0), seen(Np, 0);
+        std::vector<std::vector<uint8_t>> work(Np, std::vector<uint8_t>((size_t)(q * esz + 16)));
+        Jitter jit(jitter_seed * 31 + 104729u * e + r);
+        auto t0 = std::chrono::steady_clock::now();
+        const int64_t n = chunk_n(r), off = chunk_lo(r) * esz;
+        for (;;) {
+          bool all = true;
+          for (int u = 0; u < Np; ++u) {
+            if (step[u] >= 2 || P == 1) {
+              if (P == 1 && step[u] == 0 && me.local_ready[u].load(std::memory_order_acquire)) {
+                std::memmove(me.recvbuf + (int64_t)u * part_bytes, me.sendbuf + (int64_t)u * part_bytes,
+                             (size_t)part_bytes);
+                step[u] = 2;
+              }
+              if (step[u] < 2) all = false;
+              continue;
+            }
+            all = false;
+            if (!me.local_ready[u].load(std::memory_order_acquire)) continue;  // R23
+            if (step[u] == 0) {
+              // arrivals of S_0 reduced in rank order (R25), each exactly once
+              while (next[u] < P) {
+                const int k = next[u];
+                const uint8_t *src;
+                if (k == r) {
+                  src = me.sendbuf + (int64_t)u * part_bytes + off;
+                } else {
+                  if (me.flag[((size_t)u * 2 + 0) * P + k].load(std::memory_order_acquire) != e) break;
+                  if (last) arr[((size_t)r * Np + u) * 2 + 0]++;
+                  src = stage_ptr(r, u, k);
+                }
+                if (k == 0) {
+                  std::memcpy(work[u].data(), src, (size_t)(n * esz));
+                } else {
+                  reduce_into(dtype, op, work[u].data(), work[u].data(), src, n);
+                  if (last) red[((size_t)r * Np + u) * 2 + 0]++;
+                }
+                next[u] = k + 1;
+              }
+              if (next[u] < P) continue;
+              // parrived = |I|, pready(S_0) = |O| (the user's) -> S_1: Pready the final chunk to every O
+              std::memcpy(me.recvbuf + (int64_t)u * part_bytes + off, work[u].data(), (size_t)(n * esz));
+              for (int o = 0; o < P; ++o) {
+                if (o == r) continue;
+                std::memcpy(R[o].recvbuf + (int64_t)u * part_bytes + off, work[u].data(), (size_t)(n * esz));
+                R[o].flag[((size_t)u * 2 + 1) * P + r].store(e, std::memory_order_release);
+              }
+              step[u] = 1;
+            }
+            if (step[u] == 1) {  // S_1 arrivals: chunk i from every I_i (NOP)
+              int got = 0;
+              for (int k = 0; k < P; ++k)
+                if (k != r && me.flag[((size_t)u * 2 + 1) * P + k].load(std::memory_order_acquire) == e) ++got;
+              if (got == P - 1) {
+                if (last) arr[((size_t)r * Np + u) * 2 + 1] += (uint32_t)got;
+                step[u] = 2;  // S_k: terminal
+              }
+            }
+          }
+          if (all) break;
+          jit.maybe_yield();
+          if (std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() > 120.0) {
+            failed = 1;
+            break;
+          }
+        }
+      });
+    }
+    for (auto &t : th) t.join();
+    for (int r = 0; r < P; ++r)
+      std::memcpy((uint8_t *)y + ((int64_t)(e - 1) * P + r) * nbytes, R[r].recvbuf, (size_t)nbytes);
+    if (failed) break;
+  }
+  if (reduces)
+    for (size_t k = 0; k < red.size(); ++k) reduces[k] = red[k].load();
+  if (arrivals)
+    for (size_t k = 0; k < arr.size(); ++k) arrivals[k] = arr[k].load();
+  return failed ? ORC_ERR_TIMEOUT : ORC_OK;
+}
+
 // Alg 1 table for (P, rank): out[i*5 + {0..4}] = I, R, op, O, A for i in [0, 2(P-1)).
 int orc_alg1_table(int P, int rank, int32_t *out) {
   if (P < 1 || rank < 0 || rank >= P) return ORC_ERR_ARG;

@@ -235,3 +235,49 @@ def test_def_f64_is_exactish():
     y, a = oracle.allreduce_def_f64(x)
     np.testing.assert_allclose(y, x.astype(np.float64).sum(0), rtol=0, atol=1e-12)
     np.testing.assert_allclose(a, np.abs(x.astype(np.float64)).sum(0), rtol=1e-15)
+
+
+# ------------------------------------------------------------- DIRECT (O6)
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 5, 8])
+def test_direct_int32_bruteforce_and_counts(P):
+    for Np in (1, 3, 8):
+        for L in (0, 1, 5, 17, 64):
+            x = np.stack([synth.int32_full(13, r, 0, Np * L) for r in range(P)])
+            orders = np.stack([synth.permutation(17, r, L, Np) for r in range(P)])[None]
+            y, red, arr = oracle.pallreduce(x, Np, oracle.DIRECT, orders=orders, jitter_seed=L)
+            for r in range(P):
+                np.testing.assert_array_equal(y[r], wrap_sum(x))
+            if P > 1:
+                # S_0: P-1 arrivals, P-1 reduces (one per incoming neighbour); S_1: P-1 arrivals
+                assert (red[:, :, 0] == P - 1).all() and (red[:, :, 1] == 0).all()
+                assert (arr == P - 1).all()
+
+
+@pytest.mark.parametrize("P", [2, 3, 5, 8])
+def test_direct_fp32_rank_order_fold(P):
+    """R25: the arrivals are folded in rank order, so every element is the left
+    fold over ranks 0..P-1 (the ring fold started at rank 0), on every rank,
+    whatever the arrival order."""
+    Np, L = 3, 101
+    x = np.stack([synth.normal_f32(71, r, 0, Np * L) for r in range(P)])
+    ref = oracle.ring_fold_f32(x, np.zeros(Np * L, np.int32))
+    for s in range(4):
+        orders = np.stack([synth.permutation(300 + s, r, 0, Np) for r in range(P)])[None]
+        y, _, _ = oracle.pallreduce(x, Np, oracle.DIRECT, orders=orders, jitter_seed=s)
+        for r in range(P):
+            np.testing.assert_array_equal(y[r].view(np.uint32), ref.view(np.uint32))
+    # by hand for P = 3: ((x0 + x1) + x2)
+    if P == 3:
+        np.testing.assert_array_equal(ref, ((x[0] + x[1]) + x[2]).astype(np.float32))
+    assert (np.abs(ref - x.astype(np.float64).sum(0)) <= 1e-5 * np.abs(x.astype(np.float64)).sum(0)).all()
+
+
+def test_direct_inplace_epochs_maxmin():
+    P, Np, L, E = 4, 2, 33, 3
+    x = np.stack([np.stack([synth.int32_full(5, r, e, Np * L) for r in range(P)]) for e in range(E)])
+    y, _, _ = oracle.pallreduce(x, Np, oracle.DIRECT, inplace=True)
+    for e in range(E):
+        for r in range(P):
+            np.testing.assert_array_equal(y[e, r], wrap_sum(x[e]))
+    y, _, _ = oracle.pallreduce(x[0], Np, oracle.DIRECT, op=oracle.MAX)
+    np.testing.assert_array_equal(y[0], x[0].max(0))
