@@ -50,8 +50,11 @@ typedef enum { PC_GRAN_THREAD = 0, PC_GRAN_WARP = 1, PC_GRAN_BLOCK = 2 } pc_gran
 typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1 } pc_copy_t;
 /* Allreduce schedule (§IV-B).  RING = Alg 1; RD = recursive
  * doubling (BASELINE north_star; not in the paper; P a power of two);
- * AUTO = RD below the size threshold (env PC_RD_MAX_BYTES), ring above. */
-typedef enum { PC_ALGO_AUTO = 0, PC_ALGO_RING = 1, PC_ALGO_RD = 2 } pc_algo_t;
+ * DIRECT = two steps over neighbour SETS (the generic schedule of P:L155 with
+ * |I| = |O| = P-1: reduce-scatter to chunk owners, allgather; P <= 8; the
+ * NVSwitch-native schedule of SURVEY NEXT-1); AUTO = RD below
+ * PC_RD_MAX_BYTES, DIRECT up to PC_DIRECT_MAX_BYTES, ring above. */
+typedef enum { PC_ALGO_AUTO = 0, PC_ALGO_RING = 1, PC_ALGO_RD = 2, PC_ALGO_DIRECT = 3 } pc_algo_t;
 
 enum {
   PC_SUCCESS = 0,

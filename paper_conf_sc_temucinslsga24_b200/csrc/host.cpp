@@ -482,6 +482,14 @@ static int exchange_round(Comm *c, Request *target) {
               qrc = import_ptr(c, mod(r - 1, P), peers[mod(r - 1, P)]->ctrl, &ict);
               if (!qrc) q->rtr_targets.push_back({(uint32_t *)ict, 0});
             }
+          } else if (q->algo == PC_ALGO_DIRECT) {
+            // peer j = rank (r+1+j) mod P; in peer p's control block the RTR
+            // slot of rank r is (r - p - 1) mod P
+            for (int j = 0; j < P - 1 && !qrc; ++j) {
+              const int pj = mod(r + 1 + j, P);
+              qrc = imp(pj, j);
+              if (!qrc) q->rtr_targets.push_back({q->nb_ctrl[j], mod(r - pj - 1, P)});
+            }
           } else {
             for (int k = 0; k < q->nsteps && !qrc; ++k) {
               qrc = imp(r ^ (1 << k), k);
@@ -597,6 +605,39 @@ static RdArgs make_rd_args(Request *q) {
   return a;
 }
 
+static DirectArgs make_direct_args(Request *q) {
+  Comm *c = q->comm;
+  DirectArgs a{};
+  a.epoch = q->ctrl + q->L.epoch;
+  a.P = c->size;
+  a.r = c->rank;
+  a.Np = q->partitions;
+  a.ns = q->slices;
+  a.nunits = q->partitions * q->slices;
+  a.op = q->op;
+  a.dtype = q->dtype;
+  a.L = (int64_t)q->count;
+  a.q = q->chunk_elems;
+  a.qs = q->slice_elems;
+  a.sq = q->chunk_elems + 4;
+  a.sendbuf = (const uint8_t *)q->sbuf;
+  a.recvbuf = (uint8_t *)q->rbuf;
+  a.staging = q->staging;
+  a.cnt = q->ctrl + q->L.flags;
+  a.ready = q->ctrl + q->L.ready;
+  a.rtr = q->ctrl + q->L.rtr;
+  a.done = q->ctrl + q->L.donecnt;
+  for (int j = 0; j < c->size - 1; ++j) {
+    a.p_staging[j] = q->nb_stage[j];
+    a.p_recvbuf[j] = q->nb_buf[j];
+    a.p_cnt[j] = q->nb_ctrl[j] + q->L.flags;
+  }
+  a.err = (int32_t *)(q->ctrl + q->L.err);
+  a.timeout_ms = c->timeout_ms;
+  a.sys = q->sys_scope;
+  return a;
+}
+
 static bool needs_engine(Request *q) {
   return q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
 }
@@ -627,8 +668,9 @@ static int launch_single(Request *q) {
   int rc, tk;
   if ((rc = timing_begin(q->tlog, q->side, &tk))) return rc;
   if (q->kind == PC_KIND_PALLREDUCE) {
-    rc = q->algo == PC_ALGO_RING ? launch_ring_engine(make_ring_args(q), q->engine_warps, q->side)
-                                 : launch_rd_engine(make_rd_args(q), q->engine_warps, q->side);
+    rc = q->algo == PC_ALGO_RING     ? launch_ring_engine(make_ring_args(q), q->engine_warps, q->side)
+         : q->algo == PC_ALGO_DIRECT ? launch_direct_engine(make_direct_args(q), q->engine_warps, q->side)
+                                     : launch_rd_engine(make_rd_args(q), q->engine_warps, q->side);
   } else {
     P2pEngineArgs a{};
     a.epoch = q->ctrl + q->L.epoch;
@@ -687,6 +729,11 @@ static int group_register(Request *q, bool block, bool *launched) {
       ga.n = (int)g.members.size();
       for (int k = 0; k < ga.n; ++k) ga.a[k] = make_ring_args(g.members[k]);
       rc = launch_ring_engine_group(ga, q->engine_warps, q->side);
+    } else if (q->algo == PC_ALGO_DIRECT) {
+      DirectGroupArgs ga{};
+      ga.n = (int)g.members.size();
+      for (int k = 0; k < ga.n; ++k) ga.a[k] = make_direct_args(g.members[k]);
+      rc = launch_direct_engine_group(ga, q->engine_warps, q->side);
     } else {
       RdGroupArgs ga{};
       ga.n = (int)g.members.size();
@@ -911,7 +958,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
                        pc_op_t op, pc_algo_t algo, pc_comm_t comm, pc_request_t *req) {
   Comm *c = (Comm *)comm;
   if (!c || !req || partitions < 1 || (dtype != PC_INT32 && dtype != PC_FLOAT32) || op < 0 || op > 2 ||
-      algo < 0 || algo > 2)
+      algo < 0 || algo > 3)
     return PC_ERR_ARG;
   const int P = c->size;
   const uint64_t bytes = (uint64_t)partitions * count * 4;
@@ -923,6 +970,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
     a = (pow2 && (long long)bytes <= rd_max && P > 1) ? PC_ALGO_RD : PC_ALGO_RING;
   }
   if (a == PC_ALGO_RD && !pow2) return PC_ERR_UNSUPPORTED;
+  if (a == PC_ALGO_DIRECT && P > kMaxDirect) return PC_ERR_UNSUPPORTED;
   Request *q;
   int rc = new_request(c, PC_KIND_PALLREDUCE, req, &q);
   if (rc) return rc;
@@ -953,6 +1001,11 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
     q->chunk_elems = chunk_q(L, P);
     choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems);
     q->staging_bytes = P > 1 ? bytes : 0;
+  } else if (a == PC_ALGO_DIRECT) {
+    q->nsteps = 2;  // phase counters [u][0..1][slice]
+    q->chunk_elems = chunk_q(L, P);
+    choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems);
+    q->staging_bytes = P > 1 ? (uint64_t)partitions * P * (q->chunk_elems + 4) * 4 : 0;
   } else {
     q->nsteps = log2_exact(P);
     q->chunk_elems = L;

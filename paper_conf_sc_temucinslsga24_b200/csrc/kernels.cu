@@ -394,6 +394,156 @@ __device__ __forceinline__ void rd_body(const RdArgs &a, const int gw, const int
   }
 }
 
+// ---------------------------------------------------------------------------
+// Direct two-step schedule (generic schedule with neighbour
+// sets).  Unit (u, slice s):
+//   step 0 (after the user's Pready of u): push slice s of chunk o to owner
+//          o's staging slot [u][r] for every peer o, then bump each owner's
+//          phase-0 counter;
+//   step 1 (all P-1 phase-0 arrivals): fold the P contributions of my chunk
+//          in rank order (reading R25) in registers, store the final slice
+//          locally and into every peer's recvbuf, bump their phase-1 counters;
+//   step 2 (all P-1 phase-1 arrivals): slice final everywhere -> done[u].
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void red_add_scope(uint32_t *p, uint32_t v, bool sys) {
+  if (sys)
+    asm volatile("red.relaxed.sys.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+  else
+    asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// out_local and out_peer[j] (j < P-1) = fold over k = 0..P-1 of src[k] in rank
+// order; all pointers share one misalignment (scalar head, 16-B body, tail).
+template <int DT, int OP>
+__device__ __forceinline__ void warp_fold_direct(void *out_local, uint8_t *const *out_peer, const uint8_t *const *src,
+                                                 int P, int64_t n) {
+  using O = Op<DT, OP>;
+  using T = typename O::T;
+  const uint32_t lane = threadIdx.x & 31;
+  const uintptr_t m = reinterpret_cast<uintptr_t>(out_local) & 15;
+  int64_t head = (int64_t)(((16 - m) & 15) >> 2);
+  if (head > n) head = n;
+  auto scalar = [&](int64_t k) {
+    T acc = __ldcg(reinterpret_cast<const T *>(src[0]) + k);
+    for (int j = 1; j < P; ++j) acc = O::f(acc, __ldcg(reinterpret_cast<const T *>(src[j]) + k));
+    reinterpret_cast<T *>(out_local)[k] = acc;
+    for (int j = 0; j < P - 1; ++j) reinterpret_cast<T *>(out_peer[j])[k] = acc;
+  };
+  for (int64_t k = lane; k < head; k += 32) scalar(k);
+  const int64_t nv = (n - head) >> 2;
+  for (int64_t k = lane; k < nv; k += 32) {
+    const int64_t eo = head + 4 * k;  // element offset
+    uint4 acc = __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(src[0]) + eo));
+    for (int j = 1; j < P; ++j)
+      acc = vop<DT, OP>(acc, __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(src[j]) + eo)));
+    *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(out_local) + eo) = acc;
+    for (int j = 0; j < P - 1; ++j) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(out_peer[j]) + eo) = acc;
+  }
+  for (int64_t k = head + (nv << 2) + lane; k < n; k += 32) scalar(k);
+}
+
+template <int DT, int OP>
+__device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W) {
+  const int P = a.P, r = a.r;
+  const uint32_t e = *(const volatile uint32_t *)a.epoch;
+  const int64_t es = 4;
+  if (gw >= a.nunits) return;
+  if (P == 1) {
+    for (int x = gw; x < a.nunits; x += W) {
+      const int u = x / a.ns, s = x % a.ns;
+      if (!warp_wait(a.ready + u, e, a.err, a.timeout_ms, u, false)) return;
+      const int64_t base = (int64_t)u * a.L, lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
+      if (hi > lo && a.sendbuf != a.recvbuf)
+        warp_copy(a.recvbuf + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
+      __syncwarp();
+      if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+    }
+    return;
+  }
+  for (int j = 0; j < P - 1; ++j)  // every peer has posted ready-to-receive
+    if (!warp_wait(a.rtr + j, e, a.err, a.timeout_ms, -1, a.sys)) return;
+  const uint32_t target = e * (uint32_t)(P - 1);
+  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
+    int step[kMaxActive];
+    int remaining = 0;
+#pragma unroll
+    for (int j = 0; j < kMaxActive; ++j) {
+      const bool mine = gw + (j0 + j) * W < a.nunits;
+      step[j] = mine ? 0 : 3;
+      remaining += mine;
+    }
+    Idle idle;
+    while (remaining) {
+      bool progressed = false;
+#pragma unroll
+      for (int jj = 0; jj < kMaxActive; ++jj) {
+        if (step[jj] > 2) continue;
+        const int x = gw + (j0 + jj) * W;
+        const int u = x / a.ns, s = x % a.ns;
+        const int i = step[jj];
+        const uint32_t *dep = i == 0 ? a.ready + u : a.cnt + ((int64_t)u * 2 + (i - 1)) * a.ns + s;
+        if (!warp_poll(dep, i == 0 ? e : target, i != 0 && a.sys)) continue;
+        progressed = true;
+        const int64_t base = (int64_t)u * a.L;
+        const int64_t mis = base & 3;  // the buffers' misalignment in elements (staging mirrors it)
+        if (i == 0) {
+          for (int j = 0; j < P - 1; ++j) {
+            const int o = (r + 1 + j) % P;
+            const int64_t c_lo = min((int64_t)o * a.q, a.L), c_hi = min((int64_t)(o + 1) * a.q, a.L);
+            const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
+            if (hi > lo)
+              warp_copy(a.p_staging[j] + (((int64_t)u * P + r) * a.sq + mis + (int64_t)s * a.qs) * es,
+                        a.sendbuf + (base + lo) * es, (hi - lo) * es);
+          }
+          fence_scope(a.sys);
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0)
+            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 0) * a.ns + s, 1, a.sys);
+          step[jj] = 1;
+        } else if (i == 1) {
+          const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
+          const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
+          if (hi > lo) {
+            const uint8_t *src[kMaxDirect];
+            uint8_t *outp[kMaxDirect - 1];
+            for (int k = 0; k < P; ++k)
+              src[k] = k == r ? a.sendbuf + (base + lo) * es
+                              : a.staging + (((int64_t)u * P + k) * a.sq + mis + (int64_t)s * a.qs) * es;
+            for (int j = 0; j < P - 1; ++j) outp[j] = a.p_recvbuf[j] + (base + lo) * es;
+            warp_fold_direct<DT, OP>(a.recvbuf + (base + lo) * es, outp, src, P, hi - lo);
+          }
+          fence_scope(a.sys);
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0)
+            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
+          step[jj] = 2;
+        } else {
+          if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+          step[jj] = 3;
+          --remaining;
+        }
+      }
+      if (progressed)
+        idle.progressed();
+      else if (!idle.wait(a.err, a.timeout_ms, gw))
+        return;
+    }
+  }
+}
+
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) direct_engine(DirectArgs a) {
+  direct_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
+}
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) direct_engine_group(DirectGroupArgs g) {
+  int k = 0;
+  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
+  const int b = blockIdx.x - g.block_start[k];
+  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
+  direct_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
+}
+
 // Single-rank launches (one rank per GPU / process).
 template <int DT, int OP>
 __global__ void __launch_bounds__(kEngineBlock) ring_engine(RingArgs a) {
@@ -606,6 +756,30 @@ int launch_rd_engine_group(const RdGroupArgs &g, int warps, cudaStream_t s) {
   }
   return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
     rd_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
+    g_launches++;
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  });
+}
+
+int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s) {
+  return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
+    direct_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    g_launches++;
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  });
+}
+
+int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t s) {
+  DirectGroupArgs h = g;
+  int blocks = 0;
+  for (int k = 0; k < g.n; ++k) {
+    h.block_start[k] = blocks;
+    blocks += grid_for(warps, g.a[k].nunits);
+  }
+  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
+    direct_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
     g_launches++;
     PC_CUDA(cudaGetLastError());
     return 0;

@@ -265,6 +265,31 @@ struct RingGroupArgs {
   int block_start[kMaxLocal];
   RingArgs a[kMaxLocal];
 };
+// Direct two-step schedule (reduce-scatter to chunk owners, allgather of the
+// owned chunks) for P <= kMaxDirect ranks; peer j is rank (r + 1 + j) mod P.
+constexpr int kMaxDirect = 8;
+struct DirectArgs {
+  const uint32_t *epoch;
+  int P, r, Np, ns, nunits, op, dtype;
+  int64_t L, q, qs, sq;  // sq: staging slot stride in elements (q + 4)
+  const uint8_t *sendbuf;
+  uint8_t *recvbuf;
+  const uint8_t *staging;  // [u][sender][sq] (+ u*L mod 4 so it shares the buffers' misalignment)
+  const uint32_t *cnt, *ready, *rtr;  // cnt: [u][phase][slice] arrival counters (written by peers)
+  uint32_t *done;
+  uint8_t *p_staging[kMaxDirect - 1], *p_recvbuf[kMaxDirect - 1];
+  uint32_t *p_cnt[kMaxDirect - 1];
+  int32_t *err;
+  uint32_t timeout_ms;
+  int sys;
+};
+struct DirectGroupArgs {
+  int n;
+  int block_start[kMaxLocal];
+  DirectArgs a[kMaxLocal];
+};
+int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s);
+int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t s);
 struct RdGroupArgs {
   int n;
   int block_start[kMaxLocal];

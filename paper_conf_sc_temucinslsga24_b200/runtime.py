@@ -19,7 +19,7 @@ INT32, FLOAT32, BYTE = 0, 1, 2
 SUM, MAX, MIN = 0, 1, 2
 GRAN_THREAD, GRAN_WARP, GRAN_BLOCK = 0, 1, 2
 COPY_INLINE, COPY_ENGINE = 0, 1
-ALGO_AUTO, ALGO_RING, ALGO_RD = 0, 1, 2
+ALGO_AUTO, ALGO_RING, ALGO_RD, ALGO_DIRECT = 0, 1, 2, 3
 KIND_PSEND, KIND_PRECV, KIND_PALLREDUCE = 1, 2, 3
 
 SUCCESS, ERR_ARG, ERR_CUDA, ERR_STATE, ERR_MATCH, ERR_TIMEOUT, ERR_DEVICE, ERR_NOMEM, ERR_UNSUPPORTED = (

@@ -112,6 +112,9 @@ def check_fp32(x, y, algo, Np, L):
     if algo == pc.ALGO_RING:
         lit, _, _ = oracle.pallreduce(x, Np, oracle.RING) if x.size <= 4_000_000 else (None, 0, 0)
         cf = oracle.ring_fold_f32(x, oracle.chunk_ids(L, P, Np))
+    elif algo == pc.ALGO_DIRECT:  # R25: left fold over ranks 0..P-1
+        lit, _, _ = oracle.pallreduce(x, Np, oracle.DIRECT) if x.size <= 4_000_000 else (None, 0, 0)
+        cf = oracle.ring_fold_f32(x, np.zeros(x.shape[1], np.int32))
     else:
         lit, _, _ = oracle.pallreduce(x, Np, oracle.RD) if x.size <= 4_000_000 else (None, 0, 0)
         cf = oracle.rd_tree_f32(x)
@@ -236,3 +239,38 @@ def test_cuda_graph_replay_of_epochs():
         for q in reqs:
             assert q.error() == (0, 0)
             q.free()
+
+
+# ------------------------------------------------------------------ DIRECT
+@pytest.mark.parametrize("P", [1, 2, 3, 5, 8])
+@pytest.mark.parametrize("Np,L", [(1, 1), (3, 17), (7, 64), (2, 1000)])
+def test_direct_int32_sum(P, Np, L):
+    x = np.stack([synth.int32_full(SEED + 30, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_DIRECT)
+    for r in range(P):
+        np.testing.assert_array_equal(y[r], wrap_sum(x))
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+@pytest.mark.parametrize("Np,L", [(1, 1), (3, 17), (2, 4099)])
+def test_direct_fp32_bitexact(P, Np, L):
+    x = np.stack([synth.normal_f32(SEED + 31, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_DIRECT)
+    check_fp32(x, y, pc.ALGO_DIRECT, Np, L)
+
+
+def test_direct_ragged_inplace_epochs_producer():
+    P, Np, L = 8, 3, 300_001
+    xs = [np.stack([synth.normal_f32(SEED + 32, r, e, Np * L) for r in range(P)]) for e in range(3)]
+    ys = run_allreduce(P, Np, L, xs, pc.ALGO_DIRECT, inplace=True, producer=2)
+    for x, y in zip(xs, ys):
+        check_fp32(x, y, pc.ALGO_DIRECT, Np, L)
+
+
+@pytest.mark.parametrize("op", [pc.MAX, pc.MIN])
+def test_direct_maxmin(op):
+    P, Np, L = 5, 4, 333
+    x = np.stack([synth.int32_full(SEED + 33, r, 0, Np * L) for r in range(P)])
+    (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_DIRECT, op=op)
+    for r in range(P):
+        np.testing.assert_array_equal(y[r], oracle.allreduce_def_i32(x, op))

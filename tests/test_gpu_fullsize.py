@@ -49,7 +49,7 @@ def run_bench_shape(P, S, Np, algo, gen_rank, dtype=torch.float32, steps=2):
         return recv, count, info
 
 
-@pytest.mark.parametrize("algo,S", [(pc.ALGO_RING, 256 << 20), (pc.ALGO_RD, 64 << 20)])
+@pytest.mark.parametrize("algo,S", [(pc.ALGO_RING, 256 << 20), (pc.ALGO_RD, 64 << 20), (pc.ALGO_DIRECT, 256 << 20)])
 def test_fullsize_sampled_fp32(algo, S):
     P, Np = 8, 64
     recv, L, info = run_bench_shape(P, S, Np, algo, lambda r, n: synth.uniform_f32(SEED, r, 0, n))
@@ -60,6 +60,8 @@ def test_fullsize_sampled_fp32(algo, S):
     if algo == pc.ALGO_RING:
         chunk = oracle.chunk_ids(L, P, 1)[idx % L]
         ref = oracle.ring_fold_f32(xs, chunk)
+    elif algo == pc.ALGO_DIRECT:
+        ref = oracle.ring_fold_f32(xs, np.zeros(len(idx), np.int32))
     else:
         ref = oracle.rd_tree_f32(xs)
     y64, sabs = oracle.allreduce_def_f64(xs)
