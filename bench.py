@@ -41,7 +41,7 @@ def parse():
     ap.add_argument("--impl", default="pc", choices=["pc", "reference"])
     ap.add_argument("--bytes", type=int, default=256 << 20, help="bytes per rank (S)")
     ap.add_argument("--partitions", type=int, default=64)
-    ap.add_argument("--algo", default="ring", choices=["ring", "rd", "auto"])
+    ap.add_argument("--algo", default="ring", choices=["ring", "rd", "direct", "auto"])
     ap.add_argument("--vranks", type=int, default=8, help="virtual ranks on the one GPU when N = 1")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -353,7 +353,7 @@ def run_virtual(args):
     P, S, Np = args.vranks, args.bytes, args.partitions
     count = S // 4 // Np
     S = count * 4 * Np
-    algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "auto": pc.ALGO_AUTO}[args.algo]
+    algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "auto": pc.ALGO_AUTO}[args.algo]
     g, comms = pc.local_comms(P, 0)
     st = torch.cuda.Stream()
     gen = torch.Generator(device="cuda")
@@ -510,7 +510,7 @@ def run_multi(args):
     P, S, Np = world, args.bytes, args.partitions
     count = S // 4 // Np
     S = count * 4 * Np
-    algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "auto": pc.ALGO_AUTO}[args.algo]
+    algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "auto": pc.ALGO_AUTO}[args.algo]
     comm = pc.Comm.from_process_group(local)
     st = torch.cuda.Stream()
     gen = torch.Generator(device="cuda")

@@ -79,7 +79,7 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
     for q in reqs:
         q.free()
     ms = statistics.median(blocks)
-    return {"bytes_per_rank": n * 4, "partitions": Np, "ranks": P, "algo": ["auto", "ring", "rd"][algo],
+    return {"bytes_per_rank": n * 4, "partitions": Np, "ranks": P, "algo": ["auto", "ring", "rd", "direct"][algo],
             "us_per_step": ms * 1e3, "busbw_gbs": busbw(n * 4, ms / 1e3, P), "slices": info["slices"],
             "graph": graph, "errors": errs}
 
@@ -88,7 +88,7 @@ def sweep_allreduce(args):
     for P in [int(x) for x in args.ranks.split(",")]:
         g, cs = pc.local_comms(P, 0)
         for algo in args.algos.split(","):
-            a = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "auto": pc.ALGO_AUTO}[algo]
+            a = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "auto": pc.ALGO_AUTO}[algo]
             if a == pc.ALGO_RD and P & (P - 1):
                 continue
             S = 1 << 10
