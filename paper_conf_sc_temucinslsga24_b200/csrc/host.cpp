@@ -966,8 +966,17 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   int a = algo;
   const bool pow2 = log2_exact(P) >= 0;
   if (a == PC_ALGO_AUTO) {
-    const long rd_max = env_long("PC_RD_MAX_BYTES", 512 * 1024);
-    a = (pow2 && (long long)bytes <= rd_max && P > 1) ? PC_ALGO_RD : PC_ALGO_RING;
+    // crossovers measured on one B200 with virtual ranks (profiles/r01_sweep_*):
+    // RD (log2 P hops) wins up to ~1 MiB, DIRECT (2 steps) around 4 MiB at
+    // P = 8, the ring (bandwidth-optimal bytes) above
+    const long rd_max = env_long("PC_RD_MAX_BYTES", 1 << 20);
+    const long direct_max = env_long("PC_DIRECT_MAX_BYTES", 8 << 20);
+    if (P > 1 && pow2 && (long long)bytes <= rd_max)
+      a = PC_ALGO_RD;
+    else if (P > 4 && P <= kMaxDirect && (long long)bytes <= direct_max)
+      a = PC_ALGO_DIRECT;
+    else
+      a = PC_ALGO_RING;
   }
   if (a == PC_ALGO_RD && !pow2) return PC_ERR_UNSUPPORTED;
   if (a == PC_ALGO_DIRECT && P > kMaxDirect) return PC_ERR_UNSUPPORTED;
