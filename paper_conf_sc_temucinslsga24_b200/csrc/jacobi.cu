@@ -75,10 +75,11 @@ __device__ void tile_iter(const JacobiRank &d, int tile, int k) {
   else up = cur;  // global boundary row: not used
   const int gx = d.gx0 + x0;
   const bool colfix0 = gx == 0, colfix3 = gx + 3 == d.N - 1;
-  // Rows in batches of kRB, software-pipelined: while batch b is computed the
-  // kRB rows (and lane-0 / lane-31 edge scalars) of batch b+1 are in flight,
-  // so each warp keeps up to 2*kRB 512-B loads outstanding.
-  auto load_batch = [&](int r, float4 *nx, float *le, float *re) {
+  // Rows in batches of kRB: the kRB next rows (and the lane-0 / lane-31 edge
+  // scalars) are loaded together so each warp keeps kRB 512-B loads in flight.
+  for (int r = r0; r < r0 + d.H; r += kRB) {
+    float4 nx[kRB];
+    float le[kRB], re[kRB];
 #pragma unroll
     for (int j = 0; j < kRB; ++j) {
       const int rr = r + 1 + j;
@@ -92,13 +93,6 @@ __device__ void tile_iter(const JacobiRank &d, int tile, int k) {
       if (lane == 0) le[j] = x0 > 0 ? __ldcg(a + (size_t)rr * lx + x0 - 1) : (d.has[L] ? __ldcg(hL + rr) : 0.f);
       if (lane == 31) re[j] = x0 + 4 < lx ? __ldcg(a + (size_t)rr * lx + x0 + 4) : (d.has[R] ? __ldcg(hR + rr) : 0.f);
     }
-  };
-  float4 nx[kRB], nx2[kRB];
-  float le[kRB], re[kRB], le2[kRB], re2[kRB];
-  load_batch(r0, nx, le, re);
-  for (int r = r0; r < r0 + d.H; r += kRB) {
-    const bool more = r + kRB < r0 + d.H;
-    if (more) load_batch(r + kRB, nx2, le2, re2);
 #pragma unroll
     for (int j = 0; j < kRB; ++j) {
       const int rr = r + j;
@@ -125,14 +119,6 @@ __device__ void tile_iter(const JacobiRank &d, int tile, int k) {
       if (right && lane == 31) d.sendbuf[R][(size_t)(k + 1) * ly + rr] = o.w;
       up = cur;
       cur = dn;
-    }
-    if (more) {
-#pragma unroll
-      for (int j = 0; j < kRB; ++j) {
-        nx[j] = nx2[j];
-        le[j] = le2[j];
-        re[j] = re2[j];
-      }
     }
   }
   // Pready: push my edge segments of slot k+1 (INLINE copy by this warp)
