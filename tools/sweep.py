@@ -7,6 +7,7 @@
 Each point: busBW (allreduce) or GB/s (p2p) from CUDA events over many
 back-to-back epochs on one stream (the bench step), median of 3 blocks."""
 import argparse
+import collections
 import json
 import os
 import statistics
@@ -120,6 +121,63 @@ def sweep_dl(args):
         g.destroy()
 
 
+def sweep_dl_per_tensor(args):
+    """C3 workload (ii): one partitioned-allreduce request per gradient tensor
+    (AUTO schedule per size), one epoch of all of them captured in a CUDA graph."""
+    for P in [int(x) for x in args.ranks.split(",")]:
+        g, cs = pc.local_comms(P, 0)
+        for name, sizes in (("resnet50", synth.RESNET50_SIZES),):
+            st = torch.cuda.Stream()
+            bufs = [[torch.randn(n, device="cuda") for n in sizes] for _ in range(P)]
+            outs = [[torch.empty(n, device="cuda") for n in sizes] for _ in range(P)]
+            reqs = [[pc.pallreduce_init(bufs[r][t], outs[r][t], 1, n, pc.FLOAT32, pc.SUM, pc.ALGO_AUTO, cs[r])
+                     for t, n in enumerate(sizes)] for r in range(P)]
+            flat = [q for r in range(P) for q in reqs[r]]
+            for q in flat:
+                q.start(st)
+            pc.run_ranks([(lambda r=r: [q.pbuf_prepare(st) for q in reqs[r]]) for r in range(P)])
+
+            def epoch_rest():
+                pc.preadyall(flat, st) if len(flat) <= 16 else [pc.preadyall(flat[i:i + 16], st)
+                                                                  for i in range(0, len(flat), 16)]
+                for t in range(len(sizes)):
+                    for r in range(P):
+                        reqs[r][t].wait_on_stream(st)
+
+            epoch_rest()
+            torch.cuda.synchronize()
+
+            def epoch():
+                pc.startall(flat, st)
+                pc.pbuf_prepare_all(flat, st)
+                epoch_rest()
+
+            gr = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gr, stream=st):
+                epoch()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            it = 10
+            e0.record(st)
+            for _ in range(it):
+                with torch.cuda.stream(st):
+                    gr.replay()
+            e1.record(st)
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / it
+            total = sum(sizes) * 4
+            errs = [q.error() for q in flat if q.error()[0] != 0]
+            algos = collections.Counter(["auto", "ring", "rd", "direct"][q.info()["algo"]] for q in reqs[0])
+            print(json.dumps({"model": name, "mode": "per-tensor (graph)", "ranks": P, "tensors": len(sizes),
+                              "bytes_per_rank": total, "us_per_step": ms * 1e3,
+                              "busbw_gbs": busbw(total, ms / 1e3, P), "algos": dict(algos), "errors": errs}),
+                  flush=True)
+            for q in flat:
+                q.free()
+        for c in cs:
+            c.destroy()
+        g.destroy()
+
+
 def sweep_p2p(args):
     """C2: vector-add producer + Pready at thread/warp/block granularity with
     aggregation g, INLINE vs ENGINE; goodput = bytes / (kernel + comm) time."""
@@ -197,11 +255,11 @@ def sweep_p2p(args):
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
-    ap.add_argument("what", choices=["allreduce", "dl", "p2p"])
+    ap.add_argument("what", choices=["allreduce", "dl", "dl_tensor", "p2p"])
     ap.add_argument("--ranks", default="8")
     ap.add_argument("--algos", default="ring,rd")
     ap.add_argument("--partitions", default="1,16,64")
     ap.add_argument("--max-bytes", type=int, default=1 << 30)
     ap.add_argument("--graph", action="store_true", help="replay a captured CUDA graph of the epoch")
     a = ap.parse_args()
-    {"allreduce": sweep_allreduce, "dl": sweep_dl, "p2p": sweep_p2p}[a.what](a)
+    {"allreduce": sweep_allreduce, "dl": sweep_dl, "dl_tensor": sweep_dl_per_tensor, "p2p": sweep_p2p}[a.what](a)
