@@ -311,7 +311,7 @@ def jacobi_bench(pc, apps, torch, args):
         P = Py * Px
         g, cs = pc.local_comms(P, 0)
         st = torch.cuda.Stream()
-        js = apps.JacobiSolver(cs, list(range(P)), N, Py, Px, K, H=int(os.environ.get("PC_JACOBI_H", "32")))
+        js = apps.JacobiSolver(cs, list(range(P)), N, Py, Px, K, H=int(os.environ.get("PC_JACOBI_H", "64")))
         for s in js.local:  # perf init: top edge 1.0, rest 0
             s["grid"][0].zero_()
             if s["py"] == 0:

@@ -16,7 +16,7 @@ import re
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIBPC = os.path.join(_HERE, "libpc.so")
-LIBAPPS = os.path.join(_HERE, "libpcapps.so")
+LIBAPPS = os.environ.get("PC_APPS_LIB") or os.path.join(_HERE, "libpcapps.so")
 INCLUDE = os.path.join(os.path.dirname(_HERE), "include")
 
 P = C.c_void_p

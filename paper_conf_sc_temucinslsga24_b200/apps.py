@@ -72,7 +72,7 @@ class JacobiSolver:
     `ranks` are their comm ranks.  One epoch = one solve of `iters` iterations:
     every halo partition is (iteration slot, edge segment), readied once."""
 
-    def __init__(self, comms, ranks, N: int, Py: int, Px: int, iters: int, H: int = 32, device: int = 0):
+    def __init__(self, comms, ranks, N: int, Py: int, Px: int, iters: int, H: int = 64, device: int = 0):
         import torch
         from . import runtime as rt
         self.torch, self.rt = torch, rt

@@ -26,7 +26,13 @@
 namespace {
 
 constexpr int kStrip = 128;  // columns per warp tile (32 lanes x float4)
-constexpr int kRB = 4;       // rows loaded together per batch (tile height H % kRB == 0)
+#ifndef PC_JACOBI_MINB
+#define PC_JACOBI_MINB 4  // 4 CTAs x 8 warps per SM: enough loads in flight for HBM (measured, tools/jacobi_variants.sh)
+#endif
+#ifndef PC_JACOBI_RB
+#define PC_JACOBI_RB 4
+#endif
+constexpr int kRB = PC_JACOBI_RB;  // rows loaded together per batch (tile height H % kRB == 0)
 enum { T = 0, B = 1, L = 2, R = 3 };
 
 struct JacobiRank {
@@ -153,7 +159,7 @@ __device__ void tile_init(const JacobiRank &d, int tile) {
 
 // One launch covers the tiles of `nranks` ranks (all co-located ranks of a
 // process on this GPU, or a single rank): block b -> rank via block_start.
-__global__ void __launch_bounds__(256) jacobi_kernel(const JacobiRank *__restrict__ ranks, const int *block_start,
+__global__ void __launch_bounds__(256, PC_JACOBI_MINB) jacobi_kernel(const JacobiRank *__restrict__ ranks, const int *block_start,
                                                     int nranks, int k, int init) {
   int q = 0;
   while (q + 1 < nranks && (int)blockIdx.x >= block_start[q + 1]) ++q;
