@@ -67,3 +67,12 @@ def test_jacobi_fixed_points():
     lin = (3 * i - 5 * j + 7).astype(np.float32)
     (got,) = solve(lin, 2, 2, 10)
     np.testing.assert_array_equal(got, lin)
+
+
+@pytest.mark.parametrize("H", [4, 64, 128])
+def test_jacobi_tile_heights(H):
+    """The bench runs 64-row tiles; other legal tile heights give the same bits."""
+    N, iters = 512, 20
+    a0 = synth.jacobi_init(N, N, "random")
+    (got,) = solve(a0, 2, 2, iters, H=H)
+    np.testing.assert_array_equal(got, oracle.jacobi_seq(a0, iters))
