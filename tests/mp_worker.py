@@ -56,6 +56,35 @@ assert q.error() == (0, 0), q.error()
 if r == 1:
     res["p2p"] = rb.cpu().numpy()
 q.free()
+# ENGINE-mode p2p 1 -> 0 (library warps push), warp-granularity Pready
+if r == 1:
+    a2 = torch.from_numpy(synth.uniform_f32(synth.BASE_SEED, 1, 0, n)).cuda()
+    c2 = torch.empty(n, device="cuda")
+    q = pc.psend_init(c2, n // 64, 64, pc.FLOAT32, 0, 12, comm)
+else:
+    rb2 = torch.zeros(n, device="cuda")
+    q = pc.precv_init(rb2, n // 64, 64, pc.FLOAT32, 1, 12, comm)
+for e in range(2):
+    q.start(st)
+    q.pbuf_prepare(st)
+    if e == 0:
+        pq = q.prequest_create(pc.GRAN_WARP, 4, pc.COPY_ENGINE)
+    if r == 1:
+        apps.vecadd(a2, a2, c2, n, apps.GRAN_WARP, pq, st)
+    q.wait()
+    assert q.error() == (0, 0), q.error()
+if r == 0:
+    res["p2p_engine"] = rb2.cpu().numpy()
+q.free()
+# Jacobi 2 x 1 across the two processes (one rank each), halos over CUDA IPC
+js = apps.JacobiSolver([comm], [r], 256, 2, 1, 30, H=32)
+js.set_initial(synth.jacobi_init(256, 256, "random"))
+torch.cuda.synchronize()
+js.solve(st)
+torch.cuda.synchronize()
+assert js.errors() == [], js.errors()
+res["jacobi"] = js.result()
+js.free()
 np.savez(os.path.join(out_dir, f"rank{r}.npz"), **res)
 comm.destroy()
 dist.destroy_process_group()

@@ -36,3 +36,9 @@ def test_two_processes_ipc(tmp_path):
                                np.arange(8, dtype=np.int32)[None])
     assert (arr == 1).all()
     np.testing.assert_array_equal(res[1]["p2p"].view(np.uint8), consumed[0])
+    a2 = synth.uniform_f32(synth.BASE_SEED, 1, 0, n)
+    np.testing.assert_array_equal(res[0]["p2p_engine"], (a2 + a2).astype(np.float32))
+    # Jacobi: each process holds its own block; together they equal the oracle
+    ref = oracle.jacobi_seq(synth.jacobi_init(256, 256, "random"), 30)
+    np.testing.assert_array_equal(res[0]["jacobi"][:128], ref[:128])
+    np.testing.assert_array_equal(res[1]["jacobi"][128:], ref[128:])
