@@ -271,9 +271,11 @@ static void choose_slices(int64_t len, int nparts, int target_units, int64_t min
 // ------------------------------------------------------------------ request helpers
 static size_t dtype_size(int dt) { return dt == PC_BYTE ? 1 : 4; }
 
+// Device resources of a request are allocated lazily (first pc_start, or the
+// exchange): MPI_P*_init stays non-blocking and cheap.
 static int alloc_ctrl(Request *q) {
   Comm *c = q->comm;
-  if (c->dry) return 0;
+  if (c->dry || q->ctrl) return 0;
   PC_CUDA(cudaSetDevice(c->device));
   int lo = 0, hi = 0;
   PC_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
@@ -361,7 +363,7 @@ static int p2p_init(int kind, const void *sbuf, void *rbuf, int partitions, size
   q->L.build((size_t)partitions, (size_t)partitions);
   q->agg = 1;
   q->ntransport = partitions;
-  return alloc_ctrl(q);
+  return 0;
 }
 
 // ------------------------------------------------------------------ exchange (first pbuf_prepare)
@@ -400,7 +402,11 @@ static const ReqRec *find_rec(const std::vector<ReqRec> &all, int M, int owner, 
 static int exchange_round(Comm *c, Request *target) {
   std::vector<Request *> pending;
   for (Request *q : c->reqs)
-    if (q && !q->exchanged) pending.push_back(q);
+    if (q && !q->exchanged) {
+      int arc = alloc_ctrl(q);  // exported below
+      if (arc) return arc;
+      pending.push_back(q);
+    }
   int32_t mine = (int32_t)pending.size();
   std::vector<int32_t> counts(c->size);
   int rc = allgather(c, &mine, sizeof(mine), counts.data());
@@ -1023,7 +1029,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   }
   const size_t nflags = (size_t)partitions * (size_t)std::max(q->nsteps, 1) * (size_t)q->slices;
   q->L.build((size_t)partitions, nflags);
-  return alloc_ctrl(q);
+  return 0;
 }
 
 int pc_start(pc_request_t req, pc_stream_t stream) {
@@ -1039,6 +1045,10 @@ int pc_start(pc_request_t req, pc_stream_t stream) {
   q->user_stream = (cudaStream_t)stream;
   if (c->dry) return 0;
   PC_CUDA(cudaSetDevice(c->device));
+  if (!q->ctrl) {
+    int arc = alloc_ctrl(q);
+    if (arc) return arc;
+  }
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
   PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
   if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
@@ -1111,6 +1121,11 @@ int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream) {
     q->prepared_this_epoch = false;
     q->user_stream = (cudaStream_t)stream;
     if (q->comm->dry) continue;
+    if (!q->ctrl) {
+      PC_CUDA(cudaSetDevice(q->comm->device));
+      int arc = alloc_ctrl(q);
+      if (arc) return arc;
+    }
     a.epoch[a.n] = q->ctrl + q->L.epoch;
     a.dst[a.n] = nullptr;
     if (++a.n == kMaxCtl) {
