@@ -752,7 +752,15 @@ static int group_register(Request *q, bool block, bool *launched) {
     g.launched = true;
     g.cv.notify_all();
   }
-  if (block) g.cv.wait(lk, [&] { return g.launched || g.epoch != q->epoch; });
+  if (block && !g.cv.wait_for(lk, std::chrono::milliseconds(q->comm->timeout_ms ? q->comm->timeout_ms : 3600000),
+                              [&] { return g.launched || g.epoch != q->epoch; })) {
+    fprintf(stderr,
+            "[pc] rank %d: pc_wait timed out waiting for the other co-located ranks' waits (every rank sharing this "
+            "GPU in this process must call pc_wait/pc_wait_on_stream for the epoch; use one thread per rank or "
+            "pc_wait_on_stream)\n",
+            q->comm->rank);
+    return PC_ERR_TIMEOUT;
+  }
   *launched = g.launched && g.epoch == q->epoch;
   if (*launched) q->engine_launched = true;
   return 0;
