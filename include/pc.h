@@ -38,7 +38,10 @@ typedef struct pc_local_group_s *pc_local_group_t; /* in-process rank group (vir
 typedef struct pc_prequest_s pc_prequest_t;     /* POD device request, passed BY VALUE to kernels
                                                    (MPIX_Prequest); layout in pc_device.cuh */
 
-typedef enum { PC_INT32 = 0, PC_FLOAT32 = 1, PC_BYTE = 2 } pc_dtype_t;
+/* Element types.  BF16: bfloat16 bits (upper half of an fp32); every reduction
+ * step is one correctly rounded bf16 op (R27).  FLOAT64/BF16 are
+ * accepted by pc_pallreduce_init; p2p requests take any type (bytes moved). */
+typedef enum { PC_INT32 = 0, PC_FLOAT32 = 1, PC_BYTE = 2, PC_FLOAT64 = 3, PC_BF16 = 4 } pc_dtype_t;
 typedef enum { PC_OP_SUM = 0, PC_OP_MAX = 1, PC_OP_MIN = 2 } pc_op_t;
 /* Granularity of the device Pready call: informational — the device
  * function chosen (pc_pready / _warp / _block) decides who participates. */
@@ -108,8 +111,8 @@ int pc_precv_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, int
                   pc_comm_t comm, pc_request_t *req);
 /* Partitioned allreduce (MPIX_Pallreduce_init; schedule S of
  * P:L153-L155).  Collective: every rank calls it with identical arguments in
- * the same order.  sendbuf == recvbuf (in place) is allowed.  dtype INT32 or
- * FLOAT32; op SUM/MAX/MIN. */
+ * the same order.  sendbuf == recvbuf (in place) is allowed.  dtype INT32,
+ * FLOAT32, FLOAT64 or BF16; op SUM/MAX/MIN. */
 int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
                        pc_op_t op, pc_algo_t algo, pc_comm_t comm, pc_request_t *req);
 
@@ -170,7 +173,8 @@ int pc_schedule_ring(int P, int r, int32_t *out_rows5);
 /* Recursive-doubling schedule: rows (I, R=-1, op=1, O, A=-1); log2 P steps. */
 int pc_schedule_rd(int P, int r, int32_t *out_rows5);
 /* Chunk bounds of a partition of L elements split in P chunks (reading R4):
- * out[c] = first element of chunk c, out[P] = L. */
+ * out[c] = first element of chunk c, out[P] = L.  Quantum 4 elements, i.e.
+ * 32-bit types; for fp64 / bf16 requests the quantum is 2 / 8 (R27). */
 int pc_chunk_bounds(int64_t L, int P, int64_t *out);
 /* Request facts after the first pbuf_prepare: algo actually used, slices per
  * chunk, slice elements, engine warps. */

@@ -11,6 +11,7 @@ Functions (numpy in, numpy out):
   allreduce_def_i32(...)  O2  plain definition, int32 (sum wraps, max, min)
   allreduce_def_f64(...)  O2  plain definition, fp32 inputs summed in fp64
   pallreduce(...)         O3/O4/O6  Alg 1 (ring), RD or DIRECT schedule + Alg 2, P threads
+  bf16_round / bf16_op    R27 bf16 arithmetic (bit patterns as uint16)
   alg1_table(P, r)        Alg 1 step tuples
   ring_fold_f32 / rd_tree_f32   closed forms of O3 / O4 (pinned against them)
   jacobi_seq / jacobi_decomp    O5
@@ -27,7 +28,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
-INT32, FLOAT32 = 0, 1
+INT32, FLOAT32, FLOAT64, BF16 = 0, 1, 3, 4  # bf16 arrays are carried as uint16 bit patterns
 SUM, MAX, MIN = 0, 1, 2
 RING, RD, DIRECT = 1, 2, 3
 
@@ -52,6 +53,8 @@ def lib():
         _lib.orc_pallreduce.argtypes = [i32, i32, i32, i64, i32, i32, i32, i32, P, P, P, u64, P, P]
         _lib.orc_pallreduce_direct.argtypes = [i32, i32, i64, i32, i32, i32, i32, P, P, P, u64, P, P]
         _lib.orc_alg1_table.argtypes = [i32, i32, P]
+        _lib.orc_bf16_round.argtypes = [i64, P, P]
+        _lib.orc_bf16_op.argtypes = [i32, i64, P, P, P]
         _lib.orc_ring_fold_f32.argtypes = [i32, i64, P, P, P]
         _lib.orc_rd_tree_f32.argtypes = [i32, i64, P, P]
         _lib.orc_jacobi_seq.argtypes = [i32, i32, i32, P, P]
@@ -120,7 +123,8 @@ def n_steps(algo: int, P: int) -> int:
 
 def pallreduce(x: np.ndarray, partitions: int, algo: int = RING, op: int = SUM, inplace: bool = False,
                orders: np.ndarray | None = None, jitter_seed: int = 1):
-    """x: (epochs, P, Np*L) int32 or float32 (or (P, Np*L) for one epoch).
+    """x: (epochs, P, Np*L) int32, float32, float64 or uint16 (= bf16 bit
+    patterns, reading R27) (or (P, Np*L) for one epoch).
 
     Returns (y, reduces, arrivals): y has x's shape and holds each rank's recvbuf
     after its MPI_Wait; reduces/arrivals are (P, Np, max(nsteps,1)) counts from
@@ -128,7 +132,7 @@ def pallreduce(x: np.ndarray, partitions: int, algo: int = RING, op: int = SUM, 
     squeeze = x.ndim == 2
     if squeeze:
         x = x[None]
-    dtype = INT32 if x.dtype == np.int32 else FLOAT32
+    dtype = _DTYPES[x.dtype.type]
     x = np.ascontiguousarray(x)
     epochs, P, n = x.shape
     assert n % partitions == 0
@@ -147,6 +151,31 @@ def pallreduce(x: np.ndarray, partitions: int, algo: int = RING, op: int = SUM, 
         _check(lib().orc_pallreduce(algo, P, partitions, L, dtype, op, epochs, int(inplace), _p(x), _p(y),
                                     _p(orders), jitter_seed, _p(red), _p(arr)), "orc_pallreduce")
     return (y[0] if squeeze else y), red, arr
+
+
+_DTYPES = {np.int32: INT32, np.float32: FLOAT32, np.float64: FLOAT64, np.uint16: BF16}
+
+
+def bf16_round(x: np.ndarray) -> np.ndarray:
+    """float64 values -> nearest bf16 (ties to even), as uint16 bit patterns (R27)."""
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    out = np.zeros(x.shape, dtype=np.uint16)
+    _check(lib().orc_bf16_round(x.size, _p(x), _p(out)), "bf16_round")
+    return out
+
+
+def bf16_op(a: np.ndarray, b: np.ndarray, op: int = SUM) -> np.ndarray:
+    """Elementwise a (+) b of bf16 bit patterns (uint16), correctly rounded (R27)."""
+    a = np.ascontiguousarray(a, dtype=np.uint16)
+    b = np.ascontiguousarray(b, dtype=np.uint16)
+    out = np.zeros(a.shape, dtype=np.uint16)
+    _check(lib().orc_bf16_op(op, a.size, _p(a), _p(b), _p(out)), "bf16_op")
+    return out
+
+
+def bf16_to_f64(b: np.ndarray) -> np.ndarray:
+    """Exact decode of bf16 bit patterns (the upper half of an fp32)."""
+    return (np.asarray(b, dtype=np.uint16).astype(np.uint32) << 16).view(np.float32).astype(np.float64)
 
 
 def alg1_table(P: int, r: int) -> np.ndarray:
@@ -173,10 +202,11 @@ def rd_tree_f32(x: np.ndarray) -> np.ndarray:
     return out
 
 
-def chunk_ids(L: int, P: int, partitions: int) -> np.ndarray:
+def chunk_ids(L: int, P: int, partitions: int, esize: int = 4) -> np.ndarray:
     """Chunk id of every element of an (Np*L) buffer under reading R4
-    (q = ceil(L/(4P))*4 elements per chunk)."""
-    q = -(-L // (4 * P)) * 4 if L > 0 else 4
+    (q = ceil(L/(vP))*v elements per chunk, v = 16/esize)."""
+    v = 16 // esize
+    q = -(-L // (v * P)) * v if L > 0 else v
     j = np.arange(L)
     c = np.minimum(j // max(q, 1), P - 1).astype(np.int32)
     return np.tile(c, partitions)

@@ -38,7 +38,7 @@
 extern "C" {
 
 enum { ORC_OK = 0, ORC_ERR_ARG = -1, ORC_ERR_TIMEOUT = -5 };
-enum { ORC_INT32 = 0, ORC_FLOAT32 = 1 };
+enum { ORC_INT32 = 0, ORC_FLOAT32 = 1, ORC_FLOAT64 = 3, ORC_BF16 = 4 };
 enum { ORC_SUM = 0, ORC_MAX = 1, ORC_MIN = 2 };
 
 }  // extern "C"
@@ -98,12 +98,74 @@ inline float op_f32(int op, float local, float incoming) {
   }
 }
 
+// fp64 (R27): one IEEE binary64 add, round-to-nearest-even.
+inline double op_f64(int op, double local, double incoming) {
+  switch (op) {
+    case ORC_SUM: {
+      volatile double r = local + incoming;
+      return r;
+    }
+    case ORC_MAX: return std::fmax(local, incoming);
+    default:      return std::fmin(local, incoming);
+  }
+}
+
+// bf16 (R27): a bf16 value is the top 16 bits of an IEEE binary32 (1-8-7).
+// local ⊕ incoming = the bf16 nearest (ties to even) to the EXACT result, i.e.
+// the correctly rounded bf16 operation.  Written out here from the definition:
+// decode both operands exactly, add in binary64, round the binary64 value to
+// 8 significant bits.  (The binary64 add is itself exact or double-rounding-
+// innocuous: 53 >= 2*8+2, Figueroa's theorem.)
+inline double bf16_decode(uint16_t b) {
+  uint32_t u = (uint32_t)b << 16;
+  float f;
+  std::memcpy(&f, &u, 4);
+  return (double)f;
+}
+inline uint16_t bf16_round(double v) {
+  if (std::isnan(v)) return (uint16_t)(std::signbit(v) ? 0xFFC0 : 0x7FC0);
+  const uint16_t sign = std::signbit(v) ? 0x8000 : 0;
+  double a = std::fabs(v);
+  if (a == 0.0) return sign;
+  if (std::isinf(a)) return (uint16_t)(sign | 0x7F80);
+  int E;
+  std::frexp(a, &E);                           // a = m 2^E, m in [0.5, 1): leading bit 2^(E-1)
+  const int ulp_exp = std::max(E - 8, -133);   // 8 significant bits; bf16 subnormal quantum 2^-133
+  double r = std::nearbyint(std::ldexp(a, -ulp_exp));  // FE_TONEAREST: ties to even
+  r = std::ldexp(r, ulp_exp);
+  if (r >= std::ldexp(1.0, 128)) return (uint16_t)(sign | 0x7F80);  // overflow -> inf
+  float f = (float)r;                          // exact: r has <= 8 significant bits in range
+  uint32_t u;
+  std::memcpy(&u, &f, 4);
+  return (uint16_t)(sign | (u >> 16));
+}
+inline uint16_t op_bf16(int op, uint16_t local, uint16_t incoming) {
+  const double a = bf16_decode(local), b = bf16_decode(incoming);
+  switch (op) {
+    case ORC_SUM: return bf16_round(a + b);
+    case ORC_MAX: return bf16_round(std::fmax(a, b));
+    default:      return bf16_round(std::fmin(a, b));
+  }
+}
+
+int64_t esize_of(int dtype) { return dtype == ORC_FLOAT64 ? 8 : dtype == ORC_BF16 ? 2 : 4; }
+
 void reduce_into(int dtype, int op, void *dst, const void *local, const void *incoming, int64_t n) {
   if (dtype == ORC_INT32) {
     auto d = (int32_t *)dst;
     auto a = (const int32_t *)local;
     auto b = (const int32_t *)incoming;
     for (int64_t k = 0; k < n; ++k) d[k] = op_i32(op, a[k], b[k]);
+  } else if (dtype == ORC_FLOAT64) {
+    auto d = (double *)dst;
+    auto a = (const double *)local;
+    auto b = (const double *)incoming;
+    for (int64_t k = 0; k < n; ++k) d[k] = op_f64(op, a[k], b[k]);
+  } else if (dtype == ORC_BF16) {
+    auto d = (uint16_t *)dst;
+    auto a = (const uint16_t *)local;
+    auto b = (const uint16_t *)incoming;
+    for (int64_t k = 0; k < n; ++k) d[k] = op_bf16(op, a[k], b[k]);
   } else {
     auto d = (float *)dst;
     auto a = (const float *)local;
@@ -301,12 +363,14 @@ int orc_pallreduce(int algo, int P, int Np, int64_t L, int dtype, int op, int ep
                    uint32_t *reduces, uint32_t *arrivals) {
   if (P < 1 || Np < 1 || L < 0 || epochs < 1 || (algo != 1 && algo != 2)) return ORC_ERR_ARG;
   if (algo == 2 && (P & (P - 1))) return ORC_ERR_ARG;
-  const int64_t esz = 4;
+  const int64_t esz = esize_of(dtype);
   const int64_t part_bytes = L * esz;
   const int64_t nbytes = (int64_t)Np * part_bytes;
-  // R4: chunking of a partition of L elements into P chunks: q = ceil(L/(4P))*4
-  // elements (16-byte multiple); chunk c = [c q, min((c+1) q, L)), possibly empty.
-  const int64_t q = ((L + 4 * P - 1) / (4 * P)) * 4;
+  // R4: chunking of a partition of L elements into P chunks: q = ceil(L/(vP))*v
+  // elements with v = 16/esz (q elements are a 16-byte multiple); chunk
+  // c = [c q, min((c+1) q, L)), possibly empty.
+  const int64_t v = 16 / esz;
+  const int64_t q = ((L + v * P - 1) / (v * P)) * v;
   auto chunk_lo = [&](int c) { return std::min<int64_t>((int64_t)c * q, L); };
   auto chunk_n = [&](int c) { return std::min<int64_t>((int64_t)(c + 1) * q, L) - chunk_lo(c); };
   int nsteps_rd = 0;
@@ -474,6 +538,17 @@ int orc_pallreduce(int algo, int P, int Np, int64_t L, int dtype, int op, int ep
   return failed ? ORC_ERR_TIMEOUT : ORC_OK;
 }
 
+// bf16 arithmetic of R27, exported so tests can pin it (round-to-nearest-even
+// of binary64 values to bf16 bit patterns; the ⊕ of two bf16 operands).
+int orc_bf16_round(int64_t n, const double *x, uint16_t *out) {
+  for (int64_t k = 0; k < n; ++k) out[k] = bf16_round(x[k]);
+  return ORC_OK;
+}
+int orc_bf16_op(int op, int64_t n, const uint16_t *a, const uint16_t *b, uint16_t *out) {
+  for (int64_t k = 0; k < n; ++k) out[k] = op_bf16(op, a[k], b[k]);
+  return ORC_OK;
+}
+
 // ===========================================================================
 // O6: partitioned allreduce over the DIRECT two-step schedule (
 // the generic schedule of P:L151-L155 with neighbour SETS, progressed by Alg 2
@@ -491,8 +566,9 @@ int orc_pallreduce_direct(int P, int Np, int64_t L, int dtype, int op, int epoch
                           void *y, const int32_t *orders, uint64_t jitter_seed, uint32_t *reduces,
                           uint32_t *arrivals) {
   if (P < 1 || Np < 1 || L < 0 || epochs < 1) return ORC_ERR_ARG;
-  const int64_t esz = 4, part_bytes = L * esz, nbytes = (int64_t)Np * part_bytes;
-  const int64_t q = ((L + 4 * P - 1) / (4 * P)) * 4;  // R4
+  const int64_t esz = esize_of(dtype), part_bytes = L * esz, nbytes = (int64_t)Np * part_bytes;
+  const int64_t v = 16 / esz;
+  const int64_t q = ((L + v * P - 1) / (v * P)) * v;  // R4
   auto chunk_lo = [&](int c) { return std::min<int64_t>((int64_t)c * q, L); };
   auto chunk_n = [&](int c) { return std::min<int64_t>((int64_t)(c + 1) * q, L) - chunk_lo(c); };
   struct Rk {

@@ -231,17 +231,18 @@ static int rd_rows(int P, int r, int32_t *out) {
 
 // Reading R4: q = ceil(L / (4P)) * 4 elements per chunk (16-byte multiples);
 // trailing chunks may be short or empty.
-static int64_t chunk_q(int64_t L, int P) { return ((L + 4LL * P - 1) / (4LL * P)) * 4; }
+// epv: elements per 16-byte vector (4 for 32-bit types, 2 for fp64, 8 for bf16)
+static int64_t chunk_q(int64_t L, int P, int64_t epv = 4) { return ((L + epv * P - 1) / (epv * P)) * epv; }
 
 // Slicing policy (deterministic from arguments every rank shares): split a
 // length of `len` elements into ns slices of qs elements (multiple of 4), with
 // about `target_units / nparts` slices per part but none below min_elems.
 static void choose_slices(int64_t len, int nparts, int target_units, int64_t min_elems, int *ns_out,
-                          int64_t *qs_out) {
+                          int64_t *qs_out, int64_t epv = 4) {
   long fixed = env_long("PC_SLICE_BYTES", 0);
   int64_t qs;
   if (fixed > 0) {
-    qs = std::max<int64_t>(4, (fixed / 4 + 3) / 4 * 4);
+    qs = std::max<int64_t>(epv, (fixed / (16 / epv) + epv - 1) / epv * epv);
   } else {
     // Balance: with W = target_units warps taking units in turn, the engine
     // time is ~ ceil(nparts*ns / W) slices of len/ns elements each; pick the
@@ -261,7 +262,7 @@ static void choose_slices(int64_t len, int nparts, int target_units, int64_t min
       }
     }
     qs = (len + best - 1) / best;
-    qs = std::max<int64_t>(4, (qs + 3) / 4 * 4);
+    qs = std::max<int64_t>(epv, (qs + epv - 1) / epv * epv);
   }
   int64_t ns = len > 0 ? (len + qs - 1) / qs : 1;
   *ns_out = (int)std::max<int64_t>(1, ns);
@@ -269,7 +270,7 @@ static void choose_slices(int64_t len, int nparts, int target_units, int64_t min
 }
 
 // ------------------------------------------------------------------ request helpers
-static size_t dtype_size(int dt) { return dt == PC_BYTE ? 1 : 4; }
+static size_t dtype_size(int dt) { return dt == PC_BYTE ? 1 : dt == PC_FLOAT64 ? 8 : dt == PC_BF16 ? 2 : 4; }
 
 // Device resources of a request are allocated lazily (first pc_start, or the
 // exchange): MPI_P*_init stays non-blocking and cheap.
@@ -342,7 +343,7 @@ static int new_request(Comm *c, int kind, pc_request_t *out, Request **rq) {
 
 static int p2p_init(int kind, const void *sbuf, void *rbuf, int partitions, size_t count, int dtype, int peer,
                     int tag, Comm *c, pc_request_t *out) {
-  if (!c || !out || partitions < 1 || dtype < 0 || dtype > 2 || peer < 0 || peer >= c->size || tag < 0)
+  if (!c || !out || partitions < 1 || dtype < 0 || dtype > 4 || peer < 0 || peer >= c->size || tag < 0)
     return PC_ERR_ARG;
   const uint64_t bytes = (uint64_t)partitions * count * dtype_size(dtype);
   if (!c->dry && check_buf(kind == PC_KIND_PSEND ? sbuf : rbuf, bytes)) return PC_ERR_ARG;
@@ -600,7 +601,7 @@ static RdArgs make_rd_args(Request *q) {
   a.ready = q->ctrl + q->L.ready;
   a.rtr = q->ctrl + q->L.rtr;
   a.done = q->ctrl + q->L.donecnt;
-  const int64_t slot_bytes = (int64_t)q->partitions * (int64_t)q->count * 4;
+  const int64_t slot_bytes = (int64_t)q->partitions * (int64_t)q->count * (int64_t)q->esize;
   for (int k = 0; k < q->nsteps; ++k) {
     a.p_staging[k] = q->nb_stage[k] + (int64_t)k * slot_bytes;
     a.p_flags[k] = q->nb_ctrl[k] + q->L.flags;
@@ -625,7 +626,7 @@ static DirectArgs make_direct_args(Request *q) {
   a.L = (int64_t)q->count;
   a.q = q->chunk_elems;
   a.qs = q->slice_elems;
-  a.sq = q->chunk_elems + 4;
+  a.sq = q->chunk_elems + 16 / (int64_t)q->esize;
   a.sendbuf = (const uint8_t *)q->sbuf;
   a.recvbuf = (uint8_t *)q->rbuf;
   a.staging = q->staging;
@@ -971,11 +972,14 @@ int pc_precv_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, int
 int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
                        pc_op_t op, pc_algo_t algo, pc_comm_t comm, pc_request_t *req) {
   Comm *c = (Comm *)comm;
-  if (!c || !req || partitions < 1 || (dtype != PC_INT32 && dtype != PC_FLOAT32) || op < 0 || op > 2 ||
+  if (!c || !req || partitions < 1 ||
+      (dtype != PC_INT32 && dtype != PC_FLOAT32 && dtype != PC_FLOAT64 && dtype != PC_BF16) || op < 0 || op > 2 ||
       algo < 0 || algo > 3)
     return PC_ERR_ARG;
   const int P = c->size;
-  const uint64_t bytes = (uint64_t)partitions * count * 4;
+  const size_t esz = dtype_size(dtype);
+  const int64_t epv = 16 / (int64_t)esz;
+  const uint64_t bytes = (uint64_t)partitions * count * esz;
   if (!c->dry && (check_buf(sendbuf, bytes) || check_buf(recvbuf, bytes))) return PC_ERR_ARG;
   int a = algo;
   const bool pow2 = log2_exact(P) >= 0;
@@ -1005,34 +1009,34 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   q->op = op;
   q->algo_req = algo;
   q->algo = a;
-  q->esize = 4;
+  q->esize = esz;
   q->peer = -1;
   q->tag = 0;
-  q->part_bytes = count * 4;
+  q->part_bytes = count * esz;
   q->total_bytes = bytes;
   q->seq = c->allreduce_seq++;
   q->agg = 1;
   q->ntransport = partitions;
   q->engine_warps = c->engine_warps;
   const int64_t L = (int64_t)count;
-  const int64_t min_elems = env_long("PC_MIN_SLICE_BYTES", 8192) / 4;
+  const int64_t min_elems = env_long("PC_MIN_SLICE_BYTES", 8192) / (int64_t)esz;
   // units (partition slices) per engine warp: each warp sweeps its units
   // round-robin (Alg 2), so a few per warp absorb upstream skew
   const int upw = (int)std::max(1L, std::min(8L, env_long("PC_UNITS_PER_WARP", 1)));
   if (a == PC_ALGO_RING) {
     q->nsteps = 2 * (P - 1);
-    q->chunk_elems = chunk_q(L, P);
-    choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems);
+    q->chunk_elems = chunk_q(L, P, epv);
+    choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems, epv);
     q->staging_bytes = P > 1 ? bytes : 0;
   } else if (a == PC_ALGO_DIRECT) {
     q->nsteps = 2;  // phase counters [u][0..1][slice]
-    q->chunk_elems = chunk_q(L, P);
-    choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems);
-    q->staging_bytes = P > 1 ? (uint64_t)partitions * P * (q->chunk_elems + 4) * 4 : 0;
+    q->chunk_elems = chunk_q(L, P, epv);
+    choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems, epv);
+    q->staging_bytes = P > 1 ? (uint64_t)partitions * P * (q->chunk_elems + epv) * esz : 0;
   } else {
     q->nsteps = log2_exact(P);
     q->chunk_elems = L;
-    choose_slices(L, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems);
+    choose_slices(L, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems, epv);
     q->staging_bytes = bytes * (uint64_t)q->nsteps;
   }
   const size_t nflags = (size_t)partitions * (size_t)std::max(q->nsteps, 1) * (size_t)q->slices;

@@ -18,6 +18,7 @@
 // with W identical on every rank (agreed at comm creation), so the dependency
 // (unit x, step i) at rank r -> (unit x, step i-1) at rank r-1 can never form a
 // cycle while all engine warps are resident.
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
 #include <atomic>
@@ -100,16 +101,40 @@ struct Op<1, OP> {  // fp32: one IEEE add, round to nearest even, no contraction
   }
 };
 
+template <int OP>
+struct Op<3, OP> {  // fp64 (the paper's `double` buffers)
+  using T = double;
+  static __device__ __forceinline__ double f(double a, double b) {
+    if (OP == 0) return __dadd_rn(a, b);
+    if (OP == 1) return fmax(a, b);
+    return fmin(a, b);
+  }
+};
+template <int OP>
+struct Op<4, OP> {  // bf16 storage (uint16 bits); each op is one correctly rounded bf16 result:
+  using T = uint16_t;  // a + b of two bf16 values is exact in fp32 or the small one is below half an ulp
+  static __device__ __forceinline__ float up(uint16_t v) { return __uint_as_float((uint32_t)v << 16); }
+  static __device__ __forceinline__ uint16_t dn(float f) {
+    return __bfloat16_as_ushort(__float2bfloat16_rn(f));
+  }
+  static __device__ __forceinline__ uint16_t f(uint16_t a, uint16_t b) {
+    if (OP == 0) return dn(__fadd_rn(up(a), up(b)));
+    if (OP == 1) return dn(fmaxf(up(a), up(b)));
+    return dn(fminf(up(a), up(b)));
+  }
+};
+
 template <int DT, int OP>
 __device__ __forceinline__ uint4 vop(uint4 a, uint4 b) {
   using O = Op<DT, OP>;
   using T = typename O::T;
+  constexpr int EPV = 16 / sizeof(T);
   uint4 r;
   T *ra = reinterpret_cast<T *>(&r);
   const T *pa = reinterpret_cast<const T *>(&a);
   const T *pb = reinterpret_cast<const T *>(&b);
 #pragma unroll
-  for (int j = 0; j < 4; ++j) ra[j] = O::f(pa[j], pb[j]);
+  for (int j = 0; j < EPV; ++j) ra[j] = O::f(pa[j], pb[j]);
   return r;
 }
 
@@ -129,11 +154,12 @@ __device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *
   const T *b = reinterpret_cast<const T *>(incoming);
   T *o1 = reinterpret_cast<T *>(out1);
   T *o2 = reinterpret_cast<T *>(out2);
+  constexpr int64_t EPV = 16 / sizeof(T);
   const uintptr_t m = reinterpret_cast<uintptr_t>(out1) & 15;
   const bool same = ((reinterpret_cast<uintptr_t>(local) & 15) == m) &&
                     ((reinterpret_cast<uintptr_t>(incoming) & 15) == m) &&
-                    (!out2 || (reinterpret_cast<uintptr_t>(out2) & 15) == m) && (m & 3) == 0;
-  int64_t head = same ? (int64_t)(((16 - m) & 15) >> 2) : n;
+                    (!out2 || (reinterpret_cast<uintptr_t>(out2) & 15) == m) && (m % sizeof(T)) == 0;
+  int64_t head = same ? (int64_t)(((16 - m) & 15) / sizeof(T)) : n;
   if (head > n) head = n;
   for (int64_t k = lane; k < head; k += 32) {
     const T r = O::f(__ldcg(a + k), __ldcg(b + k));
@@ -142,7 +168,7 @@ __device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *
   }
   int64_t done = head;
   if (same && n > head) {
-    const int64_t nv = (n - head) >> 2;
+    const int64_t nv = (n - head) / EPV;
     const uint4 *av = reinterpret_cast<const uint4 *>(a + head);
     const uint4 *bv = reinterpret_cast<const uint4 *>(b + head);
     uint4 *o1v = reinterpret_cast<uint4 *>(o1 + head);
@@ -166,7 +192,7 @@ __device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *
       o1v[k] = r;
       if (o2v) o2v[k] = r;
     }
-    done = head + (nv << 2);
+    done = head + nv * EPV;
   }
   for (int64_t k = done + lane; k < n; k += 32) {
     const T r = O::f(__ldcg(a + k), __ldcg(b + k));
@@ -264,7 +290,7 @@ struct Idle {
 template <int DT, int OP>
 __device__ __forceinline__ void ring_step(const RingArgs &a, int u, int s, int i, uint32_t e) {
   const int P = a.P, r = a.r, NS = 2 * (P - 1);
-  const int64_t es = 4;
+  const int64_t es = sizeof(typename Op<DT, OP>::T);
   const int64_t base = (int64_t)u * a.L;
   const int64_t fbase = (int64_t)u * NS * a.ns + s;  // flag (u, i, s) = fbase + i * ns
   const int c = modp(r - i, P);                     // R_i = A_{i-1}
@@ -289,7 +315,7 @@ template <int DT, int OP>
 __device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const int W) {
   const int P = a.P, NS = 2 * (P - 1);
   const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
-  const int64_t es = 4;
+  const int64_t es = sizeof(typename Op<DT, OP>::T);
   if (gw >= a.nunits) return;
   if (P == 1) {
     for (int x = gw; x < a.nunits; x += W) {
@@ -352,7 +378,7 @@ template <int DT, int OP>
 __device__ __forceinline__ void rd_body(const RdArgs &a, const int gw, const int W) {
   const int NS = a.nsteps;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
-  const int64_t es = 4;
+  const int64_t es = sizeof(typename Op<DT, OP>::T);
   const int64_t stride = (int64_t)a.Np * a.L * es;  // bytes per staging slot
   uint32_t rtr_ok = 0;
   for (int x = gw; x < a.nunits; x += W) {
@@ -420,8 +446,9 @@ __device__ __forceinline__ void warp_fold_direct(void *out_local, uint8_t *const
   using O = Op<DT, OP>;
   using T = typename O::T;
   const uint32_t lane = threadIdx.x & 31;
+  constexpr int64_t EPV = 16 / sizeof(T);
   const uintptr_t m = reinterpret_cast<uintptr_t>(out_local) & 15;
-  int64_t head = (int64_t)(((16 - m) & 15) >> 2);
+  int64_t head = (int64_t)(((16 - m) & 15) / sizeof(T));
   if (head > n) head = n;
   auto scalar = [&](int64_t k) {
     T acc = __ldcg(reinterpret_cast<const T *>(src[0]) + k);
@@ -430,23 +457,23 @@ __device__ __forceinline__ void warp_fold_direct(void *out_local, uint8_t *const
     for (int j = 0; j < P - 1; ++j) reinterpret_cast<T *>(out_peer[j])[k] = acc;
   };
   for (int64_t k = lane; k < head; k += 32) scalar(k);
-  const int64_t nv = (n - head) >> 2;
+  const int64_t nv = (n - head) / EPV;
   for (int64_t k = lane; k < nv; k += 32) {
-    const int64_t eo = head + 4 * k;  // element offset
+    const int64_t eo = head + EPV * k;  // element offset
     uint4 acc = __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(src[0]) + eo));
     for (int j = 1; j < P; ++j)
       acc = vop<DT, OP>(acc, __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(src[j]) + eo)));
     *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(out_local) + eo) = acc;
     for (int j = 0; j < P - 1; ++j) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(out_peer[j]) + eo) = acc;
   }
-  for (int64_t k = head + (nv << 2) + lane; k < n; k += 32) scalar(k);
+  for (int64_t k = head + nv * EPV + lane; k < n; k += 32) scalar(k);
 }
 
 template <int DT, int OP>
 __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W) {
   const int P = a.P, r = a.r;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;
-  const int64_t es = 4;
+  const int64_t es = sizeof(typename Op<DT, OP>::T);
   if (gw >= a.nunits) return;
   if (P == 1) {
     for (int x = gw; x < a.nunits; x += W) {
@@ -485,7 +512,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
         if (!warp_poll(dep, i == 0 ? e : target, i != 0 && a.sys)) continue;
         progressed = true;
         const int64_t base = (int64_t)u * a.L;
-        const int64_t mis = base & 3;  // the buffers' misalignment in elements (staging mirrors it)
+        const int64_t mis = base % (16 / es);  // the buffers' misalignment in elements (staging mirrors it)
         if (i == 0) {
           for (int j = 0; j < P - 1; ++j) {
             const int o = (r + 1 + j) % P;
@@ -694,14 +721,21 @@ __global__ void pready_range_kernel(pc_prequest_t q, int lo, int hi) {
 
 template <typename F>
 int dispatch(int dtype, int op, F f) {
-  if (dtype == PC_INT32) {
-    if (op == PC_OP_SUM) return f(std::integral_constant<int, 0>(), std::integral_constant<int, 0>());
-    if (op == PC_OP_MAX) return f(std::integral_constant<int, 0>(), std::integral_constant<int, 1>());
-    return f(std::integral_constant<int, 0>(), std::integral_constant<int, 2>());
+  using std::integral_constant;
+#define PC_DISPATCH_OPS(DTV)                                                            \
+  do {                                                                                  \
+    if (op == PC_OP_SUM) return f(integral_constant<int, DTV>(), integral_constant<int, 0>()); \
+    if (op == PC_OP_MAX) return f(integral_constant<int, DTV>(), integral_constant<int, 1>()); \
+    return f(integral_constant<int, DTV>(), integral_constant<int, 2>());               \
+  } while (0)
+  switch (dtype) {
+    case PC_INT32: PC_DISPATCH_OPS(0);
+    case PC_FLOAT32: PC_DISPATCH_OPS(1);
+    case PC_FLOAT64: PC_DISPATCH_OPS(3);
+    case PC_BF16: PC_DISPATCH_OPS(4);
+    default: return PC_ERR_ARG;
   }
-  if (op == PC_OP_SUM) return f(std::integral_constant<int, 1>(), std::integral_constant<int, 0>());
-  if (op == PC_OP_MAX) return f(std::integral_constant<int, 1>(), std::integral_constant<int, 1>());
-  return f(std::integral_constant<int, 1>(), std::integral_constant<int, 2>());
+#undef PC_DISPATCH_OPS
 }
 
 std::atomic<uint64_t> g_launches{0};

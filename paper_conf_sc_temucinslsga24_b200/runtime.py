@@ -15,7 +15,8 @@ from typing import Callable, Sequence
 
 from . import _lib
 
-INT32, FLOAT32, BYTE = 0, 1, 2
+INT32, FLOAT32, BYTE, FLOAT64, BF16 = 0, 1, 2, 3, 4
+ESIZE = {INT32: 4, FLOAT32: 4, BYTE: 1, FLOAT64: 8, BF16: 2}
 SUM, MAX, MIN = 0, 1, 2
 GRAN_THREAD, GRAN_WARP, GRAN_BLOCK = 0, 1, 2
 COPY_INLINE, COPY_ENGINE = 0, 1
@@ -64,6 +65,10 @@ def _dtype_code(t) -> int:
         return INT32
     if t.dtype == torch.uint8:
         return BYTE
+    if t.dtype == torch.float64:
+        return FLOAT64
+    if t.dtype == torch.bfloat16:
+        return BF16
     raise TypeError(f"unsupported dtype {t.dtype}")
 
 
@@ -315,7 +320,7 @@ def psend_init(buf, partitions: int, count: int, dtype: int, dest: int, tag: int
     h = C.c_void_p()
     check(_lib.pc().pc_psend_init(_ptr(buf), partitions, count, dtype, dest, tag, comm.handle, C.byref(h)),
           "pc_psend_init")
-    es = 1 if dtype == BYTE else 4
+    es = ESIZE[dtype]
     return Request(comm, h.value, KIND_PSEND, partitions * count * es, partitions)
 
 
@@ -323,7 +328,7 @@ def precv_init(buf, partitions: int, count: int, dtype: int, source: int, tag: i
     h = C.c_void_p()
     check(_lib.pc().pc_precv_init(_ptr(buf), partitions, count, dtype, source, tag, comm.handle, C.byref(h)),
           "pc_precv_init")
-    es = 1 if dtype == BYTE else 4
+    es = ESIZE[dtype]
     return Request(comm, h.value, KIND_PRECV, partitions * count * es, partitions)
 
 
@@ -332,7 +337,7 @@ def pallreduce_init(sendbuf, recvbuf, partitions: int, count: int, dtype: int, o
     h = C.c_void_p()
     check(_lib.pc().pc_pallreduce_init(_ptr(sendbuf), _ptr(recvbuf), partitions, count, dtype, op, algo,
                                        comm.handle, C.byref(h)), "pc_pallreduce_init")
-    return Request(comm, h.value, KIND_PALLREDUCE, partitions * count * 4, partitions)
+    return Request(comm, h.value, KIND_PALLREDUCE, partitions * count * ESIZE[dtype], partitions)
 
 
 # ------------------------------------------------------------------ pure host logic

@@ -134,3 +134,24 @@ def jacobi_init(ny: int, nx: int, kind: str = "perf", seed: int = BASE_SEED) -> 
 def uniform_f32_at(seed, rank, epoch, idx, lo=-1.0, hi=1.0) -> np.ndarray:
     """uniform_f32 values at arbitrary indices (sampled parity at full size)."""
     return (lo + (hi - lo) * _unit(u64_at(seed, rank, epoch, idx))).astype(np.float32)
+
+
+def normal_f64(seed, rank, epoch, n, sigma=1.0, start=0) -> np.ndarray:
+    """Box-Muller N(0, sigma^2) kept in float64 (fp64 allreduce inputs)."""
+    raw = u64(seed, rank, epoch, 2 * n, 2 * start)
+    u1 = _unit(raw[0::2])
+    u2 = _unit(raw[1::2])
+    return sigma * np.sqrt(-2.0 * np.log1p(-u1)) * np.cos(2.0 * np.pi * u2)
+
+
+def bf16_bits(seed, rank, epoch, n, sigma=1.0, start=0) -> np.ndarray:
+    """bf16 inputs as uint16 bit patterns: the upper half of normal_f32's bits
+    (truncation is part of the random draw, not of the method)."""
+    return (normal_f32(seed, rank, epoch, n, sigma, start).view(np.uint32) >> np.uint32(16)).astype(np.uint16)
+
+
+def bf16_bits_raw(seed, rank, epoch, n, start=0) -> np.ndarray:
+    """Arbitrary finite bf16 bit patterns (every exponent incl. subnormals)."""
+    b = (u64(seed, rank, epoch, n, start) >> np.uint64(48)).astype(np.uint16)
+    exp = (b >> np.uint16(7)) & np.uint16(0xFF)
+    return np.where(exp == 0xFF, b & np.uint16(0xBFFF), b).astype(np.uint16)  # no inf/NaN

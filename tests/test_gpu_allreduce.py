@@ -21,16 +21,33 @@ pytestmark = pytest.mark.gpu
 SEED = synth.BASE_SEED
 
 
+# host arrays: bf16 travels as uint16 bit patterns (oracle reading R27)
+DTYPES = {np.int32: (pc.INT32, torch.int32), np.float32: (pc.FLOAT32, torch.float32),
+          np.float64: (pc.FLOAT64, torch.float64), np.uint16: (pc.BF16, torch.bfloat16)}
+
+
+def _to_torch(a):
+    if a.dtype == np.uint16:
+        return torch.from_numpy(a.view(np.int16).copy()).view(torch.bfloat16)
+    return torch.from_numpy(np.ascontiguousarray(a))
+
+
+def _to_numpy(t):
+    if t.dtype == torch.bfloat16:
+        return t.view(torch.int16).cpu().numpy().view(np.uint16)
+    return t.cpu().numpy()
+
+
 def run_allreduce(P, Np, L, xs_epochs, algo, op=pc.SUM, inplace=False, producer=None, gran=apps.GRAN_BLOCK):
     """xs_epochs: list over epochs of (P, Np*L) host arrays.  Returns a list over
     epochs of (P, Np*L) results (each rank's recvbuf after its wait)."""
-    dt = pc.INT32 if xs_epochs[0].dtype == np.int32 else pc.FLOAT32
+    dt, tdtype = DTYPES[xs_epochs[0].dtype.type]
+    es = pc.ESIZE[dt]
     n = Np * L
     outs = []
     with comms(P) as cs:
         streams = [torch.cuda.Stream() for _ in range(P)]
         nd = max(n, 4)
-        tdtype = torch.int32 if dt == pc.INT32 else torch.float32
         send = [torch.zeros(nd, dtype=tdtype, device="cuda") for _ in range(P)]
         recv = send if inplace else [torch.zeros(nd, dtype=tdtype, device="cuda") for _ in range(P)]
         src = [torch.zeros(nd, dtype=tdtype, device="cuda") for _ in range(P)]
@@ -39,10 +56,7 @@ def run_allreduce(P, Np, L, xs_epochs, algo, op=pc.SUM, inplace=False, producer=
         for e, xs in enumerate(xs_epochs):
             for r in range(P):
                 with torch.cuda.stream(streams[r]):
-                    if producer:
-                        src[r][:n].copy_(torch.from_numpy(xs[r]).to("cuda", non_blocking=False))
-                    else:
-                        send[r][:n].copy_(torch.from_numpy(xs[r]).to("cuda", non_blocking=False))
+                    (src if producer else send)[r][:n].copy_(_to_torch(xs[r]).to("cuda", non_blocking=False))
             torch.cuda.synchronize()
             for r in range(P):
                 reqs[r].start(streams[r])
@@ -54,7 +68,7 @@ def run_allreduce(P, Np, L, xs_epochs, algo, op=pc.SUM, inplace=False, producer=
                     reqs[r].pbuf_prepare(streams[r])
             for r in range(P):
                 if producer:
-                    apps.produce(send[r], src[r], Np, L * 4, gran, preqs[r], order_stride=producer,
+                    apps.produce(send[r], src[r], Np, L * es, gran, preqs[r], order_stride=producer,
                                  stream=streams[r])
                 else:
                     reqs[r].pready_range(0, Np - 1, streams[r])
@@ -64,7 +78,7 @@ def run_allreduce(P, Np, L, xs_epochs, algo, op=pc.SUM, inplace=False, producer=
             for r in range(P):
                 code, part = reqs[r].error()
                 assert code == 0, f"rank {r} device error {code} at {part}"
-            outs.append(np.stack([recv[r][:n].cpu().numpy() for r in range(P)]))
+            outs.append(np.stack([_to_numpy(recv[r][:n]) for r in range(P)]))
         for q in reqs:
             q.free()
     return outs
@@ -274,3 +288,61 @@ def test_direct_maxmin(op):
     (y,) = run_allreduce(P, Np, L, [x], pc.ALGO_DIRECT, op=op)
     for r in range(P):
         np.testing.assert_array_equal(y[r], oracle.allreduce_def_i32(x, op))
+
+
+# ------------------------------------------------------------ fp64 and bf16 (R27)
+def _inputs(kind, seed, P, n, e=0):
+    gen = synth.normal_f64 if kind == "f64" else synth.bf16_bits
+    return np.stack([gen(seed, r, e, n) for r in range(P)])
+
+
+def _bits(a):
+    return a.view(np.uint64) if a.dtype == np.float64 else a
+
+
+@pytest.mark.parametrize("kind", ["f64", "bf16"])
+@pytest.mark.parametrize("algo,Ps", [(pc.ALGO_RING, [2, 3, 8]), (pc.ALGO_RD, [2, 4, 8]),
+                                     (pc.ALGO_DIRECT, [3, 8])])
+@pytest.mark.parametrize("Np,L", [(1, 1), (3, 17), (7, 64), (2, 4099)])
+def test_wide_and_narrow_dtypes_bitexact(kind, algo, Ps, Np, L):
+    """fp64 / bf16 allreduce bit-exact against the schedule-faithful oracle,
+    including ragged L (partitions not 16-B aligned)."""
+    for P in Ps:
+        x = _inputs(kind, SEED + 41, P, Np * L)
+        (y,) = run_allreduce(P, Np, L, [x], algo)
+        ref, _, _ = oracle.pallreduce(x, Np, algo)
+        for r in range(P):
+            np.testing.assert_array_equal(_bits(y[r]), _bits(ref[r]))
+
+
+@pytest.mark.parametrize("kind", ["f64", "bf16"])
+@pytest.mark.parametrize("algo,P", [(pc.ALGO_RING, 8), (pc.ALGO_RD, 4), (pc.ALGO_DIRECT, 8)])
+def test_dtypes_multi_slice_ragged_epochs_inplace(kind, algo, P):
+    """Many slices per chunk, ragged tail, in place, device producer with a
+    permuted Pready order, 2 epochs; plus the fp64 error bound of the sum."""
+    Np, L = 3, 100_003
+    xs = [_inputs(kind, SEED + 42, P, Np * L, e) for e in range(2)]
+    ys = run_allreduce(P, Np, L, xs, algo, inplace=True, producer=2)
+    for x, y in zip(xs, ys):
+        ref, _, _ = oracle.pallreduce(x, Np, algo)
+        for r in range(P):
+            np.testing.assert_array_equal(_bits(y[r]), _bits(ref[r]))
+        xf = x if kind == "f64" else oracle.bf16_to_f64(x)
+        yf = y[0] if kind == "f64" else oracle.bf16_to_f64(y[0])
+        u = 2.0**-53 if kind == "f64" else 2.0**-8   # unit roundoff
+        bound = (P - 1) * u * np.abs(xf).sum(0) * 1.01 + (0 if kind == "f64" else 2.0**-133)
+        assert (np.abs(yf - xf.sum(0)) <= bound).all()
+
+
+@pytest.mark.parametrize("kind", ["f64", "bf16"])
+@pytest.mark.parametrize("op", [pc.MAX, pc.MIN])
+def test_dtypes_maxmin(kind, op):
+    P, Np, L = 5, 4, 333
+    x = _inputs(kind, SEED + 43, P, Np * L)
+    for algo in (pc.ALGO_RING, pc.ALGO_DIRECT):
+        (y,) = run_allreduce(P, Np, L, [x], algo, op=op)
+        xf = x if kind == "f64" else oracle.bf16_to_f64(x)
+        want = xf.max(0) if op == pc.MAX else xf.min(0)
+        for r in range(P):
+            got = y[r] if kind == "f64" else oracle.bf16_to_f64(y[r])
+            np.testing.assert_array_equal(got, want)
