@@ -12,6 +12,7 @@ Functions (numpy in, numpy out):
   allreduce_def_f64(...)  O2  plain definition, fp32 inputs summed in fp64
   pallreduce(...)         O3/O4/O6  Alg 1 (ring), RD or DIRECT schedule + Alg 2, P threads
   bf16_round / bf16_op    R27 bf16 arithmetic (bit patterns as uint16)
+  bce_grad(p, y, n)       O7  DL proxy producer (R28)
   alg1_table(P, r)        Alg 1 step tuples
   ring_fold_f32 / rd_tree_f32   closed forms of O3 / O4 (pinned against them)
   jacobi_seq / jacobi_decomp    O5
@@ -54,6 +55,7 @@ def lib():
         _lib.orc_pallreduce_direct.argtypes = [i32, i32, i64, i32, i32, i32, i32, P, P, P, u64, P, P]
         _lib.orc_alg1_table.argtypes = [i32, i32, P]
         _lib.orc_bf16_round.argtypes = [i64, P, P]
+        _lib.orc_bce_grad.argtypes = [i64, P, P, C.c_float, P]
         _lib.orc_bf16_op.argtypes = [i32, i64, P, P, P]
         _lib.orc_ring_fold_f32.argtypes = [i32, i64, P, P, P]
         _lib.orc_rd_tree_f32.argtypes = [i32, i64, P, P]
@@ -154,6 +156,15 @@ def pallreduce(x: np.ndarray, partitions: int, algo: int = RING, op: int = SUM, 
 
 
 _DTYPES = {np.int32: INT32, np.float32: FLOAT32, np.float64: FLOAT64, np.uint16: BF16}
+
+
+def bce_grad(p: np.ndarray, y: np.ndarray, n: float) -> np.ndarray:
+    """O7 (R28): fp32 gradient of the mean BCE w.r.t. the predictions."""
+    p = np.ascontiguousarray(p, dtype=np.float32)
+    y = np.ascontiguousarray(y, dtype=np.float32)
+    g = np.zeros_like(p)
+    _check(lib().orc_bce_grad(p.size, _p(p), _p(y), float(n), _p(g)), "bce_grad")
+    return g
 
 
 def bf16_round(x: np.ndarray) -> np.ndarray:

@@ -538,6 +538,26 @@ int orc_pallreduce(int algo, int P, int Np, int64_t L, int dtype, int op, int ep
   return failed ? ORC_ERR_TIMEOUT : ORC_OK;
 }
 
+// ===========================================================================
+// O7: DL proxy producer (§VI-D2; the BCE kernel of [34] is
+// external, reading R28): gradient of the mean binary cross-entropy
+//   l = -(1/n) sum_i [ y_i ln p_i + (1 - y_i) ln(1 - p_i) ]
+// with respect to p_i:  dl/dp_i = (p_i - y_i) / (p_i (1 - p_i) n),
+// evaluated in fp32 as five IEEE operations in this order:
+//   ((p - y) / ((p * (1 - p)) * n)).
+// ===========================================================================
+int orc_bce_grad(int64_t n, const float *p, const float *y, float nf, float *g) {
+  for (int64_t i = 0; i < n; ++i) {
+    volatile float d = p[i] - y[i];
+    volatile float t = 1.0f - p[i];
+    volatile float q = p[i] * t;
+    volatile float qn = q * nf;
+    volatile float r = d / qn;
+    g[i] = r;
+  }
+  return ORC_OK;
+}
+
 // bf16 arithmetic of R27, exported so tests can pin it (round-to-nearest-even
 // of binary64 values to bf16 bit patterns; the ⊕ of two bf16 operands).
 int orc_bf16_round(int64_t n, const double *x, uint16_t *out) {

@@ -29,6 +29,15 @@ def produce(dst, src, partitions: int, part_bytes: int, gran: int, preq: Preques
                                   preq.ptr, _stream(stream)), "produce")
 
 
+def bce_grad(p, y, g, partitions: int, L: int, nf: float, preq: Prequest | None = None, order_stride: int = 1,
+             blocks: int = 0, stream=None):
+    """DL proxy producer (R28): g = (p - y) / ((p (1 - p)) n) over partitions of L
+    fp32 elements, one block per partition; with ``preq`` each partition is
+    Preadied (block granularity) into the partitioned allreduce that reads g."""
+    _ok(_lib.apps().pcapp_bce_grad(_ptr(p), _ptr(y), _ptr(g), partitions, L, nf, order_stride, blocks,
+                                   preq.ptr if preq is not None else None, _stream(stream)), "bce_grad")
+
+
 def check_recv(preq: Prequest, recvbuf, out, partitions: int, part_bytes: int, status, blocks: int = 64,
                stream=None):
     _ok(_lib.apps().pcapp_check_recv(preq.ptr, _ptr(recvbuf), _ptr(out), partitions, part_bytes, blocks,
@@ -203,3 +212,59 @@ class JacobiSolver:
         for st in self.local:
             for q in self._reqs(st):
                 q.free()
+
+
+class DLProxy:
+    """The paper's DL kernel (§VI-D2) on co-located ranks: every
+    step each rank computes its BCE gradient (``bce_grad``) and the ranks
+    allreduce it with one persistent partitioned allreduce; ``pc_startall`` and
+    ``pc_pbuf_prepare_all`` are inside the step, as in a training loop.
+
+    mode "pready": the producer Preadies each partition from the kernel
+                   (block granularity, ENGINE copy); the engine reduces;
+    mode "serial": producer kernel, then the collective (host-side Pready of
+                   every partition, the MPI_Allreduce-after-the-kernel flow).
+    Inputs: ``p`` (predictions), ``y`` (targets), fp32, one tensor per rank."""
+
+    def __init__(self, comms, partitions: int, L: int, algo: int, p, y):
+        import torch
+
+        from . import runtime as rt
+
+        self.P, self.Np, self.L = len(comms), partitions, L
+        self.p, self.y = p, y
+        n = partitions * L
+        self.nf = float(n)
+        self.g = [torch.empty(max(n, 4), device=p[0].device) for _ in range(self.P)]
+        self.out = [torch.empty(max(n, 4), device=p[0].device) for _ in range(self.P)]
+        self.reqs = [rt.pallreduce_init(self.g[r], self.out[r], partitions, L, rt.FLOAT32, rt.SUM, algo, comms[r])
+                     for r in range(self.P)]
+        self.preqs = None
+        self.ctl = torch.cuda.Stream()
+
+    def step(self, mode: str = "pready", order_stride: int = 1):
+        from . import runtime as rt
+
+        st = self.ctl
+        if self.preqs is None:  # first epoch: exchange + mapping (collective over the ranks)
+            for q in self.reqs:
+                q.start(st)
+            rt.run_ranks([(lambda q=q: q.pbuf_prepare(st)) for q in self.reqs])
+            self.preqs = [q.prequest_create(rt.GRAN_BLOCK, 1, rt.COPY_ENGINE) for q in self.reqs]
+        else:
+            rt.startall(self.reqs, st)
+            rt.pbuf_prepare_all(self.reqs, st)
+        for r in range(self.P):
+            bce_grad(self.p[r], self.y[r], self.g[r], self.Np, self.L, self.nf,
+                     self.preqs[r] if mode == "pready" else None, order_stride, stream=st)
+        if mode == "serial":
+            rt.preadyall(self.reqs, st)
+        for q in self.reqs:
+            q.wait_on_stream(st)
+
+    def errors(self):
+        return [(r, q.error()) for r, q in enumerate(self.reqs) if q.error()[0] != 0]
+
+    def free(self):
+        for q in self.reqs:
+            q.free()

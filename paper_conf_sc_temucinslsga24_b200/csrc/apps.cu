@@ -6,6 +6,10 @@
 //                P:L229; §VI-A)
 //   produce      copy a prepared input into the send buffer partition by
 //                partition and Pready each one (allreduce producer, §VI-B)
+//   bce_grad     DL proxy (§VI-D2; reading R28): gradient of the
+//                mean binary cross-entropy w.r.t. the predictions, one
+//                partition per block, pc_pready_block into a partitioned
+//                allreduce as soon as the partition's gradient is stored
 //   check_recv   receiver kernel that waits pc_parrived per partition and
 //                consumes it (device Parrived)
 //   pingpong     Pready->Parrived latency inside one persistent kernel per side
@@ -64,6 +68,39 @@ __global__ void __launch_bounds__(512) produce_kernel(uint8_t *__restrict__ dst,
         __threadfence();
         pc_pready(p, preq);
       }
+    }
+  }
+}
+
+// R28: g = (p - y) / ((p * (1 - p)) * n), five IEEE fp32 ops in this order
+// (explicit _rn intrinsics: no contraction, IEEE division).
+__device__ __forceinline__ float bce_g(float p, float y, float nf) {
+  return __fdiv_rn(__fsub_rn(p, y), __fmul_rn(__fmul_rn(p, __fsub_rn(1.0f, p)), nf));
+}
+
+// Each block produces partitions k = blockIdx.x, +gridDim.x, ... in the order
+// p = k * order_stride mod partitions; then Preadies it (block granularity).
+// use_pready = 0: the plain kernel (the serialized baseline's producer).
+__global__ void __launch_bounds__(512) bce_grad_kernel(const float *__restrict__ P, const float *__restrict__ Y,
+                                                      float *__restrict__ G, int partitions, int64_t L, float nf,
+                                                      int order_stride, int use_pready, pc_prequest_t preq) {
+  for (int k = blockIdx.x; k < partitions; k += gridDim.x) {
+    const int u = (int)(((int64_t)k * order_stride) % partitions);
+    const int64_t off = (int64_t)u * L;
+    const float *p = P + off, *y = Y + off;
+    float *g = G + off;
+    const bool vec = ((((uintptr_t)p) | ((uintptr_t)y) | ((uintptr_t)g)) & 15) == 0;
+    const int64_t nv = vec ? L / 4 : 0;
+    const float4 *p4 = reinterpret_cast<const float4 *>(p), *y4 = reinterpret_cast<const float4 *>(y);
+    float4 *g4 = reinterpret_cast<float4 *>(g);
+#pragma unroll 4
+    for (int64_t j = threadIdx.x; j < nv; j += blockDim.x) {
+      const float4 a = __ldcs(p4 + j), b = __ldcs(y4 + j);
+      g4[j] = make_float4(bce_g(a.x, b.x, nf), bce_g(a.y, b.y, nf), bce_g(a.z, b.z, nf), bce_g(a.w, b.w, nf));
+    }
+    for (int64_t j = nv * 4 + threadIdx.x; j < L; j += blockDim.x) g[j] = bce_g(p[j], y[j], nf);
+    if (use_pready) {
+      pc_pready_block(u, preq);
     }
   }
 }
@@ -247,6 +284,17 @@ int pcapp_produce(void *dst, const void *src, int partitions, int64_t part_bytes
   if (blocks <= 0) blocks = partitions < 1184 ? partitions : 1184;
   produce_kernel<<<blocks, 512, 0, s>>>((uint8_t *)dst, (const uint8_t *)src, partitions, part_bytes, gran,
                                         order_stride < 1 ? 1 : order_stride, *preq);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_bce_grad(const float *p, const float *y, float *g, int partitions, int64_t L, float nf, int order_stride,
+                   int blocks, const pc_prequest_t *preq, cudaStream_t s) {
+  if (partitions < 1 || L < 0) return -1;
+  if (blocks <= 0) blocks = partitions < 1184 ? partitions : 1184;
+  pc_prequest_t q{};
+  if (preq) q = *preq;
+  bce_grad_kernel<<<blocks, 512, 0, s>>>(p, y, g, partitions, L, nf, order_stride < 1 ? 1 : order_stride,
+                                         preq ? 1 : 0, q);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -155,3 +155,12 @@ def bf16_bits_raw(seed, rank, epoch, n, start=0) -> np.ndarray:
     b = (u64(seed, rank, epoch, n, start) >> np.uint64(48)).astype(np.uint16)
     exp = (b >> np.uint16(7)) & np.uint16(0xFF)
     return np.where(exp == 0xFF, b & np.uint16(0xBFFF), b).astype(np.uint16)  # no inf/NaN
+
+
+def bce_inputs(seed, rank, epoch, n, start=0):
+    """DL proxy inputs (R28): predictions p uniform in [0.02, 0.98) (post-sigmoid
+    probabilities away from 0/1) and binary targets y in {0, 1}."""
+    raw = u64(seed, rank, epoch, 2 * n, 2 * start)
+    p = (0.02 + 0.96 * _unit(raw[0::2])).astype(np.float32)
+    y = (raw[1::2] >> np.uint64(63)).astype(np.float32)
+    return p, y

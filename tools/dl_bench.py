@@ -1,0 +1,87 @@
+"""DL proxy (§VI-D2, Figs 10/11 analogue) on one B200 with co-located virtual
+ranks: per step each rank computes the BCE gradient of a ResNet-50-sized flat
+buffer (25.56 M fp32) and the ranks allreduce it; pc_startall +
+pc_pbuf_prepare_all are inside the step.  Modes: pready (the producer
+Preadies each partition from the kernel), serial (producer, then host Pready
+of all partitions), and the two halves alone.
+JSON lines to stdout; CUDA-event timing on the control stream."""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
+import torch  # noqa: E402
+
+import paper_conf_sc_temucinslsga24_b200 as pc  # noqa: E402
+from paper_conf_sc_temucinslsga24_b200 import apps  # noqa: E402
+
+NPARAM = 25_557_032  # ResNet-50
+
+
+def timeit(fn, st, reps=20, warm=3):
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    for _ in range(reps):
+        fn()
+    e1.record(st)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps
+
+
+def run(P, L, algo, modes):
+    Np = -(-NPARAM // L)
+    n = Np * L
+    g, cs = pc.local_comms(P, 0)
+    gen = torch.Generator(device="cuda")
+    gen.manual_seed(0x5C24)
+    p = [(0.02 + 0.96 * torch.rand(n, device="cuda", generator=gen)) for _ in range(P)]
+    y = [torch.randint(0, 2, (n,), device="cuda", generator=gen).float() for _ in range(P)]
+    dl = apps.DLProxy(cs, Np, L, algo, p, y)
+    out = []
+    for mode in modes:
+        if mode in ("pready", "serial"):
+            ms = timeit(lambda: dl.step(mode), dl.ctl)
+        elif mode == "bce_only":
+            def f():
+                for r in range(P):
+                    apps.bce_grad(p[r], y[r], dl.g[r], Np, L, float(n), None, stream=dl.ctl)
+            ms = timeit(f, dl.ctl)
+        else:  # allreduce only (host Pready of every partition)
+            def f():
+                pc.startall(dl.reqs, dl.ctl)
+                pc.pbuf_prepare_all(dl.reqs, dl.ctl)
+                pc.preadyall(dl.reqs, dl.ctl)
+                for q in dl.reqs:
+                    q.wait_on_stream(dl.ctl)
+            ms = timeit(f, dl.ctl)
+        errs = dl.errors()
+        assert errs == [], (mode, errs)
+        out.append({"P": P, "partition_bytes": 4 * L, "partitions": Np, "algo": algo, "mode": mode,
+                    "ms_per_step": ms, "grad_GB_per_s_all_ranks": P * 4 * n / (ms / 1e3) / 1e9})
+        print(json.dumps(out[-1]), flush=True)
+    dl.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
+    return out
+
+
+if __name__ == "__main__":
+    torch.cuda.set_device(0)
+    modes = sys.argv[1].split(",") if len(sys.argv) > 1 else ["pready", "serial", "bce_only", "allreduce_only"]
+    Ps = [int(v) for v in sys.argv[2].split(",")] if len(sys.argv) > 2 else [8, 4, 2]
+    Ls = [int(v) for v in sys.argv[3].split(",")] if len(sys.argv) > 3 else [16384, 65536, 262144]
+    algos = [int(v) for v in sys.argv[4].split(",")] if len(sys.argv) > 4 else [pc.ALGO_RING, pc.ALGO_DIRECT]
+    for P in Ps:
+        for L in Ls:
+            for algo in algos:
+                try:
+                    run(P, L, algo, modes)
+                except AssertionError as ex:
+                    print(json.dumps({"P": P, "L": L, "algo": algo, "error": str(ex)}), flush=True)
