@@ -82,6 +82,7 @@ _APP_PROTOS = {
     "pcapp_bare_pingpong_pair": (I32, [P, P, I32, C.c_uint32, P, P]),
     "pcapp_prequest_size": (SZ, []),
     "pcapp_flag_variant": (I32, [P, P, I32, I32, C.c_uint32, P, P]),
+    "pcapp_lat_probe_pair": (I32, [P, P, P, P, I32, I32, P, P]),
     "pcapp_jacobi_rank_size": (SZ, []),
     "pcapp_jacobi_launch": (I32, [P, P, I32, I32, I32, I32, P]),
     "pcapp_jacobi_describe": (I32, [P, P, P, I32, I32, I32, I32, I32, I32, P, P, P, P, P]),

@@ -200,6 +200,88 @@ __global__ void bare_pingpong_pair_kernel(uint32_t *flagA, uint32_t *flagB, int 
   out_ns[side] = pc_detail::globaltimer() - t0;
 }
 
+
+// Latency decomposition probe (tools/lat_probe.py): the pair ping-pong with
+// the library wait and/or Pready replaced by raw flag operations.
+//   WLIB: pc_wait_arrived (1) or a relaxed poll of flags[k] (0)
+//   PLIB: pc_pready_warp (1), pc_pready by lane 0 (2), or raw: copy the
+//         payload, fence at the request scope, store the peer flag (0)
+template <int WLIB, int PLIB>
+__global__ void lat_probe_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, pc_prequest_t sendB,
+                                      pc_prequest_t recvB, int iters, unsigned long long *out_ns) {
+  const int side = blockIdx.x;
+  const pc_prequest_t &sq = side ? sendB : sendA;
+  const pc_prequest_t &rq = side ? recvB : recvA;
+  const uint32_t e = pc_detail::epoch_of(sq);
+  auto wait = [&](int k) {
+    if (threadIdx.x == 0) {
+      if (WLIB) {
+        pc_wait_arrived(rq, k);
+      } else {
+        while (!pc_detail::reached(pc_detail::ld_relaxed_sys(rq.flags + k), e)) {
+        }
+        if (rq.part_bytes) pc_detail::fence_gpu();
+      }
+    }
+    __syncwarp();
+  };
+  auto ready = [&](int k) {
+    if (PLIB == 1) {
+      pc_pready_warp(k, sq);
+    } else if (PLIB == 2) {
+      if (threadIdx.x == 0) pc_pready(k, sq);
+      __syncwarp();
+    } else if (PLIB == 3) {  // lane 0: epoch_rtr + publish, no shuffles
+      __syncwarp();
+      if (threadIdx.x == 0) {
+        const uint2 er = pc_detail::epoch_rtr(sq);
+        pc_detail::publish(sq, k / sq.agg, 1, er.x, k);
+      }
+      __syncwarp();
+    } else if (PLIB == 4) {  // + broadcast of e
+      __syncwarp();
+      uint32_t ee = 0;
+      if (threadIdx.x == 0) ee = pc_detail::epoch_rtr(sq).x;
+      ee = __shfl_sync(0xffffffffu, ee, 0);
+      if (threadIdx.x == 0) pc_detail::publish(sq, k / sq.agg, 1, ee, k);
+      __syncwarp();
+    } else if (PLIB == 5) {  // relaxed epoch read by lane 0 + publish
+      __syncwarp();
+      if (threadIdx.x == 0) pc_detail::publish(sq, k / sq.agg, 1, pc_detail::ld_relaxed_sys(sq.epoch), k);
+      __syncwarp();
+    } else {
+      if (sq.part_bytes) {
+        const uint64_t off = (uint64_t)k * sq.part_bytes;
+        pc_detail::copy_bytes(sq.peer_rbuf + off, sq.sbuf + off, sq.part_bytes, threadIdx.x, 32);
+        pc_detail::fence_gpu();
+        __syncwarp();
+      }
+      if (threadIdx.x == 0) {
+        pc_detail::st_relaxed_sys(sq.peer_flags + k, e);
+        pc_detail::st_relaxed_gpu(sq.sent + k, e);
+      }
+      __syncwarp();
+    }
+  };
+  const uint64_t t0 = pc_detail::globaltimer();
+  long long c_ready = 0, c_wait = 0;
+  for (int k = 0; k < iters; ++k) {
+    const long long c0 = clock64();
+    if (side == 1) wait(k);
+    const long long c1 = clock64();
+    ready(k);
+    const long long c2 = clock64();
+    if (side == 0) wait(k);
+    c_wait += c1 - c0;
+    c_ready += c2 - c1;
+  }
+  if (threadIdx.x == 0) {
+    out_ns[side] = pc_detail::globaltimer() - t0;
+    out_ns[2 + 2 * side] = (unsigned long long)c_ready;  // SM cycles inside Pready
+    out_ns[3 + 2 * side] = (unsigned long long)c_wait;   // SM cycles inside the side-1 wait
+  }
+}
+
 // Flag ping-pong microbenchmark over memory-order variants (latency floor
 // study): 0 st.release.sys/ld.acquire.sys, 1 relaxed.sys,
 // 2 release/acquire.gpu, 3 relaxed.gpu, 4 fence.acq_rel.sys+st.relaxed.sys /
@@ -343,6 +425,26 @@ int pcapp_flag_variant(uint32_t *flagA, uint32_t *flagB, int variant, int iters,
     case 4: flag_variant_kernel<4><<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns); break;
     default: flag_variant_kernel<5><<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns); break;
   }
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+
+int pcapp_lat_probe_pair(const pc_prequest_t *sendA, const pc_prequest_t *recvA, const pc_prequest_t *sendB,
+                         const pc_prequest_t *recvB, int mode, int iters, unsigned long long *out_ns, cudaStream_t s) {
+  if (!sendA || !recvA || !sendB || !recvB) return -1;
+#define PCAPP_LP(W, P_) lat_probe_pair_kernel<W, P_><<<2, 32, 0, s>>>(*sendA, *recvA, *sendB, *recvB, iters, out_ns)
+  switch (mode) {
+    case 0: PCAPP_LP(1, 1); break;
+    case 1: PCAPP_LP(0, 1); break;
+    case 2: PCAPP_LP(1, 0); break;
+    case 3: PCAPP_LP(0, 0); break;
+    case 4: PCAPP_LP(1, 2); break;
+    case 5: PCAPP_LP(0, 2); break;
+    case 6: PCAPP_LP(1, 3); break;
+    case 7: PCAPP_LP(1, 4); break;
+    default: PCAPP_LP(1, 5); break;
+  }
+#undef PCAPP_LP
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

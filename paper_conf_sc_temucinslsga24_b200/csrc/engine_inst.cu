@@ -1,0 +1,71 @@
+// One (dtype, op) instantiation of the engine launchers declared in
+// engine.cuh; the Makefile compiles this file 12 times with
+// -DPC_DT=<0|1|3|4> -DPC_OP=<0|1|2>.
+#include "engine.cuh"
+
+#if !defined(PC_DT) || !defined(PC_OP)
+#error "compile with -DPC_DT=<dtype> -DPC_OP=<op>"
+#endif
+
+namespace pc {
+
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::ring(const RingArgs &a, int warps, cudaStream_t s) {
+  ring_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::rd(const RdArgs &a, int warps, cudaStream_t s) {
+  rd_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::direct(const DirectArgs &a, int warps, cudaStream_t s) {
+  direct_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::ring_group(const RingGroupArgs &h, int blocks, cudaStream_t s) {
+  ring_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::rd_group(const RdGroupArgs &h, int blocks, cudaStream_t s) {
+  rd_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s) {
+  direct_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::occupancy(int *ctas) {
+  int a = 0, b = 0;
+  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, ring_engine<DT, OP>, kEngineBlock, 0));
+  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, rd_engine<DT, OP>, kEngineBlock, 0));
+  *ctas = a < b ? a : b;
+  return 0;
+}
+
+template struct EngineLaunch<PC_DT, PC_OP>;
+
+}  // namespace pc

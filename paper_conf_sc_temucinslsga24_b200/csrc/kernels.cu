@@ -1,608 +1,13 @@
-// libpc device engines (sm_100a).
-//
-//  ring_engine   partitioned allreduce, Alg 1 schedule progressed
-//                on the GPU: the host Progression Engine of Alg 2
-//                and its per-step reduce kernel + cudaStreamSynchronize
-//                 are replaced by warps that wait on a flag,
-//                reduce the arriving slice in registers and forward it to the
-//                next rank in the same pass (the "computation inside the device
-//                call" the paper proposes).
-//  rd_engine     the same over a recursive-doubling schedule (north_star).
-//  p2p_engine    ENGINE copy mode of partitioned send: poll local ready flags,
-//                push slices over NVLink, publish the receiver's flag.
-//  wait_words    stream-ordered MPI_Wait for send/recv requests.
-//
-// Unit of work = (user partition u, slice s) handled by ONE warp through all
-// steps of the schedule ("each partition independently executes that
-// schedule").  Warps take units in increasing order, x = gw, gw+W, ...
-// with W identical on every rank (agreed at comm creation), so the dependency
-// (unit x, step i) at rank r -> (unit x, step i-1) at rank r-1 can never form a
-// cycle while all engine warps are resident.
-#include <cuda_bf16.h>
-#include <cuda_runtime.h>
-
-#include <atomic>
-
-#include "pc_device.cuh"
-#include "pc_internal.h"
+// libpc device kernels (sm_100a): ENGINE-mode p2p copy, stream-ordered waits,
+// epoch / ready-to-receive control kernels, host-binding Pready kernels, and
+// the (dtype, op) switch onto the allreduce engines of engine.cuh (compiled
+// per instantiation in engine_inst.cu).
+#include "engine.cuh"
 
 namespace pc {
 namespace {
 
 using namespace pc_detail;
-
-#ifndef PC_ENGINE_UNROLL
-#define PC_ENGINE_UNROLL 8
-#endif
-constexpr int kU = PC_ENGINE_UNROLL;  // 16-B vectors in flight per operand per lane
-
-// Engine-side bounded spin: the awaited event is a whole slice step of the
-// upstream rank (tens of microseconds), so back off with __nanosleep early and
-// keep the L2 free of polling traffic.
-__device__ __forceinline__ bool engine_spin(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo, int part,
-                                            bool SYS) {
-  uint32_t v = SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p);
-  if (reached(v, target)) return true;
-  const uint64_t t0 = globaltimer();
-  uint32_t ns = 64, n = 0;
-  for (;;) {
-    __nanosleep(ns);
-    if (ns < 1024) ns <<= 1;
-    v = SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p);
-    if (reached(v, target)) return true;
-    if ((++n & 15) == 0) {
-      if (aborted(err)) return false;
-      if (tmo && globaltimer() - t0 > (uint64_t)tmo * 1000000ull) {
-        set_error(err, PC_DEV_ERR_TIMEOUT, part);
-        return false;
-      }
-    }
-  }
-}
-
-// Warp-wide bounded wait on a flag word; lane 0 polls, the warp follows.
-// sys: acquire at system scope (word written from another GPU).
-__device__ __forceinline__ bool warp_wait(const uint32_t *p, uint32_t target, int32_t *err, uint32_t tmo, int part,
-                                          bool sys) {
-  bool ok = true;
-  if ((threadIdx.x & 31) == 0) ok = engine_spin(p, target, err, tmo, part, sys);
-  ok = __shfl_sync(0xffffffffu, ok, 0);
-  __syncwarp();
-  return ok;
-}
-
-// Publish: every lane's (peer) stores are made visible at the request's scope
-// (system scope for a peer on another GPU), then lane 0 stores the epoch into
-// the consumer's flag.
-__device__ __forceinline__ void warp_signal(uint32_t *flag, uint32_t e, bool sys) {
-  fence_scope(sys);
-  __syncwarp();
-  if ((threadIdx.x & 31) == 0) st_relaxed_sys(flag, e);
-}
-
-template <int DT, int OP>
-struct Op;
-template <int OP>
-struct Op<0, OP> {  // int32: sum wraps mod 2^32
-  using T = int32_t;
-  static __device__ __forceinline__ int32_t f(int32_t a, int32_t b) {
-    if (OP == 0) return (int32_t)((uint32_t)a + (uint32_t)b);
-    if (OP == 1) return a > b ? a : b;
-    return a < b ? a : b;
-  }
-};
-template <int OP>
-struct Op<1, OP> {  // fp32: one IEEE add, round to nearest even, no contraction
-  using T = float;
-  static __device__ __forceinline__ float f(float a, float b) {
-    if (OP == 0) return __fadd_rn(a, b);
-    if (OP == 1) return fmaxf(a, b);
-    return fminf(a, b);
-  }
-};
-
-template <int OP>
-struct Op<3, OP> {  // fp64 (the paper's `double` buffers)
-  using T = double;
-  static __device__ __forceinline__ double f(double a, double b) {
-    if (OP == 0) return __dadd_rn(a, b);
-    if (OP == 1) return fmax(a, b);
-    return fmin(a, b);
-  }
-};
-template <int OP>
-struct Op<4, OP> {  // bf16 storage (uint16 bits); each op is one correctly rounded bf16 result:
-  using T = uint16_t;  // a + b of two bf16 values is exact in fp32 or the small one is below half an ulp
-  static __device__ __forceinline__ float up(uint16_t v) { return __uint_as_float((uint32_t)v << 16); }
-  static __device__ __forceinline__ uint16_t dn(float f) {
-    return __bfloat16_as_ushort(__float2bfloat16_rn(f));
-  }
-  static __device__ __forceinline__ uint16_t f(uint16_t a, uint16_t b) {
-    if (OP == 0) return dn(__fadd_rn(up(a), up(b)));
-    if (OP == 1) return dn(fmaxf(up(a), up(b)));
-    return dn(fminf(up(a), up(b)));
-  }
-};
-
-template <int DT, int OP>
-__device__ __forceinline__ uint4 vop(uint4 a, uint4 b) {
-  using O = Op<DT, OP>;
-  using T = typename O::T;
-  constexpr int EPV = 16 / sizeof(T);
-  uint4 r;
-  T *ra = reinterpret_cast<T *>(&r);
-  const T *pa = reinterpret_cast<const T *>(&a);
-  const T *pb = reinterpret_cast<const T *>(&b);
-#pragma unroll
-  for (int j = 0; j < EPV; ++j) ra[j] = O::f(pa[j], pb[j]);
-  return r;
-}
-
-// out1[k] (and out2[k]) = local[k] ⊕ incoming[k], k < n elements, by one warp.
-// All operands of one call sit at the same element offset of 16-B aligned
-// buffers, so they share one misalignment: a scalar head of < 4 elements
-// brings them to a 16-B boundary, the body runs on 16-B vectors (kU in flight
-// per operand per lane), a scalar tail finishes.  (Gradient buffers of
-// arbitrary tensor sizes, C3, make unaligned partitions the common case.)
-template <int DT, int OP>
-__device__ __forceinline__ void warp_reduce(void *out1, void *out2, const void *local, const void *incoming,
-                                            int64_t n) {
-  using O = Op<DT, OP>;
-  using T = typename O::T;
-  const uint32_t lane = threadIdx.x & 31;
-  const T *a = reinterpret_cast<const T *>(local);
-  const T *b = reinterpret_cast<const T *>(incoming);
-  T *o1 = reinterpret_cast<T *>(out1);
-  T *o2 = reinterpret_cast<T *>(out2);
-  constexpr int64_t EPV = 16 / sizeof(T);
-  const uintptr_t m = reinterpret_cast<uintptr_t>(out1) & 15;
-  const bool same = ((reinterpret_cast<uintptr_t>(local) & 15) == m) &&
-                    ((reinterpret_cast<uintptr_t>(incoming) & 15) == m) &&
-                    (!out2 || (reinterpret_cast<uintptr_t>(out2) & 15) == m) && (m % sizeof(T)) == 0;
-  int64_t head = same ? (int64_t)(((16 - m) & 15) / sizeof(T)) : n;
-  if (head > n) head = n;
-  for (int64_t k = lane; k < head; k += 32) {
-    const T r = O::f(__ldcg(a + k), __ldcg(b + k));
-    o1[k] = r;
-    if (o2) o2[k] = r;
-  }
-  int64_t done = head;
-  if (same && n > head) {
-    const int64_t nv = (n - head) / EPV;
-    const uint4 *av = reinterpret_cast<const uint4 *>(a + head);
-    const uint4 *bv = reinterpret_cast<const uint4 *>(b + head);
-    uint4 *o1v = reinterpret_cast<uint4 *>(o1 + head);
-    uint4 *o2v = o2 ? reinterpret_cast<uint4 *>(o2 + head) : nullptr;
-    int64_t k = lane;
-    for (; k + 32 * (kU - 1) < nv; k += 32 * kU) {
-      uint4 x[kU], y[kU];
-#pragma unroll
-      for (int j = 0; j < kU; ++j) x[j] = __ldcg(av + k + 32 * j);
-#pragma unroll
-      for (int j = 0; j < kU; ++j) y[j] = __ldcg(bv + k + 32 * j);
-#pragma unroll
-      for (int j = 0; j < kU; ++j) {
-        const uint4 r = vop<DT, OP>(x[j], y[j]);
-        o1v[k + 32 * j] = r;
-        if (o2v) o2v[k + 32 * j] = r;
-      }
-    }
-    for (; k < nv; k += 32) {
-      const uint4 r = vop<DT, OP>(__ldcg(av + k), __ldcg(bv + k));
-      o1v[k] = r;
-      if (o2v) o2v[k] = r;
-    }
-    done = head + nv * EPV;
-  }
-  for (int64_t k = done + lane; k < n; k += 32) {
-    const T r = O::f(__ldcg(a + k), __ldcg(b + k));
-    o1[k] = r;
-    if (o2) o2[k] = r;
-  }
-}
-
-__device__ __forceinline__ void warp_copy(void *dst, const void *src, int64_t nbytes) {
-  const uint32_t lane = threadIdx.x & 31;
-  const uintptr_t m = reinterpret_cast<uintptr_t>(dst) & 15;
-  if (m && (reinterpret_cast<uintptr_t>(src) & 15) == m && nbytes > (int64_t)(16 - m)) {
-    // shared misalignment: copy a head up to the 16-B boundary, then vectors
-    const int64_t h = (int64_t)(16 - m);
-    copy_bytes(reinterpret_cast<uint8_t *>(dst), reinterpret_cast<const uint8_t *>(src), (uint64_t)h, lane, 32);
-    dst = reinterpret_cast<uint8_t *>(dst) + h;
-    src = reinterpret_cast<const uint8_t *>(src) + h;
-    nbytes -= h;
-  }
-  if (((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src)) & 15) == 0) {
-    const int64_t nv = nbytes >> 4;
-    const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
-    uint4 *d4 = reinterpret_cast<uint4 *>(dst);
-    int64_t k = lane;
-    for (; k + 32 * (kU - 1) < nv; k += 32 * kU) {
-      uint4 x[kU];
-#pragma unroll
-      for (int j = 0; j < kU; ++j) x[j] = __ldcg(s4 + k + 32 * j);
-#pragma unroll
-      for (int j = 0; j < kU; ++j) d4[k + 32 * j] = x[j];
-    }
-    for (; k < nv; k += 32) d4[k] = __ldcg(s4 + k);
-    const int64_t done = nv << 4;
-    if (done < nbytes) copy_bytes(reinterpret_cast<uint8_t *>(dst) + done, reinterpret_cast<const uint8_t *>(src) + done,
-                                  (uint64_t)(nbytes - done), lane, 32);
-    return;
-  }
-  copy_bytes(reinterpret_cast<uint8_t *>(dst), reinterpret_cast<const uint8_t *>(src), (uint64_t)nbytes, lane, 32);
-}
-
-__device__ __forceinline__ int modp(int a, int p) { return ((a % p) + p) % p; }
-
-// ---------------------------------------------------------------------------
-// Ring (Alg 1).  Paper indexing: at step i rank r sends chunk R_i = r - i and
-// receives chunk A_i = r - i - 1 (mod P).  Fused engine step E_i (i >= 1)
-// consumes the arrival of step i-1 (chunk A_{i-1} = R_i) and sends step i:
-//   1 <= i <= P-2 : acc = send[c] ⊕ staging[c]  -> O.staging[c]        (RS)
-//   i  = P-1      : acc = send[c] ⊕ staging[c]  -> recv[c], O.recv[c]  (final)
-//   P <= i <= 2P-3:        recv[c]              -> O.recv[c]           (AG)
-// E_0 sends send[r] -> O.staging[r]; completion waits for step 2P-3.
-// Operand order local ⊕ incoming (reading R5); flags are per (u, step, slice)
-// (reading R3) and hold epoch values, so they are never reset.
-// ---------------------------------------------------------------------------
-// Alg 2 on a warp: the warp owns up to kMaxActive units and
-// sweeps them round-robin, polling each unit's next dependency once and
-// performing the step of every unit that is ready — exactly the per-partition
-// state machine of Alg 2, with the progression thread replaced by the warp.
-// A slow upstream unit therefore never idles the warp while another of its
-// units can advance.  Dependencies form a DAG over (unit, step, rank), so
-// progress only needs every engine warp to be resident.
-constexpr int kMaxActive = 8;
-
-__device__ __forceinline__ bool warp_poll(const uint32_t *p, uint32_t target, bool sys) {
-  bool ok = false;
-  if ((threadIdx.x & 31) == 0) ok = reached(sys ? ld_acquire_sys(p) : ld_acquire_gpu(p), target);
-  return __shfl_sync(0xffffffffu, ok, 0);
-}
-
-// Idle backoff shared by the sweeping engines; false on abort / timeout.
-struct Idle {
-  uint64_t since = 0;
-  uint32_t ns = 0, spins = 0;
-  __device__ __forceinline__ void progressed() {
-    since = 0;
-    ns = 0;
-    spins = 0;
-  }
-  __device__ __forceinline__ bool wait(int32_t *err, uint32_t tmo, int part) {
-    if (since == 0) since = globaltimer();
-    // poll back-to-back first (a hop of a small message is ~1 us away), then
-    // back off so long waits (large slices upstream) leave the L2 alone
-    if (++spins > 64) {
-      ns = ns ? (ns < 512 ? ns * 2 : 512) : 32;
-      __nanosleep(ns);
-    }
-    if (aborted(err)) return false;
-    if (tmo && globaltimer() - since > (uint64_t)tmo * 1000000ull) {
-      if ((threadIdx.x & 31) == 0) set_error(err, PC_DEV_ERR_TIMEOUT, part);
-      return false;
-    }
-    return true;
-  }
-};
-
-template <int DT, int OP>
-__device__ __forceinline__ void ring_step(const RingArgs &a, int u, int s, int i, uint32_t e) {
-  const int P = a.P, r = a.r, NS = 2 * (P - 1);
-  const int64_t es = sizeof(typename Op<DT, OP>::T);
-  const int64_t base = (int64_t)u * a.L;
-  const int64_t fbase = (int64_t)u * NS * a.ns + s;  // flag (u, i, s) = fbase + i * ns
-  const int c = modp(r - i, P);                     // R_i = A_{i-1}
-  const int64_t c_lo = min((int64_t)c * a.q, a.L), c_hi = min((int64_t)(c + 1) * a.q, a.L);
-  const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-  const int64_t n = hi > lo ? hi - lo : 0;
-  const int64_t off = (base + lo) * es;
-  if (n) {
-    if (i == 0)  // E_0: the user's Pready of S_0
-      warp_copy(a.o_staging + off, a.sendbuf + off, n * es);
-    else if (i <= P - 2)
-      warp_reduce<DT, OP>(a.o_staging + off, nullptr, a.sendbuf + off, a.staging + off, n);
-    else if (i == P - 1)
-      warp_reduce<DT, OP>(a.recvbuf + off, a.o_recvbuf + off, a.sendbuf + off, a.staging + off, n);
-    else
-      warp_copy(a.o_recvbuf + off, a.recvbuf + off, n * es);
-  }
-  warp_signal(a.o_flags + fbase + (int64_t)i * a.ns, e, a.sys);
-}
-
-template <int DT, int OP>
-__device__ __forceinline__ void ring_body(const RingArgs &a, const int gw, const int W) {
-  const int P = a.P, NS = 2 * (P - 1);
-  const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
-  const int64_t es = sizeof(typename Op<DT, OP>::T);
-  if (gw >= a.nunits) return;
-  if (P == 1) {
-    for (int x = gw; x < a.nunits; x += W) {
-      const int u = x / a.ns, s = x % a.ns;
-      if (!warp_wait(a.ready + u, e, a.err, a.timeout_ms, u, false)) return;
-      const int64_t base = (int64_t)u * a.L, lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
-      if (hi > lo && a.sendbuf != a.recvbuf)
-        warp_copy(a.recvbuf + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
-      __syncwarp();
-      if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-    }
-    return;
-  }
-  // the consumer's ready-to-receive (written by a stream memop, never by an engine)
-  if (!warp_wait(a.rtr, e, a.err, a.timeout_ms, -1, a.sys)) return;
-  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
-    int step[kMaxActive];
-    int remaining = 0;
-#pragma unroll
-    for (int j = 0; j < kMaxActive; ++j) {
-      const bool mine = gw + (j0 + j) * W < a.nunits;
-      step[j] = mine ? 0 : NS + 1;
-      remaining += mine;
-    }
-    Idle idle;
-    while (remaining) {
-      bool progressed = false;
-#pragma unroll
-      for (int j = 0; j < kMaxActive; ++j) {
-        if (step[j] > NS) continue;
-        const int x = gw + (j0 + j) * W;
-        const int u = x / a.ns, s = x % a.ns;
-        const int i = step[j];
-        const uint32_t *dep = i == 0 ? a.ready + u : a.flags + ((int64_t)u * NS + (i - 1)) * a.ns + s;
-        if (!warp_poll(dep, e, i != 0 && a.sys)) continue;
-        progressed = true;
-        if (i < NS) {
-          ring_step<DT, OP>(a, u, s, i, e);
-          step[j] = i + 1;
-        } else {  // arrival of the last AG step: partition slice final here
-          if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-          step[j] = NS + 1;
-          --remaining;
-        }
-      }
-      if (progressed)
-        idle.progressed();
-      else if (!idle.wait(a.err, a.timeout_ms, gw))
-        return;
-    }
-  }
-}
-
-// ---------------------------------------------------------------------------
-// Recursive doubling: step k exchanges the whole slice with partner r ^ 2^k
-// (its staging slot k); acc_{k+1} = acc_k ⊕ in_k is written to recv (the
-// accumulator) and pushed to the next partner in the same pass.
-// ---------------------------------------------------------------------------
-template <int DT, int OP>
-__device__ __forceinline__ void rd_body(const RdArgs &a, const int gw, const int W) {
-  const int NS = a.nsteps;
-  const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
-  const int64_t es = sizeof(typename Op<DT, OP>::T);
-  const int64_t stride = (int64_t)a.Np * a.L * es;  // bytes per staging slot
-  uint32_t rtr_ok = 0;
-  for (int x = gw; x < a.nunits; x += W) {
-    const int u = x / a.ns, s = x % a.ns;
-    const int64_t lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
-    const int64_t n = hi > lo ? hi - lo : 0;
-    const int64_t off = ((int64_t)u * a.L + lo) * es;
-    if (!warp_wait(a.ready + u, e, a.err, a.timeout_ms, u, false)) return;
-    if (NS == 0) {
-      if (n && a.sendbuf != a.recvbuf) warp_copy(a.recvbuf + off, a.sendbuf + off, n * es);
-      __syncwarp();
-      if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-      continue;
-    }
-    auto fidx = [&](int k) { return ((int64_t)u * NS + k) * a.ns + s; };
-    if (!(rtr_ok & 1u)) {
-      if (!warp_wait(a.rtr + 0, e, a.err, a.timeout_ms, -1, a.sys)) return;
-      rtr_ok |= 1u;
-    }
-    if (n) warp_copy(a.p_staging[0] + off, a.sendbuf + off, n * es);
-    warp_signal(a.p_flags[0] + fidx(0), e, a.sys);
-    for (int k = 0; k < NS; ++k) {
-      if (!warp_wait(a.flags + fidx(k), e, a.err, a.timeout_ms, u, a.sys)) return;
-      const uint8_t *acc = (k == 0) ? a.sendbuf : a.recvbuf;
-      const uint8_t *in = a.staging + (int64_t)k * stride;
-      if (k < NS - 1) {
-        if (!(rtr_ok & (1u << (k + 1)))) {
-          if (!warp_wait(a.rtr + k + 1, e, a.err, a.timeout_ms, -1, a.sys)) return;
-          rtr_ok |= 1u << (k + 1);
-        }
-        if (n) warp_reduce<DT, OP>(a.recvbuf + off, a.p_staging[k + 1] + off, acc + off, in + off, n);
-        warp_signal(a.p_flags[k + 1] + fidx(k + 1), e, a.sys);
-      } else {
-        if (n) warp_reduce<DT, OP>(a.recvbuf + off, nullptr, acc + off, in + off, n);
-        __syncwarp();
-      }
-    }
-    if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-  }
-}
-
-// ---------------------------------------------------------------------------
-// Direct two-step schedule (generic schedule with neighbour
-// sets).  Unit (u, slice s):
-//   step 0 (after the user's Pready of u): push slice s of chunk o to owner
-//          o's staging slot [u][r] for every peer o, then bump each owner's
-//          phase-0 counter;
-//   step 1 (all P-1 phase-0 arrivals): fold the P contributions of my chunk
-//          in rank order (reading R25) in registers, store the final slice
-//          locally and into every peer's recvbuf, bump their phase-1 counters;
-//   step 2 (all P-1 phase-1 arrivals): slice final everywhere -> done[u].
-// ---------------------------------------------------------------------------
-__device__ __forceinline__ void red_add_scope(uint32_t *p, uint32_t v, bool sys) {
-  if (sys)
-    asm volatile("red.relaxed.sys.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-  else
-    asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-// out_local and out_peer[j] (j < P-1) = fold over k = 0..P-1 of src[k] in rank
-// order; all pointers share one misalignment (scalar head, 16-B body, tail).
-template <int DT, int OP>
-__device__ __forceinline__ void warp_fold_direct(void *out_local, uint8_t *const *out_peer, const uint8_t *const *src,
-                                                 int P, int64_t n) {
-  using O = Op<DT, OP>;
-  using T = typename O::T;
-  const uint32_t lane = threadIdx.x & 31;
-  constexpr int64_t EPV = 16 / sizeof(T);
-  const uintptr_t m = reinterpret_cast<uintptr_t>(out_local) & 15;
-  int64_t head = (int64_t)(((16 - m) & 15) / sizeof(T));
-  if (head > n) head = n;
-  auto scalar = [&](int64_t k) {
-    T acc = __ldcg(reinterpret_cast<const T *>(src[0]) + k);
-    for (int j = 1; j < P; ++j) acc = O::f(acc, __ldcg(reinterpret_cast<const T *>(src[j]) + k));
-    reinterpret_cast<T *>(out_local)[k] = acc;
-    for (int j = 0; j < P - 1; ++j) reinterpret_cast<T *>(out_peer[j])[k] = acc;
-  };
-  for (int64_t k = lane; k < head; k += 32) scalar(k);
-  const int64_t nv = (n - head) / EPV;
-  for (int64_t k = lane; k < nv; k += 32) {
-    const int64_t eo = head + EPV * k;  // element offset
-    uint4 acc = __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(src[0]) + eo));
-    for (int j = 1; j < P; ++j)
-      acc = vop<DT, OP>(acc, __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(src[j]) + eo)));
-    *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(out_local) + eo) = acc;
-    for (int j = 0; j < P - 1; ++j) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(out_peer[j]) + eo) = acc;
-  }
-  for (int64_t k = head + nv * EPV + lane; k < n; k += 32) scalar(k);
-}
-
-template <int DT, int OP>
-__device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W) {
-  const int P = a.P, r = a.r;
-  const uint32_t e = *(const volatile uint32_t *)a.epoch;
-  const int64_t es = sizeof(typename Op<DT, OP>::T);
-  if (gw >= a.nunits) return;
-  if (P == 1) {
-    for (int x = gw; x < a.nunits; x += W) {
-      const int u = x / a.ns, s = x % a.ns;
-      if (!warp_wait(a.ready + u, e, a.err, a.timeout_ms, u, false)) return;
-      const int64_t base = (int64_t)u * a.L, lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
-      if (hi > lo && a.sendbuf != a.recvbuf)
-        warp_copy(a.recvbuf + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
-      __syncwarp();
-      if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-    }
-    return;
-  }
-  for (int j = 0; j < P - 1; ++j)  // every peer has posted ready-to-receive
-    if (!warp_wait(a.rtr + j, e, a.err, a.timeout_ms, -1, a.sys)) return;
-  const uint32_t target = e * (uint32_t)(P - 1);
-  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
-    int step[kMaxActive];
-    int remaining = 0;
-#pragma unroll
-    for (int j = 0; j < kMaxActive; ++j) {
-      const bool mine = gw + (j0 + j) * W < a.nunits;
-      step[j] = mine ? 0 : 3;
-      remaining += mine;
-    }
-    Idle idle;
-    while (remaining) {
-      bool progressed = false;
-#pragma unroll
-      for (int jj = 0; jj < kMaxActive; ++jj) {
-        if (step[jj] > 2) continue;
-        const int x = gw + (j0 + jj) * W;
-        const int u = x / a.ns, s = x % a.ns;
-        const int i = step[jj];
-        const uint32_t *dep = i == 0 ? a.ready + u : a.cnt + ((int64_t)u * 2 + (i - 1)) * a.ns + s;
-        if (!warp_poll(dep, i == 0 ? e : target, i != 0 && a.sys)) continue;
-        progressed = true;
-        const int64_t base = (int64_t)u * a.L;
-        const int64_t mis = base % (16 / es);  // the buffers' misalignment in elements (staging mirrors it)
-        if (i == 0) {
-          for (int j = 0; j < P - 1; ++j) {
-            const int o = (r + 1 + j) % P;
-            const int64_t c_lo = min((int64_t)o * a.q, a.L), c_hi = min((int64_t)(o + 1) * a.q, a.L);
-            const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-            if (hi > lo)
-              warp_copy(a.p_staging[j] + (((int64_t)u * P + r) * a.sq + mis + (int64_t)s * a.qs) * es,
-                        a.sendbuf + (base + lo) * es, (hi - lo) * es);
-          }
-          fence_scope(a.sys);
-          __syncwarp();
-          if ((threadIdx.x & 31) == 0)
-            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 0) * a.ns + s, 1, a.sys);
-          step[jj] = 1;
-        } else if (i == 1) {
-          const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
-          const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-          if (hi > lo) {
-            const uint8_t *src[kMaxDirect];
-            uint8_t *outp[kMaxDirect - 1];
-            for (int k = 0; k < P; ++k)
-              src[k] = k == r ? a.sendbuf + (base + lo) * es
-                              : a.staging + (((int64_t)u * P + k) * a.sq + mis + (int64_t)s * a.qs) * es;
-            for (int j = 0; j < P - 1; ++j) outp[j] = a.p_recvbuf[j] + (base + lo) * es;
-            warp_fold_direct<DT, OP>(a.recvbuf + (base + lo) * es, outp, src, P, hi - lo);
-          }
-          fence_scope(a.sys);
-          __syncwarp();
-          if ((threadIdx.x & 31) == 0)
-            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
-          step[jj] = 2;
-        } else {
-          if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-          step[jj] = 3;
-          --remaining;
-        }
-      }
-      if (progressed)
-        idle.progressed();
-      else if (!idle.wait(a.err, a.timeout_ms, gw))
-        return;
-    }
-  }
-}
-
-template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) direct_engine(DirectArgs a) {
-  direct_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
-}
-template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) direct_engine_group(DirectGroupArgs g) {
-  int k = 0;
-  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
-  const int b = blockIdx.x - g.block_start[k];
-  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
-  direct_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
-}
-
-// Single-rank launches (one rank per GPU / process).
-template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) ring_engine(RingArgs a) {
-  ring_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
-}
-template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) rd_engine(RdArgs a) {
-  rd_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
-}
-
-// Grouped launches: the engines of every rank that shares this GPU inside one
-// process (virtual ranks) run as ONE kernel, so they are co-resident by
-// construction and no engine can sit behind another in a hardware queue
-// (DESIGN.md §"Virtual ranks").  Block b belongs to the rank whose block range
-// contains it; warps are numbered within that rank exactly as in the
-// single-rank launch.
-template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) ring_engine_group(RingGroupArgs g) {
-  int k = 0;
-  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
-  const int b = blockIdx.x - g.block_start[k];
-  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
-  ring_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
-}
-template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) rd_engine_group(RdGroupArgs g) {
-  int k = 0;
-  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
-  const int b = blockIdx.x - g.block_start[k];
-  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
-  rd_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
-}
 
 // ---------------------------------------------------------------------------
 // ENGINE copy mode of partitioned send: unit = (transport partition t, slice s).
@@ -719,14 +124,18 @@ __global__ void pready_range_kernel(pc_prequest_t q, int lo, int hi) {
   for (int p = lo + gw; p <= hi; p += W) pc_pready_warp(p, q);
 }
 
+}  // namespace
+
+
+// (dtype, op) -> the EngineLaunch instantiation compiled in engine_inst.cu
 template <typename F>
-int dispatch(int dtype, int op, F f) {
+static int dispatch(int dtype, int op, F f) {
   using std::integral_constant;
-#define PC_DISPATCH_OPS(DTV)                                                            \
-  do {                                                                                  \
-    if (op == PC_OP_SUM) return f(integral_constant<int, DTV>(), integral_constant<int, 0>()); \
-    if (op == PC_OP_MAX) return f(integral_constant<int, DTV>(), integral_constant<int, 1>()); \
-    return f(integral_constant<int, DTV>(), integral_constant<int, 2>());               \
+#define PC_DISPATCH_OPS(DTV)                                                                    \
+  do {                                                                                          \
+    if (op == PC_OP_SUM) return f(EngineLaunch<DTV, 0>());                                      \
+    if (op == PC_OP_MAX) return f(EngineLaunch<DTV, 1>());                                      \
+    return f(EngineLaunch<DTV, 2>());                                                           \
   } while (0)
   switch (dtype) {
     case PC_INT32: PC_DISPATCH_OPS(0);
@@ -740,30 +149,16 @@ int dispatch(int dtype, int op, F f) {
 
 std::atomic<uint64_t> g_launches{0};
 
-int grid_for(int warps, int nunits) {
-  int w = warps < nunits ? warps : nunits;
-  if (w < 1) w = 1;
-  return (w * 32 + kEngineBlock - 1) / kEngineBlock;
-}
-
-}  // namespace
-
 int launch_ring_engine(const RingArgs &a, int warps, cudaStream_t s) {
-  return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
-    ring_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
-    g_launches++;
-    PC_CUDA(cudaGetLastError());
-    return 0;
-  });
+  return dispatch(a.dtype, a.op, [&](auto E) { return decltype(E)::ring(a, warps, s); });
 }
 
 int launch_rd_engine(const RdArgs &a, int warps, cudaStream_t s) {
-  return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
-    rd_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
-    g_launches++;
-    PC_CUDA(cudaGetLastError());
-    return 0;
-  });
+  return dispatch(a.dtype, a.op, [&](auto E) { return decltype(E)::rd(a, warps, s); });
+}
+
+int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s) {
+  return dispatch(a.dtype, a.op, [&](auto E) { return decltype(E)::direct(a, warps, s); });
 }
 
 int launch_ring_engine_group(const RingGroupArgs &g, int warps, cudaStream_t s) {
@@ -773,12 +168,7 @@ int launch_ring_engine_group(const RingGroupArgs &g, int warps, cudaStream_t s) 
     h.block_start[k] = blocks;
     blocks += grid_for(warps, g.a[k].nunits);
   }
-  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
-    ring_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
-    g_launches++;
-    PC_CUDA(cudaGetLastError());
-    return 0;
-  });
+  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto E) { return decltype(E)::ring_group(h, blocks, s); });
 }
 
 int launch_rd_engine_group(const RdGroupArgs &g, int warps, cudaStream_t s) {
@@ -788,21 +178,7 @@ int launch_rd_engine_group(const RdGroupArgs &g, int warps, cudaStream_t s) {
     h.block_start[k] = blocks;
     blocks += grid_for(warps, g.a[k].nunits);
   }
-  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
-    rd_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
-    g_launches++;
-    PC_CUDA(cudaGetLastError());
-    return 0;
-  });
-}
-
-int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s) {
-  return dispatch(a.dtype, a.op, [&](auto DT, auto OP) {
-    direct_engine<decltype(DT)::value, decltype(OP)::value><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
-    g_launches++;
-    PC_CUDA(cudaGetLastError());
-    return 0;
-  });
+  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto E) { return decltype(E)::rd_group(h, blocks, s); });
 }
 
 int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t s) {
@@ -812,12 +188,7 @@ int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t
     h.block_start[k] = blocks;
     blocks += grid_for(warps, g.a[k].nunits);
   }
-  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto DT, auto OP) {
-    direct_engine_group<decltype(DT)::value, decltype(OP)::value><<<blocks, kEngineBlock, 0, s>>>(h);
-    g_launches++;
-    PC_CUDA(cudaGetLastError());
-    return 0;
-  });
+  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto E) { return decltype(E)::direct_group(h, blocks, s); });
 }
 
 int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
@@ -889,12 +260,6 @@ int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s) {
 
 uint64_t launch_count() { return g_launches.load(); }
 
-int engine_occupancy_ctas_per_sm(int *ctas) {
-  int a = 0, b = 0;
-  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, ring_engine<1, 0>, kEngineBlock, 0));
-  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, rd_engine<1, 0>, kEngineBlock, 0));
-  *ctas = a < b ? a : b;
-  return 0;
-}
+int engine_occupancy_ctas_per_sm(int *ctas) { return EngineLaunch<1, 0>::occupancy(ctas); }
 
 }  // namespace pc
