@@ -183,11 +183,14 @@ def run_reference(args):
 
 
 # --------------------------------------------------------------------------- GPU legs
-def latency_pair(pc, apps, torch, comms, iters=5000, payload=0):
-    """Pready->Parrived ping-pong between two ranks inside one launch."""
+def latency_pair(pc, apps, torch, comms, iters=5000, payload=0, copy=None):
+    """Pready->Parrived ping-pong between two ranks inside one launch
+    (warp-granularity Pready; copy = INLINE flag+fence or LL lines)."""
+    copy = pc.COPY_INLINE if copy is None else copy
     cnt = payload // 4
     st = torch.cuda.Stream()
     bufs = [torch.zeros(max(iters * cnt, 4), device="cuda") for _ in range(4)]
+    bufs[0].copy_(torch.arange(bufs[0].numel(), dtype=torch.float32))
     a2b = pc.psend_init(bufs[0], iters, cnt, pc.FLOAT32, 1, 101, comms[0])
     b_in = pc.precv_init(bufs[1], iters, cnt, pc.FLOAT32, 0, 101, comms[1])
     b2a = pc.psend_init(bufs[2], iters, cnt, pc.FLOAT32, 0, 102, comms[1])
@@ -195,8 +198,8 @@ def latency_pair(pc, apps, torch, comms, iters=5000, payload=0):
     for q in (a2b, a_in, b_in, b2a):
         q.start(st)
     pc.run_ranks([lambda: [q.pbuf_prepare(st) for q in (a2b, a_in)], lambda: [q.pbuf_prepare(st) for q in (b_in, b2a)]])
-    pa, pai = a2b.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE), a_in.prequest_create(pc.GRAN_WARP, 1, 0)
-    pb, pbi = b2a.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE), b_in.prequest_create(pc.GRAN_WARP, 1, 0)
+    pa, pai = a2b.prequest_create(pc.GRAN_WARP, 1, copy), a_in.prequest_create(pc.GRAN_WARP, 1, 0)
+    pb, pbi = b2a.prequest_create(pc.GRAN_WARP, 1, copy), b_in.prequest_create(pc.GRAN_WARP, 1, 0)
     t = torch.zeros(2, dtype=torch.int64, device="cuda")
     rt = torch.zeros(iters, dtype=torch.int64, device="cuda")
     apps.pingpong_pair(pa, pai, pb, pbi, iters, apps.GRAN_WARP, t, st, rt_ns=rt)
@@ -214,8 +217,10 @@ def latency_pair(pc, apps, torch, comms, iters=5000, payload=0):
     for q in (a2b, a_in, b_in, b2a):
         q.free()
     import numpy as np
+    ok = bool(torch.equal(bufs[1], bufs[0])) if cnt else True
     return {"p50": float(np.percentile(rts, 50)), "p99": float(np.percentile(rts, 99)),
             "mean": float(rts.mean()), "payload_bytes": payload, "iters": iters, "errors": errs,
+            "copy": {0: "inline", 2: "ll"}.get(copy, copy), "payload_ok": ok,
             "bare_flag_floor_mean": bare, "frac_of_floor": bare / float(np.percentile(rts, 50))}
 
 
@@ -463,6 +468,9 @@ def run_virtual(args):
         g2, c2 = pc.local_comms(2, 0)  # the exchange of new requests is collective over the comm
         lat = {"flag_only": latency_pair(pc, apps, torch, c2, payload=0),
                "8B": latency_pair(pc, apps, torch, c2, payload=8),
+               "ll_flag_only": latency_pair(pc, apps, torch, c2, payload=0, copy=pc.COPY_LL),
+               "ll_8B": latency_pair(pc, apps, torch, c2, payload=8, copy=pc.COPY_LL),
+               "ll_256B": latency_pair(pc, apps, torch, c2, payload=256, copy=pc.COPY_LL),
                "note": "2 virtual ranks on one B200 (flags/payload in the same HBM/L2, not NVLink)"}
         for c in c2:
             c.destroy()

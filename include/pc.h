@@ -46,11 +46,20 @@ typedef enum { PC_OP_SUM = 0, PC_OP_MAX = 1, PC_OP_MIN = 2 } pc_op_t;
 /* Granularity of the device Pready call: informational — the device
  * function chosen (pc_pready / _warp / _block) decides who participates. */
 typedef enum { PC_GRAN_THREAD = 0, PC_GRAN_WARP = 1, PC_GRAN_BLOCK = 2 } pc_gran_t;
-/* Copy mechanism: INLINE = "Kernel Copy" — the contributor that
- * completes a transport partition pushes it over NVLink from inside the user
- * kernel; ENGINE = persistent library warps poll ready flags and push (the
- * GPU-resident replacement of the paper's host Progression Engine). */
-typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1 } pc_copy_t;
+/* Copy mechanism: INLINE = "Kernel Copy" — every contributor
+ * pushes its partition over NVLink from inside the user kernel and the one
+ * that completes a transport partition stores its flag; ENGINE = persistent
+ * library warps poll ready flags and push (the GPU-resident replacement of the
+ * paper's host Progression Engine); LL = Kernel Copy in 16-B lines that carry
+ * the epoch next to every 8 payload bytes (NCCL-LL-style), so a partition
+ * needs no fence and no separate flag and Pready->Parrived is one store's
+ * flight.  LL is available when part_bytes <= PC_LL_MAX_PART_BYTES and the
+ * buffer <= PC_LL_MAX_TOTAL_BYTES (else pc_prequest_create returns
+ * PC_ERR_UNSUPPORTED); aggregation then only batches the sender's completion
+ * accounting (each partition's lines are self-validating). */
+typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1, PC_COPY_LL = 2 } pc_copy_t;
+#define PC_LL_MAX_PART_BYTES 1024
+#define PC_LL_MAX_TOTAL_BYTES (16u << 20)
 /* Allreduce schedule (§IV-B).  RING = Alg 1; RD = recursive
  * doubling (BASELINE north_star; not in the paper; P a power of two);
  * DIRECT = two steps over neighbour SETS (the generic schedule of P:L155 with

@@ -6,6 +6,7 @@
  *   PC_DEVICE int  pc_pready_block(int partition, pc_prequest_t preq);  block-collective
  *   PC_DEVICE int  pc_parrived    (pc_prequest_t preq, int partition);
  *   PC_DEVICE int  pc_wait_arrived(pc_prequest_t preq, int partition);
+ *   PC_DEVICE int  pc_parrived_warp / pc_wait_arrived_warp(preq, partition);  warp-collective
  *
  * Paper: MPIX_Pready / MPIX_Pready_{thread,warp,block} / MPIX_Parrived
  * (Listing 2; §IV-A4).  PC_DEVICE plays the role of
@@ -252,6 +253,152 @@ PC_DEVICE uint2 epoch_rtr(const pc_prequest_t &q) {
   return q.sys_scope ? ld_acquire_sys_v2(q.epoch) : ld_acquire_gpu_v2(q.epoch);
 }
 
+/* The epoch alone, relaxed: for a Pready that moves no bytes (flag-only
+ * partitions, ENGINE mode) there is no receiver buffer to protect, so no
+ * ready-to-receive check and no acquire (an acquire also invalidates L1). */
+PC_DEVICE uint32_t epoch_relaxed(const pc_prequest_t &q) { return ld_relaxed_sys(q.epoch); }
+
+/* ------------------------------------------------------------ LL lines
+ * PC_COPY_LL: payload byte 8j..8j+7 of user partition p travels in line j =
+ * {d0, e, d1, e} (d0/d1 = payload bytes 0-3 / 4-7, little endian), stored as
+ * ONE st.relaxed.v2.u64 whose two 8-byte elements are each single-copy atomic:
+ * a reader that sees e in both halves has this epoch's 8 bytes.  Lines live in
+ * the receiver's control block, [epoch parity][partition][line]. */
+PC_DEVICE void st_ll(uint8_t *dst, uint64_t lo, uint64_t hi, uint32_t sys) {
+  if (sys)
+    asm volatile("st.relaxed.sys.global.v2.u64 [%0], {%1, %2};" ::"l"(dst), "l"(lo), "l"(hi) : "memory");
+  else
+    asm volatile("st.relaxed.gpu.global.v2.u64 [%0], {%1, %2};" ::"l"(dst), "l"(lo), "l"(hi) : "memory");
+}
+PC_DEVICE ulonglong2 ld_ll(const uint8_t *src, uint32_t sys) {
+  ulonglong2 v;
+  if (sys)
+    asm volatile("ld.relaxed.sys.global.v2.u64 {%0, %1}, [%2];" : "=l"(v.x), "=l"(v.y) : "l"(src) : "memory");
+  else
+    asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(v.x), "=l"(v.y) : "l"(src) : "memory");
+  return v;
+}
+/* n (1..8) payload bytes at s, little endian, zero-padded */
+PC_DEVICE uint64_t ld_payload8(const uint8_t *s, uint32_t n) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(s);
+  if (n == 8 && (a & 7) == 0) return *reinterpret_cast<const uint64_t *>(s);
+  if ((a & 3) == 0 && (n & 3) == 0) {
+    const uint64_t lo = *reinterpret_cast<const uint32_t *>(s);
+    return n == 8 ? lo | ((uint64_t)(*reinterpret_cast<const uint32_t *>(s + 4)) << 32) : lo;
+  }
+  uint64_t v = 0;
+  for (uint32_t b = 0; b < n; ++b) v |= (uint64_t)s[b] << (8 * b);
+  return v;
+}
+PC_DEVICE void st_payload8(uint8_t *d, uint64_t v, uint32_t n) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(d);
+  if (n == 8 && (a & 7) == 0) {
+    *reinterpret_cast<uint64_t *>(d) = v;
+  } else if ((a & 3) == 0 && (n & 3) == 0) {
+    *reinterpret_cast<uint32_t *>(d) = (uint32_t)v;
+    if (n == 8) *reinterpret_cast<uint32_t *>(d + 4) = (uint32_t)(v >> 32);
+  } else {
+    for (uint32_t b = 0; b < n; ++b) d[b] = (uint8_t)(v >> (8 * b));
+  }
+}
+PC_DEVICE uint32_t ll_nbytes(uint64_t part_bytes, uint32_t j) {
+  const uint64_t o = 8ull * j;
+  return o < part_bytes ? (uint32_t)(part_bytes - o < 8 ? part_bytes - o : 8) : 0u;
+}
+
+/* Sender: participant idx of n pushes lines idx, idx+n, ... of partition p and
+ * returns the epoch.  The first payload load is issued BEFORE the epoch read so
+ * the two round trips overlap, and neither is an acquire.  Ready-to-receive is
+ * not checked here: the line area of parity e&1 was last read by the receiver
+ * in epoch e-2, and the sender's completion of epoch e-1 (pc_wait / pc_test /
+ * pc_wait_on_stream) already acquired rtr >= e-1, i.e. the receiver had
+ * finished epoch e-2 — the stream order from that wait to this epoch's kernels
+ * carries the ordering (R29). */
+PC_DEVICE uint32_t ll_push(const pc_prequest_t &q, int p, uint32_t idx, uint32_t n) {
+  const uint32_t nl = q.ll_lines;
+  const uint64_t pb = q.part_bytes;
+  const uint8_t *src = q.sbuf + (uint64_t)p * pb;
+  uint64_t d = 0;
+  if (idx < nl) {
+    const uint32_t nb = ll_nbytes(pb, idx);
+    if (nb) d = ld_payload8(src + 8ull * idx, nb);
+  }
+  const uint32_t e = epoch_relaxed(q);
+  uint8_t *dst = q.peer_ll + ((uint64_t)(e & 1) * (uint64_t)q.partitions + (uint64_t)p) * nl * 16ull;
+  const uint64_t eh = (uint64_t)e << 32;
+  for (uint32_t j = idx; j < nl; j += n) {
+    if (j != idx) {
+      const uint32_t nb = ll_nbytes(pb, j);
+      d = nb ? ld_payload8(src + 8ull * j, nb) : 0;
+    }
+    st_ll(dst + 16ull * j, (d & 0xffffffffull) | eh, (d >> 32) | eh, q.sys_scope);
+  }
+  return e;
+}
+
+/* Receiver: 1 iff every line of partition p carries epoch e; then the payload
+ * is unpacked into recvbuf (by the calling thread). */
+PC_DEVICE bool ll_consume(const pc_prequest_t &q, int p, uint32_t e) {
+  const uint32_t nl = q.ll_lines;
+  const uint64_t pb = q.part_bytes;
+  const uint8_t *lines = q.ll + ((uint64_t)(e & 1) * (uint64_t)q.partitions + (uint64_t)p) * nl * 16ull;
+  uint8_t *dst = q.rbuf + (uint64_t)p * pb;
+  for (uint32_t j0 = 0; j0 < nl; j0 += 8) {
+    const uint32_t m = nl - j0 < 8 ? nl - j0 : 8;
+    ulonglong2 v[8];
+#pragma unroll
+    for (uint32_t k = 0; k < 8; ++k)
+      if (k < m) v[k] = ld_ll(lines + 16ull * (j0 + k), q.sys_scope);
+#pragma unroll
+    for (uint32_t k = 0; k < 8; ++k)
+      if (k < m && ((uint32_t)(v[k].x >> 32) != e || (uint32_t)(v[k].y >> 32) != e)) return false;
+#pragma unroll
+    for (uint32_t k = 0; k < 8; ++k)
+      if (k < m) {
+        const uint32_t nb = ll_nbytes(pb, j0 + k);
+        if (nb) st_payload8(dst + 8ull * (j0 + k), (v[k].x & 0xffffffffull) | (v[k].y << 32), nb);
+      }
+  }
+  return true;
+}
+
+/* Warp-collective receiver (all 32 lanes): lane l loads lines l, l+32, l+64,
+ * l+96 of the partition in one round trip, the warp votes, every lane unpacks
+ * its lines.  Returns the same value on every lane. */
+PC_DEVICE bool ll_consume_warp(const pc_prequest_t &q, int p, uint32_t e, uint32_t lane) {
+  const uint32_t nl = q.ll_lines;
+  const uint64_t pb = q.part_bytes;
+  const uint8_t *lines = q.ll + ((uint64_t)(e & 1) * (uint64_t)q.partitions + (uint64_t)p) * nl * 16ull;
+  uint8_t *dst = q.rbuf + (uint64_t)p * pb;
+  for (uint32_t j0 = 0; j0 < nl; j0 += 128) {
+    ulonglong2 v[4];
+    bool ok = true;
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      const uint32_t j = j0 + 32 * k + lane;
+      if (j < nl) v[k] = ld_ll(lines + 16ull * j, q.sys_scope);
+    }
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      const uint32_t j = j0 + 32 * k + lane;
+      if (j < nl) ok = ok && (uint32_t)(v[k].x >> 32) == e && (uint32_t)(v[k].y >> 32) == e;
+    }
+    if (!__all_sync(0xffffffffu, ok)) return false;
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      const uint32_t j = j0 + 32 * k + lane;
+      const uint32_t nb = j < nl ? ll_nbytes(pb, j) : 0u;
+      if (nb) st_payload8(dst + 8ull * j, (v[k].x & 0xffffffffull) | (v[k].y << 32), nb);
+    }
+  }
+  return true;
+}
+
+/* Sender completion accounting of an LL Pready (the receiver needs no flag). */
+PC_DEVICE void ll_account(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, int part) {
+  if (contribute(q, t, add, e, part)) st_relaxed_gpu(q.sent + t, e);
+}
+
 }  // namespace pc_detail
 
 /* ------------------------------------------------------------------ Pready */
@@ -278,11 +425,21 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
   const int t = partition / preq.agg;
   const unsigned grp = __match_any_sync(mask, t);
   const uint32_t leader = __ffs(grp) - 1;
+  if (preq.copy == 2) {  // LL: this lane pushes its partition's lines itself
+    const uint32_t e = ll_push(preq, partition, 0, 1);
+    __syncwarp(mask);
+    if (lane == leader) ll_account(preq, t, __popc(grp), e, partition);
+    return 0;
+  }
   uint32_t e = 0, rtr0 = 0;
   if (lane == first) {
-    const uint2 er = epoch_rtr(preq);
-    e = er.x;
-    rtr0 = er.y;
+    if (preq.copy == 0 && preq.part_bytes) {
+      const uint2 er = epoch_rtr(preq);
+      e = er.x;
+      rtr0 = er.y;
+    } else {
+      e = epoch_relaxed(preq);
+    }
   }
   e = __shfl_sync(mask, e, first);
   if (preq.copy == 1) {  // ENGINE
@@ -324,27 +481,38 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
     return 0;
   }
   const int t = partition / preq.agg;
+  if (preq.copy == 2) {  // LL: every lane loads its line, reads the epoch and stores (no broadcast)
+    const uint32_t e = ll_push(preq, partition, lane, 32);
+    __syncwarp(full);
+    if (lane == 0) ll_account(preq, t, 1, e, partition);
+    __syncwarp(full);
+    return 0;
+  }
+  if (preq.copy == 1 || preq.part_bytes == 0) {  // no bytes for this warp to move: lane 0 alone
+    if (lane == 0) {
+      const uint32_t e = epoch_relaxed(preq);
+      if (preq.copy == 1) {
+        if (contribute(preq, t, 1, e, partition)) st_release_gpu(preq.ready + t, e);
+      } else {
+        publish(preq, t, 1, e, partition);
+      }
+    }
+    __syncwarp(full);
+    return 0;
+  }
   uint32_t e = 0;
   bool ok = true;
   if (lane == 0) {
     const uint2 er = epoch_rtr(preq);
     e = er.x;
-    if (preq.copy == 0 && preq.part_bytes && !reached(er.y, e))
-      ok = spin_geq<true>(preq.rtr, e, preq.err, preq.timeout_ms, partition);
+    if (!reached(er.y, e)) ok = spin_geq<true>(preq.rtr, e, preq.err, preq.timeout_ms, partition);
   }
   e = __shfl_sync(full, e, 0);
   if (!__shfl_sync(full, ok, 0)) return PC_DEV_ERR_TIMEOUT;
-  if (preq.copy == 1) {  // ENGINE
-    if (lane == 0 && contribute(preq, t, 1, e, partition)) st_release_gpu(preq.ready + t, e);
-    __syncwarp(full);
-    return 0;
-  }
-  if (preq.part_bytes) {
-    const uint64_t off = (uint64_t)partition * preq.part_bytes;
-    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, lane, 32);
-    fence_scope(preq.sys_scope);
-    __syncwarp(full);
-  }
+  const uint64_t off = (uint64_t)partition * preq.part_bytes;
+  copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, lane, 32);
+  fence_scope(preq.sys_scope);
+  __syncwarp(full);
   if (lane == 0) publish(preq, t, 1, e, partition);
   __syncwarp(full);
   return 0;
@@ -369,26 +537,36 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
     return 0;
   }
   const int t = partition / preq.agg;
+  if (preq.copy == 2) {  // LL: every thread pushes its lines
+    const uint32_t e = ll_push(preq, partition, tid, nthr);
+    __syncthreads();
+    if (tid == 0) ll_account(preq, t, 1, e, partition);
+    return 0;
+  }
+  if (preq.copy == 1 || preq.part_bytes == 0) {  // no bytes for this block to move: thread 0 alone
+    if (tid == 0) {
+      const uint32_t e = epoch_relaxed(preq);
+      if (preq.copy == 1) {
+        if (contribute(preq, t, 1, e, partition)) st_release_gpu(preq.ready + t, e);
+      } else {
+        publish(preq, t, 1, e, partition);
+      }
+    }
+    return 0;
+  }
   if (tid == 0) {
     const uint2 er = epoch_rtr(preq);
     s_e = er.x;
     s_ok = 1;
-    if (preq.copy == 0 && preq.part_bytes && !reached(er.y, er.x))
-      s_ok = spin_geq<true>(preq.rtr, er.x, preq.err, preq.timeout_ms, partition);
+    if (!reached(er.y, er.x)) s_ok = spin_geq<true>(preq.rtr, er.x, preq.err, preq.timeout_ms, partition);
   }
   __syncthreads();
   const uint32_t e = s_e;
   if (!s_ok) return PC_DEV_ERR_TIMEOUT;
-  if (preq.copy == 1) {  // ENGINE
-    if (tid == 0 && contribute(preq, t, 1, e, partition)) st_release_gpu(preq.ready + t, e);
-    return 0;
-  }
-  if (preq.part_bytes) {
-    const uint64_t off = (uint64_t)partition * preq.part_bytes;
-    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, tid, nthr);
-    fence_scope(preq.sys_scope);
-    __syncthreads();
-  }
+  const uint64_t off = (uint64_t)partition * preq.part_bytes;
+  copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, tid, nthr);
+  fence_scope(preq.sys_scope);
+  __syncthreads();
   if (tid == 0) publish(preq, t, 1, e, partition);
   return 0;
 }
@@ -405,6 +583,7 @@ PC_DEVICE int pc_parrived(pc_prequest_t preq, int partition) {
   }
   const uint32_t g = *(const volatile uint32_t *)preq.layout;
   if (g == 0) return 0;  // sender has not published its transport layout yet
+  if (g & PC_LAYOUT_LL) return ll_consume(preq, partition, e) ? 1 : 0;
   return reached(ld_acquire_scope(preq.flags + partition / (int)g, preq.sys_scope), e);
 }
 
@@ -437,6 +616,20 @@ PC_DEVICE int pc_wait_arrived(pc_prequest_t preq, int partition) {
         __nanosleep(256);
       }
     }
+    if (g & PC_LAYOUT_LL) {  // poll the partition's lines themselves
+      n = 0;
+      while (!ll_consume(preq, partition, e)) {
+        if ((++n & 127) == 0) {
+          if (aborted(preq.err)) return PC_DEV_ERR_TIMEOUT;
+          if (preq.timeout_ms && globaltimer() - t0 > (uint64_t)preq.timeout_ms * 1000000ull) {
+            set_error(preq.err, PC_DEV_ERR_TIMEOUT, partition);
+            return PC_DEV_ERR_TIMEOUT;
+          }
+          if (n > 4096) __nanosleep(128);
+        }
+      }
+      return 0;
+    }
     w = preq.flags + partition / (int)g;
     sys = preq.sys_scope != 0;
   }
@@ -454,6 +647,58 @@ PC_DEVICE int pc_wait_arrived(pc_prequest_t preq, int partition) {
     }
   }
   return 0;
+}
+
+/* Warp-collective Parrived / wait: all 32 lanes call it with the same
+ * partition (like pc_pready_warp) and all get the result.  For an LL receive
+ * the lanes poll and unpack the partition's lines together (one round trip per
+ * poll for partitions up to 2 KiB of lines); otherwise lane 0 polls the flag.
+ * After it returns, every lane may read the partition. */
+PC_DEVICE int pc_parrived_warp(pc_prequest_t preq, int partition) {
+  using namespace pc_detail;
+  const uint32_t lane = lane_id();
+  if (preq.kind == PC_KIND_PRECV && partition >= 0 && partition < preq.partitions) {
+    const uint32_t g = *(const volatile uint32_t *)preq.layout;
+    if (g & PC_LAYOUT_LL) return ll_consume_warp(preq, partition, epoch_of(preq), lane) ? 1 : 0;
+  }
+  int r = 0;
+  if (lane == 0) r = pc_parrived(preq, partition);
+  r = __shfl_sync(0xffffffffu, r, 0);
+  return r;
+}
+
+PC_DEVICE int pc_wait_arrived_warp(pc_prequest_t preq, int partition) {
+  using namespace pc_detail;
+  const unsigned full = 0xffffffffu;
+  const uint32_t lane = lane_id();
+  if (preq.kind == PC_KIND_PRECV && partition >= 0 && partition < preq.partitions) {
+    const uint32_t e = epoch_of(preq);
+    uint32_t g = *(const volatile uint32_t *)preq.layout;
+    if (g & PC_LAYOUT_LL) {
+      const uint64_t t0 = globaltimer();
+      uint32_t n = 0;
+      while (!ll_consume_warp(preq, partition, e, lane)) {
+        if ((++n & 127) == 0) {
+          int stop = 0;
+          if (lane == 0) {
+            if (aborted(preq.err)) {
+              stop = 1;
+            } else if (preq.timeout_ms && globaltimer() - t0 > (uint64_t)preq.timeout_ms * 1000000ull) {
+              set_error(preq.err, PC_DEV_ERR_TIMEOUT, partition);
+              stop = 1;
+            }
+          }
+          if (__shfl_sync(full, stop, 0)) return PC_DEV_ERR_TIMEOUT;
+          if (n > 4096) __nanosleep(128);
+        }
+      }
+      return 0;
+    }
+  }
+  int r = 0;
+  if (lane == 0) r = pc_wait_arrived(preq, partition);
+  r = __shfl_sync(full, r, 0);
+  return r;
 }
 
 #endif /* PC_DEVICE_CUH_ */

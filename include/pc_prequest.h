@@ -46,6 +46,18 @@ struct pc_prequest_s {
                                  acquires; 0: every peer shares this GPU -> GPU scope
                                  (a system-scope fence costs ~1.5 us on B200)           */
   int32_t *err;               /* sticky device error word [2] = {code, partition}         */
+  /* LL line protocol (PC_COPY_LL): every 8 payload bytes travel
+   * with the epoch in one 16-B line {d0, e, d1, e} (two single-copy-atomic
+   * 8-B halves), so a line is its own arrival flag: no fence, no flag store. */
+  uint32_t ll_lines;          /* 16-B lines per user partition = max(1, ceil(part_bytes/8)),
+                                 0 = the request has no LL area                            */
+  uint32_t ll_pad;
+  uint8_t *peer_ll;           /* send, PC_COPY_LL: receiver's LL area (peer-mapped)        */
+  uint8_t *ll;                /* receive: own LL area [2 epoch parities][N_p][ll_lines]   */
+  uint8_t *rbuf;              /* receive: own recv buffer (LL lines are unpacked into it) */
 };
+
+/* Receive side: bit 31 of the layout word = the sender pushes LL lines. */
+#define PC_LAYOUT_LL 0x80000000u
 
 #endif /* PC_PREQUEST_H_ */

@@ -157,9 +157,14 @@ __global__ void pingpong_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, p
   const pc_prequest_t &rq = side ? recvB : recvA;
   const uint64_t t0 = pc_detail::globaltimer();
   uint64_t tk = t0;
+  // warp granularity: warp-collective Pready and wait; thread: lane 0 alone
   for (int k = 0; k < iters; ++k) {
     if (side == 1) {
-      if (threadIdx.x == 0) pc_wait_arrived(rq, k);
+      if (gran == PCAPP_GRAN_THREAD) {
+        if (threadIdx.x == 0) pc_wait_arrived(rq, k);
+      } else {
+        pc_wait_arrived_warp(rq, k);
+      }
       __syncwarp();
     }
     if (gran == PCAPP_GRAN_THREAD) {
@@ -168,8 +173,12 @@ __global__ void pingpong_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, p
       pc_pready_warp(k, sq);
     }
     if (side == 0) {
+      if (gran == PCAPP_GRAN_THREAD) {
+        if (threadIdx.x == 0) pc_wait_arrived(rq, k);
+      } else {
+        pc_wait_arrived_warp(rq, k);
+      }
       if (threadIdx.x == 0) {
-        pc_wait_arrived(rq, k);
         const uint64_t t = pc_detail::globaltimer();
         if (rt_ns) rt_ns[k] = t - tk;  // one round trip = two Pready->Parrived hops
         tk = t;
@@ -214,7 +223,9 @@ __global__ void lat_probe_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, 
   const pc_prequest_t &rq = side ? recvB : recvA;
   const uint32_t e = pc_detail::epoch_of(sq);
   auto wait = [&](int k) {
-    if (threadIdx.x == 0) {
+    if (WLIB == 2) {
+      pc_wait_arrived_warp(rq, k);
+    } else if (threadIdx.x == 0) {
       if (WLIB) {
         pc_wait_arrived(rq, k);
       } else {
@@ -244,6 +255,18 @@ __global__ void lat_probe_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, 
       if (threadIdx.x == 0) ee = pc_detail::epoch_rtr(sq).x;
       ee = __shfl_sync(0xffffffffu, ee, 0);
       if (threadIdx.x == 0) pc_detail::publish(sq, k / sq.agg, 1, ee, k);
+      __syncwarp();
+    } else if (PLIB >= 10) {  // lane 0: epoch load variant + publish
+      __syncwarp();
+      if (threadIdx.x == 0) {
+        uint32_t ee;
+        if (PLIB == 10) ee = pc_detail::ld_acquire_gpu(sq.epoch);
+        else if (PLIB == 11) ee = pc_detail::ld_acquire_sys(sq.epoch);
+        else if (PLIB == 12) asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(ee) : "l"(sq.epoch) : "memory");
+        else if (PLIB == 13) ee = pc_detail::ld_acquire_sys_v2(sq.epoch).x;
+        else ee = pc_detail::ld_acquire_gpu_v2(sq.epoch).x;
+        pc_detail::publish(sq, k / sq.agg, 1, ee, k);
+      }
       __syncwarp();
     } else if (PLIB == 5) {  // relaxed epoch read by lane 0 + publish
       __syncwarp();
@@ -442,7 +465,13 @@ int pcapp_lat_probe_pair(const pc_prequest_t *sendA, const pc_prequest_t *recvA,
     case 5: PCAPP_LP(0, 2); break;
     case 6: PCAPP_LP(1, 3); break;
     case 7: PCAPP_LP(1, 4); break;
-    default: PCAPP_LP(1, 5); break;
+    case 8: PCAPP_LP(1, 5); break;
+    case 9: PCAPP_LP(2, 1); break;
+    case 10: PCAPP_LP(1, 10); break;
+    case 11: PCAPP_LP(1, 11); break;
+    case 12: PCAPP_LP(1, 12); break;
+    case 13: PCAPP_LP(1, 13); break;
+    default: PCAPP_LP(1, 14); break;
   }
 #undef PCAPP_LP
   return cudaGetLastError() == cudaSuccess ? 0 : -2;

@@ -323,9 +323,14 @@ static void fill_prequest(Request *q, pc_prequest_t *o) {
   o->done_mul = (uint32_t)q->slices;
   o->sys_scope = (uint32_t)q->sys_scope;
   o->err = (int32_t *)(q->ctrl + q->L.err);
+  o->ll_lines = q->ll_lines;
   if (q->kind == PC_KIND_PSEND) {
     o->peer_rbuf = q->peer_buf;
     o->peer_flags = q->peer_ctrl ? q->peer_ctrl + q->L.flags : nullptr;
+    o->peer_ll = (q->peer_ctrl && q->ll_lines) ? (uint8_t *)(q->peer_ctrl + q->L.ll) : nullptr;
+  } else if (q->kind == PC_KIND_PRECV) {
+    o->ll = q->ll_lines ? (uint8_t *)(q->ctrl + q->L.ll) : nullptr;
+    o->rbuf = (uint8_t *)q->rbuf;
   }
 }
 
@@ -361,7 +366,11 @@ static int p2p_init(int kind, const void *sbuf, void *rbuf, int partitions, size
   q->part_bytes = count * q->esize;
   q->total_bytes = bytes;
   q->seq = c->post_seq[std::make_tuple(kind, peer, tag)]++;
-  q->L.build((size_t)partitions, (size_t)partitions);
+  // LL line area (PC_COPY_LL): both sides derive it from (partitions, count,
+  // dtype), which matching requires to be equal, so their layouts agree.
+  if (q->part_bytes <= PC_LL_MAX_PART_BYTES && bytes <= PC_LL_MAX_TOTAL_BYTES)
+    q->ll_lines = (uint32_t)std::max<uint64_t>(1, (q->part_bytes + 7) / 8);
+  q->L.build((size_t)partitions, (size_t)partitions, (size_t)2 * partitions * q->ll_lines * 4);
   q->agg = 1;
   q->ntransport = partitions;
   return 0;
@@ -1193,10 +1202,12 @@ int pc_pbuf_prepare_all(int n, pc_request_t *reqs, pc_stream_t stream) {
 
 int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_copy_t copy, pc_prequest_t *out) {
   Request *q = (Request *)req;
-  if (!q || !out || gran < 0 || gran > 2 || copy < 0 || copy > 1) return PC_ERR_ARG;
+  if (!q || !out || gran < 0 || gran > 2 || copy < 0 || copy > 2) return PC_ERR_ARG;
   Comm *c = q->comm;
   if (!q->exchanged || !q->matched) return PC_ERR_STATE;  // after the first pbuf_prepare (Listing 2)
   if (q->kind == PC_KIND_PALLREDUCE && aggregation != 1) return PC_ERR_ARG;
+  if (q->kind == PC_KIND_PALLREDUCE && copy == PC_COPY_LL) return PC_ERR_UNSUPPORTED;
+  if (q->kind == PC_KIND_PSEND && copy == PC_COPY_LL && !q->ll_lines) return PC_ERR_UNSUPPORTED;
   if (q->kind == PC_KIND_PSEND) {
     if (aggregation < 1 || aggregation > q->partitions) return PC_ERR_ARG;
     if (q->has_preq && (aggregation != q->agg)) return PC_ERR_STATE;  // the transport layout is fixed
@@ -1216,7 +1227,7 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
     if (!c->dry) {
       PC_CUDA(cudaSetDevice(c->device));
       // publish the transport layout (g) in the receiver's control block
-      uint32_t g = (uint32_t)aggregation;
+      uint32_t g = (uint32_t)aggregation | (copy == PC_COPY_LL ? PC_LAYOUT_LL : 0u);
       PC_CUDA(cudaMemcpyAsync(q->peer_ctrl + q->L.layout, &g, 4, cudaMemcpyHostToDevice, q->side));
       PC_CUDA(cudaStreamSynchronize(q->side));
     }
@@ -1287,10 +1298,11 @@ static int wait_common(Request *q, cudaStream_t s, bool host) {
     if (q->kind == PC_KIND_PSEND) {
       if (!q->has_preq) return PC_ERR_STATE;
       rc = launch_wait_words(q->ctrl + q->L.sent, q->ntransport, q->ctrl + q->L.epoch, 1, nullptr, q->partitions, err,
-                             c->timeout_ms, ws, false);
+                             c->timeout_ms, ws, false, q->copy == PC_COPY_LL ? q->ctrl + q->L.rtr : nullptr);
     } else {
-      rc = launch_wait_words(q->ctrl + q->L.flags, 0, q->ctrl + q->L.epoch, 1, q->ctrl + q->L.layout, q->partitions,
-                             err, c->timeout_ms, ws, q->sys_scope != 0);
+      pc_prequest_t rq;
+      fill_prequest(q, &rq);
+      rc = launch_recv_wait(rq, nullptr, ws);
     }
     if (rc) return rc;
     if (host) PC_CUDA(cudaStreamSynchronize(q->side));
@@ -1348,6 +1360,14 @@ int pc_parrived(pc_request_t req, int partition, int *flag) {
     uint32_t g = 0;
     if ((rc = read_words(q, q->L.layout, 1, &g))) return rc;
     if (g == 0) return 0;
+    if (g & PC_LAYOUT_LL) {  // check the lines and unpack them on the device
+      pc_prequest_t rq;
+      fill_prequest(q, &rq);
+      if ((rc = launch_parrived(rq, partition, (int32_t *)(q->ctrl + q->L.scratch), q->side))) return rc;
+      if ((rc = read_words(q, q->L.scratch, 1, &v))) return rc;
+      *flag = v != 0;
+      return 0;
+    }
     if ((rc = read_words(q, q->L.flags + partition / g, 1, &v))) return rc;
     *flag = reached_h(v, e);
   } else {
@@ -1392,18 +1412,36 @@ int pc_test(pc_request_t req, int *flag) {
   } else {
     int n = q->kind == PC_KIND_PSEND ? q->ntransport : 0;
     size_t off = q->kind == PC_KIND_PSEND ? q->L.sent : q->L.flags;
+    bool ll = false;
     if (q->kind == PC_KIND_PRECV) {
       uint32_t g = 0;
       if ((rc = read_words(q, q->L.layout, 1, &g))) return rc;
-      n = g ? (q->partitions + (int)g - 1) / (int)g : -1;
+      if (g & PC_LAYOUT_LL) {  // count lines not there yet (and unpack those that are) on the device
+        pc_prequest_t rq;
+        fill_prequest(q, &rq);
+        int32_t *pend = (int32_t *)(q->ctrl + q->L.scratch);
+        PC_CUDA(cudaMemsetAsync(pend, 0, 4, q->side));
+        if ((rc = launch_recv_wait(rq, pend, q->side))) return rc;
+        uint32_t np = 1;
+        if ((rc = read_words(q, q->L.scratch, 1, &np))) return rc;
+        ll = true;
+        done = np == 0;
+      } else {
+        n = g ? (q->partitions + (int)g - 1) / (int)g : -1;
+      }
     }
-    done = n >= 0;
-    if (n > 0) {
+    if (!ll) done = n >= 0;
+    if (!ll && n > 0) {
       uint32_t e = 0;
       if ((rc = current_epoch(q, &e))) return rc;
       std::vector<uint32_t> h((size_t)n);
       if ((rc = read_words(q, off, (size_t)n, h.data()))) return rc;
       for (uint32_t v : h) done = done && reached_h(v, e);
+      if (done && q->kind == PC_KIND_PSEND && q->copy == PC_COPY_LL) {  // R29: receiver posted RTR(e)
+        uint32_t r = 0;
+        if ((rc = read_words(q, q->L.rtr, 1, &r))) return rc;
+        done = reached_h(r, e);
+      }
     }
   }
   int erc = error_rc(q);

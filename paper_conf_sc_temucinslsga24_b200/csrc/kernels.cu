@@ -43,9 +43,14 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
 }
 
 __global__ void wait_words_kernel(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul,
-                                  const uint32_t *layout, int partitions, int32_t *err, uint32_t tmo, int sys) {
+                                  const uint32_t *layout, int partitions, int32_t *err, uint32_t tmo, int sys,
+                                  const uint32_t *rtr) {
   __shared__ int s_n;
   const uint32_t target = *(const volatile uint32_t *)epoch * mul;
+  // LL sender: its epoch completes only once the receiver posted ready-to-
+  // receive for this epoch (acquire), i.e. finished reading epoch e-1's lines,
+  // whose parity epoch e+1 reuses (ll_push, R29)
+  if (rtr && threadIdx.x == 32) spin_geq<true>(rtr, target, err, tmo, -3);
   if (threadIdx.x == 0) {
     int nn = n;
     if (layout) {
@@ -70,6 +75,85 @@ __global__ void wait_words_kernel(const uint32_t *words, int n, const uint32_t *
     bool ok = sys ? spin_geq<true>(words + i, target, err, tmo, i) : spin_geq<false>(words + i, target, err, tmo, i);
     if (!ok) break;
   }
+}
+
+// Receive-side MPI_Wait / MPI_Test for a request whose sender may push LL
+// lines (PC_COPY_LL): the layout word tells which protocol the sender chose.
+// LL: every thread owns lines i = (p, j) of the grid-stride range, waits (or,
+// in test mode, checks once) until the line carries this epoch in both halves
+// and unpacks its payload bytes into recvbuf.  Flags: block 0 waits on the
+// transport flags exactly as wait_words_kernel.  Test mode (pending != null):
+// no spinning; every line / flag not there yet adds 1 to *pending.
+__global__ void recv_wait_kernel(pc_prequest_t q, int32_t *pending) {
+  __shared__ uint32_t s_g;
+  const uint32_t e = *(const volatile uint32_t *)q.epoch;
+  if (threadIdx.x == 0) {
+    const uint64_t t0 = globaltimer();
+    uint32_t g;
+    while ((g = *(const volatile uint32_t *)q.layout) == 0) {  // the sender publishes g at pc_prequest_create
+      if (pending || aborted(q.err)) break;
+      if (q.timeout_ms && globaltimer() - t0 > (uint64_t)q.timeout_ms * 1000000ull) {
+        set_error(q.err, PC_DEV_ERR_TIMEOUT, -2);
+        break;
+      }
+      __nanosleep(256);
+    }
+    s_g = g;
+  }
+  __syncthreads();
+  const uint32_t g = s_g;
+  if (g == 0) {
+    if (pending && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(pending, 1);
+    return;
+  }
+  if (g & PC_LAYOUT_LL) {
+    const uint32_t nl = q.ll_lines;
+    const uint64_t nlines = (uint64_t)q.partitions * nl;
+    const uint8_t *base = q.ll + (uint64_t)(e & 1) * nlines * 16ull;
+    const uint64_t t0 = globaltimer();
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nlines; i += (uint64_t)gridDim.x * blockDim.x) {
+      ulonglong2 v = ld_ll(base + 16ull * i, q.sys_scope);
+      uint32_t n = 0;
+      while ((uint32_t)(v.x >> 32) != e || (uint32_t)(v.y >> 32) != e) {
+        if (pending) break;
+        if ((++n & 127) == 0) {
+          if (aborted(q.err)) return;
+          if (q.timeout_ms && globaltimer() - t0 > (uint64_t)q.timeout_ms * 1000000ull) {
+            set_error(q.err, PC_DEV_ERR_TIMEOUT, (int)(i / nl));
+            return;
+          }
+          __nanosleep(128);
+        }
+        v = ld_ll(base + 16ull * i, q.sys_scope);
+      }
+      if ((uint32_t)(v.x >> 32) != e || (uint32_t)(v.y >> 32) != e) {
+        atomicAdd(pending, 1);
+        continue;
+      }
+      const uint64_t p = i / nl;
+      const uint32_t j = (uint32_t)(i % nl);
+      const uint32_t nb = ll_nbytes(q.part_bytes, j);
+      if (nb) st_payload8(q.rbuf + p * q.part_bytes + 8ull * j, (v.x & 0xffffffffull) | (v.y << 32), nb);
+    }
+    return;
+  }
+  if (blockIdx.x != 0) return;
+  const int nt = (q.partitions + (int)g - 1) / (int)g;
+  for (int i = threadIdx.x; i < nt; i += blockDim.x) {
+    if (pending) {
+      if (!reached(ld_acquire_scope(q.flags + i, q.sys_scope), e)) atomicAdd(pending, 1);
+      continue;
+    }
+    bool ok = q.sys_scope ? spin_geq<true>(q.flags + i, e, q.err, q.timeout_ms, i)
+                          : spin_geq<false>(q.flags + i, e, q.err, q.timeout_ms, i);
+    if (!ok) break;
+  }
+}
+
+// Host pc_parrived of a receive request: the device binding, run by one thread
+// (for LL it also unpacks the partition's lines into recvbuf).
+__global__ void parrived_kernel(pc_prequest_t q, int partition, int32_t *out) {
+  out[0] = pc_parrived(q, partition);
 }
 
 __global__ void set_word_kernel(uint32_t *addr, uint32_t v) { st_release_sys(addr, v); }
@@ -199,8 +283,30 @@ int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
 }
 
 int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul, const uint32_t *layout,
-                      int partitions, int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys) {
-  wait_words_kernel<<<1, 256, 0, s>>>(words, n, epoch, mul, layout, partitions, err, timeout_ms, sys ? 1 : 0);
+                      int partitions, int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys,
+                      const uint32_t *rtr) {
+  wait_words_kernel<<<1, 256, 0, s>>>(words, n, epoch, mul, layout, partitions, err, timeout_ms, sys ? 1 : 0, rtr);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_recv_wait(const pc_prequest_t &q, int32_t *pending, cudaStream_t s) {
+  int blocks = 1;
+  if (q.ll_lines) {
+    const int64_t lines = (int64_t)q.partitions * q.ll_lines;
+    blocks = (int)((lines + 255) / 256);
+    if (blocks > 4 * 148) blocks = 4 * 148;
+    if (blocks < 1) blocks = 1;
+  }
+  recv_wait_kernel<<<blocks, 256, 0, s>>>(q, pending);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_parrived(const pc_prequest_t &q, int partition, int32_t *out, cudaStream_t s) {
+  parrived_kernel<<<1, 1, 0, s>>>(q, partition, out);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;

@@ -84,13 +84,17 @@ struct CtrlLayout {
   size_t sent = 0;         // [n1]
   size_t donecnt = 0;      // [n1] engine slice-completion counters / allreduce done[u]
   size_t flags = 0;        // [nflags] arrival flags
+  size_t ll = 0;           // [ll_words] LL lines (p2p, PC_COPY_LL), 256-B aligned
+  size_t scratch = 0;      // [4] host-query results (pc_parrived / pc_test on LL requests)
   size_t words = 0;
-  void build(size_t n1, size_t nflags) {
+  void build(size_t n1, size_t nflags, size_t ll_words = 0) {
     ready = cnt + n1;
     sent = ready + n1;
     donecnt = sent + n1;
     flags = donecnt + n1;
-    words = flags + nflags;
+    scratch = flags + nflags;
+    ll = (scratch + 4 + 63) & ~size_t(63);
+    words = ll + ll_words;
     words = (words + 63) & ~size_t(63);
   }
 };
@@ -180,6 +184,7 @@ struct Request {
   // prequest (p2p)
   bool has_preq = false;
   int agg = 1, ntransport = 0, copy = 0;
+  uint32_t ll_lines = 0;  // p2p: LL lines per partition (0 = no LL area; pc.h PC_LL_MAX_*)
   // engine slicing
   int nsteps = 0;
   int slices = 1;          // ns: slices per chunk (allreduce) or per transport partition (p2p ENGINE)
@@ -319,9 +324,15 @@ struct CtlArgs {
 int launch_ctl(const CtlArgs &a, cudaStream_t s);
 int launch_epoch_bump(uint32_t *epoch, cudaStream_t s);
 int launch_rtr(const RtrArgs &a, cudaStream_t s);
+// rtr != null: also acquire-wait until *rtr reached the epoch (LL sender)
 int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul, const uint32_t *layout,
-                      int partitions,
-                      int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys);
+                      int partitions, int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys,
+                      const uint32_t *rtr = nullptr);
+// receive-side wait (pending == null) or test (pending: device counter of
+// lines / flags not yet arrived, zeroed by the caller); handles LL and flags
+int launch_recv_wait(const pc_prequest_t &q, int32_t *pending, cudaStream_t s);
+// out[0] = pc_parrived(q, partition) on the device (LL receive requests)
+int launch_parrived(const pc_prequest_t &q, int partition, int32_t *out, cudaStream_t s);
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s);
 int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s);
 constexpr int kMaxPreadyAll = 16;

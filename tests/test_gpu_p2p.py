@@ -244,3 +244,152 @@ def test_pingpong_latency_roundtrip(payload):
         for q in (a2b, a_in, b_in, b2a):
             assert q.error()[0] == 0
             q.free()
+
+
+# ---------------------------------------------------------------- PC_COPY_LL
+@pytest.mark.parametrize("gran", [apps.GRAN_THREAD, apps.GRAN_WARP])
+@pytest.mark.parametrize("agg_kind", ["none", "odd", "all"])
+def test_ll_granularity_aggregation(gran, agg_kind):
+    """LL lines (8 payload bytes + the epoch per 16-B line) at thread (8 B) and
+    warp (256 B) granularity: byte-exact vs O1, in-kernel pc_wait_arrived and
+    the stream wait both unpack the lines into recvbuf."""
+    n = 3 * 2048 * 5
+    partitions = n // GRAN_ELEMS[gran]
+    agg = {"none": 1, "odd": max(1, partitions // 3 - 1), "all": partitions}[agg_kind]
+    run_vecadd(n, gran, agg, pc.COPY_LL, epochs=3)
+
+
+@pytest.mark.parametrize("pbytes", [1, 3, 8, 12, 100, 256, 1000, 1024])
+@pytest.mark.parametrize("gran", [apps.GRAN_THREAD, apps.GRAN_WARP, apps.GRAN_BLOCK])
+def test_ll_epochs_tagged_bytes(pbytes, gran):
+    """LL over many back-to-back epochs of epoch-tagged bytes (both line-area
+    parities reused many times), ragged partition sizes (partial last line,
+    unaligned partitions), permuted Pready order; recvbuf checked every epoch."""
+    partitions, E = 37, 60
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        src = torch.empty(partitions * pbytes, dtype=torch.uint8, device="cuda")
+        sbuf = torch.empty_like(src)
+        rbuf = torch.empty_like(src)
+        out = torch.zeros_like(src)
+        status = torch.zeros(1, dtype=torch.int32, device="cuda")
+        snd = pc.psend_init(sbuf, partitions, pbytes, pc.BYTE, 1, 1, cs[0])
+        rcv = pc.precv_init(rbuf, partitions, pbytes, pc.BYTE, 0, 1, cs[1])
+        for e in range(E):
+            payload = synth.bytes_tagged(SEED, 0, e, partitions * pbytes)
+            src.copy_(torch.from_numpy(payload))
+            torch.cuda.synchronize()
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                sq = snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_LL)
+                rq = rcv.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            apps.produce(sbuf, src, partitions, pbytes, gran, sq, order_stride=5, stream=s0)
+            snd.wait_on_stream(s0)
+            if e % 2:
+                apps.check_recv(rq, rbuf, out, partitions, pbytes, status, blocks=8, stream=s1)
+            rcv.wait_on_stream(s1)
+            s1.synchronize()
+            np.testing.assert_array_equal(rbuf.cpu().numpy(), payload)
+            if e % 2:
+                np.testing.assert_array_equal(out.cpu().numpy(), payload)
+        snd.wait()
+        assert int(status.item()) == 0
+        assert snd.error()[0] == 0 and rcv.error()[0] == 0
+        snd.free()
+        rcv.free()
+
+
+def test_ll_host_parrived_and_test():
+    """Host pc_parrived / pc_test on an LL receive request check (and unpack)
+    the lines on the device."""
+    partitions, count = 8, 16  # 64 B partitions
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        sbuf = torch.arange(partitions * count, dtype=torch.float32, device="cuda")
+        rbuf = torch.zeros_like(sbuf)
+        snd = pc.psend_init(sbuf, partitions, count, pc.FLOAT32, 1, 0, cs[0])
+        rcv = pc.precv_init(rbuf, partitions, count, pc.FLOAT32, 0, 0, cs[1])
+        snd.start(s0)
+        rcv.start(s1)
+        first_prepare([[snd], [rcv]], [s0, s1])
+        snd.prequest_create(pc.GRAN_WARP, 1, pc.COPY_LL)
+        assert not rcv.parrived(0)
+        assert not rcv.test()
+        snd.pready_range(0, 2, s0)
+        s0.synchronize()
+        assert rcv.parrived(1)
+        assert not rcv.parrived(5)
+        assert torch.equal(rbuf[count:2 * count], sbuf[count:2 * count])
+        assert not rcv.test()
+        snd.pready_range(3, partitions - 1, s0)
+        s0.synchronize()
+        while not rcv.test():
+            pass
+        assert torch.equal(rbuf, sbuf)
+        snd.wait()
+        snd.free()
+        rcv.free()
+
+
+def test_ll_unsupported_large_partitions():
+    """LL is for small partitions (<= PC_LL_MAX_PART_BYTES): larger ones are
+    refused at pc_prequest_create."""
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        sbuf = torch.zeros(4 * 2048, device="cuda")
+        rbuf = torch.zeros_like(sbuf)
+        snd = pc.psend_init(sbuf, 4, 2048, pc.FLOAT32, 1, 0, cs[0])
+        rcv = pc.precv_init(rbuf, 4, 2048, pc.FLOAT32, 0, 0, cs[1])
+        snd.start(s0)
+        rcv.start(s1)
+        first_prepare([[snd], [rcv]], [s0, s1])
+        with pytest.raises(pc.PcError) as ei:
+            snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_LL)
+        assert ei.value.code == pc.ERR_UNSUPPORTED
+        snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+        snd.pready_range(0, 3, s0)
+        rcv.wait()
+        snd.wait()
+        snd.free()
+        rcv.free()
+
+
+@pytest.mark.parametrize("payload", [0, 8, 256, 1024])
+def test_ll_pingpong_latency_roundtrip(payload):
+    """Pready->Parrived ping-pong with LL lines: data intact at every size."""
+    iters = 2000
+    cnt = payload // 4
+    with comms(2) as cs:
+        s0 = torch.cuda.Stream()
+        bufs = [torch.zeros(max(iters * cnt, 4), device="cuda") for _ in range(4)]
+        a2b = pc.psend_init(bufs[0], iters, cnt, pc.FLOAT32, 1, 1, cs[0])
+        b_in = pc.precv_init(bufs[1], iters, cnt, pc.FLOAT32, 0, 1, cs[1])
+        b2a = pc.psend_init(bufs[2], iters, cnt, pc.FLOAT32, 0, 2, cs[1])
+        a_in = pc.precv_init(bufs[3], iters, cnt, pc.FLOAT32, 1, 2, cs[0])
+        bufs[0].copy_(torch.arange(bufs[0].numel(), dtype=torch.float32))
+        bufs[2].copy_(-torch.arange(bufs[2].numel(), dtype=torch.float32))
+        for q in (a2b, a_in, b_in, b2a):
+            q.start(s0)
+        first_prepare([[a2b, a_in], [b_in, b2a]], [s0, s0])
+        pa = a2b.prequest_create(pc.GRAN_WARP, 1, pc.COPY_LL)
+        pai = a_in.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
+        pb = b2a.prequest_create(pc.GRAN_WARP, 1, pc.COPY_LL)
+        pbi = b_in.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
+        t = torch.zeros(2, dtype=torch.int64, device="cuda")
+        apps.pingpong_pair(pa, pai, pb, pbi, iters, apps.GRAN_WARP, t, s0)
+        for q in (a2b, b2a, a_in, b_in):
+            q.wait_on_stream(s0)
+        torch.cuda.synchronize()
+        ns = int(t[0].item()) / iters / 2
+        print(f"LL payload {payload} B: one-way {ns:.0f} ns (same-GPU virtual ranks)")
+        if cnt:
+            np.testing.assert_array_equal(bufs[1].cpu().numpy(), bufs[0].cpu().numpy())
+            np.testing.assert_array_equal(bufs[3].cpu().numpy(), bufs[2].cpu().numpy())
+        for q in (a2b, a_in, b_in, b2a):
+            assert q.error()[0] == 0
+            q.free()

@@ -12,10 +12,10 @@ from paper_conf_sc_temucinslsga24_b200 import _lib
 
 MODES = ["lib wait + lib pready_warp", "raw wait + lib pready_warp", "lib wait + raw pready",
          "raw wait + raw pready", "lib wait + lib pready(thread)", "raw wait + lib pready(thread)",
-         "lib wait + lane0 epoch_rtr+publish", "lib wait + lane0 epoch_rtr+shfl+publish", "lib wait + lane0 relaxed epoch+publish"]
+         "lib wait + lane0 epoch_rtr+publish", "lib wait + lane0 epoch_rtr+shfl+publish", "lib wait + lane0 relaxed epoch+publish", "warp wait + lib pready_warp", "lane0 ld.acquire.gpu+publish", "lane0 ld.acquire.sys+publish", "lane0 ld.relaxed.gpu+publish", "lane0 ld.acquire.sys.v2+publish", "lane0 ld.acquire.gpu.v2+publish"]
 
 
-def run(payload, iters=20000):
+def run(payload, iters=20000, copy=0):
     g, comms = pc.local_comms(2, 0)
     st = torch.cuda.Stream()
     cnt = payload // 4
@@ -28,14 +28,14 @@ def run(payload, iters=20000):
     res = {}
     first = True
     pq = None
-    for mode in range(len(MODES)):
+    for mode in (range(len(MODES)) if copy == pc.COPY_INLINE else (0, 4, 9)):
         for rep in range(2):
             for q in (a2b, a_in, b_in, b2a):
                 q.start(st)
             if first:
                 pc.run_ranks([lambda: [q.pbuf_prepare(st) for q in (a2b, a_in)],
                               lambda: [q.pbuf_prepare(st) for q in (b_in, b2a)]])
-                pq = [q.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE) for q in (a2b, a_in, b2a, b_in)]
+                pq = [q.prequest_create(pc.GRAN_WARP, 1, c) for q, c in zip((a2b, a_in, b2a, b_in), (copy, 0, copy, 0))]
                 first = False
             else:
                 for q in (a2b, a_in, b_in, b2a):
@@ -47,7 +47,7 @@ def run(payload, iters=20000):
             torch.cuda.synchronize()
         res[MODES[mode]] = t[0].item() / iters / 2
         tt = t.cpu().tolist()
-        print(f"payload {payload:4d} B  {MODES[mode]:40s} one-way {res[MODES[mode]]:8.1f} ns  "
+        print(f"copy {copy} payload {payload:4d} B  {MODES[mode]:40s} one-way {res[MODES[mode]]:8.1f} ns  "
               f"pready A {tt[2] / iters:7.0f} B {tt[4] / iters:7.0f} cyc  wait B {tt[5] / iters:7.0f} cyc", flush=True)
     for q in (a2b, a_in, b_in, b2a):
         q.free()
@@ -59,5 +59,6 @@ def run(payload, iters=20000):
 
 if __name__ == "__main__":
     torch.cuda.set_device(0)
-    for payload in (0, 8):
-        run(payload)
+    for copy in (pc.COPY_INLINE, pc.COPY_LL):
+        for payload in (0, 8, 256):
+            run(payload, copy=copy)
