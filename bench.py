@@ -41,7 +41,7 @@ def parse():
     ap.add_argument("--impl", default="pc", choices=["pc", "reference"])
     ap.add_argument("--bytes", type=int, default=256 << 20, help="bytes per rank (S)")
     ap.add_argument("--partitions", type=int, default=64)
-    ap.add_argument("--algo", default="ring", choices=["ring", "rd", "direct", "auto"])
+    ap.add_argument("--algo", default="auto", choices=["ring", "rd", "direct", "auto"])
     ap.add_argument("--vranks", type=int, default=8, help="virtual ranks on the one GPU when N = 1")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -58,6 +58,21 @@ T0 = time.time()
 
 def log(*a):
     print(f"[bench {time.time() - T0:7.1f}s]", *a, file=sys.stderr, flush=True)
+
+
+def engine_alg_bytes(algo, P, S):
+    """Algorithmic HBM bytes of one grouped engine launch of P co-located ranks
+    (DESIGN.md §6).  ring: per rank S/P*(3P-3) reads + S/P*(2P-1) writes;
+    direct (PULL): per rank S read (its chunk from all P send buffers) + S
+    written (the final chunk into all P recvbufs); rd: per rank log2P steps of
+    (read acc + read incoming + write peer staging + write acc) + the final copy."""
+    if P == 1:
+        return 2 * S
+    if algo == "direct":
+        return 2 * P * S
+    if algo == "rd":
+        return (4 * (P.bit_length() - 1) + 2) * P * S
+    return (5 * P - 4) * S
 
 
 def busbw(S, sec, P):
@@ -416,22 +431,20 @@ def run_virtual(args):
     value = busbw(S, ms / 1e3, P)
     hbm_peak, peak_src = peaks()
     eng_ms = float(np.mean(eng)) if len(eng) else None
-    # algorithmic HBM bytes of one grouped engine launch (all P co-located
-    # ranks): per rank S/P * (3P-3) reads + S/P * (2P-1) writes
-    alg_bytes = (5 * P - 4) * S if P > 1 else 2 * S
+    alg_bytes = engine_alg_bytes(info["algo_name"], P, S)
     achieved = alg_bytes / (eng_ms / 1e3) / 1e9 if eng_ms else None
     traffic = None
     tp = os.path.join(ROOT, "profiles", "engine_traffic.json")
     if os.path.exists(tp):
         try:
             t = json.load(open(tp))
-            if t.get("bytes_per_rank") == S and t.get("ranks") == P:
+            if t.get("bytes_per_rank") == S and t.get("ranks") == P and t.get("algo", "ring") == info["algo_name"]:
                 traffic = t.get("dram_bytes_per_launch")
         except Exception:
             pass
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
             "frac": (achieved / hbm_peak) if achieved else None, "traffic": traffic,
-            "kernel": "ring_engine_group (all co-located ranks' engines in one launch)",
+            "kernel": f"{info['algo_name']}_engine_group (all co-located ranks' engines in one launch)",
             "engine_ms": eng_ms, "engine_share_of_step": (eng_ms / ms) if eng_ms else None,
             "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src}
 
@@ -487,8 +500,9 @@ def run_virtual(args):
            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
            "config": {"workload": f"partitioned allreduce (C5/C3 shape) fp32 sum, {P} virtual ranks co-located on one "
-                                  f"B200, {S >> 20} MiB per rank in {Np} partitions, {args.algo} schedule",
-                      "ranks": P, "ranks_per_gpu": P, "bytes_per_rank": S, "partitions": Np, "algo": args.algo,
+                                  f"B200, {S >> 20} MiB per rank in {Np} partitions, {info['algo_name']} schedule"
+                                  f" (requested {args.algo})",
+                      "ranks": P, "ranks_per_gpu": P, "bytes_per_rank": S, "partitions": Np, "algo": info["algo_name"],
                       "slices_per_chunk": info["slices"], "slice_elems": info["slice_elems"],
                       "engine_warps_per_rank": info["engine_warps"],
                       "l2": f"no flush: working set {3 * P * S >> 20} MiB >> 126 MB L2",

@@ -63,9 +63,12 @@ typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1, PC_COPY_LL = 2 } pc_copy_
 /* Allreduce schedule (§IV-B).  RING = Alg 1; RD = recursive
  * doubling (BASELINE north_star; not in the paper; P a power of two);
  * DIRECT = two steps over neighbour SETS (the generic schedule of P:L155 with
- * |I| = |O| = P-1: reduce-scatter to chunk owners, allgather; P <= 8; the
- * NVSwitch-native schedule of SURVEY NEXT-1); AUTO = RD below
- * PC_RD_MAX_BYTES, DIRECT up to PC_DIRECT_MAX_BYTES, ring above. */
+ * |I| = |O| = P-1; P <= 8; the NVSwitch-native schedule of SURVEY NEXT-1):
+ * each chunk owner PULLS its chunk from every peer's send buffer with peer
+ * loads, folds in rank order, and pushes the result to every peer.
+ * AUTO = DIRECT for 3 <= P <= 8 (RD for P = 2 up to PC_RD_MAX_BYTES, default
+ * 4 MiB; PC_DIRECT_MAX_BYTES caps DIRECT); for P > 8 RD up to
+ * PC_RD_MAX_BYTES, ring above. */
 typedef enum { PC_ALGO_AUTO = 0, PC_ALGO_RING = 1, PC_ALGO_RD = 2, PC_ALGO_DIRECT = 3 } pc_algo_t;
 
 enum {

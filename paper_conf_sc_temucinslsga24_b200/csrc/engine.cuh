@@ -41,7 +41,10 @@ using namespace pc_detail;
 #ifndef PC_ENGINE_UNROLL
 #define PC_ENGINE_UNROLL 8
 #endif
-constexpr int kU = PC_ENGINE_UNROLL;  // 16-B vectors in flight per operand per lane
+constexpr int kU = PC_ENGINE_UNROLL;
+#ifndef PC_DIRECT_FV
+#define PC_DIRECT_FV 1
+#endif  // 16-B vectors in flight per operand per lane
 
 // Engine-side bounded spin: the awaited event is a whole slice step of the
 // upstream rank (tens of microseconds), so back off with __nanosleep early and
@@ -429,14 +432,21 @@ __device__ __forceinline__ void rd_body(const RdArgs &a, const int gw, const int
 
 // ---------------------------------------------------------------------------
 // Direct two-step schedule (generic schedule with neighbour
-// sets).  Unit (u, slice s):
-//   step 0 (after the user's Pready of u): push slice s of chunk o to owner
-//          o's staging slot [u][r] for every peer o, then bump each owner's
-//          phase-0 counter;
+// sets), PULL transport: the reduce step reads its P inputs
+// straight from the peers' send buffers with peer loads over NVSwitch (no
+// staging copy: per rank S bytes read + S written, vs. the ring's 2(P-1)/P·S
+// over the links plus staging round trips in HBM).  Unit (u, slice s):
+//   step 0 (after the user's Pready of u): announce "my partition u is final"
+//          to every owner (release: the producer's writes, acquired through
+//          ready[u], are ordered before the owner's reads) — bump each
+//          owner's phase-0 counter for slice s;
 //   step 1 (all P-1 phase-0 arrivals): fold the P contributions of my chunk
-//          in rank order (reading R25) in registers, store the final slice
-//          locally and into every peer's recvbuf, bump their phase-1 counters;
+//          in rank order (reading R25) in registers, loading peer k's slice
+//          from its send buffer, store the final slice locally and into every
+//          peer's recvbuf, bump their phase-1 counters;
 //   step 2 (all P-1 phase-1 arrivals): slice final everywhere -> done[u].
+// A peer reuses its send buffer only after its own pc_wait, which needs every
+// owner's phase-1 signal, issued after that owner's loads: no WAR hazard.
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ void red_add_scope(uint32_t *p, uint32_t v, bool sys) {
   if (sys)
@@ -445,35 +455,74 @@ __device__ __forceinline__ void red_add_scope(uint32_t *p, uint32_t v, bool sys)
     asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// out_local and out_peer[j] (j < P-1) = fold over k = 0..P-1 of src[k] in rank
-// order; all pointers share one misalignment (scalar head, 16-B body, tail).
+// recvbuf[e0 .. e0+n) of this rank and of every peer = fold over ranks
+// k = 0..P-1 (rank order, reading R25) of rank k's sendbuf[e0 ..), read with
+// peer loads (PULL).  All operands sit at the same element offset of 16-B
+// aligned buffers: scalar head, 16-B body, scalar tail.  Buffer pointers come
+// straight from the kernel parameters (no pointer arrays on the stack).
 template <int DT, int OP>
-__device__ __forceinline__ void warp_fold_direct(void *out_local, uint8_t *const *out_peer, const uint8_t *const *src,
-                                                 int P, int64_t n) {
+__device__ __forceinline__ void warp_fold_direct(const DirectArgs &a, int64_t e0, int64_t n) {
   using O = Op<DT, OP>;
   using T = typename O::T;
+  const int P = a.P, r = a.r;
   const uint32_t lane = threadIdx.x & 31;
   constexpr int64_t EPV = 16 / sizeof(T);
+  auto src = [&](int k) -> const T * {
+    return reinterpret_cast<const T *>(k == r ? a.sendbuf : a.p_sendbuf[(k - r - 1 + P) % P]) + e0;
+  };
+  T *out_local = reinterpret_cast<T *>(a.recvbuf) + e0;
   const uintptr_t m = reinterpret_cast<uintptr_t>(out_local) & 15;
   int64_t head = (int64_t)(((16 - m) & 15) / sizeof(T));
   if (head > n) head = n;
   auto scalar = [&](int64_t k) {
-    T acc = __ldcg(reinterpret_cast<const T *>(src[0]) + k);
-    for (int j = 1; j < P; ++j) acc = O::f(acc, __ldcg(reinterpret_cast<const T *>(src[j]) + k));
-    reinterpret_cast<T *>(out_local)[k] = acc;
-    for (int j = 0; j < P - 1; ++j) reinterpret_cast<T *>(out_peer[j])[k] = acc;
+    T acc = __ldcg(src(0) + k);
+    for (int j = 1; j < P; ++j) acc = O::f(acc, __ldcg(src(j) + k));
+    out_local[k] = acc;
+    for (int j = 0; j < P - 1; ++j) (reinterpret_cast<T *>(a.p_recvbuf[j]) + e0)[k] = acc;
   };
   for (int64_t k = lane; k < head; k += 32) scalar(k);
   const int64_t nv = (n - head) / EPV;
-  for (int64_t k = lane; k < nv; k += 32) {
-    const int64_t eo = head + EPV * k;  // element offset
-    uint4 acc = __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(src[0]) + eo));
-    for (int j = 1; j < P; ++j)
-      acc = vop<DT, OP>(acc, __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(src[j]) + eo)));
-    *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(out_local) + eo) = acc;
-    for (int j = 0; j < P - 1; ++j) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(out_peer[j]) + eo) = acc;
+  // all P * kFV loads of a lane are issued before the first add (the fold
+  // itself stays in rank order): one round trip per kFV vectors, not P
+  constexpr int kFV = PC_DIRECT_FV;
+  auto store_all = [&](int64_t vk, uint4 acc) {
+    const int64_t eo = head + EPV * vk;
+    *reinterpret_cast<uint4 *>(out_local + eo) = acc;
+#pragma unroll
+    for (int j = 0; j < kMaxDirect - 1; ++j)
+      if (j < P - 1) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(a.p_recvbuf[j]) + e0 + eo) = acc;
+  };
+  int64_t k = lane;
+  for (; k + 32 * (kFV - 1) < nv; k += 32 * kFV) {
+    uint4 x[kMaxDirect][kFV];
+#pragma unroll
+    for (int j = 0; j < kMaxDirect; ++j)
+      if (j < P) {
+        const uint4 *sj = reinterpret_cast<const uint4 *>(src(j) + head);
+#pragma unroll
+        for (int v = 0; v < kFV; ++v) x[j][v] = __ldcg(sj + k + 32 * v);
+      }
+#pragma unroll
+    for (int v = 0; v < kFV; ++v) {
+      uint4 acc = x[0][v];
+#pragma unroll
+      for (int j = 1; j < kMaxDirect; ++j)
+        if (j < P) acc = vop<DT, OP>(acc, x[j][v]);
+      store_all(k + 32 * v, acc);
+    }
   }
-  for (int64_t k = head + nv * EPV + lane; k < n; k += 32) scalar(k);
+  for (; k < nv; k += 32) {
+    uint4 x[kMaxDirect];
+#pragma unroll
+    for (int j = 0; j < kMaxDirect; ++j)
+      if (j < P) x[j] = __ldcg(reinterpret_cast<const uint4 *>(src(j) + head) + k);
+    uint4 acc = x[0];
+#pragma unroll
+    for (int j = 1; j < kMaxDirect; ++j)
+      if (j < P) acc = vop<DT, OP>(acc, x[j]);
+    store_all(k, acc);
+  }
+  for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
 }
 
 template <int DT, int OP>
@@ -519,16 +568,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
         if (!warp_poll(dep, i == 0 ? e : target, i != 0 && a.sys)) continue;
         progressed = true;
         const int64_t base = (int64_t)u * a.L;
-        const int64_t mis = base % (16 / es);  // the buffers' misalignment in elements (staging mirrors it)
         if (i == 0) {
-          for (int j = 0; j < P - 1; ++j) {
-            const int o = (r + 1 + j) % P;
-            const int64_t c_lo = min((int64_t)o * a.q, a.L), c_hi = min((int64_t)(o + 1) * a.q, a.L);
-            const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-            if (hi > lo)
-              warp_copy(a.p_staging[j] + (((int64_t)u * P + r) * a.sq + mis + (int64_t)s * a.qs) * es,
-                        a.sendbuf + (base + lo) * es, (hi - lo) * es);
-          }
           fence_scope(a.sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
@@ -537,15 +577,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
         } else if (i == 1) {
           const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
           const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-          if (hi > lo) {
-            const uint8_t *src[kMaxDirect];
-            uint8_t *outp[kMaxDirect - 1];
-            for (int k = 0; k < P; ++k)
-              src[k] = k == r ? a.sendbuf + (base + lo) * es
-                              : a.staging + (((int64_t)u * P + k) * a.sq + mis + (int64_t)s * a.qs) * es;
-            for (int j = 0; j < P - 1; ++j) outp[j] = a.p_recvbuf[j] + (base + lo) * es;
-            warp_fold_direct<DT, OP>(a.recvbuf + (base + lo) * es, outp, src, P, hi - lo);
-          }
+          if (hi > lo) warp_fold_direct<DT, OP>(a, base + lo, hi - lo);
           fence_scope(a.sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
@@ -566,11 +598,11 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
 }
 
 template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) direct_engine(DirectArgs a) {
+__global__ void __launch_bounds__(kEngineBlock, 2) direct_engine(DirectArgs a) {
   direct_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
 }
 template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock) direct_engine_group(DirectGroupArgs g) {
+__global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_group(DirectGroupArgs g) {
   int k = 0;
   while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
   const int b = blockIdx.x - g.block_start[k];

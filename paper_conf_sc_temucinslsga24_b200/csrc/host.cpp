@@ -397,6 +397,10 @@ static int make_rec(Request *q, ReqRec *r) {
     if ((rc = export_ptr(c, q->rbuf, q->total_bytes, &r->buf))) return rc;
   if ((rc = export_ptr(c, q->ctrl, q->L.words * 4, &r->ctrl))) return rc;
   if (q->staging && (rc = export_ptr(c, q->staging, q->staging_bytes, &r->stage))) return rc;
+  // DIRECT (PULL): the peers' reduce steps read this rank's send buffer
+  if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && c->size > 1 &&
+      (rc = export_ptr(c, q->sbuf, q->total_bytes, &r->stage)))
+    return rc;
   return 0;
 }
 
@@ -635,16 +639,14 @@ static DirectArgs make_direct_args(Request *q) {
   a.L = (int64_t)q->count;
   a.q = q->chunk_elems;
   a.qs = q->slice_elems;
-  a.sq = q->chunk_elems + 16 / (int64_t)q->esize;
   a.sendbuf = (const uint8_t *)q->sbuf;
   a.recvbuf = (uint8_t *)q->rbuf;
-  a.staging = q->staging;
   a.cnt = q->ctrl + q->L.flags;
   a.ready = q->ctrl + q->L.ready;
   a.rtr = q->ctrl + q->L.rtr;
   a.done = q->ctrl + q->L.donecnt;
   for (int j = 0; j < c->size - 1; ++j) {
-    a.p_staging[j] = q->nb_stage[j];
+    a.p_sendbuf[j] = q->nb_stage[j];  // DIRECT exports its send buffer in the stage slot
     a.p_recvbuf[j] = q->nb_buf[j];
     a.p_cnt[j] = q->nb_ctrl[j] + q->L.flags;
   }
@@ -993,14 +995,17 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   int a = algo;
   const bool pow2 = log2_exact(P) >= 0;
   if (a == PC_ALGO_AUTO) {
-    // crossovers measured on one B200 with virtual ranks (profiles/r01_sweep_*):
-    // RD (log2 P hops) wins up to ~1 MiB, DIRECT (2 steps) around 4 MiB at
-    // P = 8, the ring (bandwidth-optimal bytes) above
-    const long rd_max = env_long("PC_RD_MAX_BYTES", 1 << 20);
-    const long direct_max = env_long("PC_DIRECT_MAX_BYTES", 8 << 20);
-    if (P > 1 && pow2 && (long long)bytes <= rd_max)
+    // crossovers measured on one B200 with virtual ranks
+    // (profiles/r01_sweep_allreduce_pull.jsonl): DIRECT with PULL reduce (2
+    // steps, S read + S written per rank) is fastest at every size for
+    // 3 <= P <= 8; at P = 2 recursive doubling (one exchange) wins up to a few
+    // MiB; beyond DIRECT's peer limit: RD for small messages, ring above.
+    const long rd_max = env_long("PC_RD_MAX_BYTES", 4 << 20);
+    const long direct_max = env_long("PC_DIRECT_MAX_BYTES", -1);
+    const bool direct_ok = P > 1 && P <= kMaxDirect && (direct_max < 0 || (long long)bytes <= direct_max);
+    if (P > 1 && pow2 && (long long)bytes <= rd_max && (P == 2 || !direct_ok))
       a = PC_ALGO_RD;
-    else if (P > 4 && P <= kMaxDirect && (long long)bytes <= direct_max)
+    else if (direct_ok)
       a = PC_ALGO_DIRECT;
     else
       a = PC_ALGO_RING;
@@ -1041,7 +1046,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
     q->nsteps = 2;  // phase counters [u][0..1][slice]
     q->chunk_elems = chunk_q(L, P, epv);
     choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems, epv);
-    q->staging_bytes = P > 1 ? (uint64_t)partitions * P * (q->chunk_elems + epv) * esz : 0;
+    q->staging_bytes = 0;  // PULL: owners read the peers' send buffers directly
   } else {
     q->nsteps = log2_exact(P);
     q->chunk_elems = L;

@@ -276,13 +276,14 @@ constexpr int kMaxDirect = 8;
 struct DirectArgs {
   const uint32_t *epoch;
   int P, r, Np, ns, nunits, op, dtype;
-  int64_t L, q, qs, sq;  // sq: staging slot stride in elements (q + 4)
+  int64_t L, q, qs;
   const uint8_t *sendbuf;
   uint8_t *recvbuf;
-  const uint8_t *staging;  // [u][sender][sq] (+ u*L mod 4 so it shares the buffers' misalignment)
   const uint32_t *cnt, *ready, *rtr;  // cnt: [u][phase][slice] arrival counters (written by peers)
   uint32_t *done;
-  uint8_t *p_staging[kMaxDirect - 1], *p_recvbuf[kMaxDirect - 1];
+  // peer j = rank (r+1+j) mod P: its send buffer (read by the PULL reduce) and recvbuf
+  const uint8_t *p_sendbuf[kMaxDirect - 1];
+  uint8_t *p_recvbuf[kMaxDirect - 1];
   uint32_t *p_cnt[kMaxDirect - 1];
   int32_t *err;
   uint32_t timeout_ms;

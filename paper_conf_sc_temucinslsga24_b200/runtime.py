@@ -255,7 +255,8 @@ class Request:
         a, s, w = C.c_int32(), C.c_int32(), C.c_int32()
         q = C.c_int64()
         check(_lib.pc().pc_request_info(self.handle, C.byref(a), C.byref(s), C.byref(q), C.byref(w)), "info")
-        return {"algo": a.value, "slices": s.value, "slice_elems": q.value, "engine_warps": w.value}
+        return {"algo": a.value, "algo_name": {1: "ring", 2: "rd", 3: "direct"}.get(a.value, "?"), "slices": s.value,
+                "slice_elems": q.value, "engine_warps": w.value}
 
     def match(self) -> tuple[int, int]:
         p, i = C.c_int32(), C.c_int32()

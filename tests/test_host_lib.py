@@ -127,8 +127,9 @@ def test_dry_allreduce_agreement_and_algo_choice():
     for q in reqs + small:
         q.start()
     pc.run_ranks([(lambda r=r: (reqs[r].pbuf_prepare(), small[r].pbuf_prepare())) for r in range(4)])
-    assert all(q.info()["algo"] == pc.ALGO_RING for q in reqs)
-    assert all(q.info()["algo"] == pc.ALGO_RD for q in small)
+    # AUTO (profiles/r01_sweep_allreduce_pull.jsonl): DIRECT (pull) for 3 <= P <= 8
+    assert all(q.info()["algo"] == pc.ALGO_DIRECT for q in reqs)
+    assert all(q.info()["algo"] == pc.ALGO_DIRECT for q in small)
     infos = {tuple(sorted(q.info().items())) for q in reqs}
     assert len(infos) == 1, "every rank must derive the same slicing"
     # disagreeing allreduce (different count on rank 3) -> PC_ERR_MATCH everywhere it is checked
@@ -224,3 +225,22 @@ def test_gloo_two_process_bootstrap_and_matching(tmp_path):
     for r, (p, o) in enumerate(zip(procs, outs)):
         assert p.returncode == 0, o
         assert f"OK {r}" in o
+
+
+@pytest.mark.parametrize("P,nbytes,want", [(2, 1024, "RD"), (2, 4 << 20, "RD"), (2, 8 << 20, "DIRECT"),
+                                          (3, 1024, "DIRECT"), (8, 1024, "DIRECT"), (8, 64 << 20, "DIRECT")])
+def test_dry_auto_schedule_policy(P, nbytes, want):
+    """AUTO: RD for P = 2 up to 4 MiB, DIRECT for P <= 8 otherwise (beyond
+    DIRECT's peer limit — more ranks than one process can host dry — RD for
+    small messages, ring above)."""
+    g, cs = _dry(P)
+    reqs = [pc.pallreduce_init(0, 0, 1, nbytes // 4, pc.FLOAT32, pc.SUM, pc.ALGO_AUTO, c) for c in cs]
+    for q in reqs:
+        q.start()
+    pc.run_ranks([(lambda r=r: reqs[r].pbuf_prepare()) for r in range(P)])
+    assert all(q.info()["algo"] == getattr(pc, "ALGO_" + want) for q in reqs)
+    for q in reqs:
+        q.wait()
+    for c in cs:
+        c.destroy()
+    g.destroy()
