@@ -434,7 +434,7 @@ def run_virtual(args):
     alg_bytes = engine_alg_bytes(info["algo_name"], P, S)
     achieved = alg_bytes / (eng_ms / 1e3) / 1e9 if eng_ms else None
     traffic = None
-    tp = os.path.join(ROOT, "profiles", "engine_traffic.json")
+    tp = os.path.join(ROOT, "profiles", f"engine_traffic_{info['algo_name']}.json")
     if os.path.exists(tp):
         try:
             t = json.load(open(tp))

@@ -21,7 +21,7 @@ torch.cuda.set_device(0)
 comm = pc.Comm.from_process_group(0)
 st = torch.cuda.Stream()
 res = {}
-for name, algo in (("ring", pc.ALGO_RING), ("rd", pc.ALGO_RD)):
+for name, algo in (("ring", pc.ALGO_RING), ("rd", pc.ALGO_RD), ("direct", pc.ALGO_DIRECT)):
     Np, L = 3, 1000
     x = synth.normal_f32(synth.BASE_SEED, r, 0, Np * L)
     send = torch.from_numpy(x).cuda()
@@ -75,6 +75,28 @@ for e in range(2):
     assert q.error() == (0, 0), q.error()
 if r == 0:
     res["p2p_engine"] = rb2.cpu().numpy()
+q.free()
+# LL p2p 0 -> 1 (16-B lines over CUDA IPC), warp-granularity Pready, 3 epochs
+# (both line-area parities, the sender's completion acquires the receiver's RTR)
+nl = 2048 * 2  # whole 1024-thread blocks (vecadd launches ceil(n/2048) blocks)
+if r == 0:
+    a3 = torch.from_numpy(synth.uniform_f32(synth.BASE_SEED, 0, 7, nl)).cuda()
+    c3 = torch.empty(nl, device="cuda")
+    q = pc.psend_init(c3, nl // 64, 64, pc.FLOAT32, 1, 13, comm)
+else:
+    rb3 = torch.zeros(nl, device="cuda")
+    q = pc.precv_init(rb3, nl // 64, 64, pc.FLOAT32, 0, 13, comm)
+for e in range(3):
+    q.start(st)
+    q.pbuf_prepare(st)
+    if e == 0:
+        pq = q.prequest_create(pc.GRAN_WARP, 1, pc.COPY_LL if r == 0 else pc.COPY_INLINE)
+    if r == 0:
+        apps.vecadd(a3, a3, c3, nl, apps.GRAN_WARP, pq, st)
+    q.wait()
+    assert q.error() == (0, 0), q.error()
+if r == 1:
+    res["p2p_ll"] = rb3.cpu().numpy()
 q.free()
 # Jacobi 2 x 1 across the two processes (one rank each), halos over CUDA IPC
 js = apps.JacobiSolver([comm], [r], 256, 2, 1, 30, H=32)

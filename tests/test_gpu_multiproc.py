@@ -25,7 +25,7 @@ def test_two_processes_ipc(tmp_path):
     res = [np.load(os.path.join(tmp_path, f"rank{r}.npz")) for r in range(2)]
     Np, L = 3, 1000
     x = np.stack([synth.normal_f32(synth.BASE_SEED, r, 0, Np * L) for r in range(2)])
-    for name, algo in (("ring", oracle.RING), ("rd", oracle.RD)):
+    for name, algo in (("ring", oracle.RING), ("rd", oracle.RD), ("direct", oracle.DIRECT)):
         ref, _, _ = oracle.pallreduce(x, Np, algo)
         for r in range(2):
             np.testing.assert_array_equal(res[r][name].view(np.uint32), ref[r].view(np.uint32))
@@ -38,6 +38,8 @@ def test_two_processes_ipc(tmp_path):
     np.testing.assert_array_equal(res[1]["p2p"].view(np.uint8), consumed[0])
     a2 = synth.uniform_f32(synth.BASE_SEED, 1, 0, n)
     np.testing.assert_array_equal(res[0]["p2p_engine"], (a2 + a2).astype(np.float32))
+    a3 = synth.uniform_f32(synth.BASE_SEED, 0, 7, 2048 * 2)
+    np.testing.assert_array_equal(res[1]["p2p_ll"], (a3 + a3).astype(np.float32))
     # Jacobi: each process holds its own block; together they equal the oracle
     ref = oracle.jacobi_seq(synth.jacobi_init(256, 256, "random"), 30)
     np.testing.assert_array_equal(res[0]["jacobi"][:128], ref[:128])
