@@ -128,6 +128,33 @@ int pc_precv_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, int
 int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
                        pc_op_t op, pc_algo_t algo, pc_comm_t comm, pc_request_t *req);
 
+/* Partitioned reduce-scatter / allgather / broadcast (the two
+ * halves of the DIRECT allreduce schedule and its one-to-all case; the generic
+ * schedule of P:L151-L155 with neighbour sets).  Collective, like
+ * pc_pallreduce_init (shared posting order), P <= 8.  Schedule: reduce-scatter
+ * PULLS (owners fold the peers' blocks with peer loads, rank order, reading
+ * R25); allgather and broadcast PUSH 16-B vectors into the peers' buffers.
+ *
+ * reduce_scatter: sendbuf partitions x P x count elements (partition u = P
+ *   blocks of count, block k for rank k); recvbuf partitions x count:
+ *   recvbuf[u] = op-fold over ranks 0..P-1 (in rank order) of sendbuf_k[u][me]
+ *   (MPI_Reduce_scatter_block per partition).  dtype INT32/FLOAT32/FLOAT64/BF16.
+ *   pc_pready(u): sendbuf[u] final.  pc_parrived(u): recvbuf[u] final and every
+ *   peer done reading sendbuf[u].
+ * allgather: sendbuf partitions x count; recvbuf P x partitions x count (rank
+ *   major, as MPI_Allgather of the whole buffer): recvbuf[k][u] = sendbuf_k[u].
+ *   Any dtype (bytes move).  pc_pready(u): sendbuf[u] final.  Receive
+ *   partitions are the P x partitions blocks: pc_parrived(k * partitions + u)
+ *   = rank k's partition u is in recvbuf.
+ * bcast: buf partitions x count on every rank; the root's pc_pready(u) delivers
+ *   buf[u] to every rank; pc_parrived(u) = buf[u] holds the root's data. */
+int pc_preduce_scatter_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
+                            pc_op_t op, pc_comm_t comm, pc_request_t *req);
+int pc_pallgather_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
+                       pc_comm_t comm, pc_request_t *req);
+int pc_pbcast_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, int root, pc_comm_t comm,
+                   pc_request_t *req);
+
 /* ---------------------------------------------------------------- epoch
  * MPI_Start: epoch e <- e+1, written stream-ordered to the device
  * epoch word; for ENGINE copy and allreduce it also launches the engine on a

@@ -572,10 +572,22 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
 }
 
 /* ---------------------------------------------------------------- Parrived */
+/* Allgather receive partition u' = k * partitions + u (rank k's partition u):
+ * all of its slices' arrival epochs (written by rank k after its pushes). */
+namespace pc_detail {
+PC_DEVICE bool ag_arrived(const pc_prequest_t &q, int up, uint32_t e) {
+  for (uint32_t s = 0; s < q.done_mul; ++s)
+    if (!reached(ld_acquire_scope(q.srcflags + (uint64_t)up * q.done_mul + s, q.sys_scope), e)) return false;
+  return true;
+}
+}  // namespace pc_detail
+
 PC_DEVICE int pc_parrived(pc_prequest_t preq, int partition) {
   using namespace pc_detail;
-  if (partition < 0 || partition >= preq.partitions) return 0;
+  const bool ag = preq.kind == PC_KIND_PALLREDUCE && preq.coll == 2;
+  if (partition < 0 || partition >= (ag ? preq.nranks * preq.partitions : preq.partitions)) return 0;
   const uint32_t e = epoch_of(preq);
+  if (ag) return ag_arrived(preq, partition, e) ? 1 : 0;
   if (preq.kind == PC_KIND_PALLREDUCE) return reached(ld_acquire_gpu(preq.done + partition), e * preq.done_mul);
   if (preq.kind == PC_KIND_PSEND) {
     const int t = partition / preq.agg;
@@ -592,9 +604,24 @@ PC_DEVICE int pc_parrived(pc_prequest_t preq, int partition) {
  * ld.acquire of the partition's flag (one L2 round trip per poll). */
 PC_DEVICE int pc_wait_arrived(pc_prequest_t preq, int partition) {
   using namespace pc_detail;
-  if (partition < 0 || partition >= preq.partitions) return PC_DEV_ERR_ARG;
+  const bool ag = preq.kind == PC_KIND_PALLREDUCE && preq.coll == 2;
+  if (partition < 0 || partition >= (ag ? preq.nranks * preq.partitions : preq.partitions)) return PC_DEV_ERR_ARG;
   const uint64_t t0 = globaltimer();
   const uint32_t e = epoch_of(preq);
+  if (ag) {
+    uint32_t n = 0;
+    while (!ag_arrived(preq, partition, e)) {
+      if ((++n & 127) == 0) {
+        if (aborted(preq.err)) return PC_DEV_ERR_TIMEOUT;
+        if (preq.timeout_ms && globaltimer() - t0 > (uint64_t)preq.timeout_ms * 1000000ull) {
+          set_error(preq.err, PC_DEV_ERR_TIMEOUT, partition);
+          return PC_DEV_ERR_TIMEOUT;
+        }
+        if (n > 4096) __nanosleep(128);
+      }
+    }
+    return 0;
+  }
   const uint32_t *w;
   uint32_t target = e;
   bool sys = false;

@@ -55,6 +55,11 @@ struct pc_prequest_s {
   uint8_t *peer_ll;           /* send, PC_COPY_LL: receiver's LL area (peer-mapped)        */
   uint8_t *ll;                /* receive: own LL area [2 epoch parities][N_p][ll_lines]   */
   uint8_t *rbuf;              /* receive: own recv buffer (LL lines are unpacked into it) */
+  /* partitioned collectives (pc_preduce_scatter_init / pc_pallgather_init /
+   * pc_pbcast_init): kind PC_KIND_PALLREDUCE with coll != 0 */
+  uint32_t coll;              /* 0 allreduce, 1 reduce-scatter, 2 allgather, 3 broadcast    */
+  int32_t nranks;             /* P (allgather: receive partitions = P * partitions)        */
+  const uint32_t *srcflags;   /* allgather: [source rank][u][slice] arrival epochs         */
 };
 
 /* Receive side: bit 31 of the layout word = the sender pushes LL lines. */

@@ -16,6 +16,9 @@ Functions (numpy in, numpy out):
   alg1_table(P, r)        Alg 1 step tuples
   ring_fold_f32 / rd_tree_f32   closed forms of O3 / O4 (pinned against them)
   jacobi_seq / jacobi_decomp    O5
+  reduce_scatter_def(...) O8  partitioned reduce-scatter, plain definition (rank-order fold, R25)
+  allgather_def(...)      O9  partitioned allgather, plain definition (concatenation)
+  bcast_def(...)          O10 partitioned broadcast, plain definition (copy of the root's buffer)
 """
 from __future__ import annotations
 
@@ -237,3 +240,55 @@ def jacobi_decomp(a0: np.ndarray, iters: int, Py: int, Px: int) -> np.ndarray:
     out = np.zeros_like(a0)
     _check(lib().orc_jacobi_decomp(ny, nx, Py, Px, iters, _p(a0), _p(out)), "jacobi_decomp")
     return out
+
+
+# --------------------------------------------------------------------------- NEXT-3 collectives
+# Plain definitions (generic schedule P:L151-L155, MPI_Op P:L155).
+def _op(a: np.ndarray, b: np.ndarray, op: int) -> np.ndarray:
+    """One element-wise a ⊕ b in the element type: int32 sum wraps mod 2^32;
+    fp32/fp64 one IEEE op (RN-even; max/min = IEEE maxNum/minNum like
+    std::fmax in oracle.cpp); bf16 (uint16 bit patterns) via the R27 oracle."""
+    if a.dtype == np.uint16:
+        return bf16_op(a, b, op)
+    if a.dtype == np.int32:
+        if op == SUM:
+            return (a.view(np.uint32) + b.view(np.uint32)).view(np.int32)
+        return np.maximum(a, b) if op == MAX else np.minimum(a, b)
+    if op == SUM:
+        return a + b  # numpy float32 / float64 add: one IEEE op, round to nearest even
+    return np.fmax(a, b) if op == MAX else np.fmin(a, b)
+
+
+def reduce_scatter_def(x: np.ndarray, partitions: int, op: int = SUM) -> np.ndarray:
+    """O8.  x: (P, partitions * P * count), rank k's send buffer: partition u =
+    P blocks of count, block d destined to rank d.  Returns y: (P, partitions *
+    count), y[d][u] = x[0][u][d] ⊕ x[1][u][d] ⊕ ... ⊕ x[P-1][u][d], folded left
+    in rank order (reading R25 — the DIRECT schedule's association)."""
+    x = np.ascontiguousarray(x)
+    P = x.shape[0]
+    count = x.shape[1] // (partitions * P)
+    assert count * partitions * P == x.shape[1]
+    blocks = x.reshape(P, partitions, P, count)  # [source k][u][destination d][i]
+    y = np.empty((P, partitions, count), dtype=x.dtype)
+    for d in range(P):
+        acc = blocks[0, :, d, :].copy()
+        for k in range(1, P):
+            acc = _op(acc, blocks[k, :, d, :], op)
+        y[d] = acc
+    return y.reshape(P, partitions * count)
+
+
+def allgather_def(x: np.ndarray) -> np.ndarray:
+    """O9.  x: (P, n) send buffers.  Every rank's receive buffer is the rank-
+    major concatenation x[0] | x[1] | ... | x[P-1] (MPI_Allgather).  Returns
+    (P, P * n)."""
+    x = np.ascontiguousarray(x)
+    P = x.shape[0]
+    return np.tile(x.reshape(1, -1), (P, 1))
+
+
+def bcast_def(x: np.ndarray, root: int) -> np.ndarray:
+    """O10.  x: (P, n) buffers before the broadcast; afterwards every rank holds
+    the root's buffer."""
+    x = np.ascontiguousarray(x)
+    return np.tile(x[root][None], (x.shape[0], 1))

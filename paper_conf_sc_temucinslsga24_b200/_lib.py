@@ -42,6 +42,9 @@ _PC_PROTOS = {
     "pc_psend_init": (I32, [P, I32, SZ, I32, I32, I32, P, C.POINTER(P)]),
     "pc_precv_init": (I32, [P, I32, SZ, I32, I32, I32, P, C.POINTER(P)]),
     "pc_pallreduce_init": (I32, [P, P, I32, SZ, I32, I32, I32, P, C.POINTER(P)]),
+    "pc_preduce_scatter_init": (I32, [P, P, I32, SZ, I32, I32, P, C.POINTER(P)]),
+    "pc_pallgather_init": (I32, [P, P, I32, SZ, I32, P, C.POINTER(P)]),
+    "pc_pbcast_init": (I32, [P, I32, SZ, I32, I32, P, C.POINTER(P)]),
     "pc_start": (I32, [P, P]),
     "pc_startall": (I32, [I32, P, P]),
     "pc_pbuf_prepare_all": (I32, [I32, P, P]),

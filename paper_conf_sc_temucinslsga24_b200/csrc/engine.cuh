@@ -460,25 +460,33 @@ __device__ __forceinline__ void red_add_scope(uint32_t *p, uint32_t v, bool sys)
 // peer loads (PULL).  All operands sit at the same element offset of 16-B
 // aligned buffers: scalar head, 16-B body, scalar tail.  Buffer pointers come
 // straight from the kernel parameters (no pointer arrays on the stack).
-template <int DT, int OP>
-__device__ __forceinline__ void warp_fold_direct(const DirectArgs &a, int64_t e0, int64_t n) {
+// A: DirectArgs or CollArgs (sendbuf, p_sendbuf, recvbuf, p_recvbuf, P, r).
+// Sources at element offset s0 of every rank's send buffer, destination at d0
+// of this rank's recvbuf and (TO_PEERS) of every peer's.  When the sources and
+// the destination do not share a 16-B misalignment the whole range takes the
+// scalar path.
+template <int DT, int OP, bool TO_PEERS = true, typename A>
+__device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d0, int64_t n) {
   using O = Op<DT, OP>;
   using T = typename O::T;
   const int P = a.P, r = a.r;
   const uint32_t lane = threadIdx.x & 31;
   constexpr int64_t EPV = 16 / sizeof(T);
   auto src = [&](int k) -> const T * {
-    return reinterpret_cast<const T *>(k == r ? a.sendbuf : a.p_sendbuf[(k - r - 1 + P) % P]) + e0;
+    return reinterpret_cast<const T *>(k == r ? a.sendbuf : a.p_sendbuf[(k - r - 1 + P) % P]) + s0;
   };
+  const int64_t e0 = d0;
   T *out_local = reinterpret_cast<T *>(a.recvbuf) + e0;
   const uintptr_t m = reinterpret_cast<uintptr_t>(out_local) & 15;
   int64_t head = (int64_t)(((16 - m) & 15) / sizeof(T));
+  if ((reinterpret_cast<uintptr_t>(src(r)) & 15) != m) head = n;  // no common misalignment
   if (head > n) head = n;
   auto scalar = [&](int64_t k) {
     T acc = __ldcg(src(0) + k);
     for (int j = 1; j < P; ++j) acc = O::f(acc, __ldcg(src(j) + k));
     out_local[k] = acc;
-    for (int j = 0; j < P - 1; ++j) (reinterpret_cast<T *>(a.p_recvbuf[j]) + e0)[k] = acc;
+    if (TO_PEERS)
+      for (int j = 0; j < P - 1; ++j) (reinterpret_cast<T *>(a.p_recvbuf[j]) + e0)[k] = acc;
   };
   for (int64_t k = lane; k < head; k += 32) scalar(k);
   const int64_t nv = (n - head) / EPV;
@@ -488,9 +496,11 @@ __device__ __forceinline__ void warp_fold_direct(const DirectArgs &a, int64_t e0
   auto store_all = [&](int64_t vk, uint4 acc) {
     const int64_t eo = head + EPV * vk;
     *reinterpret_cast<uint4 *>(out_local + eo) = acc;
+    if (TO_PEERS) {
 #pragma unroll
-    for (int j = 0; j < kMaxDirect - 1; ++j)
-      if (j < P - 1) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(a.p_recvbuf[j]) + e0 + eo) = acc;
+      for (int j = 0; j < kMaxDirect - 1; ++j)
+        if (j < P - 1) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(a.p_recvbuf[j]) + e0 + eo) = acc;
+    }
   };
   int64_t k = lane;
   for (; k + 32 * (kFV - 1) < nv; k += 32 * kFV) {
@@ -577,7 +587,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
         } else if (i == 1) {
           const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
           const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-          if (hi > lo) warp_fold_direct<DT, OP>(a, base + lo, hi - lo);
+          if (hi > lo) warp_fold_pull<DT, OP>(a, base + lo, base + lo, hi - lo);
           fence_scope(a.sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
@@ -595,6 +605,136 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
         return;
     }
   }
+}
+
+// ---------------------------------------------------------------------------
+// Partitioned reduce-scatter / allgather / broadcast: the two
+// halves of the DIRECT schedule and its one-to-all special case, same unit
+// sweep (Alg 2 on a warp).  Unit (u, slice s) of one block of `count` elements.
+//  REDUCE_SCATTER (sendbuf [u][P blocks], recvbuf [u][count]), PULL:
+//    0: ready[u] -> announce to every peer (phase-0 counter)
+//    1: P-1 announcements -> fold block r of partition u over all ranks in rank
+//       order (peer loads) into my recvbuf[u]; tell every peer "done reading"
+//    2: P-1 "done reading" -> done[u]  (my send buffer is reusable)
+//  ALLGATHER (sendbuf [u][count], recvbuf [rank][u][count]), PUSH:
+//    0: ready[u] -> copy my block to recvbuf[r][u] here and at every peer,
+//       fence, per-source arrival flag + phase-0 counter at every peer
+//    1: P-1 arrivals of partition u -> done[u]
+//  BCAST (buf [u][count]) root: ready[u] -> push to every peer -> done[u];
+//    non-root: root's arrival (phase-0 counter) -> done[u]
+// ---------------------------------------------------------------------------
+template <int DT, int OP>
+__device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const int W) {
+  const int P = a.P, r = a.r;
+  const uint32_t e = *(const volatile uint32_t *)a.epoch;
+  const int64_t es = a.es;
+  if (gw >= a.nunits) return;
+  const bool rs = a.coll == PC_COLL_REDUCE_SCATTER, ag = a.coll == PC_COLL_ALLGATHER;
+  const bool bc = a.coll == PC_COLL_BCAST, root = bc && r == a.root;
+  // writers into peers' buffers need every peer's ready-to-receive
+  if (P > 1 && (ag || root))
+    for (int j = 0; j < P - 1; ++j)
+      if (!warp_wait(a.rtr + j, e, a.err, a.timeout_ms, -1, a.sys)) return;
+  const uint32_t target = e * (uint32_t)(P - 1);
+  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
+    int step[kMaxActive];
+    int remaining = 0;
+#pragma unroll
+    for (int j = 0; j < kMaxActive; ++j) {
+      const bool mine = gw + (j0 + j) * W < a.nunits;
+      step[j] = mine ? 0 : 3;
+      remaining += mine;
+    }
+    Idle idle;
+    while (remaining) {
+      bool progressed = false;
+#pragma unroll
+      for (int jj = 0; jj < kMaxActive; ++jj) {
+        if (step[jj] > 2) continue;
+        const int x = gw + (j0 + jj) * W;
+        const int u = x / a.ns, s = x % a.ns;
+        const int i = step[jj];
+        const int64_t lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.count), n = hi > lo ? hi - lo : 0;
+        const uint32_t *cnt_u = a.cnt + (int64_t)u * 2 * a.ns + s;  // phase p at cnt_u[p * ns]
+        bool finished = false;
+        if (P == 1) {  // one rank: the result is the input
+          if (!warp_poll(a.ready + u, e, false)) continue;
+          if (n && !bc) {
+            const int64_t so = rs ? (int64_t)u * a.count + lo : (int64_t)u * a.count + lo;
+            warp_copy(a.recvbuf + so * es, a.sendbuf + so * es, n * es);
+          }
+          if (ag && (threadIdx.x & 31) == 0) st_release_gpu(a.srcflags + (int64_t)u * a.ns + s, e);
+          finished = true;
+        } else if (bc && !root) {
+          if (!warp_poll(cnt_u, e, a.sys)) continue;
+          finished = true;
+        } else if (i == 0) {
+          if (!warp_poll(a.ready + u, e, false)) continue;
+          const int64_t off = ((int64_t)u * a.count + lo) * es;  // my block (AG, BCAST)
+          if (ag) {
+            const int64_t doff = (((int64_t)r * a.Np + u) * a.count + lo) * es;
+            if (n) {
+              warp_copy(a.recvbuf + doff, a.sendbuf + off, n * es);
+              for (int j = 0; j < P - 1; ++j) warp_copy(a.p_recvbuf[j] + doff, a.sendbuf + off, n * es);
+            }
+          } else if (root && n) {
+            for (int j = 0; j < P - 1; ++j) warp_copy(a.p_recvbuf[j] + off, a.sendbuf + off, n * es);
+          }
+          fence_scope(a.sys);
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0) {
+            for (int j = 0; j < P - 1; ++j) {
+              if (ag) st_relaxed_sys(a.p_srcflags[j] + ((int64_t)r * a.Np + u) * a.ns + s, e);
+              red_add_scope(a.p_cnt[j] + (int64_t)u * 2 * a.ns + s, 1, a.sys);
+            }
+            if (ag) st_release_gpu(a.srcflags + ((int64_t)r * a.Np + u) * a.ns + s, e);
+          }
+          if (root) finished = true;
+          else step[jj] = 1;
+        } else if (i == 1) {
+          if (!warp_poll(cnt_u, target, a.sys)) continue;
+          if (rs) {
+            if (n)
+              warp_fold_pull<DT, OP, false>(a, ((int64_t)u * P + r) * a.count + lo, (int64_t)u * a.count + lo, n);
+            fence_scope(a.sys);
+            __syncwarp();
+            if ((threadIdx.x & 31) == 0)
+              for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
+            step[jj] = 2;
+          } else {
+            finished = true;
+          }
+        } else {  // RS step 2: every peer finished reading my partition u
+          if (!warp_poll(cnt_u + a.ns, target, a.sys)) continue;
+          finished = true;
+        }
+        progressed = true;
+        if (finished) {
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+          step[jj] = 3;
+          --remaining;
+        }
+      }
+      if (progressed)
+        idle.progressed();
+      else if (!idle.wait(a.err, a.timeout_ms, gw))
+        return;
+    }
+  }
+}
+
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock, 2) coll_engine(CollArgs a) {
+  coll_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
+}
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock, 2) coll_engine_group(CollGroupArgs g) {
+  int k = 0;
+  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
+  const int b = blockIdx.x - g.block_start[k];
+  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
+  coll_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
 }
 
 template <int DT, int OP>
@@ -664,6 +804,8 @@ struct EngineLaunch {
   static int ring_group(const RingGroupArgs &h, int blocks, cudaStream_t s);
   static int rd_group(const RdGroupArgs &h, int blocks, cudaStream_t s);
   static int direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s);
+  static int coll(const CollArgs &a, int warps, cudaStream_t s);
+  static int coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s);
   static int occupancy(int *ctas);
 };
 

@@ -66,6 +66,22 @@ int EngineLaunch<DT, OP>::occupancy(int *ctas) {
   return 0;
 }
 
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::coll(const CollArgs &a, int warps, cudaStream_t s) {
+  coll_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s) {
+  coll_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
 template struct EngineLaunch<PC_DT, PC_OP>;
 
 }  // namespace pc

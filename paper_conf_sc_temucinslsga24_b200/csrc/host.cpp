@@ -324,6 +324,10 @@ static void fill_prequest(Request *q, pc_prequest_t *o) {
   o->sys_scope = (uint32_t)q->sys_scope;
   o->err = (int32_t *)(q->ctrl + q->L.err);
   o->ll_lines = q->ll_lines;
+  o->coll = (uint32_t)q->coll;
+  o->nranks = q->comm->size;
+  if (q->kind == PC_KIND_PALLREDUCE && q->coll == PC_COLL_ALLGATHER)
+    o->srcflags = q->ctrl + q->L.flags + (size_t)q->partitions * 2 * q->slices;
   if (q->kind == PC_KIND_PSEND) {
     o->peer_rbuf = q->peer_buf;
     o->peer_flags = q->peer_ctrl ? q->peer_ctrl + q->L.flags : nullptr;
@@ -389,6 +393,8 @@ static int make_rec(Request *q, ReqRec *r) {
   r->op = q->op;
   r->algo = q->algo;
   r->seq = q->seq;
+  r->coll = q->coll;
+  r->root = q->root;
   r->owner = c->rank;
   r->req_index = q->index;
   r->host_req = (uint64_t)(uintptr_t)q;
@@ -399,7 +405,8 @@ static int make_rec(Request *q, ReqRec *r) {
   if (q->staging && (rc = export_ptr(c, q->staging, q->staging_bytes, &r->stage))) return rc;
   // DIRECT (PULL): the peers' reduce steps read this rank's send buffer
   if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && c->size > 1 &&
-      (rc = export_ptr(c, q->sbuf, q->total_bytes, &r->stage)))
+      (q->coll == PC_COLL_ALLREDUCE || q->coll == PC_COLL_REDUCE_SCATTER) &&
+      (rc = export_ptr(c, q->sbuf, q->send_bytes, &r->stage)))
     return rc;
   return 0;
 }
@@ -473,7 +480,7 @@ static int exchange_round(Comm *c, Request *target) {
       for (int r = 0; r < c->size && !qrc; ++r) {
         const ReqRec *m = find_rec(all, M, r, PC_KIND_PALLREDUCE, -1, 0, q->seq, cnt);
         if (!m || m->partitions != q->partitions || m->count != (int64_t)q->count || m->dtype != q->dtype ||
-            m->op != q->op || m->algo != q->algo) {
+            m->op != q->op || m->algo != q->algo || m->coll != q->coll || m->root != q->root) {
           fprintf(stderr, "[pc] rank %d: allreduce #%d disagrees with rank %d\n", c->rank, q->seq, r);
           qrc = PC_ERR_MATCH;
         }
@@ -656,6 +663,42 @@ static DirectArgs make_direct_args(Request *q) {
   return a;
 }
 
+static CollArgs make_coll_args(Request *q) {
+  Comm *c = q->comm;
+  CollArgs a{};
+  a.epoch = q->ctrl + q->L.epoch;
+  a.coll = q->coll;
+  a.P = c->size;
+  a.r = c->rank;
+  a.root = q->root;
+  a.Np = q->partitions;
+  a.ns = q->slices;
+  a.nunits = q->partitions * q->slices;
+  a.op = q->op;
+  a.dtype = q->dtype;
+  a.count = (int64_t)q->count;
+  a.qs = q->slice_elems;
+  a.es = (int64_t)q->esize;
+  a.sendbuf = (const uint8_t *)q->sbuf;
+  a.recvbuf = (uint8_t *)q->rbuf;
+  a.cnt = q->ctrl + q->L.flags;
+  a.ready = q->ctrl + q->L.ready;
+  a.rtr = q->ctrl + q->L.rtr;
+  a.done = q->ctrl + q->L.donecnt;
+  const size_t sf = (size_t)q->partitions * 2 * q->slices;  // allgather source flags follow the counters
+  a.srcflags = q->ctrl + q->L.flags + sf;
+  for (int j = 0; j < c->size - 1; ++j) {
+    a.p_sendbuf[j] = q->nb_stage[j];
+    a.p_recvbuf[j] = q->nb_buf[j];
+    a.p_cnt[j] = q->nb_ctrl[j] + q->L.flags;
+    a.p_srcflags[j] = q->nb_ctrl[j] + q->L.flags + sf;
+  }
+  a.err = (int32_t *)(q->ctrl + q->L.err);
+  a.timeout_ms = c->timeout_ms;
+  a.sys = q->sys_scope;
+  return a;
+}
+
 static bool needs_engine(Request *q) {
   return q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
 }
@@ -685,7 +728,9 @@ static int launch_single(Request *q) {
   PC_CUDA(cudaStreamWaitEvent(q->side, q->ev_fork, 0));
   int rc, tk;
   if ((rc = timing_begin(q->tlog, q->side, &tk))) return rc;
-  if (q->kind == PC_KIND_PALLREDUCE) {
+  if (q->kind == PC_KIND_PALLREDUCE && q->coll != PC_COLL_ALLREDUCE) {
+    rc = launch_coll_engine(make_coll_args(q), q->engine_warps, q->side);
+  } else if (q->kind == PC_KIND_PALLREDUCE) {
     rc = q->algo == PC_ALGO_RING     ? launch_ring_engine(make_ring_args(q), q->engine_warps, q->side)
          : q->algo == PC_ALGO_DIRECT ? launch_direct_engine(make_direct_args(q), q->engine_warps, q->side)
                                      : launch_rd_engine(make_rd_args(q), q->engine_warps, q->side);
@@ -742,7 +787,12 @@ static int group_register(Request *q, bool block, bool *launched) {
     for (Request *m : g.members) PC_CUDA(cudaStreamWaitEvent(q->side, m->ev_fork, 0));
     int rc, tk;
     if ((rc = timing_begin(g.tlog, q->side, &tk))) return rc;
-    if (q->algo == PC_ALGO_RING) {
+    if (q->coll != PC_COLL_ALLREDUCE) {
+      CollGroupArgs ga{};
+      ga.n = (int)g.members.size();
+      for (int k = 0; k < ga.n; ++k) ga.a[k] = make_coll_args(g.members[k]);
+      rc = launch_coll_engine_group(ga, q->engine_warps, q->side);
+    } else if (q->algo == PC_ALGO_RING) {
       RingGroupArgs ga{};
       ga.n = (int)g.members.size();
       for (int k = 0; k < ga.n; ++k) ga.a[k] = make_ring_args(g.members[k]);
@@ -1028,6 +1078,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   q->tag = 0;
   q->part_bytes = count * esz;
   q->total_bytes = bytes;
+  q->send_bytes = bytes;
   q->seq = c->allreduce_seq++;
   q->agg = 1;
   q->ntransport = partitions;
@@ -1056,6 +1107,74 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   const size_t nflags = (size_t)partitions * (size_t)std::max(q->nsteps, 1) * (size_t)q->slices;
   q->L.build((size_t)partitions, nflags);
   return 0;
+}
+
+// Partitioned reduce-scatter / allgather / broadcast: one
+// collective request on the DIRECT machinery (all peers mapped, per-peer RTR,
+// co-located grouped launch), engine coll_body.  Collective over the comm:
+// every rank calls it with identical arguments, in the same order as its other
+// collective inits (they share the allreduce sequence numbers).
+static int coll_init(int coll, const void *sendbuf, void *recvbuf, int partitions, size_t count, int dtype, int op,
+                     int root, Comm *c, pc_request_t *req) {
+  if (!c || !req || partitions < 1 || op < 0 || op > 2) return PC_ERR_ARG;
+  const int P = c->size;
+  if (coll == PC_COLL_REDUCE_SCATTER &&
+      dtype != PC_INT32 && dtype != PC_FLOAT32 && dtype != PC_FLOAT64 && dtype != PC_BF16)
+    return PC_ERR_ARG;
+  if (dtype < 0 || dtype > 4) return PC_ERR_ARG;
+  if (coll == PC_COLL_BCAST && (root < 0 || root >= P)) return PC_ERR_ARG;
+  if (P > kMaxDirect) return PC_ERR_UNSUPPORTED;
+  const size_t esz = dtype_size(dtype);
+  const uint64_t blk = (uint64_t)partitions * count * esz;  // one rank's block set
+  const uint64_t sbytes = coll == PC_COLL_REDUCE_SCATTER ? blk * P : blk;
+  const uint64_t rbytes = coll == PC_COLL_ALLGATHER ? blk * P : blk;
+  if (!c->dry && (check_buf(sendbuf, sbytes) || check_buf(recvbuf, rbytes))) return PC_ERR_ARG;
+  Request *q;
+  int rc = new_request(c, PC_KIND_PALLREDUCE, req, &q);
+  if (rc) return rc;
+  q->coll = coll;
+  q->root = coll == PC_COLL_BCAST ? root : 0;
+  q->sbuf = sendbuf;
+  q->rbuf = recvbuf;
+  q->partitions = partitions;
+  q->count = count;
+  q->dtype = dtype;
+  q->op = coll == PC_COLL_REDUCE_SCATTER ? op : 0;
+  q->algo_req = q->algo = PC_ALGO_DIRECT;
+  q->esize = esz;
+  q->peer = -1;
+  q->part_bytes = count * esz;
+  q->total_bytes = rbytes;
+  q->send_bytes = sbytes;
+  q->seq = c->allreduce_seq++;
+  q->agg = 1;
+  q->ntransport = partitions;
+  q->engine_warps = c->engine_warps;
+  q->nsteps = 2;
+  q->chunk_elems = (int64_t)count;
+  const int64_t epv = std::max<int64_t>(1, 16 / (int64_t)esz);
+  const int64_t min_elems = std::max<int64_t>(1, env_long("PC_MIN_SLICE_BYTES", 8192) / (int64_t)esz);
+  choose_slices((int64_t)count, partitions, c->engine_warps, min_elems, &q->slices, &q->slice_elems, epv);
+  q->staging_bytes = 0;
+  size_t nflags = (size_t)partitions * 2 * (size_t)q->slices;
+  if (coll == PC_COLL_ALLGATHER) nflags += (size_t)P * partitions * (size_t)q->slices;
+  q->L.build((size_t)partitions, nflags);
+  return 0;
+}
+
+int pc_preduce_scatter_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
+                            pc_op_t op, pc_comm_t comm, pc_request_t *req) {
+  return coll_init(PC_COLL_REDUCE_SCATTER, sendbuf, recvbuf, partitions, count, dtype, op, 0, (Comm *)comm, req);
+}
+
+int pc_pallgather_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
+                       pc_comm_t comm, pc_request_t *req) {
+  return coll_init(PC_COLL_ALLGATHER, sendbuf, recvbuf, partitions, count, dtype, 0, 0, (Comm *)comm, req);
+}
+
+int pc_pbcast_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, int root, pc_comm_t comm,
+                   pc_request_t *req) {
+  return coll_init(PC_COLL_BCAST, buf, buf, partitions, count, dtype, 0, root, (Comm *)comm, req);
 }
 
 int pc_start(pc_request_t req, pc_stream_t stream) {
@@ -1351,14 +1470,21 @@ static int current_epoch(Request *q, uint32_t *e) {
 
 int pc_parrived(pc_request_t req, int partition, int *flag) {
   Request *q = (Request *)req;
-  if (!q || !flag || partition < 0 || partition >= q->partitions) return PC_ERR_ARG;
+  const bool ag = q && q->kind == PC_KIND_PALLREDUCE && q->coll == PC_COLL_ALLGATHER;
+  if (!q || !flag || partition < 0 || partition >= (ag ? q->comm->size : 1) * q->partitions) return PC_ERR_ARG;
   *flag = 0;
   if (q->comm->dry) return 0;
   PC_CUDA(cudaSetDevice(q->comm->device));
   uint32_t v = 0, e = 0;
   int rc;
   if ((rc = current_epoch(q, &e))) return rc;
-  if (q->kind == PC_KIND_PALLREDUCE) {
+  if (ag) {  // receive partition k * partitions + u: rank k's partition u, every slice
+    std::vector<uint32_t> h((size_t)q->slices);
+    const size_t off = q->L.flags + (size_t)q->partitions * 2 * q->slices + (size_t)partition * q->slices;
+    if ((rc = read_words(q, off, h.size(), h.data()))) return rc;
+    *flag = 1;
+    for (uint32_t w : h) *flag = *flag && reached_h(w, e);
+  } else if (q->kind == PC_KIND_PALLREDUCE) {
     if ((rc = read_words(q, q->L.donecnt + partition, 1, &v))) return rc;
     *flag = reached_h(v, e * (uint32_t)q->slices);
   } else if (q->kind == PC_KIND_PRECV) {

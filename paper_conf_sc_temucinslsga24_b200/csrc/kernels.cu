@@ -245,6 +245,24 @@ int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s) {
   return dispatch(a.dtype, a.op, [&](auto E) { return decltype(E)::direct(a, warps, s); });
 }
 
+// allgather / broadcast move bytes only: any instantiation serves (fp32 sum)
+static int coll_dtype(const CollArgs &a) { return a.coll == PC_COLL_REDUCE_SCATTER ? a.dtype : PC_FLOAT32; }
+static int coll_op(const CollArgs &a) { return a.coll == PC_COLL_REDUCE_SCATTER ? a.op : PC_OP_SUM; }
+
+int launch_coll_engine(const CollArgs &a, int warps, cudaStream_t s) {
+  return dispatch(coll_dtype(a), coll_op(a), [&](auto E) { return decltype(E)::coll(a, warps, s); });
+}
+
+int launch_coll_engine_group(const CollGroupArgs &g, int warps, cudaStream_t s) {
+  CollGroupArgs h = g;
+  int blocks = 0;
+  for (int k = 0; k < g.n; ++k) {
+    h.block_start[k] = blocks;
+    blocks += grid_for(warps, g.a[k].nunits);
+  }
+  return dispatch(coll_dtype(g.a[0]), coll_op(g.a[0]), [&](auto E) { return decltype(E)::coll_group(h, blocks, s); });
+}
+
 int launch_ring_engine_group(const RingGroupArgs &g, int warps, cudaStream_t s) {
   RingGroupArgs h = g;
   int blocks = 0;

@@ -51,6 +51,7 @@ struct ReqRec {
   int32_t kind, peer, tag, partitions;
   int64_t count;
   int32_t dtype, op, algo, seq;
+  int32_t coll, root;  // collective kind (PC_COLL_*) and root (broadcast)
   int32_t owner;     // exporting rank
   int32_t req_index; // index in the owner's request list
   uint64_t host_req; // Request* in the owner's process (co-located grouping)
@@ -143,7 +144,9 @@ struct Request {
   int dtype = 0, op = 0, algo_req = 0, algo = 0;
   int peer = -1, tag = 0, seq = 0;
   size_t esize = 4;
-  uint64_t part_bytes = 0, total_bytes = 0;
+  uint64_t part_bytes = 0, total_bytes = 0;  // total_bytes: recv buffer (exported to peers)
+  uint64_t send_bytes = 0;                   // collectives: send buffer bytes (PULL export)
+  int coll = 0, root = 0;                    // PC_COLL_* for collective requests; broadcast root
 
   // state
   uint32_t epoch = 0;
@@ -294,6 +297,33 @@ struct DirectGroupArgs {
   int block_start[kMaxLocal];
   DirectArgs a[kMaxLocal];
 };
+// Partitioned reduce-scatter / allgather / broadcast on the
+// DIRECT machinery (engine.cuh coll_body).  Unit (u, slice s) of a block of
+// `count` elements.
+enum { PC_COLL_ALLREDUCE = 0, PC_COLL_REDUCE_SCATTER = 1, PC_COLL_ALLGATHER = 2, PC_COLL_BCAST = 3 };
+struct CollArgs {
+  const uint32_t *epoch;
+  int coll, P, r, root, Np, ns, nunits, op, dtype;
+  int64_t count, qs, es;  // block elements, slice elements, element size (bytes)
+  const uint8_t *sendbuf;
+  uint8_t *recvbuf;
+  const uint32_t *cnt, *ready, *rtr;  // cnt: [u][phase 0..1][slice] (written by peers)
+  uint32_t *done;
+  uint32_t *srcflags;                 // allgather: [source rank][u][slice] arrival epochs
+  const uint8_t *p_sendbuf[kMaxDirect - 1];  // peer j = rank (r+1+j) mod P
+  uint8_t *p_recvbuf[kMaxDirect - 1];
+  uint32_t *p_cnt[kMaxDirect - 1], *p_srcflags[kMaxDirect - 1];
+  int32_t *err;
+  uint32_t timeout_ms;
+  int sys;
+};
+struct CollGroupArgs {
+  int n;
+  int block_start[kMaxLocal];
+  CollArgs a[kMaxLocal];
+};
+int launch_coll_engine(const CollArgs &a, int warps, cudaStream_t s);
+int launch_coll_engine_group(const CollGroupArgs &g, int warps, cudaStream_t s);
 int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s);
 int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t s);
 struct RdGroupArgs {

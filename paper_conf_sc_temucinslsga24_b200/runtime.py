@@ -341,6 +341,30 @@ def pallreduce_init(sendbuf, recvbuf, partitions: int, count: int, dtype: int, o
     return Request(comm, h.value, KIND_PALLREDUCE, partitions * count * ESIZE[dtype], partitions)
 
 
+def preduce_scatter_init(sendbuf, recvbuf, partitions: int, count: int, dtype: int, op: int, comm: Comm) -> Request:
+    """Partitioned reduce-scatter (pc.h): sendbuf partitions x P x count, recvbuf partitions x count."""
+    h = C.c_void_p()
+    check(_lib.pc().pc_preduce_scatter_init(_ptr(sendbuf), _ptr(recvbuf), partitions, count, dtype, op,
+                                            comm.handle, C.byref(h)), "pc_preduce_scatter_init")
+    return Request(comm, h.value, KIND_PALLREDUCE, partitions * count * ESIZE[dtype], partitions)
+
+
+def pallgather_init(sendbuf, recvbuf, partitions: int, count: int, dtype: int, comm: Comm) -> Request:
+    """Partitioned allgather (pc.h): sendbuf partitions x count, recvbuf P x partitions x count."""
+    h = C.c_void_p()
+    check(_lib.pc().pc_pallgather_init(_ptr(sendbuf), _ptr(recvbuf), partitions, count, dtype, comm.handle,
+                                       C.byref(h)), "pc_pallgather_init")
+    return Request(comm, h.value, KIND_PALLREDUCE, partitions * count * ESIZE[dtype], partitions)
+
+
+def pbcast_init(buf, partitions: int, count: int, dtype: int, root: int, comm: Comm) -> Request:
+    """Partitioned broadcast (pc.h): the root's Pready(u) delivers buf[u] to every rank."""
+    h = C.c_void_p()
+    check(_lib.pc().pc_pbcast_init(_ptr(buf), partitions, count, dtype, root, comm.handle, C.byref(h)),
+          "pc_pbcast_init")
+    return Request(comm, h.value, KIND_PALLREDUCE, partitions * count * ESIZE[dtype], partitions)
+
+
 # ------------------------------------------------------------------ pure host logic
 def launch_count() -> int:
     """Kernels libpc launched in this process so far."""
