@@ -332,6 +332,7 @@ def jacobi_bench(pc, apps, torch, args):
         g, cs = pc.local_comms(P, 0)
         st = torch.cuda.Stream()
         js = apps.JacobiSolver(cs, list(range(P)), N, Py, Px, K, H=int(os.environ.get("PC_JACOBI_H", "64")))
+        res["kernel"] = f"{js.kernel} (W={js.W}, H={js.H})"
         for s in js.local:  # perf init: top edge 1.0, rest 0
             s["grid"][0].zero_()
             if s["py"] == 0:

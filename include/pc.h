@@ -115,8 +115,14 @@ int pc_local_allgather(const void *send, size_t nbytes, void *recv, void *ctx);
 /* ---------------------------------------------------------------- init (non-blocking)
  * MPI-4 partitioned semantics: `count` is elements PER PARTITION, the
  * buffer holds partitions*count elements.  Matching is by (comm, peer, tag,
- * posting order).  Nothing is exchanged here; mismatches surface as
- * PC_ERR_MATCH at the first pc_pbuf_prepare. */
+ * posting order).  The two sides must agree on dtype and on the TOTAL number
+ * of elements; their partition counts may differ (MPI-4; reading R30): a
+ * receive partition is then reported arrived (pc_parrived / device
+ * pc_parrived / pc_wait_arrived) once every send transport partition that
+ * overlaps its bytes has been pushed.  PC_COPY_LL needs equal partitionings
+ * (PC_ERR_UNSUPPORTED otherwise); empty buffers need equal partitionings.
+ * Nothing is exchanged here; mismatches surface as PC_ERR_MATCH at the first
+ * pc_pbuf_prepare. */
 int pc_psend_init(const void *buf, int partitions, size_t count, pc_dtype_t dtype, int dest, int tag,
                   pc_comm_t comm, pc_request_t *req);
 int pc_precv_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, int source, int tag,

@@ -228,6 +228,43 @@ PC_DEVICE bool contribute(const pc_prequest_t &q, int t, uint32_t add, uint32_t 
   return d <= (int32_t)add;
 }
 
+/* MPI-4 partitionings that differ between the two sides (reading R30).
+ * Send side: the receive partitions [*p0, *p1] that transport partition t's
+ * bytes overlap.  Receive side: how many send transport partitions (of g user
+ * partitions of peer_part_bytes each) overlap receive partition p. */
+PC_DEVICE void xp_recv_span(int t, int partitions, int agg, uint64_t part_bytes, uint64_t peer_part_bytes,
+                            uint64_t *p0, uint64_t *p1) {
+  const uint64_t tb = (uint64_t)agg * part_bytes, total = (uint64_t)partitions * part_bytes;
+  const uint64_t lo = (uint64_t)t * tb, hi = lo + tb < total ? lo + tb : total;
+  *p0 = lo / peer_part_bytes;
+  *p1 = (hi - 1) / peer_part_bytes;
+}
+PC_DEVICE uint32_t xp_need(uint64_t p, uint64_t part_bytes, uint32_t g, uint64_t peer_part_bytes) {
+  const uint64_t tb = (uint64_t)g * peer_part_bytes;
+  const uint64_t lo = p * part_bytes, hi = lo + part_bytes;
+  return (uint32_t)((hi - 1) / tb - lo / tb + 1);
+}
+PC_DEVICE void red_add_relaxed_sys(uint32_t *p, uint32_t v) {
+  asm volatile("red.relaxed.sys.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+/* The receiver-side arrival signal of transport partition t (after the
+ * pushes are fenced): equal partitionings store flag[t] = e; different ones
+ * add 1 to the counter of every receive partition t overlaps (the receiver
+ * waits for e * xp_need). */
+PC_DEVICE void signal_transport(uint32_t *peer_flags, int t, uint32_t e, uint32_t xpart, int partitions, int agg,
+                                uint64_t part_bytes, uint64_t peer_part_bytes) {
+  if (!xpart) {
+    st_relaxed_sys(peer_flags + t, e);
+    return;
+  }
+  uint64_t p0, p1;
+  xp_recv_span(t, partitions, agg, part_bytes, peer_part_bytes, &p0, &p1);
+  for (uint64_t p = p0; p <= p1; ++p) red_add_relaxed_sys(peer_flags + p, 1);
+}
+PC_DEVICE void signal_transport(const pc_prequest_t &q, int t, uint32_t e) {
+  signal_transport(q.peer_flags, t, e, q.xpart, q.partitions, q.agg, q.part_bytes, q.peer_part_bytes);
+}
+
 /* Publish transport partition t once this contributor's own bytes are in
  * place ("Kernel Copy": every contributor assigns its data to the
  * peer address, counters aggregate, then the partition is marked).  The
@@ -237,13 +274,13 @@ PC_DEVICE bool contribute(const pc_prequest_t &q, int t, uint32_t add, uint32_t 
  * the completing contributor, which fences again and flags. */
 PC_DEVICE void publish(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, int part) {
   if (q.agg == 1) {
-    st_relaxed_sys(q.peer_flags + t, e);
+    signal_transport(q, t, e);
     st_relaxed_gpu(q.sent + t, e);
     return;
   }
   if (contribute(q, t, add, e, part)) {
     fence_scope(q.sys_scope);
-    st_relaxed_sys(q.peer_flags + t, e);
+    signal_transport(q, t, e);
     st_relaxed_gpu(q.sent + t, e);
   }
 }
@@ -596,6 +633,9 @@ PC_DEVICE int pc_parrived(pc_prequest_t preq, int partition) {
   const uint32_t g = *(const volatile uint32_t *)preq.layout;
   if (g == 0) return 0;  // sender has not published its transport layout yet
   if (g & PC_LAYOUT_LL) return ll_consume(preq, partition, e) ? 1 : 0;
+  if (g & PC_LAYOUT_XP)
+    return reached(ld_acquire_scope(preq.flags + partition, preq.sys_scope),
+                   e * xp_need((uint64_t)partition, preq.part_bytes, g & PC_LAYOUT_G, preq.peer_part_bytes));
   return reached(ld_acquire_scope(preq.flags + partition / (int)g, preq.sys_scope), e);
 }
 
@@ -657,7 +697,12 @@ PC_DEVICE int pc_wait_arrived(pc_prequest_t preq, int partition) {
       }
       return 0;
     }
-    w = preq.flags + partition / (int)g;
+    if (g & PC_LAYOUT_XP) {
+      w = preq.flags + partition;
+      target = e * xp_need((uint64_t)partition, preq.part_bytes, g & PC_LAYOUT_G, preq.peer_part_bytes);
+    } else {
+      w = preq.flags + partition / (int)g;
+    }
     sys = preq.sys_scope != 0;
   }
   // no bytes to read after the flag -> a relaxed poll is enough

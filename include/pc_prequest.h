@@ -60,9 +60,20 @@ struct pc_prequest_s {
   uint32_t coll;              /* 0 allreduce, 1 reduce-scatter, 2 allgather, 3 broadcast    */
   int32_t nranks;             /* P (allgather: receive partitions = P * partitions)        */
   const uint32_t *srcflags;   /* allgather: [source rank][u][slice] arrival epochs         */
+  /* MPI-4 partitioned p2p with DIFFERENT partition counts on the two sides
+   * (same dtype and total bytes, reading R30): the receiver's
+   * flags are then per RECEIVE partition, counters that every completed send
+   * transport partition overlapping it bumps once per epoch. */
+  uint32_t xpart;             /* 1: send and receive partitionings differ                  */
+  uint32_t xpad;
+  uint64_t peer_part_bytes;   /* send: receiver's bytes per partition; receive: sender's   */
 };
 
-/* Receive side: bit 31 of the layout word = the sender pushes LL lines. */
+/* Receive side: bit 31 of the layout word = the sender pushes LL lines; bit
+ * 30 = the partitionings differ (per-receive-partition counters); bits 0-29 =
+ * g, the sender's user partitions per transport partition. */
 #define PC_LAYOUT_LL 0x80000000u
+#define PC_LAYOUT_XP 0x40000000u
+#define PC_LAYOUT_G 0x3fffffffu
 
 #endif /* PC_PREQUEST_H_ */

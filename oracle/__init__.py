@@ -19,6 +19,8 @@ Functions (numpy in, numpy out):
   reduce_scatter_def(...) O8  partitioned reduce-scatter, plain definition (rank-order fold, R25)
   allgather_def(...)      O9  partitioned allgather, plain definition (concatenation)
   bcast_def(...)          O10 partitioned broadcast, plain definition (copy of the root's buffer)
+  xpart_arrived(...)      O11 MPI-4 different send/recv partitionings: which receive
+                              partitions are complete, by byte coverage (R30)
 """
 from __future__ import annotations
 
@@ -292,3 +294,27 @@ def bcast_def(x: np.ndarray, root: int) -> np.ndarray:
     the root's buffer."""
     x = np.ascontiguousarray(x)
     return np.tile(x[root][None], (x.shape[0], 1))
+
+
+def xpart_arrived(send_partitions: int, send_part_bytes: int, agg: int, recv_partitions: int,
+                  recv_part_bytes: int, readied: np.ndarray) -> np.ndarray:
+    """O11 (reading R30; MPI-4 partitioned semantics cited at P:L46: a receive
+    partition has arrived once every one of its bytes has).  The sender's user
+    partitions are grouped g = agg at a time into transport partitions, and a
+    transport partition's bytes move (and are announced) only once all of its
+    user partitions are readied.  readied: bool
+    [send_partitions], the user partitions Preadied so far.  Returns bool
+    [recv_partitions]: receive partition p is complete iff every byte of
+    [p * recv_part_bytes, (p + 1) * recv_part_bytes) lies in a complete
+    transport partition.  Brute force over bytes — small cases only."""
+    total = send_partitions * send_part_bytes
+    assert total == recv_partitions * recv_part_bytes
+    readied = np.asarray(readied, dtype=bool)
+    moved = np.zeros(total, dtype=bool)
+    for t0 in range(0, send_partitions, agg):
+        members = range(t0, min(t0 + agg, send_partitions))
+        if all(readied[u] for u in members):
+            for u in members:
+                moved[u * send_part_bytes:(u + 1) * send_part_bytes] = True
+    return np.array([bool(moved[p * recv_part_bytes:(p + 1) * recv_part_bytes].all())
+                     for p in range(recv_partitions)], dtype=bool)

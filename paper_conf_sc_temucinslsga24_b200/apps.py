@@ -71,7 +71,19 @@ def bare_pingpong_pair(flagA, flagB, iters: int, base: int, out_ns, stream=None)
 T, B, L, R = 0, 1, 2, 3
 _SEND_TAG = {T: 1, B: 2, L: 3, R: 4}   # tag = side of the SENDER the data leaves from
 _RECV_TAG = {T: 2, B: 1, L: 4, R: 3}   # halo on my side d comes from the neighbour's opposite side
-STRIP = 128
+STRIP = 128  # mode 0 (warp tiles): columns per tile
+JACOBI_MODES = {"warp": 0, "rows": 1}
+
+
+def jacobi_strip(lx: int, mode: int) -> int:
+    """Columns per tile: 128 for warp tiles; for the CTA row pipeline the
+    widest of 1024/512/256/128 that divides lx (4 KiB rows per CTA at 16384^2)."""
+    if mode == 0:
+        return STRIP
+    for w in (1024, 512, 256, 128):
+        if lx % w == 0:
+            return w
+    raise ValueError("lx must be a multiple of 128")
 
 
 class JacobiSolver:
@@ -81,14 +93,20 @@ class JacobiSolver:
     `ranks` are their comm ranks.  One epoch = one solve of `iters` iterations:
     every halo partition is (iteration slot, edge segment), readied once."""
 
-    def __init__(self, comms, ranks, N: int, Py: int, Px: int, iters: int, H: int = 64, device: int = 0):
+    def __init__(self, comms, ranks, N: int, Py: int, Px: int, iters: int, H: int = 64, device: int = 0,
+                 kernel: str | None = None):
+        import os
+
         import torch
         from . import runtime as rt
         self.torch, self.rt = torch, rt
         self.N, self.Py, self.Px, self.K, self.H = N, Py, Px, iters, H
         assert N % Py == 0 and N % Px == 0
         self.ly, self.lx = N // Py, N // Px
+        self.kernel = kernel or os.environ.get("PC_JACOBI_KERNEL", "rows")
+        self.mode = JACOBI_MODES[self.kernel]
         assert self.lx % STRIP == 0 and self.ly % H == 0, "lx must be a multiple of 128, ly of H"
+        self.W = jacobi_strip(self.lx, self.mode)
         self.comms, self.ranks = comms, ranks
         dev = torch.device("cuda", device)
         self.dev = dev
@@ -103,7 +121,7 @@ class JacobiSolver:
             for d, q in nb.items():
                 if q < 0:
                     continue
-                seg = STRIP if d in (T, B) else H
+                seg = self.W if d in (T, B) else H
                 nseg = (self.lx if d in (T, B) else self.ly) // seg
                 parts = (iters + 1) * nseg
                 st["send"][d] = torch.zeros(parts * seg, device=dev)
@@ -150,15 +168,15 @@ class JacobiSolver:
             sqp = (C.c_void_p * 4)(*[st["sq"][d].ptr if d in st["sq"] else 0 for d in range(4)])
             rqp = (C.c_void_p * 4)(*[st["rq"][d].ptr if d in st["rq"] else 0 for d in range(4)])
             buf = C.create_string_buffer(sz)
-            rc = lib.pcapp_jacobi_describe(buf, st["grid"][0].data_ptr(), st["grid"][1].data_ptr(), self.ly,
-                                           self.lx, self.H, st["py"] * self.ly, st["px"] * self.lx, self.N,
-                                           has, sendp, halop, sqp, rqp)
+            rc = lib.pcapp_jacobi_describe2(buf, st["grid"][0].data_ptr(), st["grid"][1].data_ptr(), self.ly,
+                                            self.lx, self.H, st["py"] * self.ly, st["px"] * self.lx, self.N,
+                                            has, sendp, halop, sqp, rqp, self.mode, self.W)
             if rc != 0:
                 raise RuntimeError("pcapp_jacobi_describe failed")
             raw[i * sz:(i + 1) * sz] = buf.raw
             starts.append(blocks)
-            tiles = (self.ly // self.H) * (self.lx // STRIP)
-            blocks += (tiles + 7) // 8
+            tiles = (self.ly // self.H) * (self.lx // self.W)
+            blocks += (tiles + 7) // 8 if self.mode == 0 else tiles
         self.desc = torch.frombuffer(raw, dtype=torch.uint8).to(self.dev)
         self.starts = torch.tensor(starts, dtype=torch.int32, device=self.dev)
         self.blocks = blocks
@@ -192,11 +210,11 @@ class JacobiSolver:
                     q.pbuf_prepare(stream)
         s = stream.cuda_stream if hasattr(stream, "cuda_stream") else (stream or 0)
         n = len(self.local)
-        _ok(lib.pcapp_jacobi_launch(self.desc.data_ptr(), self.starts.data_ptr(), n, self.blocks, 0, 1, s),
-            "jacobi init")
+        launch = lambda k, init: lib.pcapp_jacobi_launch2(self.desc.data_ptr(), self.starts.data_ptr(), n,
+                                                          self.blocks, k, init, self.mode, self.W, self.H, s)
+        _ok(launch(0, 1), "jacobi init")
         for k in range(self.K):
-            _ok(lib.pcapp_jacobi_launch(self.desc.data_ptr(), self.starts.data_ptr(), n, self.blocks, k, 0, s),
-                "jacobi iter")
+            _ok(launch(k, 0), "jacobi iter")
         for st in self.local:
             for q in st["sreq"].values():
                 q.wait_on_stream(stream)

@@ -323,15 +323,17 @@ static void fill_prequest(Request *q, pc_prequest_t *o) {
   o->done_mul = (uint32_t)q->slices;
   o->sys_scope = (uint32_t)q->sys_scope;
   o->err = (int32_t *)(q->ctrl + q->L.err);
-  o->ll_lines = q->ll_lines;
+  o->ll_lines = q->xpart ? 0 : q->ll_lines;
+  o->xpart = q->xpart ? 1u : 0u;
+  o->peer_part_bytes = q->peer_part_bytes;
   o->coll = (uint32_t)q->coll;
   o->nranks = q->comm->size;
   if (q->kind == PC_KIND_PALLREDUCE && q->coll == PC_COLL_ALLGATHER)
     o->srcflags = q->ctrl + q->L.flags + (size_t)q->partitions * 2 * q->slices;
   if (q->kind == PC_KIND_PSEND) {
     o->peer_rbuf = q->peer_buf;
-    o->peer_flags = q->peer_ctrl ? q->peer_ctrl + q->L.flags : nullptr;
-    o->peer_ll = (q->peer_ctrl && q->ll_lines) ? (uint8_t *)(q->peer_ctrl + q->L.ll) : nullptr;
+    o->peer_flags = q->peer_ctrl ? q->peer_ctrl + q->peer_flags_off : nullptr;
+    o->peer_ll = (q->peer_ctrl && q->ll_lines && !q->xpart) ? (uint8_t *)(q->peer_ctrl + q->peer_ll_off) : nullptr;
   } else if (q->kind == PC_KIND_PRECV) {
     o->ll = q->ll_lines ? (uint8_t *)(q->ctrl + q->L.ll) : nullptr;
     o->rbuf = (uint8_t *)q->rbuf;
@@ -398,6 +400,8 @@ static int make_rec(Request *q, ReqRec *r) {
   r->owner = c->rank;
   r->req_index = q->index;
   r->host_req = (uint64_t)(uintptr_t)q;
+  r->flags_off = (int64_t)q->L.flags;
+  r->ll_off = (int64_t)q->L.ll;
   int rc = 0;
   if (q->kind == PC_KIND_PRECV || q->kind == PC_KIND_PALLREDUCE)
     if ((rc = export_ptr(c, q->rbuf, q->total_bytes, &r->buf))) return rc;
@@ -449,7 +453,12 @@ static int exchange_round(Comm *c, Request *target) {
       const ReqRec *m = find_rec(all, M, q->peer, want, c->rank, q->tag, q->seq, cnt);
       if (!m) {
         qrc = PC_ERR_MATCH;
-      } else if (m->partitions != q->partitions || m->count != (int64_t)q->count || m->dtype != q->dtype) {
+      } else if (m->dtype != q->dtype ||
+                 (uint64_t)m->partitions * (uint64_t)m->count != (uint64_t)q->partitions * q->count ||
+                 ((m->partitions != q->partitions) && (uint64_t)q->partitions * q->count == 0)) {
+        // MPI-4: the partition counts may differ (reading R30), the type
+        // signature (dtype x total elements) may not; empty buffers need equal
+        // partitionings (a flag-only partition has no bytes to overlap)
         fprintf(stderr, "[pc] rank %d: %s to/from %d tag %d: partitions/count/dtype disagree (%d/%lld/%d vs %d/%lld/%d)\n",
                 c->rank, q->kind == PC_KIND_PSEND ? "psend" : "precv", q->peer, q->tag, q->partitions,
                 (long long)q->count, q->dtype, m->partitions, (long long)m->count, m->dtype);
@@ -458,6 +467,10 @@ static int exchange_round(Comm *c, Request *target) {
         q->matched = false;
       } else {
         void *pctrl = nullptr, *pbuf = nullptr;
+        q->xpart = m->partitions != q->partitions;
+        q->peer_part_bytes = (uint64_t)m->count * q->esize;
+        q->peer_flags_off = (size_t)m->flags_off;
+        q->peer_ll_off = (size_t)m->ll_off;
         if ((qrc = import_ptr(c, m->owner, m->ctrl, &pctrl)) == 0) {
           q->peer_ctrl = (uint32_t *)pctrl;
           if (q->kind == PC_KIND_PSEND) {
@@ -746,7 +759,7 @@ static int launch_single(Request *q) {
     a.partitions = q->partitions;
     a.sbuf = (const uint8_t *)q->sbuf;
     a.peer_rbuf = q->peer_buf;
-    a.peer_flags = q->peer_ctrl + q->L.flags;
+    a.peer_flags = q->peer_ctrl + q->peer_flags_off;
     a.ready = q->ctrl + q->L.ready;
     a.rtr = q->ctrl + q->L.rtr;
     a.donecnt = q->ctrl + q->L.donecnt;
@@ -754,6 +767,8 @@ static int launch_single(Request *q) {
     a.err = (int32_t *)(q->ctrl + q->L.err);
     a.timeout_ms = q->comm->timeout_ms;
     a.sys = q->sys_scope;
+    a.xpart = q->xpart ? 1u : 0u;
+    a.peer_part_bytes = q->peer_part_bytes;
     rc = launch_p2p_engine(a, q->engine_warps, q->side);
   }
   if (rc) return rc;
@@ -1331,7 +1346,7 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
   if (!q->exchanged || !q->matched) return PC_ERR_STATE;  // after the first pbuf_prepare (Listing 2)
   if (q->kind == PC_KIND_PALLREDUCE && aggregation != 1) return PC_ERR_ARG;
   if (q->kind == PC_KIND_PALLREDUCE && copy == PC_COPY_LL) return PC_ERR_UNSUPPORTED;
-  if (q->kind == PC_KIND_PSEND && copy == PC_COPY_LL && !q->ll_lines) return PC_ERR_UNSUPPORTED;
+  if (q->kind == PC_KIND_PSEND && copy == PC_COPY_LL && (!q->ll_lines || q->xpart)) return PC_ERR_UNSUPPORTED;
   if (q->kind == PC_KIND_PSEND) {
     if (aggregation < 1 || aggregation > q->partitions) return PC_ERR_ARG;
     if (q->has_preq && (aggregation != q->agg)) return PC_ERR_STATE;  // the transport layout is fixed
@@ -1351,7 +1366,7 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
     if (!c->dry) {
       PC_CUDA(cudaSetDevice(c->device));
       // publish the transport layout (g) in the receiver's control block
-      uint32_t g = (uint32_t)aggregation | (copy == PC_COPY_LL ? PC_LAYOUT_LL : 0u);
+      uint32_t g = (uint32_t)aggregation | (copy == PC_COPY_LL ? PC_LAYOUT_LL : 0u) | (q->xpart ? PC_LAYOUT_XP : 0u);
       PC_CUDA(cudaMemcpyAsync(q->peer_ctrl + q->L.layout, &g, 4, cudaMemcpyHostToDevice, q->side));
       PC_CUDA(cudaStreamSynchronize(q->side));
     }
@@ -1456,6 +1471,13 @@ static int read_words(Request *q, size_t off, size_t n, uint32_t *h) {
 
 static bool reached_h(uint32_t v, uint32_t t) { return (int32_t)(v - t) >= 0; }
 
+// R30 (host copy of pc_detail::xp_need): send transport partitions of g
+// partitions x peer_part_bytes overlapping receive partition p
+static uint32_t xp_need_h(uint64_t p, uint64_t part_bytes, uint32_t g, uint64_t peer_part_bytes) {
+  const uint64_t tb = (uint64_t)g * peer_part_bytes, lo = p * part_bytes, hi = lo + part_bytes;
+  return (uint32_t)((hi - 1) / tb - lo / tb + 1);
+}
+
 // The epoch a host-side query compares against: the later of the host's count
 // of pc_start calls and the device epoch word (which CUDA-graph replays of a
 // captured Start advance without the host seeing it).
@@ -1497,6 +1519,11 @@ int pc_parrived(pc_request_t req, int partition, int *flag) {
       if ((rc = launch_parrived(rq, partition, (int32_t *)(q->ctrl + q->L.scratch), q->side))) return rc;
       if ((rc = read_words(q, q->L.scratch, 1, &v))) return rc;
       *flag = v != 0;
+      return 0;
+    }
+    if (g & PC_LAYOUT_XP) {  // R30: counter of this receive partition, one bump per overlapping transport
+      if ((rc = read_words(q, q->L.flags + partition, 1, &v))) return rc;
+      *flag = reached_h(v, e * xp_need_h((uint64_t)partition, q->part_bytes, g & PC_LAYOUT_G, q->peer_part_bytes));
       return 0;
     }
     if ((rc = read_words(q, q->L.flags + partition / g, 1, &v))) return rc;
@@ -1547,7 +1574,8 @@ int pc_test(pc_request_t req, int *flag) {
     if (q->kind == PC_KIND_PRECV) {
       uint32_t g = 0;
       if ((rc = read_words(q, q->L.layout, 1, &g))) return rc;
-      if (g & PC_LAYOUT_LL) {  // count lines not there yet (and unpack those that are) on the device
+      if (g & (PC_LAYOUT_LL | PC_LAYOUT_XP)) {  // LL: count lines not there yet (and unpack those that
+                                                // are) on the device; XP (R30): per-partition targets
         pc_prequest_t rq;
         fill_prequest(q, &rq);
         int32_t *pend = (int32_t *)(q->ctrl + q->L.scratch);

@@ -35,7 +35,7 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
     if ((threadIdx.x & 31) == 0) {
       const uint32_t old = atom_add_acq_rel_gpu(a.donecnt + t, 1);
       if (old + 1 == e * (uint32_t)a.ns) {
-        st_relaxed_sys(a.peer_flags + t, e);
+        signal_transport(a.peer_flags, t, e, a.xpart, a.partitions, a.agg, a.part_bytes, a.peer_part_bytes);
         st_release_gpu(a.sent + t, e);
       }
     }
@@ -138,14 +138,18 @@ __global__ void recv_wait_kernel(pc_prequest_t q, int32_t *pending) {
     return;
   }
   if (blockIdx.x != 0) return;
-  const int nt = (q.partitions + (int)g - 1) / (int)g;
+  // equal partitionings: one flag per send transport partition (target e);
+  // different ones (R30): one counter per receive partition (e * overlaps)
+  const bool xp = (g & PC_LAYOUT_XP) != 0;
+  const int nt = xp ? q.partitions : (q.partitions + (int)g - 1) / (int)g;
   for (int i = threadIdx.x; i < nt; i += blockDim.x) {
+    const uint32_t target = xp ? e * xp_need((uint64_t)i, q.part_bytes, g & PC_LAYOUT_G, q.peer_part_bytes) : e;
     if (pending) {
-      if (!reached(ld_acquire_scope(q.flags + i, q.sys_scope), e)) atomicAdd(pending, 1);
+      if (!reached(ld_acquire_scope(q.flags + i, q.sys_scope), target)) atomicAdd(pending, 1);
       continue;
     }
-    bool ok = q.sys_scope ? spin_geq<true>(q.flags + i, e, q.err, q.timeout_ms, i)
-                          : spin_geq<false>(q.flags + i, e, q.err, q.timeout_ms, i);
+    bool ok = q.sys_scope ? spin_geq<true>(q.flags + i, target, q.err, q.timeout_ms, i)
+                          : spin_geq<false>(q.flags + i, target, q.err, q.timeout_ms, i);
     if (!ok) break;
   }
 }

@@ -58,6 +58,8 @@ struct ReqRec {
   ShareRec buf;      // p2p: user buffer; allreduce: recvbuf
   ShareRec ctrl;     // control block
   ShareRec stage;    // allreduce staging
+  int64_t flags_off; // word offsets of the flags / LL areas in the owner's control block
+  int64_t ll_off;    // (they depend on the owner's partition count, R30)
 };
 
 // ------------------------------------------------------------------ local group
@@ -187,6 +189,9 @@ struct Request {
   // prequest (p2p)
   bool has_preq = false;
   int agg = 1, ntransport = 0, copy = 0;
+  bool xpart = false;            // p2p: the two sides partition the buffer differently (R30)
+  uint64_t peer_part_bytes = 0;  // p2p: the partner's bytes per partition (after matching)
+  size_t peer_flags_off = 0, peer_ll_off = 0;  // p2p: word offsets in the partner's control block
   uint32_t ll_lines = 0;  // p2p: LL lines per partition (0 = no LL area; pc.h PC_LL_MAX_*)
   // engine slicing
   int nsteps = 0;
@@ -265,6 +270,8 @@ struct P2pEngineArgs {
   int32_t *err;
   uint32_t timeout_ms;
   int sys;
+  uint32_t xpart;            // partitionings differ (R30): per-receive-partition counters
+  uint64_t peer_part_bytes;  // receiver's bytes per partition
 };
 
 constexpr int kMaxLocal = 8;  // ranks of one comm sharing one GPU in one process

@@ -17,12 +17,12 @@ from gpu_util import comms
 pytestmark = pytest.mark.gpu
 
 
-def solve(a0, Py, Px, iters, H=32, epochs=1):
+def solve(a0, Py, Px, iters, H=32, epochs=1, kernel="rows"):
     N = a0.shape[0]
     P = Py * Px
     with comms(P) as cs:
         st = torch.cuda.Stream()
-        js = apps.JacobiSolver(cs, list(range(P)), N, Py, Px, iters, H=H)
+        js = apps.JacobiSolver(cs, list(range(P)), N, Py, Px, iters, H=H, kernel=kernel)
         outs = []
         for e in range(epochs):
             js.set_initial(a0)
@@ -37,11 +37,15 @@ def solve(a0, Py, Px, iters, H=32, epochs=1):
 
 
 @pytest.mark.parametrize("Py,Px,N", [(1, 1, 256), (2, 1, 256), (1, 2, 256), (2, 2, 256), (4, 1, 512),
-                                     (4, 2, 512), (8, 1, 512), (2, 4, 1024)])
-def test_jacobi_bitexact_vs_oracle(Py, Px, N):
+                                     (4, 2, 512), (8, 1, 512), (2, 4, 1024), (2, 1, 2048), (1, 2, 4096)])
+@pytest.mark.parametrize("kernel", ["rows", "warp"])
+def test_jacobi_bitexact_vs_oracle(Py, Px, N, kernel):
+    """Both tile kernels: "rows" (CTA row pipeline, strips of up to 1024
+    columns; N = 2048 / 4096 give 1024 / 2048-column blocks, i.e. 1024-wide
+    strips with and without interior strip edges) and "warp" (warp tiles)."""
     a0 = synth.jacobi_init(N, N, "random")
-    iters = 100
-    (got,) = solve(a0, Py, Px, iters)
+    iters = 100 if N <= 1024 else 12
+    (got,) = solve(a0, Py, Px, iters, kernel=kernel)
     ref = oracle.jacobi_seq(a0, iters)
     np.testing.assert_array_equal(got, ref)
     if Py * Px > 1 and N <= 512:
@@ -69,10 +73,12 @@ def test_jacobi_fixed_points():
     np.testing.assert_array_equal(got, lin)
 
 
-@pytest.mark.parametrize("H", [4, 64, 128])
-def test_jacobi_tile_heights(H):
-    """The bench runs 64-row tiles; other legal tile heights give the same bits."""
+@pytest.mark.parametrize("H", [4, 8, 16, 64, 128])
+@pytest.mark.parametrize("kernel", ["rows", "warp"])
+def test_jacobi_tile_heights(H, kernel):
+    """The bench runs 64-row tiles; other legal tile heights give the same bits
+    (rows: H + 2 below and above the 16-row shared-memory ring)."""
     N, iters = 512, 20
     a0 = synth.jacobi_init(N, N, "random")
-    (got,) = solve(a0, 2, 2, iters, H=H)
+    (got,) = solve(a0, 2, 2, iters, H=H, kernel=kernel)
     np.testing.assert_array_equal(got, oracle.jacobi_seq(a0, iters))

@@ -393,3 +393,113 @@ def test_ll_pingpong_latency_roundtrip(payload):
         for q in (a2b, a_in, b_in, b2a):
             assert q.error()[0] == 0
             q.free()
+
+
+# ---------------------------------------------------------------- MPI-4: different partition counts (R30)
+XP_TOTAL = 840 * 16  # bytes: divisible by every partition count 1..8
+
+
+@pytest.mark.parametrize("Ns,Nr", [(8, 3), (3, 8), (6, 4), (1, 5), (5, 1)])
+@pytest.mark.parametrize("agg", [1, 2])
+@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE])
+def test_xpart_different_partition_counts(Ns, Nr, agg, copy):
+    """Sender and receiver partition the same bytes differently (MPI-4, P:L46;
+    reading R30): byte-exact delivery over 3 epochs of epoch-tagged payloads,
+    device pc_wait_arrived on every RECEIVE partition (check_recv kernel),
+    stream wait, and host pc_parrived afterwards."""
+    agg = min(agg, Ns)
+    sb, rb = XP_TOTAL // Ns, XP_TOTAL // Nr
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        src = torch.empty(XP_TOTAL, dtype=torch.uint8, device="cuda")
+        sbuf, rbuf, out = torch.empty_like(src), torch.zeros_like(src), torch.zeros_like(src)
+        status = torch.zeros(1, dtype=torch.int32, device="cuda")
+        snd = pc.psend_init(sbuf, Ns, sb, pc.BYTE, 1, 9, cs[0])
+        rcv = pc.precv_init(rbuf, Nr, rb, pc.BYTE, 0, 9, cs[1])
+        for e in range(3):
+            payload = synth.bytes_tagged(SEED, 1, e, XP_TOTAL)
+            src.copy_(torch.from_numpy(payload))
+            torch.cuda.synchronize()
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                sq = snd.prequest_create(pc.GRAN_BLOCK, agg, copy)
+                rq = rcv.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            apps.produce(sbuf, src, Ns, sb, apps.GRAN_BLOCK, sq, stream=s0)
+            snd.wait_on_stream(s0)
+            apps.check_recv(rq, rbuf, out, Nr, rb, status, blocks=8, stream=s1)
+            rcv.wait_on_stream(s1)
+            torch.cuda.synchronize()
+            assert snd.error()[0] == 0 and rcv.error()[0] == 0, (snd.error(), rcv.error())
+            assert int(status.item()) == 0
+            np.testing.assert_array_equal(rbuf.cpu().numpy(), payload)
+            np.testing.assert_array_equal(out.cpu().numpy(), payload)
+            assert all(rcv.parrived(p) for p in range(Nr))
+        snd.free()
+        rcv.free()
+
+
+@pytest.mark.parametrize("Ns,Nr,agg", [(2, 3, 1), (6, 4, 2), (4, 6, 1), (5, 3, 2), (3, 5, 3)])
+def test_xpart_partial_arrival_matches_oracle(Ns, Nr, agg):
+    """Pready the send partitions one at a time (host binding, INLINE copy) in a
+    seeded order; after each, the set of receive partitions the library reports
+    arrived (host pc_parrived, pc_test) equals O11's byte-coverage definition,
+    and every arrived partition already holds its bytes."""
+    total = 960
+    sb, rb = total // Ns, total // Nr
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        payload = synth.bytes_tagged(SEED, 2, Ns * 10 + Nr, total)
+        sbuf = torch.from_numpy(payload).cuda()
+        rbuf = torch.zeros_like(sbuf)
+        snd = pc.psend_init(sbuf, Ns, sb, pc.BYTE, 1, 4, cs[0])
+        rcv = pc.precv_init(rbuf, Nr, rb, pc.BYTE, 0, 4, cs[1])
+        torch.cuda.synchronize()
+        snd.start(s0)
+        rcv.start(s1)
+        first_prepare([[snd], [rcv]], [s0, s1])
+        sq = snd.prequest_create(pc.GRAN_THREAD, agg, pc.COPY_INLINE)  # noqa: F841 (publishes the layout)
+        readied = np.zeros(Ns, dtype=bool)
+        for u in synth.permutation(SEED, 3, Ns * 10 + Nr, Ns):
+            snd.pready(int(u), s0)
+            s0.synchronize()
+            readied[u] = True
+            want = oracle.xpart_arrived(Ns, sb, agg, Nr, rb, readied)
+            got = np.array([rcv.parrived(p) for p in range(Nr)])
+            np.testing.assert_array_equal(got, want, err_msg=f"after readying {np.nonzero(readied)[0]}")
+            host = rbuf.cpu().numpy()
+            for p in np.nonzero(want)[0]:
+                np.testing.assert_array_equal(host[p * rb:(p + 1) * rb], payload[p * rb:(p + 1) * rb])
+            assert rcv.test() == bool(want.all())
+        snd.wait()
+        assert snd.error()[0] == 0 and rcv.error()[0] == 0
+        snd.free()
+        rcv.free()
+
+
+def test_xpart_ll_unsupported_and_size_mismatch():
+    """LL lines are laid out per receive partition, so a different partitioning
+    cannot use them (PC_ERR_UNSUPPORTED); different TOTAL sizes do not match."""
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        sbuf = torch.zeros(960, dtype=torch.uint8, device="cuda")
+        rbuf = torch.zeros_like(sbuf)
+        snd = pc.psend_init(sbuf, 2, 480, pc.BYTE, 1, 5, cs[0])
+        rcv = pc.precv_init(rbuf, 3, 320, pc.BYTE, 0, 5, cs[1])
+        snd.start(s0)
+        rcv.start(s1)
+        first_prepare([[snd], [rcv]], [s0, s1])
+        with pytest.raises(pc.PcError) as ei:
+            snd.prequest_create(pc.GRAN_THREAD, 1, pc.COPY_LL)
+        assert ei.value.code == pc.ERR_UNSUPPORTED
+        snd.prequest_create(pc.GRAN_THREAD, 1, pc.COPY_INLINE)
+        snd.pready(0, s0)
+        snd.pready(1, s0)
+        snd.wait()
+        rcv.wait()
+        snd.free()
+        rcv.free()

@@ -99,14 +99,23 @@ def test_dry_p2p_matching_by_tag_and_order():
     g.destroy()
 
 
-def test_dry_p2p_mismatch_is_reported():
+@pytest.mark.parametrize("recv,want", [
+    ((8, 4, "FLOAT32"), 0),                 # same bytes, different partitions: MPI-4 allows it (R30)
+    ((3, 8, "FLOAT32"), pc.ERR_MATCH),      # different total size
+    ((4, 8, "INT32"), pc.ERR_MATCH),        # different type signature
+    ((8, 0, "FLOAT32"), pc.ERR_MATCH),      # empty vs non-empty
+])
+def test_dry_p2p_matching_rules(recv, want):
     g, cs = _dry(2)
     a = pc.psend_init(0x1000, 4, 8, pc.FLOAT32, 1, 1, cs[0])
-    b = pc.precv_init(0x2000, 8, 4, pc.FLOAT32, 0, 1, cs[1])  # same bytes, different partitions
+    b = pc.precv_init(0x2000, recv[0], recv[1], getattr(pc, recv[2]), 0, 1, cs[1])
     a.start()
     b.start()
     res = pc.run_ranks([lambda: _try(a.pbuf_prepare), lambda: _try(b.pbuf_prepare)])
-    assert res == [pc.ERR_MATCH, pc.ERR_MATCH]
+    assert res == [want, want]
+    if want == 0:
+        a.wait()
+        b.wait()
     for c in cs:
         c.destroy()
     g.destroy()
