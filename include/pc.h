@@ -57,7 +57,12 @@ typedef enum { PC_GRAN_THREAD = 0, PC_GRAN_WARP = 1, PC_GRAN_BLOCK = 2 } pc_gran
  * buffer <= PC_LL_MAX_TOTAL_BYTES (else pc_prequest_create returns
  * PC_ERR_UNSUPPORTED); aggregation then only batches the sender's completion
  * accounting (each partition's lines are self-validating). */
-typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1, PC_COPY_LL = 2 } pc_copy_t;
+/* PC_COPY_HOST: the paper's host Progression Engine (
+ * SURVEY NEXT-4), kept as a comparison mode: Pready marks the transport
+ * partition in pinned host memory, a library host thread polls those flags
+ * and issues the copy (cudaMemcpyAsync) and the arrival signal (stream
+ * memop) on its own stream. */
+typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1, PC_COPY_LL = 2, PC_COPY_HOST = 3 } pc_copy_t;
 #define PC_LL_MAX_PART_BYTES 1024
 #define PC_LL_MAX_TOTAL_BYTES (16u << 20)
 /* Allreduce schedule (§IV-B).  RING = Alg 1; RD = recursive

@@ -28,6 +28,9 @@
  *     paper sent through the host, done here on the device).
  *   - ENGINE copy: the completing contributor only release-stores ready[t] = e;
  *     library engine warps move the data.
+ *   - HOST copy (the paper's Progression Engine): the completing
+ *     contributor release-stores hready[t] = e into pinned host memory; the
+ *     library's host progression thread copies and signals.
  *   - Allreduce requests: marks user partition u ready (step S_0 is the
  *     user's Pready); the library engine runs the schedule.
  * Returns 0, or a PC_ERR_* code that is also recorded in the sticky error word
@@ -226,6 +229,17 @@ PC_DEVICE bool contribute(const pc_prequest_t &q, int t, uint32_t add, uint32_t 
     return false;
   }
   return d <= (int32_t)add;
+}
+
+/* ENGINE / HOST copy: the completing contributor marks transport partition t
+ * ready for the mover — the library's engine warps (GPU-scope flag) or the
+ * host progression thread (system-scope store into pinned host memory, after
+ * which the host may read the partition's bytes). */
+PC_DEVICE void mark_ready(const pc_prequest_t &q, int t, uint32_t e) {
+  if (q.copy == 3)
+    st_release_sys(q.hready + t, e);
+  else
+    st_release_gpu(q.ready + t, e);
 }
 
 /* MPI-4 partitionings that differ between the two sides (reading R30).
@@ -479,9 +493,9 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
     }
   }
   e = __shfl_sync(mask, e, first);
-  if (preq.copy == 1) {  // ENGINE
+  if (preq.copy == 1 || preq.copy == 3) {  // ENGINE / HOST progression
     __syncwarp(mask);    // every lane's data writes are ordered before the leader's release
-    if (lane == leader && contribute(preq, t, __popc(grp), e, partition)) st_release_gpu(preq.ready + t, e);
+    if (lane == leader && contribute(preq, t, __popc(grp), e, partition)) mark_ready(preq, t, e);
     return 0;
   }
   if (preq.part_bytes) {
@@ -525,11 +539,11 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
     __syncwarp(full);
     return 0;
   }
-  if (preq.copy == 1 || preq.part_bytes == 0) {  // no bytes for this warp to move: lane 0 alone
+  if (preq.copy == 1 || preq.copy == 3 || preq.part_bytes == 0) {  // no bytes for this warp to move
     if (lane == 0) {
       const uint32_t e = epoch_relaxed(preq);
-      if (preq.copy == 1) {
-        if (contribute(preq, t, 1, e, partition)) st_release_gpu(preq.ready + t, e);
+      if (preq.copy == 1 || preq.copy == 3) {
+        if (contribute(preq, t, 1, e, partition)) mark_ready(preq, t, e);
       } else {
         publish(preq, t, 1, e, partition);
       }
@@ -580,11 +594,11 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
     if (tid == 0) ll_account(preq, t, 1, e, partition);
     return 0;
   }
-  if (preq.copy == 1 || preq.part_bytes == 0) {  // no bytes for this block to move: thread 0 alone
+  if (preq.copy == 1 || preq.copy == 3 || preq.part_bytes == 0) {  // no bytes for this block to move
     if (tid == 0) {
       const uint32_t e = epoch_relaxed(preq);
-      if (preq.copy == 1) {
-        if (contribute(preq, t, 1, e, partition)) st_release_gpu(preq.ready + t, e);
+      if (preq.copy == 1 || preq.copy == 3) {
+        if (contribute(preq, t, 1, e, partition)) mark_ready(preq, t, e);
       } else {
         publish(preq, t, 1, e, partition);
       }

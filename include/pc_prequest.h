@@ -67,6 +67,8 @@ struct pc_prequest_s {
   uint32_t xpart;             /* 1: send and receive partitionings differ                  */
   uint32_t xpad;
   uint64_t peer_part_bytes;   /* send: receiver's bytes per partition; receive: sender's   */
+  uint32_t *hready;           /* send, PC_COPY_HOST: [ntransport] ready epochs in pinned
+                                 host memory (device-mapped), polled by the progress thread */
 };
 
 /* Receive side: bit 31 of the layout word = the sender pushes LL lines; bit

@@ -15,7 +15,7 @@ import os
 import re
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIBPC = os.path.join(_HERE, "libpc.so")
+LIBPC = os.environ.get("PC_LIB") or os.path.join(_HERE, "libpc.so")
 LIBAPPS = os.environ.get("PC_APPS_LIB") or os.path.join(_HERE, "libpcapps.so")
 INCLUDE = os.path.join(os.path.dirname(_HERE), "include")
 

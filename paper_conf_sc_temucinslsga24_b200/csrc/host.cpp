@@ -59,6 +59,7 @@ typedef CUresult (*PFN_getAddrRange)(CUdeviceptr *, size_t *, CUdeviceptr);
 typedef CUresult (*PFN_writeValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 static PFN_getAddrRange g_getAddrRange = nullptr;
 static PFN_writeValue32 g_writeValue32 = nullptr;
+static PFN_writeValue32 g_waitValue32 = nullptr;  // cuStreamWaitValue32 has the same signature
 static std::once_flag g_drv_once;
 
 static void load_driver_entry_points() {
@@ -72,6 +73,10 @@ static void load_driver_entry_points() {
     if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &fn, cudaEnableDefault, &q) == cudaSuccess &&
         q == cudaDriverEntryPointSuccess)
       g_writeValue32 = (PFN_writeValue32)fn;
+    fn = nullptr;
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      g_waitValue32 = (PFN_writeValue32)fn;
     cudaGetLastError();
   });
 }
@@ -89,6 +94,120 @@ int stream_write_u32(Comm *c, cudaStream_t s, uint32_t *addr, uint32_t value) {
     c->memops = false;
   }
   return launch_set_word(addr, value, s);
+}
+
+// Stream-ordered "wait until *addr >= value" (wrap-unaware GEQ memop, or a
+// 1-block bounded spin kernel when memops are unavailable).
+int stream_wait_geq_u32(Comm *c, cudaStream_t s, const uint32_t *addr, uint32_t value, bool sys) {
+  if (c->memops && g_waitValue32) {
+    CUresult r = g_waitValue32((CUstream)s, (CUdeviceptr)addr, value, 0x0 /* CU_STREAM_WAIT_VALUE_GEQ */);
+    if (r == CUDA_SUCCESS) return 0;
+    logf("cuStreamWaitValue32 failed (%d); falling back to a wait kernel", (int)r);
+  }
+  return launch_wait_value(addr, value, s, sys, c->timeout_ms);
+}
+
+// ------------------------------------------------------------------ progression engine (PC_COPY_HOST)
+// The paper's host Progression Engine as a
+// comparison mode: device Pready stores the epoch into hready[t] (pinned host
+// memory); this thread sees it and enqueues, on its own stream, (once per
+// epoch) the wait for the receiver's ready-to-receive word, the copy of the
+// transport partition, the receiver's arrival flag and the sender's sent[t].
+static void progress_main(Comm *c) {
+  cudaSetDevice(c->device);
+  Progress &pe = c->pe;
+  int idle = 0;
+  while (!pe.stop.load(std::memory_order_acquire)) {
+    bool any = false;
+    {
+      std::lock_guard<std::mutex> lk(pe.mu);
+      for (Request *q : pe.reqs) {
+        for (int t = 0; t < q->ntransport; ++t) {
+          const uint32_t v = __atomic_load_n(q->hready + t, __ATOMIC_ACQUIRE);
+          if (v == q->pe_done[t]) continue;
+          any = true;
+          q->pe_done[t] = v;
+          int rc = 0;
+          if ((int32_t)(v - q->pe_rtr_epoch) > 0) {  // first partition of epoch v: receiver ready?
+            rc = stream_wait_geq_u32(c, pe.stream, q->ctrl + q->L.rtr, v, q->sys_scope != 0);
+            q->pe_rtr_epoch = v;
+          }
+          const int rem = q->partitions - t * q->agg;
+          const uint64_t len = (uint64_t)(rem < q->agg ? rem : q->agg) * q->part_bytes;
+          const uint64_t off = (uint64_t)t * q->agg * q->part_bytes;
+          if (!rc && len)
+            rc = cudaMemcpyAsync(q->peer_buf + off, (const uint8_t *)q->sbuf + off, len, cudaMemcpyDeviceToDevice,
+                                 pe.stream) == cudaSuccess
+                     ? 0
+                     : PC_ERR_CUDA;
+          if (!rc) rc = stream_write_u32(c, pe.stream, q->peer_ctrl + q->peer_flags_off + t, v);
+          if (!rc) rc = stream_write_u32(c, pe.stream, q->ctrl + q->L.sent + t, v);
+          if (rc) pe.err.store(rc);
+        }
+      }
+    }
+    if (any) {
+      idle = 0;
+    } else if (++idle > 1000) {
+      std::this_thread::sleep_for(std::chrono::microseconds(20));
+    } else {
+      std::this_thread::yield();
+    }
+  }
+}
+
+static int progress_register(Request *q) {
+  Comm *c = q->comm;
+  Progress &pe = c->pe;
+  if (!q->hready) {
+    PC_CUDA(cudaHostAlloc((void **)&q->hready, (size_t)q->ntransport * 4, cudaHostAllocMapped | cudaHostAllocPortable));
+    memset(q->hready, 0, (size_t)q->ntransport * 4);
+    PC_CUDA(cudaHostGetDevicePointer((void **)&q->hready_dev, q->hready, 0));
+    q->pe_done.assign((size_t)q->ntransport, 0u);
+  }
+  std::lock_guard<std::mutex> lk(pe.mu);
+  if (!pe.started) {
+    int lo = 0, hi = 0;
+    PC_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    PC_CUDA(cudaStreamCreateWithPriority(&pe.stream, cudaStreamNonBlocking, hi));
+    pe.stop.store(false);
+    pe.th = std::thread(progress_main, c);
+    pe.started = true;
+  }
+  if (!q->pe_registered) {
+    pe.reqs.push_back(q);
+    q->pe_registered = true;
+  }
+  return 0;
+}
+
+static void progress_unregister(Request *q) {
+  Progress &pe = q->comm->pe;
+  if (q->pe_registered) {
+    std::lock_guard<std::mutex> lk(pe.mu);
+    for (size_t i = 0; i < pe.reqs.size(); ++i)
+      if (pe.reqs[i] == q) {
+        pe.reqs.erase(pe.reqs.begin() + (long)i);
+        break;
+      }
+    q->pe_registered = false;
+  }
+  if (pe.stream) cudaStreamSynchronize(pe.stream);  // copies that read this request's buffers
+  if (q->hready) cudaFreeHost(q->hready);
+  q->hready = q->hready_dev = nullptr;
+}
+
+static void progress_stop(Comm *c) {
+  Progress &pe = c->pe;
+  if (!pe.started) return;
+  pe.stop.store(true, std::memory_order_release);
+  if (pe.th.joinable()) pe.th.join();
+  if (pe.stream) {
+    cudaStreamSynchronize(pe.stream);
+    cudaStreamDestroy(pe.stream);
+  }
+  pe.stream = nullptr;
+  pe.started = false;
 }
 
 // ------------------------------------------------------------------ local groups
@@ -325,6 +444,7 @@ static void fill_prequest(Request *q, pc_prequest_t *o) {
   o->err = (int32_t *)(q->ctrl + q->L.err);
   o->ll_lines = q->xpart ? 0 : q->ll_lines;
   o->xpart = q->xpart ? 1u : 0u;
+  o->hready = q->hready_dev;
   o->peer_part_bytes = q->peer_part_bytes;
   o->coll = (uint32_t)q->coll;
   o->nranks = q->comm->size;
@@ -1013,6 +1133,7 @@ int pc_comm_destroy(pc_comm_t comm) {
     if (q) return PC_ERR_STATE;  // free requests first
   if (!c->dry) {
     cudaSetDevice(c->device);
+    progress_stop(c);
     for (auto &kv : c->ipc_open) cudaIpcCloseMemHandle(kv.second);
   }
   delete c;
@@ -1341,12 +1462,15 @@ int pc_pbuf_prepare_all(int n, pc_request_t *reqs, pc_stream_t stream) {
 
 int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_copy_t copy, pc_prequest_t *out) {
   Request *q = (Request *)req;
-  if (!q || !out || gran < 0 || gran > 2 || copy < 0 || copy > 2) return PC_ERR_ARG;
+  if (!q || !out || gran < 0 || gran > 2 || copy < 0 || copy > 3) return PC_ERR_ARG;
   Comm *c = q->comm;
   if (!q->exchanged || !q->matched) return PC_ERR_STATE;  // after the first pbuf_prepare (Listing 2)
   if (q->kind == PC_KIND_PALLREDUCE && aggregation != 1) return PC_ERR_ARG;
   if (q->kind == PC_KIND_PALLREDUCE && copy == PC_COPY_LL) return PC_ERR_UNSUPPORTED;
   if (q->kind == PC_KIND_PSEND && copy == PC_COPY_LL && (!q->ll_lines || q->xpart)) return PC_ERR_UNSUPPORTED;
+  if (q->kind == PC_KIND_PALLREDUCE && copy == PC_COPY_HOST) return PC_ERR_UNSUPPORTED;
+  // the progress thread signals with stream memops (stores), not the counters R30 needs
+  if (q->kind == PC_KIND_PSEND && copy == PC_COPY_HOST && q->xpart) return PC_ERR_UNSUPPORTED;
   if (q->kind == PC_KIND_PSEND) {
     if (aggregation < 1 || aggregation > q->partitions) return PC_ERR_ARG;
     if (q->has_preq && (aggregation != q->agg)) return PC_ERR_STATE;  // the transport layout is fixed
@@ -1365,6 +1489,10 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
     q->engine_warps = c->engine_warps;
     if (!c->dry) {
       PC_CUDA(cudaSetDevice(c->device));
+      if (copy == PC_COPY_HOST) {
+        int prc = progress_register(q);
+        if (prc) return prc;
+      }
       // publish the transport layout (g) in the receiver's control block
       uint32_t g = (uint32_t)aggregation | (copy == PC_COPY_LL ? PC_LAYOUT_LL : 0u) | (q->xpart ? PC_LAYOUT_XP : 0u);
       PC_CUDA(cudaMemcpyAsync(q->peer_ctrl + q->L.layout, &g, 4, cudaMemcpyHostToDevice, q->side));
@@ -1664,6 +1792,7 @@ int pc_request_free(pc_request_t *req) {
   if (!c->dry) {
     cudaSetDevice(c->device);
     if (q->side) cudaStreamSynchronize(q->side);
+    if (q->hready || q->pe_registered) progress_unregister(q);
     if (q->ctrl) cudaFree(q->ctrl);
     if (q->staging) cudaFree(q->staging);
     if (q->side) cudaStreamDestroy(q->side);

@@ -356,6 +356,24 @@ int launch_rtr(const RtrArgs &a, cudaStream_t s) {
   return 0;
 }
 
+// Stream-ordered wait for *addr >= value (fallback for cuStreamWaitValue32):
+// one thread, bounded by tmo_ms (then it gives up; the caller's request has
+// its own timeouts downstream).
+__global__ void wait_value_kernel(const uint32_t *addr, uint32_t value, int sys, uint32_t tmo_ms) {
+  const uint64_t t0 = globaltimer();
+  while (!reached(sys ? ld_acquire_sys(addr) : ld_acquire_gpu(addr), value)) {
+    if (tmo_ms && globaltimer() - t0 > (uint64_t)tmo_ms * 1000000ull) return;
+    __nanosleep(256);
+  }
+}
+
+int launch_wait_value(const uint32_t *addr, uint32_t value, cudaStream_t s, bool sys, uint32_t tmo_ms) {
+  wait_value_kernel<<<1, 1, 0, s>>>(addr, value, sys ? 1 : 0, tmo_ms);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s) {
   set_word_kernel<<<1, 1, 0, s>>>(addr, value);
   g_launches++;

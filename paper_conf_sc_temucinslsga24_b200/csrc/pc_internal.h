@@ -9,6 +9,7 @@
 #include <map>
 #include <mutex>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "pc.h"
@@ -192,6 +193,13 @@ struct Request {
   bool xpart = false;            // p2p: the two sides partition the buffer differently (R30)
   uint64_t peer_part_bytes = 0;  // p2p: the partner's bytes per partition (after matching)
   size_t peer_flags_off = 0, peer_ll_off = 0;  // p2p: word offsets in the partner's control block
+  // PC_COPY_HOST (progression engine, NEXT-4): ready epochs in pinned host
+  // memory written by device Pready, and the progress thread's per-transport
+  // "last epoch moved" (touched only by that thread) and last RTR-checked epoch
+  uint32_t *hready = nullptr, *hready_dev = nullptr;
+  std::vector<uint32_t> pe_done;
+  uint32_t pe_rtr_epoch = 0;
+  bool pe_registered = false;
   uint32_t ll_lines = 0;  // p2p: LL lines per partition (0 = no LL area; pc.h PC_LL_MAX_*)
   // engine slicing
   int nsteps = 0;
@@ -199,6 +207,20 @@ struct Request {
   int64_t slice_elems = 0; // allreduce: elements per slice; p2p: bytes per slice
   int64_t chunk_elems = 0; // allreduce ring: q
   int engine_warps = 0;
+};
+
+// Host progression engine (PC_COPY_HOST): one thread per comm polls the
+// pinned ready flags of its HOST-mode send requests and enqueues, per ready
+// transport partition, the ready-to-receive wait, the copy and the arrival /
+// completion signals on its own stream.
+struct Progress {
+  std::thread th;
+  std::mutex mu;
+  std::vector<Request *> reqs;
+  std::atomic<bool> stop{false};
+  std::atomic<int> err{0};
+  cudaStream_t stream = nullptr;
+  bool started = false;
 };
 
 struct Comm {
@@ -217,6 +239,7 @@ struct Comm {
   std::map<std::string, void *> ipc_open;
   uint32_t timeout_ms = 10000;
   bool memops = false;  // cuStreamWriteValue32 usable
+  Progress pe;
 };
 
 // ------------------------------------------------------------------ helpers
@@ -224,6 +247,7 @@ int allgather(Comm *c, const void *send, size_t nbytes, void *recv);
 int export_ptr(Comm *c, const void *p, uint64_t bytes, ShareRec *out);
 int import_ptr(Comm *c, int owner, const ShareRec &s, void **out);
 int stream_write_u32(Comm *c, cudaStream_t s, uint32_t *addr, uint32_t value);
+int stream_wait_geq_u32(Comm *c, cudaStream_t s, const uint32_t *addr, uint32_t value, bool sys);
 bool memops_available();
 
 // ------------------------------------------------------------------ kernel launchers (kernels.cu)
@@ -372,6 +396,7 @@ int launch_recv_wait(const pc_prequest_t &q, int32_t *pending, cudaStream_t s);
 // out[0] = pc_parrived(q, partition) on the device (LL receive requests)
 int launch_parrived(const pc_prequest_t &q, int partition, int32_t *out, cudaStream_t s);
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s);
+int launch_wait_value(const uint32_t *addr, uint32_t value, cudaStream_t s, bool sys, uint32_t tmo_ms);
 int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s);
 constexpr int kMaxPreadyAll = 16;
 struct PreadyAllArgs {

@@ -19,7 +19,7 @@ INT32, FLOAT32, BYTE, FLOAT64, BF16 = 0, 1, 2, 3, 4
 ESIZE = {INT32: 4, FLOAT32: 4, BYTE: 1, FLOAT64: 8, BF16: 2}
 SUM, MAX, MIN = 0, 1, 2
 GRAN_THREAD, GRAN_WARP, GRAN_BLOCK = 0, 1, 2
-COPY_INLINE, COPY_ENGINE, COPY_LL = 0, 1, 2
+COPY_INLINE, COPY_ENGINE, COPY_LL, COPY_HOST = 0, 1, 2, 3
 ALGO_AUTO, ALGO_RING, ALGO_RD, ALGO_DIRECT = 0, 1, 2, 3
 KIND_PSEND, KIND_PRECV, KIND_PALLREDUCE = 1, 2, 3
 

@@ -91,7 +91,7 @@ def test_c1_block_agg16_inline():
 
 @pytest.mark.parametrize("gran", [apps.GRAN_THREAD, apps.GRAN_WARP, apps.GRAN_BLOCK])
 @pytest.mark.parametrize("agg_kind", ["none", "odd", "all"])
-@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE])
+@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE, pc.COPY_HOST])
 def test_granularity_aggregation_copy(gran, agg_kind, copy):
     n = 3 * 2048 * 5 + 0  # 15 blocks of 1024 threads
     partitions = n // GRAN_ELEMS[gran]
@@ -497,6 +497,75 @@ def test_xpart_ll_unsupported_and_size_mismatch():
             snd.prequest_create(pc.GRAN_THREAD, 1, pc.COPY_LL)
         assert ei.value.code == pc.ERR_UNSUPPORTED
         snd.prequest_create(pc.GRAN_THREAD, 1, pc.COPY_INLINE)
+        snd.pready(0, s0)
+        snd.pready(1, s0)
+        snd.wait()
+        rcv.wait()
+        snd.free()
+        rcv.free()
+
+
+# ---------------------------------------------------------------- host progression engine (NEXT-4)
+@pytest.mark.parametrize("agg", [1, 4])
+def test_host_progression_engine_tagged_epochs(agg):
+    """PC_COPY_HOST (the paper's Progression Engine): device
+    Pready marks pinned host flags, the library's host thread copies and
+    signals.  50 back-to-back epochs of epoch-tagged bytes with a permuted
+    Pready order, device Parrived on every partition, host wait/test."""
+    partitions, pbytes, E = 16, 4096, 50
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        src = torch.empty(partitions * pbytes, dtype=torch.uint8, device="cuda")
+        sbuf, rbuf, out = torch.empty_like(src), torch.empty_like(src), torch.zeros_like(src)
+        status = torch.zeros(1, dtype=torch.int32, device="cuda")
+        snd = pc.psend_init(sbuf, partitions, pbytes, pc.BYTE, 1, 1, cs[0])
+        rcv = pc.precv_init(rbuf, partitions, pbytes, pc.BYTE, 0, 1, cs[1])
+        for e in range(E):
+            payload = synth.bytes_tagged(SEED, 5, e, partitions * pbytes)
+            src.copy_(torch.from_numpy(payload))
+            torch.cuda.synchronize()
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                sq = snd.prequest_create(pc.GRAN_BLOCK, agg, pc.COPY_HOST)
+                rq = rcv.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            apps.produce(sbuf, src, partitions, pbytes, apps.GRAN_BLOCK, sq, order_stride=5, stream=s0)
+            apps.check_recv(rq, rbuf, out, partitions, pbytes, status, blocks=16, stream=s1)
+            if e % 2:
+                snd.wait()
+                rcv.wait()
+            else:
+                snd.wait_on_stream(s0)
+                rcv.wait_on_stream(s1)
+                torch.cuda.synchronize()
+            assert int(status.item()) == 0
+            np.testing.assert_array_equal(rbuf.cpu().numpy(), payload)
+            np.testing.assert_array_equal(out.cpu().numpy(), payload)
+        assert snd.error()[0] == 0 and rcv.error()[0] == 0
+        snd.free()
+        rcv.free()
+
+
+def test_host_progression_engine_unsupported_cases():
+    """PE mode moves p2p bytes only: no allreduce requests, no different
+    partitionings (its signals are stores, R30 needs counters)."""
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        sbuf = torch.zeros(960, dtype=torch.uint8, device="cuda")
+        rbuf = torch.zeros_like(sbuf)
+        snd = pc.psend_init(sbuf, 2, 480, pc.BYTE, 1, 6, cs[0])
+        rcv = pc.precv_init(rbuf, 3, 320, pc.BYTE, 0, 6, cs[1])
+        snd.start(s0)
+        rcv.start(s1)
+        first_prepare([[snd], [rcv]], [s0, s1])
+        with pytest.raises(pc.PcError) as ei:
+            snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_HOST)
+        assert ei.value.code == pc.ERR_UNSUPPORTED
+        snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
         snd.pready(0, s0)
         snd.pready(1, s0)
         snd.wait()
