@@ -100,6 +100,19 @@ class Clocks:
         self.lines = []
 
     def __enter__(self):
+        # NVML (nvidia_ml_py) samples every 2 ms, so even a ~100 ms timed
+        # region gets dozens of samples; nvidia-smi -lms 100 is the fallback.
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nvml = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.stop = threading.Event()
+            self.t = threading.Thread(target=self._nvml_loop, daemon=True)
+            self.t.start()
+            return self
+        except Exception:
+            self.nvml = None
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
                                        "--format=csv,noheader,nounits", "-lms", "100"],
@@ -114,7 +127,26 @@ class Clocks:
         for line in self.p.stdout:
             self.lines.append(line.strip())
 
+    def _nvml_loop(self):
+        nv = self.nvml
+        bits = [("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+                ("sw_power_cap", 0x4)]
+        mx = nv.nvmlDeviceGetMaxClockInfo(self.h, nv.NVML_CLOCK_SM)
+        while not self.stop.is_set():
+            try:
+                sm = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                f = [str(sm), str(mx), "0", hex(r)] + ["Active" if r & b else "Not Active" for _, b in bits]
+                self.lines.append(", ".join(f))
+            except Exception:
+                pass
+            time.sleep(0.002)
+
     def __exit__(self, *a):
+        if getattr(self, "nvml", None):
+            self.stop.set()
+            self.t.join(timeout=2)
+            return
         if self.p:
             self.p.terminate()
             try:

@@ -43,8 +43,14 @@ using namespace pc_detail;
 #endif
 constexpr int kU = PC_ENGINE_UNROLL;
 #ifndef PC_DIRECT_FV
-#define PC_DIRECT_FV 1
+#define PC_DIRECT_FV 2
 #endif  // 16-B vectors in flight per operand per lane
+#ifndef PC_DIRECT_MINB
+#define PC_DIRECT_MINB 1
+#endif  // min CTAs per SM of the DIRECT engines: 1 = up to 255 registers, so all
+        // P * PC_DIRECT_FV loads of a lane stay in registers (at 2 CTAs the
+        // 128-register cap spills FV = 2; measured: FV 1 @ 2 CTAs 0.92 of HBM,
+        // FV 2 @ 1 CTA 0.99, FV 4 @ 1 CTA 0.90)
 
 // Engine-side bounded spin: the awaited event is a whole slice step of the
 // upstream rank (tens of microseconds), so back off with __nanosleep early and
@@ -535,8 +541,141 @@ __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d
   for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
 }
 
+// ---------------------------------------------------------------------------
+// Bulk-copy PULL fold (DIRECT allreduce, same-GPU peers): the P source chunks
+// of 512 B (one 16-B vector per lane) reach this warp's shared-memory stage by
+// cp.async.bulk (the TMA engine), completing on the stage's mbarrier, so the
+// loads in flight are no longer bounded by registers (the register version
+// holds P vectors per lane and spills at 2).  Two stages per warp: while the
+// warp folds stage s (rank order, R25) and stores the result to every rank's
+// recvbuf, stage s^1's P copies are in flight.
+// ---------------------------------------------------------------------------
+#ifndef PC_DIRECT_BULK
+#define PC_DIRECT_BULK 0  // measured 0.80-0.87 of HBM vs 0.99 for the register fold
+#endif
+#ifndef PC_BULK_STAGES
+#define PC_BULK_STAGES 2
+#endif
+#ifndef PC_BULK_CHUNK
+#define PC_BULK_CHUNK 512
+#endif
+constexpr int kBulkStages = PC_BULK_STAGES;
+constexpr int kBulkChunk = PC_BULK_CHUNK;  // bytes per source per stage (a multiple of 512)
+constexpr int kBulkWarpBytes = (kBulkStages * kMaxDirect * kBulkChunk + 8 * kBulkStages + 127) / 128 * 128;
+constexpr size_t kDirectSmem = PC_DIRECT_BULK ? (size_t)(kEngineBlock / 32) * kBulkWarpBytes : 0;
+
+struct WarpBulk {
+  uint8_t *stage;     // [kBulkStages][kMaxDirect][kBulkChunk]
+  uint64_t *bar;      // [kBulkStages]
+  uint32_t phase;     // bit s: parity of stage s's next completion
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void warp_bulk_init(WarpBulk &wb, uint8_t *smem) {
+  const int wib = threadIdx.x >> 5;
+  wb.stage = smem + (size_t)wib * kBulkWarpBytes;
+  wb.bar = reinterpret_cast<uint64_t *>(wb.stage + kBulkStages * kMaxDirect * kBulkChunk);
+  wb.phase = 0;
+  if ((threadIdx.x & 31) == 0) {
+    for (int s = 0; s < kBulkStages; ++s)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(wb.bar + s)) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+}
+
+// lane 0: P bulk copies of `bytes` each into stage st, one mbarrier transaction
+template <typename SrcFn>
+__device__ __forceinline__ void bulk_issue(WarpBulk &wb, int st, int P, SrcFn src, uint32_t bytes) {
+  const uint32_t bar = smem_u32(wb.bar + st);
+  asm volatile("{\n .reg .b64 s;\n mbarrier.arrive.expect_tx.shared::cta.b64 s, [%0], %1;\n}" ::"r"(bar),
+               "r"(bytes * (uint32_t)P)
+               : "memory");
+  for (int j = 0; j < P; ++j)
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(wb.stage + ((size_t)st * kMaxDirect + j) * kBulkChunk)),
+                 "l"(src(j)), "r"(bytes), "r"(bar)
+                 : "memory");
+}
+
+__device__ __forceinline__ void bulk_wait(WarpBulk &wb, int st) {
+  const uint32_t bar = smem_u32(wb.bar + st), par = (wb.phase >> st) & 1u;
+  asm volatile("{\n .reg .pred p;\n W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W_%=;\n}" ::"r"(
+                   bar),
+               "r"(par)
+               : "memory");
+  wb.phase ^= 1u << st;
+}
+
+// As warp_fold_pull<.., TO_PEERS=true>, with the 16-B body moved by bulk copies.
+template <int DT, int OP, typename A>
+__device__ __forceinline__ void warp_fold_pull_bulk(const A &a, int64_t s0, int64_t d0, int64_t n, WarpBulk &wb) {
+  using O = Op<DT, OP>;
+  using T = typename O::T;
+  const int P = a.P, r = a.r;
+  const uint32_t lane = threadIdx.x & 31;
+  constexpr int64_t EPV = 16 / sizeof(T);
+  auto src = [&](int k) -> const T * {
+    return reinterpret_cast<const T *>(k == r ? a.sendbuf : a.p_sendbuf[(k - r - 1 + P) % P]) + s0;
+  };
+  T *out_local = reinterpret_cast<T *>(a.recvbuf) + d0;
+  const uintptr_t m = reinterpret_cast<uintptr_t>(out_local) & 15;
+  if ((reinterpret_cast<uintptr_t>(src(r)) & 15) != m) {  // no common misalignment: register path
+    warp_fold_pull<DT, OP, true>(a, s0, d0, n);
+    return;
+  }
+  int64_t head = (int64_t)(((16 - m) & 15) / sizeof(T));
+  if (head > n) head = n;
+  auto scalar = [&](int64_t k) {
+    T acc = __ldcg(src(0) + k);
+    for (int j = 1; j < P; ++j) acc = O::f(acc, __ldcg(src(j) + k));
+    out_local[k] = acc;
+    for (int j = 0; j < P - 1; ++j) (reinterpret_cast<T *>(a.p_recvbuf[j]) + d0)[k] = acc;
+  };
+  for (int64_t k = lane; k < head; k += 32) scalar(k);
+  constexpr int64_t VPC = kBulkChunk / 16;  // 16-B vectors per chunk per source
+  const int64_t nv = (n - head) / EPV;      // 16-B vectors of the body
+  const int64_t nch = (nv + VPC - 1) / VPC; // chunks per source
+  auto chunk_src = [&](int64_t c) {
+    return [=](int j) { return reinterpret_cast<const void *>(src(j) + head + c * VPC * EPV); };
+  };
+  auto chunk_bytes = [&](int64_t c) { return (uint32_t)((nv - c * VPC < VPC ? nv - c * VPC : VPC) * 16); };
+  if (nch > 0 && lane == 0) {
+    asm volatile("fence.proxy.async.global;" ::: "memory");  // producers' generic writes -> bulk reads
+    for (int64_t c = 0; c < nch && c < kBulkStages; ++c) bulk_issue(wb, (int)c, P, chunk_src(c), chunk_bytes(c));
+  }
+  for (int64_t c = 0; c < nch; ++c) {
+    const int st = (int)(c % kBulkStages);
+    bulk_wait(wb, st);
+#pragma unroll
+    for (int64_t v = 0; v < VPC / 32; ++v) {
+      const int64_t vk = c * VPC + v * 32 + lane;
+      if (vk < nv) {
+        const uint4 *sv =
+            reinterpret_cast<const uint4 *>(wb.stage + (size_t)st * kMaxDirect * kBulkChunk) + v * 32 + lane;
+        uint4 acc = sv[0];
+#pragma unroll
+        for (int j = 1; j < kMaxDirect; ++j)
+          if (j < P) acc = vop<DT, OP>(acc, sv[j * VPC]);
+        const int64_t eo = head + EPV * vk;
+        *reinterpret_cast<uint4 *>(out_local + eo) = acc;
+#pragma unroll
+        for (int j = 0; j < kMaxDirect - 1; ++j)
+          if (j < P - 1) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(a.p_recvbuf[j]) + d0 + eo) = acc;
+      }
+    }
+    __syncwarp();
+    if (c + kBulkStages < nch && lane == 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // our generic reads of the stage -> refill
+      bulk_issue(wb, st, P, chunk_src(c + kBulkStages), chunk_bytes(c + kBulkStages));
+    }
+  }
+  for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
+}
+
 template <int DT, int OP>
-__device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W) {
+__device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W, uint8_t *smem) {
   const int P = a.P, r = a.r;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;
   const int64_t es = sizeof(typename Op<DT, OP>::T);
@@ -553,6 +692,8 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
     }
     return;
   }
+  WarpBulk wb{};
+  if (PC_DIRECT_BULK && !a.sys) warp_bulk_init(wb, smem);
   for (int j = 0; j < P - 1; ++j)  // every peer has posted ready-to-receive
     if (!warp_wait(a.rtr + j, e, a.err, a.timeout_ms, -1, a.sys)) return;
   const uint32_t target = e * (uint32_t)(P - 1);
@@ -587,7 +728,12 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
         } else if (i == 1) {
           const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
           const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-          if (hi > lo) warp_fold_pull<DT, OP>(a, base + lo, base + lo, hi - lo);
+          if (hi > lo) {
+            if (PC_DIRECT_BULK && !a.sys)
+              warp_fold_pull_bulk<DT, OP>(a, base + lo, base + lo, hi - lo, wb);
+            else
+              warp_fold_pull<DT, OP>(a, base + lo, base + lo, hi - lo);
+          }
           fence_scope(a.sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
@@ -738,16 +884,18 @@ __global__ void __launch_bounds__(kEngineBlock, 2) coll_engine_group(CollGroupAr
 }
 
 template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock, 2) direct_engine(DirectArgs a) {
-  direct_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
+__global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine(DirectArgs a) {
+  extern __shared__ __align__(128) uint8_t dsmem[];
+  direct_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5, dsmem);
 }
 template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_group(DirectGroupArgs g) {
+__global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine_group(DirectGroupArgs g) {
   int k = 0;
   while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
   const int b = blockIdx.x - g.block_start[k];
   const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
-  direct_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
+  extern __shared__ __align__(128) uint8_t dsmem[];
+  direct_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, dsmem);
 }
 
 // Single-rank launches (one rank per GPU / process).
@@ -807,6 +955,7 @@ struct EngineLaunch {
   static int coll(const CollArgs &a, int warps, cudaStream_t s);
   static int coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s);
   static int occupancy(int *ctas);
+  static int occupancy_direct(int *ctas);
 };
 
 }  // namespace pc

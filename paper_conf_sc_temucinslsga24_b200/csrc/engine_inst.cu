@@ -25,9 +25,22 @@ int EngineLaunch<DT, OP>::rd(const RdArgs &a, int warps, cudaStream_t s) {
   return 0;
 }
 
+// The DIRECT engines take kDirectSmem of dynamic shared memory (bulk-copy
+// stages, engine.cuh): opt in once per kernel.
+template <typename K>
+static int direct_smem_attr(K kernel) {
+  static bool done = false;
+  if (!done && kDirectSmem > 48 * 1024) {
+    PC_CUDA(cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kDirectSmem));
+    done = true;
+  }
+  return 0;
+}
+
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::direct(const DirectArgs &a, int warps, cudaStream_t s) {
-  direct_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+  if (int rc = direct_smem_attr(direct_engine<DT, OP>)) return rc;
+  direct_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, kDirectSmem, s>>>(a);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -51,7 +64,8 @@ int EngineLaunch<DT, OP>::rd_group(const RdGroupArgs &h, int blocks, cudaStream_
 
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s) {
-  direct_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+  if (int rc = direct_smem_attr(direct_engine_group<DT, OP>)) return rc;
+  direct_engine_group<DT, OP><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -62,6 +76,19 @@ int EngineLaunch<DT, OP>::occupancy(int *ctas) {
   int a = 0, b = 0;
   PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, ring_engine<DT, OP>, kEngineBlock, 0));
   PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, rd_engine<DT, OP>, kEngineBlock, 0));
+  *ctas = a < b ? a : b;
+  return 0;
+}
+
+// The DIRECT engines run fewer, fatter CTAs (PC_DIRECT_MINB): their own
+// capacity, with their shared-memory stages when PC_DIRECT_BULK.
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::occupancy_direct(int *ctas) {
+  int a = 0, b = 0;
+  if (int rc = direct_smem_attr(direct_engine_group<DT, OP>)) return rc;
+  if (int rc = direct_smem_attr(direct_engine<DT, OP>)) return rc;
+  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, direct_engine_group<DT, OP>, kEngineBlock, kDirectSmem));
+  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, direct_engine<DT, OP>, kEngineBlock, kDirectSmem));
   *ctas = a < b ? a : b;
   return 0;
 }

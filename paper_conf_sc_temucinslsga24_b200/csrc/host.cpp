@@ -1078,6 +1078,13 @@ int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void
     }
     const int want = (int)env_long("PC_ENGINE_CTAS_PER_SM", 2);
     me.engine_warps = me.sms * std::max(1, std::min(occ, want)) * (kEngineBlock / 32);
+    int docc = 0;
+    if ((rc = direct_occupancy_ctas_per_sm(&docc))) {
+      delete c;
+      return rc;
+    }
+    me.direct_warps = me.sms * std::max(1, std::min(docc, (int)env_long("PC_DIRECT_CTAS_PER_SM", 1))) *
+                      (kEngineBlock / 32);
     c->sms = me.sms;
     c->memops = memops_available();
   }
@@ -1089,7 +1096,7 @@ int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void
   }
   c->ranks = all;
   c->same_proc.assign(size, false);
-  int ew = INT32_MAX;
+  int ew = INT32_MAX, dw = INT32_MAX;
   for (int q = 0; q < size; ++q) {
     const RankRec &r = all[q];
     if (r.magic != me.magic || r.size != size || r.rank != q || r.dry != me.dry) {
@@ -1102,10 +1109,14 @@ int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void
       int on_dev = 0;
       for (int k = 0; k < size; ++k)
         if (memcmp(all[k].uuid, r.uuid, 16) == 0) ++on_dev;
-      ew = std::min(ew, r.engine_warps / std::max(on_dev, 1));
+      // whole CTAs per rank, so every co-located rank's engine CTAs fit at once
+      const int wpb = kEngineBlock / 32;
+      ew = std::min(ew, r.engine_warps / std::max(on_dev, 1) / wpb * wpb);
+      dw = std::min(dw, r.direct_warps / std::max(on_dev, 1) / wpb * wpb);
     }
   }
   c->engine_warps = c->dry ? 1184 : std::max(8, (int)env_long("PC_ENGINE_WARPS", ew));
+  c->direct_warps = c->dry ? 592 : std::max(8, (int)env_long("PC_DIRECT_WARPS", dw));
   if (!c->dry) {
     for (int q = 0; q < size; ++q) {
       if (q == rank || !c->same_proc[q] || all[q].device == cuda_device) continue;
@@ -1232,7 +1243,8 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   } else if (a == PC_ALGO_DIRECT) {
     q->nsteps = 2;  // phase counters [u][0..1][slice]
     q->chunk_elems = chunk_q(L, P, epv);
-    choose_slices(q->chunk_elems, partitions, c->engine_warps * upw, min_elems, &q->slices, &q->slice_elems, epv);
+    q->engine_warps = c->direct_warps;
+    choose_slices(q->chunk_elems, partitions, c->direct_warps * upw, min_elems, &q->slices, &q->slice_elems, epv);
     q->staging_bytes = 0;  // PULL: owners read the peers' send buffers directly
   } else {
     q->nsteps = log2_exact(P);

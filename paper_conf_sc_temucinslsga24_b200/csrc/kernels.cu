@@ -407,5 +407,6 @@ int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s) {
 uint64_t launch_count() { return g_launches.load(); }
 
 int engine_occupancy_ctas_per_sm(int *ctas) { return EngineLaunch<1, 0>::occupancy(ctas); }
+int direct_occupancy_ctas_per_sm(int *ctas) { return EngineLaunch<1, 0>::occupancy_direct(ctas); }
 
 }  // namespace pc

@@ -35,7 +35,7 @@ struct RankRec {
   uint32_t magic;
   int32_t rank, size, device, dry;
   int32_t sms, engine_warps;  // this rank's engine capacity (already divided by ranks on its device)
-  int32_t pad;
+  int32_t direct_warps;  // capacity of the DIRECT engines (fewer, fatter CTAs), same division
   int64_t pid;
   uint64_t proc_token;
   uint8_t uuid[16];
@@ -231,6 +231,7 @@ struct Comm {
   std::vector<RankRec> ranks;
   std::vector<bool> same_proc;
   int engine_warps = 0;  // agreed (min over ranks)
+  int direct_warps = 0;  // the same for the DIRECT allreduce engines
   int sms = 0;
   std::vector<Request *> reqs;
   std::map<std::tuple<int, int, int>, int> post_seq;  // (kind, peer, tag) -> next seq
@@ -405,6 +406,7 @@ struct PreadyAllArgs {
 };
 int launch_pready_all(const PreadyAllArgs &a, cudaStream_t s);
 int engine_occupancy_ctas_per_sm(int *ctas);
+int direct_occupancy_ctas_per_sm(int *ctas);
 uint64_t launch_count();
 
 }  // namespace pc
