@@ -601,6 +601,7 @@ def run_multi(args):
     send = torch.randn(Np * count, device="cuda", generator=gen)
     recv = torch.empty_like(send)
     q = pc.pallreduce_init(send, recv, Np, count, pc.FLOAT32, pc.SUM, algo, comm)
+    info = q.info()
 
     def step():
         q.start(st)
@@ -674,18 +675,20 @@ def run_multi(args):
     comm.destroy()
     if rank == 0:
         eng_ms_v = eng_ms or None
-        nvl_bytes = 2 * (P - 1) / P * S  # per rank per direction (ring)
+        # NVLink bytes per rank per direction: ring and DIRECT 2(P-1)/P*S, RD log2(P)*S
+        nvl_bytes = (P.bit_length() - 1) * S if info["algo_name"] == "rd" else 2 * (P - 1) / P * S
         achieved = nvl_bytes / (eng_ms_v / 1e3) / 1e9 if eng_ms_v else None
         out = {"metric": METRIC, "value": busbw(S, ms / 1e3, P), "unit": "GB/s", "n_gpus": world,
                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
                "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                "config": {"workload": f"partitioned allreduce fp32 sum, {P} ranks (one per B200), {S >> 20} MiB "
                                       f"per rank in {Np} partitions, {args.algo} schedule", "ranks": P,
-                          "bytes_per_rank": S, "partitions": Np, "algo": args.algo,
+                          "bytes_per_rank": S, "partitions": Np, "algo": info["algo_name"],
+                          "algo_requested": args.algo,
                           "l2": "no flush: per-rank working set > 126 MB L2", "parallelism": f"dp{P}"},
                "roofline": {"bound": "nvlink", "achieved": achieved, "peak": 770.0, "unit": "GB/s",
                             "frac": achieved / 770.0 if achieved else None, "traffic": None,
-                            "kernel": "ring_engine", "engine_ms": eng_ms_v,
+                            "kernel": f"{info['algo_name']}_engine", "engine_ms": eng_ms_v,
                             "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s per direction"},
                "cpu_baseline": None, "e2e": {"value": busbw(S, ems / 1e3, P), "unit": "GB/s",
                                              "h2d_bytes_per_step": S, "d2h_bytes_per_step": S, "ms_per_step": ems},

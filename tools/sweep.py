@@ -112,10 +112,14 @@ def sweep_dl(args):
                                         ("bert_large", synth.BERT_LARGE_SIZES, 4 << 20)):
             total = sum(sizes) * 4
             Np = max(1, total // part_bytes)
-            r = time_allreduce(cs, total, Np, pc.ALGO_RING)
-            r["model"] = name
-            r["tensors"] = len(sizes)
-            print(json.dumps(r), flush=True)
+            for an in args.algos.split(","):
+                algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "auto": pc.ALGO_AUTO}[an]
+                if algo == pc.ALGO_RD and P & (P - 1):
+                    continue
+                r = time_allreduce(cs, total, Np, algo)
+                r["model"] = name
+                r["tensors"] = len(sizes)
+                print(json.dumps(r), flush=True)
         for c in cs:
             c.destroy()
         g.destroy()
