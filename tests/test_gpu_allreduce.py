@@ -346,3 +346,25 @@ def test_dtypes_maxmin(kind, op):
         for r in range(P):
             got = y[r] if kind == "f64" else oracle.bf16_to_f64(y[r])
             np.testing.assert_array_equal(got, want)
+
+
+# ------------------------------------------------------------------ c.5 matrix corners
+@pytest.mark.parametrize("algo,Ps", [(pc.ALGO_RING, [2, 3, 8]), (pc.ALGO_RD, [2, 4, 8]),
+                                     (pc.ALGO_DIRECT, [2, 3, 5, 8])])
+@pytest.mark.parametrize("Np,L", [(8, 0), (2, 3), (7, 4), (3, 16), (8, 17)])
+def test_c5_matrix_empty_and_short_chunks(algo, Ps, Np, L):
+    """SURVEY §8(c).5 corners: L = 0 (every partition empty: flags still move,
+    the wait still completes), L < P (empty trailing chunks under reading R4)
+    and non-16-B lengths; int32 wrap sum against the brute-force definition and
+    fp32 bit-exact against the schedule's fold (O3 / O4 / O6), 2 epochs."""
+    oalgo = {pc.ALGO_RING: oracle.RING, pc.ALGO_RD: oracle.RD, pc.ALGO_DIRECT: oracle.DIRECT}[algo]
+    for P in Ps:
+        xi = [np.stack([synth.int32_full(SEED + 70 + e, r, 0, Np * L) for r in range(P)]) for e in range(2)]
+        for x, y in zip(xi, run_allreduce(P, Np, L, xi, algo)):
+            for r in range(P):
+                np.testing.assert_array_equal(y[r], wrap_sum(x))
+        xf = [np.stack([synth.normal_f32(SEED + 80 + e, r, 0, Np * L) for r in range(P)]) for e in range(2)]
+        for x, y in zip(xf, run_allreduce(P, Np, L, xf, algo)):
+            ref, _, _ = oracle.pallreduce(x, Np, oalgo)
+            for r in range(P):
+                assert (y[r].view(np.uint32) == ref[r].view(np.uint32)).all(), (P, r)
