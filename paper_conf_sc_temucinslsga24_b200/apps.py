@@ -23,6 +23,14 @@ def vecadd(A, B, Cout, n: int, gran: int, preq: Prequest | None, stream=None):
                                  _stream(stream)), "vecadd")
 
 
+def pready_cost(A, B, Cout, threads: int, gran: int, preq: Prequest, out_ns, stream=None):
+    """Fig 3 analogue: one block of `threads` threads computes C = A + B and
+    Preadies at `gran`; out_ns (int64 device tensor, 1 element) receives the
+    block's Pready cost from %globaltimer."""
+    _ok(_lib.apps().pcapp_pready_cost(_ptr(A), _ptr(B), _ptr(Cout), threads, gran, preq.ptr, _ptr(out_ns),
+                                      _stream(stream)), "pready_cost")
+
+
 def produce(dst, src, partitions: int, part_bytes: int, gran: int, preq: Prequest, order_stride: int = 1,
             blocks: int = 0, stream=None):
     _ok(_lib.apps().pcapp_produce(_ptr(dst), _ptr(src), partitions, part_bytes, gran, order_stride, blocks,

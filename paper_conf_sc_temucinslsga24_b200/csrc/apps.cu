@@ -105,6 +105,30 @@ __global__ void __launch_bounds__(512) bce_grad_kernel(const float *__restrict__
   }
 }
 
+// Fig 3 analogue: ONE block of t threads computes C = A + B (8 B per
+// thread) and marks it ready at thread / warp / block granularity; thread 0
+// records %globaltimer around the Pready calls (after a block barrier on both
+// sides), i.e. the cost of the block's Pready set including the INLINE copy,
+// fences and flag stores.  Warp granularity needs t % 32 == 0.
+__global__ void pready_cost_kernel(const float2 *__restrict__ A, const float2 *__restrict__ B,
+                                   float2 *__restrict__ C, int gran, pc_prequest_t preq,
+                                   unsigned long long *out_ns) {
+  const int i = threadIdx.x;
+  C[i] = make_float2(A[i].x + B[i].x, A[i].y + B[i].y);
+  __syncthreads();
+  unsigned long long t0 = 0;
+  if (i == 0) t0 = pc_detail::globaltimer();
+  __syncthreads();
+  if (gran == PCAPP_GRAN_THREAD)
+    pc_pready(i, preq);
+  else if (gran == PCAPP_GRAN_WARP)
+    pc_pready_warp(i >> 5, preq);
+  else
+    pc_pready_block(0, preq);
+  __syncthreads();
+  if (i == 0) *out_ns = pc_detail::globaltimer() - t0;
+}
+
 __global__ void check_recv_kernel(pc_prequest_t preq, const uint8_t *recvbuf, uint8_t *out, int partitions,
                                   int64_t part_bytes, int *status) {
   __shared__ int ok;
@@ -380,6 +404,13 @@ int pcapp_vecadd(const float *A, const float *B, float *C, int64_t n, int gran, 
   if (preq) q = *preq;
   if (gran != PCAPP_GRAN_NONE && !preq) return -1;
   vecadd_kernel<<<(unsigned)blocks, 1024, 0, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, gran, q);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_pready_cost(const float *A, const float *B, float *C, int threads, int gran, const pc_prequest_t *preq,
+                      unsigned long long *out_ns, cudaStream_t s) {
+  if (threads < 1 || threads > 1024 || !preq || (gran == PCAPP_GRAN_WARP && threads % 32)) return -1;
+  pready_cost_kernel<<<1, threads, 0, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, gran, *preq, out_ns);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

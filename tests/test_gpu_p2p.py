@@ -572,3 +572,46 @@ def test_host_progression_engine_unsupported_cases():
         rcv.wait()
         snd.free()
         rcv.free()
+
+
+@pytest.mark.parametrize("t", [1, 7, 64, 1024])
+@pytest.mark.parametrize("mode", ["thread", "warp", "block", "thread_agg_block"])
+def test_fig3_single_block_pready(t, mode):
+    """Fig 3 analogue's kernel (one block of t threads, 8 B each, Pready at
+    thread / warp / block granularity or thread with aggregation to one
+    transport partition): bytes delivered every epoch, cost recorded."""
+    gran = {"thread": apps.GRAN_THREAD, "warp": apps.GRAN_WARP, "block": apps.GRAN_BLOCK,
+            "thread_agg_block": apps.GRAN_THREAD}[mode]
+    if gran == apps.GRAN_WARP and t % 32:
+        pytest.skip("warp granularity needs whole warps (reading R11)")
+    n = 2 * t
+    parts = {apps.GRAN_THREAD: t, apps.GRAN_WARP: t // 32, apps.GRAN_BLOCK: 1}[gran]
+    agg = parts if mode == "thread_agg_block" else 1
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        A = torch.from_numpy(synth.uniform_f32(SEED, 0, t, n)).cuda()
+        B = torch.from_numpy(synth.uniform_f32(SEED, 1, t, n)).cuda()
+        Cb, R = torch.empty(n, device="cuda"), torch.zeros(n, device="cuda")
+        ns = torch.zeros(1, dtype=torch.int64, device="cuda")
+        snd = pc.psend_init(Cb, parts, n // parts, pc.FLOAT32, 1, 2, cs[0])
+        rcv = pc.precv_init(R, parts, n // parts, pc.FLOAT32, 0, 2, cs[1])
+        for e in range(3):
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                sq = snd.prequest_create(gran, agg, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            R.zero_()
+            apps.pready_cost(A, B, Cb, t, gran, sq, ns, stream=s0)
+            snd.wait_on_stream(s0)
+            rcv.wait_on_stream(s1)
+            torch.cuda.synchronize()
+            want = (A.cpu().numpy() + B.cpu().numpy()).astype(np.float32)
+            np.testing.assert_array_equal(R.cpu().numpy(), want)
+            assert 0 < int(ns.item()) < 10**8
+        assert snd.error()[0] == 0 and rcv.error()[0] == 0
+        snd.free()
+        rcv.free()
