@@ -596,6 +596,8 @@ def test_fig3_single_block_pready(t, mode):
         snd = pc.psend_init(Cb, parts, n // parts, pc.FLOAT32, 1, 2, cs[0])
         rcv = pc.precv_init(R, parts, n // parts, pc.FLOAT32, 0, 2, cs[1])
         for e in range(3):
+            R.zero_()
+            torch.cuda.synchronize()
             snd.start(s0)
             rcv.start(s1)
             if e == 0:
@@ -604,7 +606,6 @@ def test_fig3_single_block_pready(t, mode):
             else:
                 rcv.pbuf_prepare(s1)
                 snd.pbuf_prepare(s0)
-            R.zero_()
             apps.pready_cost(A, B, Cb, t, gran, sq, ns, stream=s0)
             snd.wait_on_stream(s0)
             rcv.wait_on_stream(s1)
