@@ -255,12 +255,17 @@ def latency_pair(pc, apps, torch, comms, iters=5000, payload=0, copy=None):
     torch.cuda.synchronize()
     errs = [q.error()[0] for q in (a2b, b2a, a_in, b_in)]
     rts = rt.cpu().numpy()[iters // 10:] / 2.0  # one-way = round trip / 2; drop warm-up
-    # the floor: the same ping-pong with two bare flags, no library
-    flags = torch.zeros(64, dtype=torch.int32, device="cuda")
-    tb = torch.zeros(2, dtype=torch.int64, device="cuda")
-    apps.bare_pingpong_pair(flags[0:], flags[32:], iters, 0, tb, st)
-    torch.cuda.synchronize()
-    bare = float(tb[0].item()) / iters / 2.0
+    # the floor: the same ping-pong with two bare flags, no library, at the
+    # scope the library uses for these ranks (GPU: relaxed; the release/acquire
+    # and system-scope variants are reported beside it)
+    floors = {}
+    for sc, name in ((0, "relaxed_gpu"), (1, "acq_rel_gpu"), (2, "acq_rel_sys")):
+        flags = torch.zeros(64, dtype=torch.int32, device="cuda")
+        tb = torch.zeros(2, dtype=torch.int64, device="cuda")
+        apps.bare_pingpong_pair(flags[0:], flags[32:], iters, 0, tb, st, scope=sc)
+        torch.cuda.synchronize()
+        floors[name] = float(tb[0].item()) / iters / 2.0
+    bare = floors["relaxed_gpu"]
     for q in (a2b, a_in, b_in, b2a):
         q.free()
     import numpy as np
@@ -268,7 +273,8 @@ def latency_pair(pc, apps, torch, comms, iters=5000, payload=0, copy=None):
     return {"p50": float(np.percentile(rts, 50)), "p99": float(np.percentile(rts, 99)),
             "mean": float(rts.mean()), "payload_bytes": payload, "iters": iters, "errors": errs,
             "copy": {0: "inline", 2: "ll"}.get(copy, copy), "payload_ok": ok,
-            "bare_flag_floor_mean": bare, "frac_of_floor": bare / float(np.percentile(rts, 50))}
+            "bare_flag_floor_mean": bare, "bare_flag_variants_mean": floors,
+            "frac_of_floor": bare / float(np.percentile(rts, 50))}
 
 
 def c1_bench(pc, apps, torch, epochs=200):

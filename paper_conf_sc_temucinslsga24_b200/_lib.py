@@ -83,7 +83,7 @@ _APP_PROTOS = {
     "pcapp_pingpong": (I32, [P, P, I32, I32, I32, P, P]),
     "pcapp_bare_pingpong": (I32, [P, P, I32, I32, C.c_uint32, P, P]),
     "pcapp_pingpong_pair": (I32, [P, P, P, P, I32, I32, P, P, P]),
-    "pcapp_bare_pingpong_pair": (I32, [P, P, I32, C.c_uint32, P, P]),
+    "pcapp_bare_pingpong_pair": (I32, [P, P, I32, C.c_uint32, P, I32, P]),
     "pcapp_prequest_size": (SZ, []),
     "pcapp_flag_variant": (I32, [P, P, I32, I32, C.c_uint32, P, P]),
     "pcapp_lat_probe_pair": (I32, [P, P, P, P, I32, I32, P, P]),

@@ -70,8 +70,10 @@ def pingpong_pair(sendA: Prequest, recvA: Prequest, sendB: Prequest, recvB: Preq
                                         _ptr(rt_ns), _stream(stream)), "pingpong_pair")
 
 
-def bare_pingpong_pair(flagA, flagB, iters: int, base: int, out_ns, stream=None):
-    _ok(_lib.apps().pcapp_bare_pingpong_pair(_ptr(flagA), _ptr(flagB), iters, base, _ptr(out_ns),
+def bare_pingpong_pair(flagA, flagB, iters: int, base: int, out_ns, stream=None, scope: int = 2):
+    """Flag ping-pong with no library (latency floor).  scope 0: relaxed GPU
+    scope, 1: release/acquire GPU scope, 2: release/acquire system scope."""
+    _ok(_lib.apps().pcapp_bare_pingpong_pair(_ptr(flagA), _ptr(flagB), iters, base, _ptr(out_ns), scope,
                                              _stream(stream)), "bare_pingpong_pair")
 
 

@@ -110,7 +110,7 @@ __global__ void __launch_bounds__(512) bce_grad_kernel(const float *__restrict__
 // records %globaltimer around the Pready calls (after a block barrier on both
 // sides), i.e. the cost of the block's Pready set including the INLINE copy,
 // fences and flag stores.  Warp granularity needs t % 32 == 0.
-__global__ void pready_cost_kernel(const float2 *__restrict__ A, const float2 *__restrict__ B,
+__global__ void __launch_bounds__(1024) pready_cost_kernel(const float2 *__restrict__ A, const float2 *__restrict__ B,
                                    float2 *__restrict__ C, int gran, pc_prequest_t preq,
                                    unsigned long long *out_ns) {
   const int i = threadIdx.x;
@@ -213,8 +213,31 @@ __global__ void pingpong_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, p
   if (threadIdx.x == 0) out_ns[side] = pc_detail::globaltimer() - t0;
 }
 
+// The latency floor: the same ping-pong with two bare flags and no library.
+// scope 0: relaxed GPU-scope loads/stores (the hardware floor for ranks that
+// share a GPU), 1: release/acquire at GPU scope, 2: release/acquire at system
+// scope (what a flag to another GPU costs).
+__device__ __forceinline__ uint32_t bare_ld(const uint32_t *p, int scope) {
+  uint32_t v;
+  if (scope == 0)
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  else if (scope == 1)
+    v = pc_detail::ld_acquire_gpu(p);
+  else
+    v = pc_detail::ld_acquire_sys(p);
+  return v;
+}
+__device__ __forceinline__ void bare_st(uint32_t *p, uint32_t v, int scope) {
+  if (scope == 0)
+    pc_detail::st_relaxed_gpu(p, v);
+  else if (scope == 1)
+    pc_detail::st_release_gpu(p, v);
+  else
+    pc_detail::st_release_sys(p, v);
+}
+
 __global__ void bare_pingpong_pair_kernel(uint32_t *flagA, uint32_t *flagB, int iters, uint32_t base,
-                                          unsigned long long *out_ns) {
+                                          unsigned long long *out_ns, int scope) {
   if (threadIdx.x != 0) return;
   const int side = blockIdx.x;
   uint32_t *mine = side ? flagB : flagA;
@@ -223,11 +246,11 @@ __global__ void bare_pingpong_pair_kernel(uint32_t *flagA, uint32_t *flagB, int 
   for (int k = 1; k <= iters; ++k) {
     const uint32_t v = base + (uint32_t)k;
     if (side == 1)
-      while (!pc_detail::reached(pc_detail::ld_acquire_sys(mine), v)) {
+      while (!pc_detail::reached(bare_ld(mine, scope), v)) {
       }
-    pc_detail::st_release_sys(peer, v);
+    bare_st(peer, v, scope);
     if (side == 0)
-      while (!pc_detail::reached(pc_detail::ld_acquire_sys(mine), v)) {
+      while (!pc_detail::reached(bare_ld(mine, scope), v)) {
       }
   }
   out_ns[side] = pc_detail::globaltimer() - t0;
@@ -464,8 +487,9 @@ int pcapp_pingpong_pair(const pc_prequest_t *sendA, const pc_prequest_t *recvA, 
 }
 
 int pcapp_bare_pingpong_pair(uint32_t *flagA, uint32_t *flagB, int iters, uint32_t base, unsigned long long *out_ns,
+                             int scope,
                              cudaStream_t s) {
-  bare_pingpong_pair_kernel<<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns);
+  bare_pingpong_pair_kernel<<<2, 32, 0, s>>>(flagA, flagB, iters, base, out_ns, scope);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 
