@@ -425,6 +425,27 @@ def jacobi_bench(pc, apps, torch, args):
         for c in cs:
             c.destroy()
         g.destroy()
+    # C4 comparison (i): the same decomposition with kernel -> sync -> copy halos (Listing 1)
+    g, cs = pc.local_comms(8, 0)
+    st = torch.cuda.Stream()
+    js = apps.JacobiSolver(cs, list(range(8)), N, 4, 2, K, H=int(os.environ.get("PC_JACOBI_H", "64")), traditional=True)
+    js.solve(st)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    for _ in range(3):
+        js.solve(st)
+    e1.record(st)
+    torch.cuda.synchronize()
+    ms_iter = e0.elapsed_time(e1) / (3 * K)
+    res["4x2_traditional"] = {"gflops": 4.0 * (N - 2) * (N - 2) / (ms_iter / 1e3) / 1e9, "us_per_iter": ms_iter * 1e3,
+                              "hbm_frac": (8.0 * N * N / (ms_iter / 1e3) / 1e9) / hbm_peak, "ranks": 8,
+                              "halos": "kernel -> cudaStreamSynchronize -> cudaMemcpyAsync per edge (Listing 1)"}
+    res["speedup_partitioned_vs_traditional_4x2"] = res["4x2_traditional"]["us_per_iter"] / res["4x2"]["us_per_iter"]
+    js.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
     res["config"] = f"{N}^2 fp32, {K} iterations per epoch, virtual ranks on one B200, 8 B/cell-update roofline"
     return res
 

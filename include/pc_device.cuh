@@ -483,6 +483,22 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
     return 0;
   }
   uint32_t e = 0, rtr0 = 0;
+  // INLINE partitions of 8 or 16 aligned bytes (the paper's 8 B per thread):
+  // load the payload before the {epoch, rtr} acquire (round trips overlap)
+  const uint64_t off0 = (uint64_t)partition * preq.part_bytes;
+  const bool small = preq.copy == 0 && (preq.part_bytes == 8 || preq.part_bytes == 16) &&
+                     ((reinterpret_cast<uintptr_t>(preq.sbuf + off0) | reinterpret_cast<uintptr_t>(preq.peer_rbuf + off0)) &
+                      (preq.part_bytes - 1)) == 0;
+  uint4 v = make_uint4(0, 0, 0, 0);
+  if (small) {
+    if (preq.part_bytes == 16) {
+      v = __ldcg(reinterpret_cast<const uint4 *>(preq.sbuf + off0));
+    } else {
+      const uint2 h = __ldcg(reinterpret_cast<const uint2 *>(preq.sbuf + off0));
+      v.x = h.x;
+      v.y = h.y;
+    }
+  }
   if (lane == first) {
     if (preq.copy == 0 && preq.part_bytes) {
       const uint2 er = epoch_rtr(preq);
@@ -502,8 +518,14 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
     bool ok = true;
     if (lane == first && !reached(rtr0, e)) ok = spin_geq<true>(preq.rtr, e, preq.err, preq.timeout_ms, partition);
     if (!__shfl_sync(mask, ok, first)) return PC_DEV_ERR_TIMEOUT;
-    const uint64_t off = (uint64_t)partition * preq.part_bytes;
-    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, 0, 1);
+    if (small) {
+      if (preq.part_bytes == 16)
+        *reinterpret_cast<uint4 *>(preq.peer_rbuf + off0) = v;
+      else
+        *reinterpret_cast<uint2 *>(preq.peer_rbuf + off0) = make_uint2(v.x, v.y);
+    } else {
+      copy_bytes(preq.peer_rbuf + off0, preq.sbuf + off0, preq.part_bytes, 0, 1);
+    }
     fence_scope(preq.sys_scope);
   }
   __syncwarp(mask);
@@ -553,6 +575,21 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   }
   uint32_t e = 0;
   bool ok = true;
+  const uint64_t off = (uint64_t)partition * preq.part_bytes;
+  // Small aligned partition (<= one 16-B vector per lane): load the payload
+  // BEFORE the {epoch, rtr} acquire so the two L2 round trips overlap (the
+  // bytes are this kernel's own; only the peer store must follow the acquire).
+  const uintptr_t al = reinterpret_cast<uintptr_t>(preq.sbuf + off) | reinterpret_cast<uintptr_t>(preq.peer_rbuf + off);
+  const bool small16 = preq.part_bytes <= 512 && (preq.part_bytes & 15) == 0 && (al & 15) == 0;
+  const bool small8 = !small16 && preq.part_bytes <= 256 && (preq.part_bytes & 7) == 0 && (al & 7) == 0;
+  const bool small = small16 || small8;
+  uint4 v = make_uint4(0, 0, 0, 0);
+  if (small16 && 16ull * lane < preq.part_bytes) v = __ldcg(reinterpret_cast<const uint4 *>(preq.sbuf + off) + lane);
+  if (small8 && 8ull * lane < preq.part_bytes) {
+    const uint2 h = __ldcg(reinterpret_cast<const uint2 *>(preq.sbuf + off) + lane);
+    v.x = h.x;
+    v.y = h.y;
+  }
   if (lane == 0) {
     const uint2 er = epoch_rtr(preq);
     e = er.x;
@@ -560,8 +597,13 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   }
   e = __shfl_sync(full, e, 0);
   if (!__shfl_sync(full, ok, 0)) return PC_DEV_ERR_TIMEOUT;
-  const uint64_t off = (uint64_t)partition * preq.part_bytes;
-  copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, lane, 32);
+  if (small16) {
+    if (16ull * lane < preq.part_bytes) reinterpret_cast<uint4 *>(preq.peer_rbuf + off)[lane] = v;
+  } else if (small8) {
+    if (8ull * lane < preq.part_bytes) reinterpret_cast<uint2 *>(preq.peer_rbuf + off)[lane] = make_uint2(v.x, v.y);
+  } else {
+    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, lane, 32);
+  }
   fence_scope(preq.sys_scope);
   __syncwarp(full);
   if (lane == 0) publish(preq, t, 1, e, partition);

@@ -90,6 +90,7 @@ _APP_PROTOS = {
     "pcapp_jacobi_rank_size": (SZ, []),
     "pcapp_jacobi_launch": (I32, [P, P, I32, I32, I32, I32, P]),
     "pcapp_jacobi_describe": (I32, [P, P, P, I32, I32, I32, I32, I32, I32, P, P, P, P, P]),
+    "pcapp_jacobi_set_traditional": (I32, [P, I32]),
     "pcapp_jacobi_launch2": (I32, [P, P, I32, I32, I32, I32, I32, I32, I32, P]),
     "pcapp_jacobi_describe2": (I32, [P, P, P, I32, I32, I32, I32, I32, I32, P, P, P, P, P, I32, I32]),
 }

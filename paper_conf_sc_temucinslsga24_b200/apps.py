@@ -104,7 +104,7 @@ class JacobiSolver:
     every halo partition is (iteration slot, edge segment), readied once."""
 
     def __init__(self, comms, ranks, N: int, Py: int, Px: int, iters: int, H: int = 64, device: int = 0,
-                 kernel: str | None = None):
+                 kernel: str | None = None, traditional: bool = False):
         import os
 
         import torch
@@ -117,6 +117,10 @@ class JacobiSolver:
         self.mode = JACOBI_MODES[self.kernel]
         assert self.lx % STRIP == 0 and self.ly % H == 0, "lx must be a multiple of 128, ly of H"
         self.W = jacobi_strip(self.lx, self.mode)
+        # traditional = the Listing 1 baseline (C4 comparison (i)): no partitioned
+        # requests; kernel -> cudaStreamSynchronize -> peer copies of the edges
+        self.traditional = traditional
+        assert not traditional or self.mode == 1, "the traditional baseline uses the rows kernel"
         self.comms, self.ranks = comms, ranks
         dev = torch.device("cuda", device)
         self.dev = dev
@@ -136,6 +140,8 @@ class JacobiSolver:
                 parts = (iters + 1) * nseg
                 st["send"][d] = torch.zeros(parts * seg, device=dev)
                 st["halo"][d] = torch.zeros(parts * seg, device=dev)
+                if traditional:
+                    continue
                 st["sreq"][d] = rt.psend_init(st["send"][d], parts, seg, rt.FLOAT32, q, _SEND_TAG[d], comm)
                 st["rreq"][d] = rt.precv_init(st["halo"][d], parts, seg, rt.FLOAT32, q, _RECV_TAG[d], comm)
             self.local.append(st)
@@ -183,6 +189,8 @@ class JacobiSolver:
                                             has, sendp, halop, sqp, rqp, self.mode, self.W)
             if rc != 0:
                 raise RuntimeError("pcapp_jacobi_describe failed")
+            if self.traditional:
+                _ok(lib.pcapp_jacobi_set_traditional(buf, 1), "jacobi traditional")
             raw[i * sz:(i + 1) * sz] = buf.raw
             starts.append(blocks)
             tiles = (self.ly // self.H) * (self.lx // self.W)
@@ -197,6 +205,8 @@ class JacobiSolver:
         first_prepare(list_of_request_lists) runs the blocking first
         pbuf_prepare across ranks (threads for co-located ranks)."""
         lib = _lib.apps()
+        if self.traditional:
+            return self._solve_traditional(stream)
         for st in self.local:
             for q in self._reqs(st):
                 q.start(stream)
@@ -231,6 +241,38 @@ class JacobiSolver:
         for st in self.local:
             for q in st["rreq"].values():
                 q.wait_on_stream(stream)
+        self.epochs += 1
+
+    def _solve_traditional(self, stream):
+        """The Listing 1 baseline (C4 comparison (i)): every iteration is
+        kernel -> cudaStreamSynchronize -> device-to-device copies of the staged
+        edges into the neighbours' halo slots (cudaMemcpyAsync; a peer copy
+        across GPUs), the next kernel stream-ordered after the copies.  Needs
+        every rank in this process."""
+        torch = self.torch
+        assert len(self.local) == self.Py * self.Px, "traditional baseline: all ranks in this process"
+        lib = _lib.apps()
+        if self.desc is None:
+            self._build_desc()
+        s = stream.cuda_stream if hasattr(stream, "cuda_stream") else (stream or 0)
+        n = len(self.local)
+        by_rank = {st["r"]: st for st in self.local}
+        opp = {T: B, B: T, L: R, R: L}
+
+        def exchange(j):
+            with torch.cuda.stream(stream):
+                for st in self.local:
+                    for d, q in st["nb"].items():
+                        if q < 0:
+                            continue
+                        m = self.lx if d in (T, B) else self.ly
+                        by_rank[q]["halo"][opp[d]][j * m:(j + 1) * m].copy_(st["send"][d][j * m:(j + 1) * m])
+
+        for k in range(-1, self.K):
+            _ok(lib.pcapp_jacobi_launch2(self.desc.data_ptr(), self.starts.data_ptr(), n, self.blocks, max(k, 0),
+                                         1 if k < 0 else 0, self.mode, self.W, self.H, s), "jacobi traditional")
+            stream.synchronize()  # Listing 1: the host waits for the kernel before sending
+            exchange(k + 1)
         self.epochs += 1
 
     def errors(self):

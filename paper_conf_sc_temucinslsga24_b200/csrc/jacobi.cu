@@ -48,6 +48,8 @@ struct JacobiRank {
   int tiles;              // (ly/H) * (lx/W): warps (mode 0) or CTAs (mode 1)
   int W;                  // columns per tile: 128 (mode 0, one warp) or the CTA strip (mode 1)
   int mode;               // 0 warp tiles (register sliding window), 1 CTA row pipeline (bulk copies)
+  int trad;               // 1: traditional baseline (Listing 1): no Parrived / Pready in the kernel;
+                          //    the host copies the staged edges between launches
 };
 
 __device__ __forceinline__ float stencil(float up, float dn, float lf, float rt) {
@@ -274,7 +276,7 @@ __device__ void tile_rows_iter(const JacobiRank &d, int tile, int k, uint8_t *sm
       for (int j = 0; j < first; ++j)  // grid rows first: they need no arrival
         if (!halo_row(j)) issue(j);
       // Parrived: the halo segments this tile reads (slot k), then their copies
-      if (top | bot | left | right) {
+      if ((top | bot | left | right) && !d.trad) {
         halo_wait(d, top, bot, left, right, sx, rb, k);
         asm volatile("fence.proxy.async.global;" ::: "memory");
       }
@@ -349,7 +351,7 @@ __device__ void tile_rows_iter(const JacobiRank &d, int tile, int k, uint8_t *sm
     }
   }
   // Pready: push my edge segments of slot k+1 (INLINE copy by warp 0)
-  if (top | bot | left | right) {
+  if ((top | bot | left | right) && !d.trad) {
     __syncthreads();
     if (warp == 0) edge_pready(d, top, bot, left, right, sx, rb, k + 1);
   }
@@ -370,7 +372,7 @@ __device__ void tile_rows_init(const JacobiRank &d, int tile) {
     if (left) d.sendbuf[L][r] = __ldcg(a + (size_t)r * lx);
     if (right) d.sendbuf[R][r] = __ldcg(a + (size_t)r * lx + lx - 1);
   }
-  if (top | bot | left | right) {
+  if ((top | bot | left | right) && !d.trad) {
     __syncthreads();
     if (tid < 32) edge_pready(d, top, bot, left, right, sx, rb, 0);
   }
@@ -461,7 +463,7 @@ int pcapp_jacobi_describe2(void *out, float *grid0, float *grid1, int ly, int lx
     d.has[i] = has[i];
     d.sendbuf[i] = sendbuf[i];
     d.halo[i] = halo[i];
-    if (has[i]) {
+    if (has[i] && sq[i] && rq[i]) {
       d.sq[i] = *sq[i];
       d.rq[i] = *rq[i];
     }
@@ -472,6 +474,15 @@ int pcapp_jacobi_describe2(void *out, float *grid0, float *grid1, int ly, int lx
   d.W = W;
   d.mode = mode;
   *(JacobiRank *)out = d;
+  return 0;
+}
+
+// Traditional baseline switch on a filled descriptor (mode 1 only): the
+// kernel neither waits for halos nor Preadies its edges.
+int pcapp_jacobi_set_traditional(void *desc, int trad) {
+  JacobiRank *d = (JacobiRank *)desc;
+  if (trad && d->mode != 1) return -1;
+  d->trad = trad;
   return 0;
 }
 

@@ -82,3 +82,22 @@ def test_jacobi_tile_heights(H, kernel):
     a0 = synth.jacobi_init(N, N, "random")
     (got,) = solve(a0, 2, 2, iters, H=H, kernel=kernel)
     np.testing.assert_array_equal(got, oracle.jacobi_seq(a0, iters))
+
+
+@pytest.mark.parametrize("Py,Px,N", [(2, 2, 512), (4, 1, 512), (2, 4, 1024)])
+def test_jacobi_traditional_baseline_bitexact(Py, Px, N):
+    """C4 comparison (i): the same rows kernel with kernel -> sync -> copies
+    of the staged edges (Listing 1) instead of in-kernel Pready / Parrived
+    gives the same bits as the oracle."""
+    a0 = synth.jacobi_init(N, N, "random")
+    iters = 30
+    with comms(Py * Px) as cs:
+        st = torch.cuda.Stream()
+        js = apps.JacobiSolver(cs, list(range(Py * Px)), N, Py, Px, iters, H=32, traditional=True)
+        js.set_initial(a0)
+        torch.cuda.synchronize()
+        js.solve(st)
+        torch.cuda.synchronize()
+        got = js.result()
+        js.free()
+    np.testing.assert_array_equal(got, oracle.jacobi_seq(a0, iters))
