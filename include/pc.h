@@ -144,7 +144,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
  * schedule of P:L151-L155 with neighbour sets).  Collective, like
  * pc_pallreduce_init (shared posting order), P <= 8.  Schedule: reduce-scatter
  * PULLS (owners fold the peers' blocks with peer loads, rank order, reading
- * R25); allgather and broadcast PUSH 16-B vectors into the peers' buffers.
+ * R25); allgather PUSHES each 16-B vector once to all P buffers; broadcast is PULLED by the receivers.
  *
  * reduce_scatter: sendbuf partitions x P x count elements (partition u = P
  *   blocks of count, block k for rank k); recvbuf partitions x count:
@@ -158,7 +158,8 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
  *   partitions are the P x partitions blocks: pc_parrived(k * partitions + u)
  *   = rank k's partition u is in recvbuf.
  * bcast: buf partitions x count on every rank; the root's pc_pready(u) delivers
- *   buf[u] to every rank; pc_parrived(u) = buf[u] holds the root's data. */
+ *   buf[u] to every rank (the receivers PULL it with peer loads); pc_parrived(u)
+ *   = buf[u] holds the root's data (root: every rank has pulled it). */
 int pc_preduce_scatter_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,
                             pc_op_t op, pc_comm_t comm, pc_request_t *req);
 int pc_pallgather_init(const void *sendbuf, void *recvbuf, int partitions, size_t count, pc_dtype_t dtype,

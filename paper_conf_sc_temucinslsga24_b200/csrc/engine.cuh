@@ -249,6 +249,56 @@ __device__ __forceinline__ void warp_copy(void *dst, const void *src, int64_t nb
   copy_bytes(reinterpret_cast<uint8_t *>(dst), reinterpret_cast<const uint8_t *>(src), (uint64_t)nbytes, lane, 32);
 }
 
+// src -> dst0 and dsts[0 .. nd-1] at the same byte offset (the allgather
+// push): every source vector is loaded ONCE and stored nd+1 times.  The
+// destinations share one misalignment (same offset of 16-B aligned buffers);
+// if the source does not, fall back to one warp_copy per destination.
+template <int MAXD>
+__device__ __forceinline__ void warp_copy_multi(uint8_t *dst0, uint8_t *const *dsts, int nd, int64_t doff,
+                                                const uint8_t *src, int64_t nbytes) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uintptr_t m = reinterpret_cast<uintptr_t>(dst0 + doff) & 15;
+  if ((reinterpret_cast<uintptr_t>(src) & 15) != m) {
+    warp_copy(dst0 + doff, src, nbytes);
+    for (int j = 0; j < nd; ++j) warp_copy(dsts[j] + doff, src, nbytes);
+    return;
+  }
+  int64_t h = (int64_t)((16 - m) & 15);
+  if (h > nbytes) h = nbytes;
+  for (int64_t b = lane; b < h; b += 32) {
+    const uint8_t v = src[b];
+    dst0[doff + b] = v;
+    for (int j = 0; j < nd; ++j) dsts[j][doff + b] = v;
+  }
+  const int64_t nv = (nbytes - h) >> 4;
+  const uint4 *s4 = reinterpret_cast<const uint4 *>(src + h);
+  int64_t k = lane;
+  for (; k + 32 * 3 < nv; k += 32 * 4) {
+    uint4 x[4];
+#pragma unroll
+    for (int v = 0; v < 4; ++v) x[v] = __ldcg(s4 + k + 32 * v);
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+      reinterpret_cast<uint4 *>(dst0 + doff + h)[k + 32 * v] = x[v];
+#pragma unroll
+      for (int j = 0; j < MAXD; ++j)
+        if (j < nd) reinterpret_cast<uint4 *>(dsts[j] + doff + h)[k + 32 * v] = x[v];
+    }
+  }
+  for (; k < nv; k += 32) {
+    const uint4 x = __ldcg(s4 + k);
+    reinterpret_cast<uint4 *>(dst0 + doff + h)[k] = x;
+#pragma unroll
+    for (int j = 0; j < MAXD; ++j)
+      if (j < nd) reinterpret_cast<uint4 *>(dsts[j] + doff + h)[k] = x;
+  }
+  for (int64_t b = h + (nv << 4) + lane; b < nbytes; b += 32) {
+    const uint8_t v = src[b];
+    dst0[doff + b] = v;
+    for (int j = 0; j < nd; ++j) dsts[j][doff + b] = v;
+  }
+}
+
 __device__ __forceinline__ int modp(int a, int p) { return ((a % p) + p) % p; }
 
 // ---------------------------------------------------------------------------
@@ -766,8 +816,11 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
 //    0: ready[u] -> copy my block to recvbuf[r][u] here and at every peer,
 //       fence, per-source arrival flag + phase-0 counter at every peer
 //    1: P-1 arrivals of partition u -> done[u]
-//  BCAST (buf [u][count]) root: ready[u] -> push to every peer -> done[u];
-//    non-root: root's arrival (phase-0 counter) -> done[u]
+//  BCAST (buf [u][count]), PULL: root: ready[u] -> announce to every peer
+//    (phase-0 counter) -> all P-1 peers done reading (phase-1) -> done[u];
+//    non-root: root's announcement -> copy the root's slice into my buf with
+//    peer loads -> tell the root (its phase-1 counter) -> done[u]
+//  (ALLGATHER pushes each vector once to all P buffers: warp_copy_multi)
 // ---------------------------------------------------------------------------
 template <int DT, int OP>
 __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const int W) {
@@ -778,7 +831,8 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
   const bool rs = a.coll == PC_COLL_REDUCE_SCATTER, ag = a.coll == PC_COLL_ALLGATHER;
   const bool bc = a.coll == PC_COLL_BCAST, root = bc && r == a.root;
   // writers into peers' buffers need every peer's ready-to-receive
-  if (P > 1 && (ag || root))
+  // (allgather pushes; the broadcast is pulled by the receivers themselves)
+  if (P > 1 && ag)
     for (int j = 0; j < P - 1; ++j)
       if (!warp_wait(a.rtr + j, e, a.err, a.timeout_ms, -1, a.sys)) return;
   const uint32_t target = e * (uint32_t)(P - 1);
@@ -811,21 +865,23 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
           }
           if (ag && (threadIdx.x & 31) == 0) st_release_gpu(a.srcflags + (int64_t)u * a.ns + s, e);
           finished = true;
-        } else if (bc && !root) {
+        } else if (bc && !root) {  // PULL: copy the root's slice once it is announced, then tell the root
           if (!warp_poll(cnt_u, e, a.sys)) continue;
+          const int jr = (a.root - r - 1 + P) % P;
+          const int64_t off = ((int64_t)u * a.count + lo) * es;
+          if (n) warp_copy(a.recvbuf + off, a.p_recvbuf[jr] + off, n * es);
+          fence_scope(a.sys);  // our reads of the root's slice are done before it may reuse it
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0) red_add_scope(a.p_cnt[jr] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
           finished = true;
         } else if (i == 0) {
           if (!warp_poll(a.ready + u, e, false)) continue;
           const int64_t off = ((int64_t)u * a.count + lo) * es;  // my block (AG, BCAST)
           if (ag) {
             const int64_t doff = (((int64_t)r * a.Np + u) * a.count + lo) * es;
-            if (n) {
-              warp_copy(a.recvbuf + doff, a.sendbuf + off, n * es);
-              for (int j = 0; j < P - 1; ++j) warp_copy(a.p_recvbuf[j] + doff, a.sendbuf + off, n * es);
-            }
-          } else if (root && n) {
-            for (int j = 0; j < P - 1; ++j) warp_copy(a.p_recvbuf[j] + off, a.sendbuf + off, n * es);
+            if (n) warp_copy_multi<kMaxDirect - 1>(a.recvbuf, a.p_recvbuf, P - 1, doff, a.sendbuf + off, n * es);
           }
+          // (broadcast root: nothing to copy — the peers PULL the slice)
           fence_scope(a.sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0) {
@@ -835,8 +891,10 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
             }
             if (ag) st_release_gpu(a.srcflags + ((int64_t)r * a.Np + u) * a.ns + s, e);
           }
-          if (root) finished = true;
-          else step[jj] = 1;
+          step[jj] = 1;
+        } else if (i == 1 && root) {  // every peer has pulled the slice
+          if (!warp_poll(cnt_u + a.ns, target, a.sys)) continue;
+          finished = true;
         } else if (i == 1) {
           if (!warp_poll(cnt_u, target, a.sys)) continue;
           if (rs) {
@@ -871,11 +929,11 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
 }
 
 template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock, 2) coll_engine(CollArgs a) {
+__global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) coll_engine(CollArgs a) {
   coll_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
 }
 template <int DT, int OP>
-__global__ void __launch_bounds__(kEngineBlock, 2) coll_engine_group(CollGroupArgs g) {
+__global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) coll_engine_group(CollGroupArgs g) {
   int k = 0;
   while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
   const int b = blockIdx.x - g.block_start[k];

@@ -90,6 +90,11 @@ int EngineLaunch<DT, OP>::occupancy_direct(int *ctas) {
   PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, direct_engine_group<DT, OP>, kEngineBlock, kDirectSmem));
   PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, direct_engine<DT, OP>, kEngineBlock, kDirectSmem));
   *ctas = a < b ? a : b;
+  // the collective engines (reduce-scatter PULL fold) use the same fat CTAs
+  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, coll_engine<DT, OP>, kEngineBlock, 0));
+  PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, coll_engine_group<DT, OP>, kEngineBlock, 0));
+  *ctas = *ctas < a ? *ctas : a;
+  *ctas = *ctas < b ? *ctas : b;
   return 0;
 }
 

@@ -1297,12 +1297,12 @@ static int coll_init(int coll, const void *sendbuf, void *recvbuf, int partition
   q->seq = c->allreduce_seq++;
   q->agg = 1;
   q->ntransport = partitions;
-  q->engine_warps = c->engine_warps;
+  q->engine_warps = c->direct_warps;  // fat CTAs, like the DIRECT allreduce
   q->nsteps = 2;
   q->chunk_elems = (int64_t)count;
   const int64_t epv = std::max<int64_t>(1, 16 / (int64_t)esz);
   const int64_t min_elems = std::max<int64_t>(1, env_long("PC_MIN_SLICE_BYTES", 8192) / (int64_t)esz);
-  choose_slices((int64_t)count, partitions, c->engine_warps, min_elems, &q->slices, &q->slice_elems, epv);
+  choose_slices((int64_t)count, partitions, c->direct_warps, min_elems, &q->slices, &q->slice_elems, epv);
   q->staging_bytes = 0;
   size_t nflags = (size_t)partitions * 2 * (size_t)q->slices;
   if (coll == PC_COLL_ALLGATHER) nflags += (size_t)P * partitions * (size_t)q->slices;

@@ -105,6 +105,81 @@ def sweep_allreduce(args):
         g.destroy()
 
 
+def time_coll(cs, kind, S, Np, min_ms=30.0):
+    """NEXT-3 collectives, nccl-tests conventions: S = the full buffer (reduce-
+    scatter input, allgather output, broadcast buffer) per rank; busBW =
+    S/t * (P-1)/P for reduce-scatter / allgather, S/t for broadcast."""
+    P = len(cs)
+    st = torch.cuda.Stream()
+    if kind == "rs":
+        count = max(S // 4 // (Np * P), 1)
+        send = [torch.randn(Np * P * count, device="cuda") for _ in range(P)]
+        recv = [torch.empty(Np * count, device="cuda") for _ in range(P)]
+        reqs = [pc.preduce_scatter_init(send[r], recv[r], Np, count, pc.FLOAT32, pc.SUM, cs[r]) for r in range(P)]
+        full = Np * P * count * 4
+    elif kind == "ag":
+        count = max(S // 4 // (Np * P), 1)
+        send = [torch.randn(Np * count, device="cuda") for _ in range(P)]
+        recv = [torch.empty(P * Np * count, device="cuda") for _ in range(P)]
+        reqs = [pc.pallgather_init(send[r], recv[r], Np, count, pc.FLOAT32, cs[r]) for r in range(P)]
+        full = P * Np * count * 4
+    else:
+        count = max(S // 4 // Np, 1)
+        buf = [torch.randn(Np * count, device="cuda") for _ in range(P)]
+        reqs = [pc.pbcast_init(buf[r], Np, count, pc.FLOAT32, 0, cs[r]) for r in range(P)]
+        full = Np * count * 4
+    producers = reqs if kind != "bc" else reqs[:1]
+
+    def step(first=False):
+        if first:
+            for q in reqs:
+                q.start(st)
+            pc.run_ranks([(lambda q=q: q.pbuf_prepare(st)) for q in reqs])
+        else:
+            pc.startall(reqs, st)
+            pc.pbuf_prepare_all(reqs, st)
+        pc.preadyall(producers, st)
+        for q in reqs:
+            q.wait_on_stream(st)
+
+    step(True)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    step()
+    e1.record(st)
+    torch.cuda.synchronize()
+    iters = int(max(5, min(2000, min_ms / max(e0.elapsed_time(e1), 1e-3))))
+    blocks = []
+    for _ in range(3):
+        e0.record(st)
+        for _ in range(iters):
+            step()
+        e1.record(st)
+        torch.cuda.synchronize()
+        blocks.append(e0.elapsed_time(e1) / iters)
+    errs = [q.error() for q in reqs if q.error()[0] != 0]
+    for q in reqs:
+        q.free()
+    ms = statistics.median(blocks)
+    fac = 1.0 if kind == "bc" else (P - 1) / P
+    return {"coll": kind, "ranks": P, "bytes": full, "partitions": Np, "us_per_step": ms * 1e3,
+            "busbw_gbs": full / (ms / 1e3) * fac / 1e9, "errors": errs}
+
+
+def sweep_coll(args):
+    for P in [int(x) for x in args.ranks.split(",")]:
+        g, cs = pc.local_comms(P, 0)
+        for kind in ("rs", "ag", "bc"):
+            for S in [1 << 20, 16 << 20, 256 << 20, 1 << 30]:
+                if S > args.max_bytes:
+                    continue
+                print(json.dumps(time_coll(cs, kind, S, 64)), flush=True)
+        for c in cs:
+            c.destroy()
+        g.destroy()
+
+
 def sweep_dl(args):
     for P in [int(x) for x in args.ranks.split(",")]:
         g, cs = pc.local_comms(P, 0)
@@ -259,11 +334,12 @@ def sweep_p2p(args):
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
-    ap.add_argument("what", choices=["allreduce", "dl", "dl_tensor", "p2p"])
+    ap.add_argument("what", choices=["allreduce", "dl", "dl_tensor", "p2p", "coll"])
     ap.add_argument("--ranks", default="8")
     ap.add_argument("--algos", default="ring,rd")
     ap.add_argument("--partitions", default="1,16,64")
     ap.add_argument("--max-bytes", type=int, default=1 << 30)
     ap.add_argument("--graph", action="store_true", help="replay a captured CUDA graph of the epoch")
     a = ap.parse_args()
-    {"allreduce": sweep_allreduce, "dl": sweep_dl, "dl_tensor": sweep_dl_per_tensor, "p2p": sweep_p2p}[a.what](a)
+    {"allreduce": sweep_allreduce, "dl": sweep_dl, "dl_tensor": sweep_dl_per_tensor, "p2p": sweep_p2p,
+     "coll": sweep_coll}[a.what](a)
