@@ -526,10 +526,15 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
     } else {
       copy_bytes(preq.peer_rbuf + off0, preq.sbuf + off0, preq.part_bytes, 0, 1);
     }
-    fence_scope(preq.sys_scope);
   }
+  // One fence per group, not per lane: __syncwarp orders the group's pushes
+  // before the leader's fence, which is cumulative (the cooperative-groups
+  // grid.sync pattern: barrier, then one thread's fence + signal).
   __syncwarp(mask);
-  if (lane == leader) publish(preq, t, __popc(grp), e, partition);
+  if (lane == leader) {
+    if (preq.part_bytes) fence_scope(preq.sys_scope);
+    publish(preq, t, __popc(grp), e, partition);
+  }
   return 0;
 }
 
@@ -604,9 +609,11 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   } else {
     copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, lane, 32);
   }
-  fence_scope(preq.sys_scope);
-  __syncwarp(full);
-  if (lane == 0) publish(preq, t, 1, e, partition);
+  __syncwarp(full);  // the warp's pushes, then ONE cumulative fence by lane 0
+  if (lane == 0) {
+    fence_scope(preq.sys_scope);
+    publish(preq, t, 1, e, partition);
+  }
   __syncwarp(full);
   return 0;
 }
@@ -647,6 +654,20 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
     }
     return 0;
   }
+  // Partitions of at most one 16-B vector per thread (the paper's 8 KiB
+  // block = 1024 threads x 8 B): load the payload BEFORE the {epoch, rtr}
+  // acquire and the barrier, so their latencies overlap.
+  const uint64_t off = (uint64_t)partition * preq.part_bytes;
+  const uintptr_t al = reinterpret_cast<uintptr_t>(preq.sbuf + off) | reinterpret_cast<uintptr_t>(preq.peer_rbuf + off);
+  const bool v16 = preq.part_bytes <= 16ull * nthr && (preq.part_bytes & 15) == 0 && (al & 15) == 0;
+  const bool v8 = !v16 && preq.part_bytes <= 8ull * nthr && (preq.part_bytes & 7) == 0 && (al & 7) == 0;
+  uint4 v = make_uint4(0, 0, 0, 0);
+  if (v16 && 16ull * tid < preq.part_bytes) v = __ldcg(reinterpret_cast<const uint4 *>(preq.sbuf + off) + tid);
+  if (v8 && 8ull * tid < preq.part_bytes) {
+    const uint2 h = __ldcg(reinterpret_cast<const uint2 *>(preq.sbuf + off) + tid);
+    v.x = h.x;
+    v.y = h.y;
+  }
   if (tid == 0) {
     const uint2 er = epoch_rtr(preq);
     s_e = er.x;
@@ -656,11 +677,18 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
   __syncthreads();
   const uint32_t e = s_e;
   if (!s_ok) return PC_DEV_ERR_TIMEOUT;
-  const uint64_t off = (uint64_t)partition * preq.part_bytes;
-  copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, tid, nthr);
-  fence_scope(preq.sys_scope);
-  __syncthreads();
-  if (tid == 0) publish(preq, t, 1, e, partition);
+  if (v16) {
+    if (16ull * tid < preq.part_bytes) reinterpret_cast<uint4 *>(preq.peer_rbuf + off)[tid] = v;
+  } else if (v8) {
+    if (8ull * tid < preq.part_bytes) reinterpret_cast<uint2 *>(preq.peer_rbuf + off)[tid] = make_uint2(v.x, v.y);
+  } else {
+    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, tid, nthr);
+  }
+  __syncthreads();  // the block's pushes, then ONE cumulative fence by thread 0 (not one per thread)
+  if (tid == 0) {
+    fence_scope(preq.sys_scope);
+    publish(preq, t, 1, e, partition);
+  }
   return 0;
 }
 
