@@ -485,10 +485,9 @@ def run_virtual(args):
             for q in reqs:
                 q.start(st)
             pc.run_ranks([(lambda q=q: q.pbuf_prepare(st)) for q in reqs])
-        else:
-            pc.startall(reqs, st)  # one kernel for every rank's epoch
-            pc.pbuf_prepare_all(reqs, st)  # one kernel for every RTR
-        pc.preadyall(reqs, st)  # S_0: the user's Pready of every partition, one kernel
+            pc.preadyall(reqs, st)  # S_0: the user's Pready of every partition, one kernel
+        else:  # pc_epoch_all: Start + ready-to-receive + S_0 Pready of every rank, ONE kernel
+            pc.epoch_all(reqs, pready=True, stream=st)
         for q in reqs:
             q.wait_on_stream(st)
 

@@ -182,6 +182,13 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream);
 /* MPI_Startall analogue: pc_start for n requests of one GPU, with a single
  * device kernel advancing all n epochs (CUDA-graph capturable). */
 int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream);
+/* The whole control part of an epoch in ONE kernel, for n (<= 16) requests of
+ * one GPU whose first pc_pbuf_prepare (exchange + mapping) already happened:
+ * pc_startall + pc_pbuf_prepare_all, and with pready != 0 also the user's
+ * Pready of every partition of each request (allreduce-kind requests only;
+ * PC_ERR_ARG otherwise) — the small-message path, where launches dominate.
+ * PC_ERR_STATE if a request is active or not yet exchanged.  Capturable. */
+int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream);
 /* pc_pbuf_prepare for n requests whose first pc_pbuf_prepare (exchange +
  * mapping) already happened: all ready-to-receive writes in one kernel.
  * PC_ERR_STATE if a request is inactive or not yet exchanged. */

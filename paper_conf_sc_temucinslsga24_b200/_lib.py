@@ -47,6 +47,7 @@ _PC_PROTOS = {
     "pc_pbcast_init": (I32, [P, I32, SZ, I32, I32, P, C.POINTER(P)]),
     "pc_start": (I32, [P, P]),
     "pc_startall": (I32, [I32, P, P]),
+    "pc_epoch_all": (I32, [I32, P, I32, P]),
     "pc_pbuf_prepare_all": (I32, [I32, P, P]),
     "pc_pbuf_prepare": (I32, [P, P]),
     "pc_prequest_create": (I32, [P, I32, I32, I32, P]),

@@ -327,6 +327,34 @@ __device__ __forceinline__ bool warp_poll(const uint32_t *p, uint32_t target, bo
   return __shfl_sync(0xffffffffu, ok, 0);
 }
 
+// Warp-wide bounded wait until words[0 .. n-1] (n <= 32) have all reached
+// target: lane j polls word j, so the n acquires are in flight together (one
+// round trip per poll instead of n sequential waits).
+__device__ __forceinline__ bool warp_wait_all(const uint32_t *words, int n, uint32_t target, int32_t *err,
+                                              uint32_t tmo, bool sys) {
+  const uint32_t lane = threadIdx.x & 31;
+  bool mine = lane >= (uint32_t)n;
+  const uint64_t t0 = globaltimer();
+  uint32_t k = 0;
+  for (;;) {
+    if (!mine) mine = reached(sys ? ld_acquire_sys(words + lane) : ld_acquire_gpu(words + lane), target);
+    if (__all_sync(0xffffffffu, mine)) return true;
+    if ((++k & 63) == 0) {
+      int stop = 0;
+      if (lane == 0) {
+        if (aborted(err)) {
+          stop = 1;
+        } else if (tmo && globaltimer() - t0 > (uint64_t)tmo * 1000000ull) {
+          set_error(err, PC_DEV_ERR_TIMEOUT, -1);
+          stop = 1;
+        }
+      }
+      if (__shfl_sync(0xffffffffu, stop, 0)) return false;
+      if (k > 1024) __nanosleep(256);
+    }
+  }
+}
+
 // Idle backoff shared by the sweeping engines; false on abort / timeout.
 struct Idle {
   uint64_t since = 0;
@@ -744,8 +772,8 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
   }
   WarpBulk wb{};
   if (PC_DIRECT_BULK && !a.sys) warp_bulk_init(wb, smem);
-  for (int j = 0; j < P - 1; ++j)  // every peer has posted ready-to-receive
-    if (!warp_wait(a.rtr + j, e, a.err, a.timeout_ms, -1, a.sys)) return;
+  // every peer has posted ready-to-receive (all P-1 words polled at once)
+  if (!warp_wait_all(a.rtr, P - 1, e, a.err, a.timeout_ms, a.sys)) return;
   const uint32_t target = e * (uint32_t)(P - 1);
   for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
     int step[kMaxActive];
@@ -832,9 +860,7 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
   const bool bc = a.coll == PC_COLL_BCAST, root = bc && r == a.root;
   // writers into peers' buffers need every peer's ready-to-receive
   // (allgather pushes; the broadcast is pulled by the receivers themselves)
-  if (P > 1 && ag)
-    for (int j = 0; j < P - 1; ++j)
-      if (!warp_wait(a.rtr + j, e, a.err, a.timeout_ms, -1, a.sys)) return;
+  if (P > 1 && ag && !warp_wait_all(a.rtr, P - 1, e, a.err, a.timeout_ms, a.sys)) return;
   const uint32_t target = e * (uint32_t)(P - 1);
   for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
     int step[kMaxActive];

@@ -1391,6 +1391,51 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
   return 0;
 }
 
+// Start + Pbuf_prepare (+ Pready of every partition) of n already-exchanged
+// requests of one GPU in ONE kernel (the small-message epoch: one launch
+// instead of three; CUDA-graph capturable).
+int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream) {
+  if (n < 1 || !reqs || n > kMaxPreadyAll) return PC_ERR_ARG;
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    if (!q) return PC_ERR_ARG;
+    if (q->active) return PC_ERR_STATE;
+    if (!q->exchanged) return PC_ERR_STATE;
+    if (!q->matched) return PC_ERR_MATCH;
+    if (pready && q->kind != PC_KIND_PALLREDUCE) return PC_ERR_ARG;
+    if (q->comm->device != ((Request *)reqs[0])->comm->device || q->comm->dry != ((Request *)reqs[0])->comm->dry)
+      return PC_ERR_ARG;
+  }
+  const bool dry = ((Request *)reqs[0])->comm->dry;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (!dry) PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+  EpochAllArgs a{};
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
+    q->epoch++;
+    q->active = true;
+    q->engine_launched = false;
+    q->engine_registered = false;
+    q->prepared_this_epoch = true;
+    q->user_stream = (cudaStream_t)stream;
+    if (dry) continue;
+    a.epoch[a.n++] = q->ctrl + q->L.epoch;
+    for (auto &t : q->rtr_targets) {
+      if (a.nrtr == kMaxCtl) return PC_ERR_UNSUPPORTED;
+      a.rtr_dst[a.nrtr] = t.first + q->L.rtr + t.second;
+      a.rtr_epoch[a.nrtr] = q->ctrl + q->L.epoch;
+      a.rtr_sys[a.nrtr] = q->sys_scope;
+      ++a.nrtr;
+    }
+    if (pready) fill_prequest(q, &a.q[i]);
+  }
+  if (dry) return 0;
+  a.pready = pready ? 1 : 0;
+  PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
+  return launch_epoch_all(a, (cudaStream_t)stream);
+}
+
 // MPI_Startall: one device kernel advances the epochs of all n requests.
 int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream) {
   if (n < 0 || (n > 0 && !reqs)) return PC_ERR_ARG;

@@ -206,6 +206,32 @@ __global__ void pready_all_kernel(PreadyAllArgs a) {
   }
 }
 
+// One block: (1) every request's epoch e <- e + 1, (2) every ready-to-receive
+// write of the new epoch into the producers' RTR words, (3) optionally the
+// user's Pready (S_0) of every partition of every allreduce-kind request.
+// Barriers order the phases (all in one block, so CTA-scope visibility).
+__global__ void __launch_bounds__(1024) epoch_all_kernel(EpochAllArgs a) {
+  const int t = threadIdx.x;
+  if (t < a.n) a.epoch[t][0] = a.epoch[t][0] + 1;
+  __syncthreads();
+  if (t < a.nrtr) {
+    const uint32_t e = *(const volatile uint32_t *)a.rtr_epoch[t];
+    if (a.rtr_sys[t])
+      st_release_sys(a.rtr_dst[t], e);
+    else
+      st_release_gpu(a.rtr_dst[t], e);
+  }
+  if (!a.pready) return;
+  __syncthreads();
+  const int gw = t >> 5, W = blockDim.x >> 5;
+  int base = 0;
+  for (int k = 0; k < a.n; ++k) {
+    const int np = a.q[k].partitions;
+    for (int j = ((gw - base) % W + W) % W; j < np; j += W) pc_pready_warp(j, a.q[k]);
+    base += np;
+  }
+}
+
 __global__ void pready_range_kernel(pc_prequest_t q, int lo, int hi) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int W = (gridDim.x * blockDim.x) >> 5;
@@ -388,6 +414,13 @@ int launch_pready_all(const PreadyAllArgs &a, cudaStream_t s) {
   if (blocks > 148) blocks = 148;
   if (blocks < 1) blocks = 1;
   pready_all_kernel<<<blocks, 256, 0, s>>>(a);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_epoch_all(const EpochAllArgs &a, cudaStream_t s) {
+  epoch_all_kernel<<<1, 1024, 0, s>>>(a);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;

@@ -405,6 +405,17 @@ struct PreadyAllArgs {
   pc_prequest_t q[kMaxPreadyAll];
 };
 int launch_pready_all(const PreadyAllArgs &a, cudaStream_t s);
+// pc_epoch_all: Start + ready-to-receive (+ Pready of every partition of
+// allreduce-kind requests) for n requests in ONE single-block kernel.
+struct EpochAllArgs {
+  int n, nrtr, pready;
+  uint32_t *epoch[kMaxPreadyAll];
+  uint32_t *rtr_dst[kMaxCtl];
+  const uint32_t *rtr_epoch[kMaxCtl];
+  int rtr_sys[kMaxCtl];
+  pc_prequest_t q[kMaxPreadyAll];
+};
+int launch_epoch_all(const EpochAllArgs &a, cudaStream_t s);
 int engine_occupancy_ctas_per_sm(int *ctas);
 int direct_occupancy_ctas_per_sm(int *ctas);
 uint64_t launch_count();

@@ -307,6 +307,12 @@ def startall(reqs, stream=None):
     check(_lib.pc().pc_startall(len(reqs), _handles(reqs), _stream(stream)), "pc_startall")
 
 
+def epoch_all(reqs, pready: bool = False, stream=None):
+    """pc_epoch_all: Start + Pbuf_prepare (+ Pready of every partition of
+    allreduce-kind requests) of already-exchanged requests in ONE kernel."""
+    check(_lib.pc().pc_epoch_all(len(reqs), _handles(reqs), 1 if pready else 0, _stream(stream)), "pc_epoch_all")
+
+
 def pbuf_prepare_all(reqs, stream=None):
     """Ready-to-receive of already-exchanged requests in one kernel."""
     check(_lib.pc().pc_pbuf_prepare_all(len(reqs), _handles(reqs), _stream(stream)), "pc_pbuf_prepare_all")

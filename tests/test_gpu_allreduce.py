@@ -368,3 +368,53 @@ def test_c5_matrix_empty_and_short_chunks(algo, Ps, Np, L):
             ref, _, _ = oracle.pallreduce(x, Np, oalgo)
             for r in range(P):
                 assert (y[r].view(np.uint32) == ref[r].view(np.uint32)).all(), (P, r)
+
+
+@pytest.mark.parametrize("algo,P", [(pc.ALGO_RING, 4), (pc.ALGO_RD, 8), (pc.ALGO_DIRECT, 8), (pc.ALGO_DIRECT, 3)])
+@pytest.mark.parametrize("graph", [False, True])
+def test_epoch_all_single_control_kernel(algo, P, graph):
+    """pc_epoch_all (Start + Pbuf_prepare + Pready of every partition in one
+    kernel) drives correct epochs, eagerly and replayed from a CUDA graph:
+    fp32 bit-exact vs the schedule's oracle fold every epoch."""
+    Np, L = 5, 999
+    oalgo = {pc.ALGO_RING: oracle.RING, pc.ALGO_RD: oracle.RD, pc.ALGO_DIRECT: oracle.DIRECT}[algo]
+    with comms(P) as cs:
+        st = torch.cuda.Stream()
+        send = [torch.zeros(Np * L, device="cuda") for _ in range(P)]
+        recv = [torch.zeros(Np * L, device="cuda") for _ in range(P)]
+        reqs = [pc.pallreduce_init(send[r], recv[r], Np, L, pc.FLOAT32, pc.SUM, algo, cs[r]) for r in range(P)]
+        for q in reqs:
+            q.start(st)
+        first_prepare([[q] for q in reqs], [st] * P)
+        for q in reqs:
+            q.pready_range(0, Np - 1, st)
+        for q in reqs:
+            q.wait_on_stream(st)
+        torch.cuda.synchronize()
+
+        def step():
+            pc.epoch_all(reqs, pready=True, stream=st)
+            for q in reqs:
+                q.wait_on_stream(st)
+
+        g = None
+        if graph:
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=st):
+                step()
+        for e in range(4):
+            x = np.stack([synth.normal_f32(SEED + 90, r, e, Np * L) for r in range(P)])
+            for r in range(P):
+                send[r].copy_(torch.from_numpy(x[r]))
+            torch.cuda.synchronize()
+            if graph:
+                g.replay()
+            else:
+                step()
+            torch.cuda.synchronize()
+            ref, _, _ = oracle.pallreduce(x, Np, oalgo)
+            for r in range(P):
+                assert (recv[r].cpu().numpy().view(np.uint32) == ref[r].view(np.uint32)).all(), (e, r)
+        for q in reqs:
+            assert q.error() == (0, 0)
+            q.free()

@@ -42,10 +42,13 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
             for q in reqs:
                 q.start(st)
             pc.run_ranks([(lambda q=q: q.pbuf_prepare(st)) for q in reqs])
-        else:
+            pc.preadyall(reqs, st)  # S_0: the user's Pready of every partition, one kernel
+        elif os.environ.get("PC_SWEEP_SEPARATE_CTL"):
             pc.startall(reqs, st)  # one kernel for every rank's epoch
             pc.pbuf_prepare_all(reqs, st)  # one kernel for every RTR
-        pc.preadyall(reqs, st)  # S_0: the user's Pready of every partition, one kernel
+            pc.preadyall(reqs, st)
+        else:  # Start + RTR + S_0 Pready of every rank in ONE kernel
+            pc.epoch_all(reqs, pready=True, stream=st)
         for q in reqs:
             q.wait_on_stream(st)
 
