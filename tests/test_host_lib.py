@@ -253,3 +253,38 @@ def test_dry_auto_schedule_policy(P, nbytes, want):
     for c in cs:
         c.destroy()
     g.destroy()
+
+
+def test_dry_epoch_all_state_rules():
+    """pc_epoch_all bookkeeping (no device): needs exchanged, inactive
+    requests; Pready of every partition only for allreduce-kind requests;
+    at most 16 requests."""
+    g, cs = _dry(2)
+    ar = [pc.pallreduce_init(0, 0, 2, 64, pc.FLOAT32, pc.SUM, pc.ALGO_RING, c) for c in cs]
+    assert _try(lambda: pc.epoch_all(ar, pready=True)) == pc.ERR_STATE  # not exchanged yet
+    for q in ar:
+        q.start()
+    pc.run_ranks([lambda q=q: q.pbuf_prepare() for q in ar])
+    assert _try(lambda: pc.epoch_all(ar, pready=True)) == pc.ERR_STATE  # still active
+    for q in ar:
+        q.wait()
+    for _ in range(3):
+        pc.epoch_all(ar, pready=True)
+        for q in ar:
+            q.wait()
+    snd = pc.psend_init(0x1000, 4, 8, pc.FLOAT32, 1, 1, cs[0])
+    rcv = pc.precv_init(0x2000, 4, 8, pc.FLOAT32, 0, 1, cs[1])
+    snd.start()
+    rcv.start()
+    pc.run_ranks([lambda: snd.pbuf_prepare(), lambda: rcv.pbuf_prepare()])
+    snd.wait()
+    rcv.wait()
+    assert _try(lambda: pc.epoch_all([snd, rcv], pready=True)) == pc.ERR_ARG  # p2p: no library-side Pready
+    pc.epoch_all([snd, rcv], pready=False)
+    snd.wait()
+    rcv.wait()
+    for q in ar + [snd, rcv]:
+        q.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
