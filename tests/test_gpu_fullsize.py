@@ -1,6 +1,7 @@
 """GPU parity at BASELINE sizes, in the launch configuration bench.py times
-(8 virtual ranks on one B200, 256 MiB fp32 per rank, 64 partitions, ring,
-default slicing, one shared stream): sampled outputs are checked bit-exactly
+(8 virtual ranks on one B200, 256 MiB fp32 per rank, 64 partitions, ring /
+DIRECT / RD, default slicing, one shared stream, pc_epoch_all after the first
+epoch): sampled outputs are checked bit-exactly
 against the oracle's closed-form ring fold computed element by element from
 regenerated inputs, plus the R16 fp64 bound; RD at 64 MiB likewise; int32 at
 64 MiB on every element against numpy's exact sum."""
@@ -29,15 +30,14 @@ def run_bench_shape(P, S, Np, algo, gen_rank, dtype=torch.float32, steps=2):
         reqs = [pc.pallreduce_init(send[r], recv[r], Np, count, dt, pc.SUM, algo, cs[r]) for r in range(P)]
         torch.cuda.synchronize()
         for e in range(steps):  # several epochs, exactly as bench.py's step()
-            for q in reqs:
-                q.start(st)
             if e == 0:
-                first_prepare([[q] for q in reqs], [st] * P)
-            else:
                 for q in reqs:
-                    q.pbuf_prepare(st)
-            for q in reqs:
-                q.pready_range(0, Np - 1, st)
+                    q.start(st)
+                first_prepare([[q] for q in reqs], [st] * P)
+                for q in reqs:
+                    q.pready_range(0, Np - 1, st)
+            else:  # bench.py: Start + RTR + Pready of every rank in one kernel
+                pc.epoch_all(reqs, pready=True, stream=st)
             for q in reqs:
                 q.wait_on_stream(st)
         torch.cuda.synchronize()
@@ -74,9 +74,10 @@ def test_fullsize_sampled_fp32(algo, S):
         assert torch.equal(recv[r], recv[0])
 
 
-def test_fullsize_int32_every_element():
+@pytest.mark.parametrize("algo", [pc.ALGO_RING, pc.ALGO_DIRECT])
+def test_fullsize_int32_every_element(algo):
     P, Np, S = 8, 64, 64 << 20
-    recv, L, _ = run_bench_shape(P, S, Np, pc.ALGO_RING, lambda r, n: synth.int32_full(SEED, r, 1, n),
+    recv, L, _ = run_bench_shape(P, S, Np, algo, lambda r, n: synth.int32_full(SEED, r, 1, n),
                                  dtype=torch.int32)
     n = L * Np
     acc = np.zeros(n, dtype=np.int64)
