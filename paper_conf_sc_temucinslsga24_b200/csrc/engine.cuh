@@ -1040,6 +1040,7 @@ struct EngineLaunch {
   static int coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s);
   static int occupancy(int *ctas);
   static int occupancy_direct(int *ctas);
+  static int preload();  // load every engine kernel now (lazy module loading, see kernels.cu)
 };
 
 }  // namespace pc

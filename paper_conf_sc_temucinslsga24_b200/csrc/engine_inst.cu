@@ -114,6 +114,20 @@ int EngineLaunch<DT, OP>::coll_group(const CollGroupArgs &h, int blocks, cudaStr
   return 0;
 }
 
+template <int DT, int OP>
+int EngineLaunch<DT, OP>::preload() {
+  cudaFuncAttributes fa;
+  PC_CUDA(cudaFuncGetAttributes(&fa, ring_engine<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, rd_engine<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, ring_engine_group<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, rd_engine_group<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP>));
+  return 0;
+}
+
 template struct EngineLaunch<PC_DT, PC_OP>;
 
 }  // namespace pc

@@ -122,27 +122,39 @@ static void progress_main(Comm *c) {
     {
       std::lock_guard<std::mutex> lk(pe.mu);
       for (Request *q : pe.reqs) {
-        for (int t = 0; t < q->ntransport; ++t) {
+        // one sweep over the ready flags; consecutive transport partitions
+        // that became ready in the same epoch move as ONE copy and are
+        // signalled by ONE small kernel (arrival flags + sent words)
+        int t = 0;
+        while (t < q->ntransport) {
           const uint32_t v = __atomic_load_n(q->hready + t, __ATOMIC_ACQUIRE);
-          if (v == q->pe_done[t]) continue;
+          if (v == q->pe_done[t]) {
+            ++t;
+            continue;
+          }
+          int t1 = t + 1;
+          while (t1 < q->ntransport && __atomic_load_n(q->hready + t1, __ATOMIC_ACQUIRE) == v &&
+                 q->pe_done[t1] != v)
+            ++t1;
           any = true;
-          q->pe_done[t] = v;
+          for (int k = t; k < t1; ++k) q->pe_done[k] = v;
           int rc = 0;
           if ((int32_t)(v - q->pe_rtr_epoch) > 0) {  // first partition of epoch v: receiver ready?
             rc = stream_wait_geq_u32(c, pe.stream, q->ctrl + q->L.rtr, v, q->sys_scope != 0);
             q->pe_rtr_epoch = v;
           }
-          const int rem = q->partitions - t * q->agg;
-          const uint64_t len = (uint64_t)(rem < q->agg ? rem : q->agg) * q->part_bytes;
           const uint64_t off = (uint64_t)t * q->agg * q->part_bytes;
-          if (!rc && len)
-            rc = cudaMemcpyAsync(q->peer_buf + off, (const uint8_t *)q->sbuf + off, len, cudaMemcpyDeviceToDevice,
-                                 pe.stream) == cudaSuccess
+          const uint64_t end = std::min<uint64_t>((uint64_t)t1 * q->agg, (uint64_t)q->partitions) * q->part_bytes;
+          if (!rc && end > off)
+            rc = cudaMemcpyAsync(q->peer_buf + off, (const uint8_t *)q->sbuf + off, end - off,
+                                 cudaMemcpyDeviceToDevice, pe.stream) == cudaSuccess
                      ? 0
                      : PC_ERR_CUDA;
-          if (!rc) rc = stream_write_u32(c, pe.stream, q->peer_ctrl + q->peer_flags_off + t, v);
-          if (!rc) rc = stream_write_u32(c, pe.stream, q->ctrl + q->L.sent + t, v);
+          if (!rc)
+            rc = launch_pe_signal(q->peer_ctrl + q->peer_flags_off + t, q->ctrl + q->L.sent + t, t1 - t, v,
+                                  q->sys_scope != 0, pe.stream);
           if (rc) pe.err.store(rc);
+          t = t1;
         }
       }
     }
@@ -165,6 +177,7 @@ static int progress_register(Request *q) {
     PC_CUDA(cudaHostGetDevicePointer((void **)&q->hready_dev, q->hready, 0));
     q->pe_done.assign((size_t)q->ntransport, 0u);
   }
+  if (int rc = pe_kernels_preload()) return rc;  // lazy loading must not happen under spinning kernels
   std::lock_guard<std::mutex> lk(pe.mu);
   if (!pe.started) {
     int lo = 0, hi = 0;
@@ -1071,7 +1084,12 @@ int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void
     memcpy(me.uuid, &prop.uuid, 16);
     me.sms = prop.multiProcessorCount;
     int occ = 0;
-    int rc = engine_occupancy_ctas_per_sm(&occ);
+    int rc = kernels_preload();  // no lazy load may later stall behind spinning kernels
+    if (rc) {
+      delete c;
+      return rc;
+    }
+    rc = engine_occupancy_ctas_per_sm(&occ);
     if (rc) {
       delete c;
       return rc;

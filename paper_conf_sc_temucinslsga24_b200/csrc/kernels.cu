@@ -400,6 +400,61 @@ int launch_wait_value(const uint32_t *addr, uint32_t value, cudaStream_t s, bool
   return 0;
 }
 
+// Progression engine (PC_COPY_HOST): after the stream-ordered copy of
+// transport partitions [t, t+n), publish their arrival at the receiver and
+// their completion at the sender.
+__global__ void pe_signal_kernel(uint32_t *peer_flags, uint32_t *sent, int n, uint32_t v, int sys) {
+  for (int i = threadIdx.x; i < n; i += blockDim.x) {
+    if (sys)
+      st_release_sys(peer_flags + i, v);
+    else
+      st_release_gpu(peer_flags + i, v);
+    st_release_gpu(sent + i, v);
+  }
+}
+
+// With lazy module loading (the CUDA 12 default) the FIRST launch of a kernel
+// may wait for the device to go idle while it loads — fatal when that launch
+// comes from the progress thread while the user's wait kernels spin on the
+// very flags it is about to write.  Load the progress thread's kernels up
+// front (pc_prequest_create, before any epoch runs).
+// Every library kernel, loaded at pc_comm_create: no first launch may then
+// stall behind kernels that spin on the work it is about to do (engines and
+// waits are launched while producers and waits of other ranks run).
+int kernels_preload() {
+  cudaFuncAttributes fa;
+  PC_CUDA(cudaFuncGetAttributes(&fa, p2p_engine));
+  PC_CUDA(cudaFuncGetAttributes(&fa, wait_words_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, recv_wait_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, parrived_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, set_word_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, epoch_bump_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, ctl_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, rtr_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, pready_all_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, epoch_all_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, pready_range_kernel));
+  if (int rc = pe_kernels_preload()) return rc;
+  for (int dt : {PC_INT32, PC_FLOAT32, PC_FLOAT64, PC_BF16})
+    for (int op : {PC_OP_SUM, PC_OP_MAX, PC_OP_MIN})
+      if (int rc = dispatch(dt, op, [&](auto E) { return decltype(E)::preload(); })) return rc;
+  return 0;
+}
+
+int pe_kernels_preload() {
+  cudaFuncAttributes fa;
+  PC_CUDA(cudaFuncGetAttributes(&fa, pe_signal_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, wait_value_kernel));
+  return 0;
+}
+
+int launch_pe_signal(uint32_t *peer_flags, uint32_t *sent, int n, uint32_t v, bool sys, cudaStream_t s) {
+  pe_signal_kernel<<<1, 256, 0, s>>>(peer_flags, sent, n, v, sys ? 1 : 0);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s) {
   set_word_kernel<<<1, 1, 0, s>>>(addr, value);
   g_launches++;

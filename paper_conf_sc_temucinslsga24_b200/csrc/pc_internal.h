@@ -397,6 +397,9 @@ int launch_recv_wait(const pc_prequest_t &q, int32_t *pending, cudaStream_t s);
 // out[0] = pc_parrived(q, partition) on the device (LL receive requests)
 int launch_parrived(const pc_prequest_t &q, int partition, int32_t *out, cudaStream_t s);
 int launch_set_word(uint32_t *addr, uint32_t value, cudaStream_t s);
+int launch_pe_signal(uint32_t *peer_flags, uint32_t *sent, int n, uint32_t v, bool sys, cudaStream_t s);
+int pe_kernels_preload();
+int kernels_preload();
 int launch_wait_value(const uint32_t *addr, uint32_t value, cudaStream_t s, bool sys, uint32_t tmo_ms);
 int launch_pready_range(pc_prequest_t q, int lo, int hi, cudaStream_t s);
 constexpr int kMaxPreadyAll = 16;
