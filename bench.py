@@ -402,7 +402,7 @@ def jacobi_bench(pc, apps, torch, args):
     N, K = args.jacobi_n, args.jacobi_iters
     hbm_peak, _ = peaks()
     res = {}
-    for Py, Px in ((1, 1), (4, 2)):
+    for Py, Px in ((1, 1), (2, 1), (2, 2), (4, 2), (8, 1)):
         P = Py * Px
         g, cs = pc.local_comms(P, 0)
         st = torch.cuda.Stream()

@@ -223,12 +223,15 @@ __global__ void __launch_bounds__(1024) epoch_all_kernel(EpochAllArgs a) {
   }
   if (!a.pready) return;
   __syncthreads();
-  const int gw = t >> 5, W = blockDim.x >> 5;
-  int base = 0;
+  // S_0 of every partition: ready[u] = e.  No fences: the user's data was
+  // written by kernels earlier in stream order, and the only reader of
+  // ready[] is this rank's engine, launched after this kernel in stream order
+  // (kernel boundaries order both), so plain stores spread over the block
+  // replace one release per partition.
   for (int k = 0; k < a.n; ++k) {
-    const int np = a.q[k].partitions;
-    for (int j = ((gw - base) % W + W) % W; j < np; j += W) pc_pready_warp(j, a.q[k]);
-    base += np;
+    const uint32_t e = *(const volatile uint32_t *)a.epoch[k];
+    uint32_t *ready = a.q[k].ready;
+    for (int j = t; j < a.q[k].partitions; j += blockDim.x) st_relaxed_gpu(ready + j, e);
   }
 }
 
