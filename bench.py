@@ -311,10 +311,7 @@ def c1_bench(pc, apps, torch, epochs=200):
     torch.cuda.synchronize()
 
     def epoch():  # Listing 2: Start, Pbuf_prepare, kernel (Pready inside), Wait
-        snd.start(st)
-        rcv.start(st)
-        rcv.pbuf_prepare(st)
-        snd.pbuf_prepare(st)
+        pc.epoch_all([snd, rcv], pready=False, stream=st)  # Startall + Pbuf_prepare of both, one kernel
         apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
         snd.wait_on_stream(st)
         rcv.wait_on_stream(st)
@@ -368,10 +365,7 @@ def c1_bench(pc, apps, torch, epochs=200):
     st.synchronize()
     t0 = _t.perf_counter()
     for _ in range(epochs):
-        snd2.start(st)
-        rcv2.start(st)
-        rcv2.pbuf_prepare(st)
-        snd2.pbuf_prepare(st)
+        pc.epoch_all([snd2, rcv2], pready=False, stream=st)  # same control path as the Kernel Copy epochs
         apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq2, st)
         snd2.wait_on_stream(st)
         rcv2.wait_on_stream(st)
