@@ -106,9 +106,9 @@ def test_thread_granularity_warp_aggregation_large():
 
 
 def test_many_epochs_tagged_bytes():
-    """>= 200 back-to-back epochs of epoch-tagged bytes with a permuted Pready
+    """1000 back-to-back epochs of epoch-tagged bytes with a permuted Pready
     order: every epoch's bytes arrive intact and exactly once."""
-    partitions, pbytes, E = 16, 4096, 200
+    partitions, pbytes, E = 16, 4096, 1000
     with comms(2) as cs:
         s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
         src = torch.empty(partitions * pbytes, dtype=torch.uint8, device="cuda")
