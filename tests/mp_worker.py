@@ -35,6 +35,16 @@ for name, algo in (("ring", pc.ALGO_RING), ("rd", pc.ALGO_RD), ("direct", pc.ALG
     st.synchronize()
     assert q.error() == (0, 0), q.error()
     res[name] = recv.cpu().numpy()
+    # later epochs as bench.py's N > 1 step runs them: Start + RTR + Pready in
+    # one pc_epoch_all kernel (RTR words of the other PROCESS, via CUDA IPC)
+    for e in range(3):
+        recv.zero_()
+        st.wait_stream(torch.cuda.current_stream())
+        pc.epoch_all([q], pready=True, stream=st)
+        q.wait_on_stream(st)
+        st.synchronize()
+        assert q.error() == (0, 0), q.error()
+        res[name + "_epoch_all%d" % e] = recv.cpu().numpy()
     q.free()
 # p2p 0 -> 1 with block-granularity Pready from the producer kernel
 n = 2048 * 8

@@ -29,6 +29,9 @@ def test_two_processes_ipc(tmp_path):
         ref, _, _ = oracle.pallreduce(x, Np, algo)
         for r in range(2):
             np.testing.assert_array_equal(res[r][name].view(np.uint32), ref[r].view(np.uint32))
+            for e in range(3):  # pc_epoch_all epochs across processes
+                np.testing.assert_array_equal(res[r][f"{name}_epoch_all{e}"].view(np.uint32),
+                                              ref[r].view(np.uint32))
     n = 2048 * 8
     a = synth.uniform_f32(synth.BASE_SEED, 0, 0, n)
     b = synth.uniform_f32(synth.BASE_SEED, 0, 1, n)
