@@ -1438,15 +1438,19 @@ int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream) {
     q->prepared_this_epoch = true;
     q->user_stream = (cudaStream_t)stream;
     if (dry) continue;
-    a.epoch[a.n++] = q->ctrl + q->L.epoch;
+    const int k = a.n++;
+    a.epoch[k] = q->ctrl + q->L.epoch;
     for (auto &t : q->rtr_targets) {
       if (a.nrtr == kMaxCtl) return PC_ERR_UNSUPPORTED;
       a.rtr_dst[a.nrtr] = t.first + q->L.rtr + t.second;
-      a.rtr_epoch[a.nrtr] = q->ctrl + q->L.epoch;
-      a.rtr_sys[a.nrtr] = q->sys_scope;
+      a.rtr_req[a.nrtr] = (uint8_t)k;
+      if (q->sys_scope) a.rtr_sysmask |= 1ull << a.nrtr;
       ++a.nrtr;
     }
-    if (pready) fill_prequest(q, &a.q[i]);
+    if (pready) {
+      a.ready[k] = q->ctrl + q->L.ready;
+      a.partitions[k] = q->partitions;
+    }
   }
   if (dry) return 0;
   a.pready = pready ? 1 : 0;

@@ -215,8 +215,8 @@ __global__ void __launch_bounds__(1024) epoch_all_kernel(EpochAllArgs a) {
   if (t < a.n) a.epoch[t][0] = a.epoch[t][0] + 1;
   __syncthreads();
   if (t < a.nrtr) {
-    const uint32_t e = *(const volatile uint32_t *)a.rtr_epoch[t];
-    if (a.rtr_sys[t])
+    const uint32_t e = *(const volatile uint32_t *)a.epoch[a.rtr_req[t]];
+    if ((a.rtr_sysmask >> t) & 1)
       st_release_sys(a.rtr_dst[t], e);
     else
       st_release_gpu(a.rtr_dst[t], e);
@@ -230,8 +230,8 @@ __global__ void __launch_bounds__(1024) epoch_all_kernel(EpochAllArgs a) {
   // replace one release per partition.
   for (int k = 0; k < a.n; ++k) {
     const uint32_t e = *(const volatile uint32_t *)a.epoch[k];
-    uint32_t *ready = a.q[k].ready;
-    for (int j = t; j < a.q[k].partitions; j += blockDim.x) st_relaxed_gpu(ready + j, e);
+    uint32_t *ready = a.ready[k];
+    for (int j = t; j < a.partitions[k]; j += blockDim.x) st_relaxed_gpu(ready + j, e);
   }
 }
 

@@ -410,14 +410,19 @@ struct PreadyAllArgs {
 int launch_pready_all(const PreadyAllArgs &a, cudaStream_t s);
 // pc_epoch_all: Start + ready-to-receive (+ Pready of every partition of
 // allreduce-kind requests) for n requests in ONE single-block kernel.
+// Kept under 1 KB of kernel parameters (a launch's parameter bytes travel in
+// the push buffer: the earlier layout, 16 whole pc_prequest_t, was 4.6 KB and
+// made this one launch slower than pc_startall + pc_pbuf_prepare_all).
 struct EpochAllArgs {
   int n, nrtr, pready;
+  uint64_t rtr_sysmask;                 // bit k: RTR k is a system-scope release
   uint32_t *epoch[kMaxPreadyAll];
   uint32_t *rtr_dst[kMaxCtl];
-  const uint32_t *rtr_epoch[kMaxCtl];
-  int rtr_sys[kMaxCtl];
-  pc_prequest_t q[kMaxPreadyAll];
+  uint8_t rtr_req[kMaxCtl];             // RTR k carries the epoch of request rtr_req[k]
+  uint32_t *ready[kMaxPreadyAll];       // pready: allreduce S_0 ready words [partitions]
+  int partitions[kMaxPreadyAll];
 };
+static_assert(sizeof(EpochAllArgs) <= 1024, "EpochAllArgs: keep kernel parameters small");
 int launch_epoch_all(const EpochAllArgs &a, cudaStream_t s);
 int engine_occupancy_ctas_per_sm(int *ctas);
 int direct_occupancy_ctas_per_sm(int *ctas);

@@ -53,7 +53,27 @@ def ctl_only():
     pc.preadyall([snd], st)
     snd.wait_on_stream(st); rcv.wait_on_stream(st)
 
-for name, f in [("full epoch (startall/prepare_all)", full_batched), ("full epoch (start/pbuf_prepare memops)", full_memops),
+st2 = torch.cuda.Stream()
+ev_a, ev_b = torch.cuda.Event(), torch.cuda.Event()
+
+def epoch_all_serial():  # bench.py c1 epoch: one stream, both waits serialised
+    pc.epoch_all([snd, rcv], pready=False, stream=st)
+    apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
+    snd.wait_on_stream(st); rcv.wait_on_stream(st)
+
+def epoch_all_2stream():  # the receiver's wait on its own stream, as on its own GPU
+    pc.epoch_all([snd, rcv], pready=False, stream=st)
+    ev_a.record(st)
+    st2.wait_event(ev_a)
+    rcv.wait_on_stream(st2)
+    ev_b.record(st2)
+    apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
+    snd.wait_on_stream(st)
+    st.wait_event(ev_b)
+
+for name, f in [("epoch_all + vecadd + 2 waits (bench c1)", epoch_all_serial),
+                ("epoch_all; recv wait on 2nd stream", epoch_all_2stream),
+                ("full epoch (startall/prepare_all)", full_batched), ("full epoch (start/pbuf_prepare memops)", full_memops),
                 ("vecadd only", vec_only), ("vecadd + copy (device only)", trad_dev),
                 ("control only (startall, prepare_all, preadyall, waits)", ctl_only)]:
     print(f"{name:55s} {timeit(f):8.2f} us")
