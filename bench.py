@@ -313,8 +313,7 @@ def c1_bench(pc, apps, torch, epochs=200):
     def epoch():  # Listing 2: Start, Pbuf_prepare, kernel (Pready inside), Wait
         pc.epoch_all([snd, rcv], pready=False, stream=st)  # Startall + Pbuf_prepare of both, one kernel
         apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
-        snd.wait_on_stream(st)
-        rcv.wait_on_stream(st)
+        pc.waitall_on_stream([snd, rcv], st)  # both ranks' waits in one kernel
 
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(st)
@@ -367,8 +366,7 @@ def c1_bench(pc, apps, torch, epochs=200):
     for _ in range(epochs):
         pc.epoch_all([snd2, rcv2], pready=False, stream=st)  # same control path as the Kernel Copy epochs
         apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq2, st)
-        snd2.wait_on_stream(st)
-        rcv2.wait_on_stream(st)
+        pc.waitall_on_stream([snd2, rcv2], st)
         st.synchronize()
     pe_host_us = (_t.perf_counter() - t0) / epochs * 1e6
     ok = ok and bool(torch.equal(R2, Cb)) and snd2.error()[0] == 0 and rcv2.error()[0] == 0

@@ -215,6 +215,16 @@ int pc_parrived(pc_request_t req, int partition, int *flag);
 int pc_test(pc_request_t req, int *flag);
 int pc_wait(pc_request_t req);
 int pc_wait_on_stream(pc_request_t req, pc_stream_t stream);
+/* MPI_Waitall (MPI-4 §3.7.5; Listing 2 waits on each request), stream
+ * ordered: pc_wait_on_stream of n requests of one GPU, with the waits of the
+ * point-to-point requests (engine-less sends and all receives) fused into ONE
+ * kernel per group of 4 — one launch where n pc_wait_on_stream calls take n.
+ * Requests moved by library engines (allreduce, ENGINE-copy sends) take
+ * pc_wait_on_stream's path (the engine launch is the wait).  Inactive requests
+ * are skipped.  PC_ERR_ARG for n < 0 or a null array / entry, PC_ERR_STATE as
+ * pc_wait_on_stream; on an error no request of the call was marked complete
+ * unless its own wait was already enqueued. */
+int pc_waitall_on_stream(int n, pc_request_t *reqs, pc_stream_t stream);
 /* Host Pready bindings (MPI_Pready / MPI_Pready_range): enqueue a tiny kernel
  * on `stream` that marks partitions [lo, hi] ready. */
 int pc_pready(int partition, pc_request_t req, pc_stream_t stream);

@@ -57,6 +57,7 @@ _PC_PROTOS = {
     "pc_test": (I32, [P, PI32]),
     "pc_wait": (I32, [P]),
     "pc_wait_on_stream": (I32, [P, P]),
+    "pc_waitall_on_stream": (I32, [I32, P, P]),
     "pc_pready": (I32, [I32, P, P]),
     "pc_pready_range": (I32, [I32, I32, P, P]),
     "pc_preadyall": (I32, [I32, P, P]),

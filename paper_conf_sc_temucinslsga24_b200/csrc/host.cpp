@@ -1670,6 +1670,45 @@ int pc_wait_on_stream(pc_request_t req, pc_stream_t stream) {
   return wait_common(q, (cudaStream_t)stream, false);
 }
 
+int pc_waitall_on_stream(int n, pc_request_t *reqs, pc_stream_t stream) {
+  if (n < 0 || (n > 0 && !reqs)) return PC_ERR_ARG;
+  for (int i = 0; i < n; ++i)
+    if (!reqs[i]) return PC_ERR_ARG;
+  cudaStream_t s = (cudaStream_t)stream;
+  // validate first (as wait_common), then enqueue
+  std::vector<Request *> fused;
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    if (!q->active || q->comm->dry) continue;
+    const bool engine = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->copy == 1);
+    if (engine) continue;
+    if (!q->exchanged || !q->matched) return PC_ERR_STATE;
+    if (q->kind == PC_KIND_PSEND && !q->has_preq) return PC_ERR_STATE;
+    if (!fused.empty() && q->comm->device != fused[0]->comm->device) return PC_ERR_ARG;
+    fused.push_back(q);
+  }
+  for (int i = 0; i < n; ++i) {  // engine-moved and dry requests: their own path
+    Request *q = (Request *)reqs[i];
+    if (std::find(fused.begin(), fused.end(), q) != fused.end()) continue;
+    if (int rc = wait_common(q, s, false)) return rc;
+  }
+  if (fused.empty()) return 0;
+  PC_CUDA(cudaSetDevice(fused[0]->comm->device));
+  for (size_t g0 = 0; g0 < fused.size(); g0 += kMaxWaitAll) {
+    WaitAllArgs a{};
+    a.block_start[0] = 0;
+    for (size_t k = g0; k < fused.size() && a.n < kMaxWaitAll; ++k) {
+      fill_prequest(fused[k], &a.q[a.n]);
+      const int nb = fused[k]->kind == PC_KIND_PSEND ? 1 : recv_wait_blocks(a.q[a.n]);
+      a.block_start[a.n + 1] = a.block_start[a.n] + nb;
+      ++a.n;
+    }
+    if (int rc = launch_wait_all(a, s)) return rc;
+    for (size_t k = g0; k < g0 + (size_t)a.n; ++k) fused[k]->active = false;
+  }
+  return 0;
+}
+
 static int read_words(Request *q, size_t off, size_t n, uint32_t *h) {
   PC_CUDA(cudaMemcpyAsync(h, q->ctrl + off, n * 4, cudaMemcpyDeviceToHost, q->side));
   PC_CUDA(cudaStreamSynchronize(q->side));

@@ -42,9 +42,9 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
   }
 }
 
-__global__ void wait_words_kernel(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul,
-                                  const uint32_t *layout, int partitions, int32_t *err, uint32_t tmo, int sys,
-                                  const uint32_t *rtr) {
+__device__ __forceinline__ void wait_words_body(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul,
+                                                const uint32_t *layout, int partitions, int32_t *err, uint32_t tmo,
+                                                int sys, const uint32_t *rtr) {
   __shared__ int s_n;
   const uint32_t target = *(const volatile uint32_t *)epoch * mul;
   // LL sender: its epoch completes only once the receiver posted ready-to-
@@ -77,6 +77,12 @@ __global__ void wait_words_kernel(const uint32_t *words, int n, const uint32_t *
   }
 }
 
+__global__ void wait_words_kernel(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul,
+                                  const uint32_t *layout, int partitions, int32_t *err, uint32_t tmo, int sys,
+                                  const uint32_t *rtr) {
+  wait_words_body(words, n, epoch, mul, layout, partitions, err, tmo, sys, rtr);
+}
+
 // Receive-side MPI_Wait / MPI_Test for a request whose sender may push LL
 // lines (PC_COPY_LL): the layout word tells which protocol the sender chose.
 // LL: every thread owns lines i = (p, j) of the grid-stride range, waits (or,
@@ -84,7 +90,8 @@ __global__ void wait_words_kernel(const uint32_t *words, int n, const uint32_t *
 // and unpacks its payload bytes into recvbuf.  Flags: block 0 waits on the
 // transport flags exactly as wait_words_kernel.  Test mode (pending != null):
 // no spinning; every line / flag not there yet adds 1 to *pending.
-__global__ void recv_wait_kernel(pc_prequest_t q, int32_t *pending) {
+// (block `bid` of the `nb` blocks serving this request)
+__device__ __forceinline__ void recv_wait_body(const pc_prequest_t &q, int32_t *pending, uint32_t bid, uint32_t nb) {
   __shared__ uint32_t s_g;
   const uint32_t e = *(const volatile uint32_t *)q.epoch;
   if (threadIdx.x == 0) {
@@ -103,7 +110,7 @@ __global__ void recv_wait_kernel(pc_prequest_t q, int32_t *pending) {
   __syncthreads();
   const uint32_t g = s_g;
   if (g == 0) {
-    if (pending && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(pending, 1);
+    if (pending && bid == 0 && threadIdx.x == 0) atomicAdd(pending, 1);
     return;
   }
   if (g & PC_LAYOUT_LL) {
@@ -111,7 +118,7 @@ __global__ void recv_wait_kernel(pc_prequest_t q, int32_t *pending) {
     const uint64_t nlines = (uint64_t)q.partitions * nl;
     const uint8_t *base = q.ll + (uint64_t)(e & 1) * nlines * 16ull;
     const uint64_t t0 = globaltimer();
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nlines; i += (uint64_t)gridDim.x * blockDim.x) {
+    for (uint64_t i = (uint64_t)bid * blockDim.x + threadIdx.x; i < nlines; i += (uint64_t)nb * blockDim.x) {
       ulonglong2 v = ld_ll(base + 16ull * i, q.sys_scope);
       uint32_t n = 0;
       while ((uint32_t)(v.x >> 32) != e || (uint32_t)(v.y >> 32) != e) {
@@ -137,7 +144,7 @@ __global__ void recv_wait_kernel(pc_prequest_t q, int32_t *pending) {
     }
     return;
   }
-  if (blockIdx.x != 0) return;
+  if (bid != 0) return;
   // equal partitionings: one flag per send transport partition (target e);
   // different ones (R30): one counter per receive partition (e * overlaps)
   const bool xp = (g & PC_LAYOUT_XP) != 0;
@@ -151,6 +158,24 @@ __global__ void recv_wait_kernel(pc_prequest_t q, int32_t *pending) {
     bool ok = q.sys_scope ? spin_geq<true>(q.flags + i, target, q.err, q.timeout_ms, i)
                           : spin_geq<false>(q.flags + i, target, q.err, q.timeout_ms, i);
     if (!ok) break;
+  }
+}
+
+__global__ void recv_wait_kernel(pc_prequest_t q, int32_t *pending) { recv_wait_body(q, pending, blockIdx.x, gridDim.x); }
+
+// pc_waitall_on_stream: request k's wait runs on its own block range (block
+// ranges are uniform per block, so the bodies' barriers are block-uniform).
+__global__ void wait_all_kernel(WaitAllArgs a) {
+  int k = 0;
+  while (k + 1 < a.n && (int)blockIdx.x >= a.block_start[k + 1]) ++k;
+  const pc_prequest_t &q = a.q[k];
+  const uint32_t bid = blockIdx.x - a.block_start[k], nb = a.block_start[k + 1] - a.block_start[k];
+  if (q.kind == PC_KIND_PSEND) {
+    if (bid == 0)
+      wait_words_body(q.sent, q.ntransport, q.epoch, 1, nullptr, q.partitions, q.err, q.timeout_ms, 0,
+                      q.copy == PC_COPY_LL ? q.rtr : nullptr);
+  } else {
+    recv_wait_body(q, nullptr, bid, nb);
   }
 }
 
@@ -342,7 +367,7 @@ int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint3
   return 0;
 }
 
-int launch_recv_wait(const pc_prequest_t &q, int32_t *pending, cudaStream_t s) {
+int recv_wait_blocks(const pc_prequest_t &q) {
   int blocks = 1;
   if (q.ll_lines) {
     const int64_t lines = (int64_t)q.partitions * q.ll_lines;
@@ -350,7 +375,18 @@ int launch_recv_wait(const pc_prequest_t &q, int32_t *pending, cudaStream_t s) {
     if (blocks > 4 * 148) blocks = 4 * 148;
     if (blocks < 1) blocks = 1;
   }
-  recv_wait_kernel<<<blocks, 256, 0, s>>>(q, pending);
+  return blocks;
+}
+
+int launch_wait_all(const WaitAllArgs &a, cudaStream_t s) {
+  wait_all_kernel<<<a.block_start[a.n], 256, 0, s>>>(a);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_recv_wait(const pc_prequest_t &q, int32_t *pending, cudaStream_t s) {
+  recv_wait_kernel<<<recv_wait_blocks(q), 256, 0, s>>>(q, pending);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -429,6 +465,7 @@ int kernels_preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, p2p_engine));
   PC_CUDA(cudaFuncGetAttributes(&fa, wait_words_kernel));
   PC_CUDA(cudaFuncGetAttributes(&fa, recv_wait_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, wait_all_kernel));
   PC_CUDA(cudaFuncGetAttributes(&fa, parrived_kernel));
   PC_CUDA(cudaFuncGetAttributes(&fa, set_word_kernel));
   PC_CUDA(cudaFuncGetAttributes(&fa, epoch_bump_kernel));

@@ -424,6 +424,16 @@ struct EpochAllArgs {
 };
 static_assert(sizeof(EpochAllArgs) <= 1024, "EpochAllArgs: keep kernel parameters small");
 int launch_epoch_all(const EpochAllArgs &a, cudaStream_t s);
+// pc_waitall_on_stream: the p2p waits of up to kMaxWaitAll requests in one
+// kernel; request k owns blocks [block_start[k], block_start[k+1]).
+constexpr int kMaxWaitAll = 4;
+struct WaitAllArgs {
+  int n;
+  int block_start[kMaxWaitAll + 1];
+  pc_prequest_t q[kMaxWaitAll];
+};
+int recv_wait_blocks(const pc_prequest_t &q);
+int launch_wait_all(const WaitAllArgs &a, cudaStream_t s);
 int engine_occupancy_ctas_per_sm(int *ctas);
 int direct_occupancy_ctas_per_sm(int *ctas);
 uint64_t launch_count();

@@ -302,6 +302,11 @@ def _handles(reqs):
     return arr
 
 
+def waitall_on_stream(reqs, stream=None):
+    """MPI_Waitall, stream-ordered: the p2p waits of all requests in one kernel."""
+    check(_lib.pc().pc_waitall_on_stream(len(reqs), _handles(reqs), _stream(stream)), "pc_waitall_on_stream")
+
+
 def startall(reqs, stream=None):
     """MPI_Startall: one kernel advances every request's epoch."""
     check(_lib.pc().pc_startall(len(reqs), _handles(reqs), _stream(stream)), "pc_startall")

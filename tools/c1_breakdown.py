@@ -61,6 +61,11 @@ def epoch_all_serial():  # bench.py c1 epoch: one stream, both waits serialised
     apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
     snd.wait_on_stream(st); rcv.wait_on_stream(st)
 
+def epoch_all_waitall():  # bench.py c1 epoch: both waits in one pc_waitall_on_stream kernel
+    pc.epoch_all([snd, rcv], pready=False, stream=st)
+    apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
+    pc.waitall_on_stream([snd, rcv], st)
+
 def epoch_all_2stream():  # the receiver's wait on its own stream, as on its own GPU
     pc.epoch_all([snd, rcv], pready=False, stream=st)
     ev_a.record(st)
@@ -71,7 +76,8 @@ def epoch_all_2stream():  # the receiver's wait on its own stream, as on its own
     snd.wait_on_stream(st)
     st.wait_event(ev_b)
 
-for name, f in [("epoch_all + vecadd + 2 waits (bench c1)", epoch_all_serial),
+for name, f in [("epoch_all + vecadd + 2 waits", epoch_all_serial),
+                ("epoch_all + vecadd + waitall (bench c1)", epoch_all_waitall),
                 ("epoch_all; recv wait on 2nd stream", epoch_all_2stream),
                 ("full epoch (startall/prepare_all)", full_batched), ("full epoch (start/pbuf_prepare memops)", full_memops),
                 ("vecadd only", vec_only), ("vecadd + copy (device only)", trad_dev),
