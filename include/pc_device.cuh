@@ -299,6 +299,14 @@ PC_DEVICE void publish(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, 
   }
 }
 
+/* The fence a contributor issues after its pushes, before publish().  With
+ * g > 1 at GPU scope the contribution's atom.acq_rel.gpu is itself the
+ * (cumulative) release of those pushes, so the fence is dropped; g = 1
+ * (publish stores the flag directly) and system scope keep it. */
+PC_DEVICE void fence_before_publish(const pc_prequest_t &q) {
+  if (q.agg == 1 || q.sys_scope) fence_scope(q.sys_scope);
+}
+
 /* {epoch, rtr[0]} in one acquire at the request's scope (adjacent words). */
 PC_DEVICE uint2 epoch_rtr(const pc_prequest_t &q) {
   return q.sys_scope ? ld_acquire_sys_v2(q.epoch) : ld_acquire_gpu_v2(q.epoch);
@@ -532,7 +540,7 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
   // grid.sync pattern: barrier, then one thread's fence + signal).
   __syncwarp(mask);
   if (lane == leader) {
-    if (preq.part_bytes) fence_scope(preq.sys_scope);
+    if (preq.part_bytes) fence_before_publish(preq);
     publish(preq, t, __popc(grp), e, partition);
   }
   return 0;
@@ -611,7 +619,7 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   }
   __syncwarp(full);  // the warp's pushes, then ONE cumulative fence by lane 0
   if (lane == 0) {
-    fence_scope(preq.sys_scope);
+    fence_before_publish(preq);
     publish(preq, t, 1, e, partition);
   }
   __syncwarp(full);
@@ -686,7 +694,7 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
   }
   __syncthreads();  // the block's pushes, then ONE cumulative fence by thread 0 (not one per thread)
   if (tid == 0) {
-    fence_scope(preq.sys_scope);
+    fence_before_publish(preq);
     publish(preq, t, 1, e, partition);
   }
   return 0;
