@@ -288,3 +288,29 @@ def test_dry_epoch_all_state_rules():
     for c in cs:
         c.destroy()
     g.destroy()
+
+
+def test_dry_waitall_state_rules():
+    """pc_waitall_on_stream bookkeeping (no device): completes every active
+    request of the list (a later pc_epoch_all, which needs inactive requests,
+    succeeds), skips inactive ones, accepts an empty list."""
+    g, cs = _dry(2)
+    snd = pc.psend_init(0x1000, 4, 8, pc.FLOAT32, 1, 1, cs[0])
+    rcv = pc.precv_init(0x2000, 4, 8, pc.FLOAT32, 0, 1, cs[1])
+    ar = [pc.pallreduce_init(0, 0, 2, 64, pc.FLOAT32, pc.SUM, pc.ALGO_RING, c) for c in cs]
+    pc.waitall_on_stream([])
+    pc.waitall_on_stream([snd, rcv] + ar)  # nothing started: all inactive
+    for q in [snd, rcv] + ar:
+        q.start()
+    pc.run_ranks([lambda: (snd.pbuf_prepare(), ar[0].pbuf_prepare()),
+                  lambda: (rcv.pbuf_prepare(), ar[1].pbuf_prepare())])
+    assert _try(lambda: pc.epoch_all([snd, rcv] + ar)) == pc.ERR_STATE  # still active
+    pc.waitall_on_stream([snd, rcv] + ar)
+    for _ in range(3):
+        pc.epoch_all([snd, rcv] + ar)
+        pc.waitall_on_stream([rcv, snd] + ar)
+    for q in [snd, rcv] + ar:
+        q.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
