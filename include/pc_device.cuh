@@ -219,8 +219,38 @@ PC_DEVICE uint32_t transport_size(const pc_prequest_t &q, int t) {
  * (counter already at/over the target) in the sticky error word.  With g = 1
  * every Pready completes its own transport partition: no counter (the
  * latency-critical path; duplicate detection needs g > 1). */
+/* Two-level counting for large g (reading R32): with g >= 4 * kSubAgg the
+ * user partitions of a transport partition count first into sub-counters of
+ * kSubAgg consecutive partitions (words cnt[ntransport ...], unused by the
+ * one-level layout: ntransport * (1 + ceil(g / kSubAgg)) <= N_p), and only
+ * the contribution completing a sub-group adds its size to cnt[t] — a
+ * whole-buffer transport partition of 1 M warp Preadies no longer funnels
+ * 1 M atomics into one word.  The acq_rel atomics chain the releases. */
+constexpr int kSubAgg = 256;
+PC_DEVICE bool sub_agg(const pc_prequest_t &q) { return q.agg >= 4 * kSubAgg; }
+/* The counter a contribution of partition p goes to first: lanes that share
+ * it are combined into one update (thread granularity). */
+PC_DEVICE int counter_key(const pc_prequest_t &q, int p) {
+  const int t = p / q.agg;
+  if (!sub_agg(q)) return t;
+  return t * ((q.agg + kSubAgg - 1) / kSubAgg) + (p - t * q.agg) / kSubAgg;
+}
+
 PC_DEVICE bool contribute(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, int part) {
   if (q.agg == 1) return true;
+  if (sub_agg(q)) {
+    const int sl = (part - t * q.agg) / kSubAgg;
+    const int rest = (int)transport_size(q, t) - sl * kSubAgg;
+    const uint32_t ssz = (uint32_t)(rest < kSubAgg ? rest : kSubAgg);
+    const uint32_t old = atom_add_acq_rel_gpu(q.cnt + q.ntransport + counter_key(q, part), add);
+    const int32_t d = (int32_t)(e * ssz - old);
+    if (d <= 0) {
+      set_error(q.err, PC_DEV_ERR_DEVICE, part);
+      return false;
+    }
+    if (d > (int32_t)add) return false;  // sub-group not complete yet
+    add = ssz;                           // carry the whole sub-group to cnt[t]
+  }
   const uint32_t target = e * transport_size(q, t);
   const uint32_t old = atom_add_acq_rel_gpu(q.cnt + t, add);
   const int32_t d = (int32_t)(target - old);
@@ -482,7 +512,7 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
   const uint32_t lane = lane_id();
   const uint32_t first = __ffs(mask) - 1;
   const int t = partition / preq.agg;
-  const unsigned grp = __match_any_sync(mask, t);
+  const unsigned grp = __match_any_sync(mask, counter_key(preq, partition));
   const uint32_t leader = __ffs(grp) - 1;
   if (preq.copy == 2) {  // LL: this lane pushes its partition's lines itself
     const uint32_t e = ll_push(preq, partition, 0, 1);
