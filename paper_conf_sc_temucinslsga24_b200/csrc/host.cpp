@@ -618,7 +618,10 @@ static int exchange_round(Comm *c, Request *target) {
           q->exchanged = true;
           q->matched = true;
           q->match_peer_index = m->req_index;
-          q->sys_scope = c->dry || memcmp(c->ranks[q->peer].uuid, c->ranks[c->rank].uuid, 16) != 0;
+          // PC_FORCE_SYS_SCOPE=1: system-scope ordering even between ranks of one GPU
+          // (runs the cross-GPU code paths on a one-GPU box; stronger, never weaker)
+          q->sys_scope = c->dry || memcmp(c->ranks[q->peer].uuid, c->ranks[c->rank].uuid, 16) != 0 ||
+                         env_long("PC_FORCE_SYS_SCOPE", 0) != 0;
         }
       }
     } else {  // PALLREDUCE: the seq-th allreduce of every rank
@@ -673,7 +676,7 @@ static int exchange_round(Comm *c, Request *target) {
         if (!qrc) {
           q->exchanged = true;
           q->matched = true;
-          q->sys_scope = c->dry ? 1 : 0;
+          q->sys_scope = (c->dry || env_long("PC_FORCE_SYS_SCOPE", 0) != 0) ? 1 : 0;
           for (int k = 0; k < P; ++k)
             if (memcmp(c->ranks[k].uuid, c->ranks[c->rank].uuid, 16) != 0) q->sys_scope = 1;
           // ranks of this comm sharing this GPU inside this process run their

@@ -628,3 +628,40 @@ def test_two_level_aggregation_counters(gran, agg, copy):
     n = 1 << 20
     partitions = n // GRAN_ELEMS[gran]
     run_vecadd(n, gran, partitions if agg == "all" else min(agg, partitions), copy, epochs=3)
+
+
+_SCOPE_PROBE = r"""
+import ctypes, os, sys
+sys.path.insert(0, os.environ["PC_ROOT"]); sys.path.insert(0, os.path.join(os.environ["PC_ROOT"], "tests"))
+import torch
+import paper_conf_sc_temucinslsga24_b200 as pc
+from gpu_util import comms, first_prepare
+with comms(2) as cs:
+    st = torch.cuda.Stream()
+    a, b = torch.zeros(1024, device="cuda"), torch.zeros(1024, device="cuda")
+    snd = pc.psend_init(a, 4, 256, pc.FLOAT32, 1, 3, cs[0])
+    rcv = pc.precv_init(b, 4, 256, pc.FLOAT32, 0, 3, cs[1])
+    snd.start(st); rcv.start(st)
+    first_prepare([[snd], [rcv]], [st, st])
+    pq = snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+    # pc_prequest_t.sys_scope: after 6 x 4-B fields, part_bytes and 11 pointers (include/pc_prequest.h)
+    print(int.from_bytes(pq.buf.raw[128:132], "little"))
+    snd.pready_range(0, 3, st)
+    snd.wait(); rcv.wait()
+    assert snd.error() == (0, 0) and rcv.error() == (0, 0)
+    snd.free(); rcv.free()
+"""
+
+
+@pytest.mark.parametrize("force", ["0", "1"])
+def test_force_sys_scope_env(force):
+    """PC_FORCE_SYS_SCOPE=1 (tools/gpu_sys_scope_check.sh runs the whole GPU
+    suite with it) really gives ranks of one GPU system-scope ordering."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, PC_ROOT=root, PC_FORCE_SYS_SCOPE=force)
+    p = subprocess.run([sys.executable, "-c", _SCOPE_PROBE], capture_output=True, text=True, env=env, timeout=240)
+    assert p.returncode == 0, p.stderr[-2000:]
+    assert p.stdout.strip().splitlines()[-1] == force
