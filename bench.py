@@ -47,6 +47,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-latency", action="store_true")
     ap.add_argument("--no-jacobi", action="store_true")
+    ap.add_argument("--no-c1", action="store_true",
+                    help="skip the C1 leg (its host Progression Engine epochs cannot progress under ncu's serialisation)")
     ap.add_argument("--jacobi-n", type=int, default=16384)
     ap.add_argument("--jacobi-iters", type=int, default=50)
     ap.add_argument("--quiet", action="store_true", help="only the JSON line")
@@ -580,7 +582,7 @@ def run_virtual(args):
     log("latency done")
     jac = None if args.no_jacobi else jacobi_bench(pc, apps, torch, args)
     log("jacobi done")
-    c1 = c1_bench(pc, apps, torch)
+    c1 = None if args.no_c1 else c1_bench(pc, apps, torch)
     log("c1 done")
     cpu = None if args.no_cpu_baseline else oracle_sample(P=P)
     log("cpu baseline done")
