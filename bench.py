@@ -4,16 +4,22 @@
 Driver contract (one JSON line on rank 0):
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl pc|reference]
   N > 1 runs under torchrun, one rank per GPU (real ranks, CUDA IPC over
-  NVLink/NVSwitch, NCCL all_reduce timed beside it as the vendor baseline).
-  N = 1 runs the same hot path with P virtual ranks co-located on the one
-  B200 (--vranks, default 8): every rank's buffers, flags and engine live on
-  one GPU, so "NVLink" stores become HBM stores and the kernel is HBM-bound.
+  NVLink/NVSwitch); `--gpus N` outside torchrun relaunches itself under
+  torch.distributed.run.  Beside the allreduce it times NCCL all_reduce on the
+  same bytes (default tuning and NCCL_ALGO=Ring, NCCL_DEBUG=INFO on stderr),
+  a bare peer-copy floor (the NVLink roofline denominator), the C1/C2 p2p and
+  Pready->Parrived latency legs between rank pairs and the C4 Jacobi solver
+  over all ranks.  N = 1 runs the same hot path with P virtual ranks
+  co-located on the one B200 (--vranks, default 8): every rank's buffers,
+  flags and engine live on one GPU, so "NVLink" stores become HBM stores and
+  the kernel is HBM-bound.
 
-A step = one epoch of the whole hot path for every rank: pc_start (epoch
-word) -> pc_pbuf_prepare (ready-to-receive) -> Pready of every partition
-(pc_pready_range) -> engine (Alg 1 ring: reduce-in-registers + forward, all
-2(P-1) steps) -> pc_wait_on_stream.  value = bus bandwidth (nccl-tests
-convention) = S/t * 2(P-1)/P with S bytes per rank.
+A step = one epoch of the whole hot path for every rank: pc_epoch_all (Start +
+ready-to-receive + the user's Pready of every partition, one kernel for all
+ranks of the GPU) -> pc_wait_on_stream (the engine: AUTO = the DIRECT
+schedule for 3-8 ranks, PULL reduce in registers, the final chunk stored
+into every rank's recvbuf).  value = bus bandwidth (nccl-tests convention) =
+S/t * 2(P-1)/P with S bytes per rank.
 """
 from __future__ import annotations
 
@@ -229,9 +235,12 @@ def run_reference(args):
     out = {"impl": "reference", "metric": METRIC, "value": v, "unit": "GB/s", "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": sec * 1e3, "higher_is_better": True,
            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-           "config": {"workload": f"partitioned allreduce (C5/C3 shape) fp32 sum, {where}, {args.bytes >> 20} MiB "
-                                  f"per rank in {args.partitions} partitions, {aname} schedule (requested {args.algo})",
-                      "ranks": P, "bytes_per_rank": args.bytes, "partitions": args.partitions, "algo": aname},
+           "config": {"workload": f"partitioned allreduce (C5/C3 shape) fp32 sum, {where}: the CPU oracle on a "
+                                  f"bounded slice of the GPU arm's workload — {S >> 20} MiB per rank in {Np} "
+                                  f"partitions per step (GPU arm: {args.bytes >> 20} MiB in {args.partitions}), "
+                                  f"{aname} schedule (requested {args.algo})",
+                      "ranks": P, "bytes_per_rank": S, "partitions": Np, "algo": aname,
+                      "gpu_arm_bytes_per_rank": args.bytes, "gpu_arm_partitions": args.partitions},
            "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 2 * P, "host_cpus": os.cpu_count(), "kind": "oracle",
                             "sample": f"each step: the CPU oracle ({aname} schedule + the Alg 2 loop, {P} rank threads"
                                       f" + {P} Pready threads) on an {S >> 20} MiB-per-rank, {Np}-partition slice of "
@@ -559,7 +568,8 @@ def run_virtual(args):
     e2e_ms = f0.elapsed_time(f1) / ke
     log(f"e2e: {e2e_ms:.3f} ms/step")
     e2e = {"value": busbw(S, e2e_ms / 1e3, P), "unit": "GB/s", "h2d_bytes_per_step": P * S, "d2h_bytes_per_step": S,
-           "ms_per_step": e2e_ms, "api": "pc_start/pc_pbuf_prepare/pc_pready_range/pc_wait_on_stream per rank"}
+           "ms_per_step": e2e_ms, "api": "pc_epoch_all(pready) + pc_wait_on_stream per rank (host buffers copied in "
+                                         "and the result copied out each step)"}
 
     for q in reqs:
         q.free()
@@ -602,24 +612,349 @@ def run_virtual(args):
     print(json.dumps(out), flush=True)
 
 
+def _free_port():
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+class MultiCtx:
+    """One process per GPU (torchrun): rank / world / device, the process
+    group, the max-over-ranks reduction and CUDA-event timing helpers."""
+
+    def __init__(self, torch, dist):
+        self.torch, self.dist = torch, dist
+        self.rank, self.world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
+        ngpu = torch.cuda.device_count()
+        local = int(os.environ.get("LOCAL_RANK", self.rank))
+        # ranks share GPUs: a correctness run of the N > 1 path on a smaller box
+        # (e.g. torchrun --nproc-per-node 2 on the one-GPU box): gloo bootstrap,
+        # no NCCL baseline (NCCL needs one GPU per rank), the processes time-slice
+        # the GPU, so reduced sizes and no meaningful times
+        self.shared = ngpu < int(os.environ.get("LOCAL_WORLD_SIZE", self.world))
+        self.dev = local % ngpu
+        torch.cuda.set_device(self.dev)
+        if self.shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", self.dev))
+        self.tdev = "cpu" if self.shared else "cuda"
+
+    def max(self, v):
+        t = self.torch.tensor([float(v)], dtype=self.torch.float64, device=self.tdev)
+        self.dist.all_reduce(t, op=self.dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def barrier(self):
+        self.dist.barrier()
+
+    def time_ms(self, fn, iters, stream, warm=2):
+        """CUDA events on `stream` around `iters` calls, barrier + sync on both
+        sides, max over ranks (ms per call)."""
+        torch = self.torch
+        for _ in range(warm):
+            fn()
+        torch.cuda.synchronize()
+        self.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(iters):
+            fn()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        self.barrier()
+        return self.max(e0.elapsed_time(e1) / iters)
+
+
+def multi_nvlink_floor(ctx, pc, apps, torch, chunk):
+    """Bare peer-copy floor (no library): every
+    rank writes (push) / reads (pull) `chunk` bytes to / from each of its P-1
+    peers at once — the all-to-all pattern of the DIRECT schedule over
+    NVSwitch.  Peer addresses come from a pc_pallgather_init request (its
+    recvbuf holds one chunk slot per rank).  GB/s per GPU per direction."""
+    P, r = ctx.world, ctx.rank
+    n = chunk // 4
+    st = torch.cuda.Stream()
+    comm = pc.Comm.from_process_group(ctx.dev)
+    send = torch.ones(n, device="cuda")
+    recv = torch.zeros(P * n, device="cuda")
+    q = pc.pallgather_init(send, recv, 1, n, pc.FLOAT32, comm)
+    q.start(st)
+    q.pbuf_prepare(st)
+    q.pready_range(0, 0, st)
+    q.wait_on_stream(st)
+    torch.cuda.synchronize()
+    peers = [q.peer_buffer(j) for j in range(P - 1)]
+    # push: my chunk -> slot r of every peer's recvbuf; pull: slot (peer) of every peer -> my slot (peer)
+    push_dst = [p + r * chunk for p in peers]
+    pull_src = [peers[j] + ((r + 1 + j) % P) * chunk for j in range(P - 1)]
+    pull_dst = [recv.data_ptr() + ((r + 1 + j) % P) * chunk for j in range(P - 1)]
+    iters = 3 if ctx.shared else 20
+    ms_push = ctx.time_ms(lambda: apps.peer_copy([send] * (P - 1), push_dst, chunk, stream=st), iters, st)
+    ms_pull = ctx.time_ms(lambda: apps.peer_copy(pull_src, pull_dst, chunk, stream=st), iters, st)
+    out_bytes = (P - 1) * chunk
+    res = {"push_gbs_per_gpu": out_bytes / (ms_push / 1e3) / 1e9, "pull_gbs_per_gpu": out_bytes / (ms_pull / 1e3) / 1e9,
+           "bytes_per_peer": chunk, "peers": P - 1, "kernel": "peer_copy_kernel (16-B vectors, no flags)"}
+    q.free()
+    comm.destroy()
+    return res
+
+
+def multi_nccl(ctx, torch, dist, send, steps):
+    """NCCL all_reduce on the same bytes: default tuning and NCCL_ALGO=Ring (a
+    second communicator created with the variable set; NCCL_DEBUG=INFO logs
+    each communicator's nranks and the chosen algorithm / protocol)."""
+    out = {}
+    x = send.clone()
+    st = torch.cuda.current_stream()
+    out["default"] = ctx.time_ms(lambda: dist.all_reduce(x), steps, st, warm=3)
+    old = os.environ.get("NCCL_ALGO")
+    os.environ["NCCL_ALGO"] = "Ring"
+    try:
+        g_ring = dist.new_group(list(range(ctx.world)), backend="nccl")
+        out["ring"] = ctx.time_ms(lambda: dist.all_reduce(x, group=g_ring), steps, st, warm=3)
+    finally:
+        if old is None:
+            os.environ.pop("NCCL_ALGO", None)
+        else:
+            os.environ["NCCL_ALGO"] = old
+    return out
+
+
+def multi_p2p(ctx, pc, apps, torch, dist):
+    """C1 / C2 / latency between rank pairs (2k, 2k+1), all pairs at once (one
+    pc comm per pair: the first pbuf_prepare is collective over its comm).
+    Even ranks produce (vector add, 8 B/thread, 1024-thread blocks, Pready
+    inside) and send; odd ranks receive.  Reported for pair (0, 1); times are
+    max over the pair."""
+    import numpy as np
+    P, r = ctx.world, ctx.rank
+    pairs = [dist.new_group([2 * k, 2 * k + 1]) for k in range(P // 2)]
+    if r >= 2 * (P // 2):  # odd world: the last rank sits this leg out
+        return None
+    grp = pairs[r // 2]
+    side = r % 2
+    comm = pc.Comm.from_process_group(ctx.dev, group=grp)
+    st = torch.cuda.Stream()
+
+    def pmax(v):
+        t = torch.tensor([float(v)], dtype=torch.float64, device=ctx.tdev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX, group=grp)
+        return float(t.item())
+
+    def ptime(fn, iters, warm=2):
+        for _ in range(warm):
+            fn()
+        torch.cuda.synchronize()
+        dist.barrier(group=grp)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        for _ in range(iters):
+            fn()
+        e1.record(st)
+        torch.cuda.synchronize()
+        dist.barrier(group=grp)
+        return pmax(e0.elapsed_time(e1) / iters)
+
+    res = {"pair": [0, 1], "note": "ranks 2k -> 2k+1, all pairs concurrently"}
+    sizes = [1 << 24] if ctx.shared else [1 << 20, 1 << 24, 1 << 28]
+    elems = {apps.GRAN_BLOCK: 2048, apps.GRAN_WARP: 64, apps.GRAN_THREAD: 2}
+    tag = 200
+    for S in sizes:
+        n = S // 4
+        A = torch.randn(n, device="cuda")
+        B = torch.randn(n, device="cuda")
+        Cb = torch.empty(n, device="cuda")
+        Rb = torch.zeros(n, device="cuda")
+        wts = (torch.arange(n, device="cuda", dtype=torch.int64) % 1021) + 1
+        row = {}
+        # traditional (Listing 1): kernel -> cudaStreamSynchronize -> copy into
+        # the peer's buffer (cudaMemcpyAsync, peer-mapped) -> synchronize
+        snd0 = pc.psend_init(Cb, 1, n, pc.FLOAT32, 1, tag, comm) if side == 0 else None
+        rcv0 = pc.precv_init(Rb, 1, n, pc.FLOAT32, 0, tag, comm) if side == 1 else None
+        tag += 1
+        q0 = snd0 or rcv0
+        q0.start(st)
+        q0.pbuf_prepare(st)
+        if side == 0:
+            q0.pready_range(0, 0, st)
+        q0.wait_on_stream(st)
+        torch.cuda.synchronize()
+        if side == 0:
+            peer = q0.peer_buffer(0)
+
+            def trad():
+                apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st)
+                st.synchronize()
+                apps.memcpy_async(peer, Cb, S, st)
+                st.synchronize()
+        else:
+            def trad():
+                pass
+        it = 5 if ctx.shared else (50 if S <= (1 << 24) else 10)
+        for _ in range(2):
+            trad()
+        dist.barrier(group=grp)
+        t0 = time.perf_counter()
+        for _ in range(it):
+            trad()
+        torch.cuda.synchronize()
+        row["traditional_us_host"] = pmax((time.perf_counter() - t0) / it * 1e6)
+        q0.free()
+        configs = [("block", apps.GRAN_BLOCK, 1, pc.COPY_INLINE), ("block", apps.GRAN_BLOCK, 1, pc.COPY_ENGINE),
+                   ("block->1MiB", apps.GRAN_BLOCK, 128, pc.COPY_INLINE),
+                   ("warp->all", apps.GRAN_WARP, None, pc.COPY_INLINE),
+                   ("thread->all", apps.GRAN_THREAD, None, pc.COPY_INLINE)]
+        if S == (1 << 20):  # C1: 128 block partitions aggregated into 8 transport partitions (R24)
+            configs = [("C1 block->128KiB", apps.GRAN_BLOCK, 16, pc.COPY_INLINE)] + configs
+        for name, gran, agg, copy in configs:
+            cnt = elems[gran]
+            parts = n // cnt
+            g = parts if agg is None else min(agg, parts)
+            if side == 0:
+                q = pc.psend_init(Cb, parts, cnt, pc.FLOAT32, 1, tag, comm)
+            else:
+                Rb.zero_()
+                q = pc.precv_init(Rb, parts, cnt, pc.FLOAT32, 0, tag, comm)
+            tag += 1
+            q.start(st)
+            q.pbuf_prepare(st)
+            sq = q.prequest_create(gran, g, copy) if side == 0 else None
+
+            def epoch(first=False):
+                if not first:
+                    q.start(st)
+                    q.pbuf_prepare(st)
+                if side == 0:
+                    apps.vecadd(A, B, Cb, n, gran, sq, st)
+                q.wait_on_stream(st)
+
+            epoch(first=True)
+            torch.cuda.synchronize()
+            us = ptime(epoch, it) * 1e3
+            err = q.error()
+            # parity gate of the point: the receiver's bytes equal the sender's C
+            # (exact: sums of the 32-bit patterns with position weights, exchanged)
+            buf = Cb if side == 0 else Rb
+            h = torch.tensor([int((buf.view(torch.int32).long() * wts).sum().item()) if side == 0 else 0,
+                              int((buf.view(torch.int32).long() * wts).sum().item()) if side == 1 else 0],
+                             dtype=torch.int64, device=ctx.tdev)
+            dist.all_reduce(h, group=grp)
+            q.free()
+            row[f"{name} {['inline', 'engine', 'll', 'host'][copy]}"] = {
+                "us": us, "gbs": S / (us / 1e6) / 1e9, "error": list(err), "parity": bool(h[0].item() == h[1].item())}
+        res[f"{S >> 20}MiB"] = row
+    # Pready -> Parrived latency: one persistent ping-pong kernel per side
+    iters = 50 if ctx.shared else 10000
+    lat = {}
+    for name, payload, copy in (("flag_only", 0, pc.COPY_INLINE), ("8B", 8, pc.COPY_INLINE),
+                                ("ll_8B", 8, pc.COPY_LL), ("ll_256B", 256, pc.COPY_LL)):
+        cnt = payload // 4
+        sbuf = torch.arange(max(iters * cnt, 4), dtype=torch.float32, device="cuda")
+        rbuf = torch.zeros(max(iters * cnt, 4), device="cuda")
+        snd = pc.psend_init(sbuf, iters, cnt, pc.FLOAT32, 1 - side, 300 + side, comm)
+        rcv = pc.precv_init(rbuf, iters, cnt, pc.FLOAT32, 1 - side, 300 + (1 - side), comm)
+        for q in (snd, rcv):
+            q.start(st)
+        for q in (snd, rcv):
+            q.pbuf_prepare(st)
+        sq = snd.prequest_create(pc.GRAN_WARP, 1, copy)
+        rq = rcv.prequest_create(pc.GRAN_WARP, 1, pc.COPY_INLINE)
+        t = torch.zeros(1, dtype=torch.int64, device="cuda")
+        torch.cuda.synchronize()
+        dist.barrier(group=grp)
+        apps.pingpong(sq, rq, side, iters, apps.GRAN_WARP, t, st)
+        snd.wait_on_stream(st)
+        rcv.wait_on_stream(st)
+        torch.cuda.synchronize()
+        one_way = pmax(float(t.item()) / iters / 2.0)
+        lat[name] = {"mean_ns": one_way, "payload_bytes": payload, "iters": iters,
+                     "copy": ["inline", "engine", "ll"][copy], "errors": [snd.error()[0], rcv.error()[0]]}
+        snd.free()
+        rcv.free()
+    # the floor: bare release/acquire system-scope flag ping-pong, no library
+    fl = torch.zeros(64, dtype=torch.int32, device="cuda")
+    q = pc.psend_init(fl, 1, 64, pc.INT32, 1 - side, 400 + side, comm)
+    q2 = pc.precv_init(fl, 1, 64, pc.INT32, 1 - side, 400 + (1 - side), comm)
+    for x in (q, q2):
+        x.start(st)
+    for x in (q, q2):
+        x.pbuf_prepare(st)
+    q.pready_range(0, 0, st)
+    q.wait_on_stream(st)
+    q2.wait_on_stream(st)
+    torch.cuda.synchronize()
+    peer_flag = q.peer_buffer(0)
+    fl.zero_()
+    torch.cuda.synchronize()
+    dist.barrier(group=grp)
+    t = torch.zeros(1, dtype=torch.int64, device="cuda")
+    apps.bare_pingpong(fl, peer_flag, side, iters, 0, t, st)
+    torch.cuda.synchronize()
+    lat["bare_sys_flag_floor_ns"] = pmax(float(t.item()) / iters / 2.0)
+    q.free()
+    q2.free()
+    res["latency_ns"] = lat
+    comm.destroy()
+    return res
+
+
+def multi_jacobi(ctx, pc, apps, torch, args):
+    """C4 at N GPUs: 16384^2 fp32, 1D (P x 1) and 2D decompositions, halos by
+    intra-kernel partitioned sends (pc_pready_warp into the neighbour's halo
+    over NVLink); GFLOP/s over all ranks (4 flops per interior cell)."""
+    P = ctx.world
+    N = 4096 if ctx.shared else args.jacobi_n
+    K = 5 if ctx.shared else args.jacobi_iters
+    decomps = [(P, 1)] + ([{2: (2, 1), 4: (2, 2), 8: (4, 2)}[P]] if P in (4, 8) else [])
+    comm = pc.Comm.from_process_group(ctx.dev)
+    res = {}
+    for Py, Px in decomps:
+        st = torch.cuda.Stream()
+        js = apps.JacobiSolver([comm], [ctx.rank], N, Py, Px, K, H=int(os.environ.get("PC_JACOBI_H", "64")),
+                               device=ctx.dev)
+        for s_ in js.local:
+            s_["grid"][0].zero_()
+            if s_["py"] == 0:
+                s_["grid"][0][: js.lx].fill_(1.0)
+            s_["grid"][1].copy_(s_["grid"][0])
+        torch.cuda.synchronize()
+        js.solve(st)  # first epoch: exchange + mapping
+        torch.cuda.synchronize()
+        reps = 1 if ctx.shared else 3
+        ms = ctx.time_ms(lambda: js.solve(st), reps, st, warm=1)
+        ms_iter = ms / K
+        errs = js.errors()
+        nerr = ctx.max(len(errs))
+        cells = (N - 2) * (N - 2)
+        res[f"{Py}x{Px}"] = {"gflops": 4.0 * cells / (ms_iter / 1e3) / 1e9, "us_per_iter": ms_iter * 1e3,
+                             "errors": int(nerr)}
+        js.free()
+    comm.destroy()
+    res["config"] = f"{N}^2 fp32, {K} iterations per epoch, one rank per GPU"
+    return res
+
+
 def run_multi(args):
     import numpy as np
+    # NCCL logs every communicator's rank / nranks and the tuning decision
+    # (algorithm, protocol) — to stderr, so stdout keeps the one JSON line
+    os.environ.setdefault("NCCL_DEBUG", "INFO")
+    os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT,TUNING,ENV")
+    os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
     import torch
     import torch.distributed as dist
 
     import paper_conf_sc_temucinslsga24_b200 as pc
+    from paper_conf_sc_temucinslsga24_b200 import apps
 
-    rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
-    local = int(os.environ.get("LOCAL_RANK", rank))
-    ngpu = torch.cuda.device_count()
-    shared = ngpu < int(os.environ.get("LOCAL_WORLD_SIZE", world))  # ranks share GPUs (debug on a 1-GPU box)
-    local = local % ngpu
-    torch.cuda.set_device(local)
-    if shared:  # NCCL refuses two ranks on one GPU: bootstrap over gloo, no NCCL baseline
-        dist.init_process_group("gloo")
-    else:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    ctx = MultiCtx(torch, dist)
+    rank, world, local = ctx.rank, ctx.world, ctx.dev
+    shared = ctx.shared
     P, S, Np = world, args.bytes, args.partitions
+    if shared:
+        S = min(S, 16 << 20)
     count = S // 4 // Np
     S = count * 4 * Np
     algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "auto": pc.ALGO_AUTO}[args.algo]
@@ -630,7 +965,7 @@ def run_multi(args):
     send = torch.randn(Np * count, device="cuda", generator=gen)
     recv = torch.empty_like(send)
     q = pc.pallreduce_init(send, recv, Np, count, pc.FLOAT32, pc.SUM, algo, comm)
-    info = q.info()
+    steps = min(args.steps, 5) if shared else args.steps
 
     def first_step():  # the first Pbuf_prepare exchanges and maps (blocking)
         q.start(st)
@@ -643,10 +978,30 @@ def run_multi(args):
         q.wait_on_stream(st)
 
     first_step()
+    info = q.info()
     for _ in range(max(args.warmup, 1)):
         step()
     torch.cuda.synchronize()
     assert q.error()[0] == 0
+    # parity gate (sampled): the allreduce of the rank-seeded inputs equals the
+    # fp64 sum within the north_star bound (R16); bit-identical on every rank
+    xs = [torch.empty_like(send) for _ in range(P)]
+    if shared:
+        dist.all_gather(xs_cpu := [torch.empty(send.numel()) for _ in range(P)], send.cpu())
+        xs = [x.cuda() for x in xs_cpu]
+    else:
+        dist.all_gather(xs, send)
+    idx = torch.randint(0, send.numel(), (4096,), device="cuda", generator=gen)
+    ref = torch.stack([x[idx].double() for x in xs]).sum(0)
+    bound = 1e-5 * torch.stack([x[idx].double().abs() for x in xs]).sum(0)
+    parity_ok = bool(((recv[idx].double() - ref).abs() <= bound).all().item())
+    h = torch.tensor([float(recv[idx].double().sum().item())], dtype=torch.float64, device=ctx.tdev)
+    hs = [torch.empty_like(h) for _ in range(P)]
+    dist.all_gather(hs, h)
+    parity_ok = parity_ok and all(float(x.item()) == float(h.item()) for x in hs)
+    parity_ok = ctx.max(0.0 if parity_ok else 1.0) == 0.0
+    del xs
+
     q.set_timing(True)
     q.engine_times()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -655,38 +1010,24 @@ def run_multi(args):
         dist.barrier()
         torch.cuda.synchronize()
         e0.record(st)
-        for _ in range(args.steps):
+        for _ in range(steps):
             step()
         e1.record(st)
         torch.cuda.synchronize()
         dist.barrier()
     launches = pc.launch_count() - n0
-    dev = "cpu" if shared else "cuda"
-
-    def max_over_ranks(v):
-        t = torch.tensor([v], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
-
-    ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+    ms = ctx.max(e0.elapsed_time(e1) / steps)
     eng = q.engine_times()
-    eng_ms = max_over_ranks(float(np.mean(eng)) if len(eng) else 0.0)
+    eng_ms = ctx.max(float(np.mean(eng)) if len(eng) else 0.0)
     assert q.error()[0] == 0
 
-    nms = None
-    if not shared:  # NCCL baseline on the same bytes, same stream discipline
-        x = send.clone()
-        for _ in range(3):
-            dist.all_reduce(x)
-        torch.cuda.synchronize()
-        dist.barrier()
-        n0e, n1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        n0e.record()
-        for _ in range(args.steps):
-            dist.all_reduce(x)
-        n1e.record()
-        torch.cuda.synchronize()
-        nms = max_over_ranks(n0e.elapsed_time(n1e) / args.steps)
+    nccl = {"skipped": "ranks share a GPU (debug run): NCCL needs one GPU per rank"}
+    if not shared:
+        t = multi_nccl(ctx, torch, dist, send, steps)
+        nccl = {k: {"value": busbw(S, v / 1e3, P), "ms_per_step": v, "unit": "GB/s"} for k, v in t.items()}
+        nccl["call"] = "torch.distributed.all_reduce (NCCL 2.28.9); 'ring' = a communicator created with NCCL_ALGO=Ring"
+        nccl["debug_log"] = "NCCL_DEBUG=INFO, NCCL_DEBUG_SUBSYS=INIT,TUNING,ENV on stderr"
+    log("allreduce + nccl done")
 
     # e2e: H2D input, allreduce, D2H result
     host_in = send.cpu().pin_memory()
@@ -704,32 +1045,53 @@ def run_multi(args):
             host_out.copy_(recv, non_blocking=True)
     f1.record(st)
     torch.cuda.synchronize()
-    ems = max_over_ranks(f0.elapsed_time(f1) / ke)
+    ems = ctx.max(f0.elapsed_time(f1) / ke)
     q.free()
     comm.destroy()
+
+    floor = multi_nvlink_floor(ctx, pc, apps, torch, min(S, 64 << 20))
+    log("nvlink floor done")
+    p2p = None if args.no_c1 else multi_p2p(ctx, pc, apps, torch, dist)
+    log("p2p legs done")
+    jac = None if args.no_jacobi else multi_jacobi(ctx, pc, apps, torch, args)
+    log("jacobi done")
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
+        cpu = oracle_sample(P=min(P, 8))
+    dist.barrier()
     if rank == 0:
         eng_ms_v = eng_ms or None
         # NVLink bytes per rank per direction: ring and DIRECT 2(P-1)/P*S, RD log2(P)*S
         nvl_bytes = (P.bit_length() - 1) * S if info["algo_name"] == "rd" else 2 * (P - 1) / P * S
         achieved = nvl_bytes / (eng_ms_v / 1e3) / 1e9 if eng_ms_v else None
+        # the roofline denominator: the measured bare peer-copy floor of this box
+        # (DIRECT: half its bytes are peer-load responses, half peer stores)
+        peak = 0.5 * (floor["push_gbs_per_gpu"] + floor["pull_gbs_per_gpu"]) if info["algo_name"] == "direct" \
+            else floor["push_gbs_per_gpu"]
+        where = "ranks sharing GPUs (debug run: time-sliced, not a measurement)" if shared else "one per B200"
         out = {"metric": METRIC, "value": busbw(S, ms / 1e3, P), "unit": "GB/s", "n_gpus": world,
-               "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+               "steps": steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
                "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-               "config": {"workload": f"partitioned allreduce fp32 sum, {P} ranks (one per B200), {S >> 20} MiB "
-                                      f"per rank in {Np} partitions, {args.algo} schedule", "ranks": P,
+               "config": {"workload": f"partitioned allreduce fp32 sum, {P} ranks ({where}), {S >> 20} MiB "
+                                      f"per rank in {Np} partitions, {info['algo_name']} schedule "
+                                      f"(requested {args.algo})", "ranks": P,
                           "bytes_per_rank": S, "partitions": Np, "algo": info["algo_name"],
                           "algo_requested": args.algo,
-                          "l2": "no flush: per-rank working set > 126 MB L2", "parallelism": f"dp{P}"},
-               "roofline": {"bound": "nvlink", "achieved": achieved, "peak": 770.0, "unit": "GB/s",
-                            "frac": achieved / 770.0 if achieved else None, "traffic": None,
+                          "l2": "no flush: per-rank working set > 126 MB L2" if S >= (64 << 20) else
+                                "working set within L2 (debug size)",
+                          "parallelism": f"dp{P}"},
+               "parity": {"ok": parity_ok, "check": "4096 sampled elements vs the fp64 sum within 1e-5*sum|x| "
+                                                   "(R16), bit-identical on every rank"},
+               "roofline": {"bound": "nvlink", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                            "frac": achieved / peak if achieved and peak else None, "traffic": None,
                             "kernel": f"{info['algo_name']}_engine", "engine_ms": eng_ms_v,
-                            "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s per direction"},
-               "cpu_baseline": None, "e2e": {"value": busbw(S, ems / 1e3, P), "unit": "GB/s",
-                                             "h2d_bytes_per_step": S, "d2h_bytes_per_step": S, "ms_per_step": ems},
-               "gpu_launches": launches, "clocks": clk.summary(),
-               "nccl": ({"value": busbw(S, nms / 1e3, P), "ms_per_step": nms, "unit": "GB/s",
-                         "call": "torch.distributed.all_reduce (NCCL 2.28.9)"} if nms else
-                        {"skipped": "ranks share a GPU (debug run): NCCL needs one GPU per rank"})}
+                            "nvlink_bytes_per_rank_per_launch": nvl_bytes,
+                            "peak_source": "measured on this box: bare peer-copy floor (nvlink_floor)"},
+               "nvlink_floor": floor, "cpu_baseline": cpu,
+               "e2e": {"value": busbw(S, ems / 1e3, P), "unit": "GB/s", "h2d_bytes_per_step": S,
+                       "d2h_bytes_per_step": S, "ms_per_step": ems,
+                       "api": "pc_epoch_all(pready) + pc_wait_on_stream, host buffers copied in/out each step"},
+               "gpu_launches": launches, "clocks": clk.summary(), "nccl": nccl, "p2p": p2p, "jacobi": jac}
         print(json.dumps(out), flush=True)
     dist.destroy_process_group()
 
@@ -739,6 +1101,13 @@ def main():
     if args.quiet:
         sys.stderr = open(os.devnull, "w")
     world = int(os.environ.get("WORLD_SIZE", "1"))
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # --gpus N outside torchrun: relaunch as N processes, one per GPU
+        # (never fall back to virtual ranks reporting n_gpus 1)
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+        log("relaunching under torchrun:", " ".join(cmd))
+        sys.exit(subprocess.call(cmd))
     if args.impl == "reference":
         run_reference(args)
         return

@@ -105,12 +105,25 @@ int pc_comm_size(pc_comm_t comm, int *size);
  * on all ranks so per-warp work orders match — the deadlock-freedom argument
  * of DESIGN.md §"Engine"). */
 int pc_comm_engine_warps(pc_comm_t comm, int *warps);
+/* Per-rank engine warps while the engine may run beside a producer kernel
+ * (pc_start's overlap rule): whole 8-warp CTAs, the ranks of one GPU together
+ * on at most PC_OVERLAP_FRAC of its SMs (min over the comm's ranks). */
+int pc_comm_overlap_warps(pc_comm_t comm, int *warps);
 
 /* In-process rank groups: several ranks of one comm living in ONE process
  * (e.g. P virtual ranks sharing one GPU, or one process driving several GPUs).
  * Peers in the same process are addressed directly, without CUDA IPC.  Each
  * rank must be driven by its own host thread during pc_comm_create and the
- * first pc_pbuf_prepare (the all-gather blocks until every rank arrived). */
+ * first pc_pbuf_prepare (the all-gather blocks until every rank arrived).
+ * The engines of co-located ranks of one GPU (allreduce-kind requests) run as
+ * ONE grouped kernel, enqueued by the LAST member's wait of the epoch (every
+ * member's producer work is then already enqueued).  A member whose
+ * pc_wait_on_stream came earlier gets the completion ordered on its stream at
+ * that launch: work it enqueued on that stream BEFORE the group's last wait is
+ * not ordered after the collective — enqueue dependent work after every
+ * member's wait (or wait from one host thread per rank with pc_wait).  A
+ * member cannot start its next epoch before the group's engine of the current
+ * one is enqueued (PC_ERR_STATE). */
 int pc_local_group_create(int size, pc_local_group_t *group);
 int pc_local_group_destroy(pc_local_group_t group);
 /* ctx to pass to pc_comm_create together with pc_local_allgather */
@@ -169,8 +182,25 @@ int pc_pbcast_init(void *buf, int partitions, size_t count, pc_dtype_t dtype, in
 
 /* ---------------------------------------------------------------- epoch
  * MPI_Start: epoch e <- e+1, written stream-ordered to the device
- * epoch word; for ENGINE copy and allreduce it also launches the engine on a
- * library stream forked from `stream`.  PC_ERR_STATE if the request is active. */
+ * epoch word.  PC_ERR_STATE if the request is active.  If the previous epoch's
+ * completion was ordered on another stream, `stream` first waits for it.
+ *
+ * Engines (allreduce-kind requests, ENGINE-copy sends): the engine kernel is
+ * ENQUEUED on a library stream at pc_wait / pc_wait_on_stream / pc_test —
+ * after the user's producer kernels in host order (Listing 2) — but it is
+ * FORKED from the epoch's last control call (pc_start, pc_pbuf_prepare,
+ * pc_startall, pc_pbuf_prepare_all, pc_epoch_all): it starts as soon as the
+ * epoch is set up and forwards / reduces each partition as soon as its Pready
+ * arrives, while the producer still runs (§IV-B1).  While a
+ * producer may run beside it the engine takes whole CTAs on at most
+ * PC_OVERLAP_FRAC (default 0.5) of the SMs; after a host-side Pready of every
+ * partition (pc_epoch_all with pready, pc_preadyall, pc_pready_range over all
+ * partitions), which re-records the fork point, it takes the full width.  Producer
+ * kernels whose blocks need a whole SM still always find one.
+ * pc_request_set_overlap(req, 0) forks the engine at the wait instead (the
+ * engine then starts after everything enqueued before the wait: no overlap,
+ * full width).  Call it while the request is inactive; PC_ERR_STATE otherwise. */
+int pc_request_set_overlap(pc_request_t req, int on);
 int pc_start(pc_request_t req, pc_stream_t stream);
 /* MPIX_Pbuf_prepare: guarantees the remote buffers are
  * ready.  FIRST call (per batch of new requests): host-blocking exchange of
@@ -259,6 +289,14 @@ int pc_request_words(pc_request_t req, int which, int offset, int n, uint32_t *o
  * since the last call into ms[0..max) and returns how many it wrote. */
 int pc_request_set_timing(pc_request_t req, int on);
 int pc_request_engine_times(pc_request_t req, float *ms, int max);
+/* Peer-mapped address (CUDA IPC or same-process pointer, valid in this
+ * process) of a peer's receive buffer after the first pc_pbuf_prepare: a send
+ * request's receiver buffer (j = 0), or for a DIRECT-schedule collective
+ * (pc_pallgather_init, pc_pallreduce_init with PC_ALGO_DIRECT) the recvbuf of
+ * peer j = rank (r + 1 + j) mod P, 0 <= j < P - 1.  For measurement kernels
+ * outside the library (the bench's bare NVLink peer-copy and flag floors).
+ * PC_ERR_STATE before the exchange, PC_ERR_UNSUPPORTED for other kinds. */
+int pc_request_peer_buffer(pc_request_t req, int j, void **ptr);
 /* Number of kernels libpc has launched in this process (for the bench's
  * gpu_launches claim). */
 uint64_t pc_launch_count(void);

@@ -35,6 +35,7 @@ _PC_PROTOS = {
     "pc_comm_rank": (I32, [P, PI32]),
     "pc_comm_size": (I32, [P, PI32]),
     "pc_comm_engine_warps": (I32, [P, PI32]),
+    "pc_comm_overlap_warps": (I32, [P, PI32]),
     "pc_local_group_create": (I32, [I32, C.POINTER(P)]),
     "pc_local_group_destroy": (I32, [P]),
     "pc_local_group_ctx": (P, [P, I32]),
@@ -70,6 +71,8 @@ _PC_PROTOS = {
     "pc_request_error": (I32, [P, PI32, PI32]),
     "pc_request_words": (I32, [P, I32, I32, I32, P]),
     "pc_request_set_timing": (I32, [P, I32]),
+    "pc_request_set_overlap": (I32, [P, I32]),
+    "pc_request_peer_buffer": (I32, [P, I32, C.POINTER(C.c_void_p)]),
     "pc_request_engine_times": (I32, [P, P, I32]),
     "pc_launch_count": (C.c_uint64, []),
     "pc_strerror": (C.c_char_p, [I32]),
@@ -87,6 +90,9 @@ _APP_PROTOS = {
     "pcapp_pingpong_pair": (I32, [P, P, P, P, I32, I32, P, P, P]),
     "pcapp_bare_pingpong_pair": (I32, [P, P, I32, C.c_uint32, P, I32, P]),
     "pcapp_prequest_size": (SZ, []),
+    "pcapp_overlap_probe": (I32, [P, I32, C.c_uint32, P, P]),
+    "pcapp_peer_copy": (I32, [I32, C.POINTER(P), C.POINTER(P), C.c_uint64, I32, P]),
+    "pcapp_memcpy_async": (I32, [P, P, C.c_uint64, P]),
     "pcapp_flag_variant": (I32, [P, P, I32, I32, C.c_uint32, P, P]),
     "pcapp_lat_probe_pair": (I32, [P, P, P, P, I32, I32, P, P]),
     "pcapp_jacobi_rank_size": (SZ, []),

@@ -46,6 +46,29 @@ def bce_grad(p, y, g, partitions: int, L: int, nf: float, preq: Prequest | None 
                                    preq.ptr if preq is not None else None, _stream(stream)), "bce_grad")
 
 
+def peer_copy(srcs, dsts, nbytes: int, blocks: int = 0, stream=None):
+    """Bare peer copies (no library): len(srcs) concurrent copies of nbytes
+    each, srcs[j] -> dsts[j] (int addresses or tensors; one side peer-mapped)."""
+    n = len(srcs)
+    sa = (C.c_void_p * n)(*[_ptr(x) for x in srcs])
+    da = (C.c_void_p * n)(*[_ptr(x) for x in dsts])
+    _ok(_lib.apps().pcapp_peer_copy(n, sa, da, nbytes, blocks, _stream(stream)), "peer_copy")
+
+
+def memcpy_async(dst, src, nbytes: int, stream=None):
+    """cudaMemcpyAsync(cudaMemcpyDefault) of nbytes (dst / src: tensors or
+    int addresses, e.g. a peer-mapped buffer) on `stream`."""
+    _ok(_lib.apps().pcapp_memcpy_async(_ptr(dst), _ptr(src), nbytes, _stream(stream)), "memcpy_async")
+
+
+def overlap_probe(preq: Prequest, partitions: int, spin_ms: int, out_ns, stream=None):
+    """a6 concurrency probe: Pready(0), spin (<= spin_ms) until Parrived(0),
+    then Pready the rest.  out_ns: int64 device tensor [4] = %globaltimer at
+    entry, after Pready(0), when Parrived(0) was seen (0: timed out), exit."""
+    _ok(_lib.apps().pcapp_overlap_probe(preq.ptr, partitions, spin_ms, _ptr(out_ns), _stream(stream)),
+        "overlap_probe")
+
+
 def check_recv(preq: Prequest, recvbuf, out, partitions: int, part_bytes: int, status, blocks: int = 64,
                stream=None):
     _ok(_lib.apps().pcapp_check_recv(preq.ptr, _ptr(recvbuf), _ptr(out), partitions, part_bytes, blocks,
@@ -288,15 +311,22 @@ class DLProxy:
     """The paper's DL kernel (§VI-D2) on co-located ranks: every
     step each rank computes its BCE gradient (``bce_grad``) and the ranks
     allreduce it with one persistent partitioned allreduce; ``pc_startall`` and
-    ``pc_pbuf_prepare_all`` are inside the step, as in a training loop.
+    ``pc_pbuf_prepare_all`` are inside the step, as in a training loop.  Each
+    rank's producer runs on its own stream (as each GPU would run its own),
+    after the epoch's control kernels on the control stream ``ctl``.
 
     mode "pready": the producer Preadies each partition from the kernel
-                   (block granularity, ENGINE copy); the engine reduces;
-    mode "serial": producer kernel, then the collective (host-side Pready of
+                   (block granularity); the engine — forked at the epoch's
+                   pbuf_prepare, enqueued at the wait — reduces each partition
+                   as soon as every rank has produced it, while the producers
+                   still run (§8(a) a6);
+    mode "serial": producer kernels, then the collective (host-side Pready of
                    every partition, the MPI_Allreduce-after-the-kernel flow).
+    ``overlap=False`` forks the engine at the wait (pc_request_set_overlap):
+    the Pready mode without producer/engine concurrency.
     Inputs: ``p`` (predictions), ``y`` (targets), fp32, one tensor per rank."""
 
-    def __init__(self, comms, partitions: int, L: int, algo: int, p, y):
+    def __init__(self, comms, partitions: int, L: int, algo: int, p, y, overlap: bool = True):
         import torch
 
         from . import runtime as rt
@@ -309,8 +339,15 @@ class DLProxy:
         self.out = [torch.empty(max(n, 4), device=p[0].device) for _ in range(self.P)]
         self.reqs = [rt.pallreduce_init(self.g[r], self.out[r], partitions, L, rt.FLOAT32, rt.SUM, algo, comms[r])
                      for r in range(self.P)]
+        self.overlap = overlap
+        if not overlap:
+            for q in self.reqs:
+                q.set_overlap(False)
         self.preqs = None
         self.ctl = torch.cuda.Stream()
+        self.pst = [torch.cuda.Stream() for _ in range(self.P)]
+        self.ev_ctl = torch.cuda.Event()
+        self.ev_p = [torch.cuda.Event() for _ in range(self.P)]
 
     def step(self, mode: str = "pready", order_stride: int = 1):
         from . import runtime as rt
@@ -324,13 +361,22 @@ class DLProxy:
         else:
             rt.startall(self.reqs, st)
             rt.pbuf_prepare_all(self.reqs, st)
+        self.ev_ctl.record(st)
         for r in range(self.P):
+            self.pst[r].wait_event(self.ev_ctl)
             bce_grad(self.p[r], self.y[r], self.g[r], self.Np, self.L, self.nf,
-                     self.preqs[r] if mode == "pready" else None, order_stride, stream=st)
+                     self.preqs[r] if mode == "pready" else None, order_stride, stream=self.pst[r])
+            self.ev_p[r].record(self.pst[r])
+        if mode == "serial" or not self.overlap:  # the collective (or its fork point) after the kernels
+            for r in range(self.P):
+                st.wait_event(self.ev_p[r])
         if mode == "serial":
             rt.preadyall(self.reqs, st)
-        for q in self.reqs:
+        for q in self.reqs:  # (enqueues the engine: after every producer in host order)
             q.wait_on_stream(st)
+        if mode != "serial" and self.overlap:  # join the producers' tails before the next epoch
+            for r in range(self.P):
+                st.wait_event(self.ev_p[r])
 
     def errors(self):
         return [(r, q.error()) for r, q in enumerate(self.reqs) if q.error()[0] != 0]

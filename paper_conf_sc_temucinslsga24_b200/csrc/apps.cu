@@ -72,6 +72,66 @@ __global__ void __launch_bounds__(512) produce_kernel(uint8_t *__restrict__ dst,
   }
 }
 
+// Bare NVLink peer-copy floor (SURVEY §8(d) "Rooflines"): no
+// library, no flags — n concurrent copies of `bytes` each (blockIdx.y = copy),
+// 16-B vectors, 4 in flight per thread.  dst (push) or src (pull) is a
+// peer-mapped address; the bench times every rank writing to / reading from
+// its peers at once, the traffic pattern of the DIRECT schedule.
+struct PeerCopyArgs {
+  int n;
+  uint64_t bytes;
+  const uint8_t *src[8];
+  uint8_t *dst[8];
+};
+__global__ void __launch_bounds__(512) peer_copy_kernel(PeerCopyArgs a) {
+  const int j = blockIdx.y;
+  const uint4 *s = reinterpret_cast<const uint4 *>(a.src[j]);
+  uint4 *d = reinterpret_cast<uint4 *>(a.dst[j]);
+  const uint64_t nv = a.bytes / 16, stride = (uint64_t)gridDim.x * blockDim.x;
+  uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  for (; k + 3 * stride < nv; k += 4 * stride) {
+    const uint4 v0 = s[k], v1 = s[k + stride], v2 = s[k + 2 * stride], v3 = s[k + 3 * stride];
+    d[k] = v0;
+    d[k + stride] = v1;
+    d[k + 2 * stride] = v2;
+    d[k + 3 * stride] = v3;
+  }
+  for (; k < nv; k += stride) d[k] = s[k];
+}
+
+// Overlap probe (§8(a) a6, "each partition independently executes that
+// schedule"): one block Preadies partition 0 of a partitioned collective, then
+// (thread 0) spins until the collective reports partition 0 complete on this
+// rank (device pc_parrived, at most spin_ms), then Preadies partitions 1.. and
+// exits.  Partition 0 can only complete while this kernel is still running if
+// the engine runs concurrently with it.  out[0..3] = %globaltimer at entry,
+// after Pready(0), when Parrived(0) was seen (0 = never, timed out), at exit.
+__global__ void overlap_probe_kernel(pc_prequest_t preq, int partitions, uint32_t spin_ms,
+                                     unsigned long long *out) {
+  __shared__ int s_arrived;
+  if (threadIdx.x == 0) out[0] = pc_detail::globaltimer();
+  pc_pready_block(0, preq);
+  if (threadIdx.x == 0) {
+    const unsigned long long t1 = pc_detail::globaltimer();
+    out[1] = t1;
+    int arrived = 0;
+    for (;;) {
+      if (pc_parrived(preq, 0)) {
+        arrived = 1;
+        break;
+      }
+      if (pc_detail::globaltimer() - t1 > (unsigned long long)spin_ms * 1000000ull) break;
+      __nanosleep(200);
+    }
+    out[2] = arrived ? pc_detail::globaltimer() : 0ull;
+    s_arrived = arrived;
+  }
+  __syncthreads();
+  for (int p = 1; p < partitions; ++p) pc_pready_block(p, preq);
+  __syncthreads();
+  if (threadIdx.x == 0) out[3] = pc_detail::globaltimer();
+}
+
 // R28: g = (p - y) / ((p * (1 - p)) * n), five IEEE fp32 ops in this order
 // (explicit _rn intrinsics: no contraction, IEEE division).
 __device__ __forceinline__ float bce_g(float p, float y, float nf) {
@@ -529,6 +589,33 @@ int pcapp_lat_probe_pair(const pc_prequest_t *sendA, const pc_prequest_t *recvA,
     default: PCAPP_LP(1, 14); break;
   }
 #undef PCAPP_LP
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_peer_copy(int n, const void *const *src, void *const *dst, uint64_t bytes, int blocks, cudaStream_t s) {
+  if (n < 1 || n > 8 || (bytes & 15)) return -1;
+  PeerCopyArgs a{};
+  a.n = n;
+  a.bytes = bytes;
+  for (int j = 0; j < n; ++j) {
+    a.src[j] = (const uint8_t *)src[j];
+    a.dst[j] = (uint8_t *)dst[j];
+  }
+  if (blocks <= 0) blocks = 148 * 4 / n > 0 ? 148 * 4 / n : 1;
+  peer_copy_kernel<<<dim3(blocks, n), 512, 0, s>>>(a);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+// cudaMemcpyAsync (cudaMemcpyDefault: peer-mapped destinations included) —
+// the copy of the traditional model (Listing 1) in the bench's N > 1 legs.
+int pcapp_memcpy_async(void *dst, const void *src, uint64_t bytes, cudaStream_t s) {
+  return cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDefault, s) == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_overlap_probe(const pc_prequest_t *preq, int partitions, uint32_t spin_ms, unsigned long long *out,
+                        cudaStream_t s) {
+  if (!preq || partitions < 1) return -1;
+  overlap_probe_kernel<<<1, 128, 0, s>>>(*preq, partitions, spin_ms, out);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -549,7 +549,7 @@ __device__ __forceinline__ void red_add_scope(uint32_t *p, uint32_t v, bool sys)
 // of this rank's recvbuf and (TO_PEERS) of every peer's.  When the sources and
 // the destination do not share a 16-B misalignment the whole range takes the
 // scalar path.
-template <int DT, int OP, bool TO_PEERS = true, typename A>
+template <int DT, int OP, bool TO_PEERS = true, int FV = PC_DIRECT_FV, typename A>
 __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d0, int64_t n) {
   using O = Op<DT, OP>;
   using T = typename O::T;
@@ -576,7 +576,7 @@ __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d
   const int64_t nv = (n - head) / EPV;
   // all P * kFV loads of a lane are issued before the first add (the fold
   // itself stays in rank order): one round trip per kFV vectors, not P
-  constexpr int kFV = PC_DIRECT_FV;
+  constexpr int kFV = FV;
   auto store_all = [&](int64_t vk, uint4 acc) {
     const int64_t eo = head + EPV * vk;
     *reinterpret_cast<uint4 *>(out_local + eo) = acc;
@@ -752,7 +752,7 @@ __device__ __forceinline__ void warp_fold_pull_bulk(const A &a, int64_t s0, int6
   for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
 }
 
-template <int DT, int OP>
+template <int DT, int OP, int FV = PC_DIRECT_FV>
 __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W, uint8_t *smem) {
   const int P = a.P, r = a.r;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;
@@ -810,7 +810,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
             if (PC_DIRECT_BULK && !a.sys)
               warp_fold_pull_bulk<DT, OP>(a, base + lo, base + lo, hi - lo, wb);
             else
-              warp_fold_pull<DT, OP>(a, base + lo, base + lo, hi - lo);
+              warp_fold_pull<DT, OP, true, FV>(a, base + lo, base + lo, hi - lo);
           }
           fence_scope(a.sys);
           __syncwarp();
@@ -982,6 +982,24 @@ __global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine_gr
   direct_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, dsmem);
 }
 
+// "Thin" DIRECT engines for the overlap case (the engine runs beside the
+// user's producer kernels): 2 CTAs per SM (<= 128 registers) and
+// one 16-B vector per operand in flight, so an SM holding an engine CTA still
+// has half its registers and 56 warp slots for producer blocks (a fat CTA
+// leaves ~11 K registers: no 512-thread producer block fits beside it).
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_thin(DirectArgs a) {
+  direct_body<DT, OP, 1>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5, nullptr);
+}
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_group_thin(DirectGroupArgs g) {
+  int k = 0;
+  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
+  const int b = blockIdx.x - g.block_start[k];
+  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
+  direct_body<DT, OP, 1>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, nullptr);
+}
+
 // Single-rank launches (one rank per GPU / process).
 template <int DT, int OP>
 __global__ void __launch_bounds__(kEngineBlock) ring_engine(RingArgs a) {
@@ -1032,10 +1050,10 @@ template <int DT, int OP>
 struct EngineLaunch {
   static int ring(const RingArgs &a, int warps, cudaStream_t s);
   static int rd(const RdArgs &a, int warps, cudaStream_t s);
-  static int direct(const DirectArgs &a, int warps, cudaStream_t s);
+  static int direct(const DirectArgs &a, int warps, cudaStream_t s, bool thin);
   static int ring_group(const RingGroupArgs &h, int blocks, cudaStream_t s);
   static int rd_group(const RdGroupArgs &h, int blocks, cudaStream_t s);
-  static int direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s);
+  static int direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s, bool thin);
   static int coll(const CollArgs &a, int warps, cudaStream_t s);
   static int coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s);
   static int occupancy(int *ctas);

@@ -38,7 +38,13 @@ static int direct_smem_attr(K kernel) {
 }
 
 template <int DT, int OP>
-int EngineLaunch<DT, OP>::direct(const DirectArgs &a, int warps, cudaStream_t s) {
+int EngineLaunch<DT, OP>::direct(const DirectArgs &a, int warps, cudaStream_t s, bool thin) {
+  if (thin) {
+    direct_engine_thin<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    g_launches++;
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  }
   if (int rc = direct_smem_attr(direct_engine<DT, OP>)) return rc;
   direct_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, kDirectSmem, s>>>(a);
   g_launches++;
@@ -63,7 +69,13 @@ int EngineLaunch<DT, OP>::rd_group(const RdGroupArgs &h, int blocks, cudaStream_
 }
 
 template <int DT, int OP>
-int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s) {
+int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s, bool thin) {
+  if (thin) {
+    direct_engine_group_thin<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+    g_launches++;
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  }
   if (int rc = direct_smem_attr(direct_engine_group<DT, OP>)) return rc;
   direct_engine_group<DT, OP><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
   g_launches++;
@@ -123,6 +135,8 @@ int EngineLaunch<DT, OP>::preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, ring_engine_group<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, rd_engine_group<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_thin<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP>));
   return 0;

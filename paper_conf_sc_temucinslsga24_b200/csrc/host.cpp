@@ -33,6 +33,10 @@ static bool env_flag(const char *n) {
   const char *v = getenv(n);
   return v && *v && strcmp(v, "0") != 0;
 }
+static double env_double(const char *n, double dflt) {
+  const char *v = getenv(n);
+  return v && *v ? atof(v) : dflt;
+}
 static long env_long(const char *n, long dflt) {
   const char *v = getenv(n);
   if (!v || !*v) return dflt;
@@ -848,6 +852,9 @@ static CollArgs make_coll_args(Request *q) {
   return a;
 }
 
+// joined_stream value: the previous epoch's completion was observed by the host
+static const cudaStream_t kHostJoined = reinterpret_cast<cudaStream_t>(~uintptr_t(0));
+
 static bool needs_engine(Request *q) {
   return q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
 }
@@ -871,18 +878,71 @@ static int timing_end(TimingLog &T, cudaStream_t s, int a) {
   return 0;
 }
 
-// Single-rank launch on the request's side stream, forked from its user stream.
+// ---------------------------------------------------------------- overlap
+// Producer/engine overlap (§8(a) a6: "each partition forwarded and reduced as
+// soon as it is ready").  The engine is still
+// ENQUEUED at the wait (after the user's producer in host order, so no
+// spinning kernel ever depends on work submitted behind it), but it is forked
+// from ev_fork, which the epoch's control calls record: it starts as soon as
+// the epoch word and the ready-to-receive words are written and reduces each
+// partition while the producer is still running.
+static int fork_point(Request *q, cudaStream_t s) {
+  if (q->comm->dry || !q->ev_fork) return 0;
+  PC_CUDA(cudaEventRecord(q->ev_fork, s));
+  q->forked = true;
+  return 0;
+}
+
+// The engine's width.  When every partition was made ready by a host-side op
+// before ev_fork (pc_epoch_all with Pready, pc_preadyall, pc_pready_range of
+// all partitions) no user kernel can be running that the engine waits for:
+// full width.  Otherwise a producer kernel may still have blocks to place, so
+// the engine takes whole CTAs on at most PC_OVERLAP_FRAC of the SMs per GPU —
+// at least one SM carries no engine CTA, so every producer block that fits an
+// empty SM can always be placed (deadlock freedom).
+static bool full_width(const Request *q) { return !q->overlap || q->host_ready_all; }
+static int engine_width(const Request *q, bool full) {
+  return full ? q->engine_warps : std::min(q->engine_warps, q->comm->overlap_warps);
+}
+
+// Start of an epoch (pc_start / pc_startall / pc_epoch_all): reset the
+// per-epoch overlap state; a co-located group member may not start while the
+// group's engine of its previous epoch is not launched (the engine reads the
+// epoch word at entry); and when the previous epoch's completion was joined
+// on another stream, this epoch's control op waits for it first.
+static bool group_blocks_start(Request *q) {
+  if (!q->leader) return false;
+  GroupState &g = q->leader->gs;
+  std::lock_guard<std::mutex> lk(g.mu);
+  return g.epoch == q->epoch && q->engine_registered && !g.launched;
+}
+static int epoch_begin(Request *q, cudaStream_t s, bool capturing) {
+  if (group_blocks_start(q)) return PC_ERR_STATE;
+  if (!q->comm->dry && q->epoch > 0 && !capturing && q->joined_stream != s && q->joined_stream != kHostJoined &&
+      needs_engine(q) && q->engine_launched) {
+    cudaEvent_t ev = q->leader ? q->leader->gs.ev : q->ev_done;
+    if (ev) PC_CUDA(cudaStreamWaitEvent(s, ev, 0));
+  }
+  q->forked = false;
+  q->host_ready_all = false;
+  q->join_pending = false;
+  return 0;
+}
+
+// Single-rank launch on the request's side stream, forked from ev_fork.
 static int launch_single(Request *q) {
-  PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+  if (!q->forked || !q->overlap) PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
   PC_CUDA(cudaStreamWaitEvent(q->side, q->ev_fork, 0));
+  const bool full = full_width(q);
+  const int w = engine_width(q, full);
   int rc, tk;
   if ((rc = timing_begin(q->tlog, q->side, &tk))) return rc;
   if (q->kind == PC_KIND_PALLREDUCE && q->coll != PC_COLL_ALLREDUCE) {
-    rc = launch_coll_engine(make_coll_args(q), q->engine_warps, q->side);
+    rc = launch_coll_engine(make_coll_args(q), w, q->side);
   } else if (q->kind == PC_KIND_PALLREDUCE) {
-    rc = q->algo == PC_ALGO_RING     ? launch_ring_engine(make_ring_args(q), q->engine_warps, q->side)
-         : q->algo == PC_ALGO_DIRECT ? launch_direct_engine(make_direct_args(q), q->engine_warps, q->side)
-                                     : launch_rd_engine(make_rd_args(q), q->engine_warps, q->side);
+    rc = q->algo == PC_ALGO_RING     ? launch_ring_engine(make_ring_args(q), w, q->side)
+         : q->algo == PC_ALGO_DIRECT ? launch_direct_engine(make_direct_args(q), w, q->side, !full)
+                                     : launch_rd_engine(make_rd_args(q), w, q->side);
   } else {
     P2pEngineArgs a{};
     a.epoch = q->ctrl + q->L.epoch;
@@ -905,7 +965,7 @@ static int launch_single(Request *q) {
     a.sys = q->sys_scope;
     a.xpart = q->xpart ? 1u : 0u;
     a.peer_part_bytes = q->peer_part_bytes;
-    rc = launch_p2p_engine(a, q->engine_warps, q->side);
+    rc = launch_p2p_engine(a, w, q->side);
   }
   if (rc) return rc;
   if ((rc = timing_end(q->tlog, q->side, tk))) return rc;
@@ -919,7 +979,7 @@ static int launch_single(Request *q) {
 // ordered after every member's producer work (their ev_fork events).
 // *launched tells whether that launch has happened (then q->ev_done of the
 // group leader marks completion).  block: wait (host) until it has.
-static int group_register(Request *q, bool block, bool *launched) {
+static int group_register(Request *q, bool block, cudaStream_t ws, bool *launched) {
   Request *ld = q->leader;
   GroupState &g = ld->gs;
   std::unique_lock<std::mutex> lk(g.mu);
@@ -930,38 +990,53 @@ static int group_register(Request *q, bool block, bool *launched) {
     g.launched = false;
   }
   if (!q->engine_registered) {
-    PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+    if (!q->forked || !q->overlap) PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
     q->engine_registered = true;
     g.pending++;
   }
   if (!g.launched && g.pending == (int)g.members.size()) {
-    for (Request *m : g.members) PC_CUDA(cudaStreamWaitEvent(q->side, m->ev_fork, 0));
+    bool full = true;
+    for (Request *m : g.members) {
+      PC_CUDA(cudaStreamWaitEvent(q->side, m->ev_fork, 0));
+      full = full && full_width(m);
+    }
+    const int w = engine_width(q, full);
     int rc, tk;
     if ((rc = timing_begin(g.tlog, q->side, &tk))) return rc;
     if (q->coll != PC_COLL_ALLREDUCE) {
       CollGroupArgs ga{};
       ga.n = (int)g.members.size();
       for (int k = 0; k < ga.n; ++k) ga.a[k] = make_coll_args(g.members[k]);
-      rc = launch_coll_engine_group(ga, q->engine_warps, q->side);
+      rc = launch_coll_engine_group(ga, w, q->side);
     } else if (q->algo == PC_ALGO_RING) {
       RingGroupArgs ga{};
       ga.n = (int)g.members.size();
       for (int k = 0; k < ga.n; ++k) ga.a[k] = make_ring_args(g.members[k]);
-      rc = launch_ring_engine_group(ga, q->engine_warps, q->side);
+      rc = launch_ring_engine_group(ga, w, q->side);
     } else if (q->algo == PC_ALGO_DIRECT) {
       DirectGroupArgs ga{};
       ga.n = (int)g.members.size();
       for (int k = 0; k < ga.n; ++k) ga.a[k] = make_direct_args(g.members[k]);
-      rc = launch_direct_engine_group(ga, q->engine_warps, q->side);
+      rc = launch_direct_engine_group(ga, w, q->side, !full);
     } else {
       RdGroupArgs ga{};
       ga.n = (int)g.members.size();
       for (int k = 0; k < ga.n; ++k) ga.a[k] = make_rd_args(g.members[k]);
-      rc = launch_rd_engine_group(ga, q->engine_warps, q->side);
+      rc = launch_rd_engine_group(ga, w, q->side);
     }
     if (rc) return rc;
     if ((rc = timing_end(g.tlog, q->side, tk))) return rc;
     PC_CUDA(cudaEventRecord(g.ev, q->side));
+    // members that already waited on their own stream (before the group was
+    // complete) get their completion ordered there now (pc.h "In-process
+    // rank groups": work they enqueued between their wait and this launch is
+    // not covered)
+    for (Request *m : g.members)
+      if (m != q && m->join_pending) {
+        if (!ws || m->wait_stream != ws) PC_CUDA(cudaStreamWaitEvent(m->wait_stream, g.ev, 0));
+        m->joined_stream = m->wait_stream;
+        m->join_pending = false;
+      }
     g.launched = true;
     g.cv.notify_all();
   }
@@ -1117,7 +1192,8 @@ int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void
   }
   c->ranks = all;
   c->same_proc.assign(size, false);
-  int ew = INT32_MAX, dw = INT32_MAX;
+  int ew = INT32_MAX, dw = INT32_MAX, ow = INT32_MAX;
+  const double ofrac = std::min(1.0, std::max(0.0, env_double("PC_OVERLAP_FRAC", 0.5)));
   for (int q = 0; q < size; ++q) {
     const RankRec &r = all[q];
     if (r.magic != me.magic || r.size != size || r.rank != q || r.dry != me.dry) {
@@ -1134,10 +1210,14 @@ int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void
       const int wpb = kEngineBlock / 32;
       ew = std::min(ew, r.engine_warps / std::max(on_dev, 1) / wpb * wpb);
       dw = std::min(dw, r.direct_warps / std::max(on_dev, 1) / wpb * wpb);
+      // overlap width: at most ofrac of the SMs carry an engine CTA in total,
+      // so whole SMs stay free for the producer the engine waits on
+      ow = std::min(ow, (int)(r.sms * ofrac) / std::max(on_dev, 1) * wpb);
     }
   }
   c->engine_warps = c->dry ? 1184 : std::max(8, (int)env_long("PC_ENGINE_WARPS", ew));
   c->direct_warps = c->dry ? 592 : std::max(8, (int)env_long("PC_DIRECT_WARPS", dw));
+  c->overlap_warps = c->dry ? 592 : std::max(8, ow);
   if (!c->dry) {
     for (int q = 0; q < size; ++q) {
       if (q == rank || !c->same_proc[q] || all[q].device == cuda_device) continue;
@@ -1185,6 +1265,12 @@ int pc_comm_size(pc_comm_t comm, int *size) {
 int pc_comm_engine_warps(pc_comm_t comm, int *warps) {
   if (!comm || !warps) return PC_ERR_ARG;
   *warps = ((Comm *)comm)->engine_warps;
+  return 0;
+}
+
+int pc_comm_overlap_warps(pc_comm_t comm, int *warps) {
+  if (!comm || !warps) return PC_ERR_ARG;
+  *warps = ((Comm *)comm)->overlap_warps;
   return 0;
 }
 
@@ -1351,6 +1437,12 @@ int pc_start(pc_request_t req, pc_stream_t stream) {
   if (!q) return PC_ERR_ARG;
   if (q->active) return PC_ERR_STATE;
   Comm *c = q->comm;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (!c->dry) {
+    PC_CUDA(cudaSetDevice(c->device));
+    PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+  }
+  if (int rc = epoch_begin(q, (cudaStream_t)stream, cs != cudaStreamCaptureStatusNone)) return rc;
   q->epoch++;
   q->active = true;
   q->engine_launched = false;
@@ -1358,20 +1450,22 @@ int pc_start(pc_request_t req, pc_stream_t stream) {
   q->prepared_this_epoch = false;
   q->user_stream = (cudaStream_t)stream;
   if (c->dry) return 0;
-  PC_CUDA(cudaSetDevice(c->device));
   if (!q->ctrl) {
     int arc = alloc_ctrl(q);
     if (arc) return arc;
   }
-  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-  PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
   if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
   // Eager requests write the epoch with a stream memop (cheapest); once a
   // request has been captured into a CUDA graph its epoch is advanced on the
   // device, so replays produce new epochs without the host.
-  if (!q->graph_mode && c->memops) return stream_write_u32(c, (cudaStream_t)stream, q->ctrl + q->L.epoch, q->epoch);
-  q->graph_mode = true;
-  return launch_epoch_bump(q->ctrl + q->L.epoch, (cudaStream_t)stream);
+  int rc;
+  if (!q->graph_mode && c->memops) {
+    rc = stream_write_u32(c, (cudaStream_t)stream, q->ctrl + q->L.epoch, q->epoch);
+  } else {
+    q->graph_mode = true;
+    rc = launch_epoch_bump(q->ctrl + q->L.epoch, (cudaStream_t)stream);
+  }
+  return rc ? rc : fork_point(q, (cudaStream_t)stream);
 }
 
 int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
@@ -1408,6 +1502,7 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
       if (rc) return rc;
     }
     q->prepared_this_epoch = true;
+    if (int rc = fork_point(q, (cudaStream_t)stream)) return rc;
   }
   return 0;
 }
@@ -1417,22 +1512,33 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
 // instead of three; CUDA-graph capturable).
 int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream) {
   if (n < 1 || !reqs || n > kMaxPreadyAll) return PC_ERR_ARG;
+  // validate everything before any request is touched (no half-started batch)
+  int nrtr = 0;
   for (int i = 0; i < n; ++i) {
     Request *q = (Request *)reqs[i];
     if (!q) return PC_ERR_ARG;
+    for (int j = 0; j < i; ++j)
+      if (reqs[j] == reqs[i]) return PC_ERR_ARG;  // one epoch per request per call
     if (q->active) return PC_ERR_STATE;
     if (!q->exchanged) return PC_ERR_STATE;
     if (!q->matched) return PC_ERR_MATCH;
     if (pready && q->kind != PC_KIND_PALLREDUCE) return PC_ERR_ARG;
     if (q->comm->device != ((Request *)reqs[0])->comm->device || q->comm->dry != ((Request *)reqs[0])->comm->dry)
       return PC_ERR_ARG;
+    if (group_blocks_start(q)) return PC_ERR_STATE;
+    nrtr += (int)q->rtr_targets.size();
   }
   const bool dry = ((Request *)reqs[0])->comm->dry;
+  if (!dry && nrtr > kMaxCtl) return PC_ERR_UNSUPPORTED;
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-  if (!dry) PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+  if (!dry) {
+    PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
+    PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+  }
   EpochAllArgs a{};
   for (int i = 0; i < n; ++i) {
     Request *q = (Request *)reqs[i];
+    if (int rc = epoch_begin(q, (cudaStream_t)stream, cs != cudaStreamCaptureStatusNone)) return rc;
     if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
     q->epoch++;
     q->active = true;
@@ -1444,7 +1550,6 @@ int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream) {
     const int k = a.n++;
     a.epoch[k] = q->ctrl + q->L.epoch;
     for (auto &t : q->rtr_targets) {
-      if (a.nrtr == kMaxCtl) return PC_ERR_UNSUPPORTED;
       a.rtr_dst[a.nrtr] = t.first + q->L.rtr + t.second;
       a.rtr_req[a.nrtr] = (uint8_t)k;
       if (q->sys_scope) a.rtr_sysmask |= 1ull << a.nrtr;
@@ -1457,8 +1562,13 @@ int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream) {
   }
   if (dry) return 0;
   a.pready = pready ? 1 : 0;
-  PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
-  return launch_epoch_all(a, (cudaStream_t)stream);
+  if (int rc = launch_epoch_all(a, (cudaStream_t)stream)) return rc;
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    q->host_ready_all = pready != 0;
+    if (int rc = fork_point(q, (cudaStream_t)stream)) return rc;
+  }
+  return 0;
 }
 
 // MPI_Startall: one device kernel advances the epochs of all n requests.
@@ -1467,15 +1577,26 @@ int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream) {
   for (int i = 0; i < n; ++i) {
     Request *q = (Request *)reqs[i];
     if (!q) return PC_ERR_ARG;
+    for (int j = 0; j < i; ++j)
+      if (reqs[j] == reqs[i]) return PC_ERR_ARG;  // one epoch per request per call
     if (q->active) return PC_ERR_STATE;
     if (q->comm->device != ((Request *)reqs[0])->comm->device || q->comm->dry != ((Request *)reqs[0])->comm->dry)
       return PC_ERR_ARG;
+    if (group_blocks_start(q)) return PC_ERR_STATE;
   }
+  const bool dry = n == 0 || ((Request *)reqs[0])->comm->dry;
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-  if (n > 0 && !((Request *)reqs[0])->comm->dry) PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+  if (!dry) {
+    PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
+    PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+    for (int i = 0; i < n; ++i)  // device resources first: nothing below can fail half-way on allocation
+      if (int arc = alloc_ctrl((Request *)reqs[i])) return arc;
+  }
   CtlArgs a{};
+  int first = 0;  // requests [first, i] are in the pending kernel
   for (int i = 0; i < n; ++i) {
     Request *q = (Request *)reqs[i];
+    if (int rc = epoch_begin(q, (cudaStream_t)stream, cs != cudaStreamCaptureStatusNone)) return rc;
     if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
     q->epoch++;
     q->active = true;
@@ -1483,24 +1604,16 @@ int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream) {
     q->engine_registered = false;
     q->prepared_this_epoch = false;
     q->user_stream = (cudaStream_t)stream;
-    if (q->comm->dry) continue;
-    if (!q->ctrl) {
-      PC_CUDA(cudaSetDevice(q->comm->device));
-      int arc = alloc_ctrl(q);
-      if (arc) return arc;
-    }
+    if (dry) continue;
     a.epoch[a.n] = q->ctrl + q->L.epoch;
     a.dst[a.n] = nullptr;
-    if (++a.n == kMaxCtl) {
-      PC_CUDA(cudaSetDevice(q->comm->device));
-      int rc = launch_ctl(a, (cudaStream_t)stream);
-      if (rc) return rc;
+    if (++a.n == kMaxCtl || i == n - 1) {
+      if (int rc = launch_ctl(a, (cudaStream_t)stream)) return rc;
+      for (int k = first; k <= i; ++k)
+        if (int rc = fork_point((Request *)reqs[k], (cudaStream_t)stream)) return rc;
       a.n = 0;
+      first = i + 1;
     }
-  }
-  if (a.n) {
-    PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
-    return launch_ctl(a, (cudaStream_t)stream);
   }
   return 0;
 }
@@ -1518,6 +1631,7 @@ int pc_pbuf_prepare_all(int n, pc_request_t *reqs, pc_stream_t stream) {
     if (!q->matched) return PC_ERR_MATCH;
   }
   CtlArgs a{};
+  std::vector<Request *> prepared;
   for (int i = 0; i < n; ++i) {
     Request *q = (Request *)reqs[i];
     q->user_stream = (cudaStream_t)stream;
@@ -1534,11 +1648,14 @@ int pc_pbuf_prepare_all(int n, pc_request_t *reqs, pc_stream_t stream) {
       }
     }
     q->prepared_this_epoch = true;
+    prepared.push_back(q);
   }
   if (a.n) {
     PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
-    return launch_ctl(a, (cudaStream_t)stream);
+    if (int rc = launch_ctl(a, (cudaStream_t)stream)) return rc;
   }
+  for (Request *q : prepared)
+    if (int rc = fork_point(q, (cudaStream_t)stream)) return rc;
   return 0;
 }
 
@@ -1596,12 +1713,12 @@ int pc_prequest_free(pc_prequest_t *preq) {
 
 // Make sure this epoch's engine is (or will be) launched; *ev = the event that
 // completes with it, or null when a co-located group is still incomplete.
-static int ensure_engine(Request *q, bool block, cudaEvent_t *ev) {
+static int ensure_engine(Request *q, bool block, cudaStream_t ws, cudaEvent_t *ev) {
   *ev = nullptr;
   if (!needs_engine(q)) return 0;
   if (q->leader) {
     bool launched = false;
-    int rc = group_register(q, block, &launched);
+    int rc = group_register(q, block, ws, &launched);
     if (launched) *ev = q->leader->gs.ev;
     return rc;
   }
@@ -1628,12 +1745,17 @@ static int wait_common(Request *q, cudaStream_t s, bool host) {
   if (engine) {
     if (q->kind == PC_KIND_PSEND && !q->has_preq) return PC_ERR_STATE;
     cudaEvent_t ev = nullptr;
-    if ((rc = ensure_engine(q, host, &ev))) return rc;
+    if ((rc = ensure_engine(q, host, host ? nullptr : s, &ev))) return rc;
     if (host) {
       if (!ev) return PC_ERR_STATE;
       PC_CUDA(cudaEventSynchronize(ev));
+      q->joined_stream = kHostJoined;
     } else if (ev) {
       PC_CUDA(cudaStreamWaitEvent(s, ev, 0));
+      q->joined_stream = s;
+    } else {
+      q->join_pending = true;  // the group's last wait joins it on s
+      q->wait_stream = s;
     }
     // (co-located group not complete yet: the last local rank's wait launches
     //  the grouped engine on its stream; see pc.h "In-process rank groups")
@@ -1697,14 +1819,23 @@ int pc_waitall_on_stream(int n, pc_request_t *reqs, pc_stream_t stream) {
   }
   if (fused.empty()) return 0;
   PC_CUDA(cudaSetDevice(fused[0]->comm->device));
+  // The fused grid stays within what is co-resident at once (4 spinning
+  // 256-thread blocks per SM, as one recv_wait kernel): several LL receives
+  // share that budget (their bodies are grid-stride over their block range).
+  const int budget = 4 * std::max(fused[0]->comm->sms, 1) - kMaxWaitAll;
   for (size_t g0 = 0; g0 < fused.size(); g0 += kMaxWaitAll) {
     WaitAllArgs a{};
     a.block_start[0] = 0;
+    int want[kMaxWaitAll], total = 0;
     for (size_t k = g0; k < fused.size() && a.n < kMaxWaitAll; ++k) {
       fill_prequest(fused[k], &a.q[a.n]);
-      const int nb = fused[k]->kind == PC_KIND_PSEND ? 1 : recv_wait_blocks(a.q[a.n]);
-      a.block_start[a.n + 1] = a.block_start[a.n] + nb;
+      want[a.n] = fused[k]->kind == PC_KIND_PSEND ? 1 : recv_wait_blocks(a.q[a.n]);
+      total += want[a.n];
       ++a.n;
+    }
+    for (int k = 0; k < a.n; ++k) {
+      const int nb = total <= budget ? want[k] : std::max(1, (int)((int64_t)want[k] * budget / total));
+      a.block_start[k + 1] = a.block_start[k] + nb;
     }
     if (int rc = launch_wait_all(a, s)) return rc;
     for (size_t k = g0; k < g0 + (size_t)a.n; ++k) fused[k]->active = false;
@@ -1802,7 +1933,7 @@ int pc_test(pc_request_t req, int *flag) {
       *flag = 0;
       return 0;
     }
-    if ((rc = ensure_engine(q, false, &ev))) return rc;
+    if ((rc = ensure_engine(q, false, nullptr, &ev))) return rc;
     if (!ev) {
       *flag = 0;
       return 0;
@@ -1858,7 +1989,10 @@ int pc_test(pc_request_t req, int *flag) {
     return erc;
   }
   *flag = done ? 1 : 0;
-  if (done) q->active = false;
+  if (done) {
+    q->active = false;
+    q->joined_stream = kHostJoined;
+  }
   return 0;
 }
 
@@ -1883,7 +2017,15 @@ int pc_preadyall(int n, pc_request_t *reqs, pc_stream_t stream) {
   }
   if (a.n) {
     PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
-    return launch_pready_all(a, (cudaStream_t)stream);
+    if (int rc = launch_pready_all(a, (cudaStream_t)stream)) return rc;
+  }
+  // every partition is ready once this kernel ran: the engine may start after
+  // it at full width (no producer left to overlap)
+  for (int i = 0; i < n; ++i) {
+    Request *q = (Request *)reqs[i];
+    if (q->comm->dry) continue;
+    q->host_ready_all = true;
+    if (int rc = fork_point(q, (cudaStream_t)stream)) return rc;
   }
   return 0;
 }
@@ -1898,7 +2040,12 @@ int pc_pready_range(int lo, int hi, pc_request_t req, pc_stream_t stream) {
   PC_CUDA(cudaSetDevice(q->comm->device));
   pc_prequest_t p;
   fill_prequest(q, &p);
-  return launch_pready_range(p, lo, hi, (cudaStream_t)stream);
+  if (int rc = launch_pready_range(p, lo, hi, (cudaStream_t)stream)) return rc;
+  if (lo == 0 && hi == q->partitions - 1) {  // every partition: as pc_preadyall
+    q->host_ready_all = true;
+    return fork_point(q, (cudaStream_t)stream);
+  }
+  return 0;
 }
 
 int pc_pready(int partition, pc_request_t req, pc_stream_t stream) {
@@ -1966,7 +2113,32 @@ int pc_request_match(pc_request_t req, int *peer, int *peer_request_index) {
   return 0;
 }
 
+int pc_request_peer_buffer(pc_request_t req, int j, void **ptr) {
+  Request *q = (Request *)req;
+  if (!q || !ptr) return PC_ERR_ARG;
+  if (!q->exchanged || !q->matched) return PC_ERR_STATE;
+  *ptr = nullptr;
+  if (q->kind == PC_KIND_PSEND) {
+    if (j != 0) return PC_ERR_ARG;
+    *ptr = q->peer_buf;
+  } else if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT) {
+    if (j < 0 || j >= q->comm->size - 1) return PC_ERR_ARG;
+    *ptr = q->nb_buf[j];
+  } else {
+    return PC_ERR_UNSUPPORTED;
+  }
+  return 0;
+}
+
 uint64_t pc_launch_count(void) { return launch_count(); }
+
+int pc_request_set_overlap(pc_request_t req, int on) {
+  Request *q = (Request *)req;
+  if (!q) return PC_ERR_ARG;
+  if (q->active) return PC_ERR_STATE;
+  q->overlap = on != 0;
+  return 0;
+}
 
 int pc_request_set_timing(pc_request_t req, int on) {
   Request *q = (Request *)req;

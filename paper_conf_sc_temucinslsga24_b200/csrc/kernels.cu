@@ -299,8 +299,8 @@ int launch_rd_engine(const RdArgs &a, int warps, cudaStream_t s) {
   return dispatch(a.dtype, a.op, [&](auto E) { return decltype(E)::rd(a, warps, s); });
 }
 
-int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s) {
-  return dispatch(a.dtype, a.op, [&](auto E) { return decltype(E)::direct(a, warps, s); });
+int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s, bool thin) {
+  return dispatch(a.dtype, a.op, [&](auto E) { return decltype(E)::direct(a, warps, s, thin); });
 }
 
 // allgather / broadcast move bytes only: any instantiation serves (fp32 sum)
@@ -341,14 +341,14 @@ int launch_rd_engine_group(const RdGroupArgs &g, int warps, cudaStream_t s) {
   return dispatch(g.a[0].dtype, g.a[0].op, [&](auto E) { return decltype(E)::rd_group(h, blocks, s); });
 }
 
-int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t s) {
+int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t s, bool thin) {
   DirectGroupArgs h = g;
   int blocks = 0;
   for (int k = 0; k < g.n; ++k) {
     h.block_start[k] = blocks;
     blocks += grid_for(warps, g.a[k].nunits);
   }
-  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto E) { return decltype(E)::direct_group(h, blocks, s); });
+  return dispatch(g.a[0].dtype, g.a[0].op, [&](auto E) { return decltype(E)::direct_group(h, blocks, s, thin); });
 }
 
 int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {

@@ -159,6 +159,20 @@ struct Request {
   bool engine_launched = false;
   bool engine_registered = false;
   bool graph_mode = false;  // captured into a CUDA graph: epochs advance on the device only
+  // Producer/engine overlap (§8(a) a6): ev_fork is recorded at the
+  // epoch's control points (start / pbuf_prepare / epoch_all / host Pready of
+  // every partition), so the engine — still ENQUEUED at the wait, after the
+  // user's producer — starts as soon as the epoch is set up and reduces each
+  // partition while the producer is still running.
+  bool forked = false;          // ev_fork recorded at a control point of this epoch
+  bool host_ready_all = false;  // every partition was made ready by a host-side op before ev_fork
+  bool overlap = true;          // pc_request_set_overlap (0: fork at the wait, the round-1 order)
+  // stream on which the previous epoch's completion is ordered (null: host
+  // observed it); a later epoch's control op on another stream first waits
+  // for that completion (the engine reads the epoch word at entry)
+  cudaStream_t joined_stream = nullptr;
+  bool join_pending = false;    // group member waited on a stream before the group engine launched
+  cudaStream_t wait_stream = nullptr;
   bool matched = false;
   Request *leader = nullptr;  // co-located group leader (allreduce), or null
   GroupState gs;
@@ -232,6 +246,8 @@ struct Comm {
   std::vector<bool> same_proc;
   int engine_warps = 0;  // agreed (min over ranks)
   int direct_warps = 0;  // the same for the DIRECT allreduce engines
+  int overlap_warps = 0; // per-rank engine width when the engine may overlap a producer:
+                         // whole CTAs, <= PC_OVERLAP_FRAC of the SMs per GPU in total
   int sms = 0;
   std::vector<Request *> reqs;
   std::map<std::tuple<int, int, int>, int> post_seq;  // (kind, peer, tag) -> next seq
@@ -356,8 +372,9 @@ struct CollGroupArgs {
 };
 int launch_coll_engine(const CollArgs &a, int warps, cudaStream_t s);
 int launch_coll_engine_group(const CollGroupArgs &g, int warps, cudaStream_t s);
-int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s);
-int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t s);
+// thin: the 2-CTA/SM variant used while the engine overlaps producer kernels
+int launch_direct_engine(const DirectArgs &a, int warps, cudaStream_t s, bool thin = false);
+int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t s, bool thin = false);
 struct RdGroupArgs {
   int n;
   int block_start[kMaxLocal];

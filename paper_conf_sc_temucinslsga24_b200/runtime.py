@@ -84,6 +84,8 @@ class Comm:
         check(_lib.pc().pc_comm_size(handle, C.byref(s)), "pc_comm_size")
         check(_lib.pc().pc_comm_engine_warps(handle, C.byref(w)), "pc_comm_engine_warps")
         self.rank, self.size, self.engine_warps = r.value, s.value, w.value
+        check(_lib.pc().pc_comm_overlap_warps(handle, C.byref(w)), "pc_comm_overlap_warps")
+        self.overlap_warps = w.value
         self.requests: list[Request] = []
 
     @staticmethod
@@ -272,6 +274,18 @@ class Request:
         check(_lib.pc().pc_request_words(self.handle, self.WORDS[which], offset, n, out.ctypes.data),
               "pc_request_words")
         return out[:n]
+
+    def peer_buffer(self, j: int = 0) -> int:
+        """pc_request_peer_buffer: peer-mapped address of a peer's receive
+        buffer (send: the receiver's; DIRECT collective: peer (r+1+j) mod P)."""
+        p = C.c_void_p()
+        check(_lib.pc().pc_request_peer_buffer(self.handle, j, C.byref(p)), "pc_request_peer_buffer")
+        return p.value or 0
+
+    def set_overlap(self, on: bool = True):
+        """pc_request_set_overlap: fork the engine at the epoch's control calls
+        (default, overlaps the producer) or at the wait (no overlap)."""
+        check(_lib.pc().pc_request_set_overlap(self.handle, int(on)), "pc_request_set_overlap")
 
     def set_timing(self, on: bool = True):
         check(_lib.pc().pc_request_set_timing(self.handle, int(on)), "pc_request_set_timing")

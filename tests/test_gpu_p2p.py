@@ -620,11 +620,13 @@ def test_fig3_single_block_pready(t, mode):
 
 @pytest.mark.parametrize("gran", [apps.GRAN_THREAD, apps.GRAN_WARP])
 @pytest.mark.parametrize("agg", [1024, 5000, "all"])
-@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE])
+@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE, pc.COPY_LL, pc.COPY_HOST])
 def test_two_level_aggregation_counters(gran, agg, copy):
     """g >= 1024: two-level counting (reading R32) — sub-counters of 256
     partitions, ragged last sub-group (g = 5000) and last transport partition;
-    byte-exact vs O1 over several epochs."""
+    byte-exact vs O1 over several epochs.  Every copy mode goes through the
+    counters: INLINE / ENGINE (publish / mark_ready), LL (ll_account, 4 MiB
+    within the LL cap) and HOST (mark_ready into pinned host memory)."""
     n = 1 << 20
     partitions = n // GRAN_ELEMS[gran]
     run_vecadd(n, gran, partitions if agg == "all" else min(agg, partitions), copy, epochs=3)

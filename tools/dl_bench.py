@@ -2,8 +2,10 @@
 ranks: per step each rank computes the BCE gradient of a ResNet-50-sized flat
 buffer (25.56 M fp32) and the ranks allreduce it; pc_startall +
 pc_pbuf_prepare_all are inside the step.  Modes: pready (the producer
-Preadies each partition from the kernel), serial (producer, then host Pready
-of all partitions), and the two halves alone.
+Preadies each partition from the kernel; the engine overlaps the producers),
+pready_nooverlap (the same with the engine forked at the wait), serial
+(producers, then host Pready of all partitions), and the two halves alone.
+Each rank's producer runs on its own stream.
 JSON lines to stdout; CUDA-event timing on the control stream."""
 import json
 import os
@@ -43,14 +45,24 @@ def run(P, L, algo, modes):
     p = [(0.02 + 0.96 * torch.rand(n, device="cuda", generator=gen)) for _ in range(P)]
     y = [torch.randint(0, 2, (n,), device="cuda", generator=gen).float() for _ in range(P)]
     dl = apps.DLProxy(cs, Np, L, algo, p, y)
+    dl_no = None
     out = []
     for mode in modes:
         if mode in ("pready", "serial"):
             ms = timeit(lambda: dl.step(mode), dl.ctl)
-        elif mode == "bce_only":
+        elif mode == "pready_nooverlap":  # engine forked at the wait (no producer/engine concurrency)
+            if dl_no is None:
+                dl_no = apps.DLProxy(cs, Np, L, algo, p, y, overlap=False)
+            ms = timeit(lambda: dl_no.step("pready"), dl_no.ctl)
+        elif mode == "bce_only":  # the producers alone, concurrently on their per-rank streams
             def f():
+                dl.ev_ctl.record(dl.ctl)
                 for r in range(P):
-                    apps.bce_grad(p[r], y[r], dl.g[r], Np, L, float(n), None, stream=dl.ctl)
+                    dl.pst[r].wait_event(dl.ev_ctl)
+                    apps.bce_grad(p[r], y[r], dl.g[r], Np, L, float(n), None, stream=dl.pst[r])
+                    dl.ev_p[r].record(dl.pst[r])
+                for r in range(P):
+                    dl.ctl.wait_event(dl.ev_p[r])
             ms = timeit(f, dl.ctl)
         else:  # allreduce only (host Pready of every partition)
             def f():
@@ -66,6 +78,8 @@ def run(P, L, algo, modes):
                     "ms_per_step": ms, "grad_GB_per_s_all_ranks": P * 4 * n / (ms / 1e3) / 1e9})
         print(json.dumps(out[-1]), flush=True)
     dl.free()
+    if dl_no is not None:
+        dl_no.free()
     for c in cs:
         c.destroy()
     g.destroy()
