@@ -36,6 +36,13 @@
  * Returns 0, or a PC_ERR_* code that is also recorded in the sticky error word
  * (bad partition, duplicate Pready detected by counter overshoot).
  *
+ * INLINE allreduce (pc_prequest_create(..., PC_COPY_INLINE) on a DIRECT
+ * allreduce, reading R33): the Pready that completes a partition on the last
+ * rank folds it for every rank.  The fold is compiled into these bindings only
+ * in translation units built with -DPC_INLINE_ALLREDUCE (kernels that Pready
+ * into such a request), so producers of other requests keep their register
+ * allocation; elsewhere a Pready on an INLINE allreduce reports PC_DEV_ERR_ARG.
+ *
  * pc_parrived: 1 iff the partition is complete in this epoch (receive: its
  * bytes are in recvbuf; allreduce: its final result is in recvbuf).
  * It is an ld.acquire.sys of a flag in the caller's OWN memory (written
@@ -48,6 +55,7 @@
 
 #include <stdint.h>
 
+#include "pc_ops.cuh"
 #include "pc_prequest.h"
 
 typedef struct pc_prequest_s pc_prequest_t;
@@ -104,6 +112,11 @@ PC_DEVICE void st_release_gpu(uint32_t *p, uint32_t v) {
 PC_DEVICE uint32_t atom_add_acq_rel_gpu(uint32_t *p, uint32_t v) {
   uint32_t old;
   asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+PC_DEVICE uint32_t atom_add_acq_rel_sys(uint32_t *p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.acq_rel.sys.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
   return old;
 }
 PC_DEVICE void red_add_release_gpu(uint32_t *p, uint32_t v) {
@@ -492,6 +505,145 @@ PC_DEVICE void ll_account(const pc_prequest_t &q, int t, uint32_t add, uint32_t 
 
 /* ------------------------------------------------------------------ Pready */
 
+/* ------------------------------------------------------------ INLINE allreduce
+ * (reading R33: "the Pready could also trigger the computation", the
+ * paper's Kernel Copy applied to the collective).  Every rank's Pready of user
+ * partition u adds 1 to u's arrival counter in rank 0's control block
+ * (acq_rel: the caller's data writes are released; the last arrival acquires
+ * every rank's).  The contribution that completes u (target e*P) — the last
+ * rank to produce u — checks that every peer posted ready-to-receive for
+ * epoch e (implied by causality: each peer's Pready of u follows its
+ * Pbuf_prepare), folds u over the P send buffers in rank order (R25: the
+ * DIRECT schedule's bits, oracle O6), stores the result into all P recvbufs,
+ * fences once and writes done[u] = e on every rank.  No engine, no spinning
+ * kernel: the reduction runs in the producer block that completed the data,
+ * while the data is still in L2. */
+namespace pc_detail {
+
+PC_DEVICE bool ar_arrive(const pc_prequest_t &q, int u, uint32_t e) {
+  uint32_t *c = q.ar_tab->cnt + u;
+  const uint32_t old = q.sys_scope ? atom_add_acq_rel_sys(c, 1u) : atom_add_acq_rel_gpu(c, 1u);
+  const int32_t d = (int32_t)(e * (uint32_t)q.nranks - old);
+  if (d <= 0) {  // more than P arrivals in this epoch: a duplicate Pready
+    set_error(q.err, PC_DEV_ERR_DEVICE, u);
+    return false;
+  }
+  return d == 1;
+}
+
+/* Every peer posted ready-to-receive for epoch e: the P-1 words are read
+ * relaxed, all in flight at once (acquire loads would serialise), then one
+ * fence gives the acquire; only a word still behind is spun on. */
+PC_DEVICE bool ar_rtr_ok(const pc_prequest_t &q, int u, uint32_t e) {
+  const uint32_t *w = q.ar_tab->rtr;
+  uint32_t v[PC_AR_MAX - 1];
+#pragma unroll
+  for (int j = 0; j < PC_AR_MAX - 1; ++j)
+    if (j < q.nranks - 1) v[j] = ld_relaxed_sys(w + j);
+#pragma unroll
+  for (int j = 0; j < PC_AR_MAX - 1; ++j)
+    if (j < q.nranks - 1 && !reached(v[j], e)) {
+      const bool ok = q.sys_scope ? spin_geq<true>(w + j, e, q.err, q.timeout_ms, u)
+                                  : spin_geq<false>(w + j, e, q.err, q.timeout_ms, u);
+      if (!ok) return false;
+    }
+  fence_scope(q.sys_scope);
+  return true;
+}
+
+template <int DT, int OP>
+PC_DEVICE void ar_scalar(const pc_ar_tab_s *tab, int P, uint64_t b) {
+  using O = pc_ops::Op<DT, OP>;
+  using T = typename O::T;
+  T acc = __ldcg(reinterpret_cast<const T *>(tab->send[0] + b));
+  for (int k = 1; k < P; ++k) acc = O::f(acc, __ldcg(reinterpret_cast<const T *>(tab->send[k] + b)));
+  for (int k = 0; k < P; ++k) *reinterpret_cast<T *>(tab->recv[k] + b) = acc;
+}
+
+template <int DT, int OP>
+PC_DEVICE void ar_fold_t(const pc_ar_tab_s *tab, int P, uint64_t off, uint64_t nbytes, uint32_t idx,
+                         uint32_t n) {
+  using O = pc_ops::Op<DT, OP>;
+  using T = typename O::T;
+  // 16-B aligned bases (pc_pallreduce_init), the same offset in every buffer:
+  // scalar head to the 16-B boundary, 16-B body, scalar tail
+  uint64_t head = (16 - (off & 15)) & 15;
+  if (head > nbytes) head = nbytes;
+  const uint64_t nv = (nbytes - head) / 16;
+  const uint64_t body_end = head + nv * 16;
+  for (uint64_t b = (uint64_t)idx * sizeof(T); b < head; b += (uint64_t)n * sizeof(T))
+    ar_scalar<DT, OP>(tab, P, off + b);
+  for (uint64_t b = body_end + (uint64_t)idx * sizeof(T); b < nbytes; b += (uint64_t)n * sizeof(T))
+    ar_scalar<DT, OP>(tab, P, off + b);
+  const uint8_t *s0 = tab->send[0] + off + head, *s1 = tab->send[1] + off + head, *s2 = tab->send[2] + off + head,
+                *s3 = tab->send[3] + off + head, *s4 = tab->send[4] + off + head, *s5 = tab->send[5] + off + head,
+                *s6 = tab->send[6] + off + head, *s7 = tab->send[7] + off + head;
+  // destination pointers in registers too (stores could alias the table, so a
+  // pointer read inside the loop would be re-issued before every store)
+  uint8_t *d0 = tab->recv[0] + off + head, *d1 = tab->recv[1] + off + head, *d2 = tab->recv[2] + off + head,
+          *d3 = tab->recv[3] + off + head, *d4 = tab->recv[4] + off + head, *d5 = tab->recv[5] + off + head,
+          *d6 = tab->recv[6] + off + head, *d7 = tab->recv[7] + off + head;
+  for (uint64_t v = idx; v < nv; v += n) {
+    const uint64_t o = v * 16;
+    uint4 x0 = __ldcg(reinterpret_cast<const uint4 *>(s0 + o)), x1, x2, x3, x4, x5, x6, x7;
+    if (P > 1) x1 = __ldcg(reinterpret_cast<const uint4 *>(s1 + o));
+    if (P > 2) x2 = __ldcg(reinterpret_cast<const uint4 *>(s2 + o));
+    if (P > 3) x3 = __ldcg(reinterpret_cast<const uint4 *>(s3 + o));
+    if (P > 4) x4 = __ldcg(reinterpret_cast<const uint4 *>(s4 + o));
+    if (P > 5) x5 = __ldcg(reinterpret_cast<const uint4 *>(s5 + o));
+    if (P > 6) x6 = __ldcg(reinterpret_cast<const uint4 *>(s6 + o));
+    if (P > 7) x7 = __ldcg(reinterpret_cast<const uint4 *>(s7 + o));
+    uint4 acc = x0;  // rank order (R25)
+    if (P > 1) acc = pc_ops::vop<DT, OP>(acc, x1);
+    if (P > 2) acc = pc_ops::vop<DT, OP>(acc, x2);
+    if (P > 3) acc = pc_ops::vop<DT, OP>(acc, x3);
+    if (P > 4) acc = pc_ops::vop<DT, OP>(acc, x4);
+    if (P > 5) acc = pc_ops::vop<DT, OP>(acc, x5);
+    if (P > 6) acc = pc_ops::vop<DT, OP>(acc, x6);
+    if (P > 7) acc = pc_ops::vop<DT, OP>(acc, x7);
+    *reinterpret_cast<uint4 *>(d0 + o) = acc;
+    if (P > 1) *reinterpret_cast<uint4 *>(d1 + o) = acc;
+    if (P > 2) *reinterpret_cast<uint4 *>(d2 + o) = acc;
+    if (P > 3) *reinterpret_cast<uint4 *>(d3 + o) = acc;
+    if (P > 4) *reinterpret_cast<uint4 *>(d4 + o) = acc;
+    if (P > 5) *reinterpret_cast<uint4 *>(d5 + o) = acc;
+    if (P > 6) *reinterpret_cast<uint4 *>(d6 + o) = acc;
+    if (P > 7) *reinterpret_cast<uint4 *>(d7 + o) = acc;
+  }
+}
+
+/* Fold partition u by n cooperating participants (index idx).  Not inlined:
+ * the fold's P-way loads would otherwise raise the register allocation of
+ * every producer kernel that calls a Pready binding (a call on the rare
+ * completing path costs nothing measurable). */
+#ifdef PC_INLINE_ALLREDUCE
+static __device__ __noinline__ void ar_fold(const pc_prequest_t &q, int u, uint32_t idx, uint32_t n) {
+  const pc_ar_tab_s *t = q.ar_tab;
+  const uint64_t off = (uint64_t)u * q.part_bytes, nb = q.part_bytes;
+  const int P = q.nranks;
+#define PC_AR_CASE(DTV)                                      \
+  if (q.op == 0) ar_fold_t<DTV, 0>(t, P, off, nb, idx, n);   \
+  else if (q.op == 1) ar_fold_t<DTV, 1>(t, P, off, nb, idx, n); \
+  else ar_fold_t<DTV, 2>(t, P, off, nb, idx, n);
+  switch (q.dtype) {
+    case 0: PC_AR_CASE(0); break;
+    case 1: PC_AR_CASE(1); break;
+    case 3: PC_AR_CASE(3); break;
+    default: PC_AR_CASE(4); break;
+  }
+#undef PC_AR_CASE
+}
+#endif
+
+/* After the fold (every participant's stores ordered before by a barrier):
+ * one cumulative fence, then done[u] = e on every rank. */
+PC_DEVICE void ar_publish(const pc_prequest_t &q, int u, uint32_t e) {
+  fence_scope(q.sys_scope);
+  for (int k = 0; k < q.nranks; ++k) st_relaxed_sys(q.ar_tab->done[k] + u, e);
+}
+
+}  // namespace pc_detail
+
 /* Thread granularity: any subset of threads, each for its own partition.
  * INLINE: every lane pushes its own partition's bytes, lanes of the warp that
  * share a transport partition are combined (__match_any_sync) into one counter
@@ -505,8 +657,22 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
     return PC_DEV_ERR_ARG;
   }
   if (preq.kind == PC_KIND_PALLREDUCE) {
-    st_release_gpu(preq.ready + partition, epoch_of(preq));
+    if (!preq.ar_tab) {
+      st_release_gpu(preq.ready + partition, epoch_of(preq));
+      return 0;
+    }
+#ifdef PC_INLINE_ALLREDUCE
+    const uint32_t e = epoch_of(preq);  // INLINE (R33): this thread alone folds if it completes u
+    if (ar_arrive(preq, partition, e)) {
+      if (!ar_rtr_ok(preq, partition, e)) return PC_DEV_ERR_TIMEOUT;
+      ar_fold(preq, partition, 0, 1);
+      ar_publish(preq, partition, e);
+    }
     return 0;
+#else
+    set_error(preq.err, PC_DEV_ERR_ARG, partition);  // INLINE allreduce needs -DPC_INLINE_ALLREDUCE
+    return PC_DEV_ERR_ARG;
+#endif
   }
   const unsigned mask = __activemask();
   const uint32_t lane = lane_id();
@@ -592,9 +758,32 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
     return PC_DEV_ERR_ARG;
   }
   if (preq.kind == PC_KIND_PALLREDUCE) {
-    if (lane == 0) st_release_gpu(preq.ready + partition, epoch_of(preq));
+    if (!preq.ar_tab) {
+      if (lane == 0) st_release_gpu(preq.ready + partition, epoch_of(preq));
+      __syncwarp(full);
+      return 0;
+    }
+#ifdef PC_INLINE_ALLREDUCE
+    int st = 0;  // INLINE (R33): 1 = this warp completed u and folds it, -1 = RTR timeout
+    uint32_t e = 0;
+    if (lane == 0) {
+      e = epoch_of(preq);
+      st = ar_arrive(preq, partition, e) ? (ar_rtr_ok(preq, partition, e) ? 1 : -1) : 0;
+    }
+    st = __shfl_sync(full, st, 0);
+    e = __shfl_sync(full, e, 0);
+    if (st == 1) {
+      ar_fold(preq, partition, lane, 32);
+      __syncwarp(full);
+      if (lane == 0) ar_publish(preq, partition, e);
+    }
     __syncwarp(full);
-    return 0;
+    return st < 0 ? PC_DEV_ERR_TIMEOUT : 0;
+#else
+    if (lane == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);  // needs -DPC_INLINE_ALLREDUCE
+    __syncwarp(full);
+    return PC_DEV_ERR_ARG;
+#endif
   }
   const int t = partition / preq.agg;
   if (preq.copy == 2) {  // LL: every lane loads its line, reads the epoch and stores (no broadcast)
@@ -671,8 +860,29 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
   }
   __syncthreads();  // the block's data writes are complete
   if (preq.kind == PC_KIND_PALLREDUCE) {
-    if (tid == 0) st_release_gpu(preq.ready + partition, epoch_of(preq));
-    return 0;
+    if (!preq.ar_tab) {
+      if (tid == 0) st_release_gpu(preq.ready + partition, epoch_of(preq));
+      return 0;
+    }
+#ifdef PC_INLINE_ALLREDUCE
+    if (tid == 0) {  // INLINE (R33): s_ok 1 = this block completed u and folds it, -1 = RTR timeout
+      const uint32_t e = epoch_of(preq);
+      s_e = e;
+      s_ok = ar_arrive(preq, partition, e) ? (ar_rtr_ok(preq, partition, e) ? 1 : -1) : 0;
+    }
+    __syncthreads();
+    const int st = s_ok;
+    if (st == 1) {
+      ar_fold(preq, partition, tid, nthr);
+      __syncthreads();  // every thread's stores, then ONE cumulative fence + the done words
+      if (tid == 0) ar_publish(preq, partition, s_e);
+    }
+    __syncthreads();  // s_e / s_ok are reused by the block's next Pready
+    return st < 0 ? PC_DEV_ERR_TIMEOUT : 0;
+#else
+    if (tid == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);  // needs -DPC_INLINE_ALLREDUCE
+    return PC_DEV_ERR_ARG;
+#endif
   }
   const int t = partition / preq.agg;
   if (preq.copy == 2) {  // LL: every thread pushes its lines
@@ -747,7 +957,8 @@ PC_DEVICE int pc_parrived(pc_prequest_t preq, int partition) {
   if (partition < 0 || partition >= (ag ? preq.nranks * preq.partitions : preq.partitions)) return 0;
   const uint32_t e = epoch_of(preq);
   if (ag) return ag_arrived(preq, partition, e) ? 1 : 0;
-  if (preq.kind == PC_KIND_PALLREDUCE) return reached(ld_acquire_gpu(preq.done + partition), e * preq.done_mul);
+  if (preq.kind == PC_KIND_PALLREDUCE)  // INLINE: done[u] written by the folding rank (maybe another GPU)
+    return reached(ld_acquire_scope(preq.done + partition, preq.sys_scope), e * preq.done_mul);
   if (preq.kind == PC_KIND_PSEND) {
     const int t = partition / preq.agg;
     return reached(ld_acquire_gpu(preq.sent + t), e);

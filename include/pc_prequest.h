@@ -69,6 +69,25 @@ struct pc_prequest_s {
   uint64_t peer_part_bytes;   /* send: receiver's bytes per partition; receive: sender's   */
   uint32_t *hready;           /* send, PC_COPY_HOST: [ntransport] ready epochs in pinned
                                  host memory (device-mapped), polled by the progress thread */
+  /* INLINE allreduce ("Kernel Copy" for the collective, reading R33): the
+   * Pready that completes partition u on the LAST of the P ranks folds u over
+   * every rank's send buffer in rank order and stores it into every rank's
+   * recvbuf (DIRECT schedule bits, oracle O6).  NULL: the engine reduces. */
+  const struct pc_ar_tab_s *ar_tab;
+  uint32_t dtype;             /* pc_dtype_t of the collective                             */
+  uint32_t op;                /* pc_op_t of the collective                                */
+};
+
+/* Device table of an INLINE allreduce request (library-owned device memory,
+ * written once at pc_prequest_create).  Indexed by comm rank k < nranks <= 8;
+ * every pointer is valid in the owning rank's context (peer-mapped). */
+#define PC_AR_MAX 8
+struct pc_ar_tab_s {
+  const uint8_t *send[PC_AR_MAX];  /* rank k's send buffer                                      */
+  uint8_t *recv[PC_AR_MAX];        /* rank k's recv buffer                                      */
+  uint32_t *done[PC_AR_MAX];       /* rank k's INLINE completion words [N_p] (epoch e = final)  */
+  uint32_t *cnt;                   /* arrival counters [N_p] in rank 0's control block (target e*P) */
+  const uint32_t *rtr;             /* this rank's ready-to-receive words [P-1], written by the peers */
 };
 
 /* Receive side: bit 31 of the layout word = the sender pushes LL lines; bit

@@ -323,10 +323,12 @@ class DLProxy:
     mode "serial": producer kernels, then the collective (host-side Pready of
                    every partition, the MPI_Allreduce-after-the-kernel flow).
     ``overlap=False`` forks the engine at the wait (pc_request_set_overlap):
-    the Pready mode without producer/engine concurrency.
+    the Pready mode without producer/engine concurrency.  ``copy=COPY_INLINE``
+    (DIRECT schedule): no engine — the producer block whose Pready completes a
+    partition on the last rank folds it for every rank (reading R33).
     Inputs: ``p`` (predictions), ``y`` (targets), fp32, one tensor per rank."""
 
-    def __init__(self, comms, partitions: int, L: int, algo: int, p, y, overlap: bool = True):
+    def __init__(self, comms, partitions: int, L: int, algo: int, p, y, overlap: bool = True, copy: int | None = None):
         import torch
 
         from . import runtime as rt
@@ -343,6 +345,11 @@ class DLProxy:
         if not overlap:
             for q in self.reqs:
                 q.set_overlap(False)
+        from .runtime import COPY_ENGINE
+        # copy: COPY_ENGINE (the engine reduces) or COPY_INLINE (DIRECT only:
+        # the producer block completing a partition on the last rank folds it,
+        # reading R33)
+        self.copy = COPY_ENGINE if copy is None else copy
         self.preqs = None
         self.ctl = torch.cuda.Stream()
         self.pst = [torch.cuda.Stream() for _ in range(self.P)]
@@ -357,7 +364,7 @@ class DLProxy:
             for q in self.reqs:
                 q.start(st)
             rt.run_ranks([(lambda q=q: q.pbuf_prepare(st)) for q in self.reqs])
-            self.preqs = [q.prequest_create(rt.GRAN_BLOCK, 1, rt.COPY_ENGINE) for q in self.reqs]
+            self.preqs = [q.prequest_create(rt.GRAN_BLOCK, 1, self.copy) for q in self.reqs]
         else:
             rt.startall(self.reqs, st)
             rt.pbuf_prepare_all(self.reqs, st)

@@ -26,6 +26,7 @@
 #include <atomic>
 
 #include "pc_device.cuh"
+#include "pc_ops.cuh"
 #include "pc_internal.h"
 
 // engine.cuh is included by kernels.cu (control kernels, p2p engine, the
@@ -96,63 +97,10 @@ __device__ __forceinline__ void warp_signal(uint32_t *flag, uint32_t e, bool sys
   if ((threadIdx.x & 31) == 0) st_relaxed_sys(flag, e);
 }
 
-template <int DT, int OP>
-struct Op;
-template <int OP>
-struct Op<0, OP> {  // int32: sum wraps mod 2^32
-  using T = int32_t;
-  static __device__ __forceinline__ int32_t f(int32_t a, int32_t b) {
-    if (OP == 0) return (int32_t)((uint32_t)a + (uint32_t)b);
-    if (OP == 1) return a > b ? a : b;
-    return a < b ? a : b;
-  }
-};
-template <int OP>
-struct Op<1, OP> {  // fp32: one IEEE add, round to nearest even, no contraction
-  using T = float;
-  static __device__ __forceinline__ float f(float a, float b) {
-    if (OP == 0) return __fadd_rn(a, b);
-    if (OP == 1) return fmaxf(a, b);
-    return fminf(a, b);
-  }
-};
-
-template <int OP>
-struct Op<3, OP> {  // fp64 (the paper's `double` buffers)
-  using T = double;
-  static __device__ __forceinline__ double f(double a, double b) {
-    if (OP == 0) return __dadd_rn(a, b);
-    if (OP == 1) return fmax(a, b);
-    return fmin(a, b);
-  }
-};
-template <int OP>
-struct Op<4, OP> {  // bf16 storage (uint16 bits); each op is one correctly rounded bf16 result:
-  using T = uint16_t;  // a + b of two bf16 values is exact in fp32 or the small one is below half an ulp
-  static __device__ __forceinline__ float up(uint16_t v) { return __uint_as_float((uint32_t)v << 16); }
-  static __device__ __forceinline__ uint16_t dn(float f) {
-    return __bfloat16_as_ushort(__float2bfloat16_rn(f));
-  }
-  static __device__ __forceinline__ uint16_t f(uint16_t a, uint16_t b) {
-    if (OP == 0) return dn(__fadd_rn(up(a), up(b)));
-    if (OP == 1) return dn(fmaxf(up(a), up(b)));
-    return dn(fminf(up(a), up(b)));
-  }
-};
-
-template <int DT, int OP>
-__device__ __forceinline__ uint4 vop(uint4 a, uint4 b) {
-  using O = Op<DT, OP>;
-  using T = typename O::T;
-  constexpr int EPV = 16 / sizeof(T);
-  uint4 r;
-  T *ra = reinterpret_cast<T *>(&r);
-  const T *pa = reinterpret_cast<const T *>(&a);
-  const T *pb = reinterpret_cast<const T *>(&b);
-#pragma unroll
-  for (int j = 0; j < EPV; ++j) ra[j] = O::f(pa[j], pb[j]);
-  return r;
-}
+// ⊕ and its 16-B vector form: include/pc_ops.cuh (shared with the INLINE
+// allreduce fold of pc_device.cuh)
+using pc_ops::Op;
+using pc_ops::vop;
 
 // out1[k] (and out2[k]) = local[k] ⊕ incoming[k], k < n elements, by one warp.
 // All operands of one call sit at the same element offset of 16-B aligned
@@ -549,7 +497,21 @@ __device__ __forceinline__ void red_add_scope(uint32_t *p, uint32_t v, bool sys)
 // of this rank's recvbuf and (TO_PEERS) of every peer's.  When the sources and
 // the destination do not share a 16-B misalignment the whole range takes the
 // scalar path.
-template <int DT, int OP, bool TO_PEERS = true, int FV = PC_DIRECT_FV, typename A>
+// L2 prefetch by the TMA engine (cp.async.bulk.prefetch.L2): bytes the warp
+// will load soon are requested without registers or shared memory, so a thin
+// warp (one 16-B vector per operand in registers) still keeps kPfAhead blocks
+// of kPfBytes per source in flight.  16-B aligned, size a multiple of 16.
+constexpr int64_t kPfBytes = 4096;
+#ifndef PC_PF_AHEAD
+#define PC_PF_AHEAD 2
+#endif
+constexpr int kPfAhead = PC_PF_AHEAD;
+__device__ __forceinline__ void prefetch_l2(const void *p, int64_t bytes) {
+  if (bytes <= 0) return;
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"((uint32_t)bytes) : "memory");
+}
+
+template <int DT, int OP, bool TO_PEERS = true, int FV = PC_DIRECT_FV, bool PF = false, typename A>
 __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d0, int64_t n) {
   using O = Op<DT, OP>;
   using T = typename O::T;
@@ -586,8 +548,20 @@ __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d
         if (j < P - 1) *reinterpret_cast<uint4 *>(reinterpret_cast<T *>(a.p_recvbuf[j]) + e0 + eo) = acc;
     }
   };
+  // PF: lane j < P prefetches source j's 16-B body in blocks of kPfBytes,
+  // kPfAhead blocks ahead of the loads (same-GPU peers only: a.sys == 0)
+  constexpr int64_t kPfV = kPfBytes / 16;  // vectors per prefetch block
+  const bool pf = PF && !a.sys && (int)lane < P;
+  auto pf_block = [&](int64_t b) {
+    const int64_t v0 = b * kPfV;
+    if (v0 < nv)
+      prefetch_l2(reinterpret_cast<const uint4 *>(src((int)lane) + head) + v0, (min(nv - v0, kPfV)) * 16);
+  };
+  if (pf)
+    for (int b = 0; b < kPfAhead; ++b) pf_block(b);
   int64_t k = lane;
   for (; k + 32 * (kFV - 1) < nv; k += 32 * kFV) {
+    if (pf && ((k - lane) % kPfV) == 0) pf_block((k - lane) / kPfV + kPfAhead);
     uint4 x[kMaxDirect][kFV];
 #pragma unroll
     for (int j = 0; j < kMaxDirect; ++j)
@@ -752,7 +726,7 @@ __device__ __forceinline__ void warp_fold_pull_bulk(const A &a, int64_t s0, int6
   for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
 }
 
-template <int DT, int OP, int FV = PC_DIRECT_FV>
+template <int DT, int OP, int FV = PC_DIRECT_FV, bool PF = false>
 __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W, uint8_t *smem) {
   const int P = a.P, r = a.r;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;
@@ -810,7 +784,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
             if (PC_DIRECT_BULK && !a.sys)
               warp_fold_pull_bulk<DT, OP>(a, base + lo, base + lo, hi - lo, wb);
             else
-              warp_fold_pull<DT, OP, true, FV>(a, base + lo, base + lo, hi - lo);
+              warp_fold_pull<DT, OP, true, FV, PF>(a, base + lo, base + lo, hi - lo);
           }
           fence_scope(a.sys);
           __syncwarp();
@@ -989,7 +963,8 @@ __global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine_gr
 // leaves ~11 K registers: no 512-thread producer block fits beside it).
 template <int DT, int OP>
 __global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_thin(DirectArgs a) {
-  direct_body<DT, OP, 1>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5, nullptr);
+  direct_body<DT, OP, 1, true>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5,
+                               nullptr);
 }
 template <int DT, int OP>
 __global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_group_thin(DirectGroupArgs g) {
@@ -997,7 +972,7 @@ __global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_group_thin(Dire
   while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
   const int b = blockIdx.x - g.block_start[k];
   const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
-  direct_body<DT, OP, 1>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, nullptr);
+  direct_body<DT, OP, 1, true>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, nullptr);
 }
 
 // Single-rank launches (one rank per GPU / process).

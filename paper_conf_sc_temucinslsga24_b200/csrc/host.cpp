@@ -465,6 +465,13 @@ static void fill_prequest(Request *q, pc_prequest_t *o) {
   o->peer_part_bytes = q->peer_part_bytes;
   o->coll = (uint32_t)q->coll;
   o->nranks = q->comm->size;
+  o->dtype = (uint32_t)q->dtype;
+  o->op = (uint32_t)q->op;
+  if (q->inline_ar) {  // R33: completion words are the INLINE done array (epoch e = final)
+    o->ar_tab = (const pc_ar_tab_s *)q->ar_tab;
+    o->done = q->ctrl + q->L.sent;
+    o->done_mul = 1;
+  }
   if (q->kind == PC_KIND_PALLREDUCE && q->coll == PC_COLL_ALLGATHER)
     o->srcflags = q->ctrl + q->L.flags + (size_t)q->partitions * 2 * q->slices;
   if (q->kind == PC_KIND_PSEND) {
@@ -856,7 +863,7 @@ static CollArgs make_coll_args(Request *q) {
 static const cudaStream_t kHostJoined = reinterpret_cast<cudaStream_t>(~uintptr_t(0));
 
 static bool needs_engine(Request *q) {
-  return q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
+  return (q->kind == PC_KIND_PALLREDUCE && !q->inline_ar) || (q->kind == PC_KIND_PSEND && q->has_preq && q->copy == 1);
 }
 
 // Optional CUDA-event timing around an engine launch (pc_request_set_timing).
@@ -941,7 +948,7 @@ static int launch_single(Request *q) {
     rc = launch_coll_engine(make_coll_args(q), w, q->side);
   } else if (q->kind == PC_KIND_PALLREDUCE) {
     rc = q->algo == PC_ALGO_RING     ? launch_ring_engine(make_ring_args(q), w, q->side)
-         : q->algo == PC_ALGO_DIRECT ? launch_direct_engine(make_direct_args(q), w, q->side, !full)
+         : q->algo == PC_ALGO_DIRECT ? launch_direct_engine(make_direct_args(q), w, q->side, !full && q->comm->overlap_thin)
                                      : launch_rd_engine(make_rd_args(q), w, q->side);
   } else {
     P2pEngineArgs a{};
@@ -1017,7 +1024,7 @@ static int group_register(Request *q, bool block, cudaStream_t ws, bool *launche
       DirectGroupArgs ga{};
       ga.n = (int)g.members.size();
       for (int k = 0; k < ga.n; ++k) ga.a[k] = make_direct_args(g.members[k]);
-      rc = launch_direct_engine_group(ga, w, q->side, !full);
+      rc = launch_direct_engine_group(ga, w, q->side, !full && q->comm->overlap_thin);
     } else {
       RdGroupArgs ga{};
       ga.n = (int)g.members.size();
@@ -1218,6 +1225,7 @@ int pc_comm_create(int rank, int size, int cuda_device, pc_allgather_fn ag, void
   c->engine_warps = c->dry ? 1184 : std::max(8, (int)env_long("PC_ENGINE_WARPS", ew));
   c->direct_warps = c->dry ? 592 : std::max(8, (int)env_long("PC_DIRECT_WARPS", dw));
   c->overlap_warps = c->dry ? 592 : std::max(8, ow);
+  c->overlap_thin = env_long("PC_OVERLAP_THIN", 1) != 0;
   if (!c->dry) {
     for (int q = 0; q < size; ++q) {
       if (q == rank || !c->same_proc[q] || all[q].device == cuda_device) continue;
@@ -1522,7 +1530,7 @@ int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream) {
     if (q->active) return PC_ERR_STATE;
     if (!q->exchanged) return PC_ERR_STATE;
     if (!q->matched) return PC_ERR_MATCH;
-    if (pready && q->kind != PC_KIND_PALLREDUCE) return PC_ERR_ARG;
+    if (pready && (q->kind != PC_KIND_PALLREDUCE || q->inline_ar)) return PC_ERR_ARG;  // R33: Pready folds
     if (q->comm->device != ((Request *)reqs[0])->comm->device || q->comm->dry != ((Request *)reqs[0])->comm->dry)
       return PC_ERR_ARG;
     if (group_blocks_start(q)) return PC_ERR_STATE;
@@ -1698,6 +1706,33 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
       PC_CUDA(cudaStreamSynchronize(q->side));
     }
   } else {
+    if (copy == PC_COPY_INLINE) {  // R33: INLINE allreduce (DIRECT schedule bits, P <= 8)
+      if (q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT || c->size > PC_AR_MAX) return PC_ERR_UNSUPPORTED;
+      if (!c->dry && !q->ar_tab) {
+        pc_ar_tab_s t{};
+        const int P = c->size, r = c->rank;
+        for (int k = 0; k < P; ++k) {
+          if (k == r) {
+            t.send[k] = (const uint8_t *)q->sbuf;
+            t.recv[k] = (uint8_t *)q->rbuf;
+            t.done[k] = q->ctrl + q->L.sent;
+          } else {
+            const int j = mod(k - r - 1, P);  // peer j = rank (r + 1 + j) mod P
+            t.send[k] = q->nb_stage[j];        // DIRECT exports its send buffer in the stage slot
+            t.recv[k] = q->nb_buf[j];
+            t.done[k] = q->nb_ctrl[j] + q->L.sent;
+          }
+        }
+        t.cnt = (r == 0 ? q->ctrl : q->nb_ctrl[mod(0 - r - 1, P)]) + q->L.cnt;
+        t.rtr = q->ctrl + q->L.rtr;
+        PC_CUDA(cudaSetDevice(c->device));
+        PC_CUDA(cudaMalloc(&q->ar_tab, sizeof(t)));
+        PC_CUDA(cudaMemcpy(q->ar_tab, &t, sizeof(t), cudaMemcpyHostToDevice));
+      }
+      q->inline_ar = true;
+    } else {
+      q->inline_ar = false;
+    }
     q->copy = copy;
   }
   q->has_preq = true;
@@ -1740,9 +1775,20 @@ static int wait_common(Request *q, cudaStream_t s, bool host) {
   PC_CUDA(cudaSetDevice(c->device));
   if (!q->exchanged || !q->matched) return PC_ERR_STATE;
   int32_t *err = (int32_t *)(q->ctrl + q->L.err);
-  const bool engine = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->copy == 1);
+  const bool engine = (q->kind == PC_KIND_PALLREDUCE && !q->inline_ar) || (q->kind == PC_KIND_PSEND && q->copy == 1);
   int rc;
-  if (engine) {
+  if (q->inline_ar) {  // R33: every done[u] of this rank reached the epoch (written by the folding ranks)
+    cudaStream_t ws = host ? q->side : s;
+    if (host) {
+      PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+      PC_CUDA(cudaStreamWaitEvent(q->side, q->ev_fork, 0));
+    }
+    if ((rc = launch_wait_words(q->ctrl + q->L.sent, q->partitions, q->ctrl + q->L.epoch, 1, nullptr, q->partitions,
+                                err, c->timeout_ms, ws, q->sys_scope != 0)))
+      return rc;
+    if (host) PC_CUDA(cudaStreamSynchronize(q->side));
+    q->joined_stream = host ? kHostJoined : s;
+  } else if (engine) {
     if (q->kind == PC_KIND_PSEND && !q->has_preq) return PC_ERR_STATE;
     cudaEvent_t ev = nullptr;
     if ((rc = ensure_engine(q, host, host ? nullptr : s, &ev))) return rc;
@@ -1887,8 +1933,8 @@ int pc_parrived(pc_request_t req, int partition, int *flag) {
     *flag = 1;
     for (uint32_t w : h) *flag = *flag && reached_h(w, e);
   } else if (q->kind == PC_KIND_PALLREDUCE) {
-    if ((rc = read_words(q, q->L.donecnt + partition, 1, &v))) return rc;
-    *flag = reached_h(v, e * (uint32_t)q->slices);
+    if ((rc = read_words(q, (q->inline_ar ? q->L.sent : q->L.donecnt) + partition, 1, &v))) return rc;
+    *flag = reached_h(v, e * (uint32_t)(q->inline_ar ? 1 : q->slices));
   } else if (q->kind == PC_KIND_PRECV) {
     uint32_t g = 0;
     if ((rc = read_words(q, q->L.layout, 1, &g))) return rc;
@@ -1925,9 +1971,16 @@ int pc_test(pc_request_t req, int *flag) {
   }
   PC_CUDA(cudaSetDevice(q->comm->device));
   int rc;
-  const bool engine = q->kind == PC_KIND_PALLREDUCE || (q->kind == PC_KIND_PSEND && q->copy == 1);
+  const bool engine = (q->kind == PC_KIND_PALLREDUCE && !q->inline_ar) || (q->kind == PC_KIND_PSEND && q->copy == 1);
   bool done = false;
-  if (engine) {
+  if (q->inline_ar) {  // R33: every INLINE done word reached the epoch
+    uint32_t e = 0;
+    if ((rc = current_epoch(q, &e))) return rc;
+    std::vector<uint32_t> h((size_t)q->partitions);
+    if ((rc = read_words(q, q->L.sent, h.size(), h.data()))) return rc;
+    done = true;
+    for (uint32_t v : h) done = done && reached_h(v, e);
+  } else if (engine) {
     cudaEvent_t ev = nullptr;
     if (q->kind == PC_KIND_PSEND && !q->has_preq) {
       *flag = 0;
@@ -2065,6 +2118,7 @@ int pc_request_free(pc_request_t *req) {
     if (q->staging) cudaFree(q->staging);
     if (q->side) cudaStreamDestroy(q->side);
     if (q->ev_fork) cudaEventDestroy(q->ev_fork);
+    if (q->ar_tab) cudaFree(q->ar_tab);
     if (q->ev_done) cudaEventDestroy(q->ev_done);
     if (q->gs.ev) cudaEventDestroy(q->gs.ev);
     for (cudaEvent_t e : q->gs.tlog.pool) cudaEventDestroy(e);

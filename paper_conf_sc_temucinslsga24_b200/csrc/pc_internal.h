@@ -167,6 +167,10 @@ struct Request {
   bool forked = false;          // ev_fork recorded at a control point of this epoch
   bool host_ready_all = false;  // every partition was made ready by a host-side op before ev_fork
   bool overlap = true;          // pc_request_set_overlap (0: fork at the wait, the round-1 order)
+  // INLINE allreduce (reading R33): a DIRECT allreduce whose prequest was
+  // created with PC_COPY_INLINE — the completing Pready folds, no engine
+  bool inline_ar = false;
+  void *ar_tab = nullptr;       // device pc_ar_tab_s (library-owned)
   // stream on which the previous epoch's completion is ordered (null: host
   // observed it); a later epoch's control op on another stream first waits
   // for that completion (the engine reads the epoch word at entry)
@@ -246,6 +250,7 @@ struct Comm {
   std::vector<bool> same_proc;
   int engine_warps = 0;  // agreed (min over ranks)
   int direct_warps = 0;  // the same for the DIRECT allreduce engines
+  bool overlap_thin = true;  // PC_OVERLAP_THIN (measurement knob): thin DIRECT CTAs while overlapping
   int overlap_warps = 0; // per-rank engine width when the engine may overlap a producer:
                          // whole CTAs, <= PC_OVERLAP_FRAC of the SMs per GPU in total
   int sms = 0;

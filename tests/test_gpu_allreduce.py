@@ -38,9 +38,12 @@ def _to_numpy(t):
     return t.cpu().numpy()
 
 
-def run_allreduce(P, Np, L, xs_epochs, algo, op=pc.SUM, inplace=False, producer=None, gran=apps.GRAN_BLOCK):
+def run_allreduce(P, Np, L, xs_epochs, algo, op=pc.SUM, inplace=False, producer=None, gran=apps.GRAN_BLOCK,
+                  copy=pc.COPY_ENGINE):
     """xs_epochs: list over epochs of (P, Np*L) host arrays.  Returns a list over
-    epochs of (P, Np*L) results (each rank's recvbuf after its wait)."""
+    epochs of (P, Np*L) results (each rank's recvbuf after its wait).  copy:
+    the prequest's mode (COPY_INLINE on DIRECT: the completing Pready folds,
+    reading R33)."""
     dt, tdtype = DTYPES[xs_epochs[0].dtype.type]
     es = pc.ESIZE[dt]
     n = Np * L
@@ -62,7 +65,7 @@ def run_allreduce(P, Np, L, xs_epochs, algo, op=pc.SUM, inplace=False, producer=
                 reqs[r].start(streams[r])
             if e == 0:
                 first_prepare([[reqs[r]] for r in range(P)], streams)
-                preqs = [reqs[r].prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_ENGINE) for r in range(P)]
+                preqs = [reqs[r].prequest_create(pc.GRAN_BLOCK, 1, copy) for r in range(P)]
             else:
                 for r in range(P):
                     reqs[r].pbuf_prepare(streams[r])

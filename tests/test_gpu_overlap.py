@@ -28,7 +28,7 @@ SEED = synth.BASE_SEED + 700
 OALGO = {pc.ALGO_RING: oracle.RING, pc.ALGO_RD: oracle.RD, pc.ALGO_DIRECT: oracle.DIRECT}
 
 
-def _run(P, algo, overlap, Np=4, L=4099, epochs=3, spin_ms=3000):
+def _run(P, algo, overlap, Np=4, L=4099, epochs=3, spin_ms=3000, copy=pc.COPY_ENGINE):
     n = Np * L
     with comms(P, timeout_ms=20000) as cs:
         streams = [torch.cuda.Stream() for _ in range(P)]
@@ -48,7 +48,7 @@ def _run(P, algo, overlap, Np=4, L=4099, epochs=3, spin_ms=3000):
                 reqs[r].start(streams[r])
             if e == 0:
                 first_prepare([[q] for q in reqs], streams)
-                preqs = [q.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_ENGINE) for q in reqs]
+                preqs = [q.prequest_create(pc.GRAN_BLOCK, 1, copy) for q in reqs]
             else:
                 for r in range(P):
                     reqs[r].pbuf_prepare(streams[r])

@@ -45,11 +45,49 @@ def run(P, L, algo, modes):
     p = [(0.02 + 0.96 * torch.rand(n, device="cuda", generator=gen)) for _ in range(P)]
     y = [torch.randint(0, 2, (n,), device="cuda", generator=gen).float() for _ in range(P)]
     dl = apps.DLProxy(cs, Np, L, algo, p, y)
+    dl.step("serial")  # the first epoch exchanges and maps (every mode below starts from there)
+    torch.cuda.synchronize()
     dl_no = None
+    dl_in = None
     out = []
     for mode in modes:
         if mode in ("pready", "serial"):
             ms = timeit(lambda: dl.step(mode), dl.ctl)
+        elif mode in ("timeline", "timeline_serial"):  # where the time of one overlapped step goes
+            import statistics
+            sm = "pready" if mode == "timeline" else "serial"
+            dl.step(sm)
+            torch.cuda.synchronize()
+            dl.reqs[0].set_timing(True)
+            dl.reqs[0].engine_times()
+            prod, tot = [], []
+            for _ in range(10):
+                t0 = torch.cuda.Event(enable_timing=True)
+                te = [torch.cuda.Event(enable_timing=True) for _ in range(P)]
+                t1 = torch.cuda.Event(enable_timing=True)
+                dl.ev_p = te  # the step records the producers' ends into these
+                t0.record(dl.ctl)
+                dl.step(sm)
+                t1.record(dl.ctl)
+                torch.cuda.synchronize()
+                prod.append(max(t0.elapsed_time(e) for e in te))
+                tot.append(t0.elapsed_time(t1))
+            eng = dl.reqs[0].engine_times()
+            dl.reqs[0].set_timing(False)
+            dl.ev_p = [torch.cuda.Event() for _ in range(P)]
+            ms = statistics.median(tot)
+            extra = {"producers_end_ms": statistics.median(prod), "engine_ms": float(statistics.median(list(eng))) if len(eng) else None}
+            out.append({"P": P, "partition_bytes": 4 * L, "partitions": Np, "algo": algo, "mode": mode,
+                        "ms_per_step": ms, **extra})
+            print(json.dumps(out[-1]), flush=True)
+            continue
+        elif mode == "pready_inline":  # R33: the completing producer block folds (no engine)
+            if dl_in is None:
+                dl_in = apps.DLProxy(cs, Np, L, pc.ALGO_DIRECT, p, y, copy=pc.COPY_INLINE)
+                dl_in.step("pready")
+                torch.cuda.synchronize()
+            ms = timeit(lambda: dl_in.step("pready"), dl_in.ctl)
+            assert dl_in.errors() == [], dl_in.errors()
         elif mode == "pready_nooverlap":  # engine forked at the wait (no producer/engine concurrency)
             if dl_no is None:
                 dl_no = apps.DLProxy(cs, Np, L, algo, p, y, overlap=False)
@@ -63,6 +101,16 @@ def run(P, L, algo, modes):
                     dl.ev_p[r].record(dl.pst[r])
                 for r in range(P):
                     dl.ctl.wait_event(dl.ev_p[r])
+            ms = timeit(f, dl.ctl)
+        elif mode == "allreduce_bounded":  # the engine alone at its overlap width (thin CTAs)
+            def f():
+                pc.startall(dl.reqs, dl.ctl)
+                pc.pbuf_prepare_all(dl.reqs, dl.ctl)
+                for q in dl.reqs:  # two ranges: not "every partition by one host op" -> overlap width
+                    q.pready_range(0, Np - 2, dl.ctl)
+                    q.pready_range(Np - 1, Np - 1, dl.ctl)
+                for q in dl.reqs:
+                    q.wait_on_stream(dl.ctl)
             ms = timeit(f, dl.ctl)
         else:  # allreduce only (host Pready of every partition)
             def f():
@@ -80,6 +128,8 @@ def run(P, L, algo, modes):
     dl.free()
     if dl_no is not None:
         dl_no.free()
+    if dl_in is not None:
+        dl_in.free()
     for c in cs:
         c.destroy()
     g.destroy()
