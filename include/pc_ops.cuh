@@ -74,6 +74,29 @@ __device__ __forceinline__ uint4 vop(uint4 a, uint4 b) {
   return r;
 }
 
+// fp32 SUM on sm_100: packed add.rn.f32x2 (SASS FADD2) — two IEEE
+// round-to-nearest-even adds per instruction, bit-identical to __fadd_rn
+// lane by lane (no .ftz: subnormals kept), half the FADD issue slots of the
+// scalar form (the thin overlap engines are issue-bound).
+template <>
+__device__ __forceinline__ uint4 vop<1, 0>(uint4 a, uint4 b) {
+#if defined(__CUDA_ARCH__) && __CUDA_ARCH__ >= 1000
+  unsigned long long lo, hi;
+  asm("add.rn.f32x2 %0, %1, %2;"
+      : "=l"(lo)
+      : "l"(((unsigned long long)a.y << 32) | a.x), "l"(((unsigned long long)b.y << 32) | b.x));
+  asm("add.rn.f32x2 %0, %1, %2;"
+      : "=l"(hi)
+      : "l"(((unsigned long long)a.w << 32) | a.z), "l"(((unsigned long long)b.w << 32) | b.z));
+  return make_uint4((uint32_t)lo, (uint32_t)(lo >> 32), (uint32_t)hi, (uint32_t)(hi >> 32));
+#else
+  return make_uint4(__float_as_uint(__fadd_rn(__uint_as_float(a.x), __uint_as_float(b.x))),
+                    __float_as_uint(__fadd_rn(__uint_as_float(a.y), __uint_as_float(b.y))),
+                    __float_as_uint(__fadd_rn(__uint_as_float(a.z), __uint_as_float(b.z))),
+                    __float_as_uint(__fadd_rn(__uint_as_float(a.w), __uint_as_float(b.w))));
+#endif
+}
+
 }  // namespace pc_ops
 
 #endif /* PC_OPS_CUH_ */

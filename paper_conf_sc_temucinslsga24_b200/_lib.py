@@ -90,7 +90,7 @@ _APP_PROTOS = {
     "pcapp_pingpong_pair": (I32, [P, P, P, P, I32, I32, P, P, P]),
     "pcapp_bare_pingpong_pair": (I32, [P, P, I32, C.c_uint32, P, I32, P]),
     "pcapp_prequest_size": (SZ, []),
-    "pcapp_overlap_probe": (I32, [P, I32, C.c_uint32, P, P]),
+    "pcapp_overlap_probe": (I32, [C.POINTER(P), I32, I32, C.c_uint32, P, P]),
     "pcapp_peer_copy": (I32, [I32, C.POINTER(P), C.POINTER(P), C.c_uint64, I32, P]),
     "pcapp_memcpy_async": (I32, [P, P, C.c_uint64, P]),
     "pcapp_flag_variant": (I32, [P, P, I32, I32, C.c_uint32, P, P]),

@@ -61,11 +61,15 @@ def memcpy_async(dst, src, nbytes: int, stream=None):
     _ok(_lib.apps().pcapp_memcpy_async(_ptr(dst), _ptr(src), nbytes, _stream(stream)), "memcpy_async")
 
 
-def overlap_probe(preq: Prequest, partitions: int, spin_ms: int, out_ns, stream=None):
-    """a6 concurrency probe: Pready(0), spin (<= spin_ms) until Parrived(0),
-    then Pready the rest.  out_ns: int64 device tensor [4] = %globaltimer at
-    entry, after Pready(0), when Parrived(0) was seen (0: timed out), exit."""
-    _ok(_lib.apps().pcapp_overlap_probe(preq.ptr, partitions, spin_ms, _ptr(out_ns), _stream(stream)),
+def overlap_probe(preqs, partitions: int, spin_ms: int, out_ns, stream=None):
+    """a6 concurrency probe, one launch for the co-located ranks (block b =
+    rank b's producer with preqs[b]): Pready(0), spin (<= spin_ms) until
+    Parrived(0), then Pready the rest.  out_ns: int64 device tensor [P, 4] =
+    %globaltimer at entry, after Pready(0), when Parrived(0) was seen (0:
+    timed out), at exit."""
+    n = len(preqs)
+    arr = (C.c_void_p * n)(*[q.ptr for q in preqs])
+    _ok(_lib.apps().pcapp_overlap_probe(arr, n, partitions, spin_ms, _ptr(out_ns), _stream(stream)),
         "overlap_probe")
 
 

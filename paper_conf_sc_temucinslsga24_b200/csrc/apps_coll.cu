@@ -59,8 +59,16 @@ __global__ void __launch_bounds__(512) produce_kernel(uint8_t *__restrict__ dst,
 // exits.  Partition 0 can only complete while this kernel is still running if
 // the engine runs concurrently with it.  out[0..3] = %globaltimer at entry,
 // after Pready(0), when Parrived(0) was seen (0 = never, timed out), at exit.
-__global__ void overlap_probe_kernel(pc_prequest_t preq, int partitions, uint32_t spin_ms,
-                                     unsigned long long *out) {
+// Block b is rank b's producer (one launch for all co-located ranks, so the P
+// spinning producers are co-resident by construction: separate launches on P
+// streams may share a hardware queue and run one after another).
+struct ProbeArgs {
+  int n;
+  pc_prequest_t q[8];
+};
+__global__ void overlap_probe_kernel(ProbeArgs a, int partitions, uint32_t spin_ms, unsigned long long *out_all) {
+  const pc_prequest_t &preq = a.q[blockIdx.x];
+  unsigned long long *out = out_all + 4 * blockIdx.x;
   __shared__ int s_arrived;
   if (threadIdx.x == 0) out[0] = pc_detail::globaltimer();
   pc_pready_block(0, preq);
@@ -142,10 +150,14 @@ int pcapp_bce_grad(const float *p, const float *y, float *g, int partitions, int
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 
-int pcapp_overlap_probe(const pc_prequest_t *preq, int partitions, uint32_t spin_ms, unsigned long long *out,
-                        cudaStream_t s) {
-  if (!preq || partitions < 1) return -1;
-  overlap_probe_kernel<<<1, 128, 0, s>>>(*preq, partitions, spin_ms, out);
+// preqs: n prequests (one per co-located rank); out: n x 4 stamps
+int pcapp_overlap_probe(const pc_prequest_t *const *preqs, int n, int partitions, uint32_t spin_ms,
+                        unsigned long long *out, cudaStream_t s) {
+  if (!preqs || n < 1 || n > 8 || partitions < 1) return -1;
+  ProbeArgs a{};
+  a.n = n;
+  for (int i = 0; i < n; ++i) a.q[i] = *preqs[i];
+  overlap_probe_kernel<<<n, 128, 0, s>>>(a, partitions, spin_ms, out);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -1705,7 +1705,7 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
       PC_CUDA(cudaMemcpyAsync(q->peer_ctrl + q->L.layout, &g, 4, cudaMemcpyHostToDevice, q->side));
       PC_CUDA(cudaStreamSynchronize(q->side));
     }
-  } else {
+  } else if (q->kind == PC_KIND_PALLREDUCE) {
     if (copy == PC_COPY_INLINE) {  // R33: INLINE allreduce (DIRECT schedule bits, P <= 8)
       if (q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT || c->size > PC_AR_MAX) return PC_ERR_UNSUPPORTED;
       if (!c->dry && !q->ar_tab) {
@@ -1733,6 +1733,8 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
     } else {
       q->inline_ar = false;
     }
+    q->copy = copy;
+  } else {
     q->copy = copy;
   }
   q->has_preq = true;

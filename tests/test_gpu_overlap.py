@@ -2,8 +2,9 @@
 reduced as soon as it is ready", §IV-B1; the paper's own remedy of
 moving the collective's progress beside the user kernel, §VI-B).
 
-The probe producer (apps.overlap_probe, one block per rank, each rank on its
-own stream) Preadies partition 0, then spins on the DEVICE pc_parrived(0) of
+The probe producer (apps.overlap_probe: one launch, block r = rank r's
+producer, so the P spinning producers are co-resident by construction)
+Preadies partition 0, then spins on the DEVICE pc_parrived(0) of
 the partitioned collective before it Preadies the remaining partitions.
 Partition 0 can only complete while the producer is still running if the
 engine runs concurrently with it: with the default fork point (the epoch's
@@ -52,9 +53,15 @@ def _run(P, algo, overlap, Np=4, L=4099, epochs=3, spin_ms=3000, copy=pc.COPY_EN
             else:
                 for r in range(P):
                     reqs[r].pbuf_prepare(streams[r])
-            outs = [torch.zeros(4, dtype=torch.int64, device="cuda") for _ in range(P)]
-            for r in range(P):  # every rank's producer, then every rank's wait (Listing 2 order)
-                apps.overlap_probe(preqs[r], Np, spin_ms, outs[r], streams[r])
+            out = torch.zeros((P, 4), dtype=torch.int64, device="cuda")
+            # every rank's producer (one launch, block r = rank r, on rank 0's
+            # stream after every rank's control calls), then every rank's wait
+            # (Listing 2 order)
+            ev = [torch.cuda.Event() for _ in range(P)]
+            for r in range(P):
+                ev[r].record(streams[r])
+                streams[0].wait_event(ev[r])
+            apps.overlap_probe(preqs, Np, spin_ms, out, streams[0])
             for r in range(P):
                 reqs[r].wait_on_stream(streams[r])
             torch.cuda.synchronize()
@@ -64,7 +71,7 @@ def _run(P, algo, overlap, Np=4, L=4099, epochs=3, spin_ms=3000, copy=pc.COPY_EN
             for r in range(P):
                 got = recv[r].cpu().numpy()
                 np.testing.assert_array_equal(got.view(np.uint32), ref[r].view(np.uint32))
-            stamps.append(np.stack([o.cpu().numpy() for o in outs]))
+            stamps.append(out.cpu().numpy())
         return stamps
 
 
