@@ -685,7 +685,7 @@ def multi_nvlink_floor(ctx, pc, apps, torch, chunk):
     q.pready_range(0, 0, st)
     q.wait_on_stream(st)
     torch.cuda.synchronize()
-    peers = [q.peer_buffer(j) for j in range(P - 1)]
+    peers = [q.peer_buffer(j) for j in range(P - 1)]  # (allgather: DIRECT peer mapping)
     # push: my chunk -> slot r of every peer's recvbuf; pull: slot (peer) of every peer -> my slot (peer)
     push_dst = [p + r * chunk for p in peers]
     pull_src = [peers[j] + ((r + 1 + j) % P) * chunk for j in range(P - 1)]
@@ -778,6 +778,7 @@ def multi_p2p(ctx, pc, apps, torch, dist):
         q0.start(st)
         q0.pbuf_prepare(st)
         if side == 0:
+            q0.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
             q0.pready_range(0, 0, st)
         q0.wait_on_stream(st)
         torch.cuda.synchronize()
@@ -881,6 +882,7 @@ def multi_p2p(ctx, pc, apps, torch, dist):
         x.start(st)
     for x in (q, q2):
         x.pbuf_prepare(st)
+    q.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
     q.pready_range(0, 0, st)
     q.wait_on_stream(st)
     q2.wait_on_stream(st)
@@ -991,7 +993,9 @@ def run_multi(args):
         xs = [x.cuda() for x in xs_cpu]
     else:
         dist.all_gather(xs, send)
-    idx = torch.randint(0, send.numel(), (4096,), device="cuda", generator=gen)
+    gidx = torch.Generator(device="cuda")
+    gidx.manual_seed(0x5C24)  # the same sample on every rank
+    idx = torch.randint(0, send.numel(), (4096,), device="cuda", generator=gidx)
     ref = torch.stack([x[idx].double() for x in xs]).sum(0)
     bound = 1e-5 * torch.stack([x[idx].double().abs() for x in xs]).sum(0)
     parity_ok = bool(((recv[idx].double() - ref).abs() <= bound).all().item())
