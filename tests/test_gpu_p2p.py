@@ -83,6 +83,15 @@ def run_vecadd(n, gran, agg, copy, epochs=3, check_in_kernel=True):
         np.testing.assert_array_equal(np.stack(got_kernel).view(np.uint8).reshape(epochs, -1), consumed)
 
 
+@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE])
+@pytest.mark.parametrize("agg", [1, 128])
+def test_c2_block_256mib(copy, agg):
+    """C2 at its largest size (256 MiB, 32768 block partitions of 8 KiB; agg
+    128 = 1 MiB transport partitions): byte-exact vs O1 over 2 epochs with
+    seeded inputs, in-kernel Parrived consumer included."""
+    run_vecadd(1 << 26, apps.GRAN_BLOCK, agg, copy, epochs=2)
+
+
 def test_c1_block_agg16_inline():
     """C1: 1 MiB fp32, block Pready (128 x 8 KiB user partitions) aggregated
     16 per transport partition -> 8 transport partitions (reading R24)."""

@@ -28,6 +28,49 @@ def busbw(S, sec, P):
     return S / sec * 2.0 * (P - 1) / P / 1e9 if P > 1 else S / sec / 1e9
 
 
+# ------------------------------------------------------------ parity gate (§8(d).2)
+# Before a point is reported: (1) the timed fp32 run's result is bit-identical
+# on every rank and within the north_star bound |y - y64| <= 1e-5 * sum|x|
+# (reading R16) on sampled elements against the fp64 sum of the inputs; (2)
+# for S <= 64 MiB an int32 run of the same shape (partitions, count, schedule)
+# equals the plain definition, the wrapping sum mod 2^32, on every element.
+# Plain definitions only (no oracle import: tools/ is product-side).
+def fp32_gate(send, recv, nsample=65536):
+    n = send[0].numel()
+    ok = all(torch.equal(recv[0][:n], r[:n]) for r in recv[1:])
+    g = torch.Generator(device="cuda")
+    g.manual_seed(0x5C24)
+    idx = torch.randint(0, n, (min(nsample, n),), device="cuda", generator=g)
+    x = torch.stack([t[idx].double() for t in send])
+    y64, sabs = x.sum(0), x.abs().sum(0)
+    return ok and bool(((recv[0][idx].double() - y64).abs() <= 1e-5 * sabs).all().item())
+
+
+def int32_gate(cs, Np, count, algo, st):
+    P = len(cs)
+    send = [torch.randint(-2**31, 2**31 - 1, (Np * count,), dtype=torch.int32, device="cuda") for _ in range(P)]
+    recv = [torch.empty_like(send[0]) for _ in range(P)]
+    reqs = [pc.pallreduce_init(send[r], recv[r], Np, count, pc.INT32, pc.SUM, algo, cs[r]) for r in range(P)]
+    for q in reqs:
+        q.start(st)
+    pc.run_ranks([(lambda q=q: q.pbuf_prepare(st)) for q in reqs])
+    pc.preadyall(reqs, st)
+    for q in reqs:
+        q.wait_on_stream(st)
+    pc.epoch_all(reqs, pready=True, stream=st)  # and a second epoch through the bench's control path
+    for q in reqs:
+        q.wait_on_stream(st)
+    torch.cuda.synchronize()
+    tot = torch.zeros(Np * count, dtype=torch.int64, device="cuda")
+    for t in send:
+        tot += t.long()
+    want = ((tot + 2**31) % 2**32 - 2**31).int()
+    ok = all(torch.equal(r, want) for r in recv) and all(q.error()[0] == 0 for q in reqs)
+    for q in reqs:
+        q.free()
+    return ok
+
+
 def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
     P = len(cs)
     count = max(S // 4 // Np, 1)
@@ -80,12 +123,15 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
         blocks.append(e0.elapsed_time(e1) / iters)
     errs = [q.error() for q in reqs if q.error()[0] != 0]
     info = reqs[0].info()
+    parity = fp32_gate(send, recv)
     for q in reqs:
         q.free()
+    if n * 4 <= (64 << 20):
+        parity = parity and int32_gate(cs, Np, count, algo, st)
     ms = statistics.median(blocks)
     return {"bytes_per_rank": n * 4, "partitions": Np, "ranks": P, "algo": ["auto", "ring", "rd", "direct"][algo],
             "us_per_step": ms * 1e3, "busbw_gbs": busbw(n * 4, ms / 1e3, P), "slices": info["slices"],
-            "graph": graph, "errors": errs}
+            "graph": graph, "errors": errs, "parity": parity}
 
 
 def sweep_allreduce(args):
@@ -162,12 +208,28 @@ def time_coll(cs, kind, S, Np, min_ms=30.0):
         torch.cuda.synchronize()
         blocks.append(e0.elapsed_time(e1) / iters)
     errs = [q.error() for q in reqs if q.error()[0] != 0]
+    # parity gate: the plain definition of the collective on every element
+    # (reduce-scatter: the rank-order fp32 fold (R25) of block r of every
+    # partition; allgather: rank-major concatenation; broadcast: the root's)
+    if kind == "rs":
+        parity = True
+        for r in range(P):
+            blk = [send[k].view(Np, P, count)[:, r, :] for k in range(P)]
+            acc = blk[0].clone()
+            for k in range(1, P):
+                acc = acc + blk[k]  # fp32 adds in rank order, round to nearest
+            parity = parity and torch.equal(recv[r].view(Np, count), acc)
+    elif kind == "ag":
+        want = torch.cat([send[k] for k in range(P)])
+        parity = all(torch.equal(recv[r], want) for r in range(P))
+    else:
+        parity = all(torch.equal(buf[r], buf[0]) for r in range(P))
     for q in reqs:
         q.free()
     ms = statistics.median(blocks)
     fac = 1.0 if kind == "bc" else (P - 1) / P
     return {"coll": kind, "ranks": P, "bytes": full, "partitions": Np, "us_per_step": ms * 1e3,
-            "busbw_gbs": full / (ms / 1e3) * fac / 1e9, "errors": errs}
+            "busbw_gbs": full / (ms / 1e3) * fac / 1e9, "errors": errs, "parity": bool(parity)}
 
 
 def sweep_coll(args):
@@ -248,10 +310,13 @@ def sweep_dl_per_tensor(args):
             ms = e0.elapsed_time(e1) / it
             total = sum(sizes) * 4
             errs = [q.error() for q in flat if q.error()[0] != 0]
+            parity = all(fp32_gate([bufs[r][t] for r in range(P)], [outs[r][t] for r in range(P)], 4096)
+                         for t in range(len(sizes)))
             algos = collections.Counter(["auto", "ring", "rd", "direct"][q.info()["algo"]] for q in reqs[0])
             print(json.dumps({"model": name, "mode": "per-tensor (graph)", "ranks": P, "tensors": len(sizes),
                               "bytes_per_rank": total, "us_per_step": ms * 1e3,
-                              "busbw_gbs": busbw(total, ms / 1e3, P), "algos": dict(algos), "errors": errs}),
+                              "busbw_gbs": busbw(total, ms / 1e3, P), "algos": dict(algos), "errors": errs,
+                              "parity": parity}),
                   flush=True)
             for q in flat:
                 q.free()
@@ -266,7 +331,12 @@ def sweep_p2p(args):
     g2, cs = pc.local_comms(2, 0)
     st = torch.cuda.Stream()
     elems = {apps.GRAN_THREAD: 2, apps.GRAN_WARP: 64, apps.GRAN_BLOCK: 2048}
-    for S in [64 << 10, 1 << 20, 16 << 20, 256 << 20]:
+    sizes = [int(x) for x in args.sizes.split(",")] if args.sizes else [64 << 10, 1 << 20, 16 << 20, 256 << 20]
+    grans = {"thread": apps.GRAN_THREAD, "warp": apps.GRAN_WARP, "block": apps.GRAN_BLOCK}
+    gsel = [grans[g] for g in args.grans.split(",")] if args.grans else [apps.GRAN_BLOCK, apps.GRAN_WARP,
+                                                                           apps.GRAN_THREAD]
+    aggsel = args.aggs.split(",") if args.aggs else None
+    for S in sizes:
         n = S // 4
         A = torch.randn(n, device="cuda")
         B = torch.randn(n, device="cuda")
@@ -285,11 +355,13 @@ def sweep_p2p(args):
         print(json.dumps({"bytes": S, "mode": "kernel+copy (traditional, same GPU)",
                           "us": e0.elapsed_time(e1) / it * 1e3,
                           "gbs": S / (e0.elapsed_time(e1) / it / 1e3) / 1e9}), flush=True)
-        for gran in (apps.GRAN_BLOCK, apps.GRAN_WARP, apps.GRAN_THREAD):
+        for gran in gsel:
             cnt = elems[gran]
             parts = n // cnt
             for agg_name, agg in (("none", 1), ("block", max(1, 2048 // cnt)), ("1MiB", max(1, (1 << 18) // cnt)),
                                   ("all", parts)):
+                if aggsel and agg_name not in aggsel:
+                    continue
                 agg = min(agg, parts)
                 for copy in (pc.COPY_INLINE, pc.COPY_ENGINE):
                     if gran == apps.GRAN_THREAD and agg == 1 and S > (16 << 20):
@@ -343,6 +415,9 @@ if __name__ == "__main__":
     ap.add_argument("--partitions", default="1,16,64")
     ap.add_argument("--max-bytes", type=int, default=1 << 30)
     ap.add_argument("--graph", action="store_true", help="replay a captured CUDA graph of the epoch")
+    ap.add_argument("--sizes", default="", help="p2p: buffer bytes, comma separated")
+    ap.add_argument("--grans", default="", help="p2p: thread,warp,block")
+    ap.add_argument("--aggs", default="", help="p2p: none,block,1MiB,all")
     a = ap.parse_args()
     {"allreduce": sweep_allreduce, "dl": sweep_dl, "dl_tensor": sweep_dl_per_tensor, "p2p": sweep_p2p,
      "coll": sweep_coll}[a.what](a)
