@@ -806,6 +806,184 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
 }
 
 // ---------------------------------------------------------------------------
+// Batched DIRECT engine: MPI_Waitall over many partitioned allreduces of one
+// GPU in ONE launch (one request per gradient tensor).
+// Entries (request t, local rank j) live in a device table (DirectArgs are
+// epoch-invariant; each unit reads its request's epoch word).  Global units
+// are ordered [t][x][j] — a logical unit's local ranks are adjacent — and
+// every warp takes its global units in increasing order, so the smallest
+// incomplete logical unit is active on every rank whatever the width
+// (deadlock freedom).  Same steps and bits as direct_body.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ bool warp_poll_all(const uint32_t *words, int n, uint32_t target, bool sys) {
+  const uint32_t lane = threadIdx.x & 31;
+  bool mine = lane >= (uint32_t)n || reached(sys ? ld_acquire_sys(words + lane) : ld_acquire_gpu(words + lane), target);
+  return __all_sync(0xffffffffu, mine);
+}
+
+// Rank-order PULL fold of one slice with rank-indexed source pointers S[k] and
+// destinations D[0] (own recvbuf), D[1..P-1] (peers), all at the same byte
+// offset: scalar head / 16-B body (FV vectors per operand in flight) / tail.
+template <int DT, int OP, int FV>
+__device__ __forceinline__ void warp_fold_ptrs(const uint8_t *const (&S)[kMaxDirect], uint8_t *const (&D)[kMaxDirect],
+                                               int P, int64_t n) {
+  using O = Op<DT, OP>;
+  using T = typename O::T;
+  const uint32_t lane = threadIdx.x & 31;
+  constexpr int64_t EPV = 16 / sizeof(T);
+  const uintptr_t m = reinterpret_cast<uintptr_t>(D[0]) & 15;
+  int64_t head = (int64_t)(((16 - m) & 15) / sizeof(T));
+  if ((reinterpret_cast<uintptr_t>(S[0]) & 15) != m) head = n;
+  if (head > n) head = n;
+  auto scalar = [&](int64_t k) {
+    T acc = __ldcg(reinterpret_cast<const T *>(S[0]) + k);
+#pragma unroll
+    for (int j = 1; j < kMaxDirect; ++j)
+      if (j < P) acc = O::f(acc, __ldcg(reinterpret_cast<const T *>(S[j]) + k));
+#pragma unroll
+    for (int j = 0; j < kMaxDirect; ++j)
+      if (j < P) reinterpret_cast<T *>(D[j])[k] = acc;
+  };
+  for (int64_t k = lane; k < head; k += 32) scalar(k);
+  const int64_t nv = (n - head) / EPV;
+  int64_t k = lane;
+  for (; k + 32 * (FV - 1) < nv; k += 32 * FV) {
+    uint4 x[kMaxDirect][FV];
+#pragma unroll
+    for (int j = 0; j < kMaxDirect; ++j)
+      if (j < P) {
+#pragma unroll
+        for (int v = 0; v < FV; ++v)
+          x[j][v] = __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(S[j]) + head) + k + 32 * v);
+      }
+#pragma unroll
+    for (int v = 0; v < FV; ++v) {
+      uint4 acc = x[0][v];
+#pragma unroll
+      for (int j = 1; j < kMaxDirect; ++j)
+        if (j < P) acc = vop<DT, OP>(acc, x[j][v]);
+#pragma unroll
+      for (int j = 0; j < kMaxDirect; ++j)
+        if (j < P) reinterpret_cast<uint4 *>(reinterpret_cast<T *>(D[j]) + head)[k + 32 * v] = acc;
+    }
+  }
+  for (; k < nv; k += 32) {
+    uint4 acc = __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(S[0]) + head) + k);
+    uint4 x[kMaxDirect];
+#pragma unroll
+    for (int j = 1; j < kMaxDirect; ++j)
+      if (j < P) x[j] = __ldcg(reinterpret_cast<const uint4 *>(reinterpret_cast<const T *>(S[j]) + head) + k);
+#pragma unroll
+    for (int j = 1; j < kMaxDirect; ++j)
+      if (j < P) acc = vop<DT, OP>(acc, x[j]);
+#pragma unroll
+    for (int j = 0; j < kMaxDirect; ++j)
+      if (j < P) reinterpret_cast<uint4 *>(reinterpret_cast<T *>(D[j]) + head)[k] = acc;
+  }
+  for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
+}
+
+template <int DT, int OP, int FV>
+__device__ __forceinline__ void direct_batch_body(const DirectBatchArgs b, const int gw, const int W) {
+  const int R = b.R;
+  const int total = b.ubase[b.nreq];
+  for (int j0 = 0; gw + j0 * W < total; j0 += kMaxActive) {
+    int step[kMaxActive], ent[kMaxActive], unit[kMaxActive];
+    uint32_t ep[kMaxActive];
+    int remaining = 0;
+#pragma unroll
+    for (int jj = 0; jj < kMaxActive; ++jj) {
+      const int g = gw + (j0 + jj) * W;
+      step[jj] = 3;
+      ent[jj] = 0;
+      unit[jj] = 0;
+      ep[jj] = 0;
+      if (g < total) {
+        int lo = 0, hi = b.nreq;  // request t: ubase[t] <= g < ubase[t + 1]
+        while (hi - lo > 1) {
+          const int mid = (lo + hi) >> 1;
+          if (b.ubase[mid] <= g) lo = mid; else hi = mid;
+        }
+        const int off = g - b.ubase[lo];
+        ent[jj] = lo * R + off % R;
+        unit[jj] = off / R;
+        ep[jj] = *(const volatile uint32_t *)b.tab[ent[jj]].epoch;
+        step[jj] = 0;
+        ++remaining;
+      }
+    }
+    Idle idle;
+    while (remaining) {
+      bool progressed = false;
+#pragma unroll
+      for (int jj = 0; jj < kMaxActive; ++jj) {
+        if (step[jj] > 2) continue;
+        const DirectArgs &a = b.tab[ent[jj]];
+        const int P = a.P, r = a.r, ns = a.ns, sys = a.sys;
+        const int u = unit[jj] / ns, s = unit[jj] % ns;
+        const int i = step[jj];
+        const uint32_t e = ep[jj];
+        if (i == 0) {  // the user's Pready of u, and every peer's ready-to-receive
+          if (!warp_poll(a.ready + u, e, false) || !warp_poll_all(a.rtr, P - 1, e, sys)) continue;
+        } else if (!warp_poll(a.cnt + ((int64_t)u * 2 + (i - 1)) * ns + s, e * (uint32_t)(P - 1), sys)) {
+          continue;
+        }
+        progressed = true;
+        if (i == 0) {
+          fence_scope(sys);
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0)
+            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 0) * ns + s, 1, sys);
+          step[jj] = 1;
+        } else if (i == 1) {
+          const int64_t es = sizeof(typename Op<DT, OP>::T);
+          const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
+          const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
+          if (hi > lo) {
+            const int64_t boff = ((int64_t)u * a.L + lo) * es;
+            const uint8_t *S[kMaxDirect];
+            uint8_t *D[kMaxDirect];
+#pragma unroll
+            for (int k = 0; k < kMaxDirect; ++k) {  // rank-indexed sources, D[0] = own recvbuf
+              S[k] = nullptr;
+              D[k] = nullptr;
+              if (k < P) {
+                S[k] = (k == r ? a.sendbuf : a.p_sendbuf[(k - r - 1 + P) % P]) + boff;
+                D[k] = (k == 0 ? a.recvbuf : a.p_recvbuf[k - 1]) + boff;
+              }
+            }
+            warp_fold_ptrs<DT, OP, FV>(S, D, P, hi - lo);
+          }
+          fence_scope(sys);
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0)
+            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * ns + s, 1, sys);
+          step[jj] = 2;
+        } else {
+          if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+          step[jj] = 3;
+          --remaining;
+        }
+      }
+      if (progressed)
+        idle.progressed();
+      else if (!idle.wait(b.err, b.timeout_ms, gw))
+        return;
+    }
+  }
+}
+
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine_batch(DirectBatchArgs b) {
+  direct_batch_body<DT, OP, PC_DIRECT_FV>(b, (blockIdx.x * blockDim.x + threadIdx.x) >> 5,
+                                          (gridDim.x * blockDim.x) >> 5);
+}
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_batch_thin(DirectBatchArgs b) {
+  direct_batch_body<DT, OP, 1>(b, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
+}
+
+// ---------------------------------------------------------------------------
 // Partitioned reduce-scatter / allgather / broadcast: the two
 // halves of the DIRECT schedule and its one-to-all special case, same unit
 // sweep (Alg 2 on a warp).  Unit (u, slice s) of one block of `count` elements.
@@ -1029,6 +1207,7 @@ struct EngineLaunch {
   static int ring_group(const RingGroupArgs &h, int blocks, cudaStream_t s);
   static int rd_group(const RdGroupArgs &h, int blocks, cudaStream_t s);
   static int direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s, bool thin);
+  static int direct_batch(const DirectBatchArgs &b, int blocks, cudaStream_t s, bool thin);
   static int coll(const CollArgs &a, int warps, cudaStream_t s);
   static int coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s);
   static int occupancy(int *ctas);

@@ -84,6 +84,17 @@ int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cud
 }
 
 template <int DT, int OP>
+int EngineLaunch<DT, OP>::direct_batch(const DirectBatchArgs &b, int blocks, cudaStream_t s, bool thin) {
+  if (thin)
+    direct_engine_batch_thin<DT, OP><<<blocks, kEngineBlock, 0, s>>>(b);
+  else
+    direct_engine_batch<DT, OP><<<blocks, kEngineBlock, 0, s>>>(b);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+template <int DT, int OP>
 int EngineLaunch<DT, OP>::occupancy(int *ctas) {
   int a = 0, b = 0;
   PC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&a, ring_engine<DT, OP>, kEngineBlock, 0));
@@ -137,6 +148,8 @@ int EngineLaunch<DT, OP>::preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group_thin<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_batch<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_batch_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP>));
   return 0;

@@ -897,8 +897,12 @@ static int fork_point(Request *q, cudaStream_t s) {
   if (q->comm->dry || !q->ev_fork) return 0;
   PC_CUDA(cudaEventRecord(q->ev_fork, s));
   q->forked = true;
+  q->fork_ev_ext = nullptr;
   return 0;
 }
+// The event the engine forks from: the request's own, or the one a batched
+// control call recorded once for all its requests.
+static cudaEvent_t fork_event(const Request *q) { return q->fork_ev_ext ? q->fork_ev_ext : q->ev_fork; }
 
 // The engine's width.  When every partition was made ready by a host-side op
 // before ev_fork (pc_epoch_all with Pready, pc_preadyall, pc_pready_range of
@@ -926,11 +930,10 @@ static bool group_blocks_start(Request *q) {
 static int epoch_begin(Request *q, cudaStream_t s, bool capturing) {
   if (group_blocks_start(q)) return PC_ERR_STATE;
   if (!q->comm->dry && q->epoch > 0 && !capturing && q->joined_stream != s && q->joined_stream != kHostJoined &&
-      needs_engine(q) && q->engine_launched) {
-    cudaEvent_t ev = q->leader ? q->leader->gs.ev : q->ev_done;
-    if (ev) PC_CUDA(cudaStreamWaitEvent(s, ev, 0));
-  }
+      needs_engine(q) && q->engine_launched && q->last_done)
+    PC_CUDA(cudaStreamWaitEvent(s, q->last_done, 0));
   q->forked = false;
+  q->batch_launched = false;
   q->host_ready_all = false;
   q->join_pending = false;
   return 0;
@@ -938,8 +941,11 @@ static int epoch_begin(Request *q, cudaStream_t s, bool capturing) {
 
 // Single-rank launch on the request's side stream, forked from ev_fork.
 static int launch_single(Request *q) {
-  if (!q->forked || !q->overlap) PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
-  PC_CUDA(cudaStreamWaitEvent(q->side, q->ev_fork, 0));
+  if (!q->forked || !q->overlap) {
+    PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+    q->fork_ev_ext = nullptr;
+  }
+  PC_CUDA(cudaStreamWaitEvent(q->side, fork_event(q), 0));
   const bool full = full_width(q);
   const int w = engine_width(q, full);
   int rc, tk;
@@ -978,6 +984,7 @@ static int launch_single(Request *q) {
   if ((rc = timing_end(q->tlog, q->side, tk))) return rc;
   PC_CUDA(cudaEventRecord(q->ev_done, q->side));
   q->engine_launched = true;
+  q->last_done = q->ev_done;
   return 0;
 }
 
@@ -997,14 +1004,19 @@ static int group_register(Request *q, bool block, cudaStream_t ws, bool *launche
     g.launched = false;
   }
   if (!q->engine_registered) {
-    if (!q->forked || !q->overlap) PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+    if (!q->forked || !q->overlap) {
+      PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+      q->fork_ev_ext = nullptr;
+    }
     q->engine_registered = true;
     g.pending++;
   }
   if (!g.launched && g.pending == (int)g.members.size()) {
     bool full = true;
+    cudaEvent_t waited = nullptr;
     for (Request *m : g.members) {
-      PC_CUDA(cudaStreamWaitEvent(q->side, m->ev_fork, 0));
+      if (fork_event(m) != waited) PC_CUDA(cudaStreamWaitEvent(q->side, fork_event(m), 0));
+      waited = fork_event(m);  // members forked by one batched call share the event
       full = full && full_width(m);
     }
     const int w = engine_width(q, full);
@@ -1034,6 +1046,7 @@ static int group_register(Request *q, bool block, cudaStream_t ws, bool *launche
     if (rc) return rc;
     if ((rc = timing_end(g.tlog, q->side, tk))) return rc;
     PC_CUDA(cudaEventRecord(g.ev, q->side));
+    for (Request *m : g.members) m->last_done = g.ev;
     // members that already waited on their own stream (before the group was
     // complete) get their completion ordered there now (pc.h "In-process
     // rank groups": work they enqueued between their wait and this launch is
@@ -1080,6 +1093,206 @@ static int error_rc(Request *q) {
   if (code == 0) return 0;
   fprintf(stderr, "[pc] rank %d request %d: device error %d (partition %d)\n", q->comm->rank, q->index, code, part);
   return code == PC_ERR_TIMEOUT ? PC_ERR_TIMEOUT : PC_ERR_DEVICE;
+}
+
+// ---------------------------------------------------------------- batch caches
+// Device tables of batched calls over a fixed request list (BatchCache,
+// pc_internal.h).  Built eagerly on first use (a synchronous copy: not while
+// a stream captures), reused every epoch, dropped with any of its requests.
+static std::mutex g_batch_mu;
+static std::map<std::vector<Request *>, BatchCache *> g_epoch_batches, g_engine_batches;
+
+static void batch_destroy(BatchCache *b) {
+  for (Request *q : b->reqs) {
+    if (q->fork_ev_ext == b->ev) {
+      q->fork_ev_ext = nullptr;
+      q->forked = false;
+    }
+    if (q->last_done == b->ev) q->last_done = nullptr;
+  }
+  if (b->dev) cudaFree(b->dev);
+  if (b->ev) cudaEventDestroy(b->ev);
+  delete b;
+}
+
+// Drop every cache that lists q (pc_request_free).
+static void batch_drop(Request *q) {
+  std::lock_guard<std::mutex> lk(g_batch_mu);
+  for (auto *m : {&g_epoch_batches, &g_engine_batches})
+    for (auto it = m->begin(); it != m->end();) {
+      if (std::find(it->first.begin(), it->first.end(), q) != it->first.end()) {
+        batch_destroy(it->second);
+        it = m->erase(it);
+      } else {
+        ++it;
+      }
+    }
+}
+
+static int batch_upload(BatchCache *b, const void *host, size_t bytes, cudaStream_t s) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  PC_CUDA(cudaStreamIsCapturing(s, &cs));
+  if (cs != cudaStreamCaptureStatusNone) return PC_ERR_STATE;  // first use of a request list: eagerly
+  PC_CUDA(cudaMalloc(&b->dev, bytes));
+  PC_CUDA(cudaMemcpy(b->dev, host, bytes, cudaMemcpyHostToDevice));
+  b->dev_bytes = bytes;
+  PC_CUDA(cudaEventCreateWithFlags(&b->ev, cudaEventDisableTiming));
+  return 0;
+}
+
+// pc_epoch_all over more requests / RTR words than one kernel's parameters
+// hold: one single-block kernel reading the lists from device memory, one
+// fork event for all requests.
+static int epoch_all_batched(const std::vector<Request *> &rq, int pready, cudaStream_t s) {
+  BatchCache *b = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(g_batch_mu);
+    auto it = g_epoch_batches.find(rq);
+    if (it != g_epoch_batches.end()) b = it->second;
+  }
+  if (!b) {
+    b = new BatchCache();
+    b->reqs = rq;
+    std::vector<EpochEnt> ent(rq.size());
+    std::vector<RtrEnt> rtr;
+    for (size_t i = 0; i < rq.size(); ++i) {
+      Request *q = rq[i];
+      ent[i].epoch = q->ctrl + q->L.epoch;
+      ent[i].ready = q->ctrl + q->L.ready;
+      ent[i].partitions = q->partitions;
+      for (auto &t : q->rtr_targets) rtr.push_back({t.first + q->L.rtr + t.second, (int)i, q->sys_scope});
+    }
+    std::vector<int> big;
+    for (size_t i = 0; i < rq.size(); ++i)
+      if (rq[i]->partitions > kEpochSmallParts) big.push_back((int)i);
+    const size_t o_rtr = ent.size() * sizeof(EpochEnt), o_big = o_rtr + rtr.size() * sizeof(RtrEnt);
+    std::vector<uint8_t> host(o_big + big.size() * sizeof(int));
+    memcpy(host.data(), ent.data(), o_rtr);
+    if (!rtr.empty()) memcpy(host.data() + o_rtr, rtr.data(), rtr.size() * sizeof(RtrEnt));
+    if (!big.empty()) memcpy(host.data() + o_big, big.data(), big.size() * sizeof(int));
+    b->n = (int)ent.size();
+    b->nrtr = (int)rtr.size();
+    b->nreq = (int)big.size();  // (epoch batch: the large-request list)
+    if (int rc = batch_upload(b, host.data(), host.size(), s)) {
+      batch_destroy(b);
+      return rc;
+    }
+    std::lock_guard<std::mutex> lk(g_batch_mu);
+    g_epoch_batches[rq] = b;
+  }
+  EpochBatchArgs a{};
+  a.n = b->n;
+  a.nrtr = b->nrtr;
+  a.pready = pready ? 1 : 0;
+  a.ent = (const EpochEnt *)b->dev;
+  a.rtr = (const RtrEnt *)((const uint8_t *)b->dev + (size_t)b->n * sizeof(EpochEnt));
+  a.nbig = b->nreq;
+  a.big = (const int *)((const uint8_t *)a.rtr + (size_t)b->nrtr * sizeof(RtrEnt));
+  if (int rc = launch_epoch_batch(a, s)) return rc;
+  PC_CUDA(cudaEventRecord(b->ev, s));
+  for (Request *q : rq) {
+    q->host_ready_all = pready != 0;
+    q->forked = true;
+    q->fork_ev_ext = b->ev;
+  }
+  return 0;
+}
+
+// pc_waitall_on_stream over several DIRECT allreduces of one GPU: ONE
+// batched engine launch (direct_engine_batch) instead of one per request.
+// Eligible: engine-moved (not INLINE) DIRECT allreduces, one dtype / op,
+// not yet launched this epoch, and either all single-rank (R = 1) or all
+// members of co-located groups of the same size R whose members are all in
+// the list.  Returns 1 if the batch was not applicable (caller falls back).
+static int engine_batch(const std::vector<Request *> &rq, cudaStream_t s) {
+  if (rq.size() < 2) return 1;
+  Request *q0 = rq[0];
+  const int R = q0->leader ? (int)q0->leader->gs.members.size() : 1;
+  std::vector<Request *> leaders;
+  for (Request *q : rq) {
+    if (q->kind != PC_KIND_PALLREDUCE || q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT ||
+        q->inline_ar || !q->active || q->engine_registered || q->engine_launched || q->batch_launched)
+      return 1;
+    if (q->dtype != q0->dtype || q->op != q0->op || q->comm->device != q0->comm->device) return 1;
+    const int r = q->leader ? (int)q->leader->gs.members.size() : 1;
+    if (r != R || (R > 1) != (q->leader != nullptr)) return 1;
+    Request *ld = q->leader ? q->leader : q;
+    if (std::find(leaders.begin(), leaders.end(), ld) == leaders.end()) leaders.push_back(ld);
+  }
+  if ((int)(leaders.size() * R) != (int)rq.size() || leaders.size() < 2) return 1;
+  for (Request *ld : leaders)  // every group complete in the list
+    if (R > 1)
+      for (Request *m : ld->gs.members)
+        if (std::find(rq.begin(), rq.end(), m) == rq.end()) return 1;
+  BatchCache *b = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(g_batch_mu);
+    auto it = g_engine_batches.find(rq);
+    if (it != g_engine_batches.end()) b = it->second;
+  }
+  if (!b) {
+    b = new BatchCache();
+    b->reqs = rq;
+    b->nreq = (int)leaders.size();
+    b->R = R;
+    b->dtype = q0->dtype;
+    b->op = q0->op;
+    std::vector<DirectArgs> tab;
+    std::vector<int> ubase(1, 0);
+    for (Request *ld : leaders) {
+      if (R > 1)
+        for (Request *m : ld->gs.members) tab.push_back(make_direct_args(m));
+      else
+        tab.push_back(make_direct_args(ld));
+      ubase.push_back(ubase.back() + ld->partitions * ld->slices * R);
+    }
+    b->units = ubase.back();
+    std::vector<uint8_t> host(tab.size() * sizeof(DirectArgs) + ubase.size() * sizeof(int));
+    memcpy(host.data(), tab.data(), tab.size() * sizeof(DirectArgs));
+    memcpy(host.data() + tab.size() * sizeof(DirectArgs), ubase.data(), ubase.size() * sizeof(int));
+    if (int rc = batch_upload(b, host.data(), host.size(), s)) {
+      batch_destroy(b);
+      return rc;
+    }
+    std::lock_guard<std::mutex> lk(g_batch_mu);
+    g_engine_batches[rq] = b;
+  }
+  bool full = true;
+  for (Request *q : rq) full = full && full_width(q);
+  // width: the whole GPU's engine capacity (every local rank's share), or the
+  // overlap bound while producers may still run (thin CTAs)
+  const int per_rank = full ? q0->engine_warps : std::min(q0->engine_warps, q0->comm->overlap_warps);
+  const int warps = std::max(1, std::min(per_rank * R, b->units));
+  const int blocks = (warps * 32 + kEngineBlock - 1) / kEngineBlock;
+  cudaStream_t side = q0->side;
+  cudaEvent_t waited = nullptr;
+  for (Request *q : rq) {
+    if (!q->forked || !q->overlap) {
+      PC_CUDA(cudaEventRecord(q->ev_fork, q->user_stream));
+      q->fork_ev_ext = nullptr;
+    }
+    if (fork_event(q) != waited) PC_CUDA(cudaStreamWaitEvent(side, fork_event(q), 0));
+    waited = fork_event(q);
+  }
+  DirectBatchArgs a{};
+  a.tab = (const DirectArgs *)b->dev;
+  a.ubase = (const int *)((const uint8_t *)b->dev + (size_t)b->nreq * R * sizeof(DirectArgs));
+  a.nreq = b->nreq;
+  a.R = R;
+  a.err = (int32_t *)(q0->ctrl + q0->L.err);
+  a.timeout_ms = q0->comm->timeout_ms;
+  if (int rc = launch_direct_engine_batch(a, b->dtype, b->op, blocks, side, !full && q0->comm->overlap_thin))
+    return rc;
+  PC_CUDA(cudaEventRecord(b->ev, side));
+  PC_CUDA(cudaStreamWaitEvent(s, b->ev, 0));
+  for (Request *q : rq) {
+    q->engine_launched = true;
+    q->batch_launched = true;
+    q->last_done = b->ev;
+    q->joined_stream = s;
+    q->active = false;
+  }
+  return 0;
 }
 
 }  // namespace pc
@@ -1519,7 +1732,7 @@ int pc_pbuf_prepare(pc_request_t req, pc_stream_t stream) {
 // requests of one GPU in ONE kernel (the small-message epoch: one launch
 // instead of three; CUDA-graph capturable).
 int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream) {
-  if (n < 1 || !reqs || n > kMaxPreadyAll) return PC_ERR_ARG;
+  if (n < 1 || !reqs) return PC_ERR_ARG;
   // validate everything before any request is touched (no half-started batch)
   int nrtr = 0;
   for (int i = 0; i < n; ++i) {
@@ -1537,11 +1750,29 @@ int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream) {
     nrtr += (int)q->rtr_targets.size();
   }
   const bool dry = ((Request *)reqs[0])->comm->dry;
-  if (!dry && nrtr > kMaxCtl) return PC_ERR_UNSUPPORTED;
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
   if (!dry) {
     PC_CUDA(cudaSetDevice(((Request *)reqs[0])->comm->device));
     PC_CUDA(cudaStreamIsCapturing((cudaStream_t)stream, &cs));
+  }
+  if (!dry && (n > kMaxPreadyAll || nrtr > kMaxCtl)) {  // beyond one kernel's parameters: device tables
+    std::vector<Request *> rq(n);
+    for (int i = 0; i < n; ++i) rq[i] = (Request *)reqs[i];
+    {
+      std::lock_guard<std::mutex> lk(g_batch_mu);
+      if (!g_epoch_batches.count(rq) && cs != cudaStreamCaptureStatusNone) return PC_ERR_STATE;
+    }
+    for (Request *q : rq) {
+      if (int rc = epoch_begin(q, (cudaStream_t)stream, cs != cudaStreamCaptureStatusNone)) return rc;
+      if (cs != cudaStreamCaptureStatusNone) q->graph_mode = true;
+      q->epoch++;
+      q->active = true;
+      q->engine_launched = false;
+      q->engine_registered = false;
+      q->prepared_this_epoch = true;
+      q->user_stream = (cudaStream_t)stream;
+    }
+    return epoch_all_batched(rq, pready, (cudaStream_t)stream);
   }
   EpochAllArgs a{};
   for (int i = 0; i < n; ++i) {
@@ -1753,6 +1984,10 @@ int pc_prequest_free(pc_prequest_t *preq) {
 static int ensure_engine(Request *q, bool block, cudaStream_t ws, cudaEvent_t *ev) {
   *ev = nullptr;
   if (!needs_engine(q)) return 0;
+  if (q->batch_launched) {  // this epoch's engine ran in a batched waitall launch
+    *ev = q->last_done;
+    return 0;
+  }
   if (q->leader) {
     bool launched = false;
     int rc = group_register(q, block, ws, &launched);
@@ -1860,7 +2095,19 @@ int pc_waitall_on_stream(int n, pc_request_t *reqs, pc_stream_t stream) {
     if (!fused.empty() && q->comm->device != fused[0]->comm->device) return PC_ERR_ARG;
     fused.push_back(q);
   }
-  for (int i = 0; i < n; ++i) {  // engine-moved and dry requests: their own path
+  {  // several DIRECT allreduces: one batched engine launch
+    std::vector<Request *> eng;
+    for (int i = 0; i < n; ++i) {
+      Request *q = (Request *)reqs[i];
+      if (q->active && !q->comm->dry && needs_engine(q) && q->kind == PC_KIND_PALLREDUCE) eng.push_back(q);
+    }
+    if (eng.size() >= 2) {
+      PC_CUDA(cudaSetDevice(eng[0]->comm->device));
+      const int rc = engine_batch(eng, s);
+      if (rc < 0) return rc;
+    }
+  }
+  for (int i = 0; i < n; ++i) {  // engine-moved (not batched) and dry requests: their own path
     Request *q = (Request *)reqs[i];
     if (std::find(fused.begin(), fused.end(), q) != fused.end()) continue;
     if (int rc = wait_common(q, s, false)) return rc;
@@ -2115,6 +2362,7 @@ int pc_request_free(pc_request_t *req) {
   if (!c->dry) {
     cudaSetDevice(c->device);
     if (q->side) cudaStreamSynchronize(q->side);
+    batch_drop(q);
     if (q->hready || q->pe_registered) progress_unregister(q);
     if (q->ctrl) cudaFree(q->ctrl);
     if (q->staging) cudaFree(q->staging);

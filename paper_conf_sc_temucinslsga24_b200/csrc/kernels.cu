@@ -260,6 +260,56 @@ __global__ void __launch_bounds__(1024) epoch_all_kernel(EpochAllArgs a) {
   }
 }
 
+// pc_epoch_all over any number of requests: the three barrier-ordered
+// phases of epoch_all_kernel with the lists in device memory.  The new epochs
+// are kept in shared memory (no dependent global loads per RTR / Pready);
+// every thread owns whole requests for the Pready of small ones, the block
+// sweeps the few large ones together.
+constexpr int kEpochBatchSmem = 8192;
+__global__ void __launch_bounds__(1024) epoch_batch_kernel(EpochBatchArgs a) {
+  __shared__ uint32_t esh[kEpochBatchSmem];
+  const int t = threadIdx.x;
+  for (int i = t; i < a.n; i += blockDim.x) {
+    uint32_t *ep = a.ent[i].epoch;
+    const uint32_t e = *ep + 1;
+    *ep = e;
+    if (i < kEpochBatchSmem) esh[i] = e;
+  }
+  __syncthreads();
+  auto epoch = [&](int i) -> uint32_t {
+    return i < kEpochBatchSmem ? esh[i] : *(const volatile uint32_t *)a.ent[i].epoch;
+  };
+  // ready-to-receive: one fence per thread at the strongest scope it stores
+  // at, then relaxed stores (the earlier consumers of each recvbuf finished
+  // in earlier kernels of this stream)
+  bool fsys = false, fgpu = false;
+  for (int k = t; k < a.nrtr; k += blockDim.x) {
+    const RtrEnt r = a.rtr[k];
+    if (r.sys) {
+      if (!fsys) fence_sys();
+      fsys = true;
+      st_relaxed_sys(r.dst, epoch(r.req));
+    } else {
+      if (!fgpu && !fsys) fence_gpu();
+      fgpu = true;
+      st_relaxed_gpu(r.dst, epoch(r.req));
+    }
+  }
+  if (!a.pready) return;
+  for (int i = t; i < a.n; i += blockDim.x) {  // S_0 of every partition (ordering as in epoch_all_kernel)
+    const EpochEnt en = a.ent[i];
+    if (!en.ready || en.partitions > kEpochSmallParts) continue;
+    const uint32_t e = epoch(i);
+    for (int j = 0; j < en.partitions; ++j) st_relaxed_gpu(en.ready + j, e);
+  }
+  for (int b = 0; b < a.nbig; ++b) {
+    const int i = a.big[b];
+    const EpochEnt en = a.ent[i];
+    const uint32_t e = epoch(i);
+    for (int j = t; j < en.partitions; j += blockDim.x) st_relaxed_gpu(en.ready + j, e);
+  }
+}
+
 __global__ void pready_range_kernel(pc_prequest_t q, int lo, int hi) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int W = (gridDim.x * blockDim.x) >> 5;
@@ -349,6 +399,10 @@ int launch_direct_engine_group(const DirectGroupArgs &g, int warps, cudaStream_t
     blocks += grid_for(warps, g.a[k].nunits);
   }
   return dispatch(g.a[0].dtype, g.a[0].op, [&](auto E) { return decltype(E)::direct_group(h, blocks, s, thin); });
+}
+
+int launch_direct_engine_batch(const DirectBatchArgs &b, int dtype, int op, int blocks, cudaStream_t s, bool thin) {
+  return dispatch(dtype, op, [&](auto E) { return decltype(E)::direct_batch(b, blocks, s, thin); });
 }
 
 int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
@@ -473,6 +527,7 @@ int kernels_preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, rtr_kernel));
   PC_CUDA(cudaFuncGetAttributes(&fa, pready_all_kernel));
   PC_CUDA(cudaFuncGetAttributes(&fa, epoch_all_kernel));
+  PC_CUDA(cudaFuncGetAttributes(&fa, epoch_batch_kernel));
   PC_CUDA(cudaFuncGetAttributes(&fa, pready_range_kernel));
   if (int rc = pe_kernels_preload()) return rc;
   for (int dt : {PC_INT32, PC_FLOAT32, PC_FLOAT64, PC_BF16})
@@ -509,6 +564,13 @@ int launch_pready_all(const PreadyAllArgs &a, cudaStream_t s) {
   if (blocks > 148) blocks = 148;
   if (blocks < 1) blocks = 1;
   pready_all_kernel<<<blocks, 256, 0, s>>>(a);
+  g_launches++;
+  PC_CUDA(cudaGetLastError());
+  return 0;
+}
+
+int launch_epoch_batch(const EpochBatchArgs &a, cudaStream_t s) {
+  epoch_batch_kernel<<<1, 1024, 0, s>>>(a);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;

@@ -171,6 +171,9 @@ struct Request {
   // created with PC_COPY_INLINE — the completing Pready folds, no engine
   bool inline_ar = false;
   void *ar_tab = nullptr;       // device pc_ar_tab_s (library-owned)
+  cudaEvent_t fork_ev_ext = nullptr;  // fork point recorded by a batched control call (else ev_fork)
+  cudaEvent_t last_done = nullptr;    // completion of the last launched engine (single / group / batch)
+  bool batch_launched = false;        // this epoch's engine ran in a batched waitall launch
   // stream on which the previous epoch's completion is ordered (null: host
   // observed it); a later epoch's control op on another stream first waits
   // for that completion (the engine reads the epoch word at entry)
@@ -239,6 +242,21 @@ struct Progress {
   std::atomic<int> err{0};
   cudaStream_t stream = nullptr;
   bool started = false;
+};
+
+// Device tables of a batched control / wait call over a fixed list of
+// requests (pc_epoch_all with > 16 requests, pc_waitall_on_stream over many
+// allreduces), built once per distinct request list and reused every epoch;
+// dropped when one of its requests is freed.
+struct BatchCache {
+  std::vector<Request *> reqs;
+  void *dev = nullptr;       // tables (layout per kind)
+  size_t dev_bytes = 0;
+  int n = 0, nrtr = 0;       // epoch batch: request / RTR entries
+  int nreq = 0, R = 1;       // engine batch: logical requests x local ranks
+  int units = 0;
+  int dtype = 0, op = 0;
+  cudaEvent_t ev = nullptr;  // fork point (epoch batch) / completion (engine batch)
 };
 
 struct Comm {
@@ -350,6 +368,17 @@ struct DirectGroupArgs {
   int block_start[kMaxLocal];
   DirectArgs a[kMaxLocal];
 };
+// Batched DIRECT engine (pc_waitall_on_stream over many allreduces of one
+// GPU): entries (request t, local rank j) = tab[t * R + j] in device memory,
+// ubase[t] = first global unit of request t (units ordered [t][x][j]).
+struct DirectBatchArgs {
+  const DirectArgs *tab;
+  const int *ubase;  // [nreq + 1]
+  int nreq, R;
+  int32_t *err;      // the first request's error word (idle timeouts)
+  uint32_t timeout_ms;
+};
+int launch_direct_engine_batch(const DirectBatchArgs &b, int dtype, int op, int blocks, cudaStream_t s, bool thin);
 // Partitioned reduce-scatter / allgather / broadcast on the
 // DIRECT machinery (engine.cuh coll_body).  Unit (u, slice s) of a block of
 // `count` elements.
@@ -446,6 +475,27 @@ struct EpochAllArgs {
 };
 static_assert(sizeof(EpochAllArgs) <= 1024, "EpochAllArgs: keep kernel parameters small");
 int launch_epoch_all(const EpochAllArgs &a, cudaStream_t s);
+// pc_epoch_all for any number of requests (many per-tensor allreduces): the
+// same three phases in one block, the request and RTR lists in device memory.
+struct EpochEnt {
+  uint32_t *epoch;
+  uint32_t *ready;  // null: no Pready
+  int partitions;
+  int pad;
+};
+struct RtrEnt {
+  uint32_t *dst;
+  int req;  // index into the EpochEnt list (the RTR carries its epoch)
+  int sys;
+};
+struct EpochBatchArgs {
+  int n, nrtr, pready, nbig;
+  const EpochEnt *ent;
+  const RtrEnt *rtr;
+  const int *big;  // requests with more than kEpochSmallParts partitions (block-cooperative Pready)
+};
+constexpr int kEpochSmallParts = 64;
+int launch_epoch_batch(const EpochBatchArgs &a, cudaStream_t s);
 // pc_waitall_on_stream: the p2p waits of up to kMaxWaitAll requests in one
 // kernel; request k owns blocks [block_start[k], block_start[k+1]).
 constexpr int kMaxWaitAll = 4;

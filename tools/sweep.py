@@ -291,10 +291,18 @@ def sweep_dl_per_tensor(args):
             epoch_rest()
             torch.cuda.synchronize()
 
-            def epoch():
-                pc.startall(flat, st)
-                pc.pbuf_prepare_all(flat, st)
-                epoch_rest()
+            if args.batched:  # one pc_epoch_all (table kernel) + one batched engine launch
+                def epoch():
+                    pc.epoch_all(flat, pready=True, stream=st)
+                    pc.waitall_on_stream(flat, st)
+
+                epoch()  # eager first: the batch tables are built outside the capture
+                torch.cuda.synchronize()
+            else:
+                def epoch():
+                    pc.startall(flat, st)
+                    pc.pbuf_prepare_all(flat, st)
+                    epoch_rest()
 
             gr = torch.cuda.CUDAGraph()
             with torch.cuda.graph(gr, stream=st):
@@ -313,7 +321,8 @@ def sweep_dl_per_tensor(args):
             parity = all(fp32_gate([bufs[r][t] for r in range(P)], [outs[r][t] for r in range(P)], 4096)
                          for t in range(len(sizes)))
             algos = collections.Counter(["auto", "ring", "rd", "direct"][q.info()["algo"]] for q in reqs[0])
-            print(json.dumps({"model": name, "mode": "per-tensor (graph)", "ranks": P, "tensors": len(sizes),
+            print(json.dumps({"model": name, "mode": "per-tensor (graph%s)" % (", batched" if args.batched else ""),
+                              "ranks": P, "tensors": len(sizes),
                               "bytes_per_rank": total, "us_per_step": ms * 1e3,
                               "busbw_gbs": busbw(total, ms / 1e3, P), "algos": dict(algos), "errors": errs,
                               "parity": parity}),
@@ -416,6 +425,7 @@ if __name__ == "__main__":
     ap.add_argument("--max-bytes", type=int, default=1 << 30)
     ap.add_argument("--graph", action="store_true", help="replay a captured CUDA graph of the epoch")
     ap.add_argument("--sizes", default="", help="p2p: buffer bytes, comma separated")
+    ap.add_argument("--batched", action="store_true", help="dl_tensor: pc_epoch_all + pc_waitall_on_stream batch")
     ap.add_argument("--grans", default="", help="p2p: thread,warp,block")
     ap.add_argument("--aggs", default="", help="p2p: none,block,1MiB,all")
     a = ap.parse_args()
