@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--impl", default="pc", choices=["pc", "reference"])
     ap.add_argument("--bytes", type=int, default=256 << 20, help="bytes per rank (S)")
     ap.add_argument("--partitions", type=int, default=64)
-    ap.add_argument("--algo", default="auto", choices=["ring", "rd", "direct", "auto"])
+    ap.add_argument("--algo", default="auto", choices=["ring", "rd", "direct", "direct_push", "auto"])
     ap.add_argument("--vranks", type=int, default=8, help="virtual ranks on the one GPU when N = 1")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -78,6 +78,8 @@ def engine_alg_bytes(algo, P, S):
         return 2 * S
     if algo == "direct":
         return 2 * P * S
+    if algo == "direct_push":  # push (P-1)/P*S read + written, then fold S read + S written, per rank
+        return int(2 * (P - 1) * S + 2 * P * S)
     if algo == "rd":
         return (4 * (P.bit_length() - 1) + 2) * P * S
     return (5 * P - 4) * S
@@ -473,7 +475,8 @@ def run_virtual(args):
     P, S, Np = args.vranks, args.bytes, args.partitions
     count = S // 4 // Np
     S = count * 4 * Np
-    algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "auto": pc.ALGO_AUTO}[args.algo]
+    algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "direct_push": pc.ALGO_DIRECT_PUSH,
+            "auto": pc.ALGO_AUTO}[args.algo]
     g, comms = pc.local_comms(P, 0)
     st = torch.cuda.Stream()
     gen = torch.Generator(device="cuda")
@@ -959,7 +962,8 @@ def run_multi(args):
         S = min(S, 16 << 20)
     count = S // 4 // Np
     S = count * 4 * Np
-    algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "auto": pc.ALGO_AUTO}[args.algo]
+    algo = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "direct_push": pc.ALGO_DIRECT_PUSH,
+            "auto": pc.ALGO_AUTO}[args.algo]
     comm = pc.Comm.from_process_group(local)
     st = torch.cuda.Stream()
     gen = torch.Generator(device="cuda")
@@ -1024,6 +1028,29 @@ def run_multi(args):
     eng = q.engine_times()
     eng_ms = ctx.max(float(np.mean(eng)) if len(eng) else 0.0)
     assert q.error()[0] == 0
+
+    # the DIRECT schedule's other variant on the same bytes (PULL <-> PUSH):
+    # whichever direction of NVLink traffic the fabric serves better
+    other = None
+    if info["algo_name"] in ("direct", "direct_push"):
+        oalgo = pc.ALGO_DIRECT_PUSH if info["algo_name"] == "direct" else pc.ALGO_DIRECT
+        q2 = pc.pallreduce_init(send, recv, Np, count, pc.FLOAT32, pc.SUM, oalgo, comm)
+        q2.start(st)
+        q2.pbuf_prepare(st)
+        q2.pready_range(0, Np - 1, st)
+        q2.wait_on_stream(st)
+
+        def step2():
+            pc.epoch_all([q2], pready=True, stream=st)
+            q2.wait_on_stream(st)
+
+        ms2 = ctx.time_ms(step2, steps, st, warm=max(args.warmup, 1))
+        ok2 = bool(((recv[idx].double() - ref).abs() <= bound).all().item()) and q2.error()[0] == 0
+        ok2 = ctx.max(0.0 if ok2 else 1.0) == 0.0
+        other = {"algo": q2.info()["algo_name"], "value": busbw(S, ms2 / 1e3, P), "ms_per_step": ms2, "unit": "GB/s",
+                 "parity": ok2}
+        q2.free()
+    log("direct variant done")
 
     nccl = {"skipped": "ranks share a GPU (debug run): NCCL needs one GPU per rank"}
     if not shared:
@@ -1095,7 +1122,8 @@ def run_multi(args):
                "e2e": {"value": busbw(S, ems / 1e3, P), "unit": "GB/s", "h2d_bytes_per_step": S,
                        "d2h_bytes_per_step": S, "ms_per_step": ems,
                        "api": "pc_epoch_all(pready) + pc_wait_on_stream, host buffers copied in/out each step"},
-               "gpu_launches": launches, "clocks": clk.summary(), "nccl": nccl, "p2p": p2p, "jacobi": jac}
+               "gpu_launches": launches, "clocks": clk.summary(), "nccl": nccl, "direct_other_variant": other,
+               "p2p": p2p, "jacobi": jac}
         print(json.dumps(out), flush=True)
     dist.destroy_process_group()
 

@@ -74,7 +74,13 @@ typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1, PC_COPY_LL = 2, PC_COPY_H
  * AUTO = DIRECT for 3 <= P <= 8 (RD for P = 2 up to PC_RD_MAX_BYTES, default
  * 4 MiB; PC_DIRECT_MAX_BYTES caps DIRECT); for P > 8 RD up to
  * PC_RD_MAX_BYTES, ring above. */
-typedef enum { PC_ALGO_AUTO = 0, PC_ALGO_RING = 1, PC_ALGO_RD = 2, PC_ALGO_DIRECT = 3 } pc_algo_t;
+/* PC_ALGO_DIRECT: two-step schedule, owners PULL their chunk from every
+ * rank's send buffer with peer loads; PC_ALGO_DIRECT_PUSH: the same schedule
+ * and bits (rank-order fold, R25), every rank PUSHES its chunk o into owner
+ * o's staging with peer stores and the owner folds from local memory (all
+ * NVLink traffic is stores; +S staging per rank).  AUTO picks DIRECT
+ * (PULL), or PUSH with PC_DIRECT_MODE=push. */
+typedef enum { PC_ALGO_AUTO = 0, PC_ALGO_RING = 1, PC_ALGO_RD = 2, PC_ALGO_DIRECT = 3, PC_ALGO_DIRECT_PUSH = 4 } pc_algo_t;
 
 enum {
   PC_SUCCESS = 0,

@@ -726,102 +726,7 @@ __device__ __forceinline__ void warp_fold_pull_bulk(const A &a, int64_t s0, int6
   for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
 }
 
-template <int DT, int OP, int FV = PC_DIRECT_FV, bool PF = false>
-__device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W, uint8_t *smem) {
-  const int P = a.P, r = a.r;
-  const uint32_t e = *(const volatile uint32_t *)a.epoch;
-  const int64_t es = sizeof(typename Op<DT, OP>::T);
-  if (gw >= a.nunits) return;
-  if (P == 1) {
-    for (int x = gw; x < a.nunits; x += W) {
-      const int u = x / a.ns, s = x % a.ns;
-      if (!warp_wait(a.ready + u, e, a.err, a.timeout_ms, u, false)) return;
-      const int64_t base = (int64_t)u * a.L, lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
-      if (hi > lo && a.sendbuf != a.recvbuf)
-        warp_copy(a.recvbuf + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
-      __syncwarp();
-      if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-    }
-    return;
-  }
-  WarpBulk wb{};
-  if (PC_DIRECT_BULK && !a.sys) warp_bulk_init(wb, smem);
-  // every peer has posted ready-to-receive (all P-1 words polled at once)
-  if (!warp_wait_all(a.rtr, P - 1, e, a.err, a.timeout_ms, a.sys)) return;
-  const uint32_t target = e * (uint32_t)(P - 1);
-  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
-    int step[kMaxActive];
-    int remaining = 0;
-#pragma unroll
-    for (int j = 0; j < kMaxActive; ++j) {
-      const bool mine = gw + (j0 + j) * W < a.nunits;
-      step[j] = mine ? 0 : 3;
-      remaining += mine;
-    }
-    Idle idle;
-    while (remaining) {
-      bool progressed = false;
-#pragma unroll
-      for (int jj = 0; jj < kMaxActive; ++jj) {
-        if (step[jj] > 2) continue;
-        const int x = gw + (j0 + jj) * W;
-        const int u = x / a.ns, s = x % a.ns;
-        const int i = step[jj];
-        const uint32_t *dep = i == 0 ? a.ready + u : a.cnt + ((int64_t)u * 2 + (i - 1)) * a.ns + s;
-        if (!warp_poll(dep, i == 0 ? e : target, i != 0 && a.sys)) continue;
-        progressed = true;
-        const int64_t base = (int64_t)u * a.L;
-        if (i == 0) {
-          fence_scope(a.sys);
-          __syncwarp();
-          if ((threadIdx.x & 31) == 0)
-            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 0) * a.ns + s, 1, a.sys);
-          step[jj] = 1;
-        } else if (i == 1) {
-          const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
-          const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
-          if (hi > lo) {
-            if (PC_DIRECT_BULK && !a.sys)
-              warp_fold_pull_bulk<DT, OP>(a, base + lo, base + lo, hi - lo, wb);
-            else
-              warp_fold_pull<DT, OP, true, FV, PF>(a, base + lo, base + lo, hi - lo);
-          }
-          fence_scope(a.sys);
-          __syncwarp();
-          if ((threadIdx.x & 31) == 0)
-            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
-          step[jj] = 2;
-        } else {
-          if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
-          step[jj] = 3;
-          --remaining;
-        }
-      }
-      if (progressed)
-        idle.progressed();
-      else if (!idle.wait(a.err, a.timeout_ms, gw))
-        return;
-    }
-  }
-}
-
-// ---------------------------------------------------------------------------
-// Batched DIRECT engine: MPI_Waitall over many partitioned allreduces of one
-// GPU in ONE launch (SURVEY §8(d) C3 (ii): one request per gradient tensor).
-// Entries (request t, local rank j) live in a device table (DirectArgs are
-// epoch-invariant; each unit reads its request's epoch word).  Global units
-// are ordered [t][x][j] — a logical unit's local ranks are adjacent — and
-// every warp takes its global units in increasing order, so the smallest
-// incomplete logical unit is active on every rank whatever the width
-// (deadlock freedom, DESIGN §6).  Same steps and bits as direct_body.
-// ---------------------------------------------------------------------------
-__device__ __forceinline__ bool warp_poll_all(const uint32_t *words, int n, uint32_t target, bool sys) {
-  const uint32_t lane = threadIdx.x & 31;
-  bool mine = lane >= (uint32_t)n || reached(sys ? ld_acquire_sys(words + lane) : ld_acquire_gpu(words + lane), target);
-  return __all_sync(0xffffffffu, mine);
-}
-
-// Rank-order PULL fold of one slice with rank-indexed source pointers S[k] and
+// Rank-order fold of one slice with rank-indexed source pointers S[k] and
 // destinations D[0] (own recvbuf), D[1..P-1] (peers), all at the same byte
 // offset: scalar head / 16-B body (FV vectors per operand in flight) / tail.
 template <int DT, int OP, int FV>
@@ -833,7 +738,12 @@ __device__ __forceinline__ void warp_fold_ptrs(const uint8_t *const (&S)[kMaxDir
   constexpr int64_t EPV = 16 / sizeof(T);
   const uintptr_t m = reinterpret_cast<uintptr_t>(D[0]) & 15;
   int64_t head = (int64_t)(((16 - m) & 15) / sizeof(T));
-  if ((reinterpret_cast<uintptr_t>(S[0]) & 15) != m) head = n;
+  bool common = true;  // every source and destination shares D[0]'s misalignment (PUSH: the
+#pragma unroll         // 16-B aligned staging slots may not): else the scalar path
+  for (int j = 0; j < kMaxDirect; ++j)
+    if (j < P)
+      common = common && (reinterpret_cast<uintptr_t>(S[j]) & 15) == m && (reinterpret_cast<uintptr_t>(D[j]) & 15) == m;
+  if (!common) head = n;
   if (head > n) head = n;
   auto scalar = [&](int64_t k) {
     T acc = __ldcg(reinterpret_cast<const T *>(S[0]) + k);
@@ -881,6 +791,125 @@ __device__ __forceinline__ void warp_fold_ptrs(const uint8_t *const (&S)[kMaxDir
       if (j < P) reinterpret_cast<uint4 *>(reinterpret_cast<T *>(D[j]) + head)[k] = acc;
   }
   for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
+}
+
+template <int DT, int OP, int FV = PC_DIRECT_FV, bool PF = false, bool PUSH = false>
+__device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W, uint8_t *smem) {
+  const int P = a.P, r = a.r;
+  const uint32_t e = *(const volatile uint32_t *)a.epoch;
+  const int64_t es = sizeof(typename Op<DT, OP>::T);
+  if (gw >= a.nunits) return;
+  if (P == 1) {
+    for (int x = gw; x < a.nunits; x += W) {
+      const int u = x / a.ns, s = x % a.ns;
+      if (!warp_wait(a.ready + u, e, a.err, a.timeout_ms, u, false)) return;
+      const int64_t base = (int64_t)u * a.L, lo = (int64_t)s * a.qs, hi = min(lo + a.qs, a.L);
+      if (hi > lo && a.sendbuf != a.recvbuf)
+        warp_copy(a.recvbuf + (base + lo) * es, a.sendbuf + (base + lo) * es, (hi - lo) * es);
+      __syncwarp();
+      if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+    }
+    return;
+  }
+  WarpBulk wb{};
+  if (PC_DIRECT_BULK && !a.sys) warp_bulk_init(wb, smem);
+  // every peer has posted ready-to-receive (all P-1 words polled at once)
+  if (!warp_wait_all(a.rtr, P - 1, e, a.err, a.timeout_ms, a.sys)) return;
+  const uint32_t target = e * (uint32_t)(P - 1);
+  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
+    int step[kMaxActive];
+    int remaining = 0;
+#pragma unroll
+    for (int j = 0; j < kMaxActive; ++j) {
+      const bool mine = gw + (j0 + j) * W < a.nunits;
+      step[j] = mine ? 0 : 3;
+      remaining += mine;
+    }
+    Idle idle;
+    while (remaining) {
+      bool progressed = false;
+#pragma unroll
+      for (int jj = 0; jj < kMaxActive; ++jj) {
+        if (step[jj] > 2) continue;
+        const int x = gw + (j0 + jj) * W;
+        const int u = x / a.ns, s = x % a.ns;
+        const int i = step[jj];
+        const uint32_t *dep = i == 0 ? a.ready + u : a.cnt + ((int64_t)u * 2 + (i - 1)) * a.ns + s;
+        if (!warp_poll(dep, i == 0 ? e : target, i != 0 && a.sys)) continue;
+        progressed = true;
+        const int64_t base = (int64_t)u * a.L;
+        if (i == 0) {
+          if (PUSH) {  // PUSH: my slice s of chunk o -> owner o's staging slot [u][r] (peer stores)
+            for (int j = 0; j < P - 1; ++j) {
+              const int o = (r + 1 + j) % P;
+              const int64_t o_lo = min((int64_t)o * a.q, a.L), o_hi = min((int64_t)(o + 1) * a.q, a.L);
+              const int64_t lo = o_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, o_hi);
+              if (hi > lo)
+                warp_copy(const_cast<uint8_t *>(a.p_sendbuf[j]) + (((int64_t)u * P + r) * a.q + (int64_t)s * a.qs) * es,
+                          a.sendbuf + (base + lo) * es, (hi - lo) * es);
+            }
+          }
+          fence_scope(a.sys);
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0)
+            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 0) * a.ns + s, 1, a.sys);
+          step[jj] = 1;
+        } else if (i == 1) {
+          const int64_t c_lo = min((int64_t)r * a.q, a.L), c_hi = min((int64_t)(r + 1) * a.q, a.L);
+          const int64_t lo = c_lo + (int64_t)s * a.qs, hi = min(lo + a.qs, c_hi);
+          if (PUSH && hi > lo) {  // PUSH: every source is local (my send buffer / my staging slots)
+            const uint8_t *S[kMaxDirect];
+            uint8_t *D[kMaxDirect];
+#pragma unroll
+            for (int k = 0; k < kMaxDirect; ++k) {
+              S[k] = nullptr;
+              D[k] = nullptr;
+              if (k < P) {
+                S[k] = k == r ? a.sendbuf + (base + lo) * es
+                              : a.staging + (((int64_t)u * P + k) * a.q + (int64_t)s * a.qs) * es;
+                D[k] = (k == 0 ? a.recvbuf : a.p_recvbuf[k - 1]) + (base + lo) * es;
+              }
+            }
+            warp_fold_ptrs<DT, OP, FV>(S, D, P, hi - lo);
+          } else if (!PUSH && hi > lo) {
+            if (PC_DIRECT_BULK && !a.sys)
+              warp_fold_pull_bulk<DT, OP>(a, base + lo, base + lo, hi - lo, wb);
+            else
+              warp_fold_pull<DT, OP, true, FV, PF>(a, base + lo, base + lo, hi - lo);
+          }
+          fence_scope(a.sys);
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0)
+            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
+          step[jj] = 2;
+        } else {
+          if ((threadIdx.x & 31) == 0) red_add_release_gpu(a.done + u, 1);
+          step[jj] = 3;
+          --remaining;
+        }
+      }
+      if (progressed)
+        idle.progressed();
+      else if (!idle.wait(a.err, a.timeout_ms, gw))
+        return;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Batched DIRECT engine: MPI_Waitall over many partitioned allreduces of one
+// GPU in ONE launch (SURVEY §8(d) C3 (ii): one request per gradient tensor).
+// Entries (request t, local rank j) live in a device table (DirectArgs are
+// epoch-invariant; each unit reads its request's epoch word).  Global units
+// are ordered [t][x][j] — a logical unit's local ranks are adjacent — and
+// every warp takes its global units in increasing order, so the smallest
+// incomplete logical unit is active on every rank whatever the width
+// (deadlock freedom, DESIGN §6).  Same steps and bits as direct_body.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ bool warp_poll_all(const uint32_t *words, int n, uint32_t target, bool sys) {
+  const uint32_t lane = threadIdx.x & 31;
+  bool mine = lane >= (uint32_t)n || reached(sys ? ld_acquire_sys(words + lane) : ld_acquire_gpu(words + lane), target);
+  return __all_sync(0xffffffffu, mine);
 }
 
 template <int DT, int OP, int FV>
@@ -1151,6 +1180,23 @@ __global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_group_thin(Dire
   const int b = blockIdx.x - g.block_start[k];
   const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
   direct_body<DT, OP, 1, true>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, nullptr);
+}
+
+// DIRECT, PUSH variant (PC_ALGO_DIRECT_PUSH): separate kernels, so the PULL
+// kernels carry none of its registers.
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine_push(DirectArgs a) {
+  direct_body<DT, OP, PC_DIRECT_FV, false, true>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5,
+                                                 (gridDim.x * blockDim.x) >> 5, nullptr);
+}
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine_group_push(DirectGroupArgs g) {
+  int k = 0;
+  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
+  const int b = blockIdx.x - g.block_start[k];
+  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
+  direct_body<DT, OP, PC_DIRECT_FV, false, true>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5,
+                                                 (nb * blockDim.x) >> 5, nullptr);
 }
 
 // Single-rank launches (one rank per GPU / process).

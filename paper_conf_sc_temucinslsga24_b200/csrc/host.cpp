@@ -537,7 +537,7 @@ static int make_rec(Request *q, ReqRec *r) {
   r->count = (int64_t)q->count;
   r->dtype = q->dtype;
   r->op = q->op;
-  r->algo = q->algo;
+  r->algo = q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo;  // every rank must pick the same variant
   r->seq = q->seq;
   r->coll = q->coll;
   r->root = q->root;
@@ -552,7 +552,8 @@ static int make_rec(Request *q, ReqRec *r) {
   if ((rc = export_ptr(c, q->ctrl, q->L.words * 4, &r->ctrl))) return rc;
   if (q->staging && (rc = export_ptr(c, q->staging, q->staging_bytes, &r->stage))) return rc;
   // DIRECT (PULL): the peers' reduce steps read this rank's send buffer
-  if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && c->size > 1 &&
+  // (PUSH exports its staging above: the peers write into it)
+  if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && !q->direct_push && c->size > 1 &&
       (q->coll == PC_COLL_ALLREDUCE || q->coll == PC_COLL_REDUCE_SCATTER) &&
       (rc = export_ptr(c, q->sbuf, q->send_bytes, &r->stage)))
     return rc;
@@ -640,7 +641,8 @@ static int exchange_round(Comm *c, Request *target) {
       for (int r = 0; r < c->size && !qrc; ++r) {
         const ReqRec *m = find_rec(all, M, r, PC_KIND_PALLREDUCE, -1, 0, q->seq, cnt);
         if (!m || m->partitions != q->partitions || m->count != (int64_t)q->count || m->dtype != q->dtype ||
-            m->op != q->op || m->algo != q->algo || m->coll != q->coll || m->root != q->root) {
+            m->op != q->op || m->algo != (q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo) || m->coll != q->coll ||
+            m->root != q->root) {
           fprintf(stderr, "[pc] rank %d: allreduce #%d disagrees with rank %d\n", c->rank, q->seq, r);
           qrc = PC_ERR_MATCH;
         }
@@ -820,6 +822,8 @@ static DirectArgs make_direct_args(Request *q) {
   a.err = (int32_t *)(q->ctrl + q->L.err);
   a.timeout_ms = c->timeout_ms;
   a.sys = q->sys_scope;
+  a.push = q->direct_push ? 1 : 0;
+  a.staging = q->staging;
   return a;
 }
 
@@ -1211,7 +1215,8 @@ static int engine_batch(const std::vector<Request *> &rq, cudaStream_t s) {
   std::vector<Request *> leaders;
   for (Request *q : rq) {
     if (q->kind != PC_KIND_PALLREDUCE || q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT ||
-        q->inline_ar || !q->active || q->engine_registered || q->engine_launched || q->batch_launched)
+        q->direct_push || q->inline_ar || !q->active || q->engine_registered || q->engine_launched ||
+        q->batch_launched)
       return 1;
     if (q->dtype != q0->dtype || q->op != q0->op || q->comm->device != q0->comm->device) return 1;
     const int r = q->leader ? (int)q->leader->gs.members.size() : 1;
@@ -1510,7 +1515,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   Comm *c = (Comm *)comm;
   if (!c || !req || partitions < 1 ||
       (dtype != PC_INT32 && dtype != PC_FLOAT32 && dtype != PC_FLOAT64 && dtype != PC_BF16) || op < 0 || op > 2 ||
-      algo < 0 || algo > 3)
+      algo < 0 || algo > PC_ALGO_DIRECT_PUSH)
     return PC_ERR_ARG;
   const int P = c->size;
   const size_t esz = dtype_size(dtype);
@@ -1535,8 +1540,17 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
     else
       a = PC_ALGO_RING;
   }
+  bool push = false;
+  if (a == PC_ALGO_DIRECT_PUSH) {
+    a = PC_ALGO_DIRECT;
+    push = true;
+  } else if (algo == PC_ALGO_AUTO && a == PC_ALGO_DIRECT) {
+    const char *m = getenv("PC_DIRECT_MODE");
+    push = m && strcmp(m, "push") == 0;
+  }
   if (a == PC_ALGO_RD && !pow2) return PC_ERR_UNSUPPORTED;
   if (a == PC_ALGO_DIRECT && P > kMaxDirect) return PC_ERR_UNSUPPORTED;
+  if (a < PC_ALGO_RING || a > PC_ALGO_DIRECT) return PC_ERR_ARG;
   Request *q;
   int rc = new_request(c, PC_KIND_PALLREDUCE, req, &q);
   if (rc) return rc;
@@ -1548,6 +1562,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   q->op = op;
   q->algo_req = algo;
   q->algo = a;
+  q->direct_push = push && P > 1;
   q->esize = esz;
   q->peer = -1;
   q->tag = 0;
@@ -1573,7 +1588,9 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
     q->chunk_elems = chunk_q(L, P, epv);
     q->engine_warps = c->direct_warps;
     choose_slices(q->chunk_elems, partitions, c->direct_warps * upw, min_elems, &q->slices, &q->slice_elems, epv);
-    q->staging_bytes = 0;  // PULL: owners read the peers' send buffers directly
+    // PULL: owners read the peers' send buffers directly; PUSH: staging
+    // [u][source rank][q] receives every rank's copy of this rank's chunk
+    q->staging_bytes = q->direct_push ? (size_t)partitions * P * (size_t)q->chunk_elems * esz : 0;
   } else {
     q->nsteps = log2_exact(P);
     q->chunk_elems = L;
@@ -1938,7 +1955,8 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
     }
   } else if (q->kind == PC_KIND_PALLREDUCE) {
     if (copy == PC_COPY_INLINE) {  // R33: INLINE allreduce (DIRECT schedule bits, P <= 8)
-      if (q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT || c->size > PC_AR_MAX) return PC_ERR_UNSUPPORTED;
+      if (q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT || q->direct_push || c->size > PC_AR_MAX)
+        return PC_ERR_UNSUPPORTED;
       if (!c->dry && !q->ar_tab) {
         pc_ar_tab_s t{};
         const int P = c->size, r = c->rank;
@@ -2401,7 +2419,7 @@ int pc_chunk_bounds(int64_t L, int P, int64_t *out) {
 int pc_request_info(pc_request_t req, int *algo, int *slices, int64_t *slice_elems, int *engine_warps) {
   Request *q = (Request *)req;
   if (!q) return PC_ERR_ARG;
-  if (algo) *algo = q->algo;
+  if (algo) *algo = q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo;
   if (slices) *slices = q->slices;
   if (slice_elems) *slice_elems = q->slice_elems;
   if (engine_warps) *engine_warps = q->engine_warps;
@@ -2425,7 +2443,7 @@ int pc_request_peer_buffer(pc_request_t req, int j, void **ptr) {
   if (q->kind == PC_KIND_PSEND) {
     if (j != 0) return PC_ERR_ARG;
     *ptr = q->peer_buf;
-  } else if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT) {
+  } else if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && !q->direct_push) {
     if (j < 0 || j >= q->comm->size - 1) return PC_ERR_ARG;
     *ptr = q->nb_buf[j];
   } else {

@@ -169,6 +169,7 @@ struct Request {
   bool overlap = true;          // pc_request_set_overlap (0: fork at the wait, the round-1 order)
   // INLINE allreduce (reading R33): a DIRECT allreduce whose prequest was
   // created with PC_COPY_INLINE — the completing Pready folds, no engine
+  bool direct_push = false;     // DIRECT schedule, PUSH variant (PC_ALGO_DIRECT_PUSH)
   bool inline_ar = false;
   void *ar_tab = nullptr;       // device pc_ar_tab_s (library-owned)
   cudaEvent_t fork_ev_ext = nullptr;  // fork point recorded by a batched control call (else ev_fork)
@@ -356,12 +357,14 @@ struct DirectArgs {
   const uint32_t *cnt, *ready, *rtr;  // cnt: [u][phase][slice] arrival counters (written by peers)
   uint32_t *done;
   // peer j = rank (r+1+j) mod P: its send buffer (read by the PULL reduce) and recvbuf
-  const uint8_t *p_sendbuf[kMaxDirect - 1];
+  const uint8_t *p_sendbuf[kMaxDirect - 1];  // PUSH variant: peer j's STAGING (written by this rank)
   uint8_t *p_recvbuf[kMaxDirect - 1];
   uint32_t *p_cnt[kMaxDirect - 1];
   int32_t *err;
   uint32_t timeout_ms;
   int sys;
+  int push;            // PUSH variant: step 0 stores chunk o into owner o's staging slot r
+  uint8_t *staging;    // PUSH: own staging [u][source rank][q elements]
 };
 struct DirectGroupArgs {
   int n;
