@@ -12,32 +12,67 @@ using namespace pc_detail;
 // ---------------------------------------------------------------------------
 // ENGINE copy mode of partitioned send: unit = (transport partition t, slice s).
 // ---------------------------------------------------------------------------
+// Each warp sweeps up to kMaxActive of its units at a time (Alg 2 style):
+// every unit found ready in a sweep is copied, then ONE fence publishes the
+// whole set — with block-sized transport partitions (8 KiB) a fence per unit
+// was most of the engine's time.  A transport partition of one slice needs
+// no slice counter: its warp alone completes it.
 __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int W = (gridDim.x * blockDim.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
   bool rtr_ok = false;
-  for (int x = gw; x < a.nunits; x += W) {
-    const int t = x / a.ns, s = x % a.ns;
-    if (!warp_wait(a.ready + t, e, a.err, a.timeout_ms, t, false)) return;
-    if (!rtr_ok) {
-      if (!warp_wait(a.rtr, e, a.err, a.timeout_ms, -1, a.sys)) return;
-      rtr_ok = true;
-    }
-    const int rem = a.partitions - t * a.agg;
-    const uint64_t len = (uint64_t)(rem < a.agg ? rem : a.agg) * a.part_bytes;
-    const uint64_t off = (uint64_t)t * a.agg * a.part_bytes;
-    const uint64_t slo = (uint64_t)s * a.slice_bytes;
-    const uint64_t n = slo < len ? min(a.slice_bytes, len - slo) : 0;
-    if (n) warp_copy(a.peer_rbuf + off + slo, a.sbuf + off + slo, (int64_t)n);
-    fence_scope(a.sys);
-    __syncwarp();
-    if ((threadIdx.x & 31) == 0) {
-      const uint32_t old = atom_add_acq_rel_gpu(a.donecnt + t, 1);
-      if (old + 1 == e * (uint32_t)a.ns) {
-        signal_transport(a.peer_flags, t, e, a.xpart, a.partitions, a.agg, a.part_bytes, a.peer_part_bytes);
-        st_release_gpu(a.sent + t, e);
+  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
+    uint32_t pending = 0;
+#pragma unroll
+    for (int j = 0; j < kMaxActive; ++j)
+      if (gw + (j0 + j) * W < a.nunits) pending |= 1u << j;
+    Idle idle;
+    while (pending) {
+      // poll: lane j looks at unit j's ready flag (all polls in flight together)
+      bool rdy = false;
+      if (lane < (uint32_t)kMaxActive && ((pending >> lane) & 1u)) {
+        const int t = (gw + (j0 + (int)lane) * W) / a.ns;
+        rdy = reached(ld_acquire_gpu(a.ready + t), e);
       }
+      const uint32_t ready = __ballot_sync(0xffffffffu, rdy) & pending;
+      if (!ready) {
+        if (!idle.wait(a.err, a.timeout_ms, gw)) return;
+        continue;
+      }
+      idle.progressed();
+      if (!rtr_ok) {
+        if (!warp_wait(a.rtr, e, a.err, a.timeout_ms, -1, a.sys)) return;
+        rtr_ok = true;
+      }
+      for (int j = 0; j < kMaxActive; ++j) {
+        if (!((ready >> j) & 1u)) continue;
+        const int x = gw + (j0 + j) * W;
+        const int t = x / a.ns, s = x % a.ns;
+        const int rem = a.partitions - t * a.agg;
+        const uint64_t len = (uint64_t)(rem < a.agg ? rem : a.agg) * a.part_bytes;
+        const uint64_t off = (uint64_t)t * a.agg * a.part_bytes;
+        const uint64_t slo = (uint64_t)s * a.slice_bytes;
+        const uint64_t n = slo < len ? min(a.slice_bytes, len - slo) : 0;
+        if (n) warp_copy(a.peer_rbuf + off + slo, a.sbuf + off + slo, (int64_t)n);
+      }
+      fence_scope(a.sys);  // one cumulative fence for every copy of this sweep
+      __syncwarp();
+      if (lane == 0) {
+        for (int j = 0; j < kMaxActive; ++j) {
+          if (!((ready >> j) & 1u)) continue;
+          const int t = (gw + (j0 + j) * W) / a.ns;
+          const bool last = a.ns == 1 || atom_add_acq_rel_gpu(a.donecnt + t, 1) + 1 == e * (uint32_t)a.ns;
+          if (last && a.ns > 1) fence_scope(a.sys);  // the other slices' copies (acquired by the add) too
+          if (last) {
+            signal_transport(a.peer_flags, t, e, a.xpart, a.partitions, a.agg, a.part_bytes, a.peer_part_bytes);
+            st_relaxed_gpu(a.sent + t, e);  // (after the fence: the copies are delivered)
+          }
+        }
+      }
+      __syncwarp();
+      pending &= ~ready;
     }
   }
 }
