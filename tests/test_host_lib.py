@@ -314,3 +314,88 @@ def test_dry_waitall_state_rules():
     for c in cs:
         c.destroy()
     g.destroy()
+
+
+def test_dry_direct_push_variant(monkeypatch):
+    """PC_ALGO_DIRECT_PUSH is the DIRECT schedule's PUSH variant: reported as
+    such, matched only against itself (every rank must pick the same variant),
+    and AUTO picks it with PC_DIRECT_MODE=push."""
+    g, cs = _dry(4)
+    push = [pc.pallreduce_init(0, 0, 2, 4096, pc.FLOAT32, pc.SUM, pc.ALGO_DIRECT_PUSH, c) for c in cs]
+    for q in push:
+        q.start()
+    pc.run_ranks([(lambda q=q: q.pbuf_prepare()) for q in push])
+    assert all(q.info()["algo_name"] == "direct_push" for q in push)
+    mixed = [pc.pallreduce_init(0, 0, 1, 64, pc.FLOAT32, pc.SUM, pc.ALGO_DIRECT if r else pc.ALGO_DIRECT_PUSH, cs[r])
+             for r in range(4)]
+    for q in mixed:
+        q.start()
+    res = pc.run_ranks([(lambda q=q: _try(q.pbuf_prepare)) for q in mixed])
+    assert all(x == pc.ERR_MATCH for x in res)
+    monkeypatch.setenv("PC_DIRECT_MODE", "push")
+    auto = [pc.pallreduce_init(0, 0, 1, 1 << 22, pc.FLOAT32, pc.SUM, pc.ALGO_AUTO, c) for c in cs]
+    for q in auto:
+        q.start()
+    pc.run_ranks([(lambda q=q: q.pbuf_prepare()) for q in auto])
+    assert all(q.info()["algo_name"] == "direct_push" for q in auto)
+    for q in push + auto:
+        q.wait()
+    for q in push + auto + mixed:
+        q.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
+
+
+def test_dry_epoch_all_beyond_one_kernel():
+    """pc_epoch_all takes any number of requests (more than one kernel's
+    parameters hold: the device path uses a table-driven kernel); the same
+    request twice in one call is refused before any request is touched."""
+    g, cs = _dry(2)
+    ar = [[pc.pallreduce_init(0, 0, 1, 64, pc.FLOAT32, pc.SUM, pc.ALGO_DIRECT, c) for _ in range(20)] for c in cs]
+    flat = ar[0] + ar[1]
+    for q in flat:
+        q.start()
+    pc.run_ranks([(lambda r=r: [q.pbuf_prepare() for q in ar[r]]) for r in range(2)])
+    pc.waitall_on_stream(flat)
+    for _ in range(3):
+        pc.epoch_all(flat, pready=True)
+        pc.waitall_on_stream(flat)
+    assert _try(lambda: pc.epoch_all(flat + flat[:1], pready=True)) == pc.ERR_ARG
+    pc.epoch_all(flat, pready=True)  # nothing was started by the refused call
+    pc.waitall_on_stream(flat)
+    for q in flat:
+        q.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
+
+
+def test_dry_overlap_and_inline_rules():
+    """pc_request_set_overlap only on inactive requests; an INLINE prequest
+    (reading R33) only on DIRECT (PULL) allreduces; pc_epoch_all cannot Pready
+    an INLINE allreduce (its Pready folds)."""
+    g, cs = _dry(2)
+    d = [pc.pallreduce_init(0, 0, 2, 64, pc.FLOAT32, pc.SUM, pc.ALGO_DIRECT, c) for c in cs]
+    ring = [pc.pallreduce_init(0, 0, 2, 64, pc.FLOAT32, pc.SUM, pc.ALGO_RING, c) for c in cs]
+    for q in d + ring:
+        q.set_overlap(False)
+        q.set_overlap(True)
+        q.start()
+    assert _try(lambda: d[0].set_overlap(False)) == pc.ERR_STATE
+    pc.run_ranks([(lambda r=r: (d[r].pbuf_prepare(), ring[r].pbuf_prepare())) for r in range(2)])
+    for q in ring:
+        assert _try(lambda q=q: q.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)) == pc.ERR_UNSUPPORTED
+    for q in d:
+        q.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+    for q in d + ring:
+        q.wait()
+    assert _try(lambda: pc.epoch_all(d, pready=True)) == pc.ERR_ARG
+    pc.epoch_all(d, pready=False)
+    for q in d:
+        q.wait()
+    for q in d + ring:
+        q.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
