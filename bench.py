@@ -55,6 +55,7 @@ def parse():
     ap.add_argument("--no-jacobi", action="store_true")
     ap.add_argument("--no-c1", action="store_true",
                     help="skip the C1 leg (its host Progression Engine epochs cannot progress under ncu's serialisation)")
+    ap.add_argument("--no-dl", action="store_true", help="N > 1: skip the DL-proxy goodput leg")
     ap.add_argument("--jacobi-n", type=int, default=16384)
     ap.add_argument("--jacobi-iters", type=int, default=50)
     ap.add_argument("--quiet", action="store_true", help="only the JSON line")
@@ -805,6 +806,24 @@ def multi_p2p(ctx, pc, apps, torch, dist):
             trad()
         torch.cuda.synchronize()
         row["traditional_us_host"] = pmax((time.perf_counter() - t0) / it * 1e6)
+        if not ctx.shared:  # the same with NCCL point-to-point (kernel -> sync -> ncclSend / ncclRecv)
+            def trad_nccl():
+                if side == 0:
+                    apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st)
+                    st.synchronize()
+                    with torch.cuda.stream(st):
+                        dist.send(Cb, dst=r + 1, group=grp)
+                else:
+                    with torch.cuda.stream(st):
+                        dist.recv(Rb, src=r - 1, group=grp)
+                st.synchronize()
+            for _ in range(2):
+                trad_nccl()
+            dist.barrier(group=grp)
+            t0 = time.perf_counter()
+            for _ in range(it):
+                trad_nccl()
+            row["traditional_nccl_us_host"] = pmax((time.perf_counter() - t0) / it * 1e6)
         q0.free()
         configs = [("block", apps.GRAN_BLOCK, 1, pc.COPY_INLINE), ("block", apps.GRAN_BLOCK, 1, pc.COPY_ENGINE),
                    ("block->1MiB", apps.GRAN_BLOCK, 128, pc.COPY_INLINE),
@@ -901,6 +920,66 @@ def multi_p2p(ctx, pc, apps, torch, dist):
     q.free()
     q2.free()
     res["latency_ns"] = lat
+    comm.destroy()
+    return res
+
+
+def multi_dl(ctx, pc, apps, torch, dist, args):
+    """NEXT-2 / Figs 10-11 analogue across GPUs (§VI-D2): every
+    rank computes the BCE gradient of a ResNet-50-sized flat buffer (25.56 M
+    fp32, 64 KiB partitions) and the ranks allreduce it, three ways:
+      traditional: producer kernel -> NCCL all_reduce (Listing 1);
+      serial:      producer kernel -> pc_epoch_all(pready) -> engine;
+      partitioned: pc_epoch_all -> producer that Preadies each partition ->
+                   engine forked at the epoch's control call (overlap, a6).
+    ms per step (max over ranks) and the gradient goodput."""
+    NPARAM, L = 25_557_032, 16384
+    Np = -(-NPARAM // L)
+    if ctx.shared:
+        Np, L = 64, 16384
+    n = Np * L
+    gen = torch.Generator(device="cuda")
+    gen.manual_seed(0x5C24 + ctx.rank)
+    p = 0.02 + 0.96 * torch.rand(n, device="cuda", generator=gen)
+    y = torch.randint(0, 2, (n,), device="cuda", generator=gen).float()
+    g = torch.empty(n, device="cuda")
+    out = torch.empty(n, device="cuda")
+    comm = pc.Comm.from_process_group(ctx.dev)
+    st = torch.cuda.Stream()
+    q = pc.pallreduce_init(g, out, Np, L, pc.FLOAT32, pc.SUM, pc.ALGO_AUTO, comm)
+    q.start(st)
+    q.pbuf_prepare(st)
+    pq = q.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_ENGINE)
+    apps.bce_grad(p, y, g, Np, L, float(n), None, stream=st)
+    q.pready_range(0, Np - 1, st)
+    q.wait_on_stream(st)
+    torch.cuda.synchronize()
+    it = 3 if ctx.shared else 20
+
+    def serial():
+        apps.bce_grad(p, y, g, Np, L, float(n), None, stream=st)
+        pc.epoch_all([q], pready=True, stream=st)
+        q.wait_on_stream(st)
+
+    def partitioned():
+        pc.epoch_all([q], pready=False, stream=st)
+        apps.bce_grad(p, y, g, Np, L, float(n), pq, stream=st)
+        q.wait_on_stream(st)
+
+    res = {"partitions": Np, "partition_bytes": 4 * L, "bytes_per_rank": 4 * n, "algo": q.info()["algo_name"]}
+    res["serial_ms"] = ctx.time_ms(serial, it, st)
+    res["partitioned_ms"] = ctx.time_ms(partitioned, it, st)
+    assert q.error()[0] == 0
+    if not ctx.shared:
+        def traditional():
+            apps.bce_grad(p, y, g, Np, L, float(n), None, stream=st)
+            with torch.cuda.stream(st):
+                dist.all_reduce(g)
+        res["traditional_nccl_ms"] = ctx.time_ms(traditional, it, st)
+    for k in ("serial", "partitioned", "traditional_nccl"):
+        if f"{k}_ms" in res:
+            res[f"{k}_goodput_gbs"] = 4 * n * ctx.world / (res[f"{k}_ms"] / 1e3) / 1e9
+    q.free()
     comm.destroy()
     return res
 
@@ -1086,6 +1165,8 @@ def run_multi(args):
     log("p2p legs done")
     jac = None if args.no_jacobi else multi_jacobi(ctx, pc, apps, torch, args)
     log("jacobi done")
+    dl = None if args.no_dl else multi_dl(ctx, pc, apps, torch, dist, args)
+    log("dl proxy done")
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:
         cpu = oracle_sample(P=min(P, 8))
@@ -1123,7 +1204,7 @@ def run_multi(args):
                        "d2h_bytes_per_step": S, "ms_per_step": ems,
                        "api": "pc_epoch_all(pready) + pc_wait_on_stream, host buffers copied in/out each step"},
                "gpu_launches": launches, "clocks": clk.summary(), "nccl": nccl, "direct_other_variant": other,
-               "p2p": p2p, "jacobi": jac}
+               "p2p": p2p, "jacobi": jac, "dl_proxy": dl}
         print(json.dumps(out), flush=True)
     dist.destroy_process_group()
 

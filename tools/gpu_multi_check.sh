@@ -8,4 +8,4 @@ timeout 400 python -m pytest tests/test_gpu_multiproc.py -x -q > gpurun_out/mult
 timeout 900 python bench.py --gpus 2 --steps 5 --warmup 3 > gpurun_out/multi_bench_self.log 2> gpurun_out/multi_bench_self.err; echo "bench exit $?" >> gpurun_out/multi_bench_self.err
 timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29655 \
   bench.py --gpus 2 --steps 5 --warmup 3 > gpurun_out/multi_bench.log 2> gpurun_out/multi_bench.err; echo "bench exit $?" >> gpurun_out/multi_bench.err
-tail -3 gpurun_out/multi_pytest.log; tail -c 3000 gpurun_out/multi_bench_self.log; tail -5 gpurun_out/multi_bench_self.err; tail -c 600 gpurun_out/multi_bench.log; tail -3 gpurun_out/multi_bench.err
+tail -3 gpurun_out/multi_pytest.log; tail -c 1500 gpurun_out/multi_bench_self.log; tail -2 gpurun_out/multi_bench_self.err; tail -c 600 gpurun_out/multi_bench.log; tail -2 gpurun_out/multi_bench.err
