@@ -465,6 +465,51 @@ def jacobi_bench(pc, apps, torch, args):
     return res
 
 
+def e2e_pipelined(pc, torch, reqs, send, host_in, recv0, host_out, Np, count, st, steps, chunks=8):
+    """End to end through the public API with host buffers: every step copies
+    its inputs host -> device and its result device -> host.  The epoch is
+    pipelined the partitioned way: pc_epoch_all (Start + ready-to-receive, no
+    Pready) forks the engine, then the inputs arrive over PCIe in chunks of
+    partitions, each chunk Preadied (pc_pready_range) right after its copy, so
+    the engine reduces while the rest is still in flight; the result's D2H of
+    step i overlaps the H2D of step i+1 (separate copy streams, PCIe is full
+    duplex).  Returns ms per step (CUDA events, all streams joined)."""
+    st_in, st_out = torch.cuda.Stream(), torch.cuda.Stream()
+    CH = max(1, -(-Np // chunks))
+    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev_ctl, ev_done, ev_out = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
+    f0.record(st)
+    st_in.wait_event(f0)
+    st_out.wait_event(f0)
+    for i in range(steps):
+        if i:
+            st_in.wait_event(ev_done)  # step i-1's engine finished reading the send buffers
+            st.wait_event(ev_out)      # step i-1's result was read out: recvbuf is free (RTR)
+        pc.epoch_all(reqs, pready=False, stream=st)
+        ev_ctl.record(st)
+        for c0 in range(0, Np, CH):
+            c1 = min(c0 + CH, Np)
+            with torch.cuda.stream(st_in):
+                for r in range(len(reqs)):
+                    send[r][c0 * count:c1 * count].copy_(host_in[r][c0 * count:c1 * count], non_blocking=True)
+            if c0 == 0:
+                st_in.wait_event(ev_ctl)  # the Pready kernels read this epoch's word
+            for q in reqs:
+                q.pready_range(c0, c1 - 1, st_in)
+        for q in reqs:
+            q.wait_on_stream(st)
+        ev_done.record(st)
+        st_out.wait_event(ev_done)
+        with torch.cuda.stream(st_out):
+            host_out.copy_(recv0, non_blocking=True)
+        ev_out.record(st_out)
+    st.wait_event(ev_out)
+    st.wait_stream(st_in)
+    f1.record(st)
+    torch.cuda.synchronize()
+    return f0.elapsed_time(f1) / steps
+
+
 def run_virtual(args):
     import numpy as np
     import torch
@@ -557,23 +602,20 @@ def run_virtual(args):
         host_in[r].copy_(send[r].cpu())
     host_out = torch.empty(Np * count, dtype=torch.float32, pin_memory=True)
     torch.cuda.synchronize()
-    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ke = max(1, args.e2e_steps)
-    f0.record(st)
-    for _ in range(ke):
-        with torch.cuda.stream(st):
-            for r in range(P):
-                send[r].copy_(host_in[r], non_blocking=True)
-        step()
-        with torch.cuda.stream(st):
-            host_out.copy_(recv[0], non_blocking=True)
-    f1.record(st)
-    torch.cuda.synchronize()
-    e2e_ms = f0.elapsed_time(f1) / ke
+    ref0 = recv[0][: 1 << 16].clone()  # the timed steps' result: the e2e steps reduce the same inputs
+    e2e_pipelined(pc, torch, reqs, send, host_in, recv[0], host_out, Np, count, st, 1)  # warm-up
+    e2e_ms = e2e_pipelined(pc, torch, reqs, send, host_in, recv[0], host_out, Np, count, st, ke)
+    for q in reqs:
+        assert q.error()[0] == 0, f"device error {q.error()}"
+    assert torch.equal(recv[1][:4096], recv[0][:4096]) and torch.equal(recv[0][: 1 << 16], ref0)
+    assert torch.equal(host_out[: 1 << 16], ref0.cpu())
     log(f"e2e: {e2e_ms:.3f} ms/step")
     e2e = {"value": busbw(S, e2e_ms / 1e3, P), "unit": "GB/s", "h2d_bytes_per_step": P * S, "d2h_bytes_per_step": S,
-           "ms_per_step": e2e_ms, "api": "pc_epoch_all(pready) + pc_wait_on_stream per rank (host buffers copied in "
-                                         "and the result copied out each step)"}
+           "ms_per_step": e2e_ms,
+           "api": "per step: pc_epoch_all (no Pready) per GPU, then each rank's inputs host->device in 8 chunks of "
+                  "partitions, each followed by pc_pready_range (the engine reduces while PCIe delivers the rest), "
+                  "pc_wait_on_stream, the result device->host (overlapping the next step's inputs)"}
 
     for q in reqs:
         q.free()
@@ -1139,23 +1181,14 @@ def run_multi(args):
         nccl["debug_log"] = "NCCL_DEBUG=INFO, NCCL_DEBUG_SUBSYS=INIT,TUNING,ENV on stderr"
     log("allreduce + nccl done")
 
-    # e2e: H2D input, allreduce, D2H result
+    # e2e: H2D input in chunks each Preadied, allreduce, D2H result (pipelined, e2e_pipelined)
     host_in = send.cpu().pin_memory()
     host_out = torch.empty_like(host_in).pin_memory()
     torch.cuda.synchronize()
-    dist.barrier()
-    f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ke = max(1, args.e2e_steps)
-    f0.record(st)
-    for _ in range(ke):
-        with torch.cuda.stream(st):
-            send.copy_(host_in, non_blocking=True)
-        step()
-        with torch.cuda.stream(st):
-            host_out.copy_(recv, non_blocking=True)
-    f1.record(st)
-    torch.cuda.synchronize()
-    ems = ctx.max(f0.elapsed_time(f1) / ke)
+    e2e_pipelined(pc, torch, [q], [send], [host_in], recv, host_out, Np, count, st, 1)
+    dist.barrier()
+    ems = ctx.max(e2e_pipelined(pc, torch, [q], [send], [host_in], recv, host_out, Np, count, st, ke))
     q.free()
     comm.destroy()
 
@@ -1202,7 +1235,8 @@ def run_multi(args):
                "nvlink_floor": floor, "cpu_baseline": cpu,
                "e2e": {"value": busbw(S, ems / 1e3, P), "unit": "GB/s", "h2d_bytes_per_step": S,
                        "d2h_bytes_per_step": S, "ms_per_step": ems,
-                       "api": "pc_epoch_all(pready) + pc_wait_on_stream, host buffers copied in/out each step"},
+                       "api": "pc_epoch_all + chunked H2D each followed by pc_pready_range + pc_wait_on_stream + "
+                              "D2H (pipelined, e2e_pipelined)"},
                "gpu_launches": launches, "clocks": clk.summary(), "nccl": nccl, "direct_other_variant": other,
                "p2p": p2p, "jacobi": jac, "dl_proxy": dl}
         print(json.dumps(out), flush=True)
