@@ -21,7 +21,8 @@ torch.cuda.set_device(0)
 comm = pc.Comm.from_process_group(0)
 st = torch.cuda.Stream()
 res = {}
-for name, algo in (("ring", pc.ALGO_RING), ("rd", pc.ALGO_RD), ("direct", pc.ALGO_DIRECT)):
+for name, algo in (("ring", pc.ALGO_RING), ("rd", pc.ALGO_RD), ("direct", pc.ALGO_DIRECT),
+                   ("direct_push", pc.ALGO_DIRECT_PUSH)):
     Np, L = 3, 1000
     x = synth.normal_f32(synth.BASE_SEED, r, 0, Np * L)
     send = torch.from_numpy(x).cuda()
@@ -46,6 +47,46 @@ for name, algo in (("ring", pc.ALGO_RING), ("rd", pc.ALGO_RD), ("direct", pc.ALG
         assert q.error() == (0, 0), q.error()
         res[name + "_epoch_all%d" % e] = recv.cpu().numpy()
     q.free()
+# INLINE allreduce across the processes (reading R33): the producer's block
+# Pready that completes a partition on the last rank folds it for both ranks
+# (system-scope arrival counter in rank 0's control block, peer stores).
+Np, L = 5, 777
+x = synth.normal_f32(synth.BASE_SEED + 3, r, 0, Np * L)
+srcb = torch.from_numpy(x).cuda()
+send = torch.zeros_like(srcb)
+recv = torch.zeros_like(srcb)
+q = pc.pallreduce_init(send, recv, Np, L, pc.FLOAT32, pc.SUM, pc.ALGO_DIRECT, comm)
+for e in range(3):
+    recv.zero_()
+    st.wait_stream(torch.cuda.current_stream())
+    q.start(st)
+    q.pbuf_prepare(st)
+    if e == 0:
+        pq = q.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+    apps.produce(send, srcb, Np, L * 4, apps.GRAN_BLOCK, pq, order_stride=3, stream=st)
+    q.wait_on_stream(st)
+    st.synchronize()
+    assert q.error() == (0, 0), q.error()
+    res["inline%d" % e] = recv.cpu().numpy()
+q.free()
+# engine/producer overlap across the processes: each rank's producer waits on
+# the device pc_parrived(0) of the collective before it Preadies the rest
+Np, L = 4, 4099
+x = synth.normal_f32(synth.BASE_SEED + 4, r, 0, Np * L)
+send = torch.from_numpy(x).cuda()
+recv = torch.zeros_like(send)
+q = pc.pallreduce_init(send, recv, Np, L, pc.FLOAT32, pc.SUM, pc.ALGO_DIRECT, comm)
+q.start(st)
+q.pbuf_prepare(st)
+pq = q.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_ENGINE)
+stamps = torch.zeros((1, 4), dtype=torch.int64, device="cuda")
+apps.overlap_probe([pq], Np, 20000, stamps, st)
+q.wait_on_stream(st)
+st.synchronize()
+assert q.error() == (0, 0), q.error()
+res["overlap"] = recv.cpu().numpy()
+res["overlap_stamps"] = stamps.cpu().numpy()
+q.free()
 # p2p 0 -> 1 with block-granularity Pready from the producer kernel
 n = 2048 * 8
 if r == 0:

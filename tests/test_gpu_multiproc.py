@@ -20,18 +20,34 @@ def test_two_processes_ipc(tmp_path):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=29611", os.path.join(ROOT, "tests", "mp_worker.py"),
            str(tmp_path)]
-    p = subprocess.run(cmd, capture_output=True, text=True, timeout=240)
+    p = subprocess.run(cmd, capture_output=True, text=True, timeout=400)
     assert p.returncode == 0, p.stdout[-3000:] + p.stderr[-3000:]
     res = [np.load(os.path.join(tmp_path, f"rank{r}.npz")) for r in range(2)]
     Np, L = 3, 1000
     x = np.stack([synth.normal_f32(synth.BASE_SEED, r, 0, Np * L) for r in range(2)])
-    for name, algo in (("ring", oracle.RING), ("rd", oracle.RD), ("direct", oracle.DIRECT)):
+    for name, algo in (("ring", oracle.RING), ("rd", oracle.RD), ("direct", oracle.DIRECT),
+                       ("direct_push", oracle.DIRECT)):
         ref, _, _ = oracle.pallreduce(x, Np, algo)
         for r in range(2):
             np.testing.assert_array_equal(res[r][name].view(np.uint32), ref[r].view(np.uint32))
             for e in range(3):  # pc_epoch_all epochs across processes
                 np.testing.assert_array_equal(res[r][f"{name}_epoch_all{e}"].view(np.uint32),
                                               ref[r].view(np.uint32))
+    # INLINE allreduce across processes (R33): the DIRECT bits (O6), 3 epochs
+    Np, L = 5, 777
+    x = np.stack([synth.normal_f32(synth.BASE_SEED + 3, r, 0, Np * L) for r in range(2)])
+    ref, _, _ = oracle.pallreduce(x, Np, oracle.DIRECT)
+    for r in range(2):
+        for e in range(3):
+            np.testing.assert_array_equal(res[r]["inline%d" % e].view(np.uint32), ref[r].view(np.uint32))
+    # overlap across processes: partition 0 completed inside each producer
+    Np, L = 4, 4099
+    x = np.stack([synth.normal_f32(synth.BASE_SEED + 4, r, 0, Np * L) for r in range(2)])
+    ref, _, _ = oracle.pallreduce(x, Np, oracle.DIRECT)
+    for r in range(2):
+        np.testing.assert_array_equal(res[r]["overlap"].view(np.uint32), ref[r].view(np.uint32))
+        s = res[r]["overlap_stamps"][0]
+        assert 0 < s[2] < s[3], s
     n = 2048 * 8
     a = synth.uniform_f32(synth.BASE_SEED, 0, 0, n)
     b = synth.uniform_f32(synth.BASE_SEED, 0, 1, n)
