@@ -614,7 +614,19 @@ __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d
 constexpr int kBulkStages = PC_BULK_STAGES;
 constexpr int kBulkChunk = PC_BULK_CHUNK;  // bytes per source per stage (a multiple of 512)
 constexpr int kBulkWarpBytes = (kBulkStages * kMaxDirect * kBulkChunk + 8 * kBulkStages + 127) / 128 * 128;
-constexpr size_t kDirectSmem = PC_DIRECT_BULK ? (size_t)(kEngineBlock / 32) * kBulkWarpBytes : 0;
+constexpr size_t kBulkSmem = (size_t)(kEngineBlock / 32) * kBulkWarpBytes;  // a CTA's bulk stages
+constexpr size_t kDirectSmem = PC_DIRECT_BULK ? kBulkSmem : 0;
+// The thin (overlap) DIRECT engines: one 16-B vector per operand in flight in
+// registers (PC_THIN_FV), or the bulk-copy fold (PC_THIN_BULK: the P source
+// chunks staged in shared memory by cp.async.bulk, so the bytes in flight are
+// not bounded by the 128-register budget; same-GPU peers only).
+#ifndef PC_THIN_FV
+#define PC_THIN_FV 1
+#endif
+#ifndef PC_THIN_BULK
+#define PC_THIN_BULK 0
+#endif
+constexpr size_t kThinSmem = PC_THIN_BULK ? kBulkSmem : 0;
 
 struct WarpBulk {
   uint8_t *stage;     // [kBulkStages][kMaxDirect][kBulkChunk]
@@ -793,7 +805,7 @@ __device__ __forceinline__ void warp_fold_ptrs(const uint8_t *const (&S)[kMaxDir
   for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
 }
 
-template <int DT, int OP, int FV = PC_DIRECT_FV, bool PF = false, bool PUSH = false>
+template <int DT, int OP, int FV = PC_DIRECT_FV, bool PF = false, bool PUSH = false, bool BULK = PC_DIRECT_BULK>
 __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W, uint8_t *smem) {
   const int P = a.P, r = a.r;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;
@@ -812,7 +824,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
     return;
   }
   WarpBulk wb{};
-  if (PC_DIRECT_BULK && !a.sys) warp_bulk_init(wb, smem);
+  if (BULK && !a.sys) warp_bulk_init(wb, smem);
   // every peer has posted ready-to-receive (all P-1 words polled at once)
   if (!warp_wait_all(a.rtr, P - 1, e, a.err, a.timeout_ms, a.sys)) return;
   const uint32_t target = e * (uint32_t)(P - 1);
@@ -872,7 +884,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
             }
             warp_fold_ptrs<DT, OP, FV>(S, D, P, hi - lo);
           } else if (!PUSH && hi > lo) {
-            if (PC_DIRECT_BULK && !a.sys)
+            if (BULK && !a.sys)
               warp_fold_pull_bulk<DT, OP>(a, base + lo, base + lo, hi - lo, wb);
             else
               warp_fold_pull<DT, OP, true, FV, PF>(a, base + lo, base + lo, hi - lo);
@@ -1170,8 +1182,9 @@ __global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine_gr
 // leaves ~11 K registers: no 512-thread producer block fits beside it).
 template <int DT, int OP>
 __global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_thin(DirectArgs a) {
-  direct_body<DT, OP, 1, true>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5,
-                               nullptr);
+  extern __shared__ __align__(128) uint8_t tsmem[];
+  direct_body<DT, OP, PC_THIN_FV, !PC_THIN_BULK, false, PC_THIN_BULK>(
+      a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5, tsmem);
 }
 template <int DT, int OP>
 __global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_group_thin(DirectGroupArgs g) {
@@ -1179,7 +1192,9 @@ __global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_group_thin(Dire
   while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
   const int b = blockIdx.x - g.block_start[k];
   const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
-  direct_body<DT, OP, 1, true>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, nullptr);
+  extern __shared__ __align__(128) uint8_t tsmem[];
+  direct_body<DT, OP, PC_THIN_FV, !PC_THIN_BULK, false, PC_THIN_BULK>(
+      g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, tsmem);
 }
 
 // DIRECT, PUSH variant (PC_ALGO_DIRECT_PUSH): separate kernels, so the PULL

@@ -46,7 +46,10 @@ int EngineLaunch<DT, OP>::direct(const DirectArgs &a, int warps, cudaStream_t s,
     return 0;
   }
   if (thin) {
-    direct_engine_thin<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    if (kThinSmem > 48 * 1024)
+      PC_CUDA(cudaFuncSetAttribute(direct_engine_thin<DT, OP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)kThinSmem));
+    direct_engine_thin<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, kThinSmem, s>>>(a);
     g_launches++;
     PC_CUDA(cudaGetLastError());
     return 0;
@@ -83,7 +86,10 @@ int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cud
     return 0;
   }
   if (thin) {
-    direct_engine_group_thin<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+    if (kThinSmem > 48 * 1024)
+      PC_CUDA(cudaFuncSetAttribute(direct_engine_group_thin<DT, OP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)kThinSmem));
+    direct_engine_group_thin<DT, OP><<<blocks, kEngineBlock, kThinSmem, s>>>(h);
     g_launches++;
     PC_CUDA(cudaGetLastError());
     return 0;
