@@ -1114,6 +1114,7 @@ static void batch_destroy(BatchCache *b) {
     }
     if (q->last_done == b->ev) q->last_done = nullptr;
   }
+  if (b->ev) cudaEventSynchronize(b->ev);  // the last launch that read the tables has finished
   if (b->dev) cudaFree(b->dev);
   if (b->ev) cudaEventDestroy(b->ev);
   delete b;
