@@ -106,3 +106,52 @@ def test_overlap_width_bound():
         with comms(P) as cs:
             assert cs[0].overlap_warps * P <= sms * 8 // 2
             assert cs[0].overlap_warps % 8 == 0 and cs[0].overlap_warps >= 8
+
+
+@pytest.mark.parametrize("algo,P", [(pc.ALGO_DIRECT, 8), (pc.ALGO_RING, 4), (pc.ALGO_DIRECT_PUSH, 4)])
+def test_back_to_back_epochs_without_host_sync(algo, P):
+    """The early fork must keep every epoch ordered after the previous epoch's
+    consumer: 24 epochs back to back on per-rank streams with NO host
+    synchronisation — each epoch a producer kernel writes new (epoch-tagged)
+    inputs and Preadies them, the engine (forked at pbuf_prepare) reduces, and
+    a consumer copies recvbuf into that epoch's slot on the same stream before
+    the next pc_start.  Every epoch's slot must equal the oracle's fold of that
+    epoch's inputs."""
+    Np, L, E = 6, 3001, 24
+    n = Np * L
+    with comms(P, timeout_ms=20000) as cs:
+        streams = [torch.cuda.Stream() for _ in range(P)]
+        xs = [np.stack([synth.normal_f32(SEED + 9, r, e, n) for r in range(P)]) for e in range(E)]
+        src = [torch.from_numpy(np.stack([xs[e][r] for e in range(E)])).cuda() for r in range(P)]  # [E, n]
+        send = [torch.zeros(n, device="cuda") for _ in range(P)]
+        recv = [torch.zeros(n, device="cuda") for _ in range(P)]
+        slots = [torch.zeros(E, n, device="cuda") for _ in range(P)]
+        reqs = [pc.pallreduce_init(send[r], recv[r], Np, L, pc.FLOAT32, pc.SUM, algo, cs[r]) for r in range(P)]
+        torch.cuda.synchronize()
+        for e in range(E):
+            for r in range(P):
+                reqs[r].start(streams[r])
+            if e == 0:
+                first_prepare([[q] for q in reqs], streams)
+                preqs = [q.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_ENGINE) for q in reqs]
+            else:
+                for r in range(P):
+                    reqs[r].pbuf_prepare(streams[r])
+            for r in range(P):
+                apps.produce(send[r], src[r][e], Np, L * 4, apps.GRAN_BLOCK, preqs[r],
+                             order_stride=(1, 5, 7)[e % 3], stream=streams[r])  # coprime with Np = 6
+            for r in range(P):
+                reqs[r].wait_on_stream(streams[r])
+            for r in range(P):
+                with torch.cuda.stream(streams[r]):
+                    slots[r][e].copy_(recv[r])  # the consumer of this epoch's result
+        torch.cuda.synchronize()
+        for q in reqs:
+            assert q.error() == (0, 0)
+        oalgo = oracle.RING if algo == pc.ALGO_RING else oracle.DIRECT
+        for e in range(E):
+            ref, _, _ = oracle.pallreduce(xs[e], Np, oalgo)
+            for r in range(P):
+                np.testing.assert_array_equal(slots[r][e].cpu().numpy().view(np.uint32), ref[r].view(np.uint32))
+        for q in reqs:
+            q.free()
