@@ -129,7 +129,8 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
     if n * 4 <= (64 << 20):
         parity = parity and int32_gate(cs, Np, count, algo, st)
     ms = statistics.median(blocks)
-    return {"bytes_per_rank": n * 4, "partitions": Np, "ranks": P, "algo": ["auto", "ring", "rd", "direct"][algo],
+    return {"bytes_per_rank": n * 4, "partitions": Np, "ranks": P,
+            "algo": ["auto", "ring", "rd", "direct", "direct_push"][algo],
             "us_per_step": ms * 1e3, "busbw_gbs": busbw(n * 4, ms / 1e3, P), "slices": info["slices"],
             "graph": graph, "errors": errs, "parity": parity}
 
@@ -138,7 +139,8 @@ def sweep_allreduce(args):
     for P in [int(x) for x in args.ranks.split(",")]:
         g, cs = pc.local_comms(P, 0)
         for algo in args.algos.split(","):
-            a = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "auto": pc.ALGO_AUTO}[algo]
+            a = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "direct_push": pc.ALGO_DIRECT_PUSH,
+                 "auto": pc.ALGO_AUTO}[algo]
             if a == pc.ALGO_RD and P & (P - 1):
                 continue
             S = 1 << 10
@@ -413,7 +415,8 @@ def sweep_p2p(args):
                     ok = torch.equal(R, Cb)
                     print(json.dumps({"bytes": S, "gran": ["thread", "warp", "block"][gran], "agg": agg_name,
                                       "g": agg, "copy": ["inline", "engine"][copy], "us": us,
-                                      "goodput_gbs": S / (us / 1e6) / 1e9, "ok": ok, "errors": errs}), flush=True)
+                                      "goodput_gbs": S / (us / 1e6) / 1e9, "ok": ok, "parity": ok and not errs,
+                                      "errors": errs}), flush=True)
                     snd.free()
                     rcv.free()
     for c in cs:
