@@ -511,7 +511,11 @@ __device__ __forceinline__ void prefetch_l2(const void *p, int64_t bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"((uint32_t)bytes) : "memory");
 }
 
-template <int DT, int OP, bool TO_PEERS = true, int FV = PC_DIRECT_FV, bool PF = false, typename A>
+// MAXP: the largest P the call handles (P <= MAXP): the register arrays are
+// sized by it, so a small comm can keep FV * 8 / MAXP vectors per operand in
+// flight for the same registers (direct_body picks MAXP from P).
+template <int DT, int OP, bool TO_PEERS = true, int FV = PC_DIRECT_FV, bool PF = false, int MAXP = kMaxDirect,
+          typename A>
 __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d0, int64_t n) {
   using O = Op<DT, OP>;
   using T = typename O::T;
@@ -562,9 +566,9 @@ __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d
   int64_t k = lane;
   for (; k + 32 * (kFV - 1) < nv; k += 32 * kFV) {
     if (pf && ((k - lane) % kPfV) == 0) pf_block((k - lane) / kPfV + kPfAhead);
-    uint4 x[kMaxDirect][kFV];
+    uint4 x[MAXP][kFV];
 #pragma unroll
-    for (int j = 0; j < kMaxDirect; ++j)
+    for (int j = 0; j < MAXP; ++j)
       if (j < P) {
         const uint4 *sj = reinterpret_cast<const uint4 *>(src(j) + head);
 #pragma unroll
@@ -574,19 +578,19 @@ __device__ __forceinline__ void warp_fold_pull(const A &a, int64_t s0, int64_t d
     for (int v = 0; v < kFV; ++v) {
       uint4 acc = x[0][v];
 #pragma unroll
-      for (int j = 1; j < kMaxDirect; ++j)
+      for (int j = 1; j < MAXP; ++j)
         if (j < P) acc = vop<DT, OP>(acc, x[j][v]);
       store_all(k + 32 * v, acc);
     }
   }
   for (; k < nv; k += 32) {
-    uint4 x[kMaxDirect];
+    uint4 x[MAXP];
 #pragma unroll
-    for (int j = 0; j < kMaxDirect; ++j)
+    for (int j = 0; j < MAXP; ++j)
       if (j < P) x[j] = __ldcg(reinterpret_cast<const uint4 *>(src(j) + head) + k);
     uint4 acc = x[0];
 #pragma unroll
-    for (int j = 1; j < kMaxDirect; ++j)
+    for (int j = 1; j < MAXP; ++j)
       if (j < P) acc = vop<DT, OP>(acc, x[j]);
     store_all(k, acc);
   }
@@ -805,7 +809,8 @@ __device__ __forceinline__ void warp_fold_ptrs(const uint8_t *const (&S)[kMaxDir
   for (int64_t kk = head + nv * EPV + lane; kk < n; kk += 32) scalar(kk);
 }
 
-template <int DT, int OP, int FV = PC_DIRECT_FV, bool PF = false, bool PUSH = false, bool BULK = PC_DIRECT_BULK>
+template <int DT, int OP, int FV = PC_DIRECT_FV, bool PF = false, bool PUSH = false, bool BULK = PC_DIRECT_BULK,
+          int MAXP = kMaxDirect>
 __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, const int W, uint8_t *smem) {
   const int P = a.P, r = a.r;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;
@@ -886,8 +891,8 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
           } else if (!PUSH && hi > lo) {
             if (BULK && !a.sys)
               warp_fold_pull_bulk<DT, OP>(a, base + lo, base + lo, hi - lo, wb);
-            else
-              warp_fold_pull<DT, OP, true, FV, PF>(a, base + lo, base + lo, hi - lo);
+            else  // MAXP < 8: fewer sources, FV * 8 / MAXP vectors per operand in flight, same registers
+              warp_fold_pull<DT, OP, true, FV * kMaxDirect / MAXP, PF, MAXP>(a, base + lo, base + lo, hi - lo);
           }
           fence_scope(a.sys);
           __syncwarp();
@@ -1160,19 +1165,24 @@ __global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) coll_engine_grou
   coll_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
 }
 
-template <int DT, int OP>
+// MAXP: the comm size bound of the instantiation (P <= MAXP): 8, or 4 / 2
+// for small comms, which keep 2x / 4x more vectors per operand in flight
+// for the same registers (the launcher picks it from P).
+template <int DT, int OP, int MAXP = kMaxDirect>
 __global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine(DirectArgs a) {
   extern __shared__ __align__(128) uint8_t dsmem[];
-  direct_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5, dsmem);
+  direct_body<DT, OP, PC_DIRECT_FV, false, false, PC_DIRECT_BULK, MAXP>(
+      a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5, dsmem);
 }
-template <int DT, int OP>
+template <int DT, int OP, int MAXP = kMaxDirect>
 __global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) direct_engine_group(DirectGroupArgs g) {
   int k = 0;
   while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
   const int b = blockIdx.x - g.block_start[k];
   const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
   extern __shared__ __align__(128) uint8_t dsmem[];
-  direct_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, dsmem);
+  direct_body<DT, OP, PC_DIRECT_FV, false, false, PC_DIRECT_BULK, MAXP>(
+      g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5, dsmem);
 }
 
 // "Thin" DIRECT engines for the overlap case (the engine runs beside the

@@ -55,7 +55,13 @@ int EngineLaunch<DT, OP>::direct(const DirectArgs &a, int warps, cudaStream_t s,
     return 0;
   }
   if (int rc = direct_smem_attr(direct_engine<DT, OP>)) return rc;
-  direct_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, kDirectSmem, s>>>(a);
+  const int grid = grid_for(warps, a.nunits);
+  if (a.P <= 2)
+    direct_engine<DT, OP, 2><<<grid, kEngineBlock, kDirectSmem, s>>>(a);
+  else if (a.P <= 4)
+    direct_engine<DT, OP, 4><<<grid, kEngineBlock, kDirectSmem, s>>>(a);
+  else
+    direct_engine<DT, OP><<<grid, kEngineBlock, kDirectSmem, s>>>(a);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -95,7 +101,12 @@ int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cud
     return 0;
   }
   if (int rc = direct_smem_attr(direct_engine_group<DT, OP>)) return rc;
-  direct_engine_group<DT, OP><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
+  if (h.a[0].P <= 2)
+    direct_engine_group<DT, OP, 2><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
+  else if (h.a[0].P <= 4)
+    direct_engine_group<DT, OP, 4><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
+  else
+    direct_engine_group<DT, OP><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -164,6 +175,10 @@ int EngineLaunch<DT, OP>::preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, ring_engine_group<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, rd_engine_group<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP, 4>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP, 2>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine<DT, OP, 4>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine<DT, OP, 2>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_batch<DT, OP>));
