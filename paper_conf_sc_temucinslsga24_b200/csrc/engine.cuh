@@ -201,14 +201,17 @@ __device__ __forceinline__ void warp_copy(void *dst, const void *src, int64_t nb
 // push): every source vector is loaded ONCE and stored nd+1 times.  The
 // destinations share one misalignment (same offset of 16-B aligned buffers);
 // if the source does not, fall back to one warp_copy per destination.
-template <int MAXD>
+// skip: one index of dsts not written (-1: none); U source vectors per lane
+// in flight.
+template <int MAXD, int U = 4>
 __device__ __forceinline__ void warp_copy_multi(uint8_t *dst0, uint8_t *const *dsts, int nd, int64_t doff,
-                                                const uint8_t *src, int64_t nbytes) {
+                                                const uint8_t *src, int64_t nbytes, int skip = -1) {
   const uint32_t lane = threadIdx.x & 31;
   const uintptr_t m = reinterpret_cast<uintptr_t>(dst0 + doff) & 15;
   if ((reinterpret_cast<uintptr_t>(src) & 15) != m) {
     warp_copy(dst0 + doff, src, nbytes);
-    for (int j = 0; j < nd; ++j) warp_copy(dsts[j] + doff, src, nbytes);
+    for (int j = 0; j < nd; ++j)
+      if (j != skip) warp_copy(dsts[j] + doff, src, nbytes);
     return;
   }
   int64_t h = (int64_t)((16 - m) & 15);
@@ -216,21 +219,22 @@ __device__ __forceinline__ void warp_copy_multi(uint8_t *dst0, uint8_t *const *d
   for (int64_t b = lane; b < h; b += 32) {
     const uint8_t v = src[b];
     dst0[doff + b] = v;
-    for (int j = 0; j < nd; ++j) dsts[j][doff + b] = v;
+    for (int j = 0; j < nd; ++j)
+      if (j != skip) dsts[j][doff + b] = v;
   }
   const int64_t nv = (nbytes - h) >> 4;
   const uint4 *s4 = reinterpret_cast<const uint4 *>(src + h);
   int64_t k = lane;
-  for (; k + 32 * 3 < nv; k += 32 * 4) {
-    uint4 x[4];
+  for (; k + 32 * (U - 1) < nv; k += 32 * U) {
+    uint4 x[U];
 #pragma unroll
-    for (int v = 0; v < 4; ++v) x[v] = __ldcg(s4 + k + 32 * v);
+    for (int v = 0; v < U; ++v) x[v] = __ldcg(s4 + k + 32 * v);
 #pragma unroll
-    for (int v = 0; v < 4; ++v) {
+    for (int v = 0; v < U; ++v) {
       reinterpret_cast<uint4 *>(dst0 + doff + h)[k + 32 * v] = x[v];
 #pragma unroll
       for (int j = 0; j < MAXD; ++j)
-        if (j < nd) reinterpret_cast<uint4 *>(dsts[j] + doff + h)[k + 32 * v] = x[v];
+        if (j < nd && j != skip) reinterpret_cast<uint4 *>(dsts[j] + doff + h)[k + 32 * v] = x[v];
     }
   }
   for (; k < nv; k += 32) {
@@ -238,12 +242,13 @@ __device__ __forceinline__ void warp_copy_multi(uint8_t *dst0, uint8_t *const *d
     reinterpret_cast<uint4 *>(dst0 + doff + h)[k] = x;
 #pragma unroll
     for (int j = 0; j < MAXD; ++j)
-      if (j < nd) reinterpret_cast<uint4 *>(dsts[j] + doff + h)[k] = x;
+      if (j < nd && j != skip) reinterpret_cast<uint4 *>(dsts[j] + doff + h)[k] = x;
   }
   for (int64_t b = h + (nv << 4) + lane; b < nbytes; b += 32) {
     const uint8_t v = src[b];
     dst0[doff + b] = v;
-    for (int j = 0; j < nd; ++j) dsts[j][doff + b] = v;
+    for (int j = 0; j < nd; ++j)
+      if (j != skip) dsts[j][doff + b] = v;
   }
 }
 
@@ -1042,13 +1047,15 @@ __global__ void __launch_bounds__(kEngineBlock, 2) direct_engine_batch_thin(Dire
 //    0: ready[u] -> copy my block to recvbuf[r][u] here and at every peer,
 //       fence, per-source arrival flag + phase-0 counter at every peer
 //    1: P-1 arrivals of partition u -> done[u]
-//  BCAST (buf [u][count]), PULL: root: ready[u] -> announce to every peer
-//    (phase-0 counter) -> all P-1 peers done reading (phase-1) -> done[u];
-//    non-root: root's announcement -> copy the root's slice into my buf with
-//    peer loads -> tell the root (its phase-1 counter) -> done[u]
+//  BCAST (buf [u][count]): root: ready[u] -> announce to every peer
+//    (phase-0 counter) -> all P-1 parts read (phase-1) -> done[u];
+//    non-root kk (of P-1): root's announcement -> read part kk of the root's
+//    slice ONCE (peer loads) and store it into every receiver's buf -> bump
+//    the root's and every receiver's phase-1 counter -> (all P-1 parts of my
+//    slice arrived) done[u].  The root's slice leaves it once (S, not (P-1) S)
 //  (ALLGATHER pushes each vector once to all P buffers: warp_copy_multi)
 // ---------------------------------------------------------------------------
-template <int DT, int OP>
+template <int DT, int OP, int MAXP = kMaxDirect>
 __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const int W) {
   const int P = a.P, r = a.r;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;
@@ -1057,8 +1064,8 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
   const bool rs = a.coll == PC_COLL_REDUCE_SCATTER, ag = a.coll == PC_COLL_ALLGATHER;
   const bool bc = a.coll == PC_COLL_BCAST, root = bc && r == a.root;
   // writers into peers' buffers need every peer's ready-to-receive
-  // (allgather pushes; the broadcast is pulled by the receivers themselves)
-  if (P > 1 && ag && !warp_wait_all(a.rtr, P - 1, e, a.err, a.timeout_ms, a.sys)) return;
+  // (allgather pushes; broadcast receivers forward their part to the others)
+  if (P > 1 && (ag || (bc && !root)) && !warp_wait_all(a.rtr, P - 1, e, a.err, a.timeout_ms, a.sys)) return;
   const uint32_t target = e * (uint32_t)(P - 1);
   for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
     int step[kMaxActive];
@@ -1089,14 +1096,37 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
           }
           if (ag && (threadIdx.x & 31) == 0) st_release_gpu(a.srcflags + (int64_t)u * a.ns + s, e);
           finished = true;
-        } else if (bc && !root) {  // PULL: copy the root's slice once it is announced, then tell the root
+        } else if (bc && !root && P == 2) {  // one receiver: copy the root's slice, tell the root
           if (!warp_poll(cnt_u, e, a.sys)) continue;
-          const int jr = (a.root - r - 1 + P) % P;
           const int64_t off = ((int64_t)u * a.count + lo) * es;
-          if (n) warp_copy(a.recvbuf + off, a.p_recvbuf[jr] + off, n * es);
+          if (n) warp_copy(a.recvbuf + off, a.p_recvbuf[0] + off, n * es);
           fence_scope(a.sys);  // our reads of the root's slice are done before it may reuse it
           __syncwarp();
-          if ((threadIdx.x & 31) == 0) red_add_scope(a.p_cnt[jr] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
+          if ((threadIdx.x & 31) == 0) red_add_scope(a.p_cnt[0] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
+          finished = true;
+        } else if (bc && !root && i == 0) {
+          // split receive (scatter + allgather): once the root announced the
+          // slice, receiver kk (of the P-1) reads part kk of it from the root
+          // ONCE and stores it into every receiver's buffer; then it tells the
+          // root (its part was read) and every receiver (the part arrived)
+          if (!warp_poll(cnt_u, e, a.sys)) continue;
+          const int jr = (a.root - r - 1 + P) % P;          // the root's peer index
+          const int kk = (r - a.root - 1 + P) % P;          // my part, 0 .. P-2
+          const int64_t epv = 16 / es > 0 ? 16 / es : 1;
+          const int64_t pq = (((n + P - 2) / (P - 1)) + epv - 1) / epv * epv;
+          const int64_t plo = min(lo + (int64_t)kk * pq, hi), phi = min(plo + pq, hi);
+          const int64_t off = ((int64_t)u * a.count + plo) * es;
+          if (phi > plo)
+            warp_copy_multi<kMaxDirect - 1, 8>(a.recvbuf, a.p_recvbuf, P - 1, off, a.p_recvbuf[jr] + off,
+                                               (phi - plo) * es, jr);
+          fence_scope(a.sys);  // my reads of the root and my stores to the receivers, then the signals
+          __syncwarp();
+          if ((threadIdx.x & 31) == 0)
+            for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
+          if ((threadIdx.x & 31) == 0) red_add_scope(const_cast<uint32_t *>(cnt_u + a.ns), 1, a.sys);  // my own part
+          step[jj] = 1;
+        } else if (bc && !root) {  // every part of my slice arrived (P-1 receivers, me included)
+          if (!warp_poll(cnt_u + a.ns, target, a.sys)) continue;
           finished = true;
         } else if (i == 0) {
           if (!warp_poll(a.ready + u, e, false)) continue;
@@ -1123,7 +1153,8 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
           if (!warp_poll(cnt_u, target, a.sys)) continue;
           if (rs) {
             if (n)
-              warp_fold_pull<DT, OP, false>(a, ((int64_t)u * P + r) * a.count + lo, (int64_t)u * a.count + lo, n);
+              warp_fold_pull<DT, OP, false, PC_DIRECT_FV * kMaxDirect / MAXP, false, MAXP>(
+                  a, ((int64_t)u * P + r) * a.count + lo, (int64_t)u * a.count + lo, n);
             fence_scope(a.sys);
             __syncwarp();
             if ((threadIdx.x & 31) == 0)
@@ -1152,17 +1183,19 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
   }
 }
 
-template <int DT, int OP>
+// MAXP as for the DIRECT engines: the reduce-scatter fold keeps 8 / MAXP
+// times more loads in flight for small comms.
+template <int DT, int OP, int MAXP = kMaxDirect>
 __global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) coll_engine(CollArgs a) {
-  coll_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
+  coll_body<DT, OP, MAXP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
 }
-template <int DT, int OP>
+template <int DT, int OP, int MAXP = kMaxDirect>
 __global__ void __launch_bounds__(kEngineBlock, PC_DIRECT_MINB) coll_engine_group(CollGroupArgs g) {
   int k = 0;
   while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
   const int b = blockIdx.x - g.block_start[k];
   const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
-  coll_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
+  coll_body<DT, OP, MAXP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
 }
 
 // MAXP: the comm size bound of the instantiation (P <= MAXP): 8, or 4 / 2

@@ -152,7 +152,13 @@ int EngineLaunch<DT, OP>::occupancy_direct(int *ctas) {
 
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::coll(const CollArgs &a, int warps, cudaStream_t s) {
-  coll_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+  const int grid = grid_for(warps, a.nunits);
+  if (a.P <= 2)
+    coll_engine<DT, OP, 2><<<grid, kEngineBlock, 0, s>>>(a);
+  else if (a.P <= 4)
+    coll_engine<DT, OP, 4><<<grid, kEngineBlock, 0, s>>>(a);
+  else
+    coll_engine<DT, OP><<<grid, kEngineBlock, 0, s>>>(a);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -160,7 +166,12 @@ int EngineLaunch<DT, OP>::coll(const CollArgs &a, int warps, cudaStream_t s) {
 
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s) {
-  coll_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+  if (h.a[0].P <= 2)
+    coll_engine_group<DT, OP, 2><<<blocks, kEngineBlock, 0, s>>>(h);
+  else if (h.a[0].P <= 4)
+    coll_engine_group<DT, OP, 4><<<blocks, kEngineBlock, 0, s>>>(h);
+  else
+    coll_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -187,6 +198,10 @@ int EngineLaunch<DT, OP>::preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_batch_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP, 4>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP, 2>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP, 4>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP, 2>));
   return 0;
 }
 
