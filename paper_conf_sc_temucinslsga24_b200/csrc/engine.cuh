@@ -1319,4 +1319,18 @@ struct EngineLaunch {
   static int preload();  // load every engine kernel now (lazy module loading, see kernels.cu)
 };
 
+// The small-comm (MAXP = 4, 2) DIRECT / collective kernels of one (dtype, op):
+// defined in engine_small.cu, a translation unit of their own (built for the
+// gradient types' SUM only), so the long compiles run in parallel.
+template <int DT, int OP>
+struct SmallCommLaunch {
+  static int direct(const DirectArgs &a, int grid, cudaStream_t s, int maxp);
+  static int direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s, int maxp);
+  static int coll(const CollArgs &a, int grid, cudaStream_t s, int maxp);
+  static int coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s, int maxp);
+  static int preload();
+};
+template <int DT, int OP>
+constexpr bool kSmallCommKernels = (DT == 1 || DT == 4) && OP == 0;
+
 }  // namespace pc

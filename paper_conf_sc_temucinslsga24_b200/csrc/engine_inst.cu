@@ -9,6 +9,11 @@
 
 namespace pc {
 
+// The small-comm instantiations (MAXP 4 / 2, engine.cuh) exist for the
+// gradient types' SUM only (fp32, bf16; SmallCommLaunch in engine_small.cu):
+// every other (dtype, op) runs the MAXP = 8 kernels for any P (correct, fewer
+// loads in flight) — it keeps the library's build time and size in bounds.
+
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::ring(const RingArgs &a, int warps, cudaStream_t s) {
   ring_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
@@ -56,12 +61,15 @@ int EngineLaunch<DT, OP>::direct(const DirectArgs &a, int warps, cudaStream_t s,
   }
   if (int rc = direct_smem_attr(direct_engine<DT, OP>)) return rc;
   const int grid = grid_for(warps, a.nunits);
-  if (a.P <= 2)
-    direct_engine<DT, OP, 2><<<grid, kEngineBlock, kDirectSmem, s>>>(a);
-  else if (a.P <= 4)
-    direct_engine<DT, OP, 4><<<grid, kEngineBlock, kDirectSmem, s>>>(a);
-  else
+  if constexpr (kSmallCommKernels<DT, OP>) {
+    if (a.P <= 4) {
+      return SmallCommLaunch<DT, OP>::direct(a, grid, s, a.P <= 2 ? 2 : 4);
+    } else {
+      direct_engine<DT, OP><<<grid, kEngineBlock, kDirectSmem, s>>>(a);
+    }
+  } else {
     direct_engine<DT, OP><<<grid, kEngineBlock, kDirectSmem, s>>>(a);
+  }
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -101,12 +109,15 @@ int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cud
     return 0;
   }
   if (int rc = direct_smem_attr(direct_engine_group<DT, OP>)) return rc;
-  if (h.a[0].P <= 2)
-    direct_engine_group<DT, OP, 2><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
-  else if (h.a[0].P <= 4)
-    direct_engine_group<DT, OP, 4><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
-  else
+  if constexpr (kSmallCommKernels<DT, OP>) {
+    if (h.a[0].P <= 4) {
+      return SmallCommLaunch<DT, OP>::direct_group(h, blocks, s, h.a[0].P <= 2 ? 2 : 4);
+    } else {
+      direct_engine_group<DT, OP><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
+    }
+  } else {
     direct_engine_group<DT, OP><<<blocks, kEngineBlock, kDirectSmem, s>>>(h);
+  }
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -153,12 +164,15 @@ int EngineLaunch<DT, OP>::occupancy_direct(int *ctas) {
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::coll(const CollArgs &a, int warps, cudaStream_t s) {
   const int grid = grid_for(warps, a.nunits);
-  if (a.P <= 2)
-    coll_engine<DT, OP, 2><<<grid, kEngineBlock, 0, s>>>(a);
-  else if (a.P <= 4)
-    coll_engine<DT, OP, 4><<<grid, kEngineBlock, 0, s>>>(a);
-  else
+  if constexpr (kSmallCommKernels<DT, OP>) {
+    if (a.P <= 4) {
+      return SmallCommLaunch<DT, OP>::coll(a, grid, s, a.P <= 2 ? 2 : 4);
+    } else {
+      coll_engine<DT, OP><<<grid, kEngineBlock, 0, s>>>(a);
+    }
+  } else {
     coll_engine<DT, OP><<<grid, kEngineBlock, 0, s>>>(a);
+  }
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -166,12 +180,15 @@ int EngineLaunch<DT, OP>::coll(const CollArgs &a, int warps, cudaStream_t s) {
 
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::coll_group(const CollGroupArgs &h, int blocks, cudaStream_t s) {
-  if (h.a[0].P <= 2)
-    coll_engine_group<DT, OP, 2><<<blocks, kEngineBlock, 0, s>>>(h);
-  else if (h.a[0].P <= 4)
-    coll_engine_group<DT, OP, 4><<<blocks, kEngineBlock, 0, s>>>(h);
-  else
+  if constexpr (kSmallCommKernels<DT, OP>) {
+    if (h.a[0].P <= 4) {
+      return SmallCommLaunch<DT, OP>::coll_group(h, blocks, s, h.a[0].P <= 2 ? 2 : 4);
+    } else {
+      coll_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+    }
+  } else {
     coll_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+  }
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
@@ -186,10 +203,9 @@ int EngineLaunch<DT, OP>::preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, ring_engine_group<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, rd_engine_group<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP>));
-  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP, 4>));
-  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group<DT, OP, 2>));
-  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine<DT, OP, 4>));
-  PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine<DT, OP, 2>));
+  if constexpr (kSmallCommKernels<DT, OP>) {
+    if (int rc = SmallCommLaunch<DT, OP>::preload()) return rc;
+  }
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_batch<DT, OP>));
@@ -198,10 +214,7 @@ int EngineLaunch<DT, OP>::preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_batch_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP>));
-  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP, 4>));
-  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine_group<DT, OP, 2>));
-  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP, 4>));
-  PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP, 2>));
+
   return 0;
 }
 

@@ -1114,9 +1114,13 @@ static void batch_destroy(BatchCache *b) {
     }
     if (q->last_done == b->ev) q->last_done = nullptr;
   }
-  if (b->ev) cudaEventSynchronize(b->ev);  // the last launch that read the tables has finished
+  // cudaFree waits for the device (the last eager launch that read the
+  // tables); the event may have been recorded inside a graph capture, where
+  // it cannot be waited on — so no event sync, and no error left behind for
+  // the next launch's cudaGetLastError
   if (b->dev) cudaFree(b->dev);
   if (b->ev) cudaEventDestroy(b->ev);
+  cudaGetLastError();
   delete b;
 }
 
