@@ -78,9 +78,22 @@ typedef enum { PC_COPY_INLINE = 0, PC_COPY_ENGINE = 1, PC_COPY_LL = 2, PC_COPY_H
  * rank's send buffer with peer loads; PC_ALGO_DIRECT_PUSH: the same schedule
  * and bits (rank-order fold, R25), every rank PUSHES its chunk o into owner
  * o's staging with peer stores and the owner folds from local memory (all
- * NVLink traffic is stores; +S staging per rank).  AUTO picks DIRECT
- * (PULL), or PUSH with PC_DIRECT_MODE=push. */
-typedef enum { PC_ALGO_AUTO = 0, PC_ALGO_RING = 1, PC_ALGO_RD = 2, PC_ALGO_DIRECT = 3, PC_ALGO_DIRECT_PUSH = 4 } pc_algo_t;
+ * NVLink traffic is stores; +S staging per rank).  PC_ALGO_LL: one-shot for
+ * small messages — every rank stores each ready partition as 16-B LL lines
+ * {4 B data, epoch, 4 B data, epoch} into every peer's line area (no fence,
+ * no flag: a line is its own arrival flag) and every rank folds all P
+ * contributions itself in rank order (the same bits); one hop; line areas
+ * double-buffered by epoch parity (4·P·S bytes per rank).  AUTO picks LL up
+ * to PC_LL_AR_MAX_BYTES (default 64 KiB) per rank, else DIRECT (PULL), or
+ * PUSH with PC_DIRECT_MODE=push. */
+typedef enum {
+  PC_ALGO_AUTO = 0,
+  PC_ALGO_RING = 1,
+  PC_ALGO_RD = 2,
+  PC_ALGO_DIRECT = 3,
+  PC_ALGO_DIRECT_PUSH = 4,
+  PC_ALGO_LL = 5
+} pc_algo_t;
 
 enum {
   PC_SUCCESS = 0,

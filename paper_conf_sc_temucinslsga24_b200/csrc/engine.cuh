@@ -919,6 +919,149 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
 }
 
 // ---------------------------------------------------------------------------
+// One-shot LL allreduce (PC_ALGO_LL, small messages).  Unit = user partition
+// u.  Step 0 (the user's Pready of u): the warp stores partition u as 16-B
+// lines {4 B data, e, 4 B data, e} into slot [e & 1][r][u] of EVERY peer's
+// line area — no fence, no flag: each 8-B half carries the epoch, so a line is
+// its own arrival flag.  Step 1: every line of u from all P-1 peers carries
+// epoch e -> fold the P contributions in rank order (R25; my own from my send
+// buffer) and store the result into MY recvbuf only -> done[u].  One hop.
+// Parity slot e&1 was last read by the peer in epoch e-2; this rank completing
+// e-1 needed the peer's e-1 lines, pushed by the peer's engine e-1, which runs
+// after its engine e-2 finished reading — so no ready-to-receive is needed.
+// ---------------------------------------------------------------------------
+template <int DT, int OP>
+__device__ __forceinline__ uint64_t vop8(uint64_t a, uint64_t b) {
+  using O = Op<DT, OP>;
+  using T = typename O::T;
+  constexpr int EPW = 8 / sizeof(T);
+  uint64_t r;
+  T *pr = reinterpret_cast<T *>(&r);
+  const T *pa = reinterpret_cast<const T *>(&a);
+  const T *pb = reinterpret_cast<const T *>(&b);
+#pragma unroll
+  for (int j = 0; j < EPW; ++j) pr[j] = O::f(pa[j], pb[j]);
+  return r;
+}
+
+// Unit = (partition u, slice s) of 32 * kLLPerLane lines: each lane owns at
+// most kLLPerLane lines of the slice, loads them from all P-1 sources at once
+// (every load in flight together), validates, and folds straight from the
+// registers.
+constexpr int kLLPerLane = 2;
+constexpr int64_t kLLSlice = 32 * kLLPerLane;  // lines per unit
+
+template <int DT, int OP>
+__device__ __forceinline__ void ll_body(const DirectArgs &a, const int gw, const int W) {
+  const int P = a.P, r = a.r;
+  const uint32_t e = *(const volatile uint32_t *)a.epoch;
+  const uint32_t lane = threadIdx.x & 31;
+  const int64_t es = sizeof(typename Op<DT, OP>::T);
+  const uint64_t pb = (uint64_t)a.L * es;  // bytes per partition
+  const int64_t Lp = a.ll_lines;           // lines per partition
+  const int64_t par = e & 1;
+  auto line = [&](const uint8_t *area, int k, int u, int64_t j) {  // line (parity, source k, partition u, j)
+    return area + ((((par * P + k) * (int64_t)a.Np + u) * Lp + j) << 4);
+  };
+  if (gw >= a.nunits) return;
+  for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
+    int step[kMaxActive];
+    int remaining = 0;
+#pragma unroll
+    for (int j = 0; j < kMaxActive; ++j) {
+      const bool mine = gw + (j0 + j) * W < a.nunits;
+      step[j] = mine ? 0 : 2;
+      remaining += mine;
+    }
+    Idle idle;
+    while (remaining) {
+      bool progressed = false;
+#pragma unroll 1
+      for (int jj = 0; jj < kMaxActive; ++jj) {
+        if (step[jj] > 1) continue;
+        const int x = gw + (j0 + jj) * W;
+        const int u = x / a.ns;
+        const int64_t k0 = (int64_t)(x % a.ns) * kLLSlice;
+        const uint8_t *src = a.sendbuf + (uint64_t)u * pb;
+        if (step[jj] == 0) {
+          if (!warp_poll(a.ready + u, e, false)) continue;
+#pragma unroll
+          for (int t = 0; t < kLLPerLane; ++t) {  // push: my lines of the slice to every peer
+            const int64_t k = k0 + t * 32 + lane;
+            if (k >= Lp) continue;
+            const uint32_t nb = ll_nbytes(pb, (uint32_t)k);
+            const uint64_t v = nb ? ld_payload8(src + 8 * k, nb) : 0;
+            const uint64_t lo = (v & 0xffffffffull) | ((uint64_t)e << 32), hi = (v >> 32) | ((uint64_t)e << 32);
+            for (int j = 0; j < P - 1; ++j)
+              st_ll(const_cast<uint8_t *>(line(a.p_sendbuf[j], r, u, k)), lo, hi, a.sys);
+          }
+          step[jj] = 1;
+          progressed = true;
+        } else {
+          // every source's lines in flight at once, then one validity vote
+          ulonglong2 ln[kMaxDirect][kLLPerLane];
+          bool ok = true;
+#pragma unroll
+          for (int q = 0; q < kMaxDirect; ++q)
+#pragma unroll
+            for (int t = 0; t < kLLPerLane; ++t) {
+              const int64_t k = k0 + t * 32 + lane;
+              ln[q][t] = make_ulonglong2(0, 0);
+              if (q < P && q != r && k < Lp) ln[q][t] = ld_ll(line(a.staging, q, u, k), a.sys);
+            }
+#pragma unroll
+          for (int q = 0; q < kMaxDirect; ++q)
+#pragma unroll
+            for (int t = 0; t < kLLPerLane; ++t) {
+              const int64_t k = k0 + t * 32 + lane;
+              if (q < P && q != r && k < Lp)
+                ok = ok && (uint32_t)(ln[q][t].x >> 32) == e && (uint32_t)(ln[q][t].y >> 32) == e;
+            }
+          if (!__all_sync(0xffffffffu, ok)) continue;
+#pragma unroll
+          for (int t = 0; t < kLLPerLane; ++t) {  // fold in rank order, store my result
+            const int64_t k = k0 + t * 32 + lane;
+            const uint32_t nb = k < Lp ? ll_nbytes(pb, (uint32_t)k) : 0u;
+            if (!nb) continue;
+            uint64_t acc = 0;
+#pragma unroll
+            for (int q = 0; q < kMaxDirect; ++q) {
+              if (q >= P) continue;
+              const uint64_t v = q == r ? ld_payload8(src + 8 * k, nb)
+                                        : (ln[q][t].x & 0xffffffffull) | (ln[q][t].y << 32);
+              acc = q == 0 ? v : vop8<DT, OP>(acc, v);
+            }
+            st_payload8(a.recvbuf + (uint64_t)u * pb + 8 * k, acc, nb);
+          }
+          __syncwarp();
+          if (lane == 0) red_add_release_gpu(a.done + u, 1);
+          step[jj] = 2;
+          --remaining;
+          progressed = true;
+        }
+      }
+      if (progressed)
+        idle.progressed();
+      else if (!idle.wait(a.err, a.timeout_ms, gw))
+        return;
+    }
+  }
+}
+
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) ll_engine(DirectArgs a) {
+  ll_body<DT, OP>(a, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, (gridDim.x * blockDim.x) >> 5);
+}
+template <int DT, int OP>
+__global__ void __launch_bounds__(kEngineBlock) ll_engine_group(DirectGroupArgs g) {
+  int k = 0;
+  while (k + 1 < g.n && (int)blockIdx.x >= g.block_start[k + 1]) ++k;
+  const int b = blockIdx.x - g.block_start[k];
+  const int nb = (k + 1 < g.n ? g.block_start[k + 1] : (int)gridDim.x) - g.block_start[k];
+  ll_body<DT, OP>(g.a[k], (b * blockDim.x + threadIdx.x) >> 5, (nb * blockDim.x) >> 5);
+}
+
+// ---------------------------------------------------------------------------
 // Batched DIRECT engine: MPI_Waitall over many partitioned allreduces of one
 // GPU in ONE launch (one request per gradient tensor).
 // Entries (request t, local rank j) live in a device table (DirectArgs are

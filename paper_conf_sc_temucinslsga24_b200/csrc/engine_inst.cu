@@ -44,6 +44,12 @@ static int direct_smem_attr(K kernel) {
 
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::direct(const DirectArgs &a, int warps, cudaStream_t s, bool thin) {
+  if (a.ll) {
+    ll_engine<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
+    g_launches++;
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  }
   if (a.push) {
     direct_engine_push<DT, OP><<<grid_for(warps, a.nunits), kEngineBlock, 0, s>>>(a);
     g_launches++;
@@ -93,6 +99,12 @@ int EngineLaunch<DT, OP>::rd_group(const RdGroupArgs &h, int blocks, cudaStream_
 
 template <int DT, int OP>
 int EngineLaunch<DT, OP>::direct_group(const DirectGroupArgs &h, int blocks, cudaStream_t s, bool thin) {
+  if (h.a[0].ll) {
+    ll_engine_group<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
+    g_launches++;
+    PC_CUDA(cudaGetLastError());
+    return 0;
+  }
   if (h.a[0].push) {
     direct_engine_group_push<DT, OP><<<blocks, kEngineBlock, 0, s>>>(h);
     g_launches++;
@@ -210,6 +222,8 @@ int EngineLaunch<DT, OP>::preload() {
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_batch<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_push<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, ll_engine<DT, OP>));
+  PC_CUDA(cudaFuncGetAttributes(&fa, ll_engine_group<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_group_push<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, direct_engine_batch_thin<DT, OP>));
   PC_CUDA(cudaFuncGetAttributes(&fa, coll_engine<DT, OP>));

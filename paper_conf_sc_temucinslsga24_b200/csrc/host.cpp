@@ -424,6 +424,8 @@ static int alloc_ctrl(Request *q) {
   PC_CUDA(cudaMemsetAsync(q->ctrl, 0, q->L.words * 4, q->side));
   if (q->staging_bytes) {
     PC_CUDA(cudaMalloc((void **)&q->staging, q->staging_bytes));
+    // LL line areas start with epoch 0 in every line (never a valid epoch)
+    if (q->direct_ll) PC_CUDA(cudaMemsetAsync(q->staging, 0, q->staging_bytes, q->side));
   }
   PC_CUDA(cudaStreamSynchronize(q->side));
   return 0;
@@ -537,7 +539,7 @@ static int make_rec(Request *q, ReqRec *r) {
   r->count = (int64_t)q->count;
   r->dtype = q->dtype;
   r->op = q->op;
-  r->algo = q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo;  // every rank must pick the same variant
+  r->algo = q->direct_ll ? PC_ALGO_LL : q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo;  // the same variant everywhere
   r->seq = q->seq;
   r->coll = q->coll;
   r->root = q->root;
@@ -553,7 +555,7 @@ static int make_rec(Request *q, ReqRec *r) {
   if (q->staging && (rc = export_ptr(c, q->staging, q->staging_bytes, &r->stage))) return rc;
   // DIRECT (PULL): the peers' reduce steps read this rank's send buffer
   // (PUSH exports its staging above: the peers write into it)
-  if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && !q->direct_push && c->size > 1 &&
+  if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && !q->direct_push && !q->direct_ll && c->size > 1 &&
       (q->coll == PC_COLL_ALLREDUCE || q->coll == PC_COLL_REDUCE_SCATTER) &&
       (rc = export_ptr(c, q->sbuf, q->send_bytes, &r->stage)))
     return rc;
@@ -641,7 +643,8 @@ static int exchange_round(Comm *c, Request *target) {
       for (int r = 0; r < c->size && !qrc; ++r) {
         const ReqRec *m = find_rec(all, M, r, PC_KIND_PALLREDUCE, -1, 0, q->seq, cnt);
         if (!m || m->partitions != q->partitions || m->count != (int64_t)q->count || m->dtype != q->dtype ||
-            m->op != q->op || m->algo != (q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo) || m->coll != q->coll ||
+            m->op != q->op ||
+            m->algo != (q->direct_ll ? PC_ALGO_LL : q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo) || m->coll != q->coll ||
             m->root != q->root) {
           fprintf(stderr, "[pc] rank %d: allreduce #%d disagrees with rank %d\n", c->rank, q->seq, r);
           qrc = PC_ERR_MATCH;
@@ -677,7 +680,9 @@ static int exchange_round(Comm *c, Request *target) {
             for (int j = 0; j < P - 1 && !qrc; ++j) {
               const int pj = mod(r + 1 + j, P);
               qrc = imp(pj, j);
-              if (!qrc) q->rtr_targets.push_back({q->nb_ctrl[j], mod(r - pj - 1, P)});
+              // (the LL variant needs no ready-to-receive: its line areas are
+              //  double-buffered by epoch parity, engine.cuh ll_body)
+              if (!qrc && !q->direct_ll) q->rtr_targets.push_back({q->nb_ctrl[j], mod(r - pj - 1, P)});
             }
           } else {
             for (int k = 0; k < q->nsteps && !qrc; ++k) {
@@ -824,6 +829,8 @@ static DirectArgs make_direct_args(Request *q) {
   a.sys = q->sys_scope;
   a.push = q->direct_push ? 1 : 0;
   a.staging = q->staging;
+  a.ll = q->direct_ll ? 1 : 0;
+  a.ll_lines = (int64_t)std::max<uint64_t>(1, (q->part_bytes + 7) / 8);
   return a;
 }
 
@@ -1220,7 +1227,7 @@ static int engine_batch(const std::vector<Request *> &rq, cudaStream_t s) {
   std::vector<Request *> leaders;
   for (Request *q : rq) {
     if (q->kind != PC_KIND_PALLREDUCE || q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT ||
-        q->direct_push || q->inline_ar || !q->active || q->engine_registered || q->engine_launched ||
+        q->direct_push || q->direct_ll || q->inline_ar || !q->active || q->engine_registered || q->engine_launched ||
         q->batch_launched)
       return 1;
     if (q->dtype != q0->dtype || q->op != q0->op || q->comm->device != q0->comm->device) return 1;
@@ -1520,7 +1527,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   Comm *c = (Comm *)comm;
   if (!c || !req || partitions < 1 ||
       (dtype != PC_INT32 && dtype != PC_FLOAT32 && dtype != PC_FLOAT64 && dtype != PC_BF16) || op < 0 || op > 2 ||
-      algo < 0 || algo > PC_ALGO_DIRECT_PUSH)
+      algo < 0 || algo > PC_ALGO_LL)
     return PC_ERR_ARG;
   const int P = c->size;
   const size_t esz = dtype_size(dtype);
@@ -1545,8 +1552,24 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
     else
       a = PC_ALGO_RING;
   }
-  bool push = false;
-  if (a == PC_ALGO_DIRECT_PUSH) {
+  bool push = false, ll = false;
+  // small messages: the one-shot LL variant (one hop, no fences).  Measured
+  // on one B200 (virtual ranks, graph-replayed epochs, profiles/r02_ll_probe.txt)
+  // it wins from ~32 KiB to 64 KiB per rank at P = 8 (256 KiB at P <= 4;
+  // profiles/r02_sweep_small_graph.jsonl) — below, both are launch-bound
+  // and DIRECT is ~1 us ahead; across GPUs it also saves DIRECT's two
+  // system-scope fences and one NVLink hop, so it is taken from 1 byte there.
+  bool spans_gpus = false;
+  for (int k = 0; k < P && !c->dry; ++k)
+    if (memcmp(c->ranks[k].uuid, c->ranks[c->rank].uuid, 16) != 0) spans_gpus = true;
+  const long ll_min = env_long("PC_LL_AR_MIN_BYTES", spans_gpus ? 0 : 32 << 10);
+  const long ll_max = env_long("PC_LL_AR_MAX_BYTES", P <= 4 ? 256 << 10 : 64 << 10);
+  if (algo == PC_ALGO_AUTO && P > 1 && P <= kMaxDirect && (long long)bytes >= ll_min && (long long)bytes <= ll_max)
+    a = PC_ALGO_LL;
+  if (a == PC_ALGO_LL) {
+    a = PC_ALGO_DIRECT;
+    ll = P > 1;
+  } else if (a == PC_ALGO_DIRECT_PUSH) {
     a = PC_ALGO_DIRECT;
     push = true;
   } else if (algo == PC_ALGO_AUTO && a == PC_ALGO_DIRECT) {
@@ -1568,6 +1591,7 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
   q->algo_req = algo;
   q->algo = a;
   q->direct_push = push && P > 1;
+  q->direct_ll = ll;
   q->esize = esz;
   q->peer = -1;
   q->tag = 0;
@@ -1596,6 +1620,12 @@ int pc_pallreduce_init(const void *sendbuf, void *recvbuf, int partitions, size_
     // PULL: owners read the peers' send buffers directly; PUSH: staging
     // [u][source rank][q] receives every rank's copy of this rank's chunk
     q->staging_bytes = q->direct_push ? (size_t)partitions * P * (size_t)q->chunk_elems * esz : 0;
+    if (q->direct_ll) {  // [2 epoch parities][P sources][N_p][lines] of 16-B LL lines, one unit per partition
+      const size_t lines = std::max<size_t>(1, (q->part_bytes + 7) / 8);
+      q->staging_bytes = 2 * (size_t)P * partitions * lines * 16;
+      q->slices = (int)((lines + 63) / 64);  // units of 64 lines (engine.cuh kLLSlice)
+      q->slice_elems = L;
+    }
   } else {
     q->nsteps = log2_exact(P);
     q->chunk_elems = L;
@@ -1960,7 +1990,8 @@ int pc_prequest_create(pc_request_t req, pc_gran_t gran, int aggregation, pc_cop
     }
   } else if (q->kind == PC_KIND_PALLREDUCE) {
     if (copy == PC_COPY_INLINE) {  // R33: INLINE allreduce (DIRECT schedule bits, P <= 8)
-      if (q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT || q->direct_push || c->size > PC_AR_MAX)
+      if (q->coll != PC_COLL_ALLREDUCE || q->algo != PC_ALGO_DIRECT || q->direct_push || q->direct_ll ||
+          c->size > PC_AR_MAX)
         return PC_ERR_UNSUPPORTED;
       if (!c->dry && !q->ar_tab) {
         pc_ar_tab_s t{};
@@ -2424,7 +2455,7 @@ int pc_chunk_bounds(int64_t L, int P, int64_t *out) {
 int pc_request_info(pc_request_t req, int *algo, int *slices, int64_t *slice_elems, int *engine_warps) {
   Request *q = (Request *)req;
   if (!q) return PC_ERR_ARG;
-  if (algo) *algo = q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo;
+  if (algo) *algo = q->direct_ll ? PC_ALGO_LL : q->direct_push ? PC_ALGO_DIRECT_PUSH : q->algo;
   if (slices) *slices = q->slices;
   if (slice_elems) *slice_elems = q->slice_elems;
   if (engine_warps) *engine_warps = q->engine_warps;
@@ -2448,7 +2479,7 @@ int pc_request_peer_buffer(pc_request_t req, int j, void **ptr) {
   if (q->kind == PC_KIND_PSEND) {
     if (j != 0) return PC_ERR_ARG;
     *ptr = q->peer_buf;
-  } else if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && !q->direct_push) {
+  } else if (q->kind == PC_KIND_PALLREDUCE && q->algo == PC_ALGO_DIRECT && !q->direct_push && !q->direct_ll) {
     if (j < 0 || j >= q->comm->size - 1) return PC_ERR_ARG;
     *ptr = q->nb_buf[j];
   } else {

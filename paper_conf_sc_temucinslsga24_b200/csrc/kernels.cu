@@ -271,25 +271,29 @@ __global__ void pready_all_kernel(PreadyAllArgs a) {
 // user's Pready (S_0) of every partition of every allreduce-kind request.
 // Barriers order the phases (all in one block, so CTA-scope visibility).
 __global__ void __launch_bounds__(1024) epoch_all_kernel(EpochAllArgs a) {
+  __shared__ uint32_t esh[kMaxPreadyAll];  // the new epochs: no dependent global reload per RTR / request
   const int t = threadIdx.x;
-  if (t < a.n) a.epoch[t][0] = a.epoch[t][0] + 1;
+  if (t < a.n) {
+    const uint32_t e = a.epoch[t][0] + 1;
+    a.epoch[t][0] = e;
+    esh[t] = e;
+  }
   __syncthreads();
   if (t < a.nrtr) {
-    const uint32_t e = *(const volatile uint32_t *)a.epoch[a.rtr_req[t]];
+    const uint32_t e = esh[a.rtr_req[t]];
     if ((a.rtr_sysmask >> t) & 1)
       st_release_sys(a.rtr_dst[t], e);
     else
       st_release_gpu(a.rtr_dst[t], e);
   }
   if (!a.pready) return;
-  __syncthreads();
   // S_0 of every partition: ready[u] = e.  No fences: the user's data was
   // written by kernels earlier in stream order, and the only reader of
   // ready[] is this rank's engine, launched after this kernel in stream order
   // (kernel boundaries order both), so plain stores spread over the block
   // replace one release per partition.
   for (int k = 0; k < a.n; ++k) {
-    const uint32_t e = *(const volatile uint32_t *)a.epoch[k];
+    const uint32_t e = esh[k];
     uint32_t *ready = a.ready[k];
     for (int j = t; j < a.partitions[k]; j += blockDim.x) st_relaxed_gpu(ready + j, e);
   }

@@ -170,6 +170,7 @@ struct Request {
   // INLINE allreduce (reading R33): a DIRECT allreduce whose prequest was
   // created with PC_COPY_INLINE — the completing Pready folds, no engine
   bool direct_push = false;     // DIRECT schedule, PUSH variant (PC_ALGO_DIRECT_PUSH)
+  bool direct_ll = false;       // DIRECT schedule, one-shot LL variant (PC_ALGO_LL)
   bool inline_ar = false;
   void *ar_tab = nullptr;       // device pc_ar_tab_s (library-owned)
   cudaEvent_t fork_ev_ext = nullptr;  // fork point recorded by a batched control call (else ev_fork)
@@ -364,7 +365,9 @@ struct DirectArgs {
   uint32_t timeout_ms;
   int sys;
   int push;            // PUSH variant: step 0 stores chunk o into owner o's staging slot r
-  uint8_t *staging;    // PUSH: own staging [u][source rank][q elements]
+  uint8_t *staging;    // PUSH: own staging [u][source rank][q elements]; LL: own line area
+  int ll;              // LL one-shot variant: p_sendbuf[j] = peer j's line area
+  int64_t ll_lines;    // LL: 16-B lines per partition = ceil(part bytes / 8)
 };
 struct DirectGroupArgs {
   int n;

@@ -20,7 +20,7 @@ ESIZE = {INT32: 4, FLOAT32: 4, BYTE: 1, FLOAT64: 8, BF16: 2}
 SUM, MAX, MIN = 0, 1, 2
 GRAN_THREAD, GRAN_WARP, GRAN_BLOCK = 0, 1, 2
 COPY_INLINE, COPY_ENGINE, COPY_LL, COPY_HOST = 0, 1, 2, 3
-ALGO_AUTO, ALGO_RING, ALGO_RD, ALGO_DIRECT, ALGO_DIRECT_PUSH = 0, 1, 2, 3, 4
+ALGO_AUTO, ALGO_RING, ALGO_RD, ALGO_DIRECT, ALGO_DIRECT_PUSH, ALGO_LL = 0, 1, 2, 3, 4, 5
 KIND_PSEND, KIND_PRECV, KIND_PALLREDUCE = 1, 2, 3
 
 SUCCESS, ERR_ARG, ERR_CUDA, ERR_STATE, ERR_MATCH, ERR_TIMEOUT, ERR_DEVICE, ERR_NOMEM, ERR_UNSUPPORTED = (
@@ -257,7 +257,7 @@ class Request:
         a, s, w = C.c_int32(), C.c_int32(), C.c_int32()
         q = C.c_int64()
         check(_lib.pc().pc_request_info(self.handle, C.byref(a), C.byref(s), C.byref(q), C.byref(w)), "info")
-        return {"algo": a.value, "algo_name": {1: "ring", 2: "rd", 3: "direct", 4: "direct_push"}.get(a.value, "?"), "slices": s.value,
+        return {"algo": a.value, "algo_name": {1: "ring", 2: "rd", 3: "direct", 4: "direct_push", 5: "ll"}.get(a.value, "?"), "slices": s.value,
                 "slice_elems": q.value, "engine_warps": w.value}
 
     def match(self) -> tuple[int, int]:

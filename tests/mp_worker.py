@@ -22,7 +22,7 @@ comm = pc.Comm.from_process_group(0)
 st = torch.cuda.Stream()
 res = {}
 for name, algo in (("ring", pc.ALGO_RING), ("rd", pc.ALGO_RD), ("direct", pc.ALGO_DIRECT),
-                   ("direct_push", pc.ALGO_DIRECT_PUSH)):
+                   ("direct_push", pc.ALGO_DIRECT_PUSH), ("ll", pc.ALGO_LL)):
     Np, L = 3, 1000
     x = synth.normal_f32(synth.BASE_SEED, r, 0, Np * L)
     send = torch.from_numpy(x).cuda()

@@ -26,7 +26,7 @@ def test_two_processes_ipc(tmp_path):
     Np, L = 3, 1000
     x = np.stack([synth.normal_f32(synth.BASE_SEED, r, 0, Np * L) for r in range(2)])
     for name, algo in (("ring", oracle.RING), ("rd", oracle.RD), ("direct", oracle.DIRECT),
-                       ("direct_push", oracle.DIRECT)):
+                       ("direct_push", oracle.DIRECT), ("ll", oracle.DIRECT)):
         ref, _, _ = oracle.pallreduce(x, Np, algo)
         for r in range(2):
             np.testing.assert_array_equal(res[r][name].view(np.uint32), ref[r].view(np.uint32))

@@ -137,6 +137,7 @@ def test_dry_allreduce_agreement_and_algo_choice():
         q.start()
     pc.run_ranks([(lambda r=r: (reqs[r].pbuf_prepare(), small[r].pbuf_prepare())) for r in range(4)])
     # AUTO (profiles/r01_sweep_allreduce_pull.jsonl): DIRECT (pull) for 3 <= P <= 8
+    # (the one-shot LL variant only from 32 KiB per rank on one GPU)
     assert all(q.info()["algo"] == pc.ALGO_DIRECT for q in reqs)
     assert all(q.info()["algo"] == pc.ALGO_DIRECT for q in small)
     infos = {tuple(sorted(q.info().items())) for q in reqs}
@@ -236,12 +237,16 @@ def test_gloo_two_process_bootstrap_and_matching(tmp_path):
         assert f"OK {r}" in o
 
 
-@pytest.mark.parametrize("P,nbytes,want", [(2, 1024, "RD"), (2, 4 << 20, "RD"), (2, 8 << 20, "DIRECT"),
-                                          (3, 1024, "DIRECT"), (8, 1024, "DIRECT"), (8, 64 << 20, "DIRECT")])
+@pytest.mark.parametrize("P,nbytes,want", [(2, 1024, "RD"), (2, 32 << 10, "LL"), (2, 64 << 10, "LL"),
+                                          (2, 256 << 10, "LL"), (2, 512 << 10, "RD"), (2, 4 << 20, "RD"),
+                                          (2, 8 << 20, "DIRECT"), (8, 128 << 10, "DIRECT"),
+                                          (3, 1024, "DIRECT"), (8, 1024, "DIRECT"), (8, 64 << 10, "LL"),
+                                          (8, 1 << 20, "DIRECT"), (8, 64 << 20, "DIRECT")])
 def test_dry_auto_schedule_policy(P, nbytes, want):
-    """AUTO: RD for P = 2 up to 4 MiB, DIRECT for P <= 8 otherwise (beyond
-    DIRECT's peer limit — more ranks than one process can host dry — RD for
-    small messages, ring above)."""
+    """AUTO on one GPU (dry ranks count as one): the one-shot LL variant from
+    32 KiB to 64 KiB per rank (256 KiB for P <= 4), RD for P = 2 up to 4 MiB, DIRECT for P <= 8
+    otherwise (beyond DIRECT's peer limit — more ranks than one process can
+    host dry — RD for small messages, ring above)."""
     g, cs = _dry(P)
     reqs = [pc.pallreduce_init(0, 0, 1, nbytes // 4, pc.FLOAT32, pc.SUM, pc.ALGO_AUTO, c) for c in cs]
     for q in reqs:

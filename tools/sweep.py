@@ -130,7 +130,7 @@ def time_allreduce(cs, S, Np, algo, min_ms=30.0, graph=False):
         parity = parity and int32_gate(cs, Np, count, algo, st)
     ms = statistics.median(blocks)
     return {"bytes_per_rank": n * 4, "partitions": Np, "ranks": P,
-            "algo": ["auto", "ring", "rd", "direct", "direct_push"][algo],
+            "algo": ["auto", "ring", "rd", "direct", "direct_push", "ll"][algo],
             "us_per_step": ms * 1e3, "busbw_gbs": busbw(n * 4, ms / 1e3, P), "slices": info["slices"],
             "graph": graph, "errors": errs, "parity": parity}
 
@@ -140,6 +140,7 @@ def sweep_allreduce(args):
         g, cs = pc.local_comms(P, 0)
         for algo in args.algos.split(","):
             a = {"ring": pc.ALGO_RING, "rd": pc.ALGO_RD, "direct": pc.ALGO_DIRECT, "direct_push": pc.ALGO_DIRECT_PUSH,
+                 "ll": pc.ALGO_LL,
                  "auto": pc.ALGO_AUTO}[algo]
             if a == pc.ALGO_RD and P & (P - 1):
                 continue
