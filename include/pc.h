@@ -237,6 +237,12 @@ int pc_startall(int n, pc_request_t *reqs, pc_stream_t stream);
  * Pready of every partition of each request (allreduce-kind requests only;
  * PC_ERR_ARG otherwise) — the small-message path, where launches dominate.
  * PC_ERR_STATE if a request is active or not yet exchanged.  Capturable. */
+/* Any n >= 1 (round 2): beyond 16 requests or 64 ready-to-receive words the
+ * lists live in a library-owned device table built on the first call with
+ * that exact request list (a synchronous upload: that first call must not be
+ * captured into a CUDA graph, PC_ERR_STATE otherwise) and reused afterwards;
+ * the table is dropped when one of its requests is freed.  The same request
+ * twice in one call: PC_ERR_ARG, nothing started. */
 int pc_epoch_all(int n, pc_request_t *reqs, int pready, pc_stream_t stream);
 /* pc_pbuf_prepare for n requests whose first pc_pbuf_prepare (exchange +
  * mapping) already happened: all ready-to-receive writes in one kernel.
@@ -273,6 +279,11 @@ int pc_wait_on_stream(pc_request_t req, pc_stream_t stream);
  * are skipped.  PC_ERR_ARG for n < 0 or a null array / entry, PC_ERR_STATE as
  * pc_wait_on_stream; on an error no request of the call was marked complete
  * unless its own wait was already enqueued. */
+/* Round 2: two or more engine-moved DIRECT allreduces in the list (all of one
+ * dtype / op; co-located groups complete in the list) run as ONE batched
+ * engine launch over a device table built on the first call with that exact
+ * list (not capturable, like pc_epoch_all's); other requests take their own
+ * path. */
 int pc_waitall_on_stream(int n, pc_request_t *reqs, pc_stream_t stream);
 /* Host Pready bindings (MPI_Pready / MPI_Pready_range): enqueue a tiny kernel
  * on `stream` that marks partitions [lo, hi] ready. */
