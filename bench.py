@@ -300,6 +300,65 @@ def latency_pair(pc, apps, torch, comms, iters=5000, payload=0, copy=None):
             "frac_of_floor": bare / float(np.percentile(rts, 50))}
 
 
+def c2_bench(pc, apps, torch, S=256 << 20, epochs=20):
+    """C2 at its largest size (256 MiB): block-granularity Kernel Copy from
+    the persistent producer (pc_put_begin + pc_pready_block_put, reading R35;
+    Startall/Waitall control) against the traditional model (the same
+    persistent vector add with no Pready, then a device copy), device time
+    per epoch on one stream.  Parity: the receiver's buffer equals C."""
+    n = S // 4
+    g, cs = pc.local_comms(2, 0)
+    st = torch.cuda.Stream()
+    A, B = torch.randn(n, device="cuda"), torch.randn(n, device="cuda")
+    Cb, R = torch.empty(n, device="cuda"), torch.empty(n, device="cuda")
+    parts = n // 2048
+    snd = pc.psend_init(Cb, parts, 2048, pc.FLOAT32, 1, 13, cs[0])
+    rcv = pc.precv_init(R, parts, 2048, pc.FLOAT32, 0, 13, cs[1])
+    snd.start(st)
+    rcv.start(st)
+    pc.run_ranks([lambda: snd.pbuf_prepare(st), lambda: rcv.pbuf_prepare(st)])
+    sq = snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+    apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK_PUT, sq, st, persistent=True)
+    pc.waitall_on_stream([snd, rcv], st)
+
+    def epoch():
+        pc.epoch_all([snd, rcv], pready=False, stream=st)
+        apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK_PUT, sq, st, persistent=True)
+        pc.waitall_on_stream([snd, rcv], st)
+
+    def trad():
+        apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st, persistent=True)
+        with torch.cuda.stream(st):
+            R.copy_(Cb)
+
+    out = {}
+    for name, fn in (("traditional_us", trad), ("partitioned_us", epoch)):
+        for _ in range(3):
+            fn()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(st)
+        for _ in range(epochs):
+            fn()
+        e1.record(st)
+        torch.cuda.synchronize()
+        out[name] = e0.elapsed_time(e1) / epochs * 1e3
+    R.zero_()
+    epoch()
+    torch.cuda.synchronize()
+    ok = bool(torch.equal(R, Cb)) and snd.error()[0] == 0 and rcv.error()[0] == 0
+    snd.free()
+    rcv.free()
+    for c in cs:
+        c.destroy()
+    g.destroy()
+    out.update({"bytes": S, "partitions": parts, "gran": "block_put (R35), persistent producer", "copy": "inline",
+                "speedup_vs_traditional": out["traditional_us"] / out["partitioned_us"],
+                "goodput_gbs": S / (out["partitioned_us"] / 1e6) / 1e9, "ok": ok,
+                "note": "2 virtual ranks on one B200: both models move the same HBM bytes; tools/sweep.py p2p"})
+    return out
+
+
 def c1_bench(pc, apps, torch, epochs=200):
     """C1: 2 ranks, 1 MiB fp32 produced by a vector-add kernel (8 B/thread,
     1024-thread blocks) with block-granularity Pready: 128 user partitions of
@@ -639,7 +698,8 @@ def run_virtual(args):
     jac = None if args.no_jacobi else jacobi_bench(pc, apps, torch, args)
     log("jacobi done")
     c1 = None if args.no_c1 else c1_bench(pc, apps, torch)
-    log("c1 done")
+    c2p = None if args.no_c1 else c2_bench(pc, apps, torch)
+    log("c1 / c2 done")
     cpu = None if args.no_cpu_baseline else oracle_sample(P=P)
     log("cpu baseline done")
     out = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": 1, "steps": args.steps,
@@ -654,7 +714,8 @@ def run_virtual(args):
                       "l2": f"no flush: working set {3 * P * S >> 20} MiB >> 126 MB L2",
                       "parallelism": f"{P} virtual ranks / 1 GPU"},
            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-           "clocks": clk.summary(), "latency_ns": lat, "jacobi": jac, "c1_p2p": c1, "nccl": None}
+           "clocks": clk.summary(), "latency_ns": lat, "jacobi": jac, "c1_p2p": c1, "c2_p2p_256mib": c2p,
+           "nccl": None}
     print(json.dumps(out), flush=True)
 
 

@@ -4,6 +4,10 @@
  *   PC_DEVICE int  pc_pready      (int partition, pc_prequest_t preq);  any thread
  *   PC_DEVICE int  pc_pready_warp (int partition, pc_prequest_t preq);  warp-collective
  *   PC_DEVICE int  pc_pready_block(int partition, pc_prequest_t preq);  block-collective
+ *   PC_DEVICE int  pc_pready_block_put<T>(int partition, pc_prequest_t preq,
+ *                                         uint64_t idx, const T &v);     block-collective
+ *   PC_DEVICE int  pc_put_begin<T>(pc_prequest_t preq, pc_put_state *st);  block-collective
+ *   PC_DEVICE int  pc_pready_block_put<T>(partition, preq, idx, v, st);     block-collective
  *   PC_DEVICE int  pc_parrived    (pc_prequest_t preq, int partition);
  *   PC_DEVICE int  pc_wait_arrived(pc_prequest_t preq, int partition);
  *   PC_DEVICE int  pc_parrived_warp / pc_wait_arrived_warp(preq, partition);  warp-collective
@@ -36,6 +40,20 @@
  * Returns 0, or a PC_ERR_* code that is also recorded in the sticky error word
  * (bad partition, duplicate Pready detected by counter overshoot).
  *
+ * pc_pready_block_put (MPIX extension, reading R35): pc_pready_block for a
+ * block whose thread k has written element idx_k (of type T, 4/8/16 B) of the
+ * partition and still holds it in registers: the INLINE Kernel Copy assigns
+ * v straight to the receiver ("an assignment statement") instead of
+ * re-reading the partition from L2 after the barrier.  The caller writes its
+ * send buffer as usual and its threads together cover every element of the
+ * partition (idx = UINT64_MAX: this thread holds none).  Every other copy
+ * mode, request kind or alignment falls back to pc_pready_block (the send
+ * buffer already holds the data).  Persistent producers call
+ * pc_put_begin<T>(preq, &st) once per CTA before their loop and then
+ * pc_pready_block_put(partition, preq, idx, v, st): {epoch, ready-to-receive}
+ * is checked once, and each Pready is the raw chain — assign from registers,
+ * barrier, release, flag.
+ *
  * INLINE allreduce (pc_prequest_create(..., PC_COPY_INLINE) on a DIRECT
  * allreduce, reading R33): the Pready that completes a partition on the last
  * rank folds it for every rank.  The fold is compiled into these bindings only
@@ -61,6 +79,11 @@
 typedef struct pc_prequest_s pc_prequest_t;
 
 #define PC_DEVICE __device__ __forceinline__
+/* Paths a Pready rarely takes (a spin on a ready-to-receive word that is not
+ * there yet, an error, a partition of more than 16 B per thread): out of line,
+ * so the common path of a producer capped at 32 registers (two 1024-thread
+ * CTAs per SM) does not spill for them. */
+#define PC_COLD static __device__ __noinline__
 
 #ifndef PC_DEV_ERR_ARG
 #define PC_DEV_ERR_ARG (-1)
@@ -100,6 +123,22 @@ PC_DEVICE uint32_t ld_relaxed_sys(const uint32_t *p) {
   asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+PC_DEVICE uint4 ld_relaxed_gpu_v4(const uint4 *p) {
+  uint4 v;
+  asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p)
+               : "memory");
+  return v;
+}
+PC_DEVICE uint4 ld_relaxed_sys_v4(const uint4 *p) {
+  uint4 v;
+  asm volatile("ld.relaxed.sys.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p)
+               : "memory");
+  return v;
+}
 PC_DEVICE void st_release_sys(uint32_t *p, uint32_t v) {
   asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -124,13 +163,27 @@ PC_DEVICE void red_add_release_gpu(uint32_t *p, uint32_t v) {
 }
 PC_DEVICE void fence_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 PC_DEVICE void fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
-/* Release fence at the scope the request needs: system scope when a peer is
- * another GPU (NVLink), GPU scope when every peer shares this GPU. */
+/* Acquire-release fence at the scope the request needs: system scope when a
+ * peer is another GPU (NVLink), GPU scope when every peer shares this GPU.
+ * Only where the fence must ACQUIRE (relaxed flag loads before it): its
+ * acquire half invalidates the SM's L1 (CCTL.IVALL in the SASS). */
 PC_DEVICE void fence_scope(uint32_t sys) {
   if (sys)
     fence_sys();
   else
     fence_gpu();
+}
+/* Release fence (PTX fence.release): with the strong (relaxed) flag store
+ * that follows it, a release pattern — every memory operation before it (and,
+ * cumulatively, those ordered before it by a barrier) is visible at `scope`
+ * before the flag.  Same MEMBAR as fence.acq_rel without the L1 invalidation
+ * (profiles/r02_c2_floor.jsonl: st.release-style signalling 185 -> 170 us at
+ * 256 MiB).  Every Pready / engine signal releases; none acquires. */
+PC_DEVICE void fence_release(uint32_t sys) {
+  if (sys)
+    asm volatile("fence.release.sys;" ::: "memory");
+  else
+    asm volatile("fence.release.gpu;" ::: "memory");
 }
 PC_DEVICE uint32_t ld_acquire_scope(const uint32_t *p, uint32_t sys) {
   return sys ? ld_acquire_sys(p) : ld_acquire_gpu(p);
@@ -148,7 +201,7 @@ PC_DEVICE uint32_t lane_id() {
 /* wrap-aware "v has reached target" for monotonically increasing u32 words */
 PC_DEVICE bool reached(uint32_t v, uint32_t target) { return (int32_t)(v - target) >= 0; }
 
-PC_DEVICE void set_error(int32_t *err, int32_t code, int32_t part) {
+PC_COLD void set_error(int32_t *err, int32_t code, int32_t part) {
   if (atomicCAS(err, 0, code) == 0) {
     err[1] = part;
     __threadfence_system();
@@ -162,7 +215,7 @@ PC_DEVICE bool aborted(const int32_t *err) { return *(const volatile int32_t *)e
  * thread has set an error (so one failure drains every waiter instead of
  * hanging the device). */
 template <bool SYS>
-PC_DEVICE bool spin_geq(const uint32_t *p, uint32_t target, int32_t *err, uint32_t timeout_ms, int32_t part) {
+PC_COLD bool spin_geq(const uint32_t *p, uint32_t target, int32_t *err, uint32_t timeout_ms, int32_t part) {
   uint32_t v = SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p);
   if (reached(v, target)) return true;
   const uint64_t t0 = globaltimer();
@@ -218,6 +271,10 @@ PC_DEVICE void copy_bytes(uint8_t *dst, const uint8_t *src, uint64_t nbytes, uin
   } else {
     for (uint64_t b = idx; b < nbytes; b += n) dst[b] = src[b];
   }
+}
+
+PC_COLD void copy_bytes_cold(uint8_t *dst, const uint8_t *src, uint64_t nbytes, uint32_t idx, uint32_t n) {
+  copy_bytes(dst, src, nbytes, idx, n);
 }
 
 PC_DEVICE uint32_t epoch_of(const pc_prequest_t &q) { return *(const volatile uint32_t *)q.epoch; }
@@ -336,7 +393,7 @@ PC_DEVICE void publish(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, 
     return;
   }
   if (contribute(q, t, add, e, part)) {
-    fence_scope(q.sys_scope);
+    fence_release(q.sys_scope);
     signal_transport(q, t, e);
     st_relaxed_gpu(q.sent + t, e);
   }
@@ -347,7 +404,7 @@ PC_DEVICE void publish(const pc_prequest_t &q, int t, uint32_t add, uint32_t e, 
  * (cumulative) release of those pushes, so the fence is dropped; g = 1
  * (publish stores the flag directly) and system scope keep it. */
 PC_DEVICE void fence_before_publish(const pc_prequest_t &q) {
-  if (q.agg == 1 || q.sys_scope) fence_scope(q.sys_scope);
+  if (q.agg == 1 || q.sys_scope) fence_release(q.sys_scope);
 }
 
 /* {epoch, rtr[0]} in one acquire at the request's scope (adjacent words). */
@@ -638,7 +695,7 @@ static __device__ __noinline__ void ar_fold(const pc_prequest_t &q, int u, uint3
 /* After the fold (every participant's stores ordered before by a barrier):
  * one cumulative fence, then done[u] = e on every rank. */
 PC_DEVICE void ar_publish(const pc_prequest_t &q, int u, uint32_t e) {
-  fence_scope(q.sys_scope);
+  fence_release(q.sys_scope);
   for (int k = 0; k < q.nranks; ++k) st_relaxed_sys(q.ar_tab->done[k] + u, e);
 }
 
@@ -728,7 +785,7 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
       else
         *reinterpret_cast<uint2 *>(preq.peer_rbuf + off0) = make_uint2(v.x, v.y);
     } else {
-      copy_bytes(preq.peer_rbuf + off0, preq.sbuf + off0, preq.part_bytes, 0, 1);
+      copy_bytes_cold(preq.peer_rbuf + off0, preq.sbuf + off0, preq.part_bytes, 0, 1);
     }
   }
   // One fence per group, not per lane: __syncwarp orders the group's pushes
@@ -834,7 +891,7 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   } else if (small8) {
     if (8ull * lane < preq.part_bytes) reinterpret_cast<uint2 *>(preq.peer_rbuf + off)[lane] = make_uint2(v.x, v.y);
   } else {
-    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, lane, 32);
+    copy_bytes_cold(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, lane, 32);
   }
   __syncwarp(full);  // the warp's pushes, then ONE cumulative fence by lane 0
   if (lane == 0) {
@@ -857,6 +914,24 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
   if (partition < 0 || partition >= preq.partitions) {
     if (tid == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);
     return PC_DEV_ERR_ARG;
+  }
+  // INLINE Kernel Copy of a partition with bytes: thread 0 takes the epoch and
+  // checks the receiver's ready-to-receive word BEFORE the data barrier (it
+  // does not depend on the partition's bytes), so that one barrier publishes
+  // both the data and {e, ok}.  (The previous call's readers of s_e / s_ok all
+  // passed its closing barrier before thread 0 gets here.)
+  const bool inl = preq.kind != PC_KIND_PALLREDUCE && preq.copy == 0 && preq.part_bytes != 0;
+  const bool flag_only = preq.kind != PC_KIND_PALLREDUCE && (preq.copy == 1 || preq.copy == 3 || preq.part_bytes == 0);
+  uint32_t e0 = 0;
+  if (tid == 0) {
+    if (inl) {
+      const uint2 er = epoch_rtr(preq);
+      s_e = er.x;
+      s_ok = 1;
+      if (!reached(er.y, er.x)) s_ok = spin_geq<true>(preq.rtr, er.x, preq.err, preq.timeout_ms, partition);
+    } else if (flag_only) {
+      e0 = epoch_relaxed(preq);  // (ENGINE / HOST / no bytes) its latency hides behind the barrier too
+    }
   }
   __syncthreads();  // the block's data writes are complete
   if (preq.kind == PC_KIND_PALLREDUCE) {
@@ -891,9 +966,9 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
     if (tid == 0) ll_account(preq, t, 1, e, partition);
     return 0;
   }
-  if (preq.copy == 1 || preq.copy == 3 || preq.part_bytes == 0) {  // no bytes for this block to move
+  if (flag_only) {  // no bytes for this block to move
     if (tid == 0) {
-      const uint32_t e = epoch_relaxed(preq);
+      const uint32_t e = e0;
       if (preq.copy == 1 || preq.copy == 3) {
         if (contribute(preq, t, 1, e, partition)) mark_ready(preq, t, e);
       } else {
@@ -903,8 +978,10 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
     return 0;
   }
   // Partitions of at most one 16-B vector per thread (the paper's 8 KiB
-  // block = 1024 threads x 8 B): load the payload BEFORE the {epoch, rtr}
-  // acquire and the barrier, so their latencies overlap.
+  // block = 1024 threads x 8 B): one L2 read-back per thread (the user's
+  // threads wrote the partition in any layout), then its push.
+  const uint32_t e = s_e;
+  if (!s_ok) return PC_DEV_ERR_TIMEOUT;
   const uint64_t off = (uint64_t)partition * preq.part_bytes;
   const uintptr_t al = reinterpret_cast<uintptr_t>(preq.sbuf + off) | reinterpret_cast<uintptr_t>(preq.peer_rbuf + off);
   const bool v16 = preq.part_bytes <= 16ull * nthr && (preq.part_bytes & 15) == 0 && (al & 15) == 0;
@@ -916,27 +993,126 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
     v.x = h.x;
     v.y = h.y;
   }
-  if (tid == 0) {
-    const uint2 er = epoch_rtr(preq);
-    s_e = er.x;
-    s_ok = 1;
-    if (!reached(er.y, er.x)) s_ok = spin_geq<true>(preq.rtr, er.x, preq.err, preq.timeout_ms, partition);
-  }
-  __syncthreads();
-  const uint32_t e = s_e;
-  if (!s_ok) return PC_DEV_ERR_TIMEOUT;
   if (v16) {
     if (16ull * tid < preq.part_bytes) reinterpret_cast<uint4 *>(preq.peer_rbuf + off)[tid] = v;
   } else if (v8) {
     if (8ull * tid < preq.part_bytes) reinterpret_cast<uint2 *>(preq.peer_rbuf + off)[tid] = make_uint2(v.x, v.y);
   } else {
-    copy_bytes(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, tid, nthr);
+    copy_bytes_cold(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, tid, nthr);
   }
   __syncthreads();  // the block's pushes, then ONE cumulative fence by thread 0 (not one per thread)
   if (tid == 0) {
     fence_before_publish(preq);
     publish(preq, t, 1, e, partition);
   }
+  return 0;
+}
+
+/* Block granularity from registers (R35): see the header comment.  Same
+ * chain as the INLINE path of pc_pready_block minus the read-back: thread 0
+ * checks {epoch, ready-to-receive} before the barrier that also orders the
+ * block's send-buffer writes, every thread assigns its element to the
+ * receiver, a second barrier, then ONE release fence and the flag. */
+namespace pc_detail {
+template <typename T>
+PC_DEVICE bool put_eligible(const pc_prequest_t &q) {
+  return q.kind != PC_KIND_PALLREDUCE && q.copy == 0 && q.part_bytes != 0 &&
+         ((reinterpret_cast<uintptr_t>(q.peer_rbuf) | q.part_bytes) & (sizeof(T) - 1)) == 0;
+}
+/* The assignment, barrier, release and flag of a checked epoch. */
+template <typename T>
+PC_DEVICE void put_publish(int partition, const pc_prequest_t &q, uint64_t idx, const T &v, uint32_t e,
+                           uint32_t tid) {
+  if (idx < q.part_bytes / sizeof(T))
+    *reinterpret_cast<T *>(q.peer_rbuf + (uint64_t)partition * q.part_bytes + idx * sizeof(T)) = v;
+  __syncthreads();  // the block's pushes, then ONE cumulative release by thread 0
+  if (tid == 0) {
+    if (q.agg == 1 && !q.xpart) {  // the flag store itself releases (one MEMBAR, no separate fence)
+      if (q.sys_scope)
+        st_release_sys(q.peer_flags + partition, e);
+      else
+        st_release_gpu(q.peer_flags + partition, e);
+      st_relaxed_gpu(q.sent + partition, e);
+    } else {
+      fence_before_publish(q);
+      publish(q, partition / q.agg, 1, e, partition);
+    }
+  }
+}
+}  // namespace pc_detail
+
+template <typename T>
+PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t idx, const T &v) {
+  using namespace pc_detail;
+  static_assert(sizeof(T) == 4 || sizeof(T) == 8 || sizeof(T) == 16, "element of 4, 8 or 16 bytes");
+  if (!put_eligible<T>(preq)) return pc_pready_block(partition, preq);
+  __shared__ uint32_t s_e;
+  __shared__ int s_ok;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  if (partition < 0 || partition >= preq.partitions) {
+    if (tid == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);
+    return PC_DEV_ERR_ARG;
+  }
+  if (tid == 0) {  // (the previous call's readers of s_e / s_ok passed its closing barrier)
+    const uint2 er = epoch_rtr(preq);
+    s_e = er.x;
+    s_ok = 1;
+    if (!reached(er.y, er.x)) s_ok = spin_geq<true>(preq.rtr, er.x, preq.err, preq.timeout_ms, partition);
+  }
+  __syncthreads();  // {e, ok} (the elements themselves are this thread's own registers)
+  const uint32_t e = s_e;
+  if (!s_ok) return PC_DEV_ERR_TIMEOUT;
+  put_publish(partition, preq, idx, v, e, tid);
+  return 0;
+}
+
+/* Persistent producers (R35): the {epoch, ready-to-receive} check once per
+ * CTA per epoch, before its first pc_pready_block_put(..., st).  Both are
+ * fixed for the rest of the epoch once reached, so the later calls carry no
+ * load and no barrier before the assignment — the raw chain (assign from
+ * registers, barrier, release, flag) with nothing out of line in the loop.
+ * Block-collective.  Returns 0 with st->ok = 1; PC_DEV_ERR_ARG with st->ok =
+ * 0 when the request does not take the register path (not an INLINE
+ * partitioned send, or misaligned for T: use pc_pready_block); or
+ * PC_DEV_ERR_TIMEOUT. */
+struct pc_put_state {
+  uint32_t e;   /* the epoch pc_put_begin found */
+  uint32_t ok;  /* 1: checked; the fast pc_pready_block_put may be used */
+};
+
+template <typename T>
+PC_DEVICE int pc_put_begin(pc_prequest_t preq, pc_put_state *st) {
+  using namespace pc_detail;
+  __shared__ uint32_t s_e;
+  __shared__ int s_ok;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  st->e = 0;
+  st->ok = 0;
+  if (!put_eligible<T>(preq)) return PC_DEV_ERR_ARG;
+  if (tid == 0) {
+    const uint2 er = epoch_rtr(preq);
+    s_e = er.x;
+    s_ok = 1;
+    if (!reached(er.y, er.x)) s_ok = spin_geq<true>(preq.rtr, er.x, preq.err, preq.timeout_ms, -4);
+  }
+  __syncthreads();
+  if (!s_ok) return PC_DEV_ERR_TIMEOUT;
+  st->e = s_e;
+  st->ok = 1;
+  return 0;
+}
+
+template <typename T>
+PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t idx, const T &v,
+                                  const pc_put_state &st) {
+  static_assert(sizeof(T) == 4 || sizeof(T) == 8 || sizeof(T) == 16, "element of 4, 8 or 16 bytes");
+  if (!st.ok) return PC_DEV_ERR_ARG;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  if ((unsigned)partition >= (unsigned)preq.partitions) {  // (no out-of-line call in the loop)
+    if (tid == 0 && atomicCAS(preq.err, 0, PC_DEV_ERR_ARG) == 0) preq.err[1] = partition;
+    return PC_DEV_ERR_ARG;
+  }
+  pc_detail::put_publish(partition, preq, idx, v, st.e, tid);
   return 0;
 }
 

@@ -9,6 +9,7 @@ from . import _lib
 from .runtime import Prequest, _ptr, _stream
 
 GRAN_NONE, GRAN_THREAD, GRAN_WARP, GRAN_BLOCK = -1, 0, 1, 2
+GRAN_BLOCK_PUT = 3  # block granularity, Kernel Copy from registers (pc_pready_block_put, R35)
 
 
 def _ok(rc, what):
@@ -16,11 +17,16 @@ def _ok(rc, what):
         raise RuntimeError(f"{what} launch failed ({rc})")
 
 
-def vecadd(A, B, Cout, n: int, gran: int, preq: Prequest | None, stream=None):
+def vecadd(A, B, Cout, n: int, gran: int, preq: Prequest | None, stream=None, persistent: bool = False):
     """C = A + B (fp32, 8 B per thread, 1024-thread blocks) with pc_pready at
-    `gran` (thread: partition = thread, warp: = warp, block: = block)."""
-    _ok(_lib.apps().pcapp_vecadd(_ptr(A), _ptr(B), _ptr(Cout), n, gran, preq.ptr if preq else None,
-                                 _stream(stream)), "vecadd")
+    `gran` (thread: partition = thread, warp: = warp, block: = block;
+    block_put: = block, each thread's result assigned to the peer from its
+    registers).
+    persistent: the same partitions and Pready calls from one CTA per
+    resident slot walking the logical blocks (next block's operands
+    prefetched), instead of one CTA per logical block."""
+    fn = _lib.apps().pcapp_vecadd_persistent if persistent else _lib.apps().pcapp_vecadd
+    _ok(fn(_ptr(A), _ptr(B), _ptr(Cout), n, gran, preq.ptr if preq else None, _stream(stream)), "vecadd")
 
 
 def pready_cost(A, B, Cout, threads: int, gran: int, preq: Prequest, out_ns, stream=None):

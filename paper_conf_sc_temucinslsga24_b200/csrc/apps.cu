@@ -12,6 +12,7 @@
 //   bare_pingpong  the same with raw flags and no library (latency floor)
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "pc_device.cuh"
 
@@ -19,16 +20,19 @@
 #define PCAPP_GRAN_THREAD 0
 #define PCAPP_GRAN_WARP 1
 #define PCAPP_GRAN_BLOCK 2
+#define PCAPP_GRAN_BLOCK_PUT 3  // block granularity, Kernel Copy from registers (pc_pready_block_put)
 
 namespace {
 
-__global__ void __launch_bounds__(1024) vecadd_kernel(const float2 *__restrict__ A, const float2 *__restrict__ B,
-                                                      float2 *__restrict__ C, int64_t n2, int gran,
-                                                      pc_prequest_t preq) {
+template <int MINB, int gran>
+__global__ void __launch_bounds__(1024, MINB) vecadd_kernel(const float2 *__restrict__ A, const float2 *__restrict__ B,
+                                                            float2 *__restrict__ C, int64_t n2, pc_prequest_t preq) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  float2 c = make_float2(0.f, 0.f);
   if (i < n2) {
     const float2 a = A[i], b = B[i];
-    C[i] = make_float2(a.x + b.x, a.y + b.y);
+    c = make_float2(a.x + b.x, a.y + b.y);
+    C[i] = c;
   }
   if (gran == PCAPP_GRAN_THREAD) {
     if (i < n2) pc_pready((int)i, preq);
@@ -36,6 +40,157 @@ __global__ void __launch_bounds__(1024) vecadd_kernel(const float2 *__restrict__
     pc_pready_warp((int)(i >> 5), preq);
   } else if (gran == PCAPP_GRAN_BLOCK) {
     pc_pready_block((int)blockIdx.x, preq);
+  } else if (gran == PCAPP_GRAN_BLOCK_PUT) {
+    pc_pready_block_put((int)blockIdx.x, preq, i < n2 ? (uint64_t)threadIdx.x : ~0ull, c);
+  }
+}
+
+// The same C = A + B with the same partitions (logical block p = 1024 threads
+// x 8 B, warp p*32 + w, thread i) and the same Pready calls, as a persistent
+// kernel: one 1024-thread CTA per resident slot (2 per SM) walks the logical
+// blocks p = blockIdx.x, + gridDim.x, ...  The operands are staged by TMA
+// bulk copies (cp.async.bulk, one 8 KiB tile of A and of B per logical block)
+// into a ring of kStages shared-memory stages, each completing on its own
+// mbarrier, kStages - 1 logical blocks ahead — so the HBM loads overlap the
+// Pready chain (barrier, push, the release thread 0 issues before the flag)
+// without holding registers (a register prefetch spilled at the 32-register
+// budget of 2 CTAs per SM, and the spill store waited for the load).  A warp
+// arrives on the stage's "empty" mbarrier once it has read it; thread 32 (not
+// thread 0, whose Pready releases: a MEMBAR issued by the thread that has
+// bulk copies in flight waited for them, 305 -> xx us at 256 MiB) refills the
+// stage after its own Pready.  A ragged last tile moves its 16-B-aligned part
+// by TMA and the rest by plain loads.
+constexpr int kStages = 4;
+constexpr int kTile = 1024;  // float2 per logical block
+constexpr size_t kStagedSmem = (size_t)2 * kStages * kTile * sizeof(float2) + 2 * kStages * sizeof(uint64_t);
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t n) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(n) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
+  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n}" ::"r"(smem_u32(b)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *b) {
+  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.shared::cta.b64 st, [%0];\n}" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W_%=;\n}" ::"r"(
+          smem_u32(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *b) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(b))
+               : "memory");
+}
+
+template <int gran>
+__global__ void __launch_bounds__(1024, 2) vecadd_persistent_kernel(const float2 *__restrict__ A,
+                                                                    const float2 *__restrict__ B,
+                                                                    float2 *__restrict__ C, int64_t n2,
+                                                                    int64_t nblk, pc_prequest_t preq) {
+  // 32-bit loop state (the launcher guarantees n2 < 2^31) and smem offsets
+  // from one base: the loop carries few registers at the 32-register budget.
+  extern __shared__ __align__(128) uint8_t smem[];
+  constexpr uint32_t kTileBytes = kTile * sizeof(float2);
+  constexpr uint32_t kFull = 2 * kStages * kTileBytes, kEmpty = kFull + kStages * 8;
+  const uint32_t tid = threadIdx.x, base = smem_u32(smem);
+  const int N2 = (int)n2, NB = (int)nblk, G = (int)gridDim.x;
+  const int T = (NB - (int)blockIdx.x + G - 1) / G;  // logical blocks of this CTA
+  constexpr uint32_t kIssuer = 32;  // the thread that issues the bulk copies
+  auto bulk_bytes = [&](int p) -> uint32_t {
+    const int rem = N2 - p * kTile;
+    return (uint32_t)((rem < kTile ? rem : kTile) * 8) & ~15u;
+  };
+  auto issue = [&](int k) {  // thread kIssuer: tile k of this CTA into stage k % kStages
+    const int p = (int)blockIdx.x + k * G;
+    const uint32_t s = (uint32_t)(k % kStages), by = bulk_bytes(p);
+    uint64_t *f = reinterpret_cast<uint64_t *>(smem + kFull) + s;
+    mbar_expect_tx(f, 2 * by);
+    if (by) {
+      bulk_g2s(smem + s * kTileBytes, A + (int64_t)p * kTile, by, f);
+      bulk_g2s(smem + (kStages + s) * kTileBytes, B + (int64_t)p * kTile, by, f);
+    }
+  };
+  if (tid == 0) {
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(reinterpret_cast<uint64_t *>(smem + kFull) + s, 1);
+      mbar_init(reinterpret_cast<uint64_t *>(smem + kEmpty) + s, 1024 / 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (tid == kIssuer)
+    for (int k = 0; k < kStages && k < T; ++k) issue(k);
+  for (int k = 0; k < T; ++k) {
+    const int p = (int)blockIdx.x + k * G;
+    const uint32_t s = (uint32_t)(k % kStages), par = (uint32_t)(k / kStages) & 1u;
+    const int i = p * kTile + (int)tid;
+    mbar_wait(reinterpret_cast<uint64_t *>(smem + kFull) + s, par);
+    float2 c = make_float2(0.f, 0.f);
+    if (8u * tid + 8u <= bulk_bytes(p)) {
+      float2 a, b;
+      asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(a.x), "=f"(a.y) : "r"(base + s * kTileBytes + 8u * tid));
+      asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];"
+                   : "=f"(b.x), "=f"(b.y)
+                   : "r"(base + (kStages + s) * kTileBytes + 8u * tid));
+      c = make_float2(a.x + b.x, a.y + b.y);
+    } else if (i < N2) {  // ragged tail beyond the bulk copy
+      const float2 a = __ldcs(A + i), b = __ldcs(B + i);
+      c = make_float2(a.x + b.x, a.y + b.y);
+    }
+    __syncwarp();
+    if ((tid & 31) == 0) mbar_arrive(reinterpret_cast<uint64_t *>(smem + kEmpty) + s);
+    if (i < N2) C[i] = c;
+    if (gran == PCAPP_GRAN_THREAD) {
+      if (i < N2) pc_pready(i, preq);
+    } else if (gran == PCAPP_GRAN_WARP) {
+      pc_pready_warp(i >> 5, preq);
+    } else if (gran == PCAPP_GRAN_BLOCK) {
+      pc_pready_block(p, preq);
+    }
+    if (tid == kIssuer && k + kStages < T) {  // every warp has read stage s: refill it
+      mbar_wait(reinterpret_cast<uint64_t *>(smem + kEmpty) + s, par);
+      issue(k + kStages);
+    }
+  }
+}
+
+// block_put from a persistent producer (R35): the paper's 8 KiB logical
+// blocks, 1024 threads x 8 B, with pc_put_begin once per CTA and the
+// register path of pc_pready_block_put per logical block — nothing out of
+// line in the loop, so the operands of the NEXT logical block are prefetched
+// into registers (no spill at 32 registers) and their HBM latency overlaps the
+// Pready chain of this one (assign, barrier, thread 0's release + flag).
+__global__ void __launch_bounds__(1024, 2) vecadd_put_persistent_kernel(const float2 *__restrict__ A,
+                                                                        const float2 *__restrict__ B,
+                                                                        float2 *__restrict__ C, int n2, int nblk,
+                                                                        pc_prequest_t preq) {
+  pc_put_state st;
+  if (pc_put_begin<float2>(preq, &st) != 0) return;  // (the launcher checked eligibility; timeout is recorded)
+  const int G = gridDim.x;
+  int p = blockIdx.x;
+  float2 a = make_float2(0.f, 0.f), b = a;
+  int i = p * 1024 + (int)threadIdx.x;
+  if (i < n2) {
+    a = __ldcs(A + i);
+    b = __ldcs(B + i);
+  }
+  for (; p < nblk; p += G, i += G * 1024) {
+    const float2 c = make_float2(a.x + b.x, a.y + b.y);
+    const int in = i + G * 1024;
+    if (in < n2) {
+      a = __ldcs(A + in);
+      b = __ldcs(B + in);
+    }
+    if (i < n2) C[i] = c;
+    pc_pready_block_put(p, preq, i < n2 ? (uint64_t)threadIdx.x : ~0ull, c, st);
   }
 }
 
@@ -377,17 +532,93 @@ __global__ void bare_pingpong_kernel(uint32_t *my_flag, uint32_t *peer_flag, int
 
 }  // namespace
 
+// Resident 1024-thread vecadd CTAs per SM the launch asks ptxas for (1: up to
+// 64 registers per thread; 2: 32).  PCAPP_VECADD_MINB=1|2, default 2.
+int minb() {
+  static int v = 0;
+  if (!v) {
+    const char *e = getenv("PCAPP_VECADD_MINB");
+    v = (e && e[0] == '1') ? 1 : 2;
+  }
+  return v;
+}
+
+// One instantiation per (CTAs per SM, granularity): a launch carries only the
+// Pready path it calls, so the 32-register budget of 2 CTAs per SM is spent on
+// that path alone.
+using VecaddFn = void (*)(const float2 *, const float2 *, float2 *, int64_t, pc_prequest_t);
+using VecaddPersFn = void (*)(const float2 *, const float2 *, float2 *, int64_t, int64_t, pc_prequest_t);
+template <int MINB>
+VecaddFn vecadd_fn(int gran) {
+  switch (gran) {
+    case PCAPP_GRAN_THREAD: return vecadd_kernel<MINB, PCAPP_GRAN_THREAD>;
+    case PCAPP_GRAN_WARP: return vecadd_kernel<MINB, PCAPP_GRAN_WARP>;
+    case PCAPP_GRAN_BLOCK: return vecadd_kernel<MINB, PCAPP_GRAN_BLOCK>;
+    case PCAPP_GRAN_BLOCK_PUT: return vecadd_kernel<MINB, PCAPP_GRAN_BLOCK_PUT>;
+    default: return vecadd_kernel<MINB, PCAPP_GRAN_NONE>;
+  }
+}
+VecaddPersFn vecadd_pers_fn(int gran) {
+  switch (gran) {
+    case PCAPP_GRAN_THREAD: return vecadd_persistent_kernel<PCAPP_GRAN_THREAD>;
+    case PCAPP_GRAN_WARP: return vecadd_persistent_kernel<PCAPP_GRAN_WARP>;
+    case PCAPP_GRAN_BLOCK: return vecadd_persistent_kernel<PCAPP_GRAN_BLOCK>;
+    default: return vecadd_persistent_kernel<PCAPP_GRAN_NONE>;
+  }
+}
+
 extern "C" {
 
 int pcapp_vecadd(const float *A, const float *B, float *C, int64_t n, int gran, const pc_prequest_t *preq,
                  cudaStream_t s) {
-  if (n % 2) return -1;
+  if (n % 2 || gran < PCAPP_GRAN_NONE || gran > PCAPP_GRAN_BLOCK_PUT) return -1;
   const int64_t n2 = n / 2;
   const int64_t blocks = (n2 + 1023) / 1024;
   pc_prequest_t q{};
   if (preq) q = *preq;
   if (gran != PCAPP_GRAN_NONE && !preq) return -1;
-  vecadd_kernel<<<(unsigned)blocks, 1024, 0, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, gran, q);
+  if (blocks < 1) return 0;
+  const VecaddFn f = minb() == 2 ? vecadd_fn<2>(gran) : vecadd_fn<1>(gran);
+  f<<<(unsigned)blocks, 1024, 0, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, q);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_vecadd_persistent(const float *A, const float *B, float *C, int64_t n, int gran, const pc_prequest_t *preq,
+                            cudaStream_t s) {
+  if (n % 2 || gran < PCAPP_GRAN_NONE || gran > PCAPP_GRAN_BLOCK_PUT) return -1;
+  if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(B)) & 15) return -1;  // TMA: 16-B sources
+  const int64_t n2 = n / 2;
+  if (n2 + kTile >= (1ll << 31)) return -1;  // 32-bit element indices
+  const int64_t nblk = (n2 + kTile - 1) / kTile;
+  pc_prequest_t q{};
+  if (preq) q = *preq;
+  if (gran != PCAPP_GRAN_NONE && !preq) return -1;
+  if (nblk < 1) return 0;
+  const bool put_ok = q.kind != PC_KIND_PALLREDUCE && q.copy == 0 && q.part_bytes != 0 &&
+                      ((reinterpret_cast<uintptr_t>(q.peer_rbuf) | q.part_bytes) & 7) == 0;
+  if (gran == PCAPP_GRAN_BLOCK_PUT && put_ok) {
+    int dev = 0, sms = 0, per = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess ||
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, vecadd_put_persistent_kernel, 1024, 0) != cudaSuccess ||
+        per < 1)
+      return -2;
+    const int64_t grid = nblk < (int64_t)sms * per ? nblk : (int64_t)sms * per;
+    vecadd_put_persistent_kernel<<<(unsigned)grid, 1024, 0, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C,
+                                                                 (int)n2, (int)nblk, q);
+    return cudaGetLastError() == cudaSuccess ? 0 : -2;
+  }
+  if (gran == PCAPP_GRAN_BLOCK_PUT) gran = PCAPP_GRAN_BLOCK;  // same partitions: the send buffer holds the data
+  const VecaddPersFn f = vecadd_pers_fn(gran);
+  int dev = 0, sms = 0, per = 0;  // resident 1024-thread CTAs of this instantiation
+  if (cudaGetDevice(&dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
+      cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kStagedSmem) != cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, 1024, kStagedSmem) != cudaSuccess || per < 1)
+    return -2;
+  const int64_t slots = (int64_t)sms * per;
+  const int64_t grid = nblk < slots ? nblk : slots;
+  f<<<(unsigned)grid, 1024, kStagedSmem, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, nblk, q);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -92,7 +92,7 @@ __device__ __forceinline__ bool warp_wait(const uint32_t *p, uint32_t target, in
 // (system scope for a peer on another GPU), then lane 0 stores the epoch into
 // the consumer's flag.
 __device__ __forceinline__ void warp_signal(uint32_t *flag, uint32_t e, bool sys) {
-  fence_scope(sys);
+  fence_release(sys);
   __syncwarp();
   if ((threadIdx.x & 31) == 0) st_relaxed_sys(flag, e);
 }
@@ -871,7 +871,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
                           a.sendbuf + (base + lo) * es, (hi - lo) * es);
             }
           }
-          fence_scope(a.sys);
+          fence_release(a.sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
             for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 0) * a.ns + s, 1, a.sys);
@@ -899,7 +899,7 @@ __device__ __forceinline__ void direct_body(const DirectArgs &a, const int gw, c
             else  // MAXP < 8: fewer sources, FV * 8 / MAXP vectors per operand in flight, same registers
               warp_fold_pull<DT, OP, true, FV * kMaxDirect / MAXP, PF, MAXP>(a, base + lo, base + lo, hi - lo);
           }
-          fence_scope(a.sys);
+          fence_release(a.sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
             for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
@@ -1124,7 +1124,7 @@ __device__ __forceinline__ void direct_batch_body(const DirectBatchArgs b, const
         }
         progressed = true;
         if (i == 0) {
-          fence_scope(sys);
+          fence_release(sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
             for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 0) * ns + s, 1, sys);
@@ -1148,7 +1148,7 @@ __device__ __forceinline__ void direct_batch_body(const DirectBatchArgs b, const
             }
             warp_fold_ptrs<DT, OP, FV>(S, D, P, hi - lo);
           }
-          fence_scope(sys);
+          fence_release(sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
             for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * ns + s, 1, sys);
@@ -1243,7 +1243,7 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
           if (!warp_poll(cnt_u, e, a.sys)) continue;
           const int64_t off = ((int64_t)u * a.count + lo) * es;
           if (n) warp_copy(a.recvbuf + off, a.p_recvbuf[0] + off, n * es);
-          fence_scope(a.sys);  // our reads of the root's slice are done before it may reuse it
+          fence_release(a.sys);  // our reads of the root's slice are done before it may reuse it
           __syncwarp();
           if ((threadIdx.x & 31) == 0) red_add_scope(a.p_cnt[0] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
           finished = true;
@@ -1262,7 +1262,7 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
           if (phi > plo)
             warp_copy_multi<kMaxDirect - 1, 8>(a.recvbuf, a.p_recvbuf, P - 1, off, a.p_recvbuf[jr] + off,
                                                (phi - plo) * es, jr);
-          fence_scope(a.sys);  // my reads of the root and my stores to the receivers, then the signals
+          fence_release(a.sys);  // my reads of the root and my stores to the receivers, then the signals
           __syncwarp();
           if ((threadIdx.x & 31) == 0)
             for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);
@@ -1279,7 +1279,7 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
             if (n) warp_copy_multi<kMaxDirect - 1>(a.recvbuf, a.p_recvbuf, P - 1, doff, a.sendbuf + off, n * es);
           }
           // (broadcast root: nothing to copy — the peers PULL the slice)
-          fence_scope(a.sys);
+          fence_release(a.sys);
           __syncwarp();
           if ((threadIdx.x & 31) == 0) {
             for (int j = 0; j < P - 1; ++j) {
@@ -1298,7 +1298,7 @@ __device__ __forceinline__ void coll_body(const CollArgs &a, const int gw, const
             if (n)
               warp_fold_pull<DT, OP, false, PC_DIRECT_FV * kMaxDirect / MAXP, false, MAXP>(
                   a, ((int64_t)u * P + r) * a.count + lo, (int64_t)u * a.count + lo, n);
-            fence_scope(a.sys);
+            fence_release(a.sys);
             __syncwarp();
             if ((threadIdx.x & 31) == 0)
               for (int j = 0; j < P - 1; ++j) red_add_scope(a.p_cnt[j] + ((int64_t)u * 2 + 1) * a.ns + s, 1, a.sys);

@@ -2178,7 +2178,7 @@ int pc_waitall_on_stream(int n, pc_request_t *reqs, pc_stream_t stream) {
     int want[kMaxWaitAll], total = 0;
     for (size_t k = g0; k < fused.size() && a.n < kMaxWaitAll; ++k) {
       fill_prequest(fused[k], &a.q[a.n]);
-      want[a.n] = fused[k]->kind == PC_KIND_PSEND ? 1 : recv_wait_blocks(a.q[a.n]);
+      want[a.n] = fused[k]->kind == PC_KIND_PSEND ? wait_words_blocks(fused[k]->ntransport) : recv_wait_blocks(a.q[a.n]);
       total += want[a.n];
       ++a.n;
     }

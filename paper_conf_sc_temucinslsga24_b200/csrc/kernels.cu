@@ -57,14 +57,14 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
         const uint64_t n = slo < len ? min(a.slice_bytes, len - slo) : 0;
         if (n) warp_copy(a.peer_rbuf + off + slo, a.sbuf + off + slo, (int64_t)n);
       }
-      fence_scope(a.sys);  // one cumulative fence for every copy of this sweep
+      fence_release(a.sys);  // one cumulative fence for every copy of this sweep
       __syncwarp();
       if (lane == 0) {
         for (int j = 0; j < kMaxActive; ++j) {
           if (!((ready >> j) & 1u)) continue;
           const int t = (gw + (j0 + j) * W) / a.ns;
           const bool last = a.ns == 1 || atom_add_acq_rel_gpu(a.donecnt + t, 1) + 1 == e * (uint32_t)a.ns;
-          if (last && a.ns > 1) fence_scope(a.sys);  // the other slices' copies (acquired by the add) too
+          if (last && a.ns > 1) fence_release(a.sys);  // the other slices' copies (acquired by the add) too
           if (last) {
             signal_transport(a.peer_flags, t, e, a.xpart, a.partitions, a.agg, a.part_bytes, a.peer_part_bytes);
             st_relaxed_gpu(a.sent + t, e);  // (after the fence: the copies are delivered)
@@ -77,15 +77,47 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
   }
 }
 
+// Bulk wait until words[0 .. n-1] have all reached `target` (participant idx
+// of nthr, grid-stride): relaxed 16-B loads of 4 words each — one round trip
+// for the whole range once everything has arrived, instead of one dependent
+// acquire per word — a bounded acquire spin only on words still behind, then
+// one acquire fence per participant for the words it saw relaxed (the
+// "ld.relaxed; fence" acquire pattern).  Words is 4-B aligned.
+__device__ __forceinline__ bool wait_words_range(const uint32_t *w, int n, uint32_t target, int sys, int32_t *err,
+                                                 uint32_t tmo, uint32_t idx, uint32_t nthr) {
+  int head = (int)(((16u - (uint32_t)(reinterpret_cast<uintptr_t>(w) & 15u)) & 15u) >> 2);
+  if (head > n) head = n;
+  auto spin = [&](int i) {
+    return sys ? spin_geq<true>(w + i, target, err, tmo, i) : spin_geq<false>(w + i, target, err, tmo, i);
+  };
+  for (int i = (int)idx; i < head; i += (int)nthr)
+    if (!spin(i)) return false;
+  const int nv = (n - head) >> 2;
+  const uint4 *v = reinterpret_cast<const uint4 *>(w + head);
+  bool relaxed = false;
+  for (int k = (int)idx; k < nv; k += (int)nthr) {
+    const uint4 x = sys ? ld_relaxed_sys_v4(v + k) : ld_relaxed_gpu_v4(v + k);
+    relaxed = true;
+    const uint32_t xs[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (!reached(xs[j], target) && !spin(head + 4 * k + j)) return false;
+  }
+  for (int i = head + 4 * nv + (int)idx; i < n; i += (int)nthr)
+    if (!spin(i)) return false;
+  if (relaxed) fence_scope(sys);
+  return true;
+}
+
 __device__ __forceinline__ void wait_words_body(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul,
                                                 const uint32_t *layout, int partitions, int32_t *err, uint32_t tmo,
-                                                int sys, const uint32_t *rtr) {
+                                                int sys, const uint32_t *rtr, uint32_t bid, uint32_t nb) {
   __shared__ int s_n;
   const uint32_t target = *(const volatile uint32_t *)epoch * mul;
   // LL sender: its epoch completes only once the receiver posted ready-to-
   // receive for this epoch (acquire), i.e. finished reading epoch e-1's lines,
   // whose parity epoch e+1 reuses (ll_push, R29)
-  if (rtr && threadIdx.x == 32) spin_geq<true>(rtr, target, err, tmo, -3);
+  if (rtr && bid == 0 && threadIdx.x == 32) spin_geq<true>(rtr, target, err, tmo, -3);
   if (threadIdx.x == 0) {
     int nn = n;
     if (layout) {
@@ -105,17 +137,13 @@ __device__ __forceinline__ void wait_words_body(const uint32_t *words, int n, co
     s_n = nn;
   }
   __syncthreads();
-  const int nn = s_n;
-  for (int i = threadIdx.x; i < nn; i += blockDim.x) {
-    bool ok = sys ? spin_geq<true>(words + i, target, err, tmo, i) : spin_geq<false>(words + i, target, err, tmo, i);
-    if (!ok) break;
-  }
+  wait_words_range(words, s_n, target, sys, err, tmo, bid * blockDim.x + threadIdx.x, nb * blockDim.x);
 }
 
 __global__ void wait_words_kernel(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul,
                                   const uint32_t *layout, int partitions, int32_t *err, uint32_t tmo, int sys,
                                   const uint32_t *rtr) {
-  wait_words_body(words, n, epoch, mul, layout, partitions, err, tmo, sys, rtr);
+  wait_words_body(words, n, epoch, mul, layout, partitions, err, tmo, sys, rtr, blockIdx.x, gridDim.x);
 }
 
 // Receive-side MPI_Wait / MPI_Test for a request whose sender may push LL
@@ -179,12 +207,16 @@ __device__ __forceinline__ void recv_wait_body(const pc_prequest_t &q, int32_t *
     }
     return;
   }
-  if (bid != 0) return;
   // equal partitionings: one flag per send transport partition (target e);
   // different ones (R30): one counter per receive partition (e * overlaps)
   const bool xp = (g & PC_LAYOUT_XP) != 0;
   const int nt = xp ? q.partitions : (q.partitions + (int)g - 1) / (int)g;
-  for (int i = threadIdx.x; i < nt; i += blockDim.x) {
+  if (!xp && !pending) {  // MPI_Wait, uniform target: the bulk wait over every block
+    wait_words_range(q.flags, nt, e, q.sys_scope, q.err, q.timeout_ms, bid * blockDim.x + threadIdx.x,
+                     nb * blockDim.x);
+    return;
+  }
+  for (int i = (int)(bid * blockDim.x + threadIdx.x); i < nt; i += (int)(nb * blockDim.x)) {
     const uint32_t target = xp ? e * xp_need((uint64_t)i, q.part_bytes, g & PC_LAYOUT_G, q.peer_part_bytes) : e;
     if (pending) {
       if (!reached(ld_acquire_scope(q.flags + i, q.sys_scope), target)) atomicAdd(pending, 1);
@@ -206,9 +238,8 @@ __global__ void wait_all_kernel(WaitAllArgs a) {
   const pc_prequest_t &q = a.q[k];
   const uint32_t bid = blockIdx.x - a.block_start[k], nb = a.block_start[k + 1] - a.block_start[k];
   if (q.kind == PC_KIND_PSEND) {
-    if (bid == 0)
-      wait_words_body(q.sent, q.ntransport, q.epoch, 1, nullptr, q.partitions, q.err, q.timeout_ms, 0,
-                      q.copy == PC_COPY_LL ? q.rtr : nullptr);
+    wait_words_body(q.sent, q.ntransport, q.epoch, 1, nullptr, q.partitions, q.err, q.timeout_ms, 0,
+                    q.copy == PC_COPY_LL ? q.rtr : nullptr, bid, nb);
   } else {
     recv_wait_body(q, nullptr, bid, nb);
   }
@@ -325,11 +356,11 @@ __global__ void __launch_bounds__(1024) epoch_batch_kernel(EpochBatchArgs a) {
   for (int k = t; k < a.nrtr; k += blockDim.x) {
     const RtrEnt r = a.rtr[k];
     if (r.sys) {
-      if (!fsys) fence_sys();
+      if (!fsys) fence_release(1);
       fsys = true;
       st_relaxed_sys(r.dst, epoch(r.req));
     } else {
-      if (!fgpu && !fsys) fence_gpu();
+      if (!fgpu && !fsys) fence_release(0);
       fgpu = true;
       st_relaxed_gpu(r.dst, epoch(r.req));
     }
@@ -454,14 +485,23 @@ int launch_p2p_engine(const P2pEngineArgs &a, int warps, cudaStream_t s) {
 int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint32_t mul, const uint32_t *layout,
                       int partitions, int32_t *err, uint32_t timeout_ms, cudaStream_t s, bool sys,
                       const uint32_t *rtr) {
-  wait_words_kernel<<<1, 256, 0, s>>>(words, n, epoch, mul, layout, partitions, err, timeout_ms, sys ? 1 : 0, rtr);
+  // (a receiver's n is an upper bound: the sender's g may aggregate)
+  wait_words_kernel<<<wait_words_blocks(n), 256, 0, s>>>(words, n, epoch, mul, layout, partitions, err, timeout_ms,
+                                                         sys ? 1 : 0, rtr);
   g_launches++;
   PC_CUDA(cudaGetLastError());
   return 0;
 }
 
+// Flag words of a request: at most one 256-thread block per 1024 words, at
+// most one block per SM (spinning blocks never fill the GPU: DESIGN.md §7).
+int wait_words_blocks(int n) {
+  const int b = (n + 1023) / 1024;
+  return b < 1 ? 1 : (b > 148 ? 148 : b);
+}
+
 int recv_wait_blocks(const pc_prequest_t &q) {
-  int blocks = 1;
+  int blocks = wait_words_blocks(q.partitions);
   if (q.ll_lines) {
     const int64_t lines = (int64_t)q.partitions * q.ll_lines;
     blocks = (int)((lines + 255) / 256);

@@ -511,6 +511,7 @@ struct WaitAllArgs {
   pc_prequest_t q[kMaxWaitAll];
 };
 int recv_wait_blocks(const pc_prequest_t &q);
+int wait_words_blocks(int n);
 int launch_wait_all(const WaitAllArgs &a, cudaStream_t s);
 int engine_occupancy_ctas_per_sm(int *ctas);
 int direct_occupancy_ctas_per_sm(int *ctas);

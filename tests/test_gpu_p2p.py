@@ -15,11 +15,13 @@ from gpu_util import comms, first_prepare
 pytestmark = pytest.mark.gpu
 SEED = synth.BASE_SEED
 
-GRAN_ELEMS = {apps.GRAN_THREAD: 2, apps.GRAN_WARP: 64, apps.GRAN_BLOCK: 2048}  # 8 B / 256 B / 8 KiB
+GRAN_ELEMS = {apps.GRAN_THREAD: 2, apps.GRAN_WARP: 64, apps.GRAN_BLOCK: 2048,
+              apps.GRAN_BLOCK_PUT: 2048}  # 8 B / 256 B / 8 KiB / 8 KiB
 
 
-def run_vecadd(n, gran, agg, copy, epochs=3, check_in_kernel=True):
-    """C1/C2 shape: sender computes C = A + B and Preadies from the kernel."""
+def run_vecadd(n, gran, agg, copy, epochs=3, check_in_kernel=True, persistent=False):
+    """C1/C2 shape: sender computes C = A + B and Preadies from the kernel
+    (persistent: the same partitions from one CTA per resident slot)."""
     count = GRAN_ELEMS[gran]
     partitions = n // count
     with comms(2) as cs:
@@ -43,8 +45,8 @@ def run_vecadd(n, gran, agg, copy, epochs=3, check_in_kernel=True):
             rcv.start(s1)
             if e == 0:
                 first_prepare([[snd], [rcv]], [s0, s1])
-                sq = snd.prequest_create(gran, agg, copy)
-                rq = rcv.prequest_create(gran, 1, pc.COPY_INLINE)
+                sq = snd.prequest_create(min(gran, apps.GRAN_BLOCK), agg, copy)
+                rq = rcv.prequest_create(min(gran, apps.GRAN_BLOCK), 1, pc.COPY_INLINE)
             else:
                 rcv.pbuf_prepare(s1)
                 snd.pbuf_prepare(s0)
@@ -52,7 +54,7 @@ def run_vecadd(n, gran, agg, copy, epochs=3, check_in_kernel=True):
             # queues, so a spinning consumer must never be enqueued before the
             # work it waits for.  The sender's wait launches its ENGINE (lazy
             # launch), so it precedes the in-kernel Parrived consumer.
-            apps.vecadd(A, B, Cb, n, gran, sq, s0)
+            apps.vecadd(A, B, Cb, n, gran, sq, s0, persistent=persistent)
             snd.wait_on_stream(s0)
             if check_in_kernel:
                 apps.check_recv(rq, R, out, partitions, count * 4, status, blocks=64, stream=s1)
@@ -90,6 +92,31 @@ def test_c2_block_256mib(copy, agg):
     128 = 1 MiB transport partitions): byte-exact vs O1 over 2 epochs with
     seeded inputs, in-kernel Parrived consumer included."""
     run_vecadd(1 << 26, apps.GRAN_BLOCK, agg, copy, epochs=2)
+
+
+@pytest.mark.parametrize("gran", [apps.GRAN_BLOCK, apps.GRAN_BLOCK_PUT])
+@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE])
+def test_c2_persistent_256mib(gran, copy):
+    """C2 at 256 MiB from the persistent producer (296 CTAs walking 32768
+    logical blocks), block Pready with read-back and from registers
+    (pc_pready_block_put, R35): byte-exact vs O1 over 2 epochs."""
+    run_vecadd(1 << 26, gran, 1, copy, epochs=2, persistent=True)
+
+
+@pytest.mark.parametrize("persistent", [False, True])
+@pytest.mark.parametrize("gran", [apps.GRAN_THREAD, apps.GRAN_WARP, apps.GRAN_BLOCK, apps.GRAN_BLOCK_PUT])
+@pytest.mark.parametrize("agg_kind", ["none", "odd", "all"])
+@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE, pc.COPY_LL])
+def test_producer_shapes(persistent, gran, agg_kind, copy):
+    """Every granularity from both producer shapes, over more logical blocks
+    (1000) than resident CTAs so persistent CTAs loop; block_put falls back to
+    pc_pready_block for ENGINE / LL."""
+    n = 2048 * 1000
+    partitions = n // GRAN_ELEMS[gran]
+    agg = {"none": 1, "odd": max(1, partitions // 3 - 1), "all": partitions}[agg_kind]
+    if copy == pc.COPY_LL and agg * GRAN_ELEMS[gran] * 4 > 1024:
+        pytest.skip("LL: transport partitions of at most 1 KiB")
+    run_vecadd(n, gran, agg, copy, epochs=2, persistent=persistent)
 
 
 def test_c1_block_agg16_inline():

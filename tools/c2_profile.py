@@ -1,4 +1,5 @@
 """C2 profiling driver: vecadd (8 B/thread, 1024-thread blocks) at 256 MiB
+[S copies gran persistent]
 alone (GRAN_NONE) and with block-granularity Pready (INLINE / ENGINE, g=1)
 into a 2-rank partitioned send on one B200.  Run under ncu -k regex:vecadd."""
 import os
@@ -13,13 +14,15 @@ from paper_conf_sc_temucinslsga24_b200 import apps  # noqa: E402
 
 S = int(sys.argv[1]) if len(sys.argv) > 1 else 256 << 20
 copies = [int(c) for c in sys.argv[2].split(",")] if len(sys.argv) > 2 else [pc.COPY_INLINE]
+gran = int(sys.argv[3]) if len(sys.argv) > 3 else apps.GRAN_BLOCK  # 3 = block_put (R35)
+pers = len(sys.argv) > 4 and sys.argv[4] == "persistent"
 n = S // 4
 g2, cs = pc.local_comms(2, 0)
 st = torch.cuda.Stream()
 A, B = torch.randn(n, device="cuda"), torch.randn(n, device="cuda")
 Cb, R = torch.empty(n, device="cuda"), torch.empty(n, device="cuda")
 for _ in range(2):
-    apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st)
+    apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st, persistent=pers)
 torch.cuda.synchronize()
 for copy in copies:
     snd = pc.psend_init(Cb, n // 2048, 2048, pc.FLOAT32, 1, 5 + copy, cs[0])
@@ -33,7 +36,7 @@ for copy in copies:
         else:
             rcv.pbuf_prepare(st)
             snd.pbuf_prepare(st)
-        apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK, sq, st)
+        apps.vecadd(A, B, Cb, n, gran, sq, st, persistent=pers)
         snd.wait_on_stream(st)
         rcv.wait_on_stream(st)
     torch.cuda.synchronize()

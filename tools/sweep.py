@@ -342,12 +342,15 @@ def sweep_p2p(args):
     aggregation g, INLINE vs ENGINE; goodput = bytes / (kernel + comm) time."""
     g2, cs = pc.local_comms(2, 0)
     st = torch.cuda.Stream()
-    elems = {apps.GRAN_THREAD: 2, apps.GRAN_WARP: 64, apps.GRAN_BLOCK: 2048}
+    elems = {apps.GRAN_THREAD: 2, apps.GRAN_WARP: 64, apps.GRAN_BLOCK: 2048, apps.GRAN_BLOCK_PUT: 2048}
     sizes = [int(x) for x in args.sizes.split(",")] if args.sizes else [64 << 10, 1 << 20, 16 << 20, 256 << 20]
-    grans = {"thread": apps.GRAN_THREAD, "warp": apps.GRAN_WARP, "block": apps.GRAN_BLOCK}
+    grans = {"thread": apps.GRAN_THREAD, "warp": apps.GRAN_WARP, "block": apps.GRAN_BLOCK,
+             "block_put": apps.GRAN_BLOCK_PUT}
     gsel = [grans[g] for g in args.grans.split(",")] if args.grans else [apps.GRAN_BLOCK, apps.GRAN_WARP,
                                                                            apps.GRAN_THREAD]
     aggsel = args.aggs.split(",") if args.aggs else None
+    pers = args.persistent
+    producer = "persistent" if pers else "block-per-partition"
     for S in sizes:
         n = S // 4
         A = torch.randn(n, device="cuda")
@@ -358,18 +361,18 @@ def sweep_p2p(args):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         it = 20
         for _ in range(3):  # warm-up (module load, first-touch)
-            apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st)
+            apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st, persistent=pers)
             with torch.cuda.stream(st):
                 R.copy_(Cb)
         torch.cuda.synchronize()
         e0.record(st)
         for _ in range(it):
-            apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st)
+            apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st, persistent=pers)
             with torch.cuda.stream(st):
                 R.copy_(Cb)
         e1.record(st)
         torch.cuda.synchronize()
-        print(json.dumps({"bytes": S, "mode": "kernel+copy (traditional, same GPU)",
+        print(json.dumps({"bytes": S, "mode": "kernel+copy (traditional, same GPU)", "producer": producer,
                           "us": e0.elapsed_time(e1) / it * 1e3,
                           "gbs": S / (e0.elapsed_time(e1) / it / 1e3) / 1e9}), flush=True)
         for gran in gsel:
@@ -387,6 +390,11 @@ def sweep_p2p(args):
                     rcv = pc.precv_init(R, parts, cnt, pc.FLOAT32, 0, 5, cs[1])
 
                     def epoch(first=False):
+                        if args.batched:  # MPI_Startall + Pbuf_prepare in one kernel, MPI_Waitall in one kernel
+                            pc.epoch_all([snd, rcv], False, st)
+                            apps.vecadd(A, B, Cb, n, gran, sq[0], st, persistent=pers)
+                            pc.waitall_on_stream([snd, rcv], st)
+                            return
                         snd.start(st)
                         rcv.start(st)
                         if first:
@@ -394,15 +402,15 @@ def sweep_p2p(args):
                         else:
                             rcv.pbuf_prepare(st)
                             snd.pbuf_prepare(st)
-                        apps.vecadd(A, B, Cb, n, gran, sq[0], st)
+                        apps.vecadd(A, B, Cb, n, gran, sq[0], st, persistent=pers)
                         snd.wait_on_stream(st)
                         rcv.wait_on_stream(st)
 
                     snd.start(st)
                     rcv.start(st)
                     pc.run_ranks([lambda: snd.pbuf_prepare(st), lambda: rcv.pbuf_prepare(st)])
-                    sq = [snd.prequest_create(gran, agg, copy)]
-                    apps.vecadd(A, B, Cb, n, gran, sq[0], st)
+                    sq = [snd.prequest_create(min(gran, apps.GRAN_BLOCK), agg, copy)]
+                    apps.vecadd(A, B, Cb, n, gran, sq[0], st, persistent=pers)
                     snd.wait_on_stream(st)
                     rcv.wait_on_stream(st)
                     torch.cuda.synchronize()
@@ -414,8 +422,9 @@ def sweep_p2p(args):
                     us = e0.elapsed_time(e1) / it * 1e3
                     errs = [q.error() for q in (snd, rcv) if q.error()[0] != 0]
                     ok = torch.equal(R, Cb)
-                    print(json.dumps({"bytes": S, "gran": ["thread", "warp", "block"][gran], "agg": agg_name,
-                                      "g": agg, "copy": ["inline", "engine"][copy], "us": us,
+                    print(json.dumps({"bytes": S, "gran": ["thread", "warp", "block", "block_put"][gran], "agg": agg_name,
+                                      "g": agg, "copy": ["inline", "engine"][copy], "producer": producer,
+                                      "control": "epoch_all+waitall" if args.batched else "per-request", "us": us,
                                       "goodput_gbs": S / (us / 1e6) / 1e9, "ok": ok, "parity": ok and not errs,
                                       "errors": errs}), flush=True)
                     snd.free()
@@ -434,9 +443,12 @@ if __name__ == "__main__":
     ap.add_argument("--max-bytes", type=int, default=1 << 30)
     ap.add_argument("--graph", action="store_true", help="replay a captured CUDA graph of the epoch")
     ap.add_argument("--sizes", default="", help="p2p: buffer bytes, comma separated")
-    ap.add_argument("--batched", action="store_true", help="dl_tensor: pc_epoch_all + pc_waitall_on_stream batch")
+    ap.add_argument("--batched", action="store_true",
+                    help="dl_tensor / p2p: pc_epoch_all + pc_waitall_on_stream batch (one control and one wait kernel)")
     ap.add_argument("--grans", default="", help="p2p: thread,warp,block")
     ap.add_argument("--aggs", default="", help="p2p: none,block,1MiB,all")
+    ap.add_argument("--persistent", action="store_true",
+                    help="p2p: persistent vecadd producer (both arms) instead of one CTA per logical block")
     a = ap.parse_args()
     {"allreduce": sweep_allreduce, "dl": sweep_dl, "dl_tensor": sweep_dl_per_tensor, "p2p": sweep_p2p,
      "coll": sweep_coll}[a.what](a)
