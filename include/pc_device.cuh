@@ -8,6 +8,8 @@
  *                                         uint64_t idx, const T &v);     block-collective
  *   PC_DEVICE int  pc_put_begin<T>(pc_prequest_t preq, pc_put_state *st);  block-collective
  *   PC_DEVICE int  pc_pready_block_put<T>(partition, preq, idx, v, st);     block-collective
+ *   PC_DEVICE int  pc_pready_block_coop(int partition, pc_prequest_t preq);  block-collective (R36,
+ *                  INLINE allreduce, -DPC_INLINE_ALLREDUCE)
  *   PC_DEVICE int  pc_parrived    (pc_prequest_t preq, int partition);
  *   PC_DEVICE int  pc_wait_arrived(pc_prequest_t preq, int partition);
  *   PC_DEVICE int  pc_parrived_warp / pc_wait_arrived_warp(preq, partition);  warp-collective
@@ -674,21 +676,24 @@ PC_DEVICE void ar_fold_t(const pc_ar_tab_s *tab, int P, uint64_t off, uint64_t n
  * every producer kernel that calls a Pready binding (a call on the rare
  * completing path costs nothing measurable). */
 #ifdef PC_INLINE_ALLREDUCE
-static __device__ __noinline__ void ar_fold(const pc_prequest_t &q, int u, uint32_t idx, uint32_t n) {
-  const pc_ar_tab_s *t = q.ar_tab;
-  const uint64_t off = (uint64_t)u * q.part_bytes, nb = q.part_bytes;
-  const int P = q.nranks;
+/* (scalars only: a reference to the caller's by-value request would make
+ * every thread copy the whole pc_prequest_t into local memory) */
+static __device__ __noinline__ void ar_fold_scalars(const pc_ar_tab_s *t, int P, int dtype, int op, uint64_t off,
+                                                    uint64_t nb, uint32_t idx, uint32_t n) {
 #define PC_AR_CASE(DTV)                                      \
-  if (q.op == 0) ar_fold_t<DTV, 0>(t, P, off, nb, idx, n);   \
-  else if (q.op == 1) ar_fold_t<DTV, 1>(t, P, off, nb, idx, n); \
+  if (op == 0) ar_fold_t<DTV, 0>(t, P, off, nb, idx, n);   \
+  else if (op == 1) ar_fold_t<DTV, 1>(t, P, off, nb, idx, n); \
   else ar_fold_t<DTV, 2>(t, P, off, nb, idx, n);
-  switch (q.dtype) {
+  switch (dtype) {
     case 0: PC_AR_CASE(0); break;
     case 1: PC_AR_CASE(1); break;
     case 3: PC_AR_CASE(3); break;
     default: PC_AR_CASE(4); break;
   }
 #undef PC_AR_CASE
+}
+PC_DEVICE void ar_fold(const pc_prequest_t &q, int u, uint32_t idx, uint32_t n) {
+  ar_fold_scalars(q.ar_tab, q.nranks, q.dtype, q.op, (uint64_t)u * q.part_bytes, q.part_bytes, idx, n);
 }
 #endif
 
@@ -697,6 +702,17 @@ static __device__ __noinline__ void ar_fold(const pc_prequest_t &q, int u, uint3
 PC_DEVICE void ar_publish(const pc_prequest_t &q, int u, uint32_t e) {
   fence_release(q.sys_scope);
   for (int k = 0; k < q.nranks; ++k) st_relaxed_sys(q.ar_tab->done[k] + u, e);
+}
+/* A fold of the whole partition by one participant: also advance u's slice
+ * counter by P, so epochs folded this way and cooperative epochs (R36, P
+ * slices of one each) keep the same target e * P on the same request. */
+PC_DEVICE void ar_publish_all(const pc_prequest_t &q, int u, uint32_t e) {
+  uint32_t *c2 = q.ar_tab->cnt + q.partitions + u;
+  if (q.sys_scope)
+    atom_add_acq_rel_sys(c2, (uint32_t)q.nranks);
+  else
+    atom_add_acq_rel_gpu(c2, (uint32_t)q.nranks);
+  ar_publish(q, u, e);
 }
 
 }  // namespace pc_detail
@@ -723,7 +739,7 @@ PC_DEVICE int pc_pready(int partition, pc_prequest_t preq) {
     if (ar_arrive(preq, partition, e)) {
       if (!ar_rtr_ok(preq, partition, e)) return PC_DEV_ERR_TIMEOUT;
       ar_fold(preq, partition, 0, 1);
-      ar_publish(preq, partition, e);
+      ar_publish_all(preq, partition, e);
     }
     return 0;
 #else
@@ -832,7 +848,7 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
     if (st == 1) {
       ar_fold(preq, partition, lane, 32);
       __syncwarp(full);
-      if (lane == 0) ar_publish(preq, partition, e);
+      if (lane == 0) ar_publish_all(preq, partition, e);
     }
     __syncwarp(full);
     return st < 0 ? PC_DEV_ERR_TIMEOUT : 0;
@@ -950,7 +966,7 @@ PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq) {
     if (st == 1) {
       ar_fold(preq, partition, tid, nthr);
       __syncthreads();  // every thread's stores, then ONE cumulative fence + the done words
-      if (tid == 0) ar_publish(preq, partition, s_e);
+      if (tid == 0) ar_publish_all(preq, partition, s_e);
     }
     __syncthreads();  // s_e / s_ok are reused by the block's next Pready
     return st < 0 ? PC_DEV_ERR_TIMEOUT : 0;
@@ -1115,6 +1131,80 @@ PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t id
   pc_detail::put_publish(partition, preq, idx, v, st.e, tid);
   return 0;
 }
+
+#ifdef PC_INLINE_ALLREDUCE
+/* Cooperative INLINE allreduce (MPIX extension, reading R36): for producers
+ * that run the P ranks' blocks of partition u side by side (one launch over
+ * the co-located ranks, units (u, r) adjacent and all CTAs resident — the
+ * caller's construction; the spin below is bounded by the request's timeout).
+ * Block (u, r): its data writes, then one arrival on u's counter (acq_rel),
+ * a wait until all P ranks arrived and every peer is ready to receive, then it
+ * folds slice r of P of partition u (16-B aligned byte ranges) over the P
+ * send buffers in rank order (R25: the same bits as O6 / the DIRECT engine)
+ * into every rank's recv buffer; the block completing the last slice (a second
+ * counter, the INLINE request's unused ready words in rank 0's control block)
+ * writes done[u] = e on every rank.  Instead of one block folding P
+ * partitions, P blocks fold one each — and the P partitions were just written
+ * (L2).  Other request kinds: pc_pready_block. */
+PC_DEVICE int pc_pready_block_coop(int partition, pc_prequest_t preq) {
+  using namespace pc_detail;
+  if (preq.kind != PC_KIND_PALLREDUCE || !preq.ar_tab) return pc_pready_block(partition, preq);
+  __shared__ uint32_t s_e;
+  __shared__ int s_ok, s_r;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  const uint32_t nthr = blockDim.x * blockDim.y * blockDim.z;
+  if (partition < 0 || partition >= preq.partitions) {
+    if (tid == 0) set_error(preq.err, PC_DEV_ERR_ARG, partition);
+    return PC_DEV_ERR_ARG;
+  }
+  const int P = preq.nranks;
+  const pc_ar_tab_s *t = preq.ar_tab;
+  __syncthreads();  // the block's data writes are complete
+  if (tid == 0) {
+    const uint32_t e = epoch_of(preq);
+    s_e = e;
+    int r = 0;
+    for (int k = 0; k < P; ++k)
+      if (t->send[k] == preq.sbuf) r = k;
+    s_r = r;
+    uint32_t *c = t->cnt + partition;
+    const uint32_t old = preq.sys_scope ? atom_add_acq_rel_sys(c, 1u) : atom_add_acq_rel_gpu(c, 1u);
+    const int32_t d = (int32_t)(e * (uint32_t)P - old);
+    int ok = 1;
+    if (d <= 0) {  // more than P arrivals in this epoch: a duplicate Pready
+      set_error(preq.err, PC_DEV_ERR_DEVICE, partition);
+      ok = 0;
+    } else if (d > 1) {  // wait for the other ranks' blocks of u
+      ok = preq.sys_scope ? spin_geq<true>(c, e * (uint32_t)P, preq.err, preq.timeout_ms, partition)
+                          : spin_geq<false>(c, e * (uint32_t)P, preq.err, preq.timeout_ms, partition);
+    }
+    if (ok) ok = ar_rtr_ok(preq, partition, e) ? 1 : 0;
+    s_ok = ok;
+  }
+  __syncthreads();
+  const uint32_t e = s_e;
+  const int r = s_r;
+  if (!s_ok) return PC_DEV_ERR_TIMEOUT;
+  const uint64_t chunk = ((preq.part_bytes + (uint64_t)P * 16 - 1) / ((uint64_t)P * 16)) * 16;
+  const uint64_t lo = (uint64_t)r * chunk;
+  const uint64_t hi = lo + chunk < preq.part_bytes ? lo + chunk : preq.part_bytes;
+  if (lo < hi)
+    ar_fold_scalars(t, P, preq.dtype, preq.op, (uint64_t)partition * preq.part_bytes + lo, hi - lo, tid, nthr);
+  __syncthreads();  // every thread's stores, then ONE release + the slice count
+  if (tid == 0) {
+    fence_release(preq.sys_scope);
+    uint32_t *c2 = t->cnt + preq.partitions + partition;
+    const uint32_t old = preq.sys_scope ? atom_add_acq_rel_sys(c2, 1u) : atom_add_acq_rel_gpu(c2, 1u);
+    const int32_t d = (int32_t)(e * (uint32_t)P - old);
+    if (d <= 0)
+      set_error(preq.err, PC_DEV_ERR_DEVICE, partition);
+    else if (d == 1)
+      ar_publish(preq, partition, e);  // (its release covers the other slices, acquired by the add)
+  }
+  __syncthreads();  // s_e / s_ok / s_r are reused by the block's next Pready
+  return 0;
+}
+#endif
 
 /* ---------------------------------------------------------------- Parrived */
 /* Allgather receive partition u' = k * partitions + u (rank k's partition u):

@@ -85,6 +85,7 @@ _APP_PROTOS = {
     "pcapp_pready_cost": (I32, [P, P, P, I32, I32, P, P, P]),
     "pcapp_produce": (I32, [P, P, I32, I64, I32, I32, I32, P, P]),
     "pcapp_bce_grad": (I32, [P, P, P, I32, I64, C.c_float, I32, I32, P, P]),
+    "pcapp_bce_grad_multi": (I32, [I32, P, P, P, I32, I64, C.c_float, I32, P, I32, P]),
     "pcapp_check_recv": (I32, [P, P, P, I32, I64, I32, P, P]),
     "pcapp_pingpong": (I32, [P, P, I32, I32, I32, P, P]),
     "pcapp_bare_pingpong": (I32, [P, P, I32, I32, C.c_uint32, P, P]),

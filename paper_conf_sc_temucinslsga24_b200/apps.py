@@ -52,6 +52,20 @@ def bce_grad(p, y, g, partitions: int, L: int, nf: float, preq: Prequest | None 
                                    preq.ptr if preq is not None else None, _stream(stream)), "bce_grad")
 
 
+def bce_grad_multi(ps, ys, gs, partitions: int, L: int, nf: float, preqs=None, blocks: int = 0, stream=None,
+                   coop: bool = False):
+    """bce_grad of every co-located rank in ONE launch, blocks interleaved
+    (partition u of all ranks side by side), so an INLINE allreduce fold of u
+    reads the ranks' just-written partitions from L2; preqs: one Prequest per
+    rank (or None: no Pready).  coop: pc_pready_block_coop (R36) — the P
+    blocks of a partition each fold one slice of it (every CTA resident)."""
+    n = len(ps)
+    arr = lambda xs: (C.c_void_p * n)(*[_ptr(x) for x in xs])  # noqa: E731
+    qa = (C.c_void_p * n)(*[q.ptr for q in preqs]) if preqs is not None else None
+    _ok(_lib.apps().pcapp_bce_grad_multi(n, arr(ps), arr(ys), arr(gs), partitions, L, nf, blocks, qa,
+                                         1 if coop else 0, _stream(stream)), "bce_grad_multi")
+
+
 def peer_copy(srcs, dsts, nbytes: int, blocks: int = 0, stream=None):
     """Bare peer copies (no library): len(srcs) concurrent copies of nbytes
     each, srcs[j] -> dsts[j] (int addresses or tensors; one side peer-mapped)."""
@@ -338,7 +352,8 @@ class DLProxy:
     partition on the last rank folds it for every rank (reading R33).
     Inputs: ``p`` (predictions), ``y`` (targets), fp32, one tensor per rank."""
 
-    def __init__(self, comms, partitions: int, L: int, algo: int, p, y, overlap: bool = True, copy: int | None = None):
+    def __init__(self, comms, partitions: int, L: int, algo: int, p, y, overlap: bool = True, copy: int | None = None,
+                 multi: bool = False, coop: bool = False):
         import torch
 
         from . import runtime as rt
@@ -365,6 +380,10 @@ class DLProxy:
         self.pst = [torch.cuda.Stream() for _ in range(self.P)]
         self.ev_ctl = torch.cuda.Event()
         self.ev_p = [torch.cuda.Event() for _ in range(self.P)]
+        # multi: every rank's producer in ONE launch on the control stream,
+        # partition u of all ranks side by side (bce_grad_multi)
+        self.multi = multi or coop
+        self.coop = coop  # multi + pc_pready_block_coop (INLINE copy, R36)
 
     def step(self, mode: str = "pready", order_stride: int = 1):
         from . import runtime as rt
@@ -378,6 +397,14 @@ class DLProxy:
         else:
             rt.startall(self.reqs, st)
             rt.pbuf_prepare_all(self.reqs, st)
+        if self.multi:
+            bce_grad_multi(self.p, self.y, self.g, self.Np, self.L, self.nf,
+                           self.preqs if mode == "pready" else None, stream=st, coop=self.coop)
+            if mode == "serial":
+                rt.preadyall(self.reqs, st)
+            for q in self.reqs:
+                q.wait_on_stream(st)
+            return
         self.ev_ctl.record(st)
         for r in range(self.P):
             self.pst[r].wait_event(self.ev_ctl)

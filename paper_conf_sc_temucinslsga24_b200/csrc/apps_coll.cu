@@ -126,6 +126,47 @@ __global__ void __launch_bounds__(512) bce_grad_kernel(const float *__restrict__
   }
 }
 
+// The DL proxy's producers of ALL co-located ranks in one launch, unit k =
+// (partition u = k / P, rank r = k % P): the P blocks producing partition u
+// run side by side, so the Pready that completes u (INLINE, R33) folds P
+// gradient partitions that were just written and still sit in L2 instead of
+// re-reading them from HBM (one launch also makes the ranks' blocks
+// co-resident by construction).  Per rank the same arithmetic and the same
+// Pready as bce_grad_kernel.
+struct BceMultiArgs {
+  int n;
+  const float *p[8];
+  const float *y[8];
+  float *g[8];
+  pc_prequest_t q[8];
+};
+__global__ void __launch_bounds__(512) bce_grad_multi_kernel(BceMultiArgs a, int partitions, int64_t L, float nf,
+                                                            int use_pready) {
+  // use_pready: 0 none, 1 pc_pready_block, 2 pc_pready_block_coop (R36)
+  const int P = a.n;
+  const int64_t units = (int64_t)partitions * P;
+  for (int64_t k = blockIdx.x; k < units; k += gridDim.x) {
+    const int u = (int)(k / P), r = (int)(k % P);
+    const int64_t off = (int64_t)u * L;
+    const float *p = a.p[r] + off, *y = a.y[r] + off;
+    float *g = a.g[r] + off;
+    const bool vec = ((((uintptr_t)p) | ((uintptr_t)y) | ((uintptr_t)g)) & 15) == 0;
+    const int64_t nv = vec ? L / 4 : 0;
+    const float4 *p4 = reinterpret_cast<const float4 *>(p), *y4 = reinterpret_cast<const float4 *>(y);
+    float4 *g4 = reinterpret_cast<float4 *>(g);
+#pragma unroll 4
+    for (int64_t j = threadIdx.x; j < nv; j += blockDim.x) {
+      const float4 x = __ldcs(p4 + j), t = __ldcs(y4 + j);
+      g4[j] = make_float4(bce_g(x.x, t.x, nf), bce_g(x.y, t.y, nf), bce_g(x.z, t.z, nf), bce_g(x.w, t.w, nf));
+    }
+    for (int64_t j = nv * 4 + threadIdx.x; j < L; j += blockDim.x) g[j] = bce_g(p[j], y[j], nf);
+    if (use_pready == 2)
+      pc_pready_block_coop(u, a.q[r]);
+    else if (use_pready)
+      pc_pready_block(u, a.q[r]);
+  }
+}
+
 }  // namespace
 
 extern "C" {
@@ -147,6 +188,39 @@ int pcapp_bce_grad(const float *p, const float *y, float *g, int partitions, int
   if (preq) q = *preq;
   bce_grad_kernel<<<blocks, 512, 0, s>>>(p, y, g, partitions, L, nf, order_stride < 1 ? 1 : order_stride,
                                          preq ? 1 : 0, q);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_bce_grad_multi(int n, const float *const *p, const float *const *y, float *const *g, int partitions,
+                         int64_t L, float nf, int blocks, const pc_prequest_t *const *preqs, int coop,
+                         cudaStream_t s) {
+  if (n < 1 || n > 8 || partitions < 1 || L < 0 || !p || !y || !g) return -1;
+  BceMultiArgs a{};
+  a.n = n;
+  for (int r = 0; r < n; ++r) {
+    a.p[r] = p[r];
+    a.y[r] = y[r];
+    a.g[r] = g[r];
+    if (preqs) a.q[r] = *preqs[r];
+  }
+  const int64_t units = (int64_t)partitions * n;
+  if (coop && preqs) {
+    // the P blocks of a partition wait for one another: every CTA resident,
+    // and a multiple of n so the ranks' blocks of u are always in one wave
+    int dev = 0, sms = 0, per = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess ||
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, bce_grad_multi_kernel, 512, 0) != cudaSuccess || per < 1)
+      return -2;
+    int64_t cap = (int64_t)sms * per;
+    cap -= cap % n;
+    if (blocks <= 0 || blocks > cap) blocks = (int)cap;
+    blocks -= blocks % n;
+    if (blocks < n) return -1;
+  } else if (blocks <= 0) {
+    blocks = units < 1184 ? (int)units : 1184;
+  }
+  bce_grad_multi_kernel<<<blocks, 512, 0, s>>>(a, partitions, L, nf, preqs ? (coop ? 2 : 1) : 0);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -82,3 +82,37 @@ def test_dl_proxy_mode_switch_and_many_epochs():
                 for r in (0, P - 1):
                     np.testing.assert_array_equal(dl.out[r][:n].cpu().numpy(), ref[r])
         dl.free()
+
+
+@pytest.mark.parametrize("mode,copy,algo,coop", [("pready", pc.COPY_INLINE, pc.ALGO_DIRECT, False),
+                                                 ("pready", pc.COPY_INLINE, pc.ALGO_DIRECT, True),
+                                                 ("mixed", pc.COPY_INLINE, pc.ALGO_DIRECT, True),
+                                                 ("pready", None, pc.ALGO_DIRECT, False),
+                                                 ("serial", None, pc.ALGO_RING, False),
+                                                 ("pready", None, pc.ALGO_RING, False)])
+@pytest.mark.parametrize("P,Np,L", [(8, 6, 3000), (4, 13, 4099), (2, 3, 65536), (8, 700, 1024)])
+def test_dl_proxy_multi_launch(mode, copy, algo, coop, P, Np, L):
+    """All ranks' producers in one launch (bce_grad_multi, partition u of
+    every rank side by side), with the INLINE fold (R33), the cooperative
+    INLINE fold (R36: the P blocks of u fold one slice each; "mixed"
+    alternates it with host-Pready epochs on the same request) or the engine,
+    over 3 epochs: bit-exact against the oracle's gradients + pallreduce."""
+    n = Np * L
+    with comms(P) as cs:
+        inputs = [[synth.bce_inputs(SEED + 3, r, e, n) for r in range(P)] for e in range(3)]
+        p = [torch.empty(n, device="cuda") for _ in range(P)]
+        y = [torch.empty(n, device="cuda") for _ in range(P)]
+        dl = apps.DLProxy(cs, Np, L, algo, p, y, copy=copy, multi=True, coop=coop)
+        for e in range(3):
+            torch.cuda.synchronize()
+            for r in range(P):
+                p[r].copy_(torch.from_numpy(inputs[e][r][0]))
+                y[r].copy_(torch.from_numpy(inputs[e][r][1]))
+            torch.cuda.synchronize()
+            dl.step(("serial" if e == 1 else "pready") if mode == "mixed" else mode)
+            torch.cuda.synchronize()
+            assert dl.errors() == []
+            ref = _oracle_step([inputs[e][r][0] for r in range(P)], [inputs[e][r][1] for r in range(P)], Np, L, algo)
+            for r in range(P):
+                np.testing.assert_array_equal(dl.out[r][:n].cpu().numpy().view(np.uint32), ref[r].view(np.uint32))
+        dl.free()

@@ -49,6 +49,7 @@ def run(P, L, algo, modes):
     torch.cuda.synchronize()
     dl_no = None
     dl_in = None
+    multi = {}
     out = []
     for mode in modes:
         if mode in ("pready", "serial"):
@@ -88,6 +89,26 @@ def run(P, L, algo, modes):
                 torch.cuda.synchronize()
             ms = timeit(lambda: dl_in.step("pready"), dl_in.ctl)
             assert dl_in.errors() == [], dl_in.errors()
+        elif mode in ("serial_multi", "pready_multi", "pready_inline_multi", "pready_coop_multi"):
+            # every rank's producer in ONE launch, partition u of all ranks side by side (bce_grad_multi)
+            key = {"pready_inline_multi": "inline", "pready_coop_multi": "coop"}.get(mode, "engine")
+            if key not in multi:
+                multi[key] = apps.DLProxy(cs, Np, L, pc.ALGO_DIRECT if key != "engine" else algo, p, y,
+                                          copy=pc.COPY_INLINE if key != "engine" else None, multi=True,
+                                          coop=key == "coop")
+                multi[key].step("serial" if mode == "serial_multi" else "pready")
+                torch.cuda.synchronize()
+            dm = multi[key]
+            sm = "serial" if mode == "serial_multi" else "pready"
+            ms = timeit(lambda: dm.step(sm), dm.ctl)
+            assert dm.errors() == [], dm.errors()
+            if key != "engine":  # parity of the fused step against the serial one (same bits: R25 rank order)
+                ref = multi.get("engine")
+                if ref is not None:
+                    ref.step("serial")
+                    dm.step("pready")
+                    torch.cuda.synchronize()
+                    assert all(torch.equal(ref.out[r], dm.out[r]) for r in range(P)), "fused != serial"
         elif mode == "pready_nooverlap":  # engine forked at the wait (no producer/engine concurrency)
             if dl_no is None:
                 dl_no = apps.DLProxy(cs, Np, L, algo, p, y, overlap=False)
@@ -130,6 +151,8 @@ def run(P, L, algo, modes):
         dl_no.free()
     if dl_in is not None:
         dl_in.free()
+    for dm in multi.values():
+        dm.free()
     for c in cs:
         c.destroy()
     g.destroy()
