@@ -360,19 +360,27 @@ def sweep_p2p(args):
         # traditional baseline: kernel, then a device copy (no library)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         it = 20
-        for _ in range(3):  # warm-up (module load, first-touch)
+
+        def trad():
             apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st, persistent=pers)
             with torch.cuda.stream(st):
                 R.copy_(Cb)
+
+        for _ in range(3):  # warm-up (module load, first-touch)
+            trad()
+        if args.graph:  # both arms replay a captured CUDA graph of their epoch
+            gt = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gt, stream=st):
+                trad()
+            trad = gt.replay  # noqa: F811
         torch.cuda.synchronize()
         e0.record(st)
         for _ in range(it):
-            apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st, persistent=pers)
             with torch.cuda.stream(st):
-                R.copy_(Cb)
+                trad()
         e1.record(st)
         torch.cuda.synchronize()
-        print(json.dumps({"bytes": S, "mode": "kernel+copy (traditional, same GPU)", "producer": producer,
+        print(json.dumps({"bytes": S, "mode": "kernel+copy (traditional, same GPU)", "producer": producer, "graph": bool(args.graph),
                           "us": e0.elapsed_time(e1) / it * 1e3,
                           "gbs": S / (e0.elapsed_time(e1) / it / 1e3) / 1e9}), flush=True)
         for gran in gsel:
@@ -413,10 +421,20 @@ def sweep_p2p(args):
                     apps.vecadd(A, B, Cb, n, gran, sq[0], st, persistent=pers)
                     snd.wait_on_stream(st)
                     rcv.wait_on_stream(st)
+                    run = epoch
+                    if args.graph:
+                        for _ in range(2):
+                            epoch()
+                        torch.cuda.synchronize()
+                        ge = torch.cuda.CUDAGraph()
+                        with torch.cuda.graph(ge, stream=st):
+                            epoch()
+                        run = ge.replay
                     torch.cuda.synchronize()
                     e0.record(st)
                     for _ in range(it):
-                        epoch()
+                        with torch.cuda.stream(st):
+                            run()
                     e1.record(st)
                     torch.cuda.synchronize()
                     us = e0.elapsed_time(e1) / it * 1e3
@@ -424,7 +442,8 @@ def sweep_p2p(args):
                     ok = torch.equal(R, Cb)
                     print(json.dumps({"bytes": S, "gran": ["thread", "warp", "block", "block_put"][gran], "agg": agg_name,
                                       "g": agg, "copy": ["inline", "engine"][copy], "producer": producer,
-                                      "control": "epoch_all+waitall" if args.batched else "per-request", "us": us,
+                                      "control": "epoch_all+waitall" if args.batched else "per-request",
+                                      "graph": bool(args.graph), "us": us,
                                       "goodput_gbs": S / (us / 1e6) / 1e9, "ok": ok, "parity": ok and not errs,
                                       "errors": errs}), flush=True)
                     snd.free()
