@@ -25,6 +25,28 @@ def test_library_exports_every_header_symbol():
     assert lib.pc_prequest_size() == _lib.apps().pcapp_prequest_size()
 
 
+def test_app_launchers_reject_bad_arguments_before_the_gpu():
+    """The producer launchers of libpcapps (session 2: the persistent vector
+    add, the one-launch multi-rank BCE producer) validate their arguments on
+    the host and return -1 without touching the GPU."""
+    import ctypes as C
+    lib = _lib.apps()
+    for name in ("pcapp_vecadd", "pcapp_vecadd_persistent", "pcapp_bce_grad_multi"):
+        assert hasattr(lib, name)
+    a16 = C.c_void_p(0x10000)
+    a8 = C.c_void_p(0x10008)
+    assert lib.pcapp_vecadd(a16, a16, a16, 3, -1, None, None) == -1  # odd element count
+    assert lib.pcapp_vecadd(a16, a16, a16, 4, 4, None, None) == -1  # unknown granularity
+    assert lib.pcapp_vecadd(a16, a16, a16, 4, 2, None, None) == -1  # Pready without a prequest
+    assert lib.pcapp_vecadd_persistent(a8, a16, a16, 4, -1, None, None) == -1  # TMA needs 16-B sources
+    assert lib.pcapp_vecadd_persistent(a16, a16, a16, 1 << 33, -1, None, None) == -1  # 32-bit indices
+    assert lib.pcapp_vecadd_persistent(a16, a16, a16, 4, 3, None, None) == -1  # block_put needs a prequest
+    arr = (C.c_void_p * 9)(*([0x10000] * 9))
+    assert lib.pcapp_bce_grad_multi(0, arr, arr, arr, 4, 16, 1.0, 0, None, 0, None) == -1  # no ranks
+    assert lib.pcapp_bce_grad_multi(9, arr, arr, arr, 4, 16, 1.0, 0, None, 0, None) == -1  # > 8 ranks
+    assert lib.pcapp_bce_grad_multi(2, arr, arr, arr, 0, 16, 1.0, 0, None, 0, None) == -1  # no partitions
+
+
 def test_no_oracle_in_product():
     """The product never links or imports the oracle."""
     out = subprocess.run(["nm", "-D", "--defined-only", _lib.LIBPC], capture_output=True, text=True).stdout
