@@ -6,8 +6,9 @@
  *   PC_DEVICE int  pc_pready_block(int partition, pc_prequest_t preq);  block-collective
  *   PC_DEVICE int  pc_pready_block_put<T>(int partition, pc_prequest_t preq,
  *                                         uint64_t idx, const T &v);     block-collective
- *   PC_DEVICE int  pc_put_begin<T>(pc_prequest_t preq, pc_put_state *st);  block-collective
+ *   PC_DEVICE int  pc_put_begin<T>(pc_prequest_t preq, pc_put_state *st, int batch = 1);  block-collective
  *   PC_DEVICE int  pc_pready_block_put<T>(partition, preq, idx, v, st);     block-collective
+ *   PC_DEVICE void pc_put_end(pc_prequest_t preq, pc_put_state &st);       block-collective
  *   PC_DEVICE int  pc_pready_block_coop(int partition, pc_prequest_t preq);  block-collective (R36,
  *                  INLINE allreduce, -DPC_INLINE_ALLREDUCE)
  *   PC_DEVICE int  pc_parrived    (pc_prequest_t preq, int partition);
@@ -1035,6 +1036,19 @@ PC_DEVICE bool put_eligible(const pc_prequest_t &q) {
   return q.kind != PC_KIND_PALLREDUCE && q.copy == 0 && q.part_bytes != 0 &&
          ((reinterpret_cast<uintptr_t>(q.peer_rbuf) | q.part_bytes) & (sizeof(T) - 1)) == 0;
 }
+/* The release of partition p after a barrier that ordered its assignments. */
+PC_DEVICE void put_release(const pc_prequest_t &q, int partition, uint32_t e) {
+  if (q.agg == 1 && !q.xpart) {  // the flag store itself releases (one MEMBAR, no separate fence)
+    if (q.sys_scope)
+      st_release_sys(q.peer_flags + partition, e);
+    else
+      st_release_gpu(q.peer_flags + partition, e);
+    st_relaxed_gpu(q.sent + partition, e);
+  } else {
+    fence_before_publish(q);
+    publish(q, partition / q.agg, 1, e, partition);
+  }
+}
 /* The assignment, barrier, release and flag of a checked epoch. */
 template <typename T>
 PC_DEVICE void put_publish(int partition, const pc_prequest_t &q, uint64_t idx, const T &v, uint32_t e,
@@ -1042,18 +1056,7 @@ PC_DEVICE void put_publish(int partition, const pc_prequest_t &q, uint64_t idx, 
   if (idx < q.part_bytes / sizeof(T))
     *reinterpret_cast<T *>(q.peer_rbuf + (uint64_t)partition * q.part_bytes + idx * sizeof(T)) = v;
   __syncthreads();  // the block's pushes, then ONE cumulative release by thread 0
-  if (tid == 0) {
-    if (q.agg == 1 && !q.xpart) {  // the flag store itself releases (one MEMBAR, no separate fence)
-      if (q.sys_scope)
-        st_release_sys(q.peer_flags + partition, e);
-      else
-        st_release_gpu(q.peer_flags + partition, e);
-      st_relaxed_gpu(q.sent + partition, e);
-    } else {
-      fence_before_publish(q);
-      publish(q, partition / q.agg, 1, e, partition);
-    }
-  }
+  if (tid == 0) put_release(q, partition, e);
 }
 }  // namespace pc_detail
 
@@ -1083,7 +1086,12 @@ PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t id
 }
 
 /* Persistent producers (R35): the {epoch, ready-to-receive} check once per
- * CTA per epoch, before its first pc_pready_block_put(..., st).  Both are
+ * CTA per epoch, before its first pc_pready_block_put(..., st).  batch > 1:
+ * the CTA releases its Preadies `batch` at a time — one barrier and one
+ * warp-wide MEMBAR per batch instead of per logical block (lane k of warp 0
+ * releases the k-th pending partition's flag); a flag is never set before
+ * its partition's bytes are visible, only later; pc_put_end (block-
+ * collective, after the CTA's last Pready) releases the rest.  Both are
  * fixed for the rest of the epoch once reached, so the later calls carry no
  * load and no barrier before the assignment — the raw chain (assign from
  * registers, barrier, release, flag) with nothing out of line in the loop.
@@ -1092,18 +1100,24 @@ PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t id
  * partitioned send, or misaligned for T: use pc_pready_block); or
  * PC_DEV_ERR_TIMEOUT. */
 struct pc_put_state {
-  uint32_t e;   /* the epoch pc_put_begin found */
-  uint32_t ok;  /* 1: checked; the fast pc_pready_block_put may be used */
+  uint32_t e;      /* the epoch pc_put_begin found */
+  uint32_t ok;     /* 1: checked; the fast pc_pready_block_put may be used */
+  uint32_t batch;  /* logical blocks per release (1..32) */
+  uint32_t npend;  /* Preadies since the last release (the same in every thread) */
+  int mine;        /* thread k < batch: the partition of the k-th pending Pready */
 };
 
 template <typename T>
-PC_DEVICE int pc_put_begin(pc_prequest_t preq, pc_put_state *st) {
+PC_DEVICE int pc_put_begin(pc_prequest_t preq, pc_put_state *st, int batch = 1) {
   using namespace pc_detail;
   __shared__ uint32_t s_e;
   __shared__ int s_ok;
   const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
   st->e = 0;
   st->ok = 0;
+  st->batch = (uint32_t)(batch < 1 ? 1 : (batch > 32 ? 32 : batch));
+  st->npend = 0;
+  st->mine = -1;
   if (!put_eligible<T>(preq)) return PC_DEV_ERR_ARG;
   if (tid == 0) {
     const uint2 er = epoch_rtr(preq);
@@ -1119,8 +1133,7 @@ PC_DEVICE int pc_put_begin(pc_prequest_t preq, pc_put_state *st) {
 }
 
 template <typename T>
-PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t idx, const T &v,
-                                  const pc_put_state &st) {
+PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t idx, const T &v, pc_put_state &st) {
   static_assert(sizeof(T) == 4 || sizeof(T) == 8 || sizeof(T) == 16, "element of 4, 8 or 16 bytes");
   if (!st.ok) return PC_DEV_ERR_ARG;
   const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
@@ -1128,8 +1141,28 @@ PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t id
     if (tid == 0 && atomicCAS(preq.err, 0, PC_DEV_ERR_ARG) == 0) preq.err[1] = partition;
     return PC_DEV_ERR_ARG;
   }
-  pc_detail::put_publish(partition, preq, idx, v, st.e, tid);
+  if (st.batch == 1) {
+    pc_detail::put_publish(partition, preq, idx, v, st.e, tid);
+    return 0;
+  }
+  if (idx < preq.part_bytes / sizeof(T))
+    *reinterpret_cast<T *>(preq.peer_rbuf + (uint64_t)partition * preq.part_bytes + idx * sizeof(T)) = v;
+  if (tid == st.npend) st.mine = partition;
+  if (++st.npend < st.batch) return 0;
+  __syncthreads();  // the batch's assignments, then lane k of warp 0 releases pending partition k
+  if (tid < st.npend) pc_detail::put_release(preq, st.mine, st.e);
+  st.npend = 0;
   return 0;
+}
+
+/* Block-collective, after the CTA's last pc_pready_block_put of the epoch:
+ * releases the partitions still pending in a batch. */
+PC_DEVICE void pc_put_end(pc_prequest_t preq, pc_put_state &st) {
+  if (!st.ok || st.npend == 0) return;
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  __syncthreads();
+  if (tid < st.npend) pc_detail::put_release(preq, st.mine, st.e);
+  st.npend = 0;
 }
 
 #ifdef PC_INLINE_ALLREDUCE

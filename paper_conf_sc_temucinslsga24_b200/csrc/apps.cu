@@ -171,9 +171,9 @@ __global__ void __launch_bounds__(1024, 2) vecadd_persistent_kernel(const float2
 __global__ void __launch_bounds__(1024, 2) vecadd_put_persistent_kernel(const float2 *__restrict__ A,
                                                                         const float2 *__restrict__ B,
                                                                         float2 *__restrict__ C, int n2, int nblk,
-                                                                        pc_prequest_t preq) {
+                                                                        int batch, pc_prequest_t preq) {
   pc_put_state st;
-  if (pc_put_begin<float2>(preq, &st) != 0) return;  // (the launcher checked eligibility; timeout is recorded)
+  if (pc_put_begin<float2>(preq, &st, batch) != 0) return;  // (the launcher checked eligibility; timeout is recorded)
   const int G = gridDim.x;
   int p = blockIdx.x;
   float2 a = make_float2(0.f, 0.f), b = a;
@@ -192,6 +192,7 @@ __global__ void __launch_bounds__(1024, 2) vecadd_put_persistent_kernel(const fl
     if (i < n2) C[i] = c;
     pc_pready_block_put(p, preq, i < n2 ? (uint64_t)threadIdx.x : ~0ull, c, st);
   }
+  pc_put_end(preq, st);
 }
 
 // Bare NVLink peer-copy floor (SURVEY §8(d) "Rooflines"): no
@@ -567,6 +568,14 @@ VecaddPersFn vecadd_pers_fn(int gran) {
   }
 }
 
+// Logical blocks per release of the persistent register Kernel Copy producer
+// (pc_put_begin batch; PCAPP_PUT_BATCH=1..32, default 4).
+int put_batch() {  // (read at every launch: tests vary it)
+  const char *e = getenv("PCAPP_PUT_BATCH");
+  int v = e ? atoi(e) : 4;
+  return v < 1 ? 1 : (v > 32 ? 32 : v);
+}
+
 extern "C" {
 
 int pcapp_vecadd(const float *A, const float *B, float *C, int64_t n, int gran, const pc_prequest_t *preq,
@@ -605,7 +614,7 @@ int pcapp_vecadd_persistent(const float *A, const float *B, float *C, int64_t n,
       return -2;
     const int64_t grid = nblk < (int64_t)sms * per ? nblk : (int64_t)sms * per;
     vecadd_put_persistent_kernel<<<(unsigned)grid, 1024, 0, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C,
-                                                                 (int)n2, (int)nblk, q);
+                                                                 (int)n2, (int)nblk, put_batch(), q);
     return cudaGetLastError() == cudaSuccess ? 0 : -2;
   }
   if (gran == PCAPP_GRAN_BLOCK_PUT) gran = PCAPP_GRAN_BLOCK;  // same partitions: the send buffer holds the data
