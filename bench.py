@@ -118,6 +118,7 @@ class Clocks:
             pynvml.nvmlInit()
             self.nvml = pynvml
             self.h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.mx = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
             self.stop = threading.Event()
             self.t = threading.Thread(target=self._nvml_loop, daemon=True)
             self.t.start()
@@ -138,20 +139,35 @@ class Clocks:
         for line in self.p.stdout:
             self.lines.append(line.strip())
 
-    def _nvml_loop(self):
+    def _nvml_sample(self):
         nv = self.nvml
         bits = [("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
                 ("sw_power_cap", 0x4)]
-        mx = nv.nvmlDeviceGetMaxClockInfo(self.h, nv.NVML_CLOCK_SM)
+        try:
+            sm = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+            r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            f = [str(sm), str(self.mx), "0", hex(r)] + ["Active" if r & b else "Not Active" for _, b in bits]
+            self.lines.append(", ".join(f))
+        except Exception:
+            pass
+
+    def _nvml_loop(self):
         while not self.stop.is_set():
-            try:
-                sm = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
-                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
-                f = [str(sm), str(mx), "0", hex(r)] + ["Active" if r & b else "Not Active" for _, b in bits]
-                self.lines.append(", ".join(f))
-            except Exception:
-                pass
+            self._nvml_sample()
             time.sleep(0.002)
+
+    def sample_now(self):
+        """One synchronous sample (called while the timed work is still queued
+        on the GPU), so a short timed region is never left without a sample."""
+        if getattr(self, "nvml", None):
+            self._nvml_sample()
+            return
+        try:
+            out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                  "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=10)
+            self.lines.extend(x.strip() for x in out.stdout.splitlines() if x.strip())
+        except Exception:
+            pass
 
     def __exit__(self, *a):
         if getattr(self, "nvml", None):
@@ -623,6 +639,7 @@ def run_virtual(args):
         for _ in range(args.steps):
             step()
         e1.record(st)
+        clk.sample_now()  # the steps are still running: one sample inside the timed region
         torch.cuda.synchronize()
     launches = pc.launch_count() - n0
     ms = e0.elapsed_time(e1) / args.steps
@@ -1203,6 +1220,7 @@ def run_multi(args):
         for _ in range(steps):
             step()
         e1.record(st)
+        clk.sample_now()  # the steps are still running: one sample inside the timed region
         torch.cuda.synchronize()
         dist.barrier()
     launches = pc.launch_count() - n0
