@@ -945,13 +945,24 @@ def multi_p2p(ctx, pc, apps, torch, dist):
                 trad_nccl()
             row["traditional_nccl_us_host"] = pmax((time.perf_counter() - t0) / it * 1e6)
         q0.free()
-        configs = [("block", apps.GRAN_BLOCK, 1, pc.COPY_INLINE), ("block", apps.GRAN_BLOCK, 1, pc.COPY_ENGINE),
-                   ("block->1MiB", apps.GRAN_BLOCK, 128, pc.COPY_INLINE),
-                   ("warp->all", apps.GRAN_WARP, None, pc.COPY_INLINE),
-                   ("thread->all", apps.GRAN_THREAD, None, pc.COPY_INLINE)]
+        if side == 0:  # the same traditional model, device-timed, with the persistent producer (C2 leg of N = 1)
+            def trad_dev():
+                apps.vecadd(A, B, Cb, n, apps.GRAN_NONE, None, st, persistent=True)
+                apps.memcpy_async(peer, Cb, S, st)
+        else:
+            def trad_dev():
+                pass
+        row["traditional_persistent_us_device"] = ptime(trad_dev, it) * 1e3
+        configs = [("block", apps.GRAN_BLOCK, 1, pc.COPY_INLINE, False),
+                   ("block", apps.GRAN_BLOCK, 1, pc.COPY_ENGINE, False),
+                   ("block->1MiB", apps.GRAN_BLOCK, 128, pc.COPY_INLINE, False),
+                   ("block_put persistent", apps.GRAN_BLOCK_PUT, 1, pc.COPY_INLINE, True),
+                   ("warp->all", apps.GRAN_WARP, None, pc.COPY_INLINE, False),
+                   ("thread->all", apps.GRAN_THREAD, None, pc.COPY_INLINE, False)]
         if S == (1 << 20):  # C1: 128 block partitions aggregated into 8 transport partitions (R24)
-            configs = [("C1 block->128KiB", apps.GRAN_BLOCK, 16, pc.COPY_INLINE)] + configs
-        for name, gran, agg, copy in configs:
+            configs = [("C1 block->128KiB", apps.GRAN_BLOCK, 16, pc.COPY_INLINE, False)] + configs
+        elems[apps.GRAN_BLOCK_PUT] = 2048
+        for name, gran, agg, copy, pers in configs:
             cnt = elems[gran]
             parts = n // cnt
             g = parts if agg is None else min(agg, parts)
@@ -963,14 +974,14 @@ def multi_p2p(ctx, pc, apps, torch, dist):
             tag += 1
             q.start(st)
             q.pbuf_prepare(st)
-            sq = q.prequest_create(gran, g, copy) if side == 0 else None
+            sq = q.prequest_create(min(gran, apps.GRAN_BLOCK), g, copy) if side == 0 else None
 
             def epoch(first=False):
                 if not first:
                     q.start(st)
                     q.pbuf_prepare(st)
                 if side == 0:
-                    apps.vecadd(A, B, Cb, n, gran, sq, st)
+                    apps.vecadd(A, B, Cb, n, gran, sq, st, persistent=pers)
                 q.wait_on_stream(st)
 
             epoch(first=True)

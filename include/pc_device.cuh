@@ -1102,7 +1102,7 @@ PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t id
 struct pc_put_state {
   uint32_t e;      /* the epoch pc_put_begin found */
   uint32_t ok;     /* 1: checked; the fast pc_pready_block_put may be used */
-  uint32_t batch;  /* logical blocks per release (1..32) */
+  uint32_t batch;  /* logical blocks per release (1 .. min(32, threads per block)) */
   uint32_t npend;  /* Preadies since the last release (the same in every thread) */
   int mine;        /* thread k < batch: the partition of the k-th pending Pready */
 };
@@ -1115,7 +1115,9 @@ PC_DEVICE int pc_put_begin(pc_prequest_t preq, pc_put_state *st, int batch = 1) 
   const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
   st->e = 0;
   st->ok = 0;
-  st->batch = (uint32_t)(batch < 1 ? 1 : (batch > 32 ? 32 : batch));
+  const uint32_t nthr = blockDim.x * blockDim.y * blockDim.z;  // thread k < batch records pending Pready k
+  const uint32_t cap = nthr < 32 ? nthr : 32;
+  st->batch = batch < 1 ? 1u : ((uint32_t)batch > cap ? cap : (uint32_t)batch);
   st->npend = 0;
   st->mine = -1;
   if (!put_eligible<T>(preq)) return PC_DEV_ERR_ARG;

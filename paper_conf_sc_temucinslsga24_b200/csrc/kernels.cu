@@ -496,8 +496,15 @@ int launch_wait_words(const uint32_t *words, int n, const uint32_t *epoch, uint3
 // Flag words of a request: at most one 256-thread block per 1024 words, at
 // most one block per SM (spinning blocks never fill the GPU: DESIGN.md §7).
 int wait_words_blocks(int n) {
+  static int sms = 0;  // (one device per process in this library's use; B200: 148)
+  if (!sms) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) !=
+                                                   cudaSuccess || sms < 1)
+      sms = 148;
+  }
   const int b = (n + 1023) / 1024;
-  return b < 1 ? 1 : (b > 148 ? 148 : b);
+  return b < 1 ? 1 : (b > sms ? sms : b);
 }
 
 int recv_wait_blocks(const pc_prequest_t &q) {
