@@ -714,3 +714,46 @@ def test_force_sys_scope_env(force):
     p = subprocess.run([sys.executable, "-c", _SCOPE_PROBE], capture_output=True, text=True, env=env, timeout=240)
     assert p.returncode == 0, p.stderr[-2000:]
     assert p.stdout.strip().splitlines()[-1] == force
+
+
+# ------------------------------------------------ stream waits over many flag words (session 2)
+@pytest.mark.parametrize("Ns,Nr", [(100003, 100003), (3000, 5000), (5000, 3000)])
+def test_stream_wait_many_partitions(Ns, Nr):
+    """MPI_Wait on the stream over ~10^5 flag words (the bulk wait: relaxed
+    16-B loads over up to one block per SM, head / tail words at odd
+    offsets) and over per-receive-partition counters of different
+    partitionings (R30, grid-stride over several blocks): every byte
+    delivered over 3 epochs, MPI_Test false before the sender's Pready
+    (the pending-count path) and true after."""
+    total = Ns * 16 if Ns == Nr else 240000
+    sb, rb = total // Ns, total // Nr
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        sbuf = torch.empty(total, dtype=torch.uint8, device="cuda")
+        rbuf = torch.zeros_like(sbuf)
+        snd = pc.psend_init(sbuf, Ns, sb, pc.BYTE, 1, 21, cs[0])
+        rcv = pc.precv_init(rbuf, Nr, rb, pc.BYTE, 0, 21, cs[1])
+        for e in range(3):
+            payload = synth.bytes_tagged(SEED, 4, e, total)
+            sbuf.copy_(torch.from_numpy(payload))
+            torch.cuda.synchronize()
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+                rcv.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            torch.cuda.synchronize()
+            assert not rcv.test()  # nothing readied yet in this epoch
+            snd.pready_range(0, Ns - 1, s0)
+            snd.wait_on_stream(s0)
+            rcv.wait_on_stream(s1)
+            torch.cuda.synchronize()
+            assert snd.error()[0] == 0 and rcv.error()[0] == 0, (snd.error(), rcv.error())
+            np.testing.assert_array_equal(rbuf.cpu().numpy(), payload)
+            assert rcv.test()
+        snd.free()
+        rcv.free()
