@@ -82,6 +82,7 @@ _PC_PROTOS = {
 _APP_PROTOS = {
     "pcapp_vecadd": (I32, [P, P, P, I64, I32, P, P]),
     "pcapp_vecadd_persistent": (I32, [P, P, P, I64, I32, P, P]),
+    "pcapp_produce_put": (I32, [P, P, I32, I64, I32, I32, I32, P, P]),
     "pcapp_pready_cost": (I32, [P, P, P, I32, I32, P, P, P]),
     "pcapp_produce": (I32, [P, P, I32, I64, I32, I32, I32, P, P]),
     "pcapp_bce_grad": (I32, [P, P, P, I32, I64, C.c_float, I32, I32, P, P]),

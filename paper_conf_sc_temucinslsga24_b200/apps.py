@@ -43,6 +43,15 @@ def produce(dst, src, partitions: int, part_bytes: int, gran: int, preq: Preques
                                   preq.ptr, _stream(stream)), "produce")
 
 
+def produce_put(dst, src, partitions: int, part_bytes: int, elem_bytes: int, preq: Prequest, threads: int = 256,
+                blocks: int = 0, stream=None):
+    """Copy src -> dst partition by partition, handing each thread's element
+    (elem_bytes = 4 / 8 / 16) to pc_pready_block_put (R35); part_bytes <=
+    threads * elem_bytes."""
+    _ok(_lib.apps().pcapp_produce_put(_ptr(dst), _ptr(src), partitions, part_bytes, elem_bytes, threads, blocks,
+                                      preq.ptr, _stream(stream)), "produce_put")
+
+
 def bce_grad(p, y, g, partitions: int, L: int, nf: float, preq: Prequest | None = None, order_stride: int = 1,
              blocks: int = 0, stream=None):
     """DL proxy producer (R28): g = (p - y) / ((p (1 - p)) n) over partitions of L

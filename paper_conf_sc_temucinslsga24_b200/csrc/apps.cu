@@ -13,6 +13,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdlib.h>
+#include <string.h>
 
 #include "pc_device.cuh"
 
@@ -193,6 +194,28 @@ __global__ void __launch_bounds__(1024, 2) vecadd_put_persistent_kernel(const fl
     pc_pready_block_put(p, preq, i < n2 ? (uint64_t)threadIdx.x : ~0ull, c, st);
   }
   pc_put_end(preq, st);
+}
+
+// pc_pready_block_put with 4-, 8- or 16-byte elements (test producer): each
+// CTA copies its partitions src -> send buffer (one element of type T per
+// thread, partition bytes <= blockDim * sizeof(T)) and hands the element it
+// holds to pc_pready_block_put; partitions whose size or alignment does not
+// suit T take the library's pc_pready_block fallback.
+template <typename T>
+__global__ void produce_put_kernel(uint8_t *__restrict__ dst, const uint8_t *__restrict__ src, int partitions,
+                                   int64_t part_bytes, pc_prequest_t preq) {
+  const uint64_t ne = (uint64_t)part_bytes / sizeof(T), tail = (uint64_t)part_bytes % sizeof(T);
+  for (int p = blockIdx.x; p < partitions; p += gridDim.x) {
+    const uint64_t off = (uint64_t)p * part_bytes;
+    T v{};
+    const bool mine = threadIdx.x < ne;
+    if (mine) {
+      memcpy(&v, src + off + (uint64_t)threadIdx.x * sizeof(T), sizeof(T));
+      memcpy(dst + off + (uint64_t)threadIdx.x * sizeof(T), &v, sizeof(T));
+    }
+    if (threadIdx.x < tail) dst[off + ne * sizeof(T) + threadIdx.x] = src[off + ne * sizeof(T) + threadIdx.x];
+    pc_pready_block_put(p, preq, mine ? (uint64_t)threadIdx.x : ~0ull, v);
+  }
 }
 
 // Bare NVLink peer-copy floor (SURVEY §8(d) "Rooflines"): no
@@ -628,6 +651,23 @@ int pcapp_vecadd_persistent(const float *A, const float *B, float *C, int64_t n,
   const int64_t slots = (int64_t)sms * per;
   const int64_t grid = nblk < slots ? nblk : slots;
   f<<<(unsigned)grid, 1024, kStagedSmem, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, nblk, q);
+  return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+
+int pcapp_produce_put(void *dst, const void *src, int partitions, int64_t part_bytes, int elem_bytes, int threads,
+                      int blocks, const pc_prequest_t *preq, cudaStream_t s) {
+  if (!preq || partitions < 1 || threads < 32 || threads > 1024 || part_bytes < 1) return -1;
+  if ((uint64_t)part_bytes > (uint64_t)threads * (uint64_t)elem_bytes) return -1;  // one element per thread
+  if (blocks <= 0) blocks = partitions < 592 ? partitions : 592;
+  const pc_prequest_t q = *preq;
+  uint8_t *d = (uint8_t *)dst;
+  const uint8_t *sr = (const uint8_t *)src;
+  switch (elem_bytes) {
+    case 4: produce_put_kernel<uint32_t><<<blocks, threads, 0, s>>>(d, sr, partitions, part_bytes, q); break;
+    case 8: produce_put_kernel<uint2><<<blocks, threads, 0, s>>>(d, sr, partitions, part_bytes, q); break;
+    case 16: produce_put_kernel<uint4><<<blocks, threads, 0, s>>>(d, sr, partitions, part_bytes, q); break;
+    default: return -1;
+  }
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -757,3 +757,42 @@ def test_stream_wait_many_partitions(Ns, Nr):
             assert rcv.test()
         snd.free()
         rcv.free()
+
+
+@pytest.mark.parametrize("elem,pbytes,agg", [(16, 4096, 1), (4, 1024, 1), (8, 2048, 3), (16, 1000, 1), (4, 1022, 2),
+                                             (16, 16, 1)])
+@pytest.mark.parametrize("copy", [pc.COPY_INLINE, pc.COPY_ENGINE])
+def test_pready_block_put_element_types(elem, pbytes, agg, copy):
+    """pc_pready_block_put with 4-, 8- and 16-byte elements from a 256-thread
+    producer over 37 partitions (more than one per CTA), and the fallback to
+    pc_pready_block when the partition size does not suit the element type or
+    the copy mode is not INLINE: byte-exact delivery over 2 epochs."""
+    parts = 37
+    total = parts * pbytes
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        src = torch.empty(total, dtype=torch.uint8, device="cuda")
+        sbuf, rbuf = torch.zeros_like(src), torch.zeros_like(src)
+        snd = pc.psend_init(sbuf, parts, pbytes, pc.BYTE, 1, 23, cs[0])
+        rcv = pc.precv_init(rbuf, parts, pbytes, pc.BYTE, 0, 23, cs[1])
+        for e in range(2):
+            payload = synth.bytes_tagged(SEED, 5, e, total)
+            src.copy_(torch.from_numpy(payload))
+            torch.cuda.synchronize()
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                sq = snd.prequest_create(pc.GRAN_BLOCK, agg, copy)
+                rcv.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            apps.produce_put(sbuf, src, parts, pbytes, elem, sq, threads=256, blocks=8, stream=s0)
+            snd.wait_on_stream(s0)
+            rcv.wait_on_stream(s1)
+            torch.cuda.synchronize()
+            assert snd.error()[0] == 0 and rcv.error()[0] == 0, (snd.error(), rcv.error())
+            np.testing.assert_array_equal(rbuf.cpu().numpy(), payload)
+        snd.free()
+        rcv.free()
