@@ -45,6 +45,10 @@ def test_app_launchers_reject_bad_arguments_before_the_gpu():
     assert lib.pcapp_bce_grad_multi(0, arr, arr, arr, 4, 16, 1.0, 0, None, 0, None) == -1  # no ranks
     assert lib.pcapp_bce_grad_multi(9, arr, arr, arr, 4, 16, 1.0, 0, None, 0, None) == -1  # > 8 ranks
     assert lib.pcapp_bce_grad_multi(2, arr, arr, arr, 0, 16, 1.0, 0, None, 0, None) == -1  # no partitions
+    q = C.create_string_buffer(4096)  # (a request image: never read before the argument checks fail)
+    assert lib.pcapp_produce_put(a16, a16, 4, 4097, 16, 256, 0, q, None) == -1  # > one element per thread
+    assert lib.pcapp_produce_put(a16, a16, 4, 64, 16, 16, 0, q, None) == -1  # < one warp
+    assert lib.pcapp_produce_put(a16, a16, 4, 64, 16, 256, 0, None, None) == -1  # no prequest
 
 
 def test_no_oracle_in_product():
