@@ -368,6 +368,12 @@ def c2_bench(pc, apps, torch, S=256 << 20, epochs=20):
     for c in cs:
         c.destroy()
     g.destroy()
+    hbm, src = peaks()
+    alg = 4 * S  # A and B read, C written, C pushed (the peer is HBM of the same GPU here)
+    out["roofline"] = {"bound": "hbm", "algorithmic_bytes_per_epoch": alg,
+                       "achieved": alg / (out["partitioned_us"] / 1e6) / 1e9, "peak": hbm, "unit": "GB/s",
+                       "frac": alg / (out["partitioned_us"] / 1e6) / 1e9 / hbm, "peak_source": src,
+                       "note": "whole epoch (control + producer + both waits), not the producer kernel alone"}
     out.update({"bytes": S, "partitions": parts, "gran": "block_put (R35), persistent producer", "copy": "inline",
                 "speedup_vs_traditional": out["traditional_us"] / out["partitioned_us"],
                 "goodput_gbs": S / (out["partitioned_us"] / 1e6) / 1e9, "ok": ok,
