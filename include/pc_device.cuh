@@ -3,6 +3,8 @@
  *
  *   PC_DEVICE int  pc_pready      (int partition, pc_prequest_t preq);  any thread
  *   PC_DEVICE int  pc_pready_warp (int partition, pc_prequest_t preq);  warp-collective
+ *   PC_DEVICE int  pc_warp_begin(pc_prequest_t preq, pc_warp_state *st);     warp-collective
+ *   PC_DEVICE int  pc_pready_warp (int partition, pc_prequest_t preq, st);  warp-collective (checked once)
  *   PC_DEVICE int  pc_pready_block(int partition, pc_prequest_t preq);  block-collective
  *   PC_DEVICE int  pc_pready_block_put<T>(int partition, pc_prequest_t preq,
  *                                         uint64_t idx, const T &v);     block-collective
@@ -914,6 +916,81 @@ PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq) {
   if (lane == 0) {
     fence_before_publish(preq);
     publish(preq, t, 1, e, partition);
+  }
+  __syncwarp(full);
+  return 0;
+}
+
+/* Warp granularity for a persistent warp (R35's check-once, warp form):
+ * pc_warp_begin (warp-collective) checks {epoch, ready-to-receive} once per
+ * warp per epoch — both fixed once reached — and the pc_pready_warp(...,
+ * st) that follow (INLINE partitioned send, partitions of at most 16 B per
+ * lane) push straight away and release the flag with one st.release: no
+ * acquire round trip per message.  Any other request (or st.ok == 0) takes
+ * the plain pc_pready_warp. */
+struct pc_warp_state {
+  uint32_t e;   /* the epoch pc_warp_begin found */
+  uint32_t ok;  /* 1: checked; the fast path may be used */
+};
+PC_DEVICE int pc_warp_begin(pc_prequest_t preq, pc_warp_state *st) {
+  using namespace pc_detail;
+  const unsigned full = 0xffffffffu;
+  const uint32_t lane = lane_id();
+  st->e = 0;
+  st->ok = 0;
+  if (preq.kind == PC_KIND_PALLREDUCE || preq.copy != 0 || preq.part_bytes == 0 || preq.part_bytes > 512 ||
+      (preq.part_bytes & 7) != 0)
+    return PC_DEV_ERR_ARG;
+  uint32_t e = 0;
+  int ok = 1;
+  if (lane == 0) {
+    const uint2 er = epoch_rtr(preq);
+    e = er.x;
+    if (!reached(er.y, e)) ok = spin_geq<true>(preq.rtr, e, preq.err, preq.timeout_ms, -5);
+  }
+  e = __shfl_sync(full, e, 0);
+  ok = __shfl_sync(full, ok, 0);
+  __syncwarp(full);  // lane 0's acquire happens before every lane's later pushes
+  if (!ok) return PC_DEV_ERR_TIMEOUT;
+  st->e = e;
+  st->ok = 1;
+  return 0;
+}
+
+PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq);
+
+PC_DEVICE int pc_pready_warp(int partition, pc_prequest_t preq, const pc_warp_state &st) {
+  using namespace pc_detail;
+  const unsigned full = 0xffffffffu;
+  if (!st.ok) return pc_pready_warp(partition, preq);
+  const uint64_t off = (uint64_t)partition * preq.part_bytes;
+  const uintptr_t al = reinterpret_cast<uintptr_t>(preq.sbuf + off) | reinterpret_cast<uintptr_t>(preq.peer_rbuf + off);
+  const bool small16 = (preq.part_bytes & 15) == 0 && (al & 15) == 0;
+  if (!small16 && (al & 7) != 0) return pc_pready_warp(partition, preq);
+  const uint32_t lane = lane_id();
+  __syncwarp(full);  // every lane's data writes are ordered before the pushes
+  if (partition < 0 || partition >= preq.partitions) {
+    if (lane == 0 && atomicCAS(preq.err, 0, PC_DEV_ERR_ARG) == 0) preq.err[1] = partition;
+    return PC_DEV_ERR_ARG;
+  }
+  if (small16) {
+    if (16ull * lane < preq.part_bytes)
+      reinterpret_cast<uint4 *>(preq.peer_rbuf + off)[lane] = __ldcg(reinterpret_cast<const uint4 *>(preq.sbuf + off) + lane);
+  } else if (8ull * lane < preq.part_bytes) {
+    reinterpret_cast<uint2 *>(preq.peer_rbuf + off)[lane] = __ldcg(reinterpret_cast<const uint2 *>(preq.sbuf + off) + lane);
+  }
+  __syncwarp(full);  // the warp's pushes, then ONE release by lane 0
+  if (lane == 0) {
+    if (preq.agg == 1 && !preq.xpart) {  // the flag store itself releases
+      if (preq.sys_scope)
+        st_release_sys(preq.peer_flags + partition, st.e);
+      else
+        st_release_gpu(preq.peer_flags + partition, st.e);
+      st_relaxed_gpu(preq.sent + partition, st.e);
+    } else {
+      fence_before_publish(preq);
+      publish(preq, partition / preq.agg, 1, st.e, partition);
+    }
   }
   __syncwarp(full);
   return 0;

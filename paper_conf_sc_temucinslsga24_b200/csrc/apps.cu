@@ -129,6 +129,8 @@ __global__ void __launch_bounds__(1024, 2) vecadd_persistent_kernel(const float2
   __syncthreads();
   if (tid == kIssuer)
     for (int k = 0; k < kStages && k < T; ++k) issue(k);
+  pc_warp_state ws{0, 0};  // warp granularity: {epoch, ready-to-receive} checked once per warp
+  if (gran == PCAPP_GRAN_WARP) pc_warp_begin(preq, &ws);
   for (int k = 0; k < T; ++k) {
     const int p = (int)blockIdx.x + k * G;
     const uint32_t s = (uint32_t)(k % kStages), par = (uint32_t)(k / kStages) & 1u;
@@ -152,7 +154,7 @@ __global__ void __launch_bounds__(1024, 2) vecadd_persistent_kernel(const float2
     if (gran == PCAPP_GRAN_THREAD) {
       if (i < N2) pc_pready(i, preq);
     } else if (gran == PCAPP_GRAN_WARP) {
-      pc_pready_warp(i >> 5, preq);
+      pc_pready_warp(i >> 5, preq, ws);
     } else if (gran == PCAPP_GRAN_BLOCK) {
       pc_pready_block(p, preq);
     }
@@ -291,6 +293,8 @@ __global__ void check_recv_kernel(pc_prequest_t preq, const uint8_t *recvbuf, ui
 // side 0 for `iters` round trips.
 __global__ void pingpong_kernel(pc_prequest_t sendq, pc_prequest_t recvq, int side, int iters, int gran,
                                 unsigned long long *out_ns) {
+  pc_warp_state ws{0, 0};
+  if (gran != PCAPP_GRAN_THREAD) pc_warp_begin(sendq, &ws);  // (st.ok = 0: the plain Pready)
   const uint64_t t0 = pc_detail::globaltimer();
   for (int k = 0; k < iters; ++k) {
     if (side == 1) {
@@ -300,7 +304,7 @@ __global__ void pingpong_kernel(pc_prequest_t sendq, pc_prequest_t recvq, int si
     if (gran == PCAPP_GRAN_THREAD) {
       if (threadIdx.x == 0) pc_pready(k, sendq);
     } else {
-      pc_pready_warp(k, sendq);
+      pc_pready_warp(k, sendq, ws);
     }
     if (side == 0) {
       if (threadIdx.x == 0) pc_wait_arrived(recvq, k);
@@ -319,9 +323,13 @@ __global__ void pingpong_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, p
   const int side = blockIdx.x;
   const pc_prequest_t &sq = side ? sendB : sendA;
   const pc_prequest_t &rq = side ? recvB : recvA;
+  // warp granularity: {epoch, ready-to-receive} checked once per warp (the
+  // receiver's Pbuf_prepare preceded this launch), then warp-collective
+  // Pready and wait; thread: lane 0 alone
+  pc_warp_state ws{0, 0};
+  if (gran != PCAPP_GRAN_THREAD) pc_warp_begin(sq, &ws);  // (st.ok = 0: the plain Pready)
   const uint64_t t0 = pc_detail::globaltimer();
   uint64_t tk = t0;
-  // warp granularity: warp-collective Pready and wait; thread: lane 0 alone
   for (int k = 0; k < iters; ++k) {
     if (side == 1) {
       if (gran == PCAPP_GRAN_THREAD) {
@@ -334,7 +342,7 @@ __global__ void pingpong_pair_kernel(pc_prequest_t sendA, pc_prequest_t recvA, p
     if (gran == PCAPP_GRAN_THREAD) {
       if (threadIdx.x == 0) pc_pready(k, sq);
     } else {
-      pc_pready_warp(k, sq);
+      pc_pready_warp(k, sq, ws);
     }
     if (side == 0) {
       if (gran == PCAPP_GRAN_THREAD) {
