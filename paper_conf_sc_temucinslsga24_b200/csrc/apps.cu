@@ -175,16 +175,16 @@ __global__ void __launch_bounds__(1024, 2) vecadd_put_persistent_kernel(const fl
                                                                         const float2 *__restrict__ B,
                                                                         float2 *__restrict__ C, int n2, int nblk,
                                                                         int batch, pc_prequest_t preq) {
-  pc_put_state st;
-  if (pc_put_begin<float2>(preq, &st, batch) != 0) return;  // (the launcher checked eligibility; timeout is recorded)
   const int G = gridDim.x;
   int p = blockIdx.x;
   float2 a = make_float2(0.f, 0.f), b = a;
   int i = p * 1024 + (int)threadIdx.x;
-  if (i < n2) {
+  if (i < n2) {  // the first operands' HBM latency overlaps pc_put_begin's acquire
     a = __ldcs(A + i);
     b = __ldcs(B + i);
   }
+  pc_put_state st;
+  if (pc_put_begin<float2>(preq, &st, batch) != 0) return;  // (the launcher checked eligibility; timeout is recorded)
   for (; p < nblk; p += G, i += G * 1024) {
     const float2 c = make_float2(a.x + b.x, a.y + b.y);
     const int in = i + G * 1024;
