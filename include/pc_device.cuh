@@ -170,8 +170,8 @@ PC_DEVICE void fence_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 PC_DEVICE void fence_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 /* Acquire-release fence at the scope the request needs: system scope when a
  * peer is another GPU (NVLink), GPU scope when every peer shares this GPU.
- * Only where the fence must ACQUIRE (relaxed flag loads before it): its
- * acquire half invalidates the SM's L1 (CCTL.IVALL in the SASS). */
+ * (Kept for completeness; the library's acquires after relaxed loads use
+ * fence_acquire, its releases fence_release.) */
 PC_DEVICE void fence_scope(uint32_t sys) {
   if (sys)
     fence_sys();
@@ -189,6 +189,16 @@ PC_DEVICE void fence_release(uint32_t sys) {
     asm volatile("fence.release.sys;" ::: "memory");
   else
     asm volatile("fence.release.gpu;" ::: "memory");
+}
+/* Acquire fence (PTX fence.acquire): after relaxed loads of flag words, the
+ * acquire pattern for every one of them — only the L1 invalidation in the
+ * SASS (CCTL.IVALL), no MEMBAR: a wait that reads many flags relaxed and
+ * then acquires once pays no store drain. */
+PC_DEVICE void fence_acquire(uint32_t sys) {
+  if (sys)
+    asm volatile("fence.acquire.sys;" ::: "memory");
+  else
+    asm volatile("fence.acquire.gpu;" ::: "memory");
 }
 PC_DEVICE uint32_t ld_acquire_scope(const uint32_t *p, uint32_t sys) {
   return sys ? ld_acquire_sys(p) : ld_acquire_gpu(p);
@@ -609,7 +619,7 @@ PC_DEVICE bool ar_rtr_ok(const pc_prequest_t &q, int u, uint32_t e) {
                                   : spin_geq<false>(w + j, e, q.err, q.timeout_ms, u);
       if (!ok) return false;
     }
-  fence_scope(q.sys_scope);
+  fence_acquire(q.sys_scope);  // the acquire pattern for the relaxed loads above
   return true;
 }
 

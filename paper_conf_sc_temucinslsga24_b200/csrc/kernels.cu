@@ -82,7 +82,7 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
 // for the whole range once everything has arrived, instead of one dependent
 // acquire per word — a bounded acquire spin only on words still behind, then
 // one acquire fence per participant for the words it saw relaxed (the
-// "ld.relaxed; fence" acquire pattern).  Words is 4-B aligned.
+// "ld.relaxed; fence.acquire" pattern: an L1 invalidation, no MEMBAR).  Words is 4-B aligned.
 __device__ __forceinline__ bool wait_words_range(const uint32_t *w, int n, uint32_t target, int sys, int32_t *err,
                                                  uint32_t tmo, uint32_t idx, uint32_t nthr) {
   int head = (int)(((16u - (uint32_t)(reinterpret_cast<uintptr_t>(w) & 15u)) & 15u) >> 2);
@@ -105,7 +105,7 @@ __device__ __forceinline__ bool wait_words_range(const uint32_t *w, int n, uint3
   }
   for (int i = head + 4 * nv + (int)idx; i < n; i += (int)nthr)
     if (!spin(i)) return false;
-  if (relaxed) fence_scope(sys);
+  if (relaxed) fence_acquire(sys);
   return true;
 }
 
