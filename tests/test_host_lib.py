@@ -430,3 +430,43 @@ def test_dry_overlap_and_inline_rules():
     for c in cs:
         c.destroy()
     g.destroy()
+
+
+def test_device_header_compiles_in_a_user_kernel(tmp_path):
+    """include/pc_device.cuh is the user's device API: a stand-alone user
+    translation unit calling every binding (Pready at thread / warp / block
+    granularity, the register Kernel Copy with its persistent begin / end,
+    the check-once warp Pready, the cooperative INLINE fold, Parrived) builds
+    for sm_100a with nvcc alone (no GPU needed)."""
+    import shutil
+    nvcc = shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc"
+    if not os.path.exists(nvcc):
+        pytest.skip("nvcc not available")
+    src = tmp_path / "user.cu"
+    src.write_text(r'''
+#include "pc_device.cuh"
+__global__ void user_producer(float2 *out, pc_prequest_t sendq, pc_prequest_t recvq, pc_prequest_t arq, int n) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const float2 v = make_float2((float)i, 1.f);
+  if (i < n) out[i] = v;
+  pc_pready(i, sendq);
+  pc_pready_warp(i >> 5, sendq);
+  pc_pready_block(blockIdx.x, sendq);
+  pc_pready_block_put(blockIdx.x, sendq, (uint64_t)threadIdx.x, v);
+  pc_put_state st;
+  if (pc_put_begin<float2>(sendq, &st, 4) == 0) {
+    pc_pready_block_put(blockIdx.x, sendq, (uint64_t)threadIdx.x, v, st);
+    pc_put_end(sendq, st);
+  }
+  pc_warp_state ws;
+  pc_warp_begin(sendq, &ws);
+  pc_pready_warp(i >> 5, sendq, ws);
+  pc_pready_block_coop(blockIdx.x, arq);
+  if (threadIdx.x == 0 && pc_parrived(recvq, blockIdx.x)) out[0].x += 1.f;
+  pc_wait_arrived_warp(recvq, blockIdx.x);
+}
+''')
+    inc = os.path.join(ROOT, "include")
+    r = subprocess.run([nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-std=c++17", "-DPC_INLINE_ALLREDUCE",
+                        "-I", inc, "-c", "-o", str(tmp_path / "user.o"), str(src)], capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr[-2000:]
