@@ -12,7 +12,10 @@ Driver contract (one JSON line on rank 0):
   over all ranks.  N = 1 runs the same hot path with P virtual ranks
   co-located on the one B200 (--vranks, default 8): every rank's buffers,
   flags and engine live on one GPU, so "NVLink" stores become HBM stores and
-  the kernel is HBM-bound.
+  the kernel is HBM-bound.  Beside the headline line N = 1 also reports the
+  Pready->Parrived latency pairs, C4 Jacobi, C1 (1 MiB) and C2 at 256 MiB
+  (the persistent register-Kernel-Copy producer vs kernel -> copy, with its
+  own HBM roofline).
 
 A step = one epoch of the whole hot path for every rank: pc_epoch_all (Start +
 ready-to-receive + the user's Pready of every partition, one kernel for all
