@@ -11,6 +11,7 @@
  *   PC_DEVICE int  pc_put_begin<T>(pc_prequest_t preq, pc_put_state *st, int batch = 1);  block-collective
  *   PC_DEVICE int  pc_pready_block_put<T>(partition, preq, idx, v, st);     block-collective
  *   PC_DEVICE void pc_put_end(pc_prequest_t preq, pc_put_state &st);       block-collective
+ *   PC_DEVICE int  pc_pready_block(int partition, pc_prequest_t preq, pc_put_state &st);  (checked once)
  *   PC_DEVICE int  pc_pready_block_coop(int partition, pc_prequest_t preq);  block-collective (R36,
  *                  INLINE allreduce, -DPC_INLINE_ALLREDUCE)
  *   PC_DEVICE int  pc_parrived    (pc_prequest_t preq, int partition);
@@ -1240,6 +1241,40 @@ PC_DEVICE int pc_pready_block_put(int partition, pc_prequest_t preq, uint64_t id
   if (++st.npend < st.batch) return 0;
   __syncthreads();  // the batch's assignments, then lane k of warp 0 releases pending partition k
   if (tid < st.npend) pc_detail::put_release(preq, st.mine, st.e);
+  st.npend = 0;
+  return 0;
+}
+
+/* The MPI-shaped block Pready in a persistent CTA, checked once: with a
+ * state from pc_put_begin<uint8_t> (any size or alignment), the block's
+ * partition is read back after the barrier and pushed as in pc_pready_block,
+ * but {epoch, ready-to-receive} is not re-checked and the releases are
+ * batched like pc_pready_block_put's (pc_put_end flushes). */
+PC_DEVICE int pc_pready_block(int partition, pc_prequest_t preq, pc_put_state &st) {
+  using namespace pc_detail;
+  if (!st.ok) return pc_pready_block(partition, preq);
+  const uint32_t tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  const uint32_t nthr = blockDim.x * blockDim.y * blockDim.z;
+  if ((unsigned)partition >= (unsigned)preq.partitions) {
+    if (tid == 0 && atomicCAS(preq.err, 0, PC_DEV_ERR_ARG) == 0) preq.err[1] = partition;
+    return PC_DEV_ERR_ARG;
+  }
+  __syncthreads();  // the block's data writes are complete
+  const uint64_t off = (uint64_t)partition * preq.part_bytes;
+  const uintptr_t al = reinterpret_cast<uintptr_t>(preq.sbuf + off) | reinterpret_cast<uintptr_t>(preq.peer_rbuf + off);
+  if (preq.part_bytes <= 16ull * nthr && (preq.part_bytes & 15) == 0 && (al & 15) == 0) {
+    if (16ull * tid < preq.part_bytes)
+      reinterpret_cast<uint4 *>(preq.peer_rbuf + off)[tid] = __ldcg(reinterpret_cast<const uint4 *>(preq.sbuf + off) + tid);
+  } else if (preq.part_bytes <= 8ull * nthr && (preq.part_bytes & 7) == 0 && (al & 7) == 0) {
+    if (8ull * tid < preq.part_bytes)
+      reinterpret_cast<uint2 *>(preq.peer_rbuf + off)[tid] = __ldcg(reinterpret_cast<const uint2 *>(preq.sbuf + off) + tid);
+  } else {
+    copy_bytes_cold(preq.peer_rbuf + off, preq.sbuf + off, preq.part_bytes, tid, nthr);
+  }
+  if (tid == st.npend) st.mine = partition;
+  if (++st.npend < st.batch) return 0;
+  __syncthreads();  // the batch's pushes, then lane k of warp 0 releases pending partition k
+  if (tid < st.npend) put_release(preq, st.mine, st.e);
   st.npend = 0;
   return 0;
 }

@@ -95,7 +95,7 @@ template <int gran>
 __global__ void __launch_bounds__(1024, 2) vecadd_persistent_kernel(const float2 *__restrict__ A,
                                                                     const float2 *__restrict__ B,
                                                                     float2 *__restrict__ C, int64_t n2,
-                                                                    int64_t nblk, pc_prequest_t preq) {
+                                                                    int64_t nblk, int batch, pc_prequest_t preq) {
   // 32-bit loop state (the launcher guarantees n2 < 2^31) and smem offsets
   // from one base: the loop carries few registers at the 32-register budget.
   extern __shared__ __align__(128) uint8_t smem[];
@@ -131,6 +131,8 @@ __global__ void __launch_bounds__(1024, 2) vecadd_persistent_kernel(const float2
     for (int k = 0; k < kStages && k < T; ++k) issue(k);
   pc_warp_state ws{0, 0};  // warp granularity: {epoch, ready-to-receive} checked once per warp
   if (gran == PCAPP_GRAN_WARP) pc_warp_begin(preq, &ws);
+  pc_put_state bs{0, 0, 1, 0, -1};  // block granularity: checked once per CTA, releases batched
+  if (gran == PCAPP_GRAN_BLOCK) pc_put_begin<uint8_t>(preq, &bs, batch);  // (bs.ok = 0: the plain Pready)
   for (int k = 0; k < T; ++k) {
     const int p = (int)blockIdx.x + k * G;
     const uint32_t s = (uint32_t)(k % kStages), par = (uint32_t)(k / kStages) & 1u;
@@ -156,13 +158,14 @@ __global__ void __launch_bounds__(1024, 2) vecadd_persistent_kernel(const float2
     } else if (gran == PCAPP_GRAN_WARP) {
       pc_pready_warp(i >> 5, preq, ws);
     } else if (gran == PCAPP_GRAN_BLOCK) {
-      pc_pready_block(p, preq);
+      pc_pready_block(p, preq, bs);
     }
     if (tid == kIssuer && k + kStages < T) {  // every warp has read stage s: refill it
       mbar_wait(reinterpret_cast<uint64_t *>(smem + kEmpty) + s, par);
       issue(k + kStages);
     }
   }
+  if (gran == PCAPP_GRAN_BLOCK) pc_put_end(preq, bs);
 }
 
 // block_put from a persistent producer (R35): the paper's 8 KiB logical
@@ -579,7 +582,7 @@ int minb() {
 // Pready path it calls, so the 32-register budget of 2 CTAs per SM is spent on
 // that path alone.
 using VecaddFn = void (*)(const float2 *, const float2 *, float2 *, int64_t, pc_prequest_t);
-using VecaddPersFn = void (*)(const float2 *, const float2 *, float2 *, int64_t, int64_t, pc_prequest_t);
+using VecaddPersFn = void (*)(const float2 *, const float2 *, float2 *, int64_t, int64_t, int, pc_prequest_t);
 template <int MINB>
 VecaddFn vecadd_fn(int gran) {
   switch (gran) {
@@ -658,7 +661,8 @@ int pcapp_vecadd_persistent(const float *A, const float *B, float *C, int64_t n,
     return -2;
   const int64_t slots = (int64_t)sms * per;
   const int64_t grid = nblk < slots ? nblk : slots;
-  f<<<(unsigned)grid, 1024, kStagedSmem, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, nblk, q);
+  f<<<(unsigned)grid, 1024, kStagedSmem, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, nblk,
+                                              put_batch(), q);
   return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 

@@ -103,15 +103,17 @@ def test_c2_persistent_256mib(gran, copy):
     run_vecadd(1 << 26, gran, 1, copy, epochs=2, persistent=True)
 
 
+@pytest.mark.parametrize("gran", [apps.GRAN_BLOCK_PUT, apps.GRAN_BLOCK])
 @pytest.mark.parametrize("batch", ["1", "3", "32"])
 @pytest.mark.parametrize("agg", [1, 5])
-def test_put_batched_release(batch, agg, monkeypatch):
-    """Persistent register Kernel Copy releasing `batch` logical blocks at a
-    time (pc_put_begin batch, pc_put_end flushing the tail; 1000 logical
-    blocks over 296 CTAs leave partial batches), with and without
-    aggregation: byte-exact vs O1, in-kernel Parrived consumer included."""
+def test_put_batched_release(gran, batch, agg, monkeypatch):
+    """Persistent producers releasing `batch` logical blocks at a time
+    (pc_put_begin batch, pc_put_end flushing the tail; 1000 logical blocks
+    over 296 CTAs leave partial batches) — the register Kernel Copy and the
+    MPI-shaped pc_pready_block checked once — with and without aggregation:
+    byte-exact vs O1, in-kernel Parrived consumer included."""
     monkeypatch.setenv("PCAPP_PUT_BATCH", batch)
-    run_vecadd(2048 * 1000, apps.GRAN_BLOCK_PUT, agg, pc.COPY_INLINE, epochs=3, persistent=True)
+    run_vecadd(2048 * 1000, gran, agg, pc.COPY_INLINE, epochs=3, persistent=True)
 
 
 @pytest.mark.parametrize("persistent", [False, True])
