@@ -458,6 +458,11 @@ __global__ void user_producer(float2 *out, pc_prequest_t sendq, pc_prequest_t re
     pc_pready_block_put(blockIdx.x, sendq, (uint64_t)threadIdx.x, v, st);
     pc_put_end(sendq, st);
   }
+  pc_put_state bs;
+  if (pc_put_begin<uint8_t>(sendq, &bs, 2) == 0) {
+    pc_pready_block(blockIdx.x, sendq, bs);
+    pc_put_end(sendq, bs);
+  }
   pc_warp_state ws;
   pc_warp_begin(sendq, &ws);
   pc_pready_warp(i >> 5, sendq, ws);
