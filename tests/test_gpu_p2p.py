@@ -798,3 +798,41 @@ def test_pready_block_put_element_types(elem, pbytes, agg, copy):
             np.testing.assert_array_equal(rbuf.cpu().numpy(), payload)
         snd.free()
         rcv.free()
+
+
+def test_persistent_put_many_epochs():
+    """200 back-to-back epochs of the persistent register Kernel Copy with
+    batched releases (epoch-tagged inputs, no host sync between epochs except
+    every 50th): every epoch's bytes arrive intact (the last epoch checked
+    byte-exact, every 50th epoch's too), no device error."""
+    n = 2048 * 600  # 600 logical blocks over 296 CTAs: partial batches every epoch
+    with comms(2) as cs:
+        st = torch.cuda.Stream()
+        A = torch.empty(n, device="cuda")
+        B = torch.zeros(n, device="cuda")
+        Cb = torch.empty(n, device="cuda")
+        R = torch.zeros(n, device="cuda")
+        parts = n // 2048
+        snd = pc.psend_init(Cb, parts, 2048, pc.FLOAT32, 1, 31, cs[0])
+        rcv = pc.precv_init(R, parts, 2048, pc.FLOAT32, 0, 31, cs[1])
+        base = torch.arange(n, device="cuda", dtype=torch.float32)
+        torch.cuda.synchronize()
+        for e in range(200):
+            with torch.cuda.stream(st):
+                A.copy_(base + float(e))  # epoch tag in every element
+            if e == 0:
+                snd.start(st)
+                rcv.start(st)
+                first_prepare([[snd], [rcv]], [st, st])
+                sq = snd.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+                rcv.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+            else:
+                pc.epoch_all([snd, rcv], False, st)
+            apps.vecadd(A, B, Cb, n, apps.GRAN_BLOCK_PUT, sq, st, persistent=True)
+            pc.waitall_on_stream([snd, rcv], st)
+            if e % 50 == 49:
+                torch.cuda.synchronize()
+                assert snd.error()[0] == 0 and rcv.error()[0] == 0
+                assert torch.equal(R, base + float(e)), f"epoch {e}"
+        snd.free()
+        rcv.free()
