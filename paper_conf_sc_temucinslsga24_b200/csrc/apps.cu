@@ -659,7 +659,11 @@ int pcapp_vecadd_persistent(const float *A, const float *B, float *C, int64_t n,
       cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kStagedSmem) != cudaSuccess ||
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, 1024, kStagedSmem) != cudaSuccess || per < 1)
     return -2;
-  const int64_t slots = (int64_t)sms * per;
+  int64_t slots = (int64_t)sms * per;
+  // ENGINE copy: the library's engine runs beside the producer on up to half
+  // of the SMs (PC_OVERLAP_FRAC); a persistent grid over every slot would make
+  // it wait for the producer's CTAs to retire, so leave it that half.
+  if (preq && q.copy == 1 && slots > 1) slots /= 2;
   const int64_t grid = nblk < slots ? nblk : slots;
   f<<<(unsigned)grid, 1024, kStagedSmem, s>>>((const float2 *)A, (const float2 *)B, (float2 *)C, n2, nblk,
                                               put_batch(), q);
