@@ -23,6 +23,50 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
   bool rtr_ok = false;
+  // Small transport partitions (one slice of <= 512 B, 16-B aligned: thread /
+  // warp granularity): each LANE owns a unit — 32 ready flags polled at once,
+  // each lane copies its own unit with 16-B vectors, one warp-wide release,
+  // then every lane signals its own unit (the 8-unit warp-cooperative sweep
+  // below spent a poll round trip per 8 units of a few hundred bytes).
+  const uint64_t ub = (uint64_t)a.agg * a.part_bytes;
+  if (a.ns == 1 && !a.xpart && ub <= 512 && (ub & 15) == 0 &&
+      ((reinterpret_cast<uintptr_t>(a.sbuf) | reinterpret_cast<uintptr_t>(a.peer_rbuf)) & 15) == 0) {
+    for (int j0 = 0; gw + j0 * W < a.nunits; j0 += 32) {
+      const int x = gw + (j0 + (int)lane) * W;  // this lane's unit = transport partition x
+      uint32_t pending = __ballot_sync(0xffffffffu, x < a.nunits);
+      Idle idle;
+      while (pending) {
+        const bool rdy = ((pending >> lane) & 1u) && reached(ld_acquire_gpu(a.ready + x), e);
+        const uint32_t ready = __ballot_sync(0xffffffffu, rdy) & pending;
+        if (!ready) {
+          if (!idle.wait(a.err, a.timeout_ms, gw)) return;
+          continue;
+        }
+        idle.progressed();
+        if (!rtr_ok) {
+          if (!warp_wait(a.rtr, e, a.err, a.timeout_ms, -1, a.sys)) return;
+          rtr_ok = true;
+        }
+        if (rdy) {
+          const int rem = a.partitions - x * a.agg;
+          const uint64_t len = (uint64_t)(rem < a.agg ? rem : a.agg) * a.part_bytes;
+          const uint4 *src = reinterpret_cast<const uint4 *>(a.sbuf + (uint64_t)x * ub);
+          uint4 *dst = reinterpret_cast<uint4 *>(a.peer_rbuf + (uint64_t)x * ub);
+          for (uint64_t v = 0; v < len / 16; ++v) dst[v] = __ldcg(src + v);
+          for (uint64_t b = len & ~15ull; b < len; ++b)  // a ragged last transport partition
+            reinterpret_cast<uint8_t *>(dst)[b] = reinterpret_cast<const uint8_t *>(src)[b];
+        }
+        fence_release(a.sys);  // each lane's copies, before its own signal
+        if (rdy) {
+          signal_transport(a.peer_flags, x, e, 0u, a.partitions, a.agg, a.part_bytes, a.peer_part_bytes);
+          st_relaxed_gpu(a.sent + x, e);
+        }
+        __syncwarp();
+        pending &= ~ready;
+      }
+    }
+    return;
+  }
   for (int j0 = 0; gw + j0 * W < a.nunits; j0 += kMaxActive) {
     uint32_t pending = 0;
 #pragma unroll

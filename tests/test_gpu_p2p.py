@@ -836,3 +836,38 @@ def test_persistent_put_many_epochs():
                 assert torch.equal(R, base + float(e)), f"epoch {e}"
         snd.free()
         rcv.free()
+
+
+@pytest.mark.parametrize("pbytes,parts,agg", [(8, 37, 2), (16, 101, 1), (48, 33, 8), (8, 1001, 64)])
+def test_engine_small_units(pbytes, parts, agg):
+    """ENGINE copy of small transport partitions (<= 512 B: the engine gives
+    each lane a unit), including a ragged last transport partition whose
+    bytes are not a multiple of 16: byte-exact over 3 epochs."""
+    total = parts * pbytes
+    with comms(2) as cs:
+        s0, s1 = torch.cuda.Stream(), torch.cuda.Stream()
+        src = torch.empty(total, dtype=torch.uint8, device="cuda")
+        sbuf, rbuf = torch.zeros_like(src), torch.zeros_like(src)
+        snd = pc.psend_init(sbuf, parts, pbytes, pc.BYTE, 1, 25, cs[0])
+        rcv = pc.precv_init(rbuf, parts, pbytes, pc.BYTE, 0, 25, cs[1])
+        for e in range(3):
+            payload = synth.bytes_tagged(SEED, 6, e, total)
+            src.copy_(torch.from_numpy(payload))
+            torch.cuda.synchronize()
+            snd.start(s0)
+            rcv.start(s1)
+            if e == 0:
+                first_prepare([[snd], [rcv]], [s0, s1])
+                sq = snd.prequest_create(pc.GRAN_BLOCK, agg, pc.COPY_ENGINE)
+                rcv.prequest_create(pc.GRAN_BLOCK, 1, pc.COPY_INLINE)
+            else:
+                rcv.pbuf_prepare(s1)
+                snd.pbuf_prepare(s0)
+            apps.produce(sbuf, src, parts, pbytes, apps.GRAN_BLOCK, sq, stream=s0)
+            snd.wait_on_stream(s0)
+            rcv.wait_on_stream(s1)
+            torch.cuda.synchronize()
+            assert snd.error()[0] == 0 and rcv.error()[0] == 0, (snd.error(), rcv.error())
+            np.testing.assert_array_equal(rbuf.cpu().numpy(), payload)
+        snd.free()
+        rcv.free()
