@@ -23,14 +23,15 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t e = *(const volatile uint32_t *)a.epoch;  // device epoch word (graph-replayable)
   bool rtr_ok = false;
-  // Small transport partitions (one slice of <= 512 B, 16-B aligned: thread /
+  // Small transport partitions (one slice of <= 512 B, 8-B aligned: thread /
   // warp granularity): each LANE owns a unit — 32 ready flags polled at once,
-  // each lane copies its own unit with 16-B vectors, one warp-wide release,
+  // each lane copies its own unit with 16-B (or 8-B) vectors, one warp-wide release,
   // then every lane signals its own unit (the 8-unit warp-cooperative sweep
   // below spent a poll round trip per 8 units of a few hundred bytes).
   const uint64_t ub = (uint64_t)a.agg * a.part_bytes;
-  if (a.ns == 1 && !a.xpart && ub <= 512 && (ub & 15) == 0 &&
-      ((reinterpret_cast<uintptr_t>(a.sbuf) | reinterpret_cast<uintptr_t>(a.peer_rbuf)) & 15) == 0) {
+  const uintptr_t bal = reinterpret_cast<uintptr_t>(a.sbuf) | reinterpret_cast<uintptr_t>(a.peer_rbuf);
+  const bool v16 = (ub & 15) == 0 && (bal & 15) == 0;  // else 8-B vectors (thread granularity: 8-B units)
+  if (a.ns == 1 && !a.xpart && ub <= 512 && (ub & 7) == 0 && (bal & 7) == 0) {
     for (int j0 = 0; gw + j0 * W < a.nunits; j0 += 32) {
       const int x = gw + (j0 + (int)lane) * W;  // this lane's unit = transport partition x
       uint32_t pending = __ballot_sync(0xffffffffu, x < a.nunits);
@@ -50,11 +51,15 @@ __global__ void __launch_bounds__(kEngineBlock) p2p_engine(P2pEngineArgs a) {
         if (rdy) {
           const int rem = a.partitions - x * a.agg;
           const uint64_t len = (uint64_t)(rem < a.agg ? rem : a.agg) * a.part_bytes;
-          const uint4 *src = reinterpret_cast<const uint4 *>(a.sbuf + (uint64_t)x * ub);
-          uint4 *dst = reinterpret_cast<uint4 *>(a.peer_rbuf + (uint64_t)x * ub);
-          for (uint64_t v = 0; v < len / 16; ++v) dst[v] = __ldcg(src + v);
-          for (uint64_t b = len & ~15ull; b < len; ++b)  // a ragged last transport partition
-            reinterpret_cast<uint8_t *>(dst)[b] = reinterpret_cast<const uint8_t *>(src)[b];
+          const uint8_t *src = a.sbuf + (uint64_t)x * ub;
+          uint8_t *dst = a.peer_rbuf + (uint64_t)x * ub;
+          uint64_t b = 0;
+          if (v16)
+            for (; b + 16 <= len; b += 16)
+              *reinterpret_cast<uint4 *>(dst + b) = __ldcg(reinterpret_cast<const uint4 *>(src + b));
+          for (; b + 8 <= len; b += 8)
+            *reinterpret_cast<uint2 *>(dst + b) = __ldcg(reinterpret_cast<const uint2 *>(src + b));
+          for (; b < len; ++b) dst[b] = src[b];  // a ragged last transport partition
         }
         fence_release(a.sys);  // each lane's copies, before its own signal
         if (rdy) {

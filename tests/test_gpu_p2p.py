@@ -838,7 +838,8 @@ def test_persistent_put_many_epochs():
         rcv.free()
 
 
-@pytest.mark.parametrize("pbytes,parts,agg", [(8, 37, 2), (16, 101, 1), (48, 33, 8), (8, 1001, 64)])
+@pytest.mark.parametrize("pbytes,parts,agg", [(8, 37, 2), (16, 101, 1), (48, 33, 8), (8, 1001, 64), (8, 77, 1),
+                                              (24, 41, 3), (12, 50, 1)])
 def test_engine_small_units(pbytes, parts, agg):
     """ENGINE copy of small transport partitions (<= 512 B: the engine gives
     each lane a unit), including a ragged last transport partition whose
